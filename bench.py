@@ -1,0 +1,332 @@
+#!/usr/bin/env python
+"""Benchmark: trace records/s reduced to window snapshots (BASELINE.json metric) on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
+
+One step = one rtm_window_reduce over the whole workload (all 1000 windows of C2, the
+configuration BASELINE.json quotes the metric on: ~20k buffers, 90M level samples + 10M task
+events, k=64), re-armed with rtm_reset.  Inputs are resident in HBM before the timed region
+(1.6 GB > the 126 MB L2, so no flush is needed between steps).  `value` is whole-job records/s
+(max-over-ranks device time); `e2e` repeats the metric through the same C-ABI with HOST
+buffers (host->device copy of the trace and device->host read of the results inside the
+timed region).  N > 1: weak scaling, every rank holds one C2-sized shard of an N-times larger
+simulated system (owner-component sharding) and the per-window results are merged across
+ranks with an all-gather + the library's merge kernels every step.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "trace records/sec reduced to snapshot (1/2/4/8 B200) + % HBM peak"
+UNIT = "records/s"
+
+
+def _peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
+                parts = [x.strip() for x in out.stdout.strip().split(",")]
+                if len(parts) >= 7:
+                    self.rows.append(parts)
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if "Active" in r[3 + i]
+                          and "Not" not in r[3 + i]})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# ---------------------------------------------------------------------------------------------
+def cpu_reference_step(wl, n_windows_sample: int):
+    """Oracle (as it stands, one host core) over the first `n_windows_sample` windows."""
+    import gen
+    import oracle
+
+    ends = wl.t_end()[:n_windows_sample]
+    t_hi = int(ends[-1])
+    # bounded sample: the records with ts < t_hi (ts = t0 + (i*mul) >> 32 is monotone in i), plus a few
+    # beyond it that the reduction drops as early records
+    ns = min(wl.n_samples, int((t_hi - wl.t0) * wl.samples_per_tick) + 4)
+    ne = min(wl.n_events, int((t_hi - wl.t0) * wl.n_events // max(1, wl.ticks)) + 4)
+    s, e = gen.samples(wl, 0, ns), gen.events(wl, 0, ne)
+    owner, cap, tot = gen.registry(wl)
+    orc = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, t0=wl.t0, hang_windows=wl.hang_windows,
+                        k=wl.k)
+    t0 = time.perf_counter()
+    out = orc.reduce(s, e, ends, want_hung=False)
+    dt = time.perf_counter() - t0
+    assert out["rc"] == 0
+    recs = int(out["summary"]["n_samples"].sum() + out["summary"]["n_events"].sum() + out["summary"]["n_dropped"].sum())
+    return recs, dt
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle timed on the host cores, same metric/config (rank 0 only)."""
+    import gen
+
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    wl = gen.C2
+    n_win = int(os.environ.get("RTM_REF_WINDOWS", "25"))
+    for _ in range(args.warmup):
+        cpu_reference_step(wl, n_win)
+    tot_recs, tot_t = 0, 0.0
+    for _ in range(args.steps):
+        r, dt = cpu_reference_step(wl, n_win)
+        tot_recs += r
+        tot_t += dt
+    v = tot_recs / tot_t
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_t / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+            "config": {"workload": wl.description, "sample": f"first {n_win} of {wl.n_windows} windows"},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"first {n_win} windows of C2 ({tot_recs // args.steps} records/step)"},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------------------------------------
+def weak_registry(wl, world):
+    """Registry of the N-times larger system: rank r's local buffer l -> global id (comp-major)."""
+    import gen
+
+    nbl = wl.n_buffers
+    owner, cap, tot = gen.registry(wl)  # local shapes; capacity depends on (seed, local id)
+    if world == 1:
+        return owner, cap, tot
+    gb = np.arange(nbl * world, dtype=np.int64)
+    gc = gb // 4
+    r = gc % world
+    lc = gc // world
+    lb = lc * 4 + gb % 4
+    caps = np.empty(nbl * world, np.uint16)
+    for rr in range(world):
+        wr = wl.scaled(wl.name, seed=wl.seed + 1000 * rr)
+        _, cr, _ = gen.registry(wr)
+        m = r == rr
+        caps[m] = cr[lb[m]]
+    return gc.astype(np.uint32), caps, tot * world
+
+
+def run_native(args):
+    import torch
+
+    import gen
+    from paper_conf_micro_mosallaeii024_b200 import Monitor
+
+    world = args.gpus
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    wl = gen.C2
+    wr = wl.scaled(wl.name, seed=wl.seed + 1000 * rank) if world > 1 else wl
+    owner, cap, tot = weak_registry(wl, world)
+    nc = (len(owner) + 3) // 4
+    owned = None
+    if world > 1:
+        owned = (np.arange(nc) % world == rank).astype(np.uint8)
+    dev = torch.device("cuda", local)
+    ds = torch.empty(wl.n_samples * 16, dtype=torch.uint8, device=dev)
+    de = torch.empty(wl.n_events * 16, dtype=torch.uint8, device=dev)
+    st = torch.cuda.current_stream(dev).cuda_stream
+    gen.fill_device("samples", wr, ds.data_ptr(), 0, wl.n_samples, st)
+    gen.fill_device("events", wr, de.data_ptr(), 0, wl.n_events, st)
+    if world > 1:
+        gen.remap_weak(wr, ds.data_ptr(), wl.n_samples, de.data_ptr(), wl.n_events, rank, world, st)
+    torch.cuda.synchronize()
+    mon = Monitor(owner, cap, tot, n_components=nc, t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k, device=local,
+                  rank=rank, world=world, owned_components=owned)
+    t_end = wl.t_end()
+    n_rec = wl.n_samples + wl.n_events
+
+    def step():
+        mon.reset()
+        mon.ingest(ds, de)
+        return mon.window_reduce(t_end)
+
+    for _ in range(max(3, args.warmup)):
+        res = step()
+    # correctness guard on the timed configuration: every record accounted for
+    S = res["summary"]
+    assert int(S["n_samples"].sum() + S["n_events"].sum() + S["n_dropped"].sum()) == n_rec * world
+    mon.profile(True)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t_wall = time.perf_counter()
+        ev0.record()
+        for _ in range(args.steps):
+            step()
+        ev1.record()
+        torch.cuda.synchronize()
+        t_wall = time.perf_counter() - t_wall
+        if dist:
+            dist.barrier()
+    ms = ev0.elapsed_time(ev1)
+    prof = mon.profile_read()
+    mon.profile(False)
+    if dist:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    value = n_rec * world * args.steps / (ms / 1e3)
+
+    # ---- e2e through the same C-ABI with HOST buffers (pinned), results read back each step
+    hs = torch.empty(wl.n_samples * 16, dtype=torch.uint8, pin_memory=True)
+    he = torch.empty(wl.n_events * 16, dtype=torch.uint8, pin_memory=True)
+    hs.copy_(ds)
+    he.copy_(de)
+    torch.cuda.synchronize()
+    e2e_steps = max(1, min(3, args.steps))
+
+    def step_host():
+        mon.reset()
+        mon.ingest(hs, he)
+        return mon.window_reduce(t_end)
+
+    step_host()
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+    te = time.perf_counter()
+    for _ in range(e2e_steps):
+        step_host()
+    torch.cuda.synchronize()
+    te = time.perf_counter() - te
+    if dist:
+        t = torch.tensor([te], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        te = float(t.item())
+    e2e_value = n_rec * world * e2e_steps / te
+    W = wl.n_windows
+    d2h = W * (8 * 6 + wl.k * 8 + 4 + wl.n_kernels * 40 + 4)
+
+    if rank != 0:
+        if dist:
+            dist.destroy_process_group()
+        return
+    # ---- roofline of the dominant kernel (largest share of the step)
+    peaks = _peaks()
+    hbm = float(peaks.get("hbm_gbs", 6650.0))
+    dom = max((k for k in prof if prof[k]["launches"]), key=lambda k: prof[k]["total_ms"])
+    d = prof[dom]
+    hbm_kernel = "k_partition"
+    hk = prof[hbm_kernel]
+    achieved_gbs = (hk["algo_bytes"] / hk["launches"]) / (hk["total_ms"] / hk["launches"] / 1e3) / 1e9
+    step_ms = ms / args.steps
+    shares = {k: round(prof[k]["total_ms"] / args.steps / step_ms, 4) for k in prof if prof[k]["launches"]}
+    launches = sum(prof[k]["launches"] for k in prof)
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "r01_partition_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get("bytes_per_launch")
+        except Exception:
+            traffic = None
+    path_gbs = 16.0 * n_rec / (step_ms / 1e3) / 1e9
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        n_win = int(os.environ.get("RTM_CPU_WINDOWS", "40"))
+        recs, dt = cpu_reference_step(wl, n_win)
+        cpu = {"value": recs / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"first {n_win} of {W} C2 windows ({recs} records), single-threaded C oracle"}
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+        "data": "synthetic",
+        "config": {"workload": wl.description + (f" (x{world} shards, weak scaling)" if world > 1 else ""),
+                   "n_buffers": int(len(owner)), "records_per_gpu": n_rec, "windows": W, "k": wl.k,
+                   "hang_windows": wl.hang_windows, "l2": "inputs (1.6 GB/GPU) larger than L2; no flush",
+                   "parallelism": f"owner-component shards x{world}" if world > 1 else "single GPU"},
+        "roofline": {"bound": "hbm", "kernel": hbm_kernel, "achieved": achieved_gbs, "peak": hbm, "unit": "GB/s",
+                     "frac": achieved_gbs / hbm, "traffic": traffic, "peak_source": "MEASURED_PEAKS.json hbm_gbs",
+                     "path_achieved": path_gbs, "path_frac": path_gbs / hbm,
+                     "dominant_kernel": dom, "dominant_share": shares.get(dom)},
+        "kernel_share": shares,
+        "cpu_baseline": cpu,
+        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 16 * n_rec, "d2h_bytes_per_step": d2h},
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+        "wall_s_timed": t_wall,
+    }
+    print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="native", choices=["native", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_native(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -201,6 +201,9 @@ def device_lib():
         for fn in ("gen_cuda_fill_samples", "gen_cuda_fill_events", "gen_cuda_flag_samples"):
             getattr(lib, fn).argtypes = [P, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p]
             getattr(lib, fn).restype = ctypes.c_int
+        lib.gen_cuda_remap_weak.argtypes = [P, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint64,
+                                            ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p]
+        lib.gen_cuda_remap_weak.restype = ctypes.c_int
         _dev = lib
     return _dev
 
@@ -212,3 +215,12 @@ def fill_device(kind: str, wl: Workload, ptr: int, start: int, count: int, strea
     err = fn(ctypes.byref(p), start, count, ctypes.c_void_p(ptr), ctypes.c_void_p(stream))
     if err != 0:
         raise RuntimeError(f"gen_cuda fill failed: cudaError {err}")
+
+
+def remap_weak(wl: Workload, sptr: int, ns: int, eptr: int, ne: int, rank: int, world: int, stream: int = 0) -> None:
+    """Map rank `rank`'s local device trace into the id space of a `world`-times larger system."""
+    p = wl.params()
+    err = device_lib().gen_cuda_remap_weak(ctypes.byref(p), ctypes.c_void_p(sptr), ns, ctypes.c_void_p(eptr), ne,
+                                           rank, world, ctypes.c_void_p(stream))
+    if err != 0:
+        raise RuntimeError(f"gen_cuda_remap_weak failed: cudaError {err}")

@@ -27,6 +27,27 @@ __global__ void gen_samples_flag_kernel(rtm_gen_params p, uint64_t start, uint64
   }
 }
 
+// Weak-scaling shards (bench.py, N > 1): rank r's local trace is mapped into the global id space
+// of an N-times larger system, component-major: global comp = local comp * world + rank.
+__global__ void remap_weak_kernel(gen_sample_rec *s, uint64_t ns, gen_event_rec *e, uint64_t ne, uint32_t nbl,
+                                  uint32_t ncl, uint32_t bpc, uint32_t rank, uint32_t world) {
+  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < ns; t += stride) {
+    uint32_t b = s[t].buffer_id;
+    if (b < nbl) {
+      uint32_t gc = (b / bpc) * world + rank;
+      s[t].buffer_id = gc * bpc + b % bpc;
+    } else {
+      s[t].buffer_id = 0xFFFFFFF0u;
+    }
+  }
+  for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < ne; t += stride) {
+    uint32_t m = e[t].meta, c = m & 0xFFFFFu;
+    uint32_t gc = c < ncl ? c * world + rank : 0xFFFFFu;
+    e[t].meta = (m & ~0xFFFFFu) | (gc & 0xFFFFFu);
+  }
+}
+
 int grid_for(uint64_t count) {
   uint64_t g = (count + 255) / 256;
   return (int)(g > 148 * 32 ? 148 * 32 : (g ? g : 1));
@@ -52,6 +73,15 @@ int gen_cuda_fill_events(const rtm_gen_params *p, uint64_t start, uint64_t count
 int gen_cuda_flag_samples(const rtm_gen_params *p, uint64_t start, uint64_t count, void *flag, void *stream) {
   if (count == 0) return 0;
   gen_samples_flag_kernel<<<grid_for(count), 256, 0, (cudaStream_t)stream>>>(*p, start, count, (uint8_t *)flag);
+  return (int)cudaGetLastError();
+}
+
+int gen_cuda_remap_weak(const rtm_gen_params *p, void *s, uint64_t ns, void *e, uint64_t ne, uint32_t rank,
+                        uint32_t world, void *stream) {
+  uint64_t m = ns > ne ? ns : ne;
+  remap_weak_kernel<<<grid_for(m), 256, 0, (cudaStream_t)stream>>>((gen_sample_rec *)s, ns, (gen_event_rec *)e, ne,
+                                                                   p->n_buffers, p->n_components,
+                                                                   p->buffers_per_comp, rank, world);
   return (int)cudaGetLastError();
 }
 

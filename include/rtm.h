@@ -1,0 +1,196 @@
+/*
+ * include/rtm.h — C ABI of the B200 monitoring-snapshot reducer (librtm.so).
+ *
+ * The reducer turns a stream of simulator trace records into the state a real-time
+ * monitor such as AkitaRTM shows (Mosallaei, Isaacs, Sun, "Looking into the Black Box:
+ * Monitoring Computer Architecture Simulations in Real-Time with AkitaRTM"; PAPER.md):
+ *   - the Bottleneck Analyzer buffer list: a snapshot of all buffers sorted by fullness
+ *     percentage or by number of elements (Fig. 3);
+ *   - buffer fullness over time: per buffer last / max / min level and the int64
+ *     time-weighted occupancy integral (L175-L181, L199);
+ *   - progress bars with finished / executing / not-started task counts (L91, L131);
+ *   - a hang flag for components whose buffers stay full while their task counts stop
+ *     changing (T3 L67-L71; case study 2 L227-L229).
+ * The paper gives no formula; the exact definition this library computes is DESIGN.md §2
+ * and every reading where the paper is silent is listed in DESIGN.md §3.  All integer
+ * outputs are bit-exact with the CPU oracle (oracle/); mean occupancy is one IEEE division.
+ *
+ * Conventions
+ *   - Every call returns rtm_status.  RTM_E_INVALID leaves all state unchanged.
+ *     RTM_E_ORDER / RTM_E_CUDA / RTM_E_STATE are sticky: every later call on the context
+ *     returns the same code until rtm_reset() or rtm_destroy().
+ *   - A context is bound to one CUDA device and one stream and is NOT thread-safe.
+ *   - Invalid records are not errors: they are dropped and counted (rtm_window_summary).
+ *   - The caller owns every array passed in or out.  Configuration tables are copied at
+ *     rtm_create.  Host output pointers must hold the documented number of elements.
+ *   - Memory: all device buffers are allocated with cudaMalloc on cfg->device at create
+ *     (registry, per-buffer / per-component state) or on first use and grown
+ *     (per-call workspaces); nothing is freed before rtm_destroy.
+ */
+#ifndef RTM_H
+#define RTM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct rtm_ctx rtm_ctx; /* opaque, owned by the library */
+
+typedef enum {
+  RTM_OK = 0,
+  RTM_E_INVALID = -1,   /* bad argument; no state change                                  */
+  RTM_E_CUDA = -2,      /* CUDA runtime failure (sticky)                                  */
+  RTM_E_COMM = -3,      /* cross-rank exchange callback failed (sticky)                   */
+  RTM_E_ORDER = -4,     /* field-valid records not non-decreasing in ts (sticky)           */
+  RTM_E_TOO_SMALL = -5, /* output capacity too small (no state change)                    */
+  RTM_E_STATE = -6,     /* call not valid in the current state (e.g. no reduce yet)        */
+  RTM_E_NOMEM = -7      /* device allocation failed (sticky)                              */
+} rtm_status;
+
+enum { RTM_MEM_HOST = 0, RTM_MEM_DEVICE = 1 };
+/* "sort the buffers by their fullness percentage or by the number of elements" */
+enum { RTM_RANK_PERCENT = 0, RTM_RANK_SIZE = 1 };
+
+/* ---- trace records (16 B each, little-endian, naturally aligned) --------------------------
+ * rtm_level_sample: buffer `buffer_id` holds `level` elements of `capacity` from tick ts on
+ *   (the "Size" and "Cap" columns of Fig. 3; ts is an integer simulation tick).
+ * rtm_task_event: START or END of one task (e.g. a thread block of a GPU kernel, L91, L131).
+ *   meta = component_id (bits 0..19) | kernel_id (bits 20..30) | kind (bit 31: 0 START, 1 END)
+ * Field-valid sample: buffer_id < n_buffers, capacity == registered capacity, level <= capacity.
+ * Field-valid event:  component_id < n_components, kernel_id < n_kernels.
+ * Ordering contract: within the records pending at one rtm_window_reduce call, the ts of
+ * field-valid samples is non-decreasing in ingest order, and likewise for field-valid events
+ * (reading R15).  A violation makes the call fail with RTM_E_ORDER (sticky).       */
+typedef struct {
+  int64_t ts;
+  uint32_t buffer_id;
+  uint16_t level;
+  uint16_t capacity;
+} rtm_level_sample;
+
+typedef struct {
+  int64_t ts;
+  uint32_t task_id;
+  uint32_t meta;
+} rtm_task_event;
+
+#define RTM_META(comp, kernel, kind) \
+  (((uint32_t)(comp) & 0xFFFFFu) | (((uint32_t)(kernel) & 0x7FFu) << 20) | ((uint32_t)(kind) << 31))
+
+/* Cross-rank exchange hook (world > 1): gather `bytes` from every rank's device buffer `send`
+ * into `recv` (world * bytes, rank-major) on the context's device; must be complete when it
+ * returns (the library synchronises its stream before calling).  Returns 0 on success.
+ * The Python binding implements it with torch.distributed.all_gather_into_tensor (NCCL). */
+typedef int (*rtm_allgather_fn)(void *user, const void *send, void *recv, uint64_t bytes);
+
+/* ---- configuration (≈ RegisterComponent + CreateProgressBar) ------------------ */
+typedef struct {
+  uint32_t n_buffers;               /* 1 .. 2^31-1                                             */
+  uint32_t n_components;            /* 1 .. 2^20                                               */
+  uint32_t n_kernels;               /* progress bars, 1 .. 2048                                */
+  const uint32_t *buffer_owner;     /* host [n_buffers]: owning component id                   */
+  const uint16_t *buffer_capacity;  /* host [n_buffers]: 1 .. 65534 (65535 is reserved)        */
+  const int64_t *kernel_total;      /* host [n_kernels]: planned tasks per bar                 */
+  int64_t t0;                       /* begin of the first window                               */
+  uint32_t hang_windows;            /* H >= 1: consecutive windows before a hang is flagged    */
+  uint32_t k;                       /* top-k computed for every window, 1 .. 1024              */
+  int32_t rank_mode;                /* RTM_RANK_PERCENT or RTM_RANK_SIZE                       */
+  int32_t device;                   /* CUDA device ordinal                                     */
+  int32_t rank, world;              /* world == 1: single GPU; else this context is one shard  */
+  const uint8_t *owned_components;  /* host [n_components] or NULL (= all): components whose
+                                       buffers and events this rank holds (ranking restricted) */
+  rtm_allgather_fn allgather;       /* required when world > 1                                 */
+  void *allgather_user;
+  void *stream;                     /* cudaStream_t to run on (NULL = the legacy default)      */
+} rtm_config;
+
+/* ---- per-window outputs --------------------------------------------------------------------- */
+typedef struct {
+  int64_t t_begin, t_end;           /* window [t_begin, t_end)                                 */
+  uint64_t n_samples, n_events;     /* kept records                                            */
+  uint64_t n_dropped;               /* dropped samples + events charged to this window         */
+  uint64_t digest;                  /* sum over touched buffers of the DESIGN.md §2 mixer      */
+  uint32_t n_touched, n_hung;       /* buffers with >= 1 kept sample; flagged components       */
+} rtm_window_summary;               /* 56 B */
+
+typedef struct { uint32_t buffer_id; uint16_t level, capacity; } rtm_topk_entry; /* Fig. 3 row */
+typedef struct { int64_t total, started, finished, in_flight, not_started; } rtm_progress_entry;
+typedef struct { int64_t started, finished, in_flight; } rtm_component_tasks;
+typedef struct {
+  int64_t integral;                 /* sum level*dt over the window (mod 2^64)                  */
+  uint16_t last, max, min, capacity;
+  uint32_t n_samples, reserved;
+  double mean_occ;                  /* (double)integral / (double)(capacity * (t_end-t_begin)) */
+} rtm_buffer_stat;                  /* 32 B */
+
+typedef struct {
+  const char *name;                 /* kernel name                                              */
+  uint32_t launches;                /* launches timed since rtm_profile(ctx, 1)                 */
+  double total_ms;                  /* summed CUDA-event durations on the context's stream      */
+  uint64_t algo_bytes;              /* algorithmic bytes those launches had to move             */
+} rtm_kernel_time;
+
+/* ---- API -------------------------------------------------------------------------------------- */
+/* Validate cfg, copy the registry to the device, allocate state (levels start at 0: buffers
+ * start empty, L229).  *out receives the context.  RTM_E_INVALID for out-of-range fields. */
+rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out);
+void rtm_destroy(rtm_ctx *ctx);
+/* Back to the state right after rtm_create (t_prev = t0, levels 0, counters 0, no error). */
+rtm_status rtm_reset(rtm_ctx *ctx);
+
+/* Append records to the pending stream of the next rtm_window_reduce (ingest order = call
+ * order, then array order).  mem = RTM_MEM_HOST: copied host->device now (pinned memory is
+ * copied asynchronously on the context stream).  mem = RTM_MEM_DEVICE: pointers on the
+ * context's device; a single device ingest is zero-copy and must stay valid until the next
+ * rtm_window_reduce returns; further device ingests are copied into an internal buffer.
+ * Either pointer may be NULL when its count is 0. */
+rtm_status rtm_ingest(rtm_ctx *ctx, const rtm_level_sample *samples, uint64_t n_samples,
+                      const rtm_task_event *events, uint64_t n_events, int32_t mem);
+
+/* THE HOT PATH.  Reduce all pending records over n_windows consecutive windows
+ * [t_prev, t_end[0]), [t_end[0], t_end[1]), ... (t_end host array, non-decreasing,
+ * t_end[0] >= t_prev, each window shorter than 2^40 ticks).  Records outside
+ * [t_prev, t_end[n-1]) are dropped and counted, not carried.  Blocks until the per-window
+ * summaries, top-k lists and progress bars are on the host; `out` (host, nullable)
+ * receives n_windows summaries.  With world > 1 every rank must call it with the same
+ * t_end (collective); all ranks then return identical merged results. */
+rtm_status rtm_window_reduce(rtm_ctx *ctx, const int64_t *t_end, uint32_t n_windows, rtm_window_summary *out);
+
+/* Results of the most recent rtm_window_reduce; `window` indexes its batch. */
+/* Bottleneck Analyzer list (L173): min(k, eligible buffers) entries, most occupied first,
+ * ties by buffer_id ascending.  out holds k entries. */
+rtm_status rtm_topk_buffers(rtm_ctx *ctx, uint32_t window, rtm_topk_entry *out, uint32_t *n_out);
+/* Progress bars after `window` (L131): bars[n_kernels].  comps[n_components] (nullable) is
+ * only available for the last window of the batch (else RTM_E_INVALID). */
+rtm_status rtm_progress(rtm_ctx *ctx, uint32_t window, rtm_progress_entry *bars, rtm_component_tasks *comps);
+/* Hang-flagged component ids of `window`, ascending.  Writes min(cap, n) ids; *n_hung = n. */
+rtm_status rtm_hang_check(rtm_ctx *ctx, uint32_t window, uint32_t *comp_ids, uint32_t cap, uint32_t *n_hung);
+/* Full per-buffer table of the last window of the batch for buffers [first, first+count). */
+rtm_status rtm_buffer_stats(rtm_ctx *ctx, uint32_t first, uint32_t count, rtm_buffer_stat *out);
+
+/* Bulk form of the three accessors above for windows [first, first+count) of the last batch:
+ * topk[count*k] + topk_n[count], bars[count*n_kernels], summaries[count]; each nullable. */
+rtm_status rtm_window_results(rtm_ctx *ctx, uint32_t first, uint32_t count, rtm_window_summary *summaries,
+                              rtm_topk_entry *topk, uint32_t *topk_n, rtm_progress_entry *bars);
+
+/* Two-phase form of rtm_window_reduce for callers that run the exchange themselves:
+ * reduce_local computes this rank's results and packs them; *pack / *pack_bytes give the
+ * device buffer to all-gather; rtm_merge consumes world*pack_bytes gathered bytes (device). */
+rtm_status rtm_window_reduce_local(rtm_ctx *ctx, const int64_t *t_end, uint32_t n_windows,
+                                   const void **pack, uint64_t *pack_bytes);
+rtm_status rtm_merge(rtm_ctx *ctx, const void *gathered, uint32_t world, rtm_window_summary *out);
+
+/* Per-kernel CUDA-event timing on the context stream (off by default). */
+rtm_status rtm_profile(rtm_ctx *ctx, int32_t enable);
+rtm_status rtm_profile_read(rtm_ctx *ctx, rtm_kernel_time *out, uint32_t cap, uint32_t *n);
+
+const char *rtm_status_str(rtm_status s);
+/* Build identification string ("librtm sm_100a ..."). */
+const char *rtm_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RTM_H */

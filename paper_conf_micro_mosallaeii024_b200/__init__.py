@@ -1,0 +1,221 @@
+"""B200-native monitoring-snapshot reducer (AkitaRTM's dashboard state, §IV-C).
+
+Thin Python binding over the C ABI in ``include/rtm.h`` (``librtm.so``, sm_100a CUDA).  Every
+step of the reduction runs in the library's kernels; this module only marshals arguments and
+uses PyTorch for device memory, streams and ``torch.distributed`` plumbing.
+
+    mon = Monitor(owner, capacity, kernel_total, n_components=C, t0=0, hang_windows=8, k=64)
+    mon.ingest(samples_dev, events_dev)          # torch uint8/structured tensors on cuda, or numpy
+    res = mon.window_reduce(t_end)               # per-window summaries, top-k, progress bars
+    mon.hang_check(w); mon.buffer_stats(); mon.progress(w, comps=True)
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+
+from . import _native as N
+from ._native import (BSTAT_DTYPE, COMP_DTYPE, EVENT_DTYPE, PROGRESS_DTYPE, RTM_RANK_PERCENT, RTM_RANK_SIZE,
+                      SAMPLE_DTYPE, SUMMARY_DTYPE, TOPK_DTYPE, RTMError)
+
+__all__ = ["Monitor", "RTMError", "SAMPLE_DTYPE", "EVENT_DTYPE", "SUMMARY_DTYPE", "TOPK_DTYPE", "PROGRESS_DTYPE",
+           "COMP_DTYPE", "BSTAT_DTYPE", "RTM_RANK_PERCENT", "RTM_RANK_SIZE", "version"]
+
+N.lib()  # fail at import time if the native library is missing
+
+
+def version() -> str:
+    return N.lib().rtm_version().decode()
+
+
+def _records(x, dtype):
+    """(pointer, count, mem, keepalive) for a torch tensor (cuda/cpu) or a numpy array of 16-B records."""
+    if x is None:
+        return None, 0, N.RTM_MEM_DEVICE, None
+    if isinstance(x, np.ndarray):
+        a = np.ascontiguousarray(x)
+        nbytes = a.nbytes
+        if nbytes % 16:
+            raise ValueError("record arrays must hold whole 16-byte records")
+        return a.ctypes.data, nbytes // 16, N.RTM_MEM_HOST, a
+    import torch
+
+    if not isinstance(x, torch.Tensor):
+        raise TypeError("records must be a numpy array or a torch tensor")
+    if not x.is_contiguous():
+        raise ValueError("record tensor must be contiguous")
+    nbytes = x.numel() * x.element_size()
+    if nbytes % 16:
+        raise ValueError("record tensors must hold whole 16-byte records")
+    mem = N.RTM_MEM_DEVICE if x.is_cuda else N.RTM_MEM_HOST
+    return x.data_ptr(), nbytes // 16, mem, x
+
+
+class Monitor:
+    """One reducer context (rtm_create).  Not thread-safe; bound to one device and stream."""
+
+    def __init__(self, buffer_owner, buffer_capacity, kernel_total, *, n_components: int, t0: int = 0,
+                 hang_windows: int = 8, k: int = 64, rank_mode: int = RTM_RANK_PERCENT, device: int = 0,
+                 rank: int = 0, world: int = 1, owned_components=None, stream=None, process_group=None):
+        import torch
+
+        if not torch.cuda.is_available():
+            raise RuntimeError("Monitor needs a CUDA device (sm_100a); there is no CPU fallback")
+        self._owner = np.ascontiguousarray(buffer_owner, dtype=np.uint32)
+        self._cap = np.ascontiguousarray(buffer_capacity, dtype=np.uint16)
+        self._tot = np.ascontiguousarray(kernel_total, dtype=np.int64)
+        self._owned = None if owned_components is None else np.ascontiguousarray(owned_components, dtype=np.uint8)
+        self.n_buffers, self.n_components, self.n_kernels = len(self._owner), int(n_components), len(self._tot)
+        self.k, self.device, self.rank, self.world = int(k), int(device), int(rank), int(world)
+        self._pg = process_group
+        with torch.cuda.device(device):
+            self._stream = stream if stream is not None else torch.cuda.current_stream(device)
+        cfg = N.Config()
+        cfg.n_buffers, cfg.n_components, cfg.n_kernels = self.n_buffers, self.n_components, self.n_kernels
+        cfg.buffer_owner, cfg.buffer_capacity = self._owner.ctypes.data, self._cap.ctypes.data
+        cfg.kernel_total = self._tot.ctypes.data
+        cfg.t0, cfg.hang_windows, cfg.k, cfg.rank_mode = int(t0), int(hang_windows), self.k, int(rank_mode)
+        cfg.device, cfg.rank, cfg.world = self.device, self.rank, self.world
+        cfg.owned_components = None if self._owned is None else self._owned.ctypes.data
+        cfg.allgather = N.ALLGATHER_FN()  # the binding runs the exchange itself (two-phase API)
+        cfg.stream = self._stream.cuda_stream
+        h = ctypes.c_void_p()
+        N.check(N.lib().rtm_create(ctypes.byref(cfg), ctypes.byref(h)), "rtm_create")
+        self._h = h
+        self._keep = []
+        self.W = 0
+
+    # ------------------------------------------------------------------------------------------
+    def close(self):
+        if getattr(self, "_h", None):
+            N.lib().rtm_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def reset(self):
+        N.check(N.lib().rtm_reset(self._h), "rtm_reset")
+        self._keep = []
+
+    def ingest(self, samples=None, events=None):
+        sp, sn, sm, ska = _records(samples, SAMPLE_DTYPE)
+        ep, en, em, eka = _records(events, EVENT_DTYPE)
+        if sn and en and sm != em:
+            self.ingest(samples, None)
+            self.ingest(None, events)
+            return
+        mem = sm if sn else em
+        N.check(N.lib().rtm_ingest(self._h, sp, sn, ep, en, mem), "rtm_ingest")
+        self._keep.extend([ska, eka])  # zero-copy device chunks must outlive the next reduce
+
+    def window_reduce(self, t_end):
+        """THE hot path: reduce all pending records over len(t_end) windows (blocking)."""
+        t_end = np.ascontiguousarray(t_end, dtype=np.int64)
+        W = len(t_end)
+        summ = np.zeros(W, SUMMARY_DTYPE)
+        if self.world > 1:
+            self._reduce_distributed(t_end, summ)
+        else:
+            N.check(N.lib().rtm_window_reduce(self._h, t_end.ctypes.data, W, summ.ctypes.data), "rtm_window_reduce")
+        self._keep = []
+        self.W = W
+        return self.results(W)
+
+    def results(self, W=None):
+        """All per-window results of the last batch (one rtm_window_results call)."""
+        W = self.W if W is None else W
+        summ = np.zeros(W, SUMMARY_DTYPE)
+        topk = np.zeros((W, self.k), TOPK_DTYPE)
+        topk_n = np.zeros(W, np.uint32)
+        bars = np.zeros((W, self.n_kernels), PROGRESS_DTYPE)
+        N.check(N.lib().rtm_window_results(self._h, 0, W, summ.ctypes.data, topk.ctypes.data, topk_n.ctypes.data,
+                                           bars.ctypes.data), "rtm_window_results")
+        return {"summary": summ, "topk": topk, "topk_n": topk_n, "progress": bars}
+
+    def _reduce_distributed(self, t_end, summ):
+        """world > 1: local reduce -> all-gather of the packed per-window results -> merge kernels."""
+        import torch
+        import torch.distributed as dist
+
+        pack = ctypes.c_void_p()
+        nbytes = ctypes.c_uint64()
+        N.check(N.lib().rtm_window_reduce_local(self._h, t_end.ctypes.data, len(t_end), ctypes.byref(pack),
+                                                ctypes.byref(nbytes)), "rtm_window_reduce_local")
+        n = int(nbytes.value)
+        dev = torch.device("cuda", self.device)
+        send = torch.empty(n, dtype=torch.uint8, device=dev)
+        _copy_from_ptr(send, pack.value, n)
+        recv = torch.empty(self.world * n, dtype=torch.uint8, device=dev)
+        dist.all_gather_into_tensor(recv, send, group=self._pg)
+        torch.cuda.current_stream(dev).synchronize()
+        N.check(N.lib().rtm_merge(self._h, recv.data_ptr(), self.world, summ.ctypes.data), "rtm_merge")
+
+    def topk(self, window: int):
+        out = np.zeros(self.k, TOPK_DTYPE)
+        n = ctypes.c_uint32()
+        N.check(N.lib().rtm_topk_buffers(self._h, window, out.ctypes.data, ctypes.byref(n)), "rtm_topk_buffers")
+        return out[: n.value]
+
+    def progress(self, window: int, comps: bool = False):
+        bars = np.zeros(self.n_kernels, PROGRESS_DTYPE)
+        cs = np.zeros(self.n_components, COMP_DTYPE) if comps else None
+        N.check(N.lib().rtm_progress(self._h, window, bars.ctypes.data, None if cs is None else cs.ctypes.data),
+                "rtm_progress")
+        return (bars, cs) if comps else bars
+
+    def hang_check(self, window: int):
+        n = ctypes.c_uint32()
+        N.check(N.lib().rtm_hang_check(self._h, window, None, 0, ctypes.byref(n)), "rtm_hang_check")
+        ids = np.zeros(max(1, n.value), np.uint32)
+        N.check(N.lib().rtm_hang_check(self._h, window, ids.ctypes.data, len(ids), ctypes.byref(n)),
+                "rtm_hang_check")
+        return ids[: n.value]
+
+    def buffer_stats(self, first: int = 0, count: int | None = None):
+        if count is None:
+            count = self.n_buffers - first
+        out = np.zeros(count, BSTAT_DTYPE)
+        N.check(N.lib().rtm_buffer_stats(self._h, first, count, out.ctypes.data), "rtm_buffer_stats")
+        return out
+
+    def profile(self, enable: bool = True):
+        N.check(N.lib().rtm_profile(self._h, 1 if enable else 0), "rtm_profile")
+
+    def profile_read(self):
+        arr = (N.KernelTime * 32)()
+        n = ctypes.c_uint32()
+        N.check(N.lib().rtm_profile_read(self._h, arr, 32, ctypes.byref(n)), "rtm_profile_read")
+        return {arr[i].name.decode(): dict(launches=arr[i].launches, total_ms=arr[i].total_ms,
+                                           algo_bytes=arr[i].algo_bytes) for i in range(min(n.value, 32))}
+
+
+_cudart = None
+
+
+def _copy_from_ptr(dst_tensor, src_ptr: int, nbytes: int):
+    """Device-to-device copy from a raw library pointer into a torch tensor (exchange plumbing)."""
+    global _cudart
+    import torch
+
+    if _cudart is None:
+        _cudart = ctypes.CDLL("libcudart.so.12") if _try("libcudart.so.12") else ctypes.CDLL("libcudart.so")
+        _cudart.cudaMemcpyAsync.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int,
+                                            ctypes.c_void_p]
+        _cudart.cudaMemcpyAsync.restype = ctypes.c_int
+    st = torch.cuda.current_stream(dst_tensor.device)
+    err = _cudart.cudaMemcpyAsync(dst_tensor.data_ptr(), src_ptr, nbytes, 3, st.cuda_stream)
+    if err != 0:
+        raise RuntimeError(f"cudaMemcpyAsync failed: {err}")
+
+
+def _try(name):
+    try:
+        ctypes.CDLL(name)
+        return True
+    except OSError:
+        return False

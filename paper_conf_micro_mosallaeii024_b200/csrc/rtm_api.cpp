@@ -1,0 +1,765 @@
+// rtm_api.cpp — C ABI of librtm (include/rtm.h): context, ingest, the window-reduce
+// orchestration on one CUDA stream, result accessors and the multi-rank exchange.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "rtm.h"
+#include "rtm_internal.h"
+
+using namespace rtm;
+
+namespace {
+
+struct DevBuf {
+  void *p = nullptr;
+  size_t cap = 0;
+};
+
+struct Pinned {
+  void *p = nullptr;
+  size_t cap = 0;
+};
+
+struct Chunk {
+  const void *ptr;
+  uint64_t n;
+};
+
+enum KernelId { KT_SPLIT, KT_PARTITION, KT_EVENTS, KT_FOLD, KT_ORDER, KT_TOPK, KT_HANG, KT_PROGRESS, KT_MERGE, KT_N };
+const char *kKernelNames[KT_N] = {"k_split", "k_partition", "k_events", "k_fold", "k_order_check",
+                                  "k_topk", "k_hang", "k_progress", "k_merge"};
+
+}  // namespace
+
+struct rtm_ctx {
+  // registry
+  uint32_t nb, nc, nk, nbins, ncw, k, H;
+  int32_t rank_mode, device, rank, world;
+  int64_t t0;
+  rtm_allgather_fn allgather;
+  void *allgather_user;
+  cudaStream_t st;
+  int n_sms;
+  DevBuf cap, owner, elig, ktotal;
+  // persistent state
+  DevBuf carry[2];
+  int cur = 0;
+  DevBuf run, kstart, kend, cstart, cend, flags;
+  uint32_t epoch = 1;
+  int64_t t_prev;
+  int sticky = 0;
+  // pending stream
+  std::vector<Chunk> s_dev, e_dev;  // zero-copy device chunks
+  DevBuf s_own, e_own;              // internal concatenation
+  uint64_t s_own_n = 0, e_own_n = 0;
+  // per-call workspaces
+  DevBuf T, Bs, Be, rts, rte, treg_s, treg_e, soff, stage, smeta, emeta, lastlvl, win, kdelta, cdelta, active,
+      anyfull, hung, unit_ctr, status, topk, topk_n, prog, bstat, comps, pack, gathered;
+  Pinned h_small, h_res;
+  // results of the last call
+  bool have = false;
+  uint32_t W = 0;
+  std::vector<rtm_window_summary> sum;
+  std::vector<unsigned long long> topk_h;
+  std::vector<uint32_t> topk_n_h;
+  std::vector<rtm_progress_entry> prog_h;
+  std::vector<int64_t> t_end_h;
+  // profiling
+  bool prof = false;
+  KernelTimer timers[KT_N];
+  std::vector<cudaEvent_t> ev_pool;
+  struct Mark { int kid; cudaEvent_t a, b; uint64_t bytes; };
+  std::vector<Mark> marks;
+  size_t ev_next = 0;
+};
+
+namespace {
+
+rtm_status cuda_fail(rtm_ctx *c, cudaError_t e) {
+  (void)e;
+  cudaGetLastError();
+  if (c) c->sticky = RTM_E_CUDA;
+  return RTM_E_CUDA;
+}
+
+#define CK(call)                                     \
+  do {                                               \
+    cudaError_t e_ = (call);                         \
+    if (e_ != cudaSuccess) return cuda_fail(c, e_);  \
+  } while (0)
+
+rtm_status ensure(rtm_ctx *c, DevBuf &b, size_t bytes, bool zero_new = false) {
+  if (bytes == 0) bytes = 8;
+  if (b.cap >= bytes) return RTM_OK;
+  if (b.p) cudaFree(b.p);
+  b.p = nullptr;
+  b.cap = 0;
+  size_t want = bytes + bytes / 4;
+  cudaError_t e = cudaMalloc(&b.p, want);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    e = cudaMalloc(&b.p, bytes);
+    want = bytes;
+  }
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    b.p = nullptr;
+    c->sticky = RTM_E_NOMEM;
+    return RTM_E_NOMEM;
+  }
+  b.cap = want;
+  if (zero_new && cudaMemset(b.p, 0, want) != cudaSuccess) return cuda_fail(c, cudaGetLastError());
+  return RTM_OK;
+}
+
+// grow keeping the first `keep` bytes (used for the ingest concatenation buffer)
+rtm_status grow_keep(rtm_ctx *c, DevBuf &b, size_t bytes, size_t keep) {
+  if (b.cap >= bytes) return RTM_OK;
+  size_t want = std::max(bytes + bytes / 2, (size_t)1 << 20);
+  void *np = nullptr;
+  if (cudaMalloc(&np, want) != cudaSuccess) {
+    cudaGetLastError();
+    c->sticky = RTM_E_NOMEM;
+    return RTM_E_NOMEM;
+  }
+  if (keep) CK(cudaMemcpyAsync(np, b.p, keep, cudaMemcpyDeviceToDevice, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  if (b.p) cudaFree(b.p);
+  b.p = np;
+  b.cap = want;
+  return RTM_OK;
+}
+
+rtm_status ensure_pinned(rtm_ctx *c, Pinned &h, size_t bytes) {
+  if (h.cap >= bytes) return RTM_OK;
+  if (h.p) cudaFreeHost(h.p);
+  h.p = nullptr;
+  size_t want = std::max(bytes + bytes / 4, (size_t)1 << 16);
+  if (cudaMallocHost(&h.p, want) != cudaSuccess) {
+    cudaGetLastError();
+    h.cap = 0;
+    c->sticky = RTM_E_NOMEM;
+    return RTM_E_NOMEM;
+  }
+  h.cap = want;
+  return RTM_OK;
+}
+
+void prof_begin(rtm_ctx *c, int kid, uint64_t bytes) {
+  if (!c->prof) return;
+  if (c->ev_next + 2 > c->ev_pool.size()) {
+    for (int i = 0; i < 32; ++i) {
+      cudaEvent_t e;
+      cudaEventCreate(&e);
+      c->ev_pool.push_back(e);
+    }
+  }
+  rtm_ctx::Mark m;
+  m.kid = kid;
+  m.a = c->ev_pool[c->ev_next++];
+  m.b = c->ev_pool[c->ev_next++];
+  m.bytes = bytes;
+  cudaEventRecord(m.a, c->st);
+  c->marks.push_back(m);
+}
+void prof_end(rtm_ctx *c) {
+  if (!c->prof || c->marks.empty()) return;
+  cudaEventRecord(c->marks.back().b, c->st);
+}
+void prof_collect(rtm_ctx *c) {  // after a stream sync
+  for (auto &m : c->marks) {
+    float ms = 0;
+    if (cudaEventElapsedTime(&ms, m.a, m.b) == cudaSuccess) {
+      c->timers[m.kid].launches++;
+      c->timers[m.kid].total_ms += ms;
+      c->timers[m.kid].algo_bytes += m.bytes;
+    } else {
+      cudaGetLastError();
+    }
+  }
+  c->marks.clear();
+  c->ev_next = 0;
+}
+
+#define LAUNCH(kid, bytes, stmt) \
+  do {                           \
+    prof_begin(c, kid, bytes);   \
+    stmt;                        \
+    prof_end(c);                 \
+  } while (0)
+
+void free_buf(DevBuf &b) {
+  if (b.p) cudaFree(b.p);
+  b.p = nullptr;
+  b.cap = 0;
+}
+
+rtm_status zero_state(rtm_ctx *c) {
+  CK(cudaMemsetAsync(c->carry[0].p, 0, (size_t)c->nb * 2, c->st));
+  CK(cudaMemsetAsync(c->carry[1].p, 0, (size_t)c->nb * 2, c->st));
+  CK(cudaMemsetAsync(c->run.p, 0, (size_t)c->nc * 4, c->st));
+  CK(cudaMemsetAsync(c->kstart.p, 0, (size_t)c->nk * 8, c->st));
+  CK(cudaMemsetAsync(c->kend.p, 0, (size_t)c->nk * 8, c->st));
+  CK(cudaMemsetAsync(c->cstart.p, 0, (size_t)c->nc * 8, c->st));
+  CK(cudaMemsetAsync(c->cend.p, 0, (size_t)c->nc * 8, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  c->cur = 0;
+  c->t_prev = c->t0;
+  c->have = false;
+  c->W = 0;
+  c->s_dev.clear();
+  c->e_dev.clear();
+  c->s_own_n = c->e_own_n = 0;
+  return RTM_OK;
+}
+
+// Pending stream of one kind as a single device array.
+void pending(const std::vector<Chunk> &dev, const DevBuf &own, uint64_t own_n, const void **ptr, uint64_t *n) {
+  if (own_n) { *ptr = own.p; *n = own_n; }
+  else if (!dev.empty()) { *ptr = dev[0].ptr; *n = dev[0].n; }
+  else { *ptr = nullptr; *n = 0; }
+}
+
+rtm_status append(rtm_ctx *c, std::vector<Chunk> &dev, DevBuf &own, uint64_t &own_n, const void *src, uint64_t n,
+                  int32_t mem) {
+  if (n == 0) return RTM_OK;
+  const size_t rec = 16;
+  if (mem == RTM_MEM_DEVICE && dev.empty() && own_n == 0) {
+    dev.push_back({src, n});  // zero-copy
+    return RTM_OK;
+  }
+  // move a pending zero-copy chunk into the internal buffer first
+  if (!dev.empty()) {
+    rtm_status s = grow_keep(c, own, (size_t)(own_n + dev[0].n) * rec, (size_t)own_n * rec);
+    if (s) return s;
+    CK(cudaMemcpyAsync((char *)own.p + own_n * rec, dev[0].ptr, dev[0].n * rec, cudaMemcpyDeviceToDevice, c->st));
+    own_n += dev[0].n;
+    dev.clear();
+  }
+  rtm_status s = grow_keep(c, own, (size_t)(own_n + n) * rec, (size_t)own_n * rec);
+  if (s) return s;
+  CK(cudaMemcpyAsync((char *)own.p + own_n * rec, src, n * rec,
+                     mem == RTM_MEM_DEVICE ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, c->st));
+  own_n += n;
+  return RTM_OK;
+}
+
+// Host-side region/tile bookkeeping from the split positions.
+uint32_t regions_to_tiles(std::vector<long long> &B, uint64_t N, uint32_t W, int tile, std::vector<uint32_t> &rt) {
+  B[0] = 0;
+  B[W + 2] = (long long)N;
+  for (uint32_t r = 1; r <= W + 2; ++r) {
+    if (B[r] < B[r - 1]) B[r] = B[r - 1];  // only for unsorted input (reported as RTM_E_ORDER)
+    if (B[r] > (long long)N) B[r] = (long long)N;
+  }
+  rt.assign(W + 3, 0);
+  uint32_t t = 0;
+  for (uint32_t r = 0; r <= W + 1; ++r) {
+    rt[r] = t;
+    t += (uint32_t)((B[r + 1] - B[r] + tile - 1) / tile);
+  }
+  rt[W + 2] = t;
+  return t;
+}
+
+// The local (per-rank) part of a reduce call.  On success the device result arrays hold this
+// rank's per-window results for n_windows windows.
+rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p) {
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (!t_end || W == 0) return RTM_E_INVALID;
+  if (t_end[0] < c->t_prev) return RTM_E_INVALID;
+  if (t_end[0] - c->t_prev >= kMaxWindowLen) return RTM_E_INVALID;
+  for (uint32_t w = 1; w < W; ++w)
+    if (t_end[w] < t_end[w - 1] || t_end[w] - t_end[w - 1] >= kMaxWindowLen) return RTM_E_INVALID;
+  CK(cudaSetDevice(c->device));
+
+  const void *sp, *ep;
+  uint64_t ns, ne;
+  pending(c->s_dev, c->s_own, c->s_own_n, &sp, &ns);
+  pending(c->e_dev, c->e_own, c->e_own_n, &ep, &ne);
+
+  rtm_status s;
+  // ---- window bounds T[0..W] and split positions
+  if ((s = ensure(c, c->T, (size_t)(W + 1) * 8))) return s;
+  if ((s = ensure(c, c->Bs, (size_t)(W + 3) * 8))) return s;
+  if ((s = ensure(c, c->Be, (size_t)(W + 3) * 8))) return s;
+  if ((s = ensure(c, c->rts, (size_t)(W + 3) * 4))) return s;
+  if ((s = ensure(c, c->rte, (size_t)(W + 3) * 4))) return s;
+  const size_t small = (size_t)(W + 3) * 8 * 2 + (size_t)(W + 3) * 4 * 2 + (size_t)(W + 1) * 8;
+  if ((s = ensure_pinned(c, c->h_small, small))) return s;
+  long long *hT = (long long *)c->h_small.p;
+  long long *hBs = hT + (W + 1);
+  long long *hBe = hBs + (W + 3);
+  uint32_t *hrts = (uint32_t *)(hBe + (W + 3));
+  uint32_t *hrte = hrts + (W + 3);
+  hT[0] = c->t_prev;
+  for (uint32_t w = 0; w < W; ++w) hT[w + 1] = t_end[w];
+  CK(cudaMemcpyAsync(c->T.p, hT, (size_t)(W + 1) * 8, cudaMemcpyHostToDevice, c->st));
+
+  memset(&p, 0, sizeof(p));
+  p.nb = c->nb; p.nc = c->nc; p.nk = c->nk; p.nbins = c->nbins; p.ncw = c->ncw; p.k = c->k;
+  p.rank_mode = c->rank_mode; p.H = c->H;
+  p.cap = (const uint16_t *)c->cap.p; p.owner = (const uint32_t *)c->owner.p;
+  p.elig = (const uint8_t *)c->elig.p; p.ktotal = (const int64_t *)c->ktotal.p;
+  p.W = W; p.epoch = c->epoch;
+  p.T = (const long long *)c->T.p;
+  p.s = (const rtm_level_sample *)sp; p.ns = ns;
+  p.e = (const rtm_task_event *)ep; p.ne = ne;
+
+  LAUNCH(KT_SPLIT, 0, launch_split(p, true, (long long *)c->Bs.p + 1, c->st));
+  LAUNCH(KT_SPLIT, 0, launch_split(p, false, (long long *)c->Be.p + 1, c->st));
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(hBs + 1, (long long *)c->Bs.p + 1, (size_t)(W + 1) * 8, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaMemcpyAsync(hBe + 1, (long long *)c->Be.p + 1, (size_t)(W + 1) * 8, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  std::vector<long long> Bs(hBs, hBs + W + 3), Be(hBe, hBe + W + 3);
+  std::vector<uint32_t> rts, rte;
+  const uint32_t nts = regions_to_tiles(Bs, ns, W, kTileS, rts);
+  const uint32_t nte = regions_to_tiles(Be, ne, W, kTileE, rte);
+  memcpy(hBs, Bs.data(), (W + 3) * 8);
+  memcpy(hBe, Be.data(), (W + 3) * 8);
+  memcpy(hrts, rts.data(), (W + 3) * 4);
+  memcpy(hrte, rte.data(), (W + 3) * 4);
+  CK(cudaMemcpyAsync(c->Bs.p, hBs, (size_t)(W + 3) * 8, cudaMemcpyHostToDevice, c->st));
+  CK(cudaMemcpyAsync(c->Be.p, hBe, (size_t)(W + 3) * 8, cudaMemcpyHostToDevice, c->st));
+  CK(cudaMemcpyAsync(c->rts.p, hrts, (size_t)(W + 3) * 4, cudaMemcpyHostToDevice, c->st));
+  CK(cudaMemcpyAsync(c->rte.p, hrte, (size_t)(W + 3) * 4, cudaMemcpyHostToDevice, c->st));
+
+  // ---- workspaces
+  const size_t Wn = W;
+  if ((s = ensure(c, c->treg_s, (size_t)nts * 4))) return s;
+  if ((s = ensure(c, c->treg_e, (size_t)nte * 4))) return s;
+  if ((s = ensure(c, c->soff, (size_t)nts * (c->nbins + 1) * 4))) return s;
+  if ((s = ensure(c, c->stage, (size_t)nts * kTileS * 8))) return s;
+  if ((s = ensure(c, c->smeta, (size_t)nts * sizeof(TileMeta)))) return s;
+  if ((s = ensure(c, c->emeta, (size_t)nte * sizeof(TileMeta)))) return s;
+  if ((s = ensure(c, c->lastlvl, Wn * c->nb * 2))) return s;
+  if (c->flags.cap < Wn * c->nbins * 4) {
+    if ((s = ensure(c, c->flags, Wn * c->nbins * 4, true))) return s;
+  }
+  if ((s = ensure(c, c->win, (size_t)kWinFields * Wn * 8))) return s;
+  if ((s = ensure(c, c->kdelta, Wn * c->nk * 2 * 4))) return s;
+  if ((s = ensure(c, c->cdelta, (size_t)c->nc * 2 * 8))) return s;
+  if ((s = ensure(c, c->active, Wn * c->ncw * 4))) return s;
+  if ((s = ensure(c, c->anyfull, Wn * c->ncw * 4))) return s;
+  if ((s = ensure(c, c->hung, Wn * c->ncw * 4))) return s;
+  if ((s = ensure(c, c->unit_ctr, 8))) return s;
+  if ((s = ensure(c, c->status, 8))) return s;
+  if ((s = ensure(c, c->topk, Wn * c->k * 8))) return s;
+  if ((s = ensure(c, c->topk_n, Wn * 4))) return s;
+  if ((s = ensure(c, c->prog, Wn * c->nk * 5 * 8))) return s;
+  if ((s = ensure(c, c->bstat, (size_t)c->nb * sizeof(rtm_buffer_stat)))) return s;
+  if ((s = ensure(c, c->comps, (size_t)c->nc * sizeof(rtm_component_tasks)))) return s;
+
+  CK(cudaMemsetAsync(c->win.p, 0, (size_t)kWinFields * Wn * 8, c->st));
+  CK(cudaMemsetAsync(c->kdelta.p, 0, Wn * c->nk * 2 * 4, c->st));
+  CK(cudaMemsetAsync(c->cdelta.p, 0, (size_t)c->nc * 2 * 8, c->st));
+  CK(cudaMemsetAsync(c->active.p, 0, Wn * c->ncw * 4, c->st));
+  CK(cudaMemsetAsync(c->anyfull.p, 0, Wn * c->ncw * 4, c->st));
+  CK(cudaMemsetAsync(c->unit_ctr.p, 0, 8, c->st));
+  CK(cudaMemsetAsync(c->status.p, 0, 8, c->st));
+
+  p.Bs = (const long long *)c->Bs.p; p.Be = (const long long *)c->Be.p;
+  p.rts = (const uint32_t *)c->rts.p; p.rte = (const uint32_t *)c->rte.p;
+  p.tile_reg_s = (const uint32_t *)c->treg_s.p; p.tile_reg_e = (const uint32_t *)c->treg_e.p;
+  p.n_tiles_s = nts; p.n_tiles_e = nte;
+  p.soff = (uint32_t *)c->soff.p; p.stage = (unsigned long long *)c->stage.p;
+  p.smeta = (TileMeta *)c->smeta.p; p.emeta = (TileMeta *)c->emeta.p;
+  p.lastlvl = (uint16_t *)c->lastlvl.p; p.flags = (uint32_t *)c->flags.p;
+  p.win = (unsigned long long *)c->win.p; p.kdelta = (uint32_t *)c->kdelta.p;
+  p.cdelta = (unsigned long long *)c->cdelta.p; p.active = (uint32_t *)c->active.p;
+  p.anyfull = (uint32_t *)c->anyfull.p; p.hung = (uint32_t *)c->hung.p;
+  p.unit_ctr = (uint32_t *)c->unit_ctr.p; p.status = (uint32_t *)c->status.p;
+  p.carry_in = (const uint16_t *)c->carry[c->cur].p; p.carry_out = (uint16_t *)c->carry[c->cur ^ 1].p;
+  p.run = (uint32_t *)c->run.p;
+  p.kstart = (long long *)c->kstart.p; p.kend = (long long *)c->kend.p;
+  p.cstart = (long long *)c->cstart.p; p.cend = (long long *)c->cend.p;
+  p.topk = (unsigned long long *)c->topk.p; p.topk_n = (uint32_t *)c->topk_n.p;
+  p.prog = (long long *)c->prog.p; p.bstat = (rtm_buffer_stat *)c->bstat.p;
+  p.comps = (rtm_component_tasks *)c->comps.p;
+
+  launch_fill_tile_regions(p, c->st);
+  LAUNCH(KT_PARTITION, (uint64_t)ns * 16, launch_partition(p, c->st));
+  LAUNCH(KT_EVENTS, (uint64_t)ne * 16, launch_events(p, c->st));
+  LAUNCH(KT_FOLD, 0, launch_fold(p, c->n_sms, c->st));
+  LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
+  LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
+  LAUNCH(KT_HANG, 0, launch_hang(p, c->st));
+  LAUNCH(KT_PROGRESS, 0, launch_progress(p, c->st));
+  CK(cudaGetLastError());
+  return RTM_OK;
+}
+
+// D2H of the per-window results and bookkeeping after a (local or merged) reduce.
+rtm_status finish(rtm_ctx *c, const int64_t *t_end, uint32_t W, rtm_window_summary *out) {
+  const size_t Wn = W;
+  const size_t bytes = (size_t)kWinFields * Wn * 8 + Wn * c->k * 8 + Wn * 4 + Wn * c->nk * 5 * 8 + 16;
+  rtm_status s;
+  if ((s = ensure_pinned(c, c->h_res, bytes))) return s;
+  char *h = (char *)c->h_res.p;
+  unsigned long long *hwin = (unsigned long long *)h;
+  unsigned long long *htopk = hwin + kWinFields * Wn;
+  long long *hprog = (long long *)(htopk + Wn * c->k);
+  uint32_t *htopk_n = (uint32_t *)(hprog + Wn * c->nk * 5);
+  uint32_t *hstatus = htopk_n + Wn;
+  CK(cudaMemcpyAsync(hwin, c->win.p, (size_t)kWinFields * Wn * 8, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaMemcpyAsync(htopk, c->topk.p, Wn * c->k * 8, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaMemcpyAsync(hprog, c->prog.p, Wn * c->nk * 5 * 8, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaMemcpyAsync(htopk_n, c->topk_n.p, Wn * 4, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaMemcpyAsync(hstatus, c->status.p, 4, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  prof_collect(c);
+  if (*hstatus & 4u) {  // look-back wait timed out: internal error, never expected
+    c->sticky = RTM_E_CUDA;
+    return RTM_E_CUDA;
+  }
+  if (*hstatus) {
+    c->sticky = RTM_E_ORDER;
+    return RTM_E_ORDER;
+  }
+  c->sum.resize(Wn);
+  c->t_end_h.assign(t_end, t_end + W);
+  for (uint32_t w = 0; w < W; ++w) {
+    rtm_window_summary &S = c->sum[w];
+    S.t_begin = w ? t_end[w - 1] : c->t_prev;
+    S.t_end = t_end[w];
+    S.n_samples = hwin[WF_SAMPLES * Wn + w];
+    S.n_events = hwin[WF_EVENTS * Wn + w];
+    S.n_dropped = hwin[WF_DROPPED * Wn + w];
+    S.digest = hwin[WF_DIGEST * Wn + w];
+    S.n_touched = (uint32_t)hwin[WF_TOUCHED * Wn + w];
+    S.n_hung = (uint32_t)hwin[WF_HUNG * Wn + w];
+  }
+  c->topk_h.assign(htopk, htopk + Wn * c->k);
+  c->topk_n_h.assign(htopk_n, htopk_n + Wn);
+  c->prog_h.resize(Wn * c->nk);
+  memcpy(c->prog_h.data(), hprog, Wn * c->nk * 5 * 8);
+  if (out) memcpy(out, c->sum.data(), Wn * sizeof(rtm_window_summary));
+  c->t_prev = t_end[W - 1];
+  c->cur ^= 1;
+  c->epoch = c->epoch == 0xFFFFFFFFu ? 1u : c->epoch + 1u;
+  c->have = true;
+  c->W = W;
+  c->s_dev.clear();
+  c->e_dev.clear();
+  c->s_own_n = c->e_own_n = 0;
+  return RTM_OK;
+}
+
+}  // namespace
+
+// ================================================================================================
+extern "C" {
+
+const char *rtm_status_str(rtm_status s) {
+  switch (s) {
+    case RTM_OK: return "ok";
+    case RTM_E_INVALID: return "invalid argument";
+    case RTM_E_CUDA: return "CUDA error";
+    case RTM_E_COMM: return "cross-rank exchange failed";
+    case RTM_E_ORDER: return "field-valid records not non-decreasing in ts";
+    case RTM_E_TOO_SMALL: return "output capacity too small";
+    case RTM_E_STATE: return "call not valid in the current state";
+    case RTM_E_NOMEM: return "device allocation failed";
+  }
+  return "unknown status";
+}
+
+const char *rtm_version(void) { return "librtm 0.1 sm_100a (window-snapshot reducer)"; }
+
+rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
+  if (!cfg || !out) return RTM_E_INVALID;
+  *out = nullptr;
+  if (cfg->n_buffers == 0 || cfg->n_buffers > (uint32_t)kMaxBins * kBin) return RTM_E_INVALID;
+  if (cfg->n_components == 0 || cfg->n_components > (1u << 20)) return RTM_E_INVALID;
+  if (cfg->n_kernels == 0 || cfg->n_kernels > 2048) return RTM_E_INVALID;
+  if (cfg->k == 0 || cfg->k > 1024 || cfg->hang_windows == 0) return RTM_E_INVALID;
+  if (cfg->rank_mode != RTM_RANK_PERCENT && cfg->rank_mode != RTM_RANK_SIZE) return RTM_E_INVALID;
+  if (!cfg->buffer_owner || !cfg->buffer_capacity || !cfg->kernel_total) return RTM_E_INVALID;
+  if (cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world) return RTM_E_INVALID;
+  for (uint32_t b = 0; b < cfg->n_buffers; ++b)
+    if (cfg->buffer_capacity[b] == 0 || cfg->buffer_capacity[b] == 0xFFFFu || cfg->buffer_owner[b] >= cfg->n_components)
+      return RTM_E_INVALID;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || cfg->device < 0 || cfg->device >= ndev) {
+    cudaGetLastError();
+    return RTM_E_INVALID;
+  }
+  rtm_ctx *c = new rtm_ctx();
+  c->nb = cfg->n_buffers;
+  c->nc = cfg->n_components;
+  c->nk = cfg->n_kernels;
+  c->nbins = (c->nb + kBin - 1) / kBin;
+  c->ncw = (c->nc + 31) / 32;
+  c->k = cfg->k;
+  c->H = cfg->hang_windows;
+  c->rank_mode = cfg->rank_mode;
+  c->device = cfg->device;
+  c->rank = cfg->rank;
+  c->world = cfg->world;
+  c->t0 = cfg->t0;
+  c->t_prev = cfg->t0;
+  c->allgather = cfg->allgather;
+  c->allgather_user = cfg->allgather_user;
+  c->st = (cudaStream_t)cfg->stream;
+  if (cudaSetDevice(c->device) != cudaSuccess) { cudaGetLastError(); delete c; return RTM_E_CUDA; }
+  configure_kernels_once();
+  cudaDeviceGetAttribute(&c->n_sms, cudaDevAttrMultiProcessorCount, c->device);
+  rtm_status s = RTM_OK;
+  auto fail = [&](rtm_status e) { rtm_destroy(c); return e; };
+  if ((s = ensure(c, c->cap, (size_t)c->nb * 2)) || (s = ensure(c, c->owner, (size_t)c->nb * 4)) ||
+      (s = ensure(c, c->elig, (size_t)c->nb)) || (s = ensure(c, c->ktotal, (size_t)c->nk * 8)) ||
+      (s = ensure(c, c->carry[0], (size_t)c->nb * 2)) || (s = ensure(c, c->carry[1], (size_t)c->nb * 2)) ||
+      (s = ensure(c, c->run, (size_t)c->nc * 4)) || (s = ensure(c, c->kstart, (size_t)c->nk * 8)) ||
+      (s = ensure(c, c->kend, (size_t)c->nk * 8)) || (s = ensure(c, c->cstart, (size_t)c->nc * 8)) ||
+      (s = ensure(c, c->cend, (size_t)c->nc * 8)))
+    return fail(s);
+  std::vector<uint8_t> elig(c->nb);
+  for (uint32_t b = 0; b < c->nb; ++b)
+    elig[b] = cfg->owned_components ? (cfg->owned_components[cfg->buffer_owner[b]] != 0) : 1;
+  if (cudaMemcpy(c->cap.p, cfg->buffer_capacity, (size_t)c->nb * 2, cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaMemcpy(c->owner.p, cfg->buffer_owner, (size_t)c->nb * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaMemcpy(c->elig.p, elig.data(), (size_t)c->nb, cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaMemcpy(c->ktotal.p, cfg->kernel_total, (size_t)c->nk * 8, cudaMemcpyHostToDevice) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(RTM_E_CUDA);
+  }
+  if ((s = zero_state(c))) return fail(s);
+  *out = c;
+  return RTM_OK;
+}
+
+void rtm_destroy(rtm_ctx *c) {
+  if (!c) return;
+  cudaSetDevice(c->device);
+  cudaStreamSynchronize(c->st);
+  DevBuf *bufs[] = {&c->cap, &c->owner, &c->elig, &c->ktotal, &c->carry[0], &c->carry[1], &c->run, &c->kstart,
+                    &c->kend, &c->cstart, &c->cend, &c->flags, &c->s_own, &c->e_own, &c->T, &c->Bs, &c->Be,
+                    &c->rts, &c->rte, &c->treg_s, &c->treg_e, &c->soff, &c->stage, &c->smeta, &c->emeta,
+                    &c->lastlvl, &c->win, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
+                    &c->unit_ctr, &c->status, &c->topk, &c->topk_n, &c->prog, &c->bstat, &c->comps, &c->pack,
+                    &c->gathered};
+  for (DevBuf *b : bufs) free_buf(*b);
+  if (c->h_small.p) cudaFreeHost(c->h_small.p);
+  if (c->h_res.p) cudaFreeHost(c->h_res.p);
+  for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
+  cudaGetLastError();
+  delete c;
+}
+
+rtm_status rtm_reset(rtm_ctx *c) {
+  if (!c) return RTM_E_INVALID;
+  cudaSetDevice(c->device);
+  cudaStreamSynchronize(c->st);
+  cudaGetLastError();
+  c->sticky = 0;
+  return zero_state(c);
+}
+
+rtm_status rtm_ingest(rtm_ctx *c, const rtm_level_sample *samples, uint64_t n_samples, const rtm_task_event *events,
+                      uint64_t n_events, int32_t mem) {
+  if (!c) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (mem != RTM_MEM_HOST && mem != RTM_MEM_DEVICE) return RTM_E_INVALID;
+  if ((n_samples && !samples) || (n_events && !events)) return RTM_E_INVALID;
+  if (mem == RTM_MEM_DEVICE && ((((uintptr_t)samples) & 15) || (((uintptr_t)events) & 15))) return RTM_E_INVALID;
+  CK(cudaSetDevice(c->device));
+  rtm_status s = append(c, c->s_dev, c->s_own, c->s_own_n, samples, n_samples, mem);
+  if (s) return s;
+  return append(c, c->e_dev, c->e_own, c->e_own_n, events, n_events, mem);
+}
+
+rtm_status rtm_window_reduce(rtm_ctx *c, const int64_t *t_end, uint32_t n_windows, rtm_window_summary *out) {
+  if (!c) return RTM_E_INVALID;
+  if (c->world > 1 && !c->allgather) return RTM_E_INVALID;
+  Params p;
+  rtm_status s = reduce_local(c, t_end, n_windows, p);
+  if (s) return s;
+  if (c->world > 1) {
+    const uint64_t pb = pack_bytes(p);
+    if ((s = ensure(c, c->pack, pb))) return s;
+    if ((s = ensure(c, c->gathered, pb * c->world))) return s;
+    launch_pack(p, c->pack.p, c->st);
+    CK(cudaStreamSynchronize(c->st));
+    if (c->allgather(c->allgather_user, c->pack.p, c->gathered.p, pb) != 0) {
+      c->sticky = RTM_E_COMM;
+      return RTM_E_COMM;
+    }
+    LAUNCH(KT_MERGE, 0, launch_merge(p, c->gathered.p, c->world, c->st));
+    CK(cudaGetLastError());
+  }
+  return finish(c, t_end, n_windows, out);
+}
+
+rtm_status rtm_window_reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t n_windows, const void **pack,
+                                   uint64_t *pack_bytes_out) {
+  if (!c || !pack || !pack_bytes_out) return RTM_E_INVALID;
+  Params p;
+  rtm_status s = reduce_local(c, t_end, n_windows, p);
+  if (s) return s;
+  const uint64_t pb = pack_bytes(p);
+  if ((s = ensure(c, c->pack, pb))) return s;
+  launch_pack(p, c->pack.p, c->st);
+  CK(cudaGetLastError());
+  CK(cudaStreamSynchronize(c->st));
+  *pack = c->pack.p;
+  *pack_bytes_out = pb;
+  // remember the call for rtm_merge
+  c->t_end_h.assign(t_end, t_end + n_windows);
+  c->W = n_windows;
+  c->have = false;
+  return RTM_OK;
+}
+
+rtm_status rtm_merge(rtm_ctx *c, const void *gathered, uint32_t world, rtm_window_summary *out) {
+  if (!c || !gathered || world == 0) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (c->t_end_h.empty() || c->have) return RTM_E_STATE;
+  CK(cudaSetDevice(c->device));
+  const uint32_t W = (uint32_t)c->t_end_h.size();
+  Params p;
+  memset(&p, 0, sizeof(p));
+  p.nb = c->nb; p.nc = c->nc; p.nk = c->nk; p.nbins = c->nbins; p.ncw = c->ncw; p.k = c->k;
+  p.rank_mode = c->rank_mode; p.W = W;
+  p.ktotal = (const int64_t *)c->ktotal.p;
+  p.win = (unsigned long long *)c->win.p; p.topk = (unsigned long long *)c->topk.p;
+  p.topk_n = (uint32_t *)c->topk_n.p; p.prog = (long long *)c->prog.p; p.hung = (uint32_t *)c->hung.p;
+  p.comps = (rtm_component_tasks *)c->comps.p; p.bstat = (rtm_buffer_stat *)c->bstat.p;
+  p.status = (uint32_t *)c->status.p;
+  LAUNCH(KT_MERGE, 0, launch_merge(p, gathered, world, c->st));
+  CK(cudaGetLastError());
+  std::vector<int64_t> te = c->t_end_h;
+  return finish(c, te.data(), W, out);
+}
+
+rtm_status rtm_topk_buffers(rtm_ctx *c, uint32_t window, rtm_topk_entry *out, uint32_t *n_out) {
+  if (!c || !out || !n_out) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (!c->have) return RTM_E_STATE;
+  if (window >= c->W) return RTM_E_INVALID;
+  const uint32_t n = c->topk_n_h[window];
+  for (uint32_t i = 0; i < c->k; ++i) {
+    const unsigned long long e = c->topk_h[(size_t)window * c->k + i];
+    out[i].buffer_id = i < n ? (uint32_t)(e & 0xFFFFFFFFu) : 0xFFFFFFFFu;
+    out[i].level = i < n ? (uint16_t)((e >> 32) & 0xFFFFu) : 0;
+    out[i].capacity = i < n ? (uint16_t)(e >> 48) : 0;
+  }
+  *n_out = n;
+  return RTM_OK;
+}
+
+rtm_status rtm_window_results(rtm_ctx *c, uint32_t first, uint32_t count, rtm_window_summary *summaries,
+                              rtm_topk_entry *topk, uint32_t *topk_n, rtm_progress_entry *bars) {
+  if (!c) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (!c->have) return RTM_E_STATE;
+  if ((uint64_t)first + count > c->W) return RTM_E_INVALID;
+  if (summaries) memcpy(summaries, c->sum.data() + first, (size_t)count * sizeof(rtm_window_summary));
+  if (topk_n) memcpy(topk_n, c->topk_n_h.data() + first, (size_t)count * 4);
+  if (bars)
+    memcpy(bars, c->prog_h.data() + (size_t)first * c->nk, (size_t)count * c->nk * sizeof(rtm_progress_entry));
+  if (topk) {
+    const unsigned long long *src = c->topk_h.data() + (size_t)first * c->k;
+    for (uint32_t w = 0; w < count; ++w) {
+      const uint32_t n = c->topk_n_h[first + w];
+      rtm_topk_entry *o = topk + (size_t)w * c->k;
+      for (uint32_t i = 0; i < c->k; ++i) {
+        const unsigned long long e = src[(size_t)w * c->k + i];
+        o[i].buffer_id = i < n ? (uint32_t)(e & 0xFFFFFFFFu) : 0xFFFFFFFFu;
+        o[i].level = i < n ? (uint16_t)((e >> 32) & 0xFFFFu) : 0;
+        o[i].capacity = i < n ? (uint16_t)(e >> 48) : 0;
+      }
+    }
+  }
+  return RTM_OK;
+}
+
+rtm_status rtm_progress(rtm_ctx *c, uint32_t window, rtm_progress_entry *bars, rtm_component_tasks *comps) {
+  if (!c || !bars) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (!c->have) return RTM_E_STATE;
+  if (window >= c->W) return RTM_E_INVALID;
+  if (comps && window != c->W - 1) return RTM_E_INVALID;
+  memcpy(bars, c->prog_h.data() + (size_t)window * c->nk, (size_t)c->nk * sizeof(rtm_progress_entry));
+  if (comps) {
+    CK(cudaSetDevice(c->device));
+    CK(cudaMemcpyAsync(comps, c->comps.p, (size_t)c->nc * sizeof(rtm_component_tasks), cudaMemcpyDeviceToHost,
+                       c->st));
+    CK(cudaStreamSynchronize(c->st));
+  }
+  return RTM_OK;
+}
+
+rtm_status rtm_hang_check(rtm_ctx *c, uint32_t window, uint32_t *comp_ids, uint32_t cap, uint32_t *n_hung) {
+  if (!c || !n_hung || (cap && !comp_ids)) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (!c->have) return RTM_E_STATE;
+  if (window >= c->W) return RTM_E_INVALID;
+  std::vector<uint32_t> bits(c->ncw);
+  CK(cudaSetDevice(c->device));
+  CK(cudaMemcpyAsync(bits.data(), (uint32_t *)c->hung.p + (size_t)window * c->ncw, (size_t)c->ncw * 4,
+                     cudaMemcpyDeviceToHost, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  uint32_t n = 0;
+  for (uint32_t q = 0; q < c->ncw; ++q) {
+    uint32_t x = bits[q];
+    while (x) {
+      const int bpos = __builtin_ctz(x);
+      x &= x - 1;
+      const uint32_t comp = q * 32 + bpos;
+      if (comp >= c->nc) continue;
+      if (n < cap) comp_ids[n] = comp;
+      ++n;
+    }
+  }
+  *n_hung = n;
+  return RTM_OK;
+}
+
+rtm_status rtm_buffer_stats(rtm_ctx *c, uint32_t first, uint32_t count, rtm_buffer_stat *out) {
+  if (!c || (count && !out)) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (!c->have) return RTM_E_STATE;
+  if ((uint64_t)first + count > c->nb) return RTM_E_INVALID;
+  if (!count) return RTM_OK;
+  CK(cudaSetDevice(c->device));
+  CK(cudaMemcpyAsync(out, (rtm_buffer_stat *)c->bstat.p + first, (size_t)count * sizeof(rtm_buffer_stat),
+                     cudaMemcpyDeviceToHost, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  for (uint32_t i = 0; i < count; ++i) out[i].reserved = 0;
+  return RTM_OK;
+}
+
+rtm_status rtm_profile(rtm_ctx *c, int32_t enable) {
+  if (!c) return RTM_E_INVALID;
+  c->prof = enable != 0;
+  for (int i = 0; i < KT_N; ++i) {
+    c->timers[i] = KernelTimer();
+    c->timers[i].name = kKernelNames[i];
+  }
+  c->marks.clear();
+  c->ev_next = 0;
+  return RTM_OK;
+}
+
+rtm_status rtm_profile_read(rtm_ctx *c, rtm_kernel_time *out, uint32_t cap, uint32_t *n) {
+  if (!c || !n || (cap && !out)) return RTM_E_INVALID;
+  uint32_t m = 0;
+  for (int i = 0; i < KT_N; ++i) {
+    if (m < cap) {
+      out[m].name = kKernelNames[i];
+      out[m].launches = c->timers[i].launches;
+      out[m].total_ms = c->timers[i].total_ms;
+      out[m].algo_bytes = c->timers[i].algo_bytes;
+    }
+    ++m;
+  }
+  *n = m;
+  return RTM_OK;
+}
+
+}  // extern "C"

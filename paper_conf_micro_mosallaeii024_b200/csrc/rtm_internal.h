@@ -1,0 +1,126 @@
+// rtm_internal.h — device data layout and kernel launchers of librtm (sm_100a).
+//
+// Data path of one rtm_window_reduce call (DESIGN.md §4 has the rationale and rooflines):
+//   K0 split      : per window boundary, warp 33-ary search for the first record position whose
+//                   field-valid successors all have ts >= boundary  -> region [B_r, B_r+1) per window
+//   K1 partition  : one CTA per 4096-sample tile of one region; validate, order-check, stable
+//                   multisplit of kept samples by 256-buffer bin into 8-byte staging entries
+//   K3 events     : one CTA per 4096-event tile; progress deltas, component activity bitmaps
+//   K2 fold       : one warp per (window, bin) unit, dequeued in window order; in-order fold of
+//                   the bin's samples (delta form of the integral), carry-in resolved by
+//                   decoupled look-back over earlier windows' last levels, finalize + digest
+//   K4 order check: cross-tile ts monotonicity of field-valid records
+//   K5 top-k      : one CTA per window, MSB radix select on the exact 32-bit fullness key
+//   K6 hang       : per component run length over windows
+//   K7 progress   : per kernel prefix over windows, component totals
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "rtm.h"
+
+namespace rtm {
+
+constexpr int kBinLog = 8;                  // 256 buffers per bin
+constexpr int kBin = 1 << kBinLog;
+constexpr int kTileS = 4096;                // samples per partition tile
+constexpr int kTileE = 4096;                // events per event tile
+constexpr int kK1Threads = 256;             // 8 warps x 16 records per lane
+constexpr int kK3Threads = 256;
+constexpr int kFoldWarps = 4;               // warps per fold CTA
+constexpr uint16_t kSent = 0xFFFFu;         // "no kept sample in this window" marker
+constexpr uint32_t kMaxBins = 4096;         // n_buffers <= 2^20 for the partition kernel
+constexpr uint32_t kTopkSmemKeys = 40960;   // keys held in shared memory by the top-k kernel
+constexpr int64_t kMaxWindowLen = (int64_t)1 << 40;  // ts offset field of a staging entry
+
+// per-window scalar accumulators, SoA [kWinFields][W] u64
+enum { WF_SAMPLES = 0, WF_EVENTS, WF_DROPPED, WF_DIGEST, WF_TOUCHED, WF_HUNG, kWinFields };
+
+struct TileMeta {            // per tile, for the cross-tile order check
+  long long first_ts;
+  long long last_ts;
+  unsigned flags;            // bit0 has valid record, bit1 in-tile order / range violation
+  unsigned pad;
+};
+
+struct KernelTimer {
+  const char *name;
+  uint32_t launches = 0;
+  double total_ms = 0;
+  uint64_t algo_bytes = 0;
+};
+
+// Everything a launch needs, by value (kernel parameter).
+struct Params {
+  // registry
+  uint32_t nb, nc, nk, nbins, ncw, k;
+  int32_t rank_mode;
+  uint32_t H;
+  const uint16_t *cap;
+  const uint32_t *owner;
+  const uint8_t *elig;       // [nb] 1 if buffer ranks on this rank
+  const int64_t *ktotal;
+  // call
+  uint32_t W;                // windows in the call
+  uint32_t epoch;
+  const long long *T;        // [W+1]: T[0] = t_begin, T[w+1] = t_end[w]
+  const rtm_level_sample *s;
+  uint64_t ns;
+  const rtm_task_event *e;
+  uint64_t ne;
+  const long long *Bs;       // [W+3] sample region boundaries (positions)
+  const long long *Be;
+  const uint32_t *rts;       // [W+3] first tile of each sample region; rts[W+2] = total
+  const uint32_t *rte;
+  const uint32_t *tile_reg_s;// [n_tiles_s] region of each tile
+  const uint32_t *tile_reg_e;
+  uint32_t n_tiles_s, n_tiles_e;
+  // outputs / workspaces
+  uint32_t *soff;            // [n_tiles_s * (nbins+1)]
+  unsigned long long *stage; // [n_tiles_s * kTileS]
+  TileMeta *smeta, *emeta;
+  uint16_t *lastlvl;         // [W * nb]
+  uint32_t *flags;           // [W * nbins]
+  unsigned long long *win;   // [kWinFields * W]
+  uint32_t *kdelta;          // [W * nk * 2]
+  unsigned long long *cdelta;// [nc * 2]
+  uint32_t *active;          // [W * ncw]
+  uint32_t *anyfull;         // [W * ncw]
+  uint32_t *hung;            // [W * ncw]
+  uint32_t *unit_ctr;
+  uint32_t *status;          // bit0 sample order, bit1 event order
+  const uint16_t *carry_in;  // [nb]
+  uint16_t *carry_out;       // [nb]
+  uint32_t *run;             // [nc]
+  long long *kstart, *kend;  // [nk] cumulative
+  long long *cstart, *cend;  // [nc] cumulative
+  unsigned long long *topk;  // [W * k] packed (id | level<<32 | cap<<48)
+  uint32_t *topk_n;          // [W]
+  long long *prog;           // [W * nk * 5]
+  rtm_buffer_stat *bstat;    // [nb]
+  rtm_component_tasks *comps;// [nc]
+};
+
+// launchers (rtm_kernels.cu); all asynchronous on `st`
+void launch_split(const Params &p, bool samples, long long *outB, cudaStream_t st);
+void launch_fill_tile_regions(const Params &p, cudaStream_t st);
+void launch_partition(const Params &p, cudaStream_t st);
+void launch_events(const Params &p, cudaStream_t st);
+void launch_fold(const Params &p, int n_sms, cudaStream_t st);
+void launch_order_check(const Params &p, cudaStream_t st);
+void launch_topk(const Params &p, cudaStream_t st);
+void launch_hang(const Params &p, cudaStream_t st);
+void launch_progress(const Params &p, cudaStream_t st);
+// multi-rank exchange
+uint64_t pack_bytes(const Params &p);
+void launch_pack(const Params &p, void *pack, cudaStream_t st);
+void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStream_t st);
+void configure_kernels_once();  // opt-in shared-memory limits, once per device
+size_t fold_smem_bytes();
+size_t partition_smem_bytes(uint32_t nbins);
+size_t topk_smem_bytes(uint32_t nb);
+
+}  // namespace rtm

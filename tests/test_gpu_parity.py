@@ -1,0 +1,282 @@
+"""GPU parity: the CUDA path (through the C-ABI) vs the CPU oracle, element by element.
+
+Integer outputs must be bit-exact; mean occupancy must agree within 1e-12 relative
+(BASELINE.json north_star) — the path uses the same single IEEE division, so it is exact.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+from tests.helpers import event_array, random_tiny_case, sample_array
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+from paper_conf_micro_mosallaeii024_b200 import Monitor, RTMError  # noqa: E402
+from paper_conf_micro_mosallaeii024_b200 import _native as N  # noqa: E402
+
+SUM_FIELDS = ("t_begin", "t_end", "n_samples", "n_events", "n_dropped", "digest", "n_touched", "n_hung")
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a).view(np.uint8)).cuda()
+
+
+def _pair(owner, cap, tot, nc, **kw):
+    orc = oracle.Oracle(owner, cap, tot, n_components=nc, **kw)
+    mon = Monitor(owner, cap, tot, n_components=nc, **kw)
+    return orc, mon
+
+
+def assert_same(got, ref, mon, *, stats=True, comps=True, hung=True):
+    W = len(ref["summary"])
+    for f in SUM_FIELDS:
+        assert np.array_equal(got["summary"][f], ref["summary"][f]), (f, got["summary"][f], ref["summary"][f])
+    assert np.array_equal(got["topk_n"], ref["topk_n"])
+    for w in range(W):
+        n = int(ref["topk_n"][w])
+        assert np.array_equal(got["topk"][w][:n], ref["topk"][w][:n]), w
+    for f in ("total", "started", "finished", "in_flight", "not_started"):
+        assert np.array_equal(got["progress"][f], ref["progress"][f]), f
+    for w in (0, W - 1):  # single-window accessors agree with the bulk one
+        assert np.array_equal(mon.topk(w), got["topk"][w][: int(got["topk_n"][w])])
+        assert np.array_equal(mon.progress(w), got["progress"][w])
+    if hung:
+        for w in range(W):
+            assert np.array_equal(mon.hang_check(w), np.nonzero(ref["hung"][w])[0].astype(np.uint32)), w
+    if stats:
+        st = mon.buffer_stats()
+        rs = ref["stats"]
+        for f in ("integral", "last", "max", "min", "capacity", "n_samples"):
+            assert np.array_equal(st[f], rs[f]), f
+        np.testing.assert_allclose(st["mean_occ"], rs["mean_occ"], rtol=1e-12, atol=0)
+        assert np.array_equal(st["mean_occ"], rs["mean_occ"])  # same single IEEE division
+    if comps:
+        _, cs = mon.progress(W - 1, comps=True)
+        for f in ("started", "finished", "in_flight"):
+            assert np.array_equal(cs[f], ref["comps"][f]), f
+
+
+# ---------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("seed", range(40))
+def test_random_tiny_traces(seed):
+    rng = np.random.default_rng(5000 + seed)
+    case = random_tiny_case(rng, allow_disorder=(seed % 5 == 4))
+    kw = dict(t0=case["t0"], hang_windows=case["H"], k=case["k"], rank_mode=case["mode"])
+    orc, mon = _pair(case["owner"], case["caps"], case["totals"], case["nc"], **kw)
+    for srows, erows, ends in case["calls"]:
+        s, e = sample_array(srows), event_array(erows)
+        ref = orc.reduce(s, e, ends)
+        mon.ingest(_dev(s) if len(s) else None, _dev(e) if len(e) else None)
+        if ref["rc"] == -4:
+            with pytest.raises(RTMError) as ei:
+                mon.window_reduce(ends)
+            assert ei.value.code == N.RTM_E_ORDER
+            break
+        got = mon.window_reduce(ends)
+        assert_same(got, ref, mon)
+
+
+def test_fig3_and_size_mode():
+    size = [8, 8, 8, 8, 8, 8, 7, 4, 4, 4, 4, 4]
+    cap = np.array([8] * 7 + [4] * 5, np.uint16)
+    s = sample_array([(i, i, size[i], int(cap[i])) for i in range(12)])
+    for mode, expected in ((1, list(range(12))), (0, [0, 1, 2, 3, 4, 5, 7, 8, 9, 10, 11, 6])):
+        mon = Monitor(np.arange(12, dtype=np.uint32), cap, np.ones(1, np.int64), n_components=12, t0=0,
+                      hang_windows=1, k=12, rank_mode=mode)
+        mon.ingest(_dev(s), None)
+        got = mon.window_reduce([100])
+        assert [int(x) for x in got["topk"][0]["buffer_id"]] == expected
+
+
+def test_c1_full_parity():
+    wl = gen.C1
+    owner, cap, tot = gen.registry(wl)
+    s, e = gen.samples(wl), gen.events(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    ref = orc.reduce(s, e, wl.t_end())
+    mon.ingest(_dev(s), _dev(e))
+    got = mon.window_reduce(wl.t_end())
+    assert_same(got, ref, mon)
+    assert int(ref["summary"]["n_hung"].sum()) >= 0
+
+
+def test_c1_invalid_records_parity():
+    wl = gen.C1_INVALID
+    owner, cap, tot = gen.registry(wl)
+    s, e = gen.samples(wl), gen.events(wl)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k)
+    # windows starting after t0 and ending before the trace end: late and early drops too
+    ends = wl.t_end()[2:8]
+    orc.reduce(s[:0], e[:0], [wl.t_end()[1]])
+    mon.ingest(None, None)
+    mon.window_reduce([wl.t_end()[1]])
+    ref = orc.reduce(s, e, ends)
+    mon.ingest(_dev(s), _dev(e))
+    got = mon.window_reduce(ends)
+    assert int(ref["summary"]["n_dropped"].sum()) > 0
+    assert_same(got, ref, mon)
+
+
+def test_windows_one_call_each_full_tables():
+    """Every window's full per-buffer table (reduce one window per call) and batch invariance."""
+    wl = gen.C1.scaled("C1-small", n_samples=300_000, n_events=30_000, n_buffers=900, n_windows=12)
+    owner, cap, tot = gen.registry(wl)
+    s, e = gen.samples(wl), gen.events(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    ref = orc.reduce(s, e, wl.t_end(), want_all_stats=True)
+    ends = wl.t_end()
+    for w in range(wl.n_windows):
+        lo = wl.t0 if w == 0 else ends[w - 1]
+        ss = s[(s["ts"] >= lo) & (s["ts"] < ends[w])]
+        ee = e[(e["ts"] >= lo) & (e["ts"] < ends[w])]
+        mon.ingest(_dev(ss) if len(ss) else None, _dev(ee) if len(ee) else None)
+        got = mon.window_reduce(ends[w:w + 1])
+        st = mon.buffer_stats()
+        for f in ("integral", "last", "max", "min", "n_samples"):
+            assert np.array_equal(st[f], ref["all_stats"][w][f]), (w, f)
+        for f in ("n_samples", "digest", "n_touched", "n_hung"):
+            assert got["summary"][f][0] == ref["summary"][f][w], (w, f)
+        assert np.array_equal(got["topk"][0], ref["topk"][w])
+
+
+def test_edge_cases_empty_zero_length_and_k_above_n():
+    owner = np.array([0, 0, 1], np.uint32)
+    cap = np.array([4, 8, 16], np.uint16)
+    tot = np.array([10, 3], np.int64)
+    kw = dict(t0=0, hang_windows=1, k=8)
+    orc, mon = _pair(owner, cap, tot, 2, **kw)
+    # no records at all, zero-length windows included
+    ends = [0, 5, 5, 9]
+    ref = orc.reduce(sample_array([]), event_array([]), ends)
+    mon.ingest(None, None)
+    got = mon.window_reduce(ends)
+    assert_same(got, ref, mon)
+    # only dropped records (late, early, invalid)
+    s = sample_array([(3, 0, 1, 4), (10, 9, 1, 4), (12, 1, 9, 8), (20, 2, 1, 16)])
+    ref = orc.reduce(s, event_array([]), [15, 18])
+    mon.ingest(s, None)  # host ingest path
+    got = mon.window_reduce([15, 18])
+    assert_same(got, ref, mon)
+
+
+def test_multiple_ingest_chunks_host_and_device():
+    wl = gen.C1.scaled("C1-chunks", n_samples=100_000, n_events=10_000, n_windows=5)
+    owner, cap, tot = gen.registry(wl)
+    s, e = gen.samples(wl), gen.events(wl)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, t0=wl.t0, hang_windows=2, k=wl.k)
+    ref = orc.reduce(s, e, wl.t_end())
+    mon.ingest(_dev(s[:30000]), _dev(e[:1000]))
+    mon.ingest(s[30000:70000], e[1000:5000])
+    mon.ingest(_dev(s[70000:]), _dev(e[5000:]))
+    got = mon.window_reduce(wl.t_end())
+    assert_same(got, ref, mon)
+
+
+def test_order_violation_is_sticky_until_reset():
+    owner = np.zeros(2, np.uint32)
+    cap = np.array([4, 4], np.uint16)
+    mon = Monitor(owner, cap, np.ones(1, np.int64), n_components=1, t0=0, hang_windows=1, k=2)
+    mon.ingest(_dev(sample_array([(5, 0, 1, 4), (3, 1, 2, 4)])), None)
+    with pytest.raises(RTMError) as ei:
+        mon.window_reduce([10])
+    assert ei.value.code == N.RTM_E_ORDER
+    with pytest.raises(RTMError):
+        mon.window_reduce([20])
+    mon.reset()
+    mon.ingest(_dev(sample_array([(3, 1, 2, 4), (5, 0, 1, 4)])), None)
+    got = mon.window_reduce([10])
+    assert int(got["summary"]["n_samples"][0]) == 2
+
+
+def test_invalid_arguments():
+    mon = Monitor(np.zeros(1, np.uint32), np.array([4], np.uint16), np.ones(1, np.int64), n_components=1, t0=10,
+                  hang_windows=1, k=1)
+    for ends in ([5], [20, 15], [10 + (1 << 40)]):
+        with pytest.raises(RTMError) as ei:
+            mon.window_reduce(ends)
+        assert ei.value.code == N.RTM_E_INVALID
+    got = mon.window_reduce([20])  # state unchanged by the rejected calls
+    assert int(got["summary"]["t_begin"][0]) == 10
+
+
+def test_case_study_deadlock_on_gpu():
+    from tests.test_oracle import _deadlock_trace
+
+    caps, S, E = _deadlock_trace()
+    owner = np.arange(5, dtype=np.uint32)
+    orc, mon = _pair(owner, np.array(caps, np.uint16), np.array([100], np.int64), 5, t0=0, hang_windows=2, k=5)
+    ends = [100 * (w + 1) for w in range(6)]
+    ref = orc.reduce(sample_array(S), event_array(E), ends)
+    mon.ingest(_dev(sample_array(S)), _dev(event_array(E)))
+    got = mon.window_reduce(ends)
+    assert_same(got, ref, mon)
+    assert [list(mon.hang_check(w)) for w in range(6)] == [[], [], [], [], [1, 2], [0, 1, 2, 3]]
+
+
+def test_virtual_shards_merge_equals_whole():
+    """Three shard contexts on one GPU (owner-component sharding) + the library's merge kernels."""
+    import ctypes
+
+    from paper_conf_micro_mosallaeii024_b200 import _copy_from_ptr
+
+    wl = gen.C1.scaled("C1-vshard", n_samples=200_000, n_events=20_000, n_windows=6)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    ref = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw).reduce(gen.samples(wl), gen.events(wl),
+                                                                                   wl.t_end())
+    G = 3
+    mons, packs = [], []
+    for r in range(G):
+        owned = (np.arange(wl.n_components) % G == r).astype(np.uint8)
+        m = Monitor(owner, cap, tot, n_components=wl.n_components, rank=r, world=G, owned_components=owned, **kw)
+        m.ingest(_dev(gen.samples(wl, shard=(G, r))), _dev(gen.events(wl, shard=(G, r))))
+        ends = np.ascontiguousarray(wl.t_end())
+        pack, nbytes = ctypes.c_void_p(), ctypes.c_uint64()
+        N.check(N.lib().rtm_window_reduce_local(m._h, ends.ctypes.data, len(ends), ctypes.byref(pack),
+                                                ctypes.byref(nbytes)), "local")
+        t = torch.empty(int(nbytes.value), dtype=torch.uint8, device="cuda")
+        _copy_from_ptr(t, pack.value, int(nbytes.value))
+        torch.cuda.synchronize()
+        mons.append(m)
+        packs.append(t)
+    gathered = torch.cat(packs)
+    for m in mons:
+        summ = np.zeros(wl.n_windows, N.SUMMARY_DTYPE)
+        N.check(N.lib().rtm_merge(m._h, gathered.data_ptr(), G, summ.ctypes.data), "merge")
+        m.W = wl.n_windows
+        got = m.results()
+        assert np.array_equal(got["summary"], summ)
+        assert_same(got, ref, m)
+
+
+@pytest.mark.slow
+def test_c2_full_size_parity():
+    """BASELINE configs[1] at full size, in the launch configuration bench.py times."""
+    wl = gen.C2
+    owner, cap, tot = gen.registry(wl)
+    ds = torch.empty(wl.n_samples * 16, dtype=torch.uint8, device="cuda")
+    de = torch.empty(wl.n_events * 16, dtype=torch.uint8, device="cuda")
+    gen.fill_device("samples", wl, ds.data_ptr(), 0, wl.n_samples)
+    gen.fill_device("events", wl, de.data_ptr(), 0, wl.n_events)
+    torch.cuda.synchronize()
+    kw = dict(t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k)
+    mon = Monitor(owner, cap, tot, n_components=wl.n_components, **kw)
+    mon.ingest(ds, de)
+    got = mon.window_reduce(wl.t_end())
+    # device generator == host generator (spot check), then the oracle on the host copy
+    s = gen.samples(wl)
+    e = gen.events(wl)
+    idx = np.random.default_rng(0).integers(0, wl.n_samples, 4096)
+    assert np.array_equal(ds.view(-1, 16)[torch.from_numpy(idx).cuda()].cpu().numpy().view(gen.SAMPLE_DTYPE).ravel(),
+                          s[idx])
+    ref = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw).reduce(s, e, wl.t_end())
+    assert_same(got, ref, mon)
