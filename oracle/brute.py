@@ -29,11 +29,12 @@ def fmix64(z: int) -> int:
 
 
 def digest_term(b, last, mx, mn, cap, n, integral) -> int:
-    h = fmix64(0x9E3779B97F4A7C15 ^ b)
-    h = fmix64(h ^ (last | (mx << 16) | (mn << 32) | (cap << 48)))
-    h = fmix64(h ^ n)
-    h = fmix64(h ^ (integral & M64))
-    return h
+    levels = last | (mx << 16) | (mn << 32) | (cap << 48)
+    ident = (n << 32) | b
+    x = ((integral & M64) * 0x9E3779B97F4A7C15) & M64
+    x ^= (ident * 0xC2B2AE3D27D4EB4F) & M64
+    x ^= (levels * 0x165667B19E3779F9) & M64
+    return fmix64(x)
 
 
 class OrderError(Exception):

@@ -28,7 +28,9 @@ struct orc_ctx {
   int sticky;
 };
 
-/* ---- digest mixer (DESIGN.md §2 "digest"): splitmix64 finalizer absorbed four times ---- */
+/* ---- digest mixer (DESIGN.md §2 "digest", reading R17): three fields folded by odd-constant
+ * products (bijections of Z/2^64), XORed, then one splitmix64 finalizer.  A change in any single
+ * field changes the term. ---- */
 static uint64_t fmix64(uint64_t z) {
   z ^= z >> 30;
   z *= 0xbf58476d1ce4e5b9ULL;
@@ -40,11 +42,10 @@ static uint64_t fmix64(uint64_t z) {
 
 uint64_t orc_digest_term(uint32_t b, uint16_t last, uint16_t mx, uint16_t mn, uint16_t cap, uint32_t n,
                          int64_t integral) {
-  uint64_t h = fmix64(0x9E3779B97F4A7C15ULL ^ (uint64_t)b);
-  h = fmix64(h ^ ((uint64_t)last | ((uint64_t)mx << 16) | ((uint64_t)mn << 32) | ((uint64_t)cap << 48)));
-  h = fmix64(h ^ (uint64_t)n);
-  h = fmix64(h ^ (uint64_t)integral);
-  return h;
+  const uint64_t levels = (uint64_t)last | ((uint64_t)mx << 16) | ((uint64_t)mn << 32) | ((uint64_t)cap << 48);
+  const uint64_t ident = ((uint64_t)n << 32) | (uint64_t)b;
+  return fmix64(((uint64_t)integral * 0x9E3779B97F4A7C15ULL) ^ (ident * 0xC2B2AE3D27D4EB4FULL) ^
+                (levels * 0x165667B19E3779F9ULL));
 }
 
 orc_ctx *orc_create(const orc_config *cfg) {

@@ -11,7 +11,7 @@ import os
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "librtm.so")
+LIB_PATH = os.environ.get("RTM_LIB_PATH") or os.path.join(HERE, "librtm.so")  # override: profiling builds
 
 RTM_OK, RTM_E_INVALID, RTM_E_CUDA, RTM_E_COMM, RTM_E_ORDER, RTM_E_TOO_SMALL, RTM_E_STATE, RTM_E_NOMEM = (
     0, -1, -2, -3, -4, -5, -6, -7)

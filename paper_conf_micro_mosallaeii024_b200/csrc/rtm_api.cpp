@@ -2,6 +2,7 @@
 // orchestration on one CUDA stream, result accessors and the multi-rank exchange.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdio.h>
 #include <string.h>
 
 #include <algorithm>
@@ -44,11 +45,12 @@ struct rtm_ctx {
   void *allgather_user;
   cudaStream_t st;
   int n_sms;
-  DevBuf cap, owner, elig, ktotal;
+  DevBuf cap, owner, elig, ktotal, rcp, elig_ids;
+  uint32_t n_elig = 0;
   // persistent state
   DevBuf carry[2];
   int cur = 0;
-  DevBuf run, kstart, kend, cstart, cend, flags;
+  DevBuf run[2], kstart, kend, cstart, cend, flags;
   uint32_t epoch = 1;
   int64_t t_prev;
   int sticky = 0;
@@ -201,7 +203,8 @@ void free_buf(DevBuf &b) {
 rtm_status zero_state(rtm_ctx *c) {
   CK(cudaMemsetAsync(c->carry[0].p, 0, (size_t)c->nb * 2, c->st));
   CK(cudaMemsetAsync(c->carry[1].p, 0, (size_t)c->nb * 2, c->st));
-  CK(cudaMemsetAsync(c->run.p, 0, (size_t)c->nc * 4, c->st));
+  CK(cudaMemsetAsync(c->run[0].p, 0, (size_t)c->nc * 4, c->st));
+  CK(cudaMemsetAsync(c->run[1].p, 0, (size_t)c->nc * 4, c->st));
   CK(cudaMemsetAsync(c->kstart.p, 0, (size_t)c->nk * 8, c->st));
   CK(cudaMemsetAsync(c->kend.p, 0, (size_t)c->nk * 8, c->st));
   CK(cudaMemsetAsync(c->cstart.p, 0, (size_t)c->nc * 8, c->st));
@@ -305,7 +308,11 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.rank_mode = c->rank_mode; p.H = c->H;
   p.cap = (const uint16_t *)c->cap.p; p.owner = (const uint32_t *)c->owner.p;
   p.elig = (const uint8_t *)c->elig.p; p.ktotal = (const int64_t *)c->ktotal.p;
+  p.rcp = (const unsigned long long *)c->rcp.p; p.elig_ids = (const uint32_t *)c->elig_ids.p; p.n_elig = c->n_elig;
   p.W = W; p.epoch = c->epoch;
+  p.narrow = 1;
+  for (uint32_t w = 0; w < W; ++w)
+    if (t_end[w] - (w ? t_end[w - 1] : c->t_prev) >= ((int64_t)1 << 32)) p.narrow = 0;
   p.T = (const long long *)c->T.p;
   p.s = (const rtm_level_sample *)sp; p.ns = ns;
   p.e = (const rtm_task_event *)ep; p.ne = ne;
@@ -375,15 +382,22 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.anyfull = (uint32_t *)c->anyfull.p; p.hung = (uint32_t *)c->hung.p;
   p.unit_ctr = (uint32_t *)c->unit_ctr.p; p.status = (uint32_t *)c->status.p;
   p.carry_in = (const uint16_t *)c->carry[c->cur].p; p.carry_out = (uint16_t *)c->carry[c->cur ^ 1].p;
-  p.run = (uint32_t *)c->run.p;
+  p.run = (const uint32_t *)c->run[c->cur].p;
+  p.run_out = (uint32_t *)c->run[c->cur ^ 1].p;
   p.kstart = (long long *)c->kstart.p; p.kend = (long long *)c->kend.p;
   p.cstart = (long long *)c->cstart.p; p.cend = (long long *)c->cend.p;
   p.topk = (unsigned long long *)c->topk.p; p.topk_n = (uint32_t *)c->topk_n.p;
   p.prog = (long long *)c->prog.p; p.bstat = (rtm_buffer_stat *)c->bstat.p;
   p.comps = (rtm_component_tasks *)c->comps.p;
 
+#ifdef RTM_PHASE_TIMING
+  static unsigned long long *dbg = nullptr;
+  if (!dbg) cudaMalloc(&dbg, 64);
+  cudaMemsetAsync(dbg, 0, 64, c->st);
+  p.dbg = dbg;
+#endif
   launch_fill_tile_regions(p, c->st);
-  LAUNCH(KT_PARTITION, (uint64_t)ns * 16, launch_partition(p, c->st));
+  LAUNCH(KT_PARTITION, (uint64_t)ns * 16, launch_partition(p, c->n_sms, c->st));
   LAUNCH(KT_EVENTS, (uint64_t)ne * 16, launch_events(p, c->st));
   LAUNCH(KT_FOLD, 0, launch_fold(p, c->n_sms, c->st));
   LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
@@ -391,6 +405,19 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   LAUNCH(KT_HANG, 0, launch_hang(p, c->st));
   LAUNCH(KT_PROGRESS, 0, launch_progress(p, c->st));
   CK(cudaGetLastError());
+#ifdef RTM_PHASE_TIMING
+  {
+    unsigned long long h[8];
+    cudaMemcpyAsync(h, p.dbg, 64, cudaMemcpyDeviceToHost, c->st);
+    cudaStreamSynchronize(c->st);
+    if (h[3])
+      fprintf(stderr,
+              "[phase] tiles=%llu wait=%.0f scan=%.0f finish=%.0f | fin: summary=%.0f prefix=%.0f scatter=%.0f | "
+              "scan: cap_prefetch=%.0f (cycles/tile)\n",
+              h[3], (double)h[0] / h[3], (double)h[1] / h[3], (double)h[2] / h[3], (double)h[4] / h[3],
+              (double)h[5] / h[3], (double)h[6] / h[3], (double)h[7] / h[3]);
+  }
+#endif
   return RTM_OK;
 }
 
@@ -514,13 +541,27 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   if ((s = ensure(c, c->cap, (size_t)c->nb * 2)) || (s = ensure(c, c->owner, (size_t)c->nb * 4)) ||
       (s = ensure(c, c->elig, (size_t)c->nb)) || (s = ensure(c, c->ktotal, (size_t)c->nk * 8)) ||
       (s = ensure(c, c->carry[0], (size_t)c->nb * 2)) || (s = ensure(c, c->carry[1], (size_t)c->nb * 2)) ||
-      (s = ensure(c, c->run, (size_t)c->nc * 4)) || (s = ensure(c, c->kstart, (size_t)c->nk * 8)) ||
+      (s = ensure(c, c->run[0], (size_t)c->nc * 4)) || (s = ensure(c, c->run[1], (size_t)c->nc * 4)) ||
+      (s = ensure(c, c->kstart, (size_t)c->nk * 8)) ||
       (s = ensure(c, c->kend, (size_t)c->nk * 8)) || (s = ensure(c, c->cstart, (size_t)c->nc * 8)) ||
-      (s = ensure(c, c->cend, (size_t)c->nc * 8)))
+      (s = ensure(c, c->cend, (size_t)c->nc * 8)) || (s = ensure(c, c->rcp, (size_t)65536 * 8)) ||
+      (s = ensure(c, c->elig_ids, (size_t)c->nb * 4)))
     return fail(s);
   std::vector<uint8_t> elig(c->nb);
-  for (uint32_t b = 0; b < c->nb; ++b)
+  std::vector<uint32_t> elig_ids;
+  for (uint32_t b = 0; b < c->nb; ++b) {
     elig[b] = cfg->owned_components ? (cfg->owned_components[cfg->buffer_owner[b]] != 0) : 1;
+    if (elig[b]) elig_ids.push_back(b);
+  }
+  c->n_elig = (uint32_t)elig_ids.size();
+  std::vector<unsigned long long> rcp(65536, 0);
+  for (uint32_t cc = 2; cc < 65536; ++cc) rcp[cc] = (1ull << 48) / cc;  // c == 1: only l == 0 < c
+  if (cudaMemcpy(c->rcp.p, rcp.data(), 65536 * 8, cudaMemcpyHostToDevice) != cudaSuccess ||
+      (c->n_elig && cudaMemcpy(c->elig_ids.p, elig_ids.data(), (size_t)c->n_elig * 4, cudaMemcpyHostToDevice) !=
+                        cudaSuccess)) {
+    cudaGetLastError();
+    return fail(RTM_E_CUDA);
+  }
   if (cudaMemcpy(c->cap.p, cfg->buffer_capacity, (size_t)c->nb * 2, cudaMemcpyHostToDevice) != cudaSuccess ||
       cudaMemcpy(c->owner.p, cfg->buffer_owner, (size_t)c->nb * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
       cudaMemcpy(c->elig.p, elig.data(), (size_t)c->nb, cudaMemcpyHostToDevice) != cudaSuccess ||
@@ -537,7 +578,8 @@ void rtm_destroy(rtm_ctx *c) {
   if (!c) return;
   cudaSetDevice(c->device);
   cudaStreamSynchronize(c->st);
-  DevBuf *bufs[] = {&c->cap, &c->owner, &c->elig, &c->ktotal, &c->carry[0], &c->carry[1], &c->run, &c->kstart,
+  DevBuf *bufs[] = {&c->cap, &c->owner, &c->elig, &c->ktotal, &c->carry[0], &c->carry[1], &c->run[0], &c->run[1],
+                    &c->kstart, &c->rcp, &c->elig_ids,
                     &c->kend, &c->cstart, &c->cend, &c->flags, &c->s_own, &c->e_own, &c->T, &c->Bs, &c->Be,
                     &c->rts, &c->rte, &c->treg_s, &c->treg_e, &c->soff, &c->stage, &c->smeta, &c->emeta,
                     &c->lastlvl, &c->win, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
@@ -625,7 +667,7 @@ rtm_status rtm_merge(rtm_ctx *c, const void *gathered, uint32_t world, rtm_windo
   memset(&p, 0, sizeof(p));
   p.nb = c->nb; p.nc = c->nc; p.nk = c->nk; p.nbins = c->nbins; p.ncw = c->ncw; p.k = c->k;
   p.rank_mode = c->rank_mode; p.W = W;
-  p.ktotal = (const int64_t *)c->ktotal.p;
+  p.ktotal = (const int64_t *)c->ktotal.p; p.rcp = (const unsigned long long *)c->rcp.p;
   p.win = (unsigned long long *)c->win.p; p.topk = (unsigned long long *)c->topk.p;
   p.topk_n = (uint32_t *)c->topk_n.p; p.prog = (long long *)c->prog.p; p.hung = (uint32_t *)c->hung.p;
   p.comps = (rtm_component_tasks *)c->comps.p; p.bstat = (rtm_buffer_stat *)c->bstat.p;

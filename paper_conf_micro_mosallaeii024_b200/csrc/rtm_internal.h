@@ -28,11 +28,11 @@ constexpr int kBinLog = 8;                  // 256 buffers per bin
 constexpr int kBin = 1 << kBinLog;
 constexpr int kTileS = 4096;                // samples per partition tile
 constexpr int kTileE = 4096;                // events per event tile
-constexpr int kK1Threads = 256;             // 8 warps x 16 records per lane
+constexpr int kK1Threads = 512;             // 16 warps x 8 records per lane
 constexpr int kK3Threads = 256;
 constexpr int kFoldWarps = 4;               // warps per fold CTA
 constexpr uint16_t kSent = 0xFFFFu;         // "no kept sample in this window" marker
-constexpr uint32_t kMaxBins = 4096;         // n_buffers <= 2^20 for the partition kernel
+constexpr uint32_t kMaxBins = 3072;         // n_buffers <= 786432 (partition smem <= 204 KB)
 constexpr uint32_t kTopkSmemKeys = 40960;   // keys held in shared memory by the top-k kernel
 constexpr int64_t kMaxWindowLen = (int64_t)1 << 40;  // ts offset field of a staging entry
 
@@ -63,8 +63,12 @@ struct Params {
   const uint32_t *owner;
   const uint8_t *elig;       // [nb] 1 if buffer ranks on this rank
   const int64_t *ktotal;
+  const unsigned long long *rcp;  // [65536] floor(2^48 / c) (exact fullness key, K5)
+  const uint32_t *elig_ids;  // [n_elig] ascending ids of ranked buffers
+  uint32_t n_elig;
   // call
   uint32_t W;                // windows in the call
+  int32_t narrow;            // every window shorter than 2^32 ticks (32-bit order check)
   uint32_t epoch;
   const long long *T;        // [W+1]: T[0] = t_begin, T[w+1] = t_end[w]
   const rtm_level_sample *s;
@@ -94,7 +98,8 @@ struct Params {
   uint32_t *status;          // bit0 sample order, bit1 event order
   const uint16_t *carry_in;  // [nb]
   uint16_t *carry_out;       // [nb]
-  uint32_t *run;             // [nc]
+  const uint32_t *run;       // [nc] carried hang run length (in)
+  uint32_t *run_out;         // [nc] (out, ping-pong with run)
   long long *kstart, *kend;  // [nk] cumulative
   long long *cstart, *cend;  // [nc] cumulative
   unsigned long long *topk;  // [W * k] packed (id | level<<32 | cap<<48)
@@ -102,12 +107,13 @@ struct Params {
   long long *prog;           // [W * nk * 5]
   rtm_buffer_stat *bstat;    // [nb]
   rtm_component_tasks *comps;// [nc]
+  unsigned long long *dbg;   // phase-timing scratch (RTM_PHASE_TIMING builds only)
 };
 
 // launchers (rtm_kernels.cu); all asynchronous on `st`
 void launch_split(const Params &p, bool samples, long long *outB, cudaStream_t st);
 void launch_fill_tile_regions(const Params &p, cudaStream_t st);
-void launch_partition(const Params &p, cudaStream_t st);
+void launch_partition(const Params &p, int n_sms, cudaStream_t st);
 void launch_events(const Params &p, cudaStream_t st);
 void launch_fold(const Params &p, int n_sms, cudaStream_t st);
 void launch_order_check(const Params &p, cudaStream_t st);

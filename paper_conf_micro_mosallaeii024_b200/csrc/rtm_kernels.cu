@@ -3,6 +3,7 @@
 // the one compulsory HBM read of 16 B per trace record.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "rtm_internal.h"
 
@@ -159,161 +160,373 @@ __global__ void k_fill_tile_regions(const uint32_t *rt, uint32_t *tile_reg, uint
 }
 
 // ============================================================================================
-// K1: sample partition.  One CTA per tile of <= 4096 samples of ONE region.  8 warps; warp w
-// owns tile positions [512w, 512w+512), lane l handles positions 512w + 32j + l (j = 0..15),
-// so each warp load is 512 contiguous bytes.  Kept samples are stably multisplit by bin
-// (buffer_id >> 8): per-(warp, bin) running counters give a stable rank, a block scan gives
-// bin offsets, the tile is permuted through shared memory and written out coalesced as
-// 8-byte entries  ts_off<<24 | level<<8 | (buffer_id & 255).
+// K1: sample partition.  A tile is <= 4096 samples of ONE region, processed by 16 warps; warp w
+// owns tile positions [256w, 256w+256), lane l handles 256w + 32j + l (j = 0..7).  Per sample:
+// field validity, range + order check against the previous field-valid sample (warp order;
+// 32-bit offsets when windows are < 2^32 ticks), and a stable multisplit by bin
+// (buffer_id >> 8): __match_any_sync + the group leader's shared atomicAdd on per-(warp, bin)
+// u16 counters give the stable rank (onesweep-style), a block scan gives bin offsets.  Kept
+// samples become 8-byte entries  (ts - t_begin) << 24 | level << 8 | (buffer_id & 255),
+// staged in shared memory (tile order) and scattered to the tile's staging slot.
+//
+// k_partition_tma (n_bins <= 1024): persistent, one CTA per SM; tiles stream into a double
+// buffer with cp.async.bulk (TMA) + mbarrier, so the next tile's HBM read is in flight while the
+// current one is ranked.  k_partition: one CTA per tile, register loads (any n_bins).
 // ============================================================================================
-constexpr int kRecPerLane = kTileS / kK1Threads;  // 16
+constexpr int kRecPerLane = kTileS / kK1Threads;  // 8
+constexpr int kK1Warps = kK1Threads / 32;         // 16
 constexpr unsigned kNoKey = 0xFFFFu;
+constexpr uint32_t kTmaMaxBins = 1024;
 
-__global__ void __launch_bounds__(kK1Threads, 2) k_partition(Params p) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  unsigned long long *sbuf = reinterpret_cast<unsigned long long *>(smem);                 // [4096]
-  unsigned *binoff = reinterpret_cast<unsigned *>(sbuf + kTileS);                           // [nbins+1]
-  unsigned short *cnt = reinterpret_cast<unsigned short *>(binoff + p.nbins + 1);          // [8][nbins]
-  __shared__ unsigned scan_scratch[32];
-  __shared__ long long wfirst[8], wlast[8];
-  __shared__ unsigned whas[8], wviol[8], wkept[8];
+#ifdef RTM_PHASE_TIMING
+#define PT_MARK(p_, slot_, t0_)                                                     \
+  do {                                                                              \
+    __syncthreads();                                                                \
+    if (threadIdx.x == 0 && (p_).dbg) {                                             \
+      const long long t1_ = clock64();                                              \
+      atomicAdd((p_).dbg + (slot_), (unsigned long long)(t1_ - (t0_)));            \
+      (t0_) = t1_;                                                                  \
+    }                                                                               \
+  } while (0)
+#else
+#define PT_MARK(p_, slot_, t0_) \
+  do {                          \
+  } while (0)
+#endif
 
-  const unsigned tile = blockIdx.x;
-  const unsigned r = p.tile_reg_s[tile];
-  const long long start = p.Bs[r] + (long long)(tile - p.rts[r]) * kTileS;
-  long long endp = p.Bs[r + 1];
-  if (endp > start + kTileS) endp = start + kTileS;
-  const int n = (int)(endp - start);
-  const Region g = region_of(p, r);
-  const bool is_win = g.window >= 0;
+struct K1Warp {
+  unsigned long long first, last;  // offsets (from lo) of the first / last field-valid record
+  unsigned has, viol, kept;
+};
+
+__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long *bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long *bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long *bar, unsigned parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, unsigned long long *bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+
+template <bool NARROW, bool SMEM>
+__device__ __forceinline__ void partition_scan(const Params &p, const int4 *src, int n, long long lo,
+                                               unsigned long long wlen, bool keep_ok, unsigned long long *ebuf,
+                                               unsigned *cnt, unsigned *kbuf, K1Warp &wr) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
-
-  if (is_win)
-    for (unsigned i = threadIdx.x; i < 8u * p.nbins; i += blockDim.x) cnt[i] = 0;
-  __syncthreads();
-
-  const int4 *src = reinterpret_cast<const int4 *>(p.s) + start;
-  unsigned long long ent[kRecPerLane];
-  unsigned kp[kRecPerLane];  // key << 16 | pos (kNoKey << 16: not kept)
-  long long carry = kTsMin, first = kTsMax;
+  const unsigned nbins = p.nbins;
+  unsigned long long carry = 0, first = 0;
   bool has = false, viol = false;
   unsigned kept = 0;
+  // registered capacities of all 8 records, fetched up front: the table (2 B/buffer) lives in
+  // L2 and its lookups must not sit on the per-record dependency chain
+  unsigned capj[kRecPerLane];
+  if (SMEM) {
 #pragma unroll
-  for (int h = 0; h < 2; ++h) {
-    int4 v[8];
+    for (int j = 0; j < kRecPerLane; ++j) {
+      const int i = warp * 256 + j * 32 + lane;
+      const unsigned b = i < n ? (unsigned)reinterpret_cast<const int *>(src + i)[2] : 0u;
+      capj[j] = __ldg(p.cap + (b < p.nb ? b : 0u));
+    }
+#ifdef RTM_PHASE_TIMING
+    unsigned sink = 0;
 #pragma unroll
-    for (int jj = 0; jj < 8; ++jj) {
-      int i = warp * 512 + (h * 8 + jj) * 32 + lane;
-      v[jj] = i < n ? ld_stream(src + i) : make_int4(0, 0, 0, 0);
+    for (int j = 0; j < kRecPerLane; ++j) sink += capj[j];
+    if (sink == 0xFFFFFFFFu) capj[0] ^= 1;  // force the cap loads to complete here
+    long long ptc = clock64();
+    PT_MARK(p, 7, ptc);
+#endif
+  }
+  constexpr int G = 4;
+#pragma unroll
+  for (int h = 0; h < kRecPerLane / G; ++h) {
+    int4 v[G];
+#pragma unroll
+    for (int jj = 0; jj < G; ++jj) {
+      const int i = warp * 256 + (h * G + jj) * 32 + lane;
+      if (SMEM) v[jj] = i < n ? src[i] : make_int4(0, 0, 0, 0);
+      else v[jj] = i < n ? ld_stream(src + i) : make_int4(0, 0, 0, 0);
     }
 #pragma unroll
-    for (int jj = 0; jj < 8; ++jj) {
-      const int j = h * 8 + jj;
-      const int i = warp * 512 + j * 32 + lane;
-      const bool valid = i < n && sample_valid(p, v[jj]);
-      const long long ts = rec_ts(v[jj]);
-      const unsigned b = (unsigned)v[jj].z;
-      // in-tile order: each field-valid record vs the previous field-valid record (warp order)
+    for (int jj = 0; jj < G; ++jj) {
+      const int i = warp * 256 + (h * G + jj) * 32 + lane;
+      const unsigned b = (unsigned)v[jj].z, lvl = (unsigned)v[jj].w & 0xFFFFu, c = (unsigned)v[jj].w >> 16;
+      const unsigned capb = SMEM ? capj[h * G + jj] : __ldg(p.cap + (b < p.nb ? b : 0u));
+      const bool valid = (i < n) & (b < p.nb) & (c == capb) & (lvl <= c);
+      const unsigned long long off = (unsigned long long)(rec_ts(v[jj]) - lo);
+      const bool inr = off < wlen;
       const unsigned vm = __ballot_sync(kFull, valid);
       const unsigned lower = vm & lt;
-      const long long prev = shfl_ll(ts, lower ? 31 - __clz(lower) : lane);
-      if (valid && ((lower ? prev : carry) > ts || ts < g.lo_ts || ts >= g.hi_ts)) viol = true;
-      if (vm) {
-        if (!has) first = shfl_ll(ts, __ffs(vm) - 1);
-        has = true;
-        carry = shfl_ll(ts, 31 - __clz(vm));
+      const int srcl = lower ? 31 - __clz(lower) : lane;
+      bool bad;
+      if (NARROW) {
+        const unsigned o = (unsigned)off;
+        const unsigned pv = __shfl_sync(kFull, o, srcl);
+        bad = valid & ((!inr) | (o < (lower ? pv : (unsigned)carry)));
+        if (vm) carry = __shfl_sync(kFull, o, 31 - __clz(vm));
+      } else {
+        const unsigned long long pv = __shfl_sync(kFull, off, srcl);
+        bad = valid & ((!inr) | (off < (lower ? pv : carry)));
+        if (vm) carry = __shfl_sync(kFull, off, 31 - __clz(vm));
       }
-      const bool keep = valid && is_win;
+      viol |= bad;
+      if (!has && vm) {
+        first = __shfl_sync(kFull, off, __ffs(vm) - 1);
+        has = true;
+      }
+      const bool keep = valid & keep_ok;
       kept += keep;
-      unsigned key = keep ? (b >> kBinLog) : kNoKey;
+      const unsigned key = keep ? (b >> kBinLog) : kNoKey;
       unsigned pos = 0;
-      if (is_win) {
+      if (keep_ok) {
+        // onesweep-style stable rank: the group leader's shared atomicAdd returns the base
+        // stable rank: every peer reads the (warp, bin) counter, the group leader stores the new
+        // value (plain shared stores: shared atomics cost ~2 cycles per lane on this part)
         const unsigned peers = __match_any_sync(kFull, key);
-        unsigned basec = 0;
-        if (keep) basec = cnt[warp * p.nbins + key];
+        unsigned short *c16 = reinterpret_cast<unsigned short *>(cnt) + warp * nbins;
+        const unsigned basec = keep ? c16[key] : 0u;
         __syncwarp();
-        if (keep && lane == __ffs(peers) - 1) cnt[warp * p.nbins + key] = (unsigned short)(basec + __popc(peers));
+        if (keep && lane == __ffs(peers) - 1) c16[key] = (unsigned short)(basec + __popc(peers));
         __syncwarp();
         pos = basec + __popc(peers & lt);
-        ent[j] = ((unsigned long long)(ts - g.lo_ts) << 24) |
-                 ((unsigned long long)((unsigned)v[jj].w & 0xFFFFu) << 8) | (b & (kBin - 1));
+        if (keep) ebuf[i] = (off << 24) | ((unsigned long long)lvl << 8) | (b & (kBin - 1));
       }
-      kp[j] = (key << 16) | pos;
+      kbuf[i] = (key << 16) | pos;
     }
   }
-  // warp summaries -> tile summary
   kept = warp_sum(kept);
-  const bool wv = __any_sync(kFull, viol);
-  if (lane == 0) {
-    wfirst[warp] = first;
-    wlast[warp] = carry;
-    whas[warp] = has;
-    wviol[warp] = wv;
-    wkept[warp] = kept;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    long long run = kTsMin, tf = 0;
-    bool th = false, tv = false;
-    unsigned tk = 0;
-    for (int w = 0; w < 8; ++w) {
-      tk += wkept[w];
-      tv |= wviol[w] != 0;
-      if (whas[w]) {
-        if (wfirst[w] < run) tv = true;
-        if (!th) tf = wfirst[w];
-        th = true;
-        run = wlast[w];
-      }
-    }
-    TileMeta m;
-    m.first_ts = tf;
-    m.last_ts = run;
-    m.flags = (th ? 1u : 0u) | (tv ? 2u : 0u);
-    m.pad = 0;
-    p.smeta[tile] = m;
-    if ((unsigned)n > tk) atomicAdd(p.win + WF_DROPPED * p.W + g.charge, (unsigned long long)(n - tk));
-    if (tk) atomicAdd(p.win + WF_SAMPLES * p.W + g.window, (unsigned long long)tk);
-    wkept[0] = tk;
-  }
-  if (!is_win) return;
-  __syncthreads();
-  const unsigned total_kept = wkept[0];
+  wr.first = first;
+  wr.last = carry;
+  wr.has = has;
+  wr.viol = __any_sync(kFull, viol);
+  wr.kept = kept;
+}
 
-  // per-bin exclusive prefix over warps, bin totals, exclusive scan over bins
-  const unsigned nb = p.nbins;
-  const unsigned chunk = (nb + blockDim.x - 1) / blockDim.x;
-  const unsigned b0 = threadIdx.x * chunk;
-  unsigned csum = 0;
-  for (unsigned bb = b0; bb < b0 + chunk && bb < nb; ++bb) {
-    unsigned run = 0;
-    for (int w = 0; w < 8; ++w) {
-      unsigned c = cnt[w * nb + bb];
-      cnt[w * nb + bb] = (unsigned short)run;
-      run += c;
+struct K1Smem {            // static shared part of both partition kernels
+  unsigned scan_scratch[32];
+  K1Warp wsum[kK1Warps];
+  unsigned kept;
+};
+
+// Tile bookkeeping shared by both kernels: region, position range, bounds.
+struct TileInfo {
+  long long start;
+  int n;
+  Region g;
+  long long lo;
+  unsigned long long wlen;
+};
+__device__ __forceinline__ TileInfo tile_info(const Params &p, unsigned tile) {
+  TileInfo t;
+  const unsigned r = p.tile_reg_s[tile];
+  t.start = p.Bs[r] + (long long)(tile - p.rts[r]) * kTileS;
+  long long endp = p.Bs[r + 1];
+  if (endp > t.start + kTileS) endp = t.start + kTileS;
+  t.n = (int)(endp - t.start);
+  t.g = region_of(p, r);
+  t.lo = t.g.lo_ts;  // field-valid records of the region need (u64)(ts - lo) < wlen
+  t.wlen = t.g.hi_ts == kTsMax ? (unsigned long long)(kTsMax - t.lo) + 1ull : (unsigned long long)(t.g.hi_ts - t.lo);
+  return t;
+}
+
+// Everything after the per-sample scan: tile meta + drop / kept counts, bin offsets, scatter.
+// Ends with __syncthreads() (the caller may reuse all shared buffers afterwards).
+__device__ __forceinline__ void partition_finish(const Params &p, unsigned tile, const TileInfo &t, K1Smem &K,
+                                                 const K1Warp &wr, const unsigned long long *ebuf, unsigned *binoff,
+                                                 unsigned *cnt, const unsigned *kbuf, unsigned long long *sbuf) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const unsigned nbins = p.nbins;
+  const bool is_win = t.g.window >= 0;
+  if (lane == 0) K.wsum[warp] = wr;
+  __syncthreads();
+  if (warp == 0) {  // tile summary over the 16 warps (lanes 0..15), in warp order
+    K1Warp x;
+    x.first = x.last = 0;
+    x.has = x.viol = x.kept = 0;
+    if (lane < kK1Warps) x = K.wsum[lane];
+    const unsigned hm = __ballot_sync(kFull, x.has != 0);
+    // order across warps: each warp's first valid offset >= the last valid offset of the nearest
+    // earlier warp with valid records (within-warp order was checked in the scan)
+    const unsigned lower = hm & lanemask_lt();
+    const unsigned long long prev_last = __shfl_sync(kFull, x.last, lower ? 31 - __clz(lower) : lane);
+    const bool bad = (x.viol != 0) | ((x.has != 0) & (lower != 0) & (x.first < prev_last));
+    const bool tv = __any_sync(kFull, bad);
+    const unsigned tk = warp_sum(x.kept);
+    const unsigned long long tf = hm ? __shfl_sync(kFull, x.first, __ffs(hm) - 1) : 0ull;
+    const unsigned long long tl = hm ? __shfl_sync(kFull, x.last, 31 - __clz(hm)) : 0ull;
+    if (lane == 0) {
+      TileMeta m;
+      m.first_ts = (long long)((unsigned long long)t.lo + tf);
+      m.last_ts = (long long)((unsigned long long)t.lo + tl);
+      m.flags = (hm ? 1u : 0u) | (tv ? 2u : 0u);
+      m.pad = 0;
+      p.smeta[tile] = m;
+      if ((unsigned)t.n > tk) atomicAdd(p.win + WF_DROPPED * p.W + t.g.charge, (unsigned long long)(t.n - tk));
+      if (tk) atomicAdd(p.win + WF_SAMPLES * p.W + t.g.window, (unsigned long long)tk);
+      K.kept = tk;
     }
-    binoff[bb] = run;
-    csum += run;
   }
-  unsigned base = block_excl_scan(csum, scan_scratch, nullptr);
-  for (unsigned bb = b0; bb < b0 + chunk && bb < nb; ++bb) {
-    unsigned t = binoff[bb];
-    binoff[bb] = base;
-    base += t;
+  long long ptt = clock64();
+  PT_MARK(p, 4, ptt);
+  if (!is_win) {
+    __syncthreads();
+    return;
   }
-  if (threadIdx.x == 0) binoff[nb] = total_kept;
-  __syncthreads();
-  uint32_t *offs = p.soff + (size_t)tile * (nb + 1);
-  for (unsigned bb = threadIdx.x; bb <= nb; bb += blockDim.x) offs[bb] = binoff[bb];
+  // per-bin exclusive prefix over the 16 warps: 16 consecutive lanes hold one bin's warp counts
+  unsigned short *cnt16 = reinterpret_cast<unsigned short *>(cnt);  // u16 [16][nbins]
+  for (unsigned base = 0; base < kK1Warps * nbins; base += blockDim.x) {
+    const unsigned q = base + threadIdx.x;
+    const unsigned bb = q >> 4, w = q & 15u;
+    const bool in = q < kK1Warps * nbins;
+    const unsigned c = in ? cnt16[w * nbins + bb] : 0u;
+    unsigned x = c;
 #pragma unroll
-  for (int j = 0; j < kRecPerLane; ++j) {
-    unsigned key = kp[j] >> 16;
-    if (key != kNoKey) sbuf[binoff[key] + cnt[warp * nb + key] + (kp[j] & 0xFFFFu)] = ent[j];
+    for (int o = 1; o < 16; o <<= 1) {
+      const unsigned y = __shfl_up_sync(kFull, x, o, 16);
+      if (w >= (unsigned)o) x += y;
+    }
+    if (in) {
+      cnt16[w * nbins + bb] = (unsigned short)(x - c);
+      if (w == 15) binoff[bb] = x;  // bin total
+    }
   }
   __syncthreads();
+  const unsigned total_kept = K.kept;
+  if (warp == 0) {  // exclusive scan over bins (nbins <= 3072: <= 96 per lane)
+    unsigned carry = 0;
+    for (unsigned b0 = 0; b0 < nbins; b0 += 32) {
+      const unsigned bb = b0 + lane;
+      const unsigned v = bb < nbins ? binoff[bb] : 0u;
+      unsigned x = v;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned y = __shfl_up_sync(kFull, x, o);
+        if (lane >= o) x += y;
+      }
+      if (bb < nbins) binoff[bb] = carry + x - v;
+      carry += __shfl_sync(kFull, x, 31);
+    }
+    if (lane == 0) binoff[nbins] = total_kept;
+  }
+  __syncthreads();
+  PT_MARK(p, 5, ptt);
+  uint32_t *offs = p.soff + (size_t)tile * (nbins + 1);
+  for (unsigned bb = threadIdx.x; bb <= nbins; bb += blockDim.x) offs[bb] = binoff[bb];
   unsigned long long *dst = p.stage + (size_t)tile * kTileS;
-  for (unsigned i = threadIdx.x; i < total_kept; i += blockDim.x) dst[i] = sbuf[i];
+  unsigned long long *out = sbuf ? sbuf : dst;  // permute in shared memory when a buffer is free
+#pragma unroll 4
+  for (int j = 0; j < kRecPerLane; ++j) {
+    const int i = warp * 256 + j * 32 + lane;
+    const unsigned kv = kbuf[i], key = kv >> 16;
+    if (key != kNoKey && i < t.n) out[binoff[key] + cnt16[warp * nbins + key] + (kv & 0xFFFFu)] = ebuf[i];
+  }
+  __syncthreads();
+  if (sbuf) {  // coalesced 16-byte copy-out of the bin-sorted tile
+    const uint4 *s4 = reinterpret_cast<const uint4 *>(sbuf);
+    uint4 *d4 = reinterpret_cast<uint4 *>(dst);
+    for (unsigned q = threadIdx.x; q < (total_kept + 1) / 2; q += blockDim.x) d4[q] = s4[q];
+    __syncthreads();
+  }
+  PT_MARK(p, 6, ptt);
+  (void)ptt;
+}
+
+__device__ __forceinline__ void zero_counters(const Params &p, unsigned *cnt) {
+  for (unsigned i = threadIdx.x; i < kK1Warps * p.nbins / 2 + 1; i += blockDim.x) cnt[i] = 0;
+}
+
+__global__ void __launch_bounds__(kK1Threads, 2) k_partition(Params p, int narrow) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  unsigned long long *ebuf = reinterpret_cast<unsigned long long *>(smem);  // [4096]
+  unsigned *kbuf = reinterpret_cast<unsigned *>(ebuf + kTileS);             // [4096] key<<16|pos
+  unsigned *binoff = kbuf + kTileS;                                         // [nbins+1]
+  unsigned *cnt = binoff + p.nbins + 1;                                     // u16 [16][nbins]
+  __shared__ K1Smem K;
+  const unsigned tile = blockIdx.x;
+  const TileInfo t = tile_info(p, tile);
+  const bool is_win = t.g.window >= 0;
+  if (is_win) zero_counters(p, cnt);
+  __syncthreads();
+  const int4 *src = reinterpret_cast<const int4 *>(p.s) + t.start;
+  K1Warp wr;
+  if (is_win && narrow) partition_scan<true, false>(p, src, t.n, t.lo, t.wlen, true, ebuf, cnt, kbuf, wr);
+  else partition_scan<false, false>(p, src, t.n, t.lo, t.wlen, is_win, ebuf, cnt, kbuf, wr);
+  partition_finish(p, tile, t, K, wr, ebuf, binoff, cnt, kbuf, nullptr);
+}
+
+__global__ void __launch_bounds__(kK1Threads, 1) k_partition_tma(Params p, int narrow) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  int4 *raw = reinterpret_cast<int4 *>(smem);                                 // [2][4096] records
+  unsigned long long *ebuf = reinterpret_cast<unsigned long long *>(raw + 2 * kTileS);  // [4096]
+  unsigned *kbuf = reinterpret_cast<unsigned *>(ebuf + kTileS);                  // [4096]
+  unsigned *binoff = kbuf + kTileS;                                              // [nbins+1]
+  unsigned *cnt = binoff + p.nbins + 1;                                          // u16 [16][nbins]
+  __shared__ K1Smem K;
+  __shared__ __align__(8) unsigned long long bar[2];
+  if (threadIdx.x == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  auto issue = [&](unsigned tile, int buf) {
+    const TileInfo t = tile_info(p, tile);
+    const unsigned bytes = (unsigned)t.n * 16u;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    mbar_expect_tx(&bar[buf], bytes);
+    bulk_g2s(raw + buf * kTileS, reinterpret_cast<const int4 *>(p.s) + t.start, bytes, &bar[buf]);
+  };
+  unsigned tile = blockIdx.x;
+  if (threadIdx.x == 0 && tile < p.n_tiles_s) issue(tile, 0);
+  for (unsigned it = 0; tile < p.n_tiles_s; ++it, tile += gridDim.x) {
+    const int buf = it & 1;
+    const unsigned next = tile + gridDim.x;
+    if (threadIdx.x == 0 && next < p.n_tiles_s) issue(next, buf ^ 1);  // buffer freed at end of it-1
+    const TileInfo t = tile_info(p, tile);
+    const bool is_win = t.g.window >= 0;
+    if (is_win) zero_counters(p, cnt);
+    __syncthreads();
+#ifdef RTM_PHASE_TIMING
+    long long c0 = clock64();
+#endif
+    mbar_wait(&bar[buf], (it >> 1) & 1u);
+#ifdef RTM_PHASE_TIMING
+    long long c1 = clock64();
+#endif
+    const int4 *src = raw + buf * kTileS;
+    K1Warp wr;
+    if (is_win && narrow) partition_scan<true, true>(p, src, t.n, t.lo, t.wlen, true, ebuf, cnt, kbuf, wr);
+    else partition_scan<false, true>(p, src, t.n, t.lo, t.wlen, is_win, ebuf, cnt, kbuf, wr);
+#ifdef RTM_PHASE_TIMING
+    __syncthreads();
+    long long c2 = clock64();
+#endif
+    // the tile's raw records are consumed: its TMA slot holds the permuted entries
+    partition_finish(p, tile, t, K, wr, ebuf, binoff, cnt, kbuf,
+                     reinterpret_cast<unsigned long long *>(raw + buf * kTileS));
+#ifdef RTM_PHASE_TIMING
+    long long c3 = clock64();
+    if (threadIdx.x == 0 && p.dbg) {
+      atomicAdd(p.dbg + 0, (unsigned long long)(c1 - c0));
+      atomicAdd(p.dbg + 1, (unsigned long long)(c2 - c1));
+      atomicAdd(p.dbg + 2, (unsigned long long)(c3 - c2));
+      atomicAdd(p.dbg + 3, 1ull);
+    }
+#endif
+  }
 }
 
 // ============================================================================================
@@ -437,14 +650,59 @@ __global__ void __launch_bounds__(kK3Threads) k_events(Params p) {
 // L_in from the nearest earlier window with a resolved level (decoupled look-back), finalizes
 // and resolves its own untouched cells.
 // ============================================================================================
+constexpr unsigned kRows = 32;  // bucket rows per lane (8 KB per warp)
 struct FoldSmem {
-  unsigned long long D[kBin];
-  unsigned long long ts0[kBin];
-  unsigned n[kBin];
-  unsigned short cur[kBin], pmax[kBin], pmin[kBin];
-  unsigned long long sc[32];
-  unsigned short sl[32];
+  unsigned long long D[kBin];      // sum_i (l_i - l_{i-1}) * (t_end - ts_i), l_{-1} = 0
+  unsigned long long ts0[kBin];    // offset of the first kept sample in the window
+  unsigned long long cml[kBin];    // cur | max << 16 | min << 32   (levels seen this window)
+  unsigned n[kBin];                // kept samples this window (0: untouched, other fields stale)
+  unsigned bcnt[32];               // records queued per lane bucket
+  unsigned long long bucket[kRows * 32];  // [row][lane]: lane l's bucket holds lids == l (mod 32)
 };
+
+// Lane-private fold of the queued records: lane l owns lids l, l+32, ..., so state updates
+// never conflict; each bucket holds its records in ingest order.
+__device__ __forceinline__ void fold_drain(FoldSmem &S, int lane, unsigned long long Wlen) {
+  const unsigned cnt = S.bcnt[lane];
+  const unsigned mx = __reduce_max_sync(kFull, cnt);
+  for (unsigned r = 0; r < mx; ++r) {
+    if (r < cnt) {
+      const unsigned long long e = S.bucket[r * 32 + lane];
+      const unsigned lid = (unsigned)(e & (kBin - 1));
+      const unsigned lvl = (unsigned)(e >> 8) & 0xFFFFu;
+      const unsigned long long off = e >> 24;
+      const unsigned c0 = S.n[lid];
+      const unsigned long long st = S.cml[lid];
+      const unsigned prev = c0 ? (unsigned)(st & 0xFFFFu) : 0u;
+      unsigned hi = c0 ? (unsigned)(st >> 16) & 0xFFFFu : lvl;
+      unsigned lo = c0 ? (unsigned)(st >> 32) & 0xFFFFu : lvl;
+      hi = lvl > hi ? lvl : hi;
+      lo = lvl < lo ? lvl : lo;
+      const unsigned long long contrib =
+          (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off));
+      S.D[lid] = (c0 ? S.D[lid] : 0ull) + contrib;
+      if (!c0) S.ts0[lid] = off;
+      S.n[lid] = c0 + 1;
+      S.cml[lid] = (unsigned long long)lvl | ((unsigned long long)hi << 16) | ((unsigned long long)lo << 32);
+    }
+  }
+  __syncwarp();
+  S.bcnt[lane] = 0;
+  __syncwarp();
+}
+
+// Queue one chunk of <= 32 records (act lanes) into the lane buckets, preserving ingest order.
+__device__ __forceinline__ void fold_insert(FoldSmem &S, int lane, unsigned lt, bool act, unsigned long long e,
+                                            unsigned long long Wlen) {
+  const unsigned key = act ? (unsigned)(e & 31u) : 32u + (unsigned)lane;
+  const unsigned peers = __match_any_sync(kFull, key);
+  const int leader = __ffs(peers) - 1;
+  if (__any_sync(kFull, act && S.bcnt[key] + __popc(peers) > kRows)) fold_drain(S, lane, Wlen);
+  unsigned base = 0;
+  if (act && lane == leader) base = atomicAdd(&S.bcnt[key], (unsigned)__popc(peers));
+  base = __shfl_sync(kFull, base, leader);
+  if (act) S.bucket[(base + __popc(peers & lt)) * 32 + key] = e;
+}
 
 __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -462,16 +720,10 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
     const unsigned long long Wlen = (unsigned long long)(te - tb);
     const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
 #pragma unroll
-    for (int i = 0; i < kBin / 32; ++i) {
-      const int l = lane + 32 * i;
-      S.D[l] = 0;
-      S.n[l] = 0;
-      S.cur[l] = 0;
-      S.pmax[l] = 0;
-      S.pmin[l] = 0xFFFFu;
-    }
+    for (int i = 0; i < kBin / 32; ++i) S.n[lane + 32 * i] = 0;
+    S.bcnt[lane] = 0;
     __syncwarp();
-    // ---- phase 1: in-order fold over the (tile, bin) segments of window w
+    // ---- phase 1: queue the (tile, bin) segments of window w in tile order, fold per lane
     for (unsigned tg = t_lo; tg < t_hi; tg += 32) {
       unsigned seg_lo = 0, seg_len = 0;
       if (tg + lane < t_hi) {
@@ -480,61 +732,37 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
         seg_len = __ldg(o + 1) - seg_lo;
       }
       const unsigned nseg = min(32u, t_hi - tg);
+      // software pipeline: the first 64 records of segment sg+1 load while sg is queued
+      unsigned len = __shfl_sync(kFull, seg_len, 0);
+      const unsigned long long *seg = p.stage + (size_t)tg * kTileS + __shfl_sync(kFull, seg_lo, 0);
+      unsigned long long e0 = lane < len ? __ldcg(seg + lane) : 0ull;
+      unsigned long long e1 = lane + 32 < len ? __ldcg(seg + 32 + lane) : 0ull;
       for (unsigned sg = 0; sg < nseg; ++sg) {
-        const unsigned lo = __shfl_sync(kFull, seg_lo, sg), len = __shfl_sync(kFull, seg_len, sg);
-        const unsigned long long *seg = p.stage + (size_t)(tg + sg) * kTileS + lo;
-        for (unsigned c = 0; c < len; c += 32) {
+        const unsigned nlen = sg + 1 < nseg ? __shfl_sync(kFull, seg_len, sg + 1) : 0u;
+        const unsigned nlo = __shfl_sync(kFull, seg_lo, sg + 1 < nseg ? sg + 1 : sg);
+        const unsigned long long *nseg_p = p.stage + (size_t)(tg + sg + 1) * kTileS + nlo;
+        const unsigned long long n0 = lane < nlen ? __ldcg(nseg_p + lane) : 0ull;
+        const unsigned long long n1 = lane + 32 < nlen ? __ldcg(nseg_p + 32 + lane) : 0ull;
+        if (len) fold_insert(S, lane, lt, lane < len, e0, Wlen);
+        if (len > 32) fold_insert(S, lane, lt, lane + 32 < len, e1, Wlen);
+        for (unsigned c = 64; c < len; c += 32) {
           const bool act = c + lane < len;
-          const unsigned long long e = act ? __ldcg(seg + c + lane) : 0ull;
-          const unsigned lid = act ? (unsigned)(e & (kBin - 1)) : (unsigned)(kBin + lane);
-          const unsigned lvl = (unsigned)(e >> 8) & 0xFFFFu;
-          const unsigned long long off = e >> 24;
-          const unsigned peers = __match_any_sync(kFull, lid);
-          const unsigned lower = peers & lt;
-          const unsigned plv = __shfl_sync(kFull, lvl, lower ? 31 - __clz(lower) : lane);
-          unsigned long long contrib = 0;
-          if (act) {
-            unsigned prev;
-            if (lower) {
-              prev = plv;
-            } else {
-              prev = S.cur[lid];
-              if (S.n[lid] == 0) S.ts0[lid] = off;
-            }
-            contrib = (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off));
-          }
-          S.sc[lane] = contrib;
-          S.sl[lane] = (unsigned short)lvl;
-          __syncwarp();
-          if (act && (peers >> lane) == 1u) {  // last lane of its group applies the group
-            unsigned long long sum = 0;
-            unsigned mx = 0, mn = 0xFFFFu;
-            unsigned m = peers;
-            while (m) {
-              const int j = __ffs(m) - 1;
-              m &= m - 1;
-              sum += S.sc[j];
-              const unsigned x = S.sl[j];
-              mx = x > mx ? x : mx;
-              mn = x < mn ? x : mn;
-            }
-            S.D[lid] += sum;
-            S.n[lid] += __popc(peers);
-            S.cur[lid] = (unsigned short)lvl;
-            if (mx > S.pmax[lid]) S.pmax[lid] = (unsigned short)mx;
-            if (mn < S.pmin[lid]) S.pmin[lid] = (unsigned short)mn;
-          }
-          __syncwarp();
+          fold_insert(S, lane, lt, act, act ? __ldcg(seg + c + lane) : 0ull, Wlen);
         }
+        seg = nseg_p;
+        len = nlen;
+        e0 = n0;
+        e1 = n1;
       }
     }
+    fold_drain(S, lane, Wlen);
     // ---- publish this window's last levels (kSent: untouched) and the phase-1 flag
     const unsigned b_base = bin * kBin;
     uint16_t *lw = p.lastlvl + (size_t)w * p.nb;
 #pragma unroll
     for (int i = 0; i < kBin / 32; ++i) {
       const unsigned l = lane + 32 * i, b = b_base + l;
-      if (b < p.nb) lw[b] = S.n[l] ? S.cur[l] : kSent;
+      if (b < p.nb) lw[b] = S.n[l] ? (uint16_t)(S.cml[l] & 0xFFFFu) : kSent;
     }
     __threadfence();
     __syncwarp();
@@ -593,10 +821,12 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
       unsigned long long I;
       unsigned mx, mn, last;
       if (cnt) {
+        const unsigned long long st = S.cml[l];
+        const unsigned hi = (unsigned)(st >> 16) & 0xFFFFu, lo = (unsigned)(st >> 32) & 0xFFFFu;
         I = (unsigned long long)L * S.ts0[l] + S.D[l];
-        mx = S.pmax[l] > L ? S.pmax[l] : L;
-        mn = S.pmin[l] < L ? S.pmin[l] : L;
-        last = S.cur[l];
+        mx = hi > L ? hi : L;
+        mn = lo < L ? lo : L;
+        last = (unsigned)(st & 0xFFFFu);
       } else {
         I = (unsigned long long)L * Wlen;
         mx = mn = last = L;
@@ -608,20 +838,17 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
         atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
       }
       if (cnt) {
-        // digest term: splitmix64 finalizer absorbed four times
-        auto fm = [](unsigned long long z) {
-          z ^= z >> 30;
-          z *= 0xbf58476d1ce4e5b9ULL;
-          z ^= z >> 27;
-          z *= 0x94d049bb133111ebULL;
-          z ^= z >> 31;
-          return z;
-        };
-        unsigned long long h = fm(0x9E3779B97F4A7C15ULL ^ (unsigned long long)b);
-        h = fm(h ^ ((unsigned long long)last | ((unsigned long long)mx << 16) | ((unsigned long long)mn << 32) |
-                    ((unsigned long long)capb << 48)));
-        h = fm(h ^ (unsigned long long)cnt);
-        h = fm(h ^ I);
+        // digest term: odd-constant products of (I, n|b, levels), XOR, one fmix64
+        unsigned long long h = (I * 0x9E3779B97F4A7C15ULL) ^
+                               ((((unsigned long long)cnt << 32) | b) * 0xC2B2AE3D27D4EB4FULL) ^
+                               (((unsigned long long)last | ((unsigned long long)mx << 16) |
+                                 ((unsigned long long)mn << 32) | ((unsigned long long)capb << 48)) *
+                                0x165667B19E3779F9ULL);
+        h ^= h >> 30;
+        h *= 0xbf58476d1ce4e5b9ULL;
+        h ^= h >> 27;
+        h *= 0x94d049bb133111ebULL;
+        h ^= h >> 31;
         dig += h;
         ++touched;
       }
@@ -706,64 +933,60 @@ __global__ void __launch_bounds__(1024) k_order_check(const TileMeta *meta, unsi
 // ============================================================================================
 constexpr int kTopkThreads = 512;
 
-__device__ __forceinline__ unsigned fullness_key(unsigned l, unsigned c, int mode) {
+// key32 = floor(l * 2^32 / c) for l < c, exact: m = floor(2^48 / c) (rcp table), q0 = (l*m) >> 16
+// is floor or floor-1 (error < l / 2^16 < 1), one remainder test fixes it.
+__device__ __forceinline__ unsigned fullness_key(unsigned l, unsigned c, int mode, const unsigned long long *rcp) {
   if (mode == RTM_RANK_SIZE) return l;
-  if (l == c) return 0xFFFFFFFFu;
-  return (unsigned)(((unsigned long long)l << 32) / c);
+  if (l >= c) return 0xFFFFFFFFu;  // l == c for field-valid data
+  unsigned long long q = ((unsigned long long)l * __ldg(rcp + c)) >> 16;
+  const unsigned long long r = ((unsigned long long)l << 32) - q * c;
+  if (r >= c) ++q;
+  return (unsigned)q;
 }
 
+template <bool ALL>
 __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
-  const unsigned nb = p.nb;
-  const bool keys_in_smem = nb <= kTopkSmemKeys;
-  unsigned *keys = reinterpret_cast<unsigned *>(smem);                                  // [nb] or none
-  unsigned *hist = keys + (keys_in_smem ? ((nb + 1) & ~1u) : 0);                        // [16][256]
-  unsigned long long *sel = reinterpret_cast<unsigned long long *>(hist + 16 * 256);    // [1024]
+  const unsigned ne = ALL ? p.nb : p.n_elig;  // ranked buffers (ids ascending)
+  const bool keys_in_smem = ne <= kTopkSmemKeys;
+  unsigned *keys = reinterpret_cast<unsigned *>(smem);                                  // [ne] or none
+  unsigned *hist = keys + (keys_in_smem ? ((ne + 1) & ~1u) : 0);                        // [8][256]
+  unsigned long long *sel = reinterpret_cast<unsigned long long *>(hist + 8 * 256);     // [1024]
   __shared__ unsigned scan_scratch[32];
   __shared__ unsigned s_digit, s_need, s_ngt;
   const unsigned w = blockIdx.x;
-  const uint16_t *lv = p.lastlvl + (size_t)w * nb;
+  const uint16_t *lv = p.lastlvl + (size_t)w * p.nb;
   const int warp = threadIdx.x >> 5;
-
-  auto key_of = [&](unsigned b, bool &el) -> unsigned {
-    el = __ldg(p.elig + b) != 0;
-    return fullness_key(lv[b], __ldg(p.cap + b), p.rank_mode);
+  auto id_of = [&](unsigned i) -> unsigned { return ALL ? i : __ldg(p.elig_ids + i); };
+  auto key_at = [&](unsigned i) -> unsigned {
+    if (keys_in_smem) return keys[i];
+    const unsigned b = id_of(i);
+    return fullness_key(lv[b], __ldg(p.cap + b), p.rank_mode, p.rcp);
   };
-  unsigned n_el = 0;
-  if (keys_in_smem) {
-    for (unsigned b = threadIdx.x; b < nb; b += blockDim.x) {
-      bool el;
-      unsigned k = key_of(b, el);
-      keys[b] = k;
-      n_el += el;
+  if (keys_in_smem)
+    for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) {
+      const unsigned b = id_of(i);
+      keys[i] = fullness_key(lv[b], __ldg(p.cap + b), p.rank_mode, p.rcp);
     }
-  } else {
-    for (unsigned b = threadIdx.x; b < nb; b += blockDim.x) n_el += __ldg(p.elig + b) != 0;
-  }
-  unsigned tot_el;
-  block_excl_scan(n_el, scan_scratch, &tot_el);
-  const unsigned keff = p.k < tot_el ? p.k : tot_el;
+  const unsigned keff = p.k < ne ? p.k : ne;
   if (keff == 0) {
     if (threadIdx.x == 0) p.topk_n[w] = 0;
     return;
   }
   unsigned prefix = 0, mask = 0, need = keff;
   for (int d = 3; d >= 0; --d) {
-    for (unsigned i = threadIdx.x; i < 16 * 256; i += blockDim.x) hist[i] = 0;
+    for (unsigned i = threadIdx.x; i < 8 * 256; i += blockDim.x) hist[i] = 0;
     __syncthreads();
-    unsigned *myh = hist + (warp & 15) * 256;
-    for (unsigned b = threadIdx.x; b < nb; b += blockDim.x) {
-      bool el;
-      unsigned k;
-      if (keys_in_smem) { k = keys[b]; el = __ldg(p.elig + b) != 0; }
-      else k = key_of(b, el);
-      if (el && (k & mask) == prefix) atomicAdd(&myh[(k >> (8 * d)) & 255u], 1u);
+    unsigned *myh = hist + (warp & 7) * 256;
+    for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) {
+      const unsigned k = key_at(i);
+      if ((k & mask) == prefix) atomicAdd(&myh[(k >> (8 * d)) & 255u], 1u);
     }
     __syncthreads();
     if (threadIdx.x < 256) {
-      unsigned s = 0;
-      for (int q = 0; q < 16; ++q) s += hist[q * 256 + threadIdx.x];
-      hist[threadIdx.x] = s;  // row 0 now holds totals (rows read before overwrite by owner only)
+      unsigned t = 0;
+      for (int q = 0; q < 8; ++q) t += hist[q * 256 + threadIdx.x];
+      hist[threadIdx.x] = t;  // row 0 <- totals (each thread owns its column)
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -785,38 +1008,24 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
   const unsigned tau = prefix;  // k-th key; `need` keys equal to tau are taken (lowest ids)
   if (threadIdx.x == 0) s_ngt = 0;
   __syncthreads();
-  // keys > tau (count keff - need), any order
-  for (unsigned b = threadIdx.x; b < nb; b += blockDim.x) {
-    bool el;
-    unsigned k;
-    if (keys_in_smem) { k = keys[b]; el = __ldg(p.elig + b) != 0; }
-    else k = key_of(b, el);
-    if (el && k > tau) {
-      unsigned slot = atomicAdd(&s_ngt, 1u);
-      sel[slot] = ((unsigned long long)k << 32) | (0xFFFFFFFFu - b);
-    }
-  }
-  __syncthreads();
-  const unsigned ngt = s_ngt;
-  // keys == tau in id order: contiguous id chunk per thread, block scan for stable ranks
-  const unsigned chunk = (nb + blockDim.x - 1) / blockDim.x;
+  // one pass over contiguous index chunks: keys > tau (any order) and the first `need` keys == tau
+  const unsigned chunk = (ne + blockDim.x - 1) / blockDim.x;
   const unsigned c0 = threadIdx.x * chunk;
   unsigned ceq = 0;
-  for (unsigned b = c0; b < c0 + chunk && b < nb; ++b) {
-    bool el;
-    unsigned k;
-    if (keys_in_smem) { k = keys[b]; el = __ldg(p.elig + b) != 0; }
-    else k = key_of(b, el);
-    ceq += (el && k == tau);
+  for (unsigned i = c0; i < c0 + chunk && i < ne; ++i) {
+    const unsigned k = key_at(i);
+    if (k > tau) {
+      const unsigned slot = atomicAdd(&s_ngt, 1u);
+      sel[slot] = ((unsigned long long)k << 32) | (0xFFFFFFFFu - id_of(i));
+    }
+    ceq += (k == tau);
   }
-  unsigned rank = block_excl_scan(ceq, scan_scratch, nullptr);
-  for (unsigned b = c0; b < c0 + chunk && b < nb && rank < need; ++b) {
-    bool el;
-    unsigned k;
-    if (keys_in_smem) { k = keys[b]; el = __ldg(p.elig + b) != 0; }
-    else k = key_of(b, el);
-    if (el && k == tau) {
-      sel[ngt + rank] = ((unsigned long long)k << 32) | (0xFFFFFFFFu - b);
+  unsigned rank = block_excl_scan(ceq, scan_scratch, nullptr);  // syncs: s_ngt final after it
+  const unsigned ngt = s_ngt;
+  for (unsigned i = c0; i < c0 + chunk && i < ne && rank < need; ++i) {
+    const unsigned k = key_at(i);
+    if (k == tau) {
+      sel[ngt + rank] = ((unsigned long long)k << 32) | (0xFFFFFFFFu - id_of(i));
       ++rank;
     }
   }
@@ -853,29 +1062,46 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
 // ============================================================================================
 // K6: hang flag (L227-L229): cond_c(w) = any buffer of c full for the whole window AND no task
 // event of c in w; run_c counts consecutive cond windows; flagged when run_c >= H.
-// One thread per component; a warp covers one 32-component bitmap word.
+// run_c(w) >= H  <=>  cond_c holds in windows w-H+1..w (reaching back into the carried run_in
+// when w < H-1), so every (window, 32-component word) is flagged independently with bitwise ANDs.
+// Threads [W*ncw, W*ncw + nc) compute the carried run length for the next call.
 // ============================================================================================
+__device__ __forceinline__ unsigned hang_cond(const Params &p, unsigned j, unsigned q) {
+  const size_t i = (size_t)j * p.ncw + q;
+  return __ldg(p.anyfull + i) & ~__ldg(p.active + i);
+}
+
 __global__ void k_hang(Params p) {
-  const unsigned c = blockIdx.x * blockDim.x + threadIdx.x;
-  const unsigned word = c >> 5, bit = c & 31;
-  const bool in = c < p.nc;
-  unsigned run = in ? p.run[c] : 0u;
-  const bool wordok = word < p.ncw;
-  for (unsigned w = 0; w < p.W; ++w) {
-    unsigned f = 0, a = 0;
-    if (wordok) {
-      f = __ldg(p.anyfull + (size_t)w * p.ncw + word);
-      a = __ldg(p.active + (size_t)w * p.ncw + word);
+  const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const size_t nflag = (size_t)p.W * p.ncw;
+  if (tid < nflag) {
+    const unsigned w = (unsigned)(tid / p.ncw), q = (unsigned)(tid % p.ncw);
+    const long long first = (long long)w - (long long)p.H + 1;
+    unsigned acc = 0xFFFFFFFFu;
+    for (long long j = w; j >= (first > 0 ? first : 0) && acc; --j) acc &= hang_cond(p, (unsigned)j, q);
+    if (acc && first < 0) {  // the run must continue the carried run: run_in >= H - (w+1)
+      const unsigned need = p.H - (w + 1);
+      unsigned m = 0;
+      for (unsigned x = acc; x; x &= x - 1) {
+        const unsigned bit = __ffs(x) - 1, c = q * 32 + bit;
+        if (c < p.nc && p.run[c] >= need) m |= 1u << bit;
+      }
+      acc = m;
     }
-    const bool cond = in && ((f >> bit) & 1u) && !((a >> bit) & 1u);
-    run = cond ? run + 1 : 0u;
-    const unsigned fl = __ballot_sync(kFull, in && run >= p.H);
-    if ((threadIdx.x & 31) == 0 && wordok) {
-      p.hung[(size_t)w * p.ncw + word] = fl;
-      if (fl) atomicAdd(p.win + WF_HUNG * p.W + w, (unsigned long long)__popc(fl));
+    if (q == p.ncw - 1 && (p.nc & 31)) acc &= (1u << (p.nc & 31)) - 1u;
+    p.hung[(size_t)w * p.ncw + q] = acc;
+    if (acc) atomicAdd(p.win + WF_HUNG * p.W + w, (unsigned long long)__popc(acc));
+  } else if (tid < nflag + p.nc) {
+    const unsigned c = (unsigned)(tid - nflag), q = c >> 5, bit = c & 31;
+    unsigned r = 0;
+    long long j = (long long)p.W - 1;
+    for (; j >= 0; --j) {
+      if ((hang_cond(p, (unsigned)j, q) >> bit) & 1u) ++r;
+      else break;
     }
+    if (j < 0) r += p.run[c];
+    p.run_out[c] = r;
   }
-  if (in) p.run[c] = run;
 }
 
 // ============================================================================================
@@ -951,10 +1177,11 @@ __host__ __device__ inline PackLayout pack_layout(const Params &p) {
   return L;
 }
 
-__device__ __forceinline__ unsigned long long topk_composite(unsigned long long ent, int mode) {
+__device__ __forceinline__ unsigned long long topk_composite(unsigned long long ent, int mode,
+                                                             const unsigned long long *rcp) {
   const unsigned b = (unsigned)(ent & 0xFFFFFFFFu);
   const unsigned l = (unsigned)(ent >> 32) & 0xFFFFu, c = (unsigned)(ent >> 48);
-  return ((unsigned long long)fullness_key(l, c, mode) << 32) | (0xFFFFFFFFu - b);
+  return ((unsigned long long)fullness_key(l, c, mode, rcp) << 32) | (0xFFFFFFFFu - b);
 }
 
 // one CTA per window: merge world x k candidates; sums of scalar fields; progress sums; hang OR
@@ -976,7 +1203,7 @@ __global__ void __launch_bounds__(256) k_merge_windows(Params p, const unsigned 
       const unsigned n = reinterpret_cast<const unsigned *>(base + L.topk_n)[w];
       if (s < n) {
         en = reinterpret_cast<const unsigned long long *>(base + L.topk)[(size_t)w * p.k + s];
-        key = topk_composite(en, p.rank_mode);
+        key = topk_composite(en, p.rank_mode, p.rcp);
       }
     }
     cand[i] = key;
@@ -1065,10 +1292,14 @@ __global__ void k_merge_tables(Params p, const unsigned char *g, unsigned world,
 // ============================================================================================
 size_t fold_smem_bytes() { return sizeof(FoldSmem) * kFoldWarps; }
 size_t partition_smem_bytes(uint32_t nbins) {
-  return (size_t)kTileS * 8 + (size_t)(nbins + 1) * 4 + (size_t)8 * nbins * 2 + 16;
+  return (size_t)kTileS * 8 + (size_t)kTileS * 4 + (size_t)(nbins + 1) * 4 + ((size_t)kK1Warps * nbins / 2 + 1) * 4 + 16;
 }
+size_t partition_tma_smem_bytes(uint32_t nbins) { return (size_t)2 * kTileS * 16 + partition_smem_bytes(nbins); }
+static_assert((size_t)2 * kTileS * 16 + (size_t)kTileS * 12 + (size_t)(kTmaMaxBins + 1) * 4 +
+                      ((size_t)kK1Warps * kTmaMaxBins / 2 + 1) * 4 + 16 <= 227 * 1024,
+              "TMA partition shared memory exceeds the 227 KB opt-in limit");
 size_t topk_smem_bytes(uint32_t nb) {
-  return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 16 * 256 * 4 + 1024 * 8;
+  return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8;
 }
 
 void launch_split(const Params &p, bool samples, long long *outB, cudaStream_t st) {
@@ -1086,10 +1317,15 @@ void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
   if (p.n_tiles_e) k_fill_tile_regions<<<blocks, 64, 0, st>>>(p.rte, const_cast<uint32_t *>(p.tile_reg_e), nr);
 }
 
-void launch_partition(const Params &p, cudaStream_t st) {
+void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   if (!p.n_tiles_s) return;
-  const size_t sm = partition_smem_bytes(p.nbins);
-  k_partition<<<p.n_tiles_s, kK1Threads, sm, st>>>(p);
+  static const bool use_tma = getenv("RTM_TMA") != nullptr;  // measured slower on C2
+  if (p.nbins <= kTmaMaxBins && use_tma) {
+    const unsigned grid = p.n_tiles_s < (unsigned)n_sms ? p.n_tiles_s : (unsigned)n_sms;
+    k_partition_tma<<<grid, kK1Threads, partition_tma_smem_bytes(p.nbins), st>>>(p, p.narrow);
+  } else {
+    k_partition<<<p.n_tiles_s, kK1Threads, partition_smem_bytes(p.nbins), st>>>(p, p.narrow);
+  }
 }
 
 void launch_events(const Params &p, cudaStream_t st) {
@@ -1117,13 +1353,14 @@ void launch_order_check(const Params &p, cudaStream_t st) {
 }
 
 void launch_topk(const Params &p, cudaStream_t st) {
-  k_topk<<<p.W, kTopkThreads, topk_smem_bytes(p.nb), st>>>(p);
+  if (p.n_elig == p.nb) k_topk<true><<<p.W, kTopkThreads, topk_smem_bytes(p.nb), st>>>(p);
+  else k_topk<false><<<p.W, kTopkThreads, topk_smem_bytes(p.n_elig), st>>>(p);
 }
 
 void launch_hang(const Params &p, cudaStream_t st) {
-  const unsigned threads = 128;
-  const unsigned blocks = (p.ncw * 32 + threads - 1) / threads;
-  k_hang<<<blocks, threads, 0, st>>>(p);
+  const unsigned threads = 256;
+  const size_t n = (size_t)p.W * p.ncw + p.nc;
+  k_hang<<<(unsigned)((n + threads - 1) / threads), threads, 0, st>>>(p);
 }
 
 void launch_progress(const Params &p, cudaStream_t st) {
@@ -1141,7 +1378,11 @@ void configure_kernels_once() {
   done[dev] = true;
   cudaFuncSetAttribute(k_partition, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)partition_smem_bytes(kMaxBins));
-  cudaFuncSetAttribute(k_topk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
+  cudaFuncSetAttribute(k_partition_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       (int)partition_tma_smem_bytes(kTmaMaxBins));
+  cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
+  cudaFuncSetAttribute(k_topk<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       (int)topk_smem_bytes(kTopkSmemKeys));
   cudaFuncSetAttribute(k_fold, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
   cudaGetLastError();
 }

@@ -33,6 +33,22 @@ def test_splitmix64_known_vector():
     assert brute.fmix64(0x9E3779B97F4A7C15) == 0xE220A8397B1DCDAF
 
 
+def test_digest_term_detects_any_single_field_change():
+    """DESIGN.md reading R17: odd-constant products are bijections and fmix64 is a bijection, so
+    changing exactly one field (buffer, last, max, min, cap, n, integral) always changes the term."""
+    rng = np.random.default_rng(9)
+    for _ in range(300):
+        f = [int(rng.integers(0, 2**31)), *(int(x) for x in rng.integers(0, 65536, 4)), int(rng.integers(0, 2**32)),
+             int(rng.integers(-(2**62), 2**62))]
+        base = oracle.digest_term(*f)
+        for i in range(7):
+            g = list(f)
+            g[i] = g[i] + 1 if i != 6 else g[i] - 12345
+            if i in (1, 2, 3, 4):
+                g[i] &= 0xFFFF
+            assert oracle.digest_term(*g) != base, i
+
+
 def test_digest_term_matches_spec_retyped():
     rng = np.random.default_rng(7)
     for _ in range(200):
@@ -387,3 +403,30 @@ def test_shard_merge_equals_whole():
     for sh in shards:
         hung |= sh["hung"]
     assert np.array_equal(hung, whole["hung"])
+
+
+def test_gpu_fullness_key_reciprocal_formula_is_exact():
+    """The CUDA top-k computes floor(l*2^32/c) as q0 = (l*m)>>16, m = floor(2^48/c), plus one
+    remainder fix-up (DESIGN.md §4 K5).  Emulated here exhaustively for small caps and on random
+    pairs for large ones; it must equal the exact floor."""
+    def gpu_key(l, c):
+        if l >= c:
+            return 0xFFFFFFFF
+        m = (1 << 48) // c if c >= 2 else 0
+        q = (l * m) >> 16
+        r = (l << 32) - q * c
+        if r >= c:
+            q += 1
+        return q
+
+    for c in range(1, 300):
+        for l in range(0, c):
+            assert gpu_key(l, c) == (l << 32) // c
+    rng = np.random.default_rng(11)
+    for _ in range(50000):
+        c = int(rng.integers(2, 65535))
+        l = int(rng.integers(0, c))
+        assert gpu_key(l, c) == (l << 32) // c
+    for c in (65533, 65534, 40961, 32768, 32769):
+        for l in (0, 1, c // 2, c - 2, c - 1):
+            assert gpu_key(l, c) == (l << 32) // c
