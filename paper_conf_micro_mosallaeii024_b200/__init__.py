@@ -140,7 +140,8 @@ class Monitor:
     def _reduce_distributed(self, t_end, summ):
         """world > 1: local reduce -> all-gather of the packed per-window results -> merge kernels."""
         import torch
-        import torch.distributed as dist
+
+        from .dist import allgather_packs
 
         pack = ctypes.c_void_p()
         nbytes = ctypes.c_uint64()
@@ -150,8 +151,7 @@ class Monitor:
         dev = torch.device("cuda", self.device)
         send = torch.empty(n, dtype=torch.uint8, device=dev)
         _copy_from_ptr(send, pack.value, n)
-        recv = torch.empty(self.world * n, dtype=torch.uint8, device=dev)
-        dist.all_gather_into_tensor(recv, send, group=self._pg)
+        recv = allgather_packs(send, self.world, self._pg)
         torch.cuda.current_stream(dev).synchronize()
         N.check(N.lib().rtm_merge(self._h, recv.data_ptr(), self.world, summ.ctypes.data), "rtm_merge")
 
