@@ -650,58 +650,67 @@ __global__ void __launch_bounds__(kK3Threads) k_events(Params p) {
 // L_in from the nearest earlier window with a resolved level (decoupled look-back), finalizes
 // and resolves its own untouched cells.
 // ============================================================================================
-constexpr unsigned kRows = 32;  // bucket rows per lane (8 KB per warp)
 struct FoldSmem {
   unsigned long long D[kBin];      // sum_i (l_i - l_{i-1}) * (t_end - ts_i), l_{-1} = 0
   unsigned long long ts0[kBin];    // offset of the first kept sample in the window
   unsigned long long cml[kBin];    // cur | max << 16 | min << 32   (levels seen this window)
   unsigned n[kBin];                // kept samples this window (0: untouched, other fields stale)
-  unsigned bcnt[32];               // records queued per lane bucket
-  unsigned long long bucket[kRows * 32];  // [row][lane]: lane l's bucket holds lids == l (mod 32)
 };
 
-// Lane-private fold of the queued records: lane l owns lids l, l+32, ..., so state updates
-// never conflict; each bucket holds its records in ingest order.
-__device__ __forceinline__ void fold_drain(FoldSmem &S, int lane, unsigned long long Wlen) {
-  const unsigned cnt = S.bcnt[lane];
-  const unsigned mx = __reduce_max_sync(kFull, cnt);
-  for (unsigned r = 0; r < mx; ++r) {
-    if (r < cnt) {
-      const unsigned long long e = S.bucket[r * 32 + lane];
-      const unsigned lid = (unsigned)(e & (kBin - 1));
-      const unsigned lvl = (unsigned)(e >> 8) & 0xFFFFu;
-      const unsigned long long off = e >> 24;
-      const unsigned c0 = S.n[lid];
-      const unsigned long long st = S.cml[lid];
-      const unsigned prev = c0 ? (unsigned)(st & 0xFFFFu) : 0u;
-      unsigned hi = c0 ? (unsigned)(st >> 16) & 0xFFFFu : lvl;
-      unsigned lo = c0 ? (unsigned)(st >> 32) & 0xFFFFu : lvl;
-      hi = lvl > hi ? lvl : hi;
-      lo = lvl < lo ? lvl : lo;
-      const unsigned long long contrib =
-          (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off));
-      S.D[lid] = (c0 ? S.D[lid] : 0ull) + contrib;
-      if (!c0) S.ts0[lid] = off;
-      S.n[lid] = c0 + 1;
-      S.cml[lid] = (unsigned long long)lvl | ((unsigned long long)hi << 16) | ((unsigned long long)lo << 32);
+// One chunk of <= 32 consecutive records (ingest order) of one (window, bin) unit.  Records of
+// the same buffer (peers, found with __match_any_sync) form a chain in lane order: each record's
+// predecessor level is the previous peer's (shuffle) or, for the chain head, the buffer's state.
+// Contributions are computed in parallel; the group's sum / max / min travel down the chain in
+// `maxrank` shuffle steps and only the chain's last lane updates the shared state, so every
+// state update in a chunk touches a distinct buffer.
+__device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, bool act, unsigned long long e,
+                                           unsigned long long Wlen) {
+  const unsigned lid = act ? (unsigned)(e & (kBin - 1)) : (unsigned)(kBin + lane);
+  const unsigned lvl = (unsigned)(e >> 8) & 0xFFFFu;
+  const unsigned long long off = e >> 24;
+  const unsigned peers = __match_any_sync(kFull, lid);
+  const unsigned lower = peers & lt;
+  const int pred = lower ? 31 - __clz(lower) : lane;
+  const unsigned rank = __popc(lower);
+  const bool tail = (peers >> lane) == 1u;
+  const unsigned plv = __shfl_sync(kFull, lvl, pred);
+  unsigned c0 = 0;
+  unsigned long long st = 0;
+  if (act && (!lower || tail)) {  // chain heads need the state's level, tails update the state
+    c0 = S.n[lid];
+    st = S.cml[lid];
+  }
+  const unsigned prev = lower ? plv : (c0 ? (unsigned)(st & 0xFFFFu) : 0u);
+  const unsigned long long contrib =
+      act ? (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off)) : 0ull;
+  unsigned long long sum = contrib;
+  unsigned mm = (lvl << 16) | lvl;  // max << 16 | min over the chain so far
+  const unsigned maxrank = __reduce_max_sync(kFull, rank);
+  for (unsigned k = 0; k < maxrank; ++k) {
+    const unsigned long long su = __shfl_sync(kFull, sum, pred);
+    const unsigned mu = __shfl_sync(kFull, mm, pred);
+    if (lower) {
+      sum = contrib + su;
+      const unsigned hi = max(lvl, mu >> 16), lo = min(lvl, mu & 0xFFFFu);
+      mm = (hi << 16) | lo;
     }
   }
+  const unsigned long long off0 = __shfl_sync(kFull, off, __ffs(peers) - 1);  // chain head's offset
+  if (act && tail) {
+    unsigned hi = mm >> 16, lo = mm & 0xFFFFu;
+    unsigned long long d = sum;
+    if (c0) {
+      hi = max(hi, (unsigned)(st >> 16) & 0xFFFFu);
+      lo = min(lo, (unsigned)(st >> 32) & 0xFFFFu);
+      d += S.D[lid];
+    } else {
+      S.ts0[lid] = off0;
+    }
+    S.D[lid] = d;
+    S.n[lid] = c0 + rank + 1;
+    S.cml[lid] = (unsigned long long)lvl | ((unsigned long long)hi << 16) | ((unsigned long long)lo << 32);
+  }
   __syncwarp();
-  S.bcnt[lane] = 0;
-  __syncwarp();
-}
-
-// Queue one chunk of <= 32 records (act lanes) into the lane buckets, preserving ingest order.
-__device__ __forceinline__ void fold_insert(FoldSmem &S, int lane, unsigned lt, bool act, unsigned long long e,
-                                            unsigned long long Wlen) {
-  const unsigned key = act ? (unsigned)(e & 31u) : 32u + (unsigned)lane;
-  const unsigned peers = __match_any_sync(kFull, key);
-  const int leader = __ffs(peers) - 1;
-  if (__any_sync(kFull, act && S.bcnt[key] + __popc(peers) > kRows)) fold_drain(S, lane, Wlen);
-  unsigned base = 0;
-  if (act && lane == leader) base = atomicAdd(&S.bcnt[key], (unsigned)__popc(peers));
-  base = __shfl_sync(kFull, base, leader);
-  if (act) S.bucket[(base + __popc(peers & lt)) * 32 + key] = e;
 }
 
 __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
@@ -721,9 +730,8 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
     const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
 #pragma unroll
     for (int i = 0; i < kBin / 32; ++i) S.n[lane + 32 * i] = 0;
-    S.bcnt[lane] = 0;
     __syncwarp();
-    // ---- phase 1: queue the (tile, bin) segments of window w in tile order, fold per lane
+    // ---- phase 1: the (tile, bin) segments of window w, flattened into one stream of chunks
     for (unsigned tg = t_lo; tg < t_hi; tg += 32) {
       unsigned seg_lo = 0, seg_len = 0;
       if (tg + lane < t_hi) {
@@ -731,31 +739,34 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
         seg_lo = __ldg(o);
         seg_len = __ldg(o + 1) - seg_lo;
       }
-      const unsigned nseg = min(32u, t_hi - tg);
-      // software pipeline: the first 64 records of segment sg+1 load while sg is queued
-      unsigned len = __shfl_sync(kFull, seg_len, 0);
-      const unsigned long long *seg = p.stage + (size_t)tg * kTileS + __shfl_sync(kFull, seg_lo, 0);
-      unsigned long long e0 = lane < len ? __ldcg(seg + lane) : 0ull;
-      unsigned long long e1 = lane + 32 < len ? __ldcg(seg + 32 + lane) : 0ull;
-      for (unsigned sg = 0; sg < nseg; ++sg) {
-        const unsigned nlen = sg + 1 < nseg ? __shfl_sync(kFull, seg_len, sg + 1) : 0u;
-        const unsigned nlo = __shfl_sync(kFull, seg_lo, sg + 1 < nseg ? sg + 1 : sg);
-        const unsigned long long *nseg_p = p.stage + (size_t)(tg + sg + 1) * kTileS + nlo;
-        const unsigned long long n0 = lane < nlen ? __ldcg(nseg_p + lane) : 0ull;
-        const unsigned long long n1 = lane + 32 < nlen ? __ldcg(nseg_p + 32 + lane) : 0ull;
-        if (len) fold_insert(S, lane, lt, lane < len, e0, Wlen);
-        if (len > 32) fold_insert(S, lane, lt, lane + 32 < len, e1, Wlen);
-        for (unsigned c = 64; c < len; c += 32) {
-          const bool act = c + lane < len;
-          fold_insert(S, lane, lt, act, act ? __ldcg(seg + c + lane) : 0ull, Wlen);
+      unsigned pre = seg_len;  // inclusive prefix of segment lengths over lanes
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned y = __shfl_up_sync(kFull, pre, o);
+        if (lane >= o) pre += y;
+      }
+      const unsigned total = __shfl_sync(kFull, pre, 31);
+      unsigned sgi = 0;  // this lane's current segment (cursor)
+      auto fetch = [&](unsigned g) -> unsigned long long {
+        // advance the cursor to the segment holding flattened index g (< 32 segments)
+        for (;;) {
+          const unsigned end = __shfl_sync(kFull, pre, sgi & 31);
+          const bool adv = g < total && g >= end;
+          if (!__any_sync(kFull, adv)) break;
+          if (adv) ++sgi;
         }
-        seg = nseg_p;
-        len = nlen;
-        e0 = n0;
-        e1 = n1;
+        const unsigned base = __shfl_sync(kFull, pre - seg_len, sgi & 31);
+        const unsigned lo = __shfl_sync(kFull, seg_lo, sgi & 31);
+        if (g >= total) return 0ull;
+        return __ldcg(p.stage + (size_t)(tg + sgi) * kTileS + lo + (g - base));
+      };
+      unsigned long long e = fetch(lane);
+      for (unsigned c = 0; c < total; c += 32) {
+        const unsigned long long en = fetch(c + 32 + lane);  // prefetch the next chunk
+        fold_chunk(S, lane, lt, c + lane < total, e, Wlen);
+        e = en;
       }
     }
-    fold_drain(S, lane, Wlen);
     // ---- publish this window's last levels (kSent: untouched) and the phase-1 flag
     const unsigned b_base = bin * kBin;
     uint16_t *lw = p.lastlvl + (size_t)w * p.nb;
