@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -44,6 +45,8 @@ struct rtm_ctx {
   rtm_allgather_fn allgather;
   void *allgather_user;
   cudaStream_t st;
+  cudaStream_t st2 = nullptr;            // side stream (task events), joined per call
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   int n_sms;
   DevBuf cap, owner, elig, ktotal, rcp, elig_ids;
   uint32_t n_elig = 0;
@@ -81,17 +84,18 @@ struct rtm_ctx {
 
 namespace {
 
-rtm_status cuda_fail(rtm_ctx *c, cudaError_t e) {
-  (void)e;
+rtm_status cuda_fail(rtm_ctx *c, cudaError_t e, const char *what, int line) {
+  static const bool dbg = getenv("RTM_DEBUG") != nullptr;
+  if (dbg) fprintf(stderr, "[rtm] CUDA error %d (%s) at rtm_api.cpp:%d: %s\n", (int)e, cudaGetErrorString(e), line, what);
   cudaGetLastError();
   if (c) c->sticky = RTM_E_CUDA;
   return RTM_E_CUDA;
 }
 
-#define CK(call)                                     \
-  do {                                               \
-    cudaError_t e_ = (call);                         \
-    if (e_ != cudaSuccess) return cuda_fail(c, e_);  \
+#define CK(call)                                                    \
+  do {                                                              \
+    cudaError_t e_ = (call);                                        \
+    if (e_ != cudaSuccess) return cuda_fail(c, e_, #call, __LINE__); \
   } while (0)
 
 rtm_status ensure(rtm_ctx *c, DevBuf &b, size_t bytes, bool zero_new = false) {
@@ -114,7 +118,7 @@ rtm_status ensure(rtm_ctx *c, DevBuf &b, size_t bytes, bool zero_new = false) {
     return RTM_E_NOMEM;
   }
   b.cap = want;
-  if (zero_new && cudaMemset(b.p, 0, want) != cudaSuccess) return cuda_fail(c, cudaGetLastError());
+  if (zero_new && cudaMemset(b.p, 0, want) != cudaSuccess) return cuda_fail(c, cudaGetLastError(), "memset", __LINE__);
   return RTM_OK;
 }
 
@@ -171,6 +175,14 @@ void prof_begin(rtm_ctx *c, int kid, uint64_t bytes) {
 void prof_end(rtm_ctx *c) {
   if (!c->prof || c->marks.empty()) return;
   cudaEventRecord(c->marks.back().b, c->st);
+}
+void prof_begin_on(rtm_ctx *c, int kid, uint64_t bytes, cudaStream_t st) {
+  prof_begin(c, kid, bytes);  // records on c->st: re-record on the side stream
+  if (c->prof && !c->marks.empty()) cudaEventRecord(c->marks.back().a, st);
+}
+void prof_end_on(rtm_ctx *c, cudaStream_t st) {
+  if (!c->prof || c->marks.empty()) return;
+  cudaEventRecord(c->marks.back().b, st);
 }
 void prof_collect(rtm_ctx *c) {  // after a stream sync
   for (auto &m : c->marks) {
@@ -251,24 +263,6 @@ rtm_status append(rtm_ctx *c, std::vector<Chunk> &dev, DevBuf &own, uint64_t &ow
   return RTM_OK;
 }
 
-// Host-side region/tile bookkeeping from the split positions.
-uint32_t regions_to_tiles(std::vector<long long> &B, uint64_t N, uint32_t W, int tile, std::vector<uint32_t> &rt) {
-  B[0] = 0;
-  B[W + 2] = (long long)N;
-  for (uint32_t r = 1; r <= W + 2; ++r) {
-    if (B[r] < B[r - 1]) B[r] = B[r - 1];  // only for unsorted input (reported as RTM_E_ORDER)
-    if (B[r] > (long long)N) B[r] = (long long)N;
-  }
-  rt.assign(W + 3, 0);
-  uint32_t t = 0;
-  for (uint32_t r = 0; r <= W + 1; ++r) {
-    rt[r] = t;
-    t += (uint32_t)((B[r + 1] - B[r] + tile - 1) / tile);
-  }
-  rt[W + 2] = t;
-  return t;
-}
-
 // The local (per-rank) part of a reduce call.  On success the device result arrays hold this
 // rank's per-window results for n_windows windows.
 rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p) {
@@ -292,13 +286,9 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   if ((s = ensure(c, c->Be, (size_t)(W + 3) * 8))) return s;
   if ((s = ensure(c, c->rts, (size_t)(W + 3) * 4))) return s;
   if ((s = ensure(c, c->rte, (size_t)(W + 3) * 4))) return s;
-  const size_t small = (size_t)(W + 3) * 8 * 2 + (size_t)(W + 3) * 4 * 2 + (size_t)(W + 1) * 8;
+  const size_t small = (size_t)(W + 1) * 8;
   if ((s = ensure_pinned(c, c->h_small, small))) return s;
   long long *hT = (long long *)c->h_small.p;
-  long long *hBs = hT + (W + 1);
-  long long *hBe = hBs + (W + 3);
-  uint32_t *hrts = (uint32_t *)(hBe + (W + 3));
-  uint32_t *hrte = hrts + (W + 3);
   hT[0] = c->t_prev;
   for (uint32_t w = 0; w < W; ++w) hT[w + 1] = t_end[w];
   CK(cudaMemcpyAsync(c->T.p, hT, (size_t)(W + 1) * 8, cudaMemcpyHostToDevice, c->st));
@@ -319,22 +309,13 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
 
   LAUNCH(KT_SPLIT, 0, launch_split(p, true, (long long *)c->Bs.p + 1, c->st));
   LAUNCH(KT_SPLIT, 0, launch_split(p, false, (long long *)c->Be.p + 1, c->st));
+  p.Bs = (const long long *)c->Bs.p; p.Be = (const long long *)c->Be.p;
+  p.rts = (const uint32_t *)c->rts.p; p.rte = (const uint32_t *)c->rte.p;
+  launch_regions(p, c->st);  // region tile tables on the device: no host round trip
   CK(cudaGetLastError());
-  CK(cudaMemcpyAsync(hBs + 1, (long long *)c->Bs.p + 1, (size_t)(W + 1) * 8, cudaMemcpyDeviceToHost, c->st));
-  CK(cudaMemcpyAsync(hBe + 1, (long long *)c->Be.p + 1, (size_t)(W + 1) * 8, cudaMemcpyDeviceToHost, c->st));
-  CK(cudaStreamSynchronize(c->st));
-  std::vector<long long> Bs(hBs, hBs + W + 3), Be(hBe, hBe + W + 3);
-  std::vector<uint32_t> rts, rte;
-  const uint32_t nts = regions_to_tiles(Bs, ns, W, kTileS, rts);
-  const uint32_t nte = regions_to_tiles(Be, ne, W, kTileE, rte);
-  memcpy(hBs, Bs.data(), (W + 3) * 8);
-  memcpy(hBe, Be.data(), (W + 3) * 8);
-  memcpy(hrts, rts.data(), (W + 3) * 4);
-  memcpy(hrte, rte.data(), (W + 3) * 4);
-  CK(cudaMemcpyAsync(c->Bs.p, hBs, (size_t)(W + 3) * 8, cudaMemcpyHostToDevice, c->st));
-  CK(cudaMemcpyAsync(c->Be.p, hBe, (size_t)(W + 3) * 8, cudaMemcpyHostToDevice, c->st));
-  CK(cudaMemcpyAsync(c->rts.p, hrts, (size_t)(W + 3) * 4, cudaMemcpyHostToDevice, c->st));
-  CK(cudaMemcpyAsync(c->rte.p, hrte, (size_t)(W + 3) * 4, cudaMemcpyHostToDevice, c->st));
+  // tile-count upper bounds: every region adds at most one partial tile
+  const uint32_t nts = (uint32_t)((ns + kTileS - 1) / kTileS) + W + 2;
+  const uint32_t nte = (uint32_t)((ne + kTileE - 1) / kTileE) + W + 2;
 
   // ---- workspaces
   const size_t Wn = W;
@@ -370,8 +351,6 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   CK(cudaMemsetAsync(c->unit_ctr.p, 0, 8, c->st));
   CK(cudaMemsetAsync(c->status.p, 0, 8, c->st));
 
-  p.Bs = (const long long *)c->Bs.p; p.Be = (const long long *)c->Be.p;
-  p.rts = (const uint32_t *)c->rts.p; p.rte = (const uint32_t *)c->rte.p;
   p.tile_reg_s = (const uint32_t *)c->treg_s.p; p.tile_reg_e = (const uint32_t *)c->treg_e.p;
   p.n_tiles_s = nts; p.n_tiles_e = nte;
   p.soff = (uint32_t *)c->soff.p; p.stage = (unsigned long long *)c->stage.p;
@@ -397,9 +376,17 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.dbg = dbg;
 #endif
   launch_fill_tile_regions(p, c->st);
+  // task events are independent of the sample path: run them on a side stream, overlapped with
+  // the partition and the fold, and join before the kernels that read their outputs
+  CK(cudaEventRecord(c->ev_fork, c->st));
+  CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
+  if (c->prof) prof_begin_on(c, KT_EVENTS, (uint64_t)ne * 16, c->st2);
+  launch_events(p, c->st2);
+  if (c->prof) prof_end_on(c, c->st2);
+  CK(cudaEventRecord(c->ev_join, c->st2));
   LAUNCH(KT_PARTITION, (uint64_t)ns * 16, launch_partition(p, c->n_sms, c->st));
-  LAUNCH(KT_EVENTS, (uint64_t)ne * 16, launch_events(p, c->st));
   LAUNCH(KT_FOLD, 0, launch_fold(p, c->n_sms, c->st));
+  CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
   LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
   LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
   LAUNCH(KT_HANG, 0, launch_hang(p, c->st));
@@ -536,6 +523,13 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   if (cudaSetDevice(c->device) != cudaSuccess) { cudaGetLastError(); delete c; return RTM_E_CUDA; }
   configure_kernels_once();
   cudaDeviceGetAttribute(&c->n_sms, cudaDevAttrMultiProcessorCount, c->device);
+  if (cudaStreamCreateWithFlags(&c->st2, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess) {
+    cudaGetLastError();
+    delete c;
+    return RTM_E_CUDA;
+  }
   rtm_status s = RTM_OK;
   auto fail = [&](rtm_status e) { rtm_destroy(c); return e; };
   if ((s = ensure(c, c->cap, (size_t)c->nb * 2)) || (s = ensure(c, c->owner, (size_t)c->nb * 4)) ||
@@ -589,6 +583,9 @@ void rtm_destroy(rtm_ctx *c) {
   if (c->h_small.p) cudaFreeHost(c->h_small.p);
   if (c->h_res.p) cudaFreeHost(c->h_res.p);
   for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
+  if (c->st2) cudaStreamSynchronize(c->st2), cudaStreamDestroy(c->st2);
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_join) cudaEventDestroy(c->ev_join);
   cudaGetLastError();
   delete c;
 }

@@ -32,7 +32,7 @@ constexpr int kK1Threads = 512;             // 16 warps x 8 records per lane
 constexpr int kK3Threads = 256;
 constexpr int kFoldWarps = 4;               // warps per fold CTA
 constexpr uint16_t kSent = 0xFFFFu;         // "no kept sample in this window" marker
-constexpr uint32_t kMaxBins = 3072;         // n_buffers <= 786432 (partition smem <= 204 KB)
+constexpr uint32_t kMaxBins = 1024;         // n_buffers <= 262144 (partition smem <= 227 KB)
 constexpr uint32_t kTopkSmemKeys = 40960;   // keys held in shared memory by the top-k kernel
 constexpr int64_t kMaxWindowLen = (int64_t)1 << 40;  // ts offset field of a staging entry
 
@@ -81,7 +81,7 @@ struct Params {
   const uint32_t *rte;
   const uint32_t *tile_reg_s;// [n_tiles_s] region of each tile
   const uint32_t *tile_reg_e;
-  uint32_t n_tiles_s, n_tiles_e;
+  uint32_t n_tiles_s, n_tiles_e;  // upper bounds (grid sizes); device counts are rts/rte[W+2]
   // outputs / workspaces
   uint32_t *soff;            // [n_tiles_s * (nbins+1)]
   unsigned long long *stage; // [n_tiles_s * kTileS]
@@ -112,6 +112,7 @@ struct Params {
 
 // launchers (rtm_kernels.cu); all asynchronous on `st`
 void launch_split(const Params &p, bool samples, long long *outB, cudaStream_t st);
+void launch_regions(const Params &p, cudaStream_t st);
 void launch_fill_tile_regions(const Params &p, cudaStream_t st);
 void launch_partition(const Params &p, int n_sms, cudaStream_t st);
 void launch_events(const Params &p, cudaStream_t st);

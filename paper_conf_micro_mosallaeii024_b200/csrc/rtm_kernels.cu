@@ -5,6 +5,8 @@
 #include <stdint.h>
 #include <stdlib.h>
 
+#include <type_traits>
+
 #include "rtm_internal.h"
 
 namespace rtm {
@@ -41,6 +43,26 @@ __device__ __forceinline__ unsigned short ld_relaxed_u16(const unsigned short *p
   unsigned short v;
   asm volatile("ld.relaxed.gpu.global.u16 %0, [%1];" : "=h"(v) : "l"(p) : "memory");
   return v;
+}
+
+// Lanes holding the same BITS-bit key: one ballot per key bit.  On sm_100 __match_any_sync costs
+// ~59 cycles of SM throughput per warp instruction; this costs ~2.5 per bit (tools/microbench.cu).
+template <int BITS>
+__device__ __forceinline__ unsigned match_bits(unsigned key) {
+  unsigned m = kFull;
+#pragma unroll
+  for (int k = 0; k < BITS; ++k) {
+    // m &= bit_k(key) ? ballot : ~ballot   -- predicate, VOTE, two predicated LOP3s
+    asm("{\n .reg .pred p;\n .reg .b32 b;\n"
+        " setp.ne.u32 p, %1, 0;\n"
+        " vote.sync.ballot.b32 b, p, 0xffffffff;\n"
+        " @p  and.b32 %0, %0, b;\n"
+        " not.b32 b, b;\n"
+        " @!p and.b32 %0, %0, b;\n}"
+        : "+r"(m)
+        : "r"(key & (1u << k)));
+  }
+  return m;
 }
 
 // field validity (include/rtm.h)
@@ -154,6 +176,58 @@ __global__ void k_split(Params p, long long *outB) {
   if (lane == 0) outB[q] = (long long)ans;
 }
 
+// Region boundaries -> tile table on the device (no host round trip): B[0] = 0, B[W+2] = N, the
+// split positions made monotone (only an unsorted stream can break that; it is reported by the
+// order check), rt[r] = first tile of region r, rt[W+2] = number of tiles.  One CTA.
+__global__ void __launch_bounds__(1024) k_regions(long long *B, unsigned long long N, uint32_t W, uint32_t *rt,
+                                                   int tile) {
+  __shared__ long long wmax[32];
+  __shared__ unsigned wsum[32];
+  __shared__ long long carry_m;
+  __shared__ unsigned carry_s;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const unsigned nr = W + 3;
+  if (threadIdx.x == 0) { carry_m = 0; carry_s = 0; }
+  __syncthreads();
+  for (unsigned base = 0; base < nr; base += blockDim.x) {  // prefix max of the positions
+    const unsigned r = base + threadIdx.x;
+    long long x = 0;
+    if (r < nr) x = r == 0 ? 0 : (r == nr - 1 ? (long long)N : B[r]);
+    if (x > (long long)N) x = (long long)N;
+    for (int o = 1; o < 32; o <<= 1) {
+      const long long y = __shfl_up_sync(kFull, x, o);
+      if (lane >= o && y > x) x = y;
+    }
+    if (lane == 31) wmax[warp] = x;
+    __syncthreads();
+    long long pre = carry_m;
+    for (int w = 0; w < warp; ++w) pre = wmax[w] > pre ? wmax[w] : pre;
+    if (pre > x) x = pre;
+    __syncthreads();
+    if (r < nr) B[r] = x;
+    if (threadIdx.x == blockDim.x - 1) carry_m = x;
+    __syncthreads();
+  }
+  for (unsigned base = 0; base < nr; base += blockDim.x) {  // tiles per region, exclusive sum
+    const unsigned r = base + threadIdx.x;
+    unsigned cnt = 0;
+    if (r + 1 < nr) cnt = (unsigned)((B[r + 1] - B[r] + tile - 1) / tile);
+    unsigned x = cnt;
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned y = __shfl_up_sync(kFull, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) wsum[warp] = x;
+    __syncthreads();
+    unsigned pre = carry_s;
+    for (int w = 0; w < warp; ++w) pre += wsum[w];
+    __syncthreads();
+    if (r < nr) rt[r] = pre + x - cnt;
+    if (threadIdx.x == blockDim.x - 1) carry_s = pre + x;
+    __syncthreads();
+  }
+}
+
 __global__ void k_fill_tile_regions(const uint32_t *rt, uint32_t *tile_reg, uint32_t n_regions) {
   for (uint32_t r = blockIdx.x; r < n_regions; r += gridDim.x)
     for (uint32_t t = rt[r] + threadIdx.x; t < rt[r + 1]; t += blockDim.x) tile_reg[t] = r;
@@ -176,7 +250,7 @@ __global__ void k_fill_tile_regions(const uint32_t *rt, uint32_t *tile_reg, uint
 constexpr int kRecPerLane = kTileS / kK1Threads;  // 8
 constexpr int kK1Warps = kK1Threads / 32;         // 16
 constexpr unsigned kNoKey = 0xFFFFu;
-constexpr uint32_t kTmaMaxBins = 1024;
+constexpr uint32_t kTmaMaxBins = 256;
 
 #ifdef RTM_PHASE_TIMING
 #define PT_MARK(p_, slot_, t0_)                                                     \
@@ -221,34 +295,36 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned by
                : "memory");
 }
 
-template <bool NARROW, bool SMEM>
+// Per-warp scan of 8 steps x 32 records.  No cross-step dependency chain: each step ranks its
+// records within the step (match_any + popc) and its group leaders store the step's per-bin
+// counts (u8) into `stepc[j][bin]`; the order check compares each record with the previous
+// field-valid record of the same step, and the step-to-step part of the check is resolved
+// afterwards from per-step first/last offsets.  A per-bin prefix over the 8 steps then gives
+// each record's rank within (warp, bin) and the warp's bin totals (for the CTA-level prefix).
+template <bool NARROW, bool SMEM, int KB>
 __device__ __forceinline__ void partition_scan(const Params &p, const int4 *src, int n, long long lo,
                                                unsigned long long wlen, bool keep_ok, unsigned long long *ebuf,
-                                               unsigned *cnt, unsigned *kbuf, K1Warp &wr) {
+                                               unsigned *cnt, unsigned *kbuf, unsigned char *stepc, K1Warp &wr) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
   const unsigned nbins = p.nbins;
-  unsigned long long carry = 0, first = 0;
-  bool has = false, viol = false;
+  bool viol = false;
   unsigned kept = 0;
-  // registered capacities of all 8 records, fetched up front: the table (2 B/buffer) lives in
-  // L2 and its lookups must not sit on the per-record dependency chain
+  unsigned vmj[kRecPerLane];
+  unsigned long long firstj[kRecPerLane], lastj[kRecPerLane];
+  if (keep_ok) {  // zero this warp's step counts
+    unsigned *z = reinterpret_cast<unsigned *>(stepc);
+    for (unsigned q = lane; q < (unsigned)kRecPerLane * nbins / 4u; q += 32) z[q] = 0u;
+    __syncwarp();
+  }
   unsigned capj[kRecPerLane];
-  if (SMEM) {
+  if (SMEM) {  // registered capacities fetched up front (the table lives in L2)
 #pragma unroll
     for (int j = 0; j < kRecPerLane; ++j) {
       const int i = warp * 256 + j * 32 + lane;
       const unsigned b = i < n ? (unsigned)reinterpret_cast<const int *>(src + i)[2] : 0u;
       capj[j] = __ldg(p.cap + (b < p.nb ? b : 0u));
     }
-#ifdef RTM_PHASE_TIMING
-    unsigned sink = 0;
-#pragma unroll
-    for (int j = 0; j < kRecPerLane; ++j) sink += capj[j];
-    if (sink == 0xFFFFFFFFu) capj[0] ^= 1;  // force the cap loads to complete here
-    long long ptc = clock64();
-    PT_MARK(p, 7, ptc);
-#endif
   }
   constexpr int G = 4;
 #pragma unroll
@@ -262,9 +338,10 @@ __device__ __forceinline__ void partition_scan(const Params &p, const int4 *src,
     }
 #pragma unroll
     for (int jj = 0; jj < G; ++jj) {
-      const int i = warp * 256 + (h * G + jj) * 32 + lane;
+      const int j = h * G + jj;
+      const int i = warp * 256 + j * 32 + lane;
       const unsigned b = (unsigned)v[jj].z, lvl = (unsigned)v[jj].w & 0xFFFFu, c = (unsigned)v[jj].w >> 16;
-      const unsigned capb = SMEM ? capj[h * G + jj] : __ldg(p.cap + (b < p.nb ? b : 0u));
+      const unsigned capb = SMEM ? capj[j] : __ldg(p.cap + (b < p.nb ? b : 0u));
       const bool valid = (i < n) & (b < p.nb) & (c == capb) & (lvl <= c);
       const unsigned long long off = (unsigned long long)(rec_ts(v[jj]) - lo);
       const bool inr = off < wlen;
@@ -275,36 +352,52 @@ __device__ __forceinline__ void partition_scan(const Params &p, const int4 *src,
       if (NARROW) {
         const unsigned o = (unsigned)off;
         const unsigned pv = __shfl_sync(kFull, o, srcl);
-        bad = valid & ((!inr) | (o < (lower ? pv : (unsigned)carry)));
-        if (vm) carry = __shfl_sync(kFull, o, 31 - __clz(vm));
+        bad = valid & ((!inr) | ((lower != 0) & (o < pv)));
       } else {
         const unsigned long long pv = __shfl_sync(kFull, off, srcl);
-        bad = valid & ((!inr) | (off < (lower ? pv : carry)));
-        if (vm) carry = __shfl_sync(kFull, off, 31 - __clz(vm));
+        bad = valid & ((!inr) | ((lower != 0) & (off < pv)));
       }
       viol |= bad;
-      if (!has && vm) {
-        first = __shfl_sync(kFull, off, __ffs(vm) - 1);
-        has = true;
-      }
+      vmj[j] = vm;
+      firstj[j] = __shfl_sync(kFull, off, vm ? __ffs(vm) - 1 : 0);
+      lastj[j] = __shfl_sync(kFull, off, vm ? 31 - __clz(vm) : 0);
       const bool keep = valid & keep_ok;
       kept += keep;
       const unsigned key = keep ? (b >> kBinLog) : kNoKey;
-      unsigned pos = 0;
+      unsigned rank = 0;
       if (keep_ok) {
-        // onesweep-style stable rank: the group leader's shared atomicAdd returns the base
-        // stable rank: every peer reads the (warp, bin) counter, the group leader stores the new
-        // value (plain shared stores: shared atomics cost ~2 cycles per lane on this part)
-        const unsigned peers = __match_any_sync(kFull, key);
-        unsigned short *c16 = reinterpret_cast<unsigned short *>(cnt) + warp * nbins;
-        const unsigned basec = keep ? c16[key] : 0u;
-        __syncwarp();
-        if (keep && lane == __ffs(peers) - 1) c16[key] = (unsigned short)(basec + __popc(peers));
-        __syncwarp();
-        pos = basec + __popc(peers & lt);
+        const unsigned peers = __match_any_sync(kFull, key);  // measured faster than match_bits here
+        rank = __popc(peers & lt);
+        if (keep && rank == 0) stepc[j * nbins + key] = (unsigned char)__popc(peers);
         if (keep) ebuf[i] = (off << 24) | ((unsigned long long)lvl << 8) | (b & (kBin - 1));
       }
-      kbuf[i] = (key << 16) | pos;
+      kbuf[i] = (key << 16) | rank;
+    }
+  }
+  // step-to-step order: each step's first field-valid offset >= the previous steps' last one
+  bool has = false;
+  unsigned long long carry = 0, first = 0;
+#pragma unroll
+  for (int j = 0; j < kRecPerLane; ++j) {
+    if (vmj[j]) {
+      if (has && firstj[j] < carry) viol = true;
+      if (!has) first = firstj[j];
+      has = true;
+      carry = lastj[j];
+    }
+  }
+  if (keep_ok) {  // per-bin exclusive prefix over the steps; warp totals -> the CTA counters
+    __syncwarp();
+    unsigned short *c16 = reinterpret_cast<unsigned short *>(cnt) + warp * nbins;
+    for (unsigned k = lane; k < nbins; k += 32) {
+      unsigned run = 0;
+#pragma unroll
+      for (int j = 0; j < kRecPerLane; ++j) {
+        const unsigned x = stepc[j * nbins + k];
+        stepc[j * nbins + k] = (unsigned char)run;
+        run += x;
+      }
+      c16[k] = (unsigned short)run;
     }
   }
   kept = warp_sum(kept);
@@ -313,6 +406,25 @@ __device__ __forceinline__ void partition_scan(const Params &p, const int4 *src,
   wr.has = has;
   wr.viol = __any_sync(kFull, viol);
   wr.kept = kept;
+}
+
+// key width: bins are 0..nbins-1 and the all-ones key marks "not kept", so nbins < 2^KB - 1 + 1
+template <bool SMEM>
+__device__ __forceinline__ void partition_scan_dispatch(const Params &p, const int4 *src, int n, long long lo,
+                                                        unsigned long long wlen, bool keep_ok, bool narrow,
+                                                        unsigned long long *ebuf, unsigned *cnt, unsigned *kbuf,
+                                                        unsigned char *stepc, K1Warp &wr) {
+  const unsigned need = 32 - __clz(p.nbins);  // smallest KB with nbins <= 2^KB - 1
+#define RTM_SCAN_CASE(KB_)                                                                                   \
+  case KB_:                                                                                                  \
+    if (narrow) partition_scan<true, SMEM, KB_>(p, src, n, lo, wlen, keep_ok, ebuf, cnt, kbuf, stepc, wr);   \
+    else partition_scan<false, SMEM, KB_>(p, src, n, lo, wlen, keep_ok, ebuf, cnt, kbuf, stepc, wr);         \
+    break;
+  switch (need < 2 ? 2u : need) {
+    RTM_SCAN_CASE(2) RTM_SCAN_CASE(3) RTM_SCAN_CASE(4) RTM_SCAN_CASE(5) RTM_SCAN_CASE(6) RTM_SCAN_CASE(7)
+    RTM_SCAN_CASE(8) RTM_SCAN_CASE(9) RTM_SCAN_CASE(10) default : RTM_SCAN_CASE(11)
+  }
+#undef RTM_SCAN_CASE
 }
 
 struct K1Smem {            // static shared part of both partition kernels
@@ -346,7 +458,8 @@ __device__ __forceinline__ TileInfo tile_info(const Params &p, unsigned tile) {
 // Ends with __syncthreads() (the caller may reuse all shared buffers afterwards).
 __device__ __forceinline__ void partition_finish(const Params &p, unsigned tile, const TileInfo &t, K1Smem &K,
                                                  const K1Warp &wr, const unsigned long long *ebuf, unsigned *binoff,
-                                                 unsigned *cnt, const unsigned *kbuf, unsigned long long *sbuf) {
+                                                 unsigned *cnt, const unsigned *kbuf, const unsigned char *stepc,
+                                                 unsigned long long *sbuf) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned nbins = p.nbins;
   const bool is_win = t.g.window >= 0;
@@ -431,7 +544,9 @@ __device__ __forceinline__ void partition_finish(const Params &p, unsigned tile,
   for (int j = 0; j < kRecPerLane; ++j) {
     const int i = warp * 256 + j * 32 + lane;
     const unsigned kv = kbuf[i], key = kv >> 16;
-    if (key != kNoKey && i < t.n) out[binoff[key] + cnt16[warp * nbins + key] + (kv & 0xFFFFu)] = ebuf[i];
+    if (key != kNoKey && i < t.n)
+      out[binoff[key] + cnt16[warp * nbins + key] + stepc[(size_t)warp * kRecPerLane * nbins + j * nbins + key] +
+          (kv & 0xFFFFu)] = ebuf[i];
   }
   __syncthreads();
   if (sbuf) {  // coalesced 16-byte copy-out of the bin-sorted tile
@@ -448,32 +563,40 @@ __device__ __forceinline__ void zero_counters(const Params &p, unsigned *cnt) {
   for (unsigned i = threadIdx.x; i < kK1Warps * p.nbins / 2 + 1; i += blockDim.x) cnt[i] = 0;
 }
 
-__global__ void __launch_bounds__(kK1Threads, 2) k_partition(Params p, int narrow) {
+__global__ void __launch_bounds__(kK1Threads, 2) k_partition(Params p, int narrow, unsigned tile0) {
+  if (tile0 + blockIdx.x >= p.rts[p.W + 2]) return;  // grid sized by an upper bound
   extern __shared__ __align__(16) unsigned char smem[];
   unsigned long long *ebuf = reinterpret_cast<unsigned long long *>(smem);  // [4096]
   unsigned *kbuf = reinterpret_cast<unsigned *>(ebuf + kTileS);             // [4096] key<<16|pos
   unsigned *binoff = kbuf + kTileS;                                         // [nbins+1]
   unsigned *cnt = binoff + p.nbins + 1;                                     // u16 [16][nbins]
+  unsigned char *stepc = reinterpret_cast<unsigned char *>(cnt + kK1Warps * p.nbins / 2 + 1);  // u8 [16][8][nbins]
   __shared__ K1Smem K;
-  const unsigned tile = blockIdx.x;
+  const unsigned tile = tile0 + blockIdx.x;
   const TileInfo t = tile_info(p, tile);
   const bool is_win = t.g.window >= 0;
   if (is_win) zero_counters(p, cnt);
   __syncthreads();
   const int4 *src = reinterpret_cast<const int4 *>(p.s) + t.start;
   K1Warp wr;
-  if (is_win && narrow) partition_scan<true, false>(p, src, t.n, t.lo, t.wlen, true, ebuf, cnt, kbuf, wr);
-  else partition_scan<false, false>(p, src, t.n, t.lo, t.wlen, is_win, ebuf, cnt, kbuf, wr);
-  partition_finish(p, tile, t, K, wr, ebuf, binoff, cnt, kbuf, nullptr);
+  unsigned char *wstep = stepc + (size_t)(threadIdx.x >> 5) * kRecPerLane * p.nbins;
+#ifdef RTM_PHASE_TIMING
+  long long pt0 = clock64();
+  if (threadIdx.x == 0 && p.dbg) atomicAdd(p.dbg + 3, 1ull);
+#endif
+  partition_scan_dispatch<false>(p, src, t.n, t.lo, t.wlen, is_win, is_win && narrow, ebuf, cnt, kbuf, wstep, wr);
+  PT_MARK(p, 1, pt0);
+  partition_finish(p, tile, t, K, wr, ebuf, binoff, cnt, kbuf, stepc, nullptr);
 }
 
 __global__ void __launch_bounds__(kK1Threads, 1) k_partition_tma(Params p, int narrow) {
-  extern __shared__ __align__(128) unsigned char smem[];
+  extern __shared__ __align__(16) unsigned char smem[];
   int4 *raw = reinterpret_cast<int4 *>(smem);                                 // [2][4096] records
   unsigned long long *ebuf = reinterpret_cast<unsigned long long *>(raw + 2 * kTileS);  // [4096]
   unsigned *kbuf = reinterpret_cast<unsigned *>(ebuf + kTileS);                  // [4096]
   unsigned *binoff = kbuf + kTileS;                                              // [nbins+1]
   unsigned *cnt = binoff + p.nbins + 1;                                          // u16 [16][nbins]
+  unsigned char *stepc = reinterpret_cast<unsigned char *>(cnt + kK1Warps * p.nbins / 2 + 1);  // u8 [16][8][nbins]
   __shared__ K1Smem K;
   __shared__ __align__(8) unsigned long long bar[2];
   if (threadIdx.x == 0) {
@@ -489,12 +612,13 @@ __global__ void __launch_bounds__(kK1Threads, 1) k_partition_tma(Params p, int n
     mbar_expect_tx(&bar[buf], bytes);
     bulk_g2s(raw + buf * kTileS, reinterpret_cast<const int4 *>(p.s) + t.start, bytes, &bar[buf]);
   };
+  const unsigned n_tiles = p.rts[p.W + 2];  // device count (the grid is sized by an upper bound)
   unsigned tile = blockIdx.x;
-  if (threadIdx.x == 0 && tile < p.n_tiles_s) issue(tile, 0);
-  for (unsigned it = 0; tile < p.n_tiles_s; ++it, tile += gridDim.x) {
+  if (threadIdx.x == 0 && tile < n_tiles) issue(tile, 0);
+  for (unsigned it = 0; tile < n_tiles; ++it, tile += gridDim.x) {
     const int buf = it & 1;
     const unsigned next = tile + gridDim.x;
-    if (threadIdx.x == 0 && next < p.n_tiles_s) issue(next, buf ^ 1);  // buffer freed at end of it-1
+    if (threadIdx.x == 0 && next < n_tiles) issue(next, buf ^ 1);  // buffer freed at end of it-1
     const TileInfo t = tile_info(p, tile);
     const bool is_win = t.g.window >= 0;
     if (is_win) zero_counters(p, cnt);
@@ -508,14 +632,14 @@ __global__ void __launch_bounds__(kK1Threads, 1) k_partition_tma(Params p, int n
 #endif
     const int4 *src = raw + buf * kTileS;
     K1Warp wr;
-    if (is_win && narrow) partition_scan<true, true>(p, src, t.n, t.lo, t.wlen, true, ebuf, cnt, kbuf, wr);
-    else partition_scan<false, true>(p, src, t.n, t.lo, t.wlen, is_win, ebuf, cnt, kbuf, wr);
+    unsigned char *wstep = stepc + (size_t)(threadIdx.x >> 5) * kRecPerLane * p.nbins;
+    partition_scan_dispatch<true>(p, src, t.n, t.lo, t.wlen, is_win, is_win && narrow, ebuf, cnt, kbuf, wstep, wr);
 #ifdef RTM_PHASE_TIMING
     __syncthreads();
     long long c2 = clock64();
 #endif
     // the tile's raw records are consumed: its TMA slot holds the permuted entries
-    partition_finish(p, tile, t, K, wr, ebuf, binoff, cnt, kbuf,
+    partition_finish(p, tile, t, K, wr, ebuf, binoff, cnt, kbuf, stepc,
                      reinterpret_cast<unsigned long long *>(raw + buf * kTileS));
 #ifdef RTM_PHASE_TIMING
     long long c3 = clock64();
@@ -535,6 +659,7 @@ __global__ void __launch_bounds__(kK1Threads, 1) k_partition_tma(Params p, int n
 // per-component START/END deltas (progress bars, L131; "task counts stop changing", L227).
 // ============================================================================================
 __global__ void __launch_bounds__(kK3Threads) k_events(Params p) {
+  if (blockIdx.x >= p.rte[p.W + 2]) return;  // grid sized by an upper bound
   extern __shared__ __align__(16) unsigned char smem[];
   unsigned *khist = reinterpret_cast<unsigned *>(smem);  // [nk*2]
   unsigned *abits = khist + 2 * p.nk;                     // [ncw] if smem_bits
@@ -655,6 +780,8 @@ struct FoldSmem {
   unsigned long long ts0[kBin];    // offset of the first kept sample in the window
   unsigned long long cml[kBin];    // cur | max << 16 | min << 32   (levels seen this window)
   unsigned n[kBin];                // kept samples this window (0: untouched, other fields stale)
+  unsigned seg_end[32];            // flattened segment table of the current tile group
+  unsigned long long seg_ptr[32];
 };
 
 // One chunk of <= 32 consecutive records (ingest order) of one (window, bin) unit.  Records of
@@ -665,10 +792,12 @@ struct FoldSmem {
 // state update in a chunk touches a distinct buffer.
 __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, bool act, unsigned long long e,
                                            unsigned long long Wlen) {
-  const unsigned lid = act ? (unsigned)(e & (kBin - 1)) : (unsigned)(kBin + lane);
+  const unsigned lid = (unsigned)(e & (kBin - 1));
   const unsigned lvl = (unsigned)(e >> 8) & 0xFFFFu;
   const unsigned long long off = e >> 24;
-  const unsigned peers = __match_any_sync(kFull, lid);
+  const unsigned am = __ballot_sync(kFull, act);
+  const unsigned mb = match_bits<kBinLog>(lid);  // all lanes (ballots are collective)
+  const unsigned peers = act ? (mb & am) : (1u << lane);
   const unsigned lower = peers & lt;
   const int pred = lower ? 31 - __clz(lower) : lane;
   const unsigned rank = __popc(lower);
@@ -746,25 +875,26 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
         if (lane >= o) pre += y;
       }
       const unsigned total = __shfl_sync(kFull, pre, 31);
-      unsigned sgi = 0;  // this lane's current segment (cursor)
+      // per-warp segment table: end (inclusive prefix) and the staging address of each segment
+      S.seg_end[lane] = pre;
+      S.seg_ptr[lane] = (unsigned long long)(p.stage + (size_t)(tg + lane) * kTileS + seg_lo) -
+                        (unsigned long long)(pre - seg_len) * 8ull;
+      __syncwarp();
+      unsigned sgi = 0;  // this lane's current segment (cursor), advanced without warp collectives
       auto fetch = [&](unsigned g) -> unsigned long long {
-        // advance the cursor to the segment holding flattened index g (< 32 segments)
-        for (;;) {
-          const unsigned end = __shfl_sync(kFull, pre, sgi & 31);
-          const bool adv = g < total && g >= end;
-          if (!__any_sync(kFull, adv)) break;
-          if (adv) ++sgi;
-        }
-        const unsigned base = __shfl_sync(kFull, pre - seg_len, sgi & 31);
-        const unsigned lo = __shfl_sync(kFull, seg_lo, sgi & 31);
         if (g >= total) return 0ull;
-        return __ldcg(p.stage + (size_t)(tg + sgi) * kTileS + lo + (g - base));
+        while (g >= S.seg_end[sgi]) ++sgi;
+        return __ldcg(reinterpret_cast<const unsigned long long *>(S.seg_ptr[sgi]) + g);
       };
-      unsigned long long e = fetch(lane);
+      // 4-deep software pipeline: staging reads are DRAM/L2 round trips
+      unsigned long long e0 = fetch(lane), e1 = fetch(32 + lane), e2 = fetch(64 + lane), e3 = fetch(96 + lane);
       for (unsigned c = 0; c < total; c += 32) {
-        const unsigned long long en = fetch(c + 32 + lane);  // prefetch the next chunk
-        fold_chunk(S, lane, lt, c + lane < total, e, Wlen);
-        e = en;
+        const unsigned long long en = fetch(c + 128 + lane);
+        fold_chunk(S, lane, lt, c + lane < total, e0, Wlen);
+        e0 = e1;
+        e1 = e2;
+        e2 = e3;
+        e3 = en;
       }
     }
     // ---- publish this window's last levels (kSent: untouched) and the phase-1 flag
@@ -891,8 +1021,9 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
 // K4: cross-tile order check (single CTA).  Tile t violates the contract if its own flag is set
 // or its first field-valid ts is below the max ts of all earlier tiles.
 // ============================================================================================
-__global__ void __launch_bounds__(1024) k_order_check(const TileMeta *meta, unsigned n, unsigned *status,
-                                                       unsigned bit) {
+__global__ void __launch_bounds__(1024) k_order_check(const TileMeta *meta, unsigned n_max, const uint32_t *n_dev,
+                                                       unsigned *status, unsigned bit) {
+  const unsigned n = *n_dev < n_max ? *n_dev : n_max;
   __shared__ long long wmax[32];
   __shared__ long long carry_s;
   __shared__ unsigned bad_s;
@@ -1303,11 +1434,17 @@ __global__ void k_merge_tables(Params p, const unsigned char *g, unsigned world,
 // ============================================================================================
 size_t fold_smem_bytes() { return sizeof(FoldSmem) * kFoldWarps; }
 size_t partition_smem_bytes(uint32_t nbins) {
-  return (size_t)kTileS * 8 + (size_t)kTileS * 4 + (size_t)(nbins + 1) * 4 + ((size_t)kK1Warps * nbins / 2 + 1) * 4 + 16;
+  return (size_t)kTileS * 8 + (size_t)kTileS * 4 + (size_t)(nbins + 1) * 4 + ((size_t)kK1Warps * nbins / 2 + 1) * 4 +
+         (size_t)kK1Warps * kRecPerLane * ((nbins + 3) & ~3u) + 16;
 }
+static_assert((size_t)kTileS * 12 + (size_t)(kMaxBins + 1) * 4 + ((size_t)kK1Warps * kMaxBins / 2 + 1) * 4 +
+                      (size_t)kK1Warps * kRecPerLane * kMaxBins + 16 <= 227 * 1024,
+              "partition shared memory exceeds the 227 KB opt-in limit");
 size_t partition_tma_smem_bytes(uint32_t nbins) { return (size_t)2 * kTileS * 16 + partition_smem_bytes(nbins); }
+static_assert(227 * 1024 >= 0, "");
 static_assert((size_t)2 * kTileS * 16 + (size_t)kTileS * 12 + (size_t)(kTmaMaxBins + 1) * 4 +
-                      ((size_t)kK1Warps * kTmaMaxBins / 2 + 1) * 4 + 16 <= 227 * 1024,
+                      ((size_t)kK1Warps * kTmaMaxBins / 2 + 1) * 4 + (size_t)kK1Warps * kRecPerLane * kTmaMaxBins +
+                      16 <= 227 * 1024,
               "TMA partition shared memory exceeds the 227 KB opt-in limit");
 size_t topk_smem_bytes(uint32_t nb) {
   return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8;
@@ -1321,6 +1458,11 @@ void launch_split(const Params &p, bool samples, long long *outB, cudaStream_t s
   else k_split<false><<<blocks, threads, 0, st>>>(p, outB);
 }
 
+void launch_regions(const Params &p, cudaStream_t st) {
+  k_regions<<<1, 1024, 0, st>>>(const_cast<long long *>(p.Bs), p.ns, p.W, const_cast<uint32_t *>(p.rts), kTileS);
+  k_regions<<<1, 1024, 0, st>>>(const_cast<long long *>(p.Be), p.ne, p.W, const_cast<uint32_t *>(p.rte), kTileE);
+}
+
 void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
   const unsigned nr = p.W + 2;
   const unsigned blocks = nr < 4096 ? nr : 4096;
@@ -1330,12 +1472,12 @@ void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
 
 void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   if (!p.n_tiles_s) return;
-  static const bool use_tma = getenv("RTM_TMA") != nullptr;  // measured slower on C2
+  static const bool use_tma = getenv("RTM_TMA") != nullptr;     // measured slower on C2
   if (p.nbins <= kTmaMaxBins && use_tma) {
     const unsigned grid = p.n_tiles_s < (unsigned)n_sms ? p.n_tiles_s : (unsigned)n_sms;
     k_partition_tma<<<grid, kK1Threads, partition_tma_smem_bytes(p.nbins), st>>>(p, p.narrow);
   } else {
-    k_partition<<<p.n_tiles_s, kK1Threads, partition_smem_bytes(p.nbins), st>>>(p, p.narrow);
+    k_partition<<<p.n_tiles_s, kK1Threads, partition_smem_bytes(p.nbins), st>>>(p, p.narrow, 0u);
   }
 }
 
@@ -1359,8 +1501,8 @@ void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
 }
 
 void launch_order_check(const Params &p, cudaStream_t st) {
-  if (p.n_tiles_s) k_order_check<<<1, 1024, 0, st>>>(p.smeta, p.n_tiles_s, p.status, 1u);
-  if (p.n_tiles_e) k_order_check<<<1, 1024, 0, st>>>(p.emeta, p.n_tiles_e, p.status, 2u);
+  if (p.n_tiles_s) k_order_check<<<1, 1024, 0, st>>>(p.smeta, p.n_tiles_s, p.rts + p.W + 2, p.status, 1u);
+  if (p.n_tiles_e) k_order_check<<<1, 1024, 0, st>>>(p.emeta, p.n_tiles_e, p.rte + p.W + 2, p.status, 2u);
 }
 
 void launch_topk(const Params &p, cudaStream_t st) {
