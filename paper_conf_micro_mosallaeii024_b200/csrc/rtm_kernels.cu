@@ -420,9 +420,8 @@ __device__ __forceinline__ void partition_scan_dispatch(const Params &p, const i
     if (narrow) partition_scan<true, SMEM, KB_>(p, src, n, lo, wlen, keep_ok, ebuf, cnt, kbuf, stepc, wr);   \
     else partition_scan<false, SMEM, KB_>(p, src, n, lo, wlen, keep_ok, ebuf, cnt, kbuf, stepc, wr);         \
     break;
-  switch (need < 2 ? 2u : need) {
-    RTM_SCAN_CASE(2) RTM_SCAN_CASE(3) RTM_SCAN_CASE(4) RTM_SCAN_CASE(5) RTM_SCAN_CASE(6) RTM_SCAN_CASE(7)
-    RTM_SCAN_CASE(8) RTM_SCAN_CASE(9) RTM_SCAN_CASE(10) default : RTM_SCAN_CASE(11)
+  switch (need <= 7 ? 7u : 11u) {  // two instantiations keep the hot code small
+    RTM_SCAN_CASE(7) default : RTM_SCAN_CASE(11)
   }
 #undef RTM_SCAN_CASE
 }
@@ -1074,6 +1073,7 @@ __global__ void __launch_bounds__(1024) k_order_check(const TileMeta *meta, unsi
 // (tie-break), and the k winners are bitonic-sorted by (key desc, id asc).
 // ============================================================================================
 constexpr int kTopkThreads = 512;
+constexpr unsigned kTopkCand = 4096;  // candidate list capacity after the first radix digit
 
 // key32 = floor(l * 2^32 / c) for l < c, exact: m = floor(2^48 / c) (rcp table), q0 = (l*m) >> 16
 // is floor or floor-1 (error < l / 2^16 < 1), one remainder test fixes it.
@@ -1094,8 +1094,9 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
   unsigned *keys = reinterpret_cast<unsigned *>(smem);                                  // [ne] or none
   unsigned *hist = keys + (keys_in_smem ? ((ne + 1) & ~1u) : 0);                        // [8][256]
   unsigned long long *sel = reinterpret_cast<unsigned long long *>(hist + 8 * 256);     // [1024]
+  unsigned *cand = reinterpret_cast<unsigned *>(sel + 1024);                             // [kTopkCand]
   __shared__ unsigned scan_scratch[32];
-  __shared__ unsigned s_digit, s_need, s_ngt;
+  __shared__ unsigned s_digit, s_need, s_ngt, s_ncand;
   const unsigned w = blockIdx.x;
   const uint16_t *lv = p.lastlvl + (size_t)w * p.nb;
   const int warp = threadIdx.x >> 5;
@@ -1115,13 +1116,18 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     if (threadIdx.x == 0) p.topk_n[w] = 0;
     return;
   }
+  // MSB radix select.  After the first digit only candidates (top byte >= the selected digit,
+  // at most k + the selected bucket) can matter: they are compacted in id order when they fit,
+  // so the remaining passes and the selection scan ~1k keys instead of every buffer.
   unsigned prefix = 0, mask = 0, need = keff;
+  unsigned n_it = ne;  // iteration space: all keys, or the candidate list
+  bool use_c = false;
   for (int d = 3; d >= 0; --d) {
     for (unsigned i = threadIdx.x; i < 8 * 256; i += blockDim.x) hist[i] = 0;
     __syncthreads();
     unsigned *myh = hist + (warp & 7) * 256;
-    for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) {
-      const unsigned k = key_at(i);
+    for (unsigned j = threadIdx.x; j < n_it; j += blockDim.x) {
+      const unsigned k = key_at(use_c ? cand[j] : j);
       if ((k & mask) == prefix) atomicAdd(&myh[(k >> (8 * d)) & 255u], 1u);
     }
     __syncthreads();
@@ -1140,9 +1146,21 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
       }
       s_digit = (unsigned)x;
       s_need = need - cum;
+      s_ncand = cum + hist[x];
     }
     __syncthreads();
-    prefix |= s_digit << (8 * d);
+    const unsigned digit = s_digit;
+    if (d == 3 && s_ncand <= kTopkCand) {  // compact candidates (stable, id order)
+      const unsigned chunk = (ne + blockDim.x - 1) / blockDim.x, c0 = threadIdx.x * chunk;
+      unsigned cnt = 0;
+      for (unsigned i = c0; i < c0 + chunk && i < ne; ++i) cnt += (key_at(i) >> 24) >= digit;
+      unsigned pos = block_excl_scan(cnt, scan_scratch, nullptr);
+      for (unsigned i = c0; i < c0 + chunk && i < ne; ++i)
+        if ((key_at(i) >> 24) >= digit) cand[pos++] = i;
+      n_it = s_ncand;
+      use_c = true;
+    }
+    prefix |= digit << (8 * d);
     mask |= 255u << (8 * d);
     need = s_need;
     __syncthreads();
@@ -1150,11 +1168,12 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
   const unsigned tau = prefix;  // k-th key; `need` keys equal to tau are taken (lowest ids)
   if (threadIdx.x == 0) s_ngt = 0;
   __syncthreads();
-  // one pass over contiguous index chunks: keys > tau (any order) and the first `need` keys == tau
-  const unsigned chunk = (ne + blockDim.x - 1) / blockDim.x;
+  // one pass over contiguous chunks (id order): keys > tau (any order) and the first `need` == tau
+  const unsigned chunk = (n_it + blockDim.x - 1) / blockDim.x;
   const unsigned c0 = threadIdx.x * chunk;
   unsigned ceq = 0;
-  for (unsigned i = c0; i < c0 + chunk && i < ne; ++i) {
+  for (unsigned j = c0; j < c0 + chunk && j < n_it; ++j) {
+    const unsigned i = use_c ? cand[j] : j;
     const unsigned k = key_at(i);
     if (k > tau) {
       const unsigned slot = atomicAdd(&s_ngt, 1u);
@@ -1164,7 +1183,8 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
   }
   unsigned rank = block_excl_scan(ceq, scan_scratch, nullptr);  // syncs: s_ngt final after it
   const unsigned ngt = s_ngt;
-  for (unsigned i = c0; i < c0 + chunk && i < ne && rank < need; ++i) {
+  for (unsigned j = c0; j < c0 + chunk && j < n_it && rank < need; ++j) {
+    const unsigned i = use_c ? cand[j] : j;
     const unsigned k = key_at(i);
     if (k == tau) {
       sel[ngt + rank] = ((unsigned long long)k << 32) | (0xFFFFFFFFu - id_of(i));
@@ -1447,7 +1467,7 @@ static_assert((size_t)2 * kTileS * 16 + (size_t)kTileS * 12 + (size_t)(kTmaMaxBi
                       16 <= 227 * 1024,
               "TMA partition shared memory exceeds the 227 KB opt-in limit");
 size_t topk_smem_bytes(uint32_t nb) {
-  return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8;
+  return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8 + kTopkCand * 4;
 }
 
 void launch_split(const Params &p, bool samples, long long *outB, cudaStream_t st) {
