@@ -321,7 +321,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   const size_t Wn = W;
   if ((s = ensure(c, c->treg_s, (size_t)nts * 4))) return s;
   if ((s = ensure(c, c->treg_e, (size_t)nte * 4))) return s;
-  if ((s = ensure(c, c->soff, (size_t)nts * (c->nbins + 1) * 4))) return s;
+  if ((s = ensure(c, c->soff, (size_t)nts * (c->nbins + 1) * 2))) return s;
   if ((s = ensure(c, c->stage, (size_t)nts * kTileS * 8))) return s;
   if ((s = ensure(c, c->smeta, (size_t)nts * sizeof(TileMeta)))) return s;
   if ((s = ensure(c, c->emeta, (size_t)nte * sizeof(TileMeta)))) return s;
@@ -353,7 +353,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
 
   p.tile_reg_s = (const uint32_t *)c->treg_s.p; p.tile_reg_e = (const uint32_t *)c->treg_e.p;
   p.n_tiles_s = nts; p.n_tiles_e = nte;
-  p.soff = (uint32_t *)c->soff.p; p.stage = (unsigned long long *)c->stage.p;
+  p.soff = (uint16_t *)c->soff.p; p.stage = (unsigned long long *)c->stage.p;
   p.smeta = (TileMeta *)c->smeta.p; p.emeta = (TileMeta *)c->emeta.p;
   p.lastlvl = (uint16_t *)c->lastlvl.p; p.flags = (uint32_t *)c->flags.p;
   p.win = (unsigned long long *)c->win.p; p.kdelta = (uint32_t *)c->kdelta.p;

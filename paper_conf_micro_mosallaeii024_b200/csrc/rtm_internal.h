@@ -28,11 +28,11 @@ constexpr int kBinLog = 8;                  // 256 buffers per bin
 constexpr int kBin = 1 << kBinLog;
 constexpr int kTileS = 4096;                // samples per partition tile
 constexpr int kTileE = 4096;                // events per event tile
-constexpr int kK1Threads = 512;             // 16 warps x 8 records per lane
+constexpr int kK1Threads = 256;             // 8 warps x 512-sample sub-tiles
 constexpr int kK3Threads = 256;
 constexpr int kFoldWarps = 4;               // warps per fold CTA
 constexpr uint16_t kSent = 0xFFFFu;         // "no kept sample in this window" marker
-constexpr uint32_t kMaxBins = 1024;         // n_buffers <= 262144 (partition smem <= 227 KB)
+constexpr uint32_t kMaxBins = 4096;         // n_buffers <= 2^20 (fallback partition smem 160 KB)
 constexpr uint32_t kTopkSmemKeys = 40960;   // keys held in shared memory by the top-k kernel
 constexpr int64_t kMaxWindowLen = (int64_t)1 << 40;  // ts offset field of a staging entry
 
@@ -83,7 +83,7 @@ struct Params {
   const uint32_t *tile_reg_e;
   uint32_t n_tiles_s, n_tiles_e;  // upper bounds (grid sizes); device counts are rts/rte[W+2]
   // outputs / workspaces
-  uint32_t *soff;            // [n_tiles_s * (nbins+1)]
+  uint16_t *soff;            // [n_tiles_s * (nbins+1)] tile-local bin offsets
   unsigned long long *stage; // [n_tiles_s * kTileS]
   TileMeta *smeta, *emeta;
   uint16_t *lastlvl;         // [W * nb]
@@ -127,7 +127,7 @@ void launch_pack(const Params &p, void *pack, cudaStream_t st);
 void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStream_t st);
 void configure_kernels_once();  // opt-in shared-memory limits, once per device
 size_t fold_smem_bytes();
-size_t partition_smem_bytes(uint32_t nbins);
+size_t partition_smem_bytes(uint32_t nbins, uint32_t nb);
 size_t topk_smem_bytes(uint32_t nb);
 
 }  // namespace rtm

@@ -234,214 +234,63 @@ __global__ void k_fill_tile_regions(const uint32_t *rt, uint32_t *tile_reg, uint
 }
 
 // ============================================================================================
-// K1: sample partition.  A tile is <= 4096 samples of ONE region, processed by 16 warps; warp w
-// owns tile positions [256w, 256w+256), lane l handles 256w + 32j + l (j = 0..7).  Per sample:
-// field validity, range + order check against the previous field-valid sample (warp order;
-// 32-bit offsets when windows are < 2^32 ticks), and a stable multisplit by bin
-// (buffer_id >> 8): __match_any_sync + the group leader's shared atomicAdd on per-(warp, bin)
-// u16 counters give the stable rank (onesweep-style), a block scan gives bin offsets.  Kept
-// samples become 8-byte entries  (ts - t_begin) << 24 | level << 8 | (buffer_id & 255),
-// staged in shared memory (tile order) and scattered to the tile's staging slot.
+// K1: sample partition.  A tile is <= 4096 samples of ONE region, handled by one CTA of 8 warps;
+// warp w owns the sub-tile [512w, 512w + 512).  Per sample: field validity, range + order check
+// against the previous field-valid sample, and a stable multisplit by bin (buffer_id >> 8).  Kept
+// samples become 8-byte entries  (ts - t_begin) << 24 | level << 8 | (buffer_id & 255).
 //
-// k_partition_tma (n_bins <= 1024): persistent, one CTA per SM; tiles stream into a double
-// buffer with cp.async.bulk (TMA) + mbarrier, so the next tile's HBM read is in flight while the
-// current one is ranked.  k_partition: one CTA per tile, register loads (any n_bins).
+// k_partition_lm (lane-major, n_bins <= 128; persistent, 1-2 CTAs per SM): the buffer-capacity
+// table lives in shared memory (the field check is a gather per sample: from L1 it was the
+// kernel's bottleneck).  Each warp stages its 512 raw records in shared memory (XOR-swizzled
+// 16-byte slots) and lane l takes the CONSECUTIVE records 16l .. 16l+15, so the stable order
+// inside a bin is (lane, slot).  Rank = equal keys among the lane's earlier samples (register
+// compares, no warp collectives); per-(bin, lane) counts go to a u16 matrix that reuses the
+// warp's raw slot, one row (= bin) per lane is prefix-scanned.
+// k_partition_mx (fallback, any n_bins): lanes take strided records; __match_any_sync peers +
+// the warp's bin counters give the rank.
+//
+// Both: one barrier publishes every warp's bin totals; each warp derives its bin bases (CTA bin
+// offsets + earlier warps' counts) and permutes its entries into a CTA buffer that reuses the raw
+// staging; a second barrier precedes the coalesced copy-out.  soff gets the tile's u16 bin offsets.
 // ============================================================================================
-constexpr int kRecPerLane = kTileS / kK1Threads;  // 8
-constexpr int kK1Warps = kK1Threads / 32;         // 16
+constexpr int kSub = kTileS / (kK1Threads / 32);  // 512 samples per warp
+constexpr int kPerLane = kSub / 32;               // 16
+constexpr int kK1Warps = kK1Threads / 32;         // 8
 constexpr unsigned kNoKey = 0xFFFFu;
-constexpr uint32_t kTmaMaxBins = 256;
+constexpr uint32_t kLmMaxBins = 128;              // the count matrix (nbins x 64 B) fits the warp's raw slot
+static_assert(kPerLane == 16, "lane-major swizzle assumes 16 records per lane");
+static_assert((size_t)kLmMaxBins * 64 <= (size_t)kSub * 16, "count matrix must fit the raw slot");
 
-#ifdef RTM_PHASE_TIMING
-#define PT_MARK(p_, slot_, t0_)                                                     \
-  do {                                                                              \
-    __syncthreads();                                                                \
-    if (threadIdx.x == 0 && (p_).dbg) {                                             \
-      const long long t1_ = clock64();                                              \
-      atomicAdd((p_).dbg + (slot_), (unsigned long long)(t1_ - (t0_)));            \
-      (t0_) = t1_;                                                                  \
-    }                                                                               \
-  } while (0)
-#else
-#define PT_MARK(p_, slot_, t0_) \
-  do {                          \
-  } while (0)
-#endif
-
-struct K1Warp {
-  unsigned long long first, last;  // offsets (from lo) of the first / last field-valid record
-  unsigned has, viol, kept;
+struct K1WarpSum {
+  unsigned long long first, last;  // offsets of the first / last field-valid record
+  unsigned has, viol, kept, pad;
 };
 
-__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(unsigned long long *bar, unsigned count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+__host__ __device__ constexpr size_t k1_align16(size_t x) { return (x + 15) & ~(size_t)15; }
+__host__ __device__ constexpr size_t k1_vec_bytes(uint32_t nbins) { return k1_align16((size_t)kK1Warps * nbins * 2); }
+// dynamic shared memory.  lm: raw 16 B x 4096 | wt | wb | cap[nb];  mx: sbuf 8 B x 4096 | wt | wb
+// (wt: 8 x nbins u16 bin totals / live counters, wb: 8 x nbins u16 bin bases)
+__host__ __device__ constexpr size_t k1_smem_lm(uint32_t nbins, uint32_t nb) {
+  return (size_t)kTileS * 16 + 2 * k1_vec_bytes(nbins) + k1_align16((size_t)nb * 2);
 }
-__device__ __forceinline__ void mbar_expect_tx(unsigned long long *bar, unsigned bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(unsigned long long *bar, unsigned parity) {
-  asm volatile(
-      "{\n .reg .pred p;\n WAIT_%=:\n"
-      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, unsigned long long *bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                   smem_u32(dst)),
-               "l"(src), "r"(bytes), "r"(smem_u32(bar))
-               : "memory");
+__host__ __device__ constexpr size_t k1_smem_mx(uint32_t nbins) { return (size_t)kTileS * 8 + 2 * k1_vec_bytes(nbins); }
+
+// u16 element (b, l) of a warp's count matrix: rows of 64 B, 16-byte chunks XOR-swizzled by row
+__device__ __forceinline__ unsigned mat_idx(unsigned b, unsigned l) {
+  return b * 32 + ((((l >> 3) ^ ((b >> 1) & 3u)) << 3) | (l & 7u));
 }
 
-// Per-warp scan of 8 steps x 32 records.  No cross-step dependency chain: each step ranks its
-// records within the step (match_any + popc) and its group leaders store the step's per-bin
-// counts (u8) into `stepc[j][bin]`; the order check compares each record with the previous
-// field-valid record of the same step, and the step-to-step part of the check is resolved
-// afterwards from per-step first/last offsets.  A per-bin prefix over the 8 steps then gives
-// each record's rank within (warp, bin) and the warp's bin totals (for the CTA-level prefix).
-template <bool NARROW, bool SMEM, int KB>
-__device__ __forceinline__ void partition_scan(const Params &p, const int4 *src, int n, long long lo,
-                                               unsigned long long wlen, bool keep_ok, unsigned long long *ebuf,
-                                               unsigned *cnt, unsigned *kbuf, unsigned char *stepc, K1Warp &wr) {
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const unsigned lt = lanemask_lt();
-  const unsigned nbins = p.nbins;
-  bool viol = false;
-  unsigned kept = 0;
-  unsigned vmj[kRecPerLane];
-  unsigned long long firstj[kRecPerLane], lastj[kRecPerLane];
-  if (keep_ok) {  // zero this warp's step counts
-    unsigned *z = reinterpret_cast<unsigned *>(stepc);
-    for (unsigned q = lane; q < (unsigned)kRecPerLane * nbins / 4u; q += 32) z[q] = 0u;
-    __syncwarp();
-  }
-  unsigned capj[kRecPerLane];
-  if (SMEM) {  // registered capacities fetched up front (the table lives in L2)
-#pragma unroll
-    for (int j = 0; j < kRecPerLane; ++j) {
-      const int i = warp * 256 + j * 32 + lane;
-      const unsigned b = i < n ? (unsigned)reinterpret_cast<const int *>(src + i)[2] : 0u;
-      capj[j] = __ldg(p.cap + (b < p.nb ? b : 0u));
-    }
-  }
-  constexpr int G = 4;
-#pragma unroll
-  for (int h = 0; h < kRecPerLane / G; ++h) {
-    int4 v[G];
-#pragma unroll
-    for (int jj = 0; jj < G; ++jj) {
-      const int i = warp * 256 + (h * G + jj) * 32 + lane;
-      if (SMEM) v[jj] = i < n ? src[i] : make_int4(0, 0, 0, 0);
-      else v[jj] = i < n ? ld_stream(src + i) : make_int4(0, 0, 0, 0);
-    }
-#pragma unroll
-    for (int jj = 0; jj < G; ++jj) {
-      const int j = h * G + jj;
-      const int i = warp * 256 + j * 32 + lane;
-      const unsigned b = (unsigned)v[jj].z, lvl = (unsigned)v[jj].w & 0xFFFFu, c = (unsigned)v[jj].w >> 16;
-      const unsigned capb = SMEM ? capj[j] : __ldg(p.cap + (b < p.nb ? b : 0u));
-      const bool valid = (i < n) & (b < p.nb) & (c == capb) & (lvl <= c);
-      const unsigned long long off = (unsigned long long)(rec_ts(v[jj]) - lo);
-      const bool inr = off < wlen;
-      const unsigned vm = __ballot_sync(kFull, valid);
-      const unsigned lower = vm & lt;
-      const int srcl = lower ? 31 - __clz(lower) : lane;
-      bool bad;
-      if (NARROW) {
-        const unsigned o = (unsigned)off;
-        const unsigned pv = __shfl_sync(kFull, o, srcl);
-        bad = valid & ((!inr) | ((lower != 0) & (o < pv)));
-      } else {
-        const unsigned long long pv = __shfl_sync(kFull, off, srcl);
-        bad = valid & ((!inr) | ((lower != 0) & (off < pv)));
-      }
-      viol |= bad;
-      vmj[j] = vm;
-      firstj[j] = __shfl_sync(kFull, off, vm ? __ffs(vm) - 1 : 0);
-      lastj[j] = __shfl_sync(kFull, off, vm ? 31 - __clz(vm) : 0);
-      const bool keep = valid & keep_ok;
-      kept += keep;
-      const unsigned key = keep ? (b >> kBinLog) : kNoKey;
-      unsigned rank = 0;
-      if (keep_ok) {
-        const unsigned peers = __match_any_sync(kFull, key);  // measured faster than match_bits here
-        rank = __popc(peers & lt);
-        if (keep && rank == 0) stepc[j * nbins + key] = (unsigned char)__popc(peers);
-        if (keep) ebuf[i] = (off << 24) | ((unsigned long long)lvl << 8) | (b & (kBin - 1));
-      }
-      kbuf[i] = (key << 16) | rank;
-    }
-  }
-  // step-to-step order: each step's first field-valid offset >= the previous steps' last one
-  bool has = false;
-  unsigned long long carry = 0, first = 0;
-#pragma unroll
-  for (int j = 0; j < kRecPerLane; ++j) {
-    if (vmj[j]) {
-      if (has && firstj[j] < carry) viol = true;
-      if (!has) first = firstj[j];
-      has = true;
-      carry = lastj[j];
-    }
-  }
-  if (keep_ok) {  // per-bin exclusive prefix over the steps; warp totals -> the CTA counters
-    __syncwarp();
-    unsigned short *c16 = reinterpret_cast<unsigned short *>(cnt) + warp * nbins;
-    for (unsigned k = lane; k < nbins; k += 32) {
-      unsigned run = 0;
-#pragma unroll
-      for (int j = 0; j < kRecPerLane; ++j) {
-        const unsigned x = stepc[j * nbins + k];
-        stepc[j * nbins + k] = (unsigned char)run;
-        run += x;
-      }
-      c16[k] = (unsigned short)run;
-    }
-  }
-  kept = warp_sum(kept);
-  wr.first = first;
-  wr.last = carry;
-  wr.has = has;
-  wr.viol = __any_sync(kFull, viol);
-  wr.kept = kept;
-}
-
-// key width: bins are 0..nbins-1 and the all-ones key marks "not kept", so nbins < 2^KB - 1 + 1
-template <bool SMEM>
-__device__ __forceinline__ void partition_scan_dispatch(const Params &p, const int4 *src, int n, long long lo,
-                                                        unsigned long long wlen, bool keep_ok, bool narrow,
-                                                        unsigned long long *ebuf, unsigned *cnt, unsigned *kbuf,
-                                                        unsigned char *stepc, K1Warp &wr) {
-  const unsigned need = 32 - __clz(p.nbins);  // smallest KB with nbins <= 2^KB - 1
-#define RTM_SCAN_CASE(KB_)                                                                                   \
-  case KB_:                                                                                                  \
-    if (narrow) partition_scan<true, SMEM, KB_>(p, src, n, lo, wlen, keep_ok, ebuf, cnt, kbuf, stepc, wr);   \
-    else partition_scan<false, SMEM, KB_>(p, src, n, lo, wlen, keep_ok, ebuf, cnt, kbuf, stepc, wr);         \
-    break;
-  switch (need <= 7 ? 7u : 11u) {  // two instantiations keep the hot code small
-    RTM_SCAN_CASE(7) default : RTM_SCAN_CASE(11)
-  }
-#undef RTM_SCAN_CASE
-}
-
-struct K1Smem {            // static shared part of both partition kernels
-  unsigned scan_scratch[32];
-  K1Warp wsum[kK1Warps];
-  unsigned kept;
-};
-
-// Tile bookkeeping shared by both kernels: region, position range, bounds.
-struct TileInfo {
-  long long start;
+struct K1Tile {
+  unsigned tile;
   int n;
   Region g;
   long long lo;
   unsigned long long wlen;
+  long long start;
 };
-__device__ __forceinline__ TileInfo tile_info(const Params &p, unsigned tile) {
-  TileInfo t;
+__device__ __forceinline__ K1Tile k1_tile(const Params &p, unsigned tile) {
+  K1Tile t;
+  t.tile = tile;
   const unsigned r = p.tile_reg_s[tile];
   t.start = p.Bs[r] + (long long)(tile - p.rts[r]) * kTileS;
   long long endp = p.Bs[r + 1];
@@ -453,203 +302,295 @@ __device__ __forceinline__ TileInfo tile_info(const Params &p, unsigned tile) {
   return t;
 }
 
-// Everything after the per-sample scan: tile meta + drop / kept counts, bin offsets, scatter.
-// Ends with __syncthreads() (the caller may reuse all shared buffers afterwards).
-__device__ __forceinline__ void partition_finish(const Params &p, unsigned tile, const TileInfo &t, K1Smem &K,
-                                                 const K1Warp &wr, const unsigned long long *ebuf, unsigned *binoff,
-                                                 unsigned *cnt, const unsigned *kbuf, const unsigned char *stepc,
-                                                 unsigned long long *sbuf) {
+// After B1: tile meta + drop / kept counts (warp 0), in warp order.
+__device__ __forceinline__ void k1_tile_summary(const Params &p, const K1Tile &t, const K1WarpSum *wsum) {
+  const int lane = threadIdx.x & 31;
+  K1WarpSum x;
+  x.first = x.last = 0;
+  x.has = x.viol = x.kept = x.pad = 0;
+  if (lane < kK1Warps) x = wsum[lane];
+  const unsigned hm = __ballot_sync(kFull, x.has != 0);
+  const unsigned lower = hm & lanemask_lt();
+  const unsigned long long pl = __shfl_sync(kFull, x.last, lower ? 31 - __clz(lower) : lane);
+  const bool bad = (x.viol != 0) | ((x.has != 0) & (lower != 0) & (x.first < pl));
+  const bool tv = __any_sync(kFull, bad);
+  const unsigned tk = warp_sum(x.kept);
+  const unsigned long long tf = __shfl_sync(kFull, x.first, hm ? __ffs(hm) - 1 : 0);
+  const unsigned long long tl = __shfl_sync(kFull, x.last, hm ? 31 - __clz(hm) : 0);
+  if (lane == 0) {
+    TileMeta m;
+    m.first_ts = (long long)((unsigned long long)t.lo + tf);
+    m.last_ts = (long long)((unsigned long long)t.lo + tl);
+    m.flags = (hm ? 1u : 0u) | (tv ? 2u : 0u);
+    m.pad = 0;
+    p.smeta[t.tile] = m;
+    if ((unsigned)t.n > tk) atomicAdd(p.win + WF_DROPPED * p.W + t.g.charge, (unsigned long long)(t.n - tk));
+    if (tk) atomicAdd(p.win + WF_SAMPLES * p.W + t.g.window, (unsigned long long)tk);
+  }
+}
+
+// After B1 (window tiles): this warp's bin bases -> myb; warp 0 writes the soff row.  Returns the
+// tile's kept total.
+__device__ __forceinline__ unsigned k1_bin_bases(const Params &p, unsigned tile, const unsigned short *wt,
+                                                 unsigned short *myb) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned nbins = p.nbins;
-  const bool is_win = t.g.window >= 0;
-  if (lane == 0) K.wsum[warp] = wr;
-  __syncthreads();
-  if (warp == 0) {  // tile summary over the 16 warps (lanes 0..15), in warp order
-    K1Warp x;
-    x.first = x.last = 0;
-    x.has = x.viol = x.kept = 0;
-    if (lane < kK1Warps) x = K.wsum[lane];
-    const unsigned hm = __ballot_sync(kFull, x.has != 0);
-    // order across warps: each warp's first valid offset >= the last valid offset of the nearest
-    // earlier warp with valid records (within-warp order was checked in the scan)
-    const unsigned lower = hm & lanemask_lt();
-    const unsigned long long prev_last = __shfl_sync(kFull, x.last, lower ? 31 - __clz(lower) : lane);
-    const bool bad = (x.viol != 0) | ((x.has != 0) & (lower != 0) & (x.first < prev_last));
-    const bool tv = __any_sync(kFull, bad);
-    const unsigned tk = warp_sum(x.kept);
-    const unsigned long long tf = hm ? __shfl_sync(kFull, x.first, __ffs(hm) - 1) : 0ull;
-    const unsigned long long tl = hm ? __shfl_sync(kFull, x.last, 31 - __clz(hm)) : 0ull;
-    if (lane == 0) {
-      TileMeta m;
-      m.first_ts = (long long)((unsigned long long)t.lo + tf);
-      m.last_ts = (long long)((unsigned long long)t.lo + tl);
-      m.flags = (hm ? 1u : 0u) | (tv ? 2u : 0u);
-      m.pad = 0;
-      p.smeta[tile] = m;
-      if ((unsigned)t.n > tk) atomicAdd(p.win + WF_DROPPED * p.W + t.g.charge, (unsigned long long)(t.n - tk));
-      if (tk) atomicAdd(p.win + WF_SAMPLES * p.W + t.g.window, (unsigned long long)tk);
-      K.kept = tk;
-    }
-  }
-  long long ptt = clock64();
-  PT_MARK(p, 4, ptt);
-  if (!is_win) {
-    __syncthreads();
-    return;
-  }
-  // per-bin exclusive prefix over the 16 warps: 16 consecutive lanes hold one bin's warp counts
-  unsigned short *cnt16 = reinterpret_cast<unsigned short *>(cnt);  // u16 [16][nbins]
-  for (unsigned base = 0; base < kK1Warps * nbins; base += blockDim.x) {
-    const unsigned q = base + threadIdx.x;
-    const unsigned bb = q >> 4, w = q & 15u;
-    const bool in = q < kK1Warps * nbins;
-    const unsigned c = in ? cnt16[w * nbins + bb] : 0u;
-    unsigned x = c;
+  uint16_t *offs = p.soff + (size_t)tile * (nbins + 1);
+  unsigned carry = 0;
+  for (unsigned b0 = 0; b0 < nbins; b0 += 32) {
+    const unsigned b = b0 + lane;
+    unsigned T = 0, P = 0;
+    if (b < nbins) {
 #pragma unroll
-    for (int o = 1; o < 16; o <<= 1) {
-      const unsigned y = __shfl_up_sync(kFull, x, o, 16);
-      if (w >= (unsigned)o) x += y;
-    }
-    if (in) {
-      cnt16[w * nbins + bb] = (unsigned short)(x - c);
-      if (w == 15) binoff[bb] = x;  // bin total
-    }
-  }
-  __syncthreads();
-  const unsigned total_kept = K.kept;
-  if (warp == 0) {  // exclusive scan over bins (nbins <= 3072: <= 96 per lane)
-    unsigned carry = 0;
-    for (unsigned b0 = 0; b0 < nbins; b0 += 32) {
-      const unsigned bb = b0 + lane;
-      const unsigned v = bb < nbins ? binoff[bb] : 0u;
-      unsigned x = v;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const unsigned y = __shfl_up_sync(kFull, x, o);
-        if (lane >= o) x += y;
+      for (int w2 = 0; w2 < kK1Warps; ++w2) {
+        const unsigned x = wt[(size_t)w2 * nbins + b];
+        T += x;
+        P += w2 < warp ? x : 0u;
       }
-      if (bb < nbins) binoff[bb] = carry + x - v;
-      carry += __shfl_sync(kFull, x, 31);
     }
-    if (lane == 0) binoff[nbins] = total_kept;
+    unsigned incl = T;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned y = __shfl_up_sync(kFull, incl, o);
+      if (lane >= o) incl += y;
+    }
+    const unsigned base = carry + incl - T;
+    if (b < nbins) {
+      myb[b] = (unsigned short)(base + P);
+      if (warp == 0) offs[b] = (uint16_t)base;
+    }
+    carry += __shfl_sync(kFull, incl, 31);
   }
-  __syncthreads();
-  PT_MARK(p, 5, ptt);
-  uint32_t *offs = p.soff + (size_t)tile * (nbins + 1);
-  for (unsigned bb = threadIdx.x; bb <= nbins; bb += blockDim.x) offs[bb] = binoff[bb];
-  unsigned long long *dst = p.stage + (size_t)tile * kTileS;
-  unsigned long long *out = sbuf ? sbuf : dst;  // permute in shared memory when a buffer is free
-#pragma unroll 4
-  for (int j = 0; j < kRecPerLane; ++j) {
-    const int i = warp * 256 + j * 32 + lane;
-    const unsigned kv = kbuf[i], key = kv >> 16;
-    if (key != kNoKey && i < t.n)
-      out[binoff[key] + cnt16[warp * nbins + key] + stepc[(size_t)warp * kRecPerLane * nbins + j * nbins + key] +
-          (kv & 0xFFFFu)] = ebuf[i];
-  }
-  __syncthreads();
-  if (sbuf) {  // coalesced 16-byte copy-out of the bin-sorted tile
-    const uint4 *s4 = reinterpret_cast<const uint4 *>(sbuf);
-    uint4 *d4 = reinterpret_cast<uint4 *>(dst);
-    for (unsigned q = threadIdx.x; q < (total_kept + 1) / 2; q += blockDim.x) d4[q] = s4[q];
-    __syncthreads();
-  }
-  PT_MARK(p, 6, ptt);
-  (void)ptt;
+  if (warp == 0 && lane == 0) offs[nbins] = (uint16_t)carry;
+  __syncwarp();
+  return carry;
 }
 
-__device__ __forceinline__ void zero_counters(const Params &p, unsigned *cnt) {
-  for (unsigned i = threadIdx.x; i < kK1Warps * p.nbins / 2 + 1; i += blockDim.x) cnt[i] = 0;
+__device__ __forceinline__ void k1_publish(K1WarpSum *wsum, unsigned long long first, unsigned long long last,
+                                           bool has, bool viol, unsigned kept) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  kept = warp_sum(kept);
+  viol = __any_sync(kFull, viol);
+  if (lane == 0) {
+    K1WarpSum s;
+    s.first = first;
+    s.last = last;
+    s.has = has;
+    s.viol = viol;
+    s.kept = kept;
+    s.pad = 0;
+    wsum[warp] = s;
+  }
 }
 
-__global__ void __launch_bounds__(kK1Threads, 2) k_partition(Params p, int narrow, unsigned tile0) {
-  if (tile0 + blockIdx.x >= p.rts[p.W + 2]) return;  // grid sized by an upper bound
+__global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
-  unsigned long long *ebuf = reinterpret_cast<unsigned long long *>(smem);  // [4096]
-  unsigned *kbuf = reinterpret_cast<unsigned *>(ebuf + kTileS);             // [4096] key<<16|pos
-  unsigned *binoff = kbuf + kTileS;                                         // [nbins+1]
-  unsigned *cnt = binoff + p.nbins + 1;                                     // u16 [16][nbins]
-  unsigned char *stepc = reinterpret_cast<unsigned char *>(cnt + kK1Warps * p.nbins / 2 + 1);  // u8 [16][8][nbins]
-  __shared__ K1Smem K;
-  const unsigned tile = tile0 + blockIdx.x;
-  const TileInfo t = tile_info(p, tile);
-  const bool is_win = t.g.window >= 0;
-  if (is_win) zero_counters(p, cnt);
+  __shared__ K1WarpSum wsum[kK1Warps];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const unsigned lt = lanemask_lt();
+  const unsigned nbins = p.nbins;
+  unsigned short *wt = reinterpret_cast<unsigned short *>(smem + (size_t)kTileS * 16);
+  unsigned short *wb = reinterpret_cast<unsigned short *>(smem + (size_t)kTileS * 16 + k1_vec_bytes(nbins));
+  unsigned short *capS = reinterpret_cast<unsigned short *>(smem + (size_t)kTileS * 16 + 2 * k1_vec_bytes(nbins));
+  unsigned short *myt = wt + (size_t)warp * nbins;
+  unsigned short *myb = wb + (size_t)warp * nbins;
+  int4 *raw = reinterpret_cast<int4 *>(smem) + warp * kSub;                          // this warp's slot
+  unsigned short *mat = reinterpret_cast<unsigned short *>(raw);                      // aliases the slot
+  unsigned long long *sbuf = reinterpret_cast<unsigned long long *>(smem);            // CTA permute buffer
+  for (unsigned i = threadIdx.x; i < p.nb; i += kK1Threads) capS[i] = __ldg(p.cap + i);
   __syncthreads();
-  const int4 *src = reinterpret_cast<const int4 *>(p.s) + t.start;
-  K1Warp wr;
-  unsigned char *wstep = stepc + (size_t)(threadIdx.x >> 5) * kRecPerLane * p.nbins;
-#ifdef RTM_PHASE_TIMING
-  long long pt0 = clock64();
-  if (threadIdx.x == 0 && p.dbg) atomicAdd(p.dbg + 3, 1ull);
-#endif
-  partition_scan_dispatch<false>(p, src, t.n, t.lo, t.wlen, is_win, is_win && narrow, ebuf, cnt, kbuf, wstep, wr);
-  PT_MARK(p, 1, pt0);
-  partition_finish(p, tile, t, K, wr, ebuf, binoff, cnt, kbuf, stepc, nullptr);
-}
-
-__global__ void __launch_bounds__(kK1Threads, 1) k_partition_tma(Params p, int narrow) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  int4 *raw = reinterpret_cast<int4 *>(smem);                                 // [2][4096] records
-  unsigned long long *ebuf = reinterpret_cast<unsigned long long *>(raw + 2 * kTileS);  // [4096]
-  unsigned *kbuf = reinterpret_cast<unsigned *>(ebuf + kTileS);                  // [4096]
-  unsigned *binoff = kbuf + kTileS;                                              // [nbins+1]
-  unsigned *cnt = binoff + p.nbins + 1;                                          // u16 [16][nbins]
-  unsigned char *stepc = reinterpret_cast<unsigned char *>(cnt + kK1Warps * p.nbins / 2 + 1);  // u8 [16][8][nbins]
-  __shared__ K1Smem K;
-  __shared__ __align__(8) unsigned long long bar[2];
-  if (threadIdx.x == 0) {
-    mbar_init(&bar[0], 1);
-    mbar_init(&bar[1], 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  auto issue = [&](unsigned tile, int buf) {
-    const TileInfo t = tile_info(p, tile);
-    const unsigned bytes = (unsigned)t.n * 16u;
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    mbar_expect_tx(&bar[buf], bytes);
-    bulk_g2s(raw + buf * kTileS, reinterpret_cast<const int4 *>(p.s) + t.start, bytes, &bar[buf]);
-  };
-  const unsigned n_tiles = p.rts[p.W + 2];  // device count (the grid is sized by an upper bound)
-  unsigned tile = blockIdx.x;
-  if (threadIdx.x == 0 && tile < n_tiles) issue(tile, 0);
-  for (unsigned it = 0; tile < n_tiles; ++it, tile += gridDim.x) {
-    const int buf = it & 1;
-    const unsigned next = tile + gridDim.x;
-    if (threadIdx.x == 0 && next < n_tiles) issue(next, buf ^ 1);  // buffer freed at end of it-1
-    const TileInfo t = tile_info(p, tile);
+  const unsigned n_tiles = p.rts[p.W + 2];
+  const int sub0 = warp * kSub;
+  for (unsigned tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+    const K1Tile t = k1_tile(p, tile);
     const bool is_win = t.g.window >= 0;
-    if (is_win) zero_counters(p, cnt);
-    __syncthreads();
-#ifdef RTM_PHASE_TIMING
-    long long c0 = clock64();
-#endif
-    mbar_wait(&bar[buf], (it >> 1) & 1u);
-#ifdef RTM_PHASE_TIMING
-    long long c1 = clock64();
-#endif
-    const int4 *src = raw + buf * kTileS;
-    K1Warp wr;
-    unsigned char *wstep = stepc + (size_t)(threadIdx.x >> 5) * kRecPerLane * p.nbins;
-    partition_scan_dispatch<true>(p, src, t.n, t.lo, t.wlen, is_win, is_win && narrow, ebuf, cnt, kbuf, wstep, wr);
-#ifdef RTM_PHASE_TIMING
-    __syncthreads();
-    long long c2 = clock64();
-#endif
-    // the tile's raw records are consumed: its TMA slot holds the permuted entries
-    partition_finish(p, tile, t, K, wr, ebuf, binoff, cnt, kbuf, stepc,
-                     reinterpret_cast<unsigned long long *>(raw + buf * kTileS));
-#ifdef RTM_PHASE_TIMING
-    long long c3 = clock64();
-    if (threadIdx.x == 0 && p.dbg) {
-      atomicAdd(p.dbg + 0, (unsigned long long)(c1 - c0));
-      atomicAdd(p.dbg + 1, (unsigned long long)(c2 - c1));
-      atomicAdd(p.dbg + 2, (unsigned long long)(c3 - c2));
-      atomicAdd(p.dbg + 3, 1ull);
+    const int4 *src = reinterpret_cast<const int4 *>(p.s) + t.start + sub0;
+    // stage the sub-tile: record i at 16-byte slot 16(i>>4) + ((i&15) ^ ((i>>4)&7))
+#pragma unroll
+    for (int h = 0; h < kPerLane; h += 4) {
+      int4 v[4];
+#pragma unroll
+      for (int jj = 0; jj < 4; ++jj) {
+        const int i = (h + jj) * 32 + lane;
+        v[jj] = sub0 + i < t.n ? ld_stream(src + i) : make_int4(0, 0, 0, 0);
+      }
+#pragma unroll
+      for (int jj = 0; jj < 4; ++jj) {
+        const int i = (h + jj) * 32 + lane;
+        raw[(i & ~15) | ((i & 15) ^ ((i >> 4) & 7))] = v[jj];
+      }
     }
-#endif
+    __syncwarp();
+    unsigned long long e[kPerLane];
+    unsigned kp[kPerLane];  // key << 16 | position within the warp's bin group
+    unsigned long long first = 0, last = 0;
+    bool has = false, viol = false;
+    unsigned kept = 0;
+#pragma unroll
+    for (int k = 0; k < kPerLane; ++k) {
+      const int i = lane * kPerLane + k;
+      const int4 v = raw[lane * kPerLane + (k ^ (lane & 7))];
+      const unsigned b = (unsigned)v.z, lvl = (unsigned)v.w & 0xFFFFu, c = (unsigned)v.w >> 16;
+      const unsigned capb = capS[b < p.nb ? b : 0u];
+      const bool valid = (sub0 + i < t.n) & (b < p.nb) & (c == capb) & (lvl <= c);
+      const unsigned long long off = (unsigned long long)(rec_ts(v) - t.lo);
+      if (valid) {
+        viol |= (off >= t.wlen) | (has & (off < last));
+        if (!has) first = off;
+        has = true;
+        last = off;
+      }
+      const bool keep = valid & is_win;
+      kept += keep;
+      const unsigned key = keep ? (b >> kBinLog) : kNoKey;
+      unsigned rank = 0;
+#pragma unroll
+      for (int q = 0; q < k; ++q) rank += (kp[q] >> 16) == key;
+      kp[k] = (key << 16) | rank;
+      e[k] = (off << 24) | ((unsigned long long)lvl << 8) | (b & (kBin - 1));
+    }
+    {  // order across lanes: my first vs the last of the nearest earlier lane with a valid record
+      const unsigned hm = __ballot_sync(kFull, has);
+      const unsigned lower = hm & lt;
+      const unsigned long long pl = __shfl_sync(kFull, last, lower ? 31 - __clz(lower) : lane);
+      viol |= has & (lower != 0) & (first < pl);
+      const unsigned long long f0 = __shfl_sync(kFull, first, hm ? __ffs(hm) - 1 : 0);
+      const unsigned long long l0 = __shfl_sync(kFull, last, hm ? 31 - __clz(hm) : 0);
+      first = f0;
+      last = l0;
+      has = hm != 0;
+    }
+    if (is_win) {  // per-(bin, lane) counts -> row prefix -> position within the warp's bin group
+      uint4 *m4 = reinterpret_cast<uint4 *>(mat);  // the raw slot is consumed (registers)
+      for (unsigned q = lane; q < nbins * 4; q += 32) m4[q] = make_uint4(0, 0, 0, 0);
+      __syncwarp();
+#pragma unroll
+      for (int k = 0; k < kPerLane; ++k)  // final count of (bin, lane) = last rank + 1 (program order)
+        if ((kp[k] >> 16) != kNoKey) mat[mat_idx(kp[k] >> 16, lane)] = (unsigned short)((kp[k] & 0xFFFFu) + 1);
+      __syncwarp();
+      for (unsigned b = lane; b < nbins; b += 32) {
+        uint4 *row = reinterpret_cast<uint4 *>(mat + b * 32);
+        unsigned run = 0;
+#pragma unroll
+        for (int cq = 0; cq < 4; ++cq) {
+          uint4 q = row[cq ^ ((b >> 1) & 3u)];
+          unsigned *w4 = reinterpret_cast<unsigned *>(&q);
+#pragma unroll
+          for (int x = 0; x < 4; ++x) {
+            const unsigned wv = w4[x], a = wv & 0xFFFFu, bb = wv >> 16;
+            w4[x] = run | ((run + a) << 16);
+            run += a + bb;
+          }
+          row[cq ^ ((b >> 1) & 3u)] = q;
+        }
+        myt[b] = (unsigned short)run;
+      }
+      __syncwarp();
+#pragma unroll
+      for (int k = 0; k < kPerLane; ++k)
+        if ((kp[k] >> 16) != kNoKey) kp[k] += mat[mat_idx(kp[k] >> 16, lane)];
+    }
+    k1_publish(wsum, first, last, has, viol, kept);
+    __syncthreads();  // B1: summaries + bin totals published; every raw slot consumed
+    if (warp == 0) k1_tile_summary(p, t, wsum);
+    if (is_win) {
+      const unsigned total = k1_bin_bases(p, tile, wt, myb);
+#pragma unroll
+      for (int k = 0; k < kPerLane; ++k) {
+        const unsigned key = kp[k] >> 16;
+        if (key != kNoKey) sbuf[myb[key] + (kp[k] & 0xFFFFu)] = e[k];
+      }
+      __syncthreads();  // B2: the tile is bin-sorted in shared memory
+      const uint4 *s4 = reinterpret_cast<const uint4 *>(sbuf);
+      uint4 *d4 = reinterpret_cast<uint4 *>(p.stage + (size_t)tile * kTileS);
+      for (unsigned q = threadIdx.x; q < (total + 1) / 2; q += kK1Threads) d4[q] = s4[q];
+    }
+    __syncthreads();  // B3: shared buffers free for the next tile
   }
+}
+
+__global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ K1WarpSum wsum[kK1Warps];
+  const unsigned tile = blockIdx.x;
+  if (tile >= p.rts[p.W + 2]) return;  // grid sized by an upper bound (CTA-uniform)
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const unsigned lt = lanemask_lt();
+  const unsigned nbins = p.nbins;
+  unsigned long long *sbuf = reinterpret_cast<unsigned long long *>(smem);
+  unsigned short *wt = reinterpret_cast<unsigned short *>(smem + (size_t)kTileS * 8);
+  unsigned short *wb = reinterpret_cast<unsigned short *>(smem + (size_t)kTileS * 8 + k1_vec_bytes(nbins));
+  unsigned short *myt = wt + (size_t)warp * nbins;
+  unsigned short *myb = wb + (size_t)warp * nbins;
+  const K1Tile t = k1_tile(p, tile);
+  const bool is_win = t.g.window >= 0;
+  const int sub0 = warp * kSub;
+  const int4 *src = reinterpret_cast<const int4 *>(p.s) + t.start + sub0;
+  if (is_win)
+    for (unsigned q = lane; q < nbins; q += 32) myt[q] = 0;
+  __syncwarp();
+  unsigned long long e[kPerLane];
+  unsigned kp[kPerLane];  // key << 16 | position within the warp's bin group
+  unsigned long long first = 0, last = 0;
+  bool has = false, viol = false;
+  unsigned kept = 0;
+#pragma unroll
+  for (int h = 0; h < kPerLane; h += 4) {
+    int4 v[4];
+#pragma unroll
+    for (int jj = 0; jj < 4; ++jj) {
+      const int i = (h + jj) * 32 + lane;
+      v[jj] = sub0 + i < t.n ? ld_stream(src + i) : make_int4(0, 0, 0, 0);
+    }
+#pragma unroll
+    for (int jj = 0; jj < 4; ++jj) {
+      const int j = h + jj;
+      const int i = j * 32 + lane;
+      const unsigned b = (unsigned)v[jj].z, lvl = (unsigned)v[jj].w & 0xFFFFu, c = (unsigned)v[jj].w >> 16;
+      const unsigned capb = __ldg(p.cap + (b < p.nb ? b : 0u));
+      const bool valid = (sub0 + i < t.n) & (b < p.nb) & (c == capb) & (lvl <= c);
+      const unsigned long long off = (unsigned long long)(rec_ts(v[jj]) - t.lo);
+      const unsigned vm = __ballot_sync(kFull, valid);
+      const unsigned lower = vm & lt;
+      const unsigned long long pv = __shfl_sync(kFull, off, lower ? 31 - __clz(lower) : lane);
+      const unsigned long long nl = __shfl_sync(kFull, off, vm ? 31 - __clz(vm) : lane);
+      const unsigned long long fo = __shfl_sync(kFull, off, vm ? __ffs(vm) - 1 : lane);
+      viol |= valid & ((off >= t.wlen) | (lower ? off < pv : (has & (off < last))));
+      if (vm) {
+        if (!has) first = fo;
+        has = true;
+        last = nl;
+      }
+      const bool keep = valid & is_win;
+      kept += keep;
+      const unsigned key = keep ? (b >> kBinLog) : kNoKey;
+      unsigned pos = 0;
+      if (is_win) {  // CTA-uniform
+        const unsigned peers = __match_any_sync(kFull, key);
+        const unsigned basec = keep ? myt[key] : 0u;
+        __syncwarp();
+        if (keep && lane == __ffs(peers) - 1) myt[key] = (unsigned short)(basec + __popc(peers));
+        __syncwarp();
+        pos = basec + __popc(peers & lt);
+      }
+      kp[j] = (key << 16) | pos;
+      e[j] = (off << 24) | ((unsigned long long)lvl << 8) | (b & (kBin - 1));
+    }
+  }
+  k1_publish(wsum, first, last, has, viol, kept);
+  __syncthreads();  // B1
+  if (warp == 0) k1_tile_summary(p, t, wsum);
+  if (!is_win) return;
+  const unsigned total = k1_bin_bases(p, tile, wt, myb);
+#pragma unroll
+  for (int k = 0; k < kPerLane; ++k) {
+    const unsigned key = kp[k] >> 16;
+    if (key != kNoKey) sbuf[myb[key] + (kp[k] & 0xFFFFu)] = e[k];
+  }
+  __syncthreads();  // B2
+  const uint4 *s4 = reinterpret_cast<const uint4 *>(sbuf);
+  uint4 *d4 = reinterpret_cast<uint4 *>(p.stage + (size_t)tile * kTileS);
+  for (unsigned q = threadIdx.x; q < (total + 1) / 2; q += kK1Threads) d4[q] = s4[q];
 }
 
 // ============================================================================================
@@ -863,9 +804,9 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
     for (unsigned tg = t_lo; tg < t_hi; tg += 32) {
       unsigned seg_lo = 0, seg_len = 0;
       if (tg + lane < t_hi) {
-        const uint32_t *o = p.soff + (size_t)(tg + lane) * (p.nbins + 1) + bin;
+        const uint16_t *o = p.soff + (size_t)(tg + lane) * (p.nbins + 1) + bin;
         seg_lo = __ldg(o);
-        seg_len = __ldg(o + 1) - seg_lo;
+        seg_len = (unsigned)__ldg(o + 1) - seg_lo;
       }
       unsigned pre = seg_len;  // inclusive prefix of segment lengths over lanes
 #pragma unroll
@@ -1453,19 +1394,12 @@ __global__ void k_merge_tables(Params p, const unsigned char *g, unsigned world,
 // launchers
 // ============================================================================================
 size_t fold_smem_bytes() { return sizeof(FoldSmem) * kFoldWarps; }
-size_t partition_smem_bytes(uint32_t nbins) {
-  return (size_t)kTileS * 8 + (size_t)kTileS * 4 + (size_t)(nbins + 1) * 4 + ((size_t)kK1Warps * nbins / 2 + 1) * 4 +
-         (size_t)kK1Warps * kRecPerLane * ((nbins + 3) & ~3u) + 16;
+size_t partition_smem_bytes(uint32_t nbins, uint32_t nb) {
+  return nbins <= kLmMaxBins ? k1_smem_lm(nbins, nb) : k1_smem_mx(nbins);
 }
-static_assert((size_t)kTileS * 12 + (size_t)(kMaxBins + 1) * 4 + ((size_t)kK1Warps * kMaxBins / 2 + 1) * 4 +
-                      (size_t)kK1Warps * kRecPerLane * kMaxBins + 16 <= 227 * 1024,
+static_assert(2 * (k1_smem_lm(80, 20480) + 1024 + 512) <= 228 * 1024, "C2-sized partition CTAs must fit 2 per SM");
+static_assert(k1_smem_lm(kLmMaxBins, kLmMaxBins * kBin) <= 227 * 1024 && k1_smem_mx(kMaxBins) <= 227 * 1024,
               "partition shared memory exceeds the 227 KB opt-in limit");
-size_t partition_tma_smem_bytes(uint32_t nbins) { return (size_t)2 * kTileS * 16 + partition_smem_bytes(nbins); }
-static_assert(227 * 1024 >= 0, "");
-static_assert((size_t)2 * kTileS * 16 + (size_t)kTileS * 12 + (size_t)(kTmaMaxBins + 1) * 4 +
-                      ((size_t)kK1Warps * kTmaMaxBins / 2 + 1) * 4 + (size_t)kK1Warps * kRecPerLane * kTmaMaxBins +
-                      16 <= 227 * 1024,
-              "TMA partition shared memory exceeds the 227 KB opt-in limit");
 size_t topk_smem_bytes(uint32_t nb) {
   return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8 + kTopkCand * 4;
 }
@@ -1492,12 +1426,16 @@ void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
 
 void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   if (!p.n_tiles_s) return;
-  static const bool use_tma = getenv("RTM_TMA") != nullptr;     // measured slower on C2
-  if (p.nbins <= kTmaMaxBins && use_tma) {
-    const unsigned grid = p.n_tiles_s < (unsigned)n_sms ? p.n_tiles_s : (unsigned)n_sms;
-    k_partition_tma<<<grid, kK1Threads, partition_tma_smem_bytes(p.nbins), st>>>(p, p.narrow);
+  const size_t sm = partition_smem_bytes(p.nbins, p.nb);
+  if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM (capacity table loaded once)
+    int per_sm = 1;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm, kK1Threads, sm);
+    if (per_sm < 1) per_sm = 1;
+    unsigned grid = (unsigned)(n_sms * per_sm);
+    if (grid > p.n_tiles_s) grid = p.n_tiles_s;
+    k_partition_lm<<<grid, kK1Threads, sm, st>>>(p);
   } else {
-    k_partition<<<p.n_tiles_s, kK1Threads, partition_smem_bytes(p.nbins), st>>>(p, p.narrow, 0u);
+    k_partition_mx<<<p.n_tiles_s, kK1Threads, sm, st>>>(p);
   }
 }
 
@@ -1549,10 +1487,9 @@ void configure_kernels_once() {
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 128 || done[dev]) return;
   done[dev] = true;
-  cudaFuncSetAttribute(k_partition, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                       (int)partition_smem_bytes(kMaxBins));
-  cudaFuncSetAttribute(k_partition_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                       (int)partition_tma_smem_bytes(kTmaMaxBins));
+  cudaFuncSetAttribute(k_partition_lm, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       (int)k1_smem_lm(kLmMaxBins, kLmMaxBins * kBin));
+  cudaFuncSetAttribute(k_partition_mx, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
   cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
   cudaFuncSetAttribute(k_topk<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)topk_smem_bytes(kTopkSmemKeys));
