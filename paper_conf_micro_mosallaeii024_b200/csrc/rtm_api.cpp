@@ -62,7 +62,7 @@ struct rtm_ctx {
   DevBuf s_own, e_own;              // internal concatenation
   uint64_t s_own_n = 0, e_own_n = 0;
   // per-call workspaces
-  DevBuf T, Bs, Be, rts, rte, treg_s, treg_e, soff, stage, smeta, emeta, lastlvl, win, kdelta, cdelta, active,
+  DevBuf T, Bs, Be, rts, rte, treg_s, treg_e, tdesc, soff, stage, smeta, emeta, lastlvl, win, kdelta, cdelta, active,
       anyfull, hung, unit_ctr, status, topk, topk_n, prog, bstat, comps, pack, gathered;
   Pinned h_small, h_res;
   // results of the last call
@@ -321,6 +321,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   const size_t Wn = W;
   if ((s = ensure(c, c->treg_s, (size_t)nts * 4))) return s;
   if ((s = ensure(c, c->treg_e, (size_t)nte * 4))) return s;
+  if ((s = ensure(c, c->tdesc, (size_t)nts * sizeof(TileDesc)))) return s;
   if ((s = ensure(c, c->soff, (size_t)nts * (c->nbins + 1) * 2))) return s;
   if ((s = ensure(c, c->stage, (size_t)nts * kTileS * 8))) return s;
   if ((s = ensure(c, c->smeta, (size_t)nts * sizeof(TileMeta)))) return s;
@@ -351,7 +352,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   CK(cudaMemsetAsync(c->unit_ctr.p, 0, 8, c->st));
   CK(cudaMemsetAsync(c->status.p, 0, 8, c->st));
 
-  p.tile_reg_s = (const uint32_t *)c->treg_s.p; p.tile_reg_e = (const uint32_t *)c->treg_e.p;
+  p.tdesc = (TileDesc *)c->tdesc.p; p.tile_reg_s = (const uint32_t *)c->treg_s.p; p.tile_reg_e = (const uint32_t *)c->treg_e.p;
   p.n_tiles_s = nts; p.n_tiles_e = nte;
   p.soff = (uint16_t *)c->soff.p; p.stage = (unsigned long long *)c->stage.p;
   p.smeta = (TileMeta *)c->smeta.p; p.emeta = (TileMeta *)c->emeta.p;
@@ -397,12 +398,10 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     unsigned long long h[8];
     cudaMemcpyAsync(h, p.dbg, 64, cudaMemcpyDeviceToHost, c->st);
     cudaStreamSynchronize(c->st);
-    if (h[3])
-      fprintf(stderr,
-              "[phase] tiles=%llu wait=%.0f scan=%.0f finish=%.0f | fin: summary=%.0f prefix=%.0f scatter=%.0f | "
-              "scan: cap_prefetch=%.0f (cycles/tile)\n",
-              h[3], (double)h[0] / h[3], (double)h[1] / h[3], (double)h[2] / h[3], (double)h[4] / h[3],
-              (double)h[5] / h[3], (double)h[6] / h[3], (double)h[7] / h[3]);
+    if (h[7])
+      fprintf(stderr, "[phase] tiles=%llu  -=%.0f wait_raw=%.0f scan=%.0f rank=%.0f B1=%.0f bases+scatter=%.0f -=%.0f (cycles/tile, thread 0)\n",
+              h[7], (double)h[0] / h[7], (double)h[1] / h[7], (double)h[2] / h[7], (double)h[3] / h[7],
+              (double)h[4] / h[7], (double)h[5] / h[7], (double)h[6] / h[7]);
   }
 #endif
   return RTM_OK;
@@ -575,7 +574,7 @@ void rtm_destroy(rtm_ctx *c) {
   DevBuf *bufs[] = {&c->cap, &c->owner, &c->elig, &c->ktotal, &c->carry[0], &c->carry[1], &c->run[0], &c->run[1],
                     &c->kstart, &c->rcp, &c->elig_ids,
                     &c->kend, &c->cstart, &c->cend, &c->flags, &c->s_own, &c->e_own, &c->T, &c->Bs, &c->Be,
-                    &c->rts, &c->rte, &c->treg_s, &c->treg_e, &c->soff, &c->stage, &c->smeta, &c->emeta,
+                    &c->rts, &c->rte, &c->treg_s, &c->treg_e, &c->tdesc, &c->soff, &c->stage, &c->smeta, &c->emeta,
                     &c->lastlvl, &c->win, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
                     &c->unit_ctr, &c->status, &c->topk, &c->topk_n, &c->prog, &c->bstat, &c->comps, &c->pack,
                     &c->gathered};

@@ -39,6 +39,17 @@ constexpr int64_t kMaxWindowLen = (int64_t)1 << 40;  // ts offset field of a sta
 // per-window scalar accumulators, SoA [kWinFields][W] u64
 enum { WF_SAMPLES = 0, WF_EVENTS, WF_DROPPED, WF_DIGEST, WF_TOUCHED, WF_HUNG, kWinFields };
 
+struct TileDesc {            // per sample tile, precomputed so the partition reads one 48-byte record
+  long long start;           // first record (index into the sample stream)
+  long long lo;              // region lower bound: field-valid records need (u64)(ts - lo) < wlen
+  unsigned long long wlen;
+  int n;                     // records in the tile
+  int window;                // -1: head / tail region
+  unsigned charge;           // window the tile's drops are charged to
+  unsigned pad[3];
+};
+static_assert(sizeof(TileDesc) == 48, "TileDesc is three 16-byte chunks");
+
 struct TileMeta {            // per tile, for the cross-tile order check
   long long first_ts;
   long long last_ts;
@@ -83,6 +94,7 @@ struct Params {
   const uint32_t *tile_reg_e;
   uint32_t n_tiles_s, n_tiles_e;  // upper bounds (grid sizes); device counts are rts/rte[W+2]
   // outputs / workspaces
+  TileDesc *tdesc;           // [n_tiles_s]
   uint16_t *soff;            // [n_tiles_s * (nbins+1)] tile-local bin offsets
   unsigned long long *stage; // [n_tiles_s * kTileS]
   TileMeta *smeta, *emeta;

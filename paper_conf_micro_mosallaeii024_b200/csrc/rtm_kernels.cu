@@ -228,6 +228,31 @@ __global__ void __launch_bounds__(1024) k_regions(long long *B, unsigned long lo
   }
 }
 
+// sample tiles: region id + descriptor (start, bounds, size, window) per tile
+__global__ void k_fill_tile_desc(Params p) {
+  const uint32_t nr = p.W + 2;
+  for (uint32_t r = blockIdx.x; r < nr; r += gridDim.x) {
+    const Region g = region_of(p, r);
+    const long long lo = g.lo_ts;
+    const unsigned long long wlen =
+        g.hi_ts == kTsMax ? (unsigned long long)(kTsMax - lo) + 1ull : (unsigned long long)(g.hi_ts - lo);
+    for (uint32_t t = p.rts[r] + threadIdx.x; t < p.rts[r + 1]; t += blockDim.x) {
+      const_cast<uint32_t *>(p.tile_reg_s)[t] = r;
+      TileDesc d;
+      d.start = p.Bs[r] + (long long)(t - p.rts[r]) * kTileS;
+      long long endp = p.Bs[r + 1];
+      if (endp > d.start + kTileS) endp = d.start + kTileS;
+      d.n = (int)(endp - d.start);
+      d.lo = lo;
+      d.wlen = wlen;
+      d.window = g.window;
+      d.charge = g.charge;
+      d.pad[0] = d.pad[1] = d.pad[2] = 0;
+      p.tdesc[t] = d;
+    }
+  }
+}
+
 __global__ void k_fill_tile_regions(const uint32_t *rt, uint32_t *tile_reg, uint32_t n_regions) {
   for (uint32_t r = blockIdx.x; r < n_regions; r += gridDim.x)
     for (uint32_t t = rt[r] + threadIdx.x; t < rt[r + 1]; t += blockDim.x) tile_reg[t] = r;
@@ -243,9 +268,9 @@ __global__ void k_fill_tile_regions(const uint32_t *rt, uint32_t *tile_reg, uint
 // table lives in shared memory (the field check is a gather per sample: from L1 it was the
 // kernel's bottleneck).  Each warp stages its 512 raw records in shared memory (XOR-swizzled
 // 16-byte slots) and lane l takes the CONSECUTIVE records 16l .. 16l+15, so the stable order
-// inside a bin is (lane, slot).  Rank = equal keys among the lane's earlier samples (register
-// compares, no warp collectives); per-(bin, lane) counts go to a u16 matrix that reuses the
-// warp's raw slot, one row (= bin) per lane is prefix-scanned.
+// inside a bin is (lane, slot).  No warp collectives: rank = a u8 (bin, lane) counter in the
+// warp's (consumed) raw slot; each lane then prefix-scans whole bin rows with byte-SIMD
+// multiplies, so position = rank + earlier lanes' counts of the bin.
 // k_partition_mx (fallback, any n_bins): lanes take strided records; __match_any_sync peers +
 // the warp's bin counters give the rank.
 //
@@ -257,9 +282,9 @@ constexpr int kSub = kTileS / (kK1Threads / 32);  // 512 samples per warp
 constexpr int kPerLane = kSub / 32;               // 16
 constexpr int kK1Warps = kK1Threads / 32;         // 8
 constexpr unsigned kNoKey = 0xFFFFu;
-constexpr uint32_t kLmMaxBins = 128;              // the count matrix (nbins x 64 B) fits the warp's raw slot
+constexpr uint32_t kLmMaxBins = 128;              // count rows (nbins x 48 B) fit the raw slot; cap <= 64 KB
 static_assert(kPerLane == 16, "lane-major swizzle assumes 16 records per lane");
-static_assert((size_t)kLmMaxBins * 64 <= (size_t)kSub * 16, "count matrix must fit the raw slot");
+static_assert((size_t)kLmMaxBins * 48 <= (size_t)kSub * 16, "count rows must fit the raw slot");
 
 struct K1WarpSum {
   unsigned long long first, last;  // offsets of the first / last field-valid record
@@ -268,17 +293,14 @@ struct K1WarpSum {
 
 __host__ __device__ constexpr size_t k1_align16(size_t x) { return (x + 15) & ~(size_t)15; }
 __host__ __device__ constexpr size_t k1_vec_bytes(uint32_t nbins) { return k1_align16((size_t)kK1Warps * nbins * 2); }
-// dynamic shared memory.  lm: raw 16 B x 4096 | wt | wb | cap[nb];  mx: sbuf 8 B x 4096 | wt | wb
+// dynamic shared memory.  lm: raw 16 B x 4096 | wt x 2 (tile parity) | wb | tile descriptors
+// (8 warps x 2) | cap[nb];  mx: sbuf 8 B x 4096 | wt | wb
 // (wt: 8 x nbins u16 bin totals / live counters, wb: 8 x nbins u16 bin bases)
 __host__ __device__ constexpr size_t k1_smem_lm(uint32_t nbins, uint32_t nb) {
-  return (size_t)kTileS * 16 + 2 * k1_vec_bytes(nbins) + k1_align16((size_t)nb * 2);
+  return (size_t)kTileS * 16 + 3 * k1_vec_bytes(nbins) + (size_t)kK1Warps * 2 * sizeof(TileDesc) +
+         k1_align16((size_t)nb * 2);
 }
 __host__ __device__ constexpr size_t k1_smem_mx(uint32_t nbins) { return (size_t)kTileS * 8 + 2 * k1_vec_bytes(nbins); }
-
-// u16 element (b, l) of a warp's count matrix: rows of 64 B, 16-byte chunks XOR-swizzled by row
-__device__ __forceinline__ unsigned mat_idx(unsigned b, unsigned l) {
-  return b * 32 + ((((l >> 3) ^ ((b >> 1) & 3u)) << 3) | (l & 7u));
-}
 
 struct K1Tile {
   unsigned tile;
@@ -288,19 +310,28 @@ struct K1Tile {
   unsigned long long wlen;
   long long start;
 };
-__device__ __forceinline__ K1Tile k1_tile(const Params &p, unsigned tile) {
+__device__ __forceinline__ K1Tile k1_tile_from(const TileDesc &d, unsigned tile) {
   K1Tile t;
   t.tile = tile;
-  const unsigned r = p.tile_reg_s[tile];
-  t.start = p.Bs[r] + (long long)(tile - p.rts[r]) * kTileS;
-  long long endp = p.Bs[r + 1];
-  if (endp > t.start + kTileS) endp = t.start + kTileS;
-  t.n = (int)(endp - t.start);
-  t.g = region_of(p, r);
-  t.lo = t.g.lo_ts;  // field-valid records of the region need (u64)(ts - lo) < wlen
-  t.wlen = t.g.hi_ts == kTsMax ? (unsigned long long)(kTsMax - t.lo) + 1ull : (unsigned long long)(t.g.hi_ts - t.lo);
+  t.start = d.start;
+  t.n = d.n;
+  t.g.lo_ts = d.lo;
+  t.g.hi_ts = 0;  // unused: the bound is (lo, wlen)
+  t.g.window = d.window;
+  t.g.charge = d.charge;
+  t.lo = d.lo;
+  t.wlen = d.wlen;
   return t;
 }
+__device__ __forceinline__ K1Tile k1_tile(const Params &p, unsigned tile) { return k1_tile_from(p.tdesc[tile], tile); }
+
+__device__ __forceinline__ void cp_async16(void *smem_dst, const void *gsrc) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(smem_dst);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_1() { asm volatile("cp.async.wait_group 1;\n" ::: "memory"); }
 
 // After B1: tile meta + drop / kept counts (warp 0), in warp order.
 __device__ __forceinline__ void k1_tile_summary(const Params &p, const K1Tile &t, const K1WarpSum *wsum) {
@@ -383,72 +414,138 @@ __device__ __forceinline__ void k1_publish(K1WarpSum *wsum, unsigned long long f
   }
 }
 
+// One lane's 16 consecutive records: field check, running min / max of the field-valid offsets
+// (an inversion inside the lane shows up as an offset below the running max), entries, keys.
+// NAR: windows shorter than 2^32 ticks, so offsets are compared and packed in 32 bits.
+template <bool NAR>
+__device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool is_win, const int4 *raw,
+                                        const unsigned short *capS, int sub0, unsigned long long (&e)[kPerLane],
+                                        unsigned (&kp)[kPerLane], unsigned long long &first,
+                                        unsigned long long &last, bool &has, bool &viol, unsigned &kept) {
+  const int lane = threadIdx.x & 31;
+  unsigned mn = ~0u, mx = 0u, hiacc = 0u;
+  unsigned long long mn64 = ~0ull, mx64 = 0ull;
+  bool hv = false, bad = false;
+#pragma unroll
+  for (int k = 0; k < kPerLane; ++k) {
+    const int i = lane * kPerLane + k;
+    const int4 v = raw[lane * kPerLane + (k ^ (lane & 7))];
+    const unsigned b = (unsigned)v.z, lvl = (unsigned)v.w & 0xFFFFu, c = (unsigned)v.w >> 16;
+    const unsigned capb = capS[b < p.nb ? b : 0u];
+    const bool valid = (sub0 + i < t.n) & (b < p.nb) & (c == capb) & (lvl <= c);
+    const unsigned long long off = (unsigned long long)(rec_ts(v) - t.lo);
+    hv |= valid;
+    if (NAR) {
+      const unsigned o = (unsigned)off;
+      bad |= valid & (o < mx);
+      mx = max(mx, valid ? o : 0u);
+      mn = min(mn, valid ? o : ~0u);
+      hiacc |= valid ? (unsigned)(off >> 32) : 0u;
+      // (o << 24) | (level << 8) | (buffer_id & 255), o < 2^32
+      const unsigned lo = __byte_perm(__byte_perm((unsigned)v.z, (unsigned)v.w, 0x0540), o, 0x4210);
+      e[k] = ((unsigned long long)(o >> 8) << 32) | lo;
+    } else {
+      bad |= valid & (off < mx64);
+      mx64 = max(mx64, valid ? off : 0ull);
+      mn64 = min(mn64, valid ? off : ~0ull);
+      e[k] = (off << 24) | ((unsigned long long)lvl << 8) | (b & (kBin - 1));
+    }
+    const bool keep = valid & is_win;
+    kept += keep;
+    kp[k] = (keep ? (b >> kBinLog) : kNoKey) << 16;
+  }
+  if (NAR) {
+    bad |= hv & ((hiacc != 0u) | ((unsigned long long)mx >= t.wlen));
+    first = mn;
+    last = mx;
+  } else {
+    bad |= hv & (mx64 >= t.wlen);
+    first = mn64;
+    last = mx64;
+  }
+  has = hv;
+  viol = bad;
+}
+
+#ifdef RTM_PHASE_TIMING
+// thread 0's view of a persistent kernel's per-tile phases (cycles), summed into p.dbg[slot]
+#define PTM(slot_)                                                       \
+  do {                                                                   \
+    if (threadIdx.x == 0 && p.dbg) {                                     \
+      const long long t1_ = clock64();                                   \
+      atomicAdd(p.dbg + (slot_), (unsigned long long)(t1_ - pt_));       \
+      pt_ = t1_;                                                         \
+    }                                                                    \
+  } while (0)
+#else
+#define PTM(slot_) \
+  do {             \
+  } while (0)
+#endif
+
 __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
-  __shared__ K1WarpSum wsum[kK1Warps];
+  __shared__ K1WarpSum wsum[2][kK1Warps];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
   const unsigned nbins = p.nbins;
-  unsigned short *wt = reinterpret_cast<unsigned short *>(smem + (size_t)kTileS * 16);
-  unsigned short *wb = reinterpret_cast<unsigned short *>(smem + (size_t)kTileS * 16 + k1_vec_bytes(nbins));
-  unsigned short *capS = reinterpret_cast<unsigned short *>(smem + (size_t)kTileS * 16 + 2 * k1_vec_bytes(nbins));
-  unsigned short *myt = wt + (size_t)warp * nbins;
-  unsigned short *myb = wb + (size_t)warp * nbins;
-  int4 *raw = reinterpret_cast<int4 *>(smem) + warp * kSub;                          // this warp's slot
-  unsigned short *mat = reinterpret_cast<unsigned short *>(raw);                      // aliases the slot
-  unsigned long long *sbuf = reinterpret_cast<unsigned long long *>(smem);            // CTA permute buffer
+  const size_t vb = k1_vec_bytes(nbins);
+  unsigned char *tail = smem + (size_t)kTileS * 16;
+  unsigned short *wt2 = reinterpret_cast<unsigned short *>(tail);            // [2][8][nbins]
+  unsigned short *myb = reinterpret_cast<unsigned short *>(tail + 2 * vb) + (size_t)warp * nbins;
+  TileDesc *dsm = reinterpret_cast<TileDesc *>(tail + 3 * vb) + warp * 2;     // this warp's [2]
+  unsigned short *capS = reinterpret_cast<unsigned short *>(tail + 3 * vb + (size_t)kK1Warps * 2 * sizeof(TileDesc));
+  int4 *raw = reinterpret_cast<int4 *>(smem) + warp * kSub;  // this warp's slot
+  // after the scan the slot holds the count rows: 48 B per bin = 32 u8 lane counters (later the
+  // exclusive in-word prefixes) + 8 u16 word bases
+  unsigned char *rows = reinterpret_cast<unsigned char *>(raw);
   for (unsigned i = threadIdx.x; i < p.nb; i += kK1Threads) capS[i] = __ldg(p.cap + i);
-  __syncthreads();
   const unsigned n_tiles = p.rts[p.W + 2];
   const int sub0 = warp * kSub;
-  for (unsigned tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
-    const K1Tile t = k1_tile(p, tile);
-    const bool is_win = t.g.window >= 0;
-    const int4 *src = reinterpret_cast<const int4 *>(p.s) + t.start + sub0;
-    // stage the sub-tile: record i at 16-byte slot 16(i>>4) + ((i&15) ^ ((i>>4)&7))
+  // async prefetch of a tile (descriptor already in dsm[slot]): this warp's 512 raw records,
+  // record i to the 16-byte slot 16(i>>4) + ((i&15) ^ ((i>>4)&7))
+  auto prefetch_raw = [&](const TileDesc &d) {
+    const int4 *src = reinterpret_cast<const int4 *>(p.s) + d.start + sub0;
+    const int m = d.n - sub0;
 #pragma unroll
-    for (int h = 0; h < kPerLane; h += 4) {
-      int4 v[4];
-#pragma unroll
-      for (int jj = 0; jj < 4; ++jj) {
-        const int i = (h + jj) * 32 + lane;
-        v[jj] = sub0 + i < t.n ? ld_stream(src + i) : make_int4(0, 0, 0, 0);
-      }
-#pragma unroll
-      for (int jj = 0; jj < 4; ++jj) {
-        const int i = (h + jj) * 32 + lane;
-        raw[(i & ~15) | ((i & 15) ^ ((i >> 4) & 7))] = v[jj];
-      }
+    for (int j = 0; j < kPerLane; ++j) {
+      const int i = j * 32 + lane;
+      if (i < m) cp_async16(raw + ((i & ~15) | ((i & 15) ^ ((i >> 4) & 7))), src + i);
     }
+  };
+  unsigned tile = blockIdx.x;
+  if (tile < n_tiles) {
+    if (lane < 3) cp_async16(reinterpret_cast<int4 *>(dsm) + lane, reinterpret_cast<const int4 *>(p.tdesc + tile) + lane);
+    cp_async_commit();
+    cp_async_wait_all();
     __syncwarp();
+    prefetch_raw(dsm[0]);
+  }
+  cp_async_commit();
+  __syncthreads();  // capacity table
+  long long pt_ = clock64();
+  (void)pt_;
+  for (unsigned par = 0; tile < n_tiles; tile += gridDim.x, par ^= 1) {
+    const unsigned nxt = tile + gridDim.x;
+    const K1Tile t = k1_tile_from(dsm[par], tile);
+    const bool is_win = t.g.window >= 0;
+    unsigned short *wt = wt2 + (size_t)par * (vb / 2);
+    unsigned short *myt = wt + (size_t)warp * nbins;
+    __syncwarp();  // dsm[par] read by every lane before it is reused
+    if (nxt < n_tiles && lane < 3)
+      cp_async16(reinterpret_cast<int4 *>(dsm + (par ^ 1)) + lane, reinterpret_cast<const int4 *>(p.tdesc + nxt) + lane);
+    cp_async_commit();
+    cp_async_wait_1();  // this tile's raw records (the descriptor group may still be in flight)
+    __syncwarp();
+    PTM(1);
+    if (threadIdx.x == 0 && p.dbg) atomicAdd(p.dbg + 7, 1ull);
     unsigned long long e[kPerLane];
     unsigned kp[kPerLane];  // key << 16 | position within the warp's bin group
-    unsigned long long first = 0, last = 0;
-    bool has = false, viol = false;
+    unsigned long long first, last;
+    bool has, viol;
     unsigned kept = 0;
-#pragma unroll
-    for (int k = 0; k < kPerLane; ++k) {
-      const int i = lane * kPerLane + k;
-      const int4 v = raw[lane * kPerLane + (k ^ (lane & 7))];
-      const unsigned b = (unsigned)v.z, lvl = (unsigned)v.w & 0xFFFFu, c = (unsigned)v.w >> 16;
-      const unsigned capb = capS[b < p.nb ? b : 0u];
-      const bool valid = (sub0 + i < t.n) & (b < p.nb) & (c == capb) & (lvl <= c);
-      const unsigned long long off = (unsigned long long)(rec_ts(v) - t.lo);
-      if (valid) {
-        viol |= (off >= t.wlen) | (has & (off < last));
-        if (!has) first = off;
-        has = true;
-        last = off;
-      }
-      const bool keep = valid & is_win;
-      kept += keep;
-      const unsigned key = keep ? (b >> kBinLog) : kNoKey;
-      unsigned rank = 0;
-#pragma unroll
-      for (int q = 0; q < k; ++q) rank += (kp[q] >> 16) == key;
-      kp[k] = (key << 16) | rank;
-      e[k] = (off << 24) | ((unsigned long long)lvl << 8) | (b & (kBin - 1));
-    }
+    if (p.narrow && is_win) lm_scan<true>(p, t, is_win, raw, capS, sub0, e, kp, first, last, has, viol, kept);
+    else lm_scan<false>(p, t, is_win, raw, capS, sub0, e, kp, first, last, has, viol, kept);
     {  // order across lanes: my first vs the last of the nearest earlier lane with a valid record
       const unsigned hm = __ballot_sync(kFull, has);
       const unsigned lower = hm & lt;
@@ -460,53 +557,73 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
       last = l0;
       has = hm != 0;
     }
-    if (is_win) {  // per-(bin, lane) counts -> row prefix -> position within the warp's bin group
-      uint4 *m4 = reinterpret_cast<uint4 *>(mat);  // the raw slot is consumed (registers)
-      for (unsigned q = lane; q < nbins * 4; q += 32) m4[q] = make_uint4(0, 0, 0, 0);
+    PTM(2);
+    __syncwarp();  // every lane has consumed its raw records
+    if (is_win) {  // rank = (lane, bin) counter; position = rank + earlier lanes' counts of the bin
+      uint4 *r4 = reinterpret_cast<uint4 *>(rows);
+      for (unsigned q = lane; q < nbins * 3; q += 32) r4[q] = make_uint4(0, 0, 0, 0);
       __syncwarp();
-#pragma unroll
-      for (int k = 0; k < kPerLane; ++k)  // final count of (bin, lane) = last rank + 1 (program order)
-        if ((kp[k] >> 16) != kNoKey) mat[mat_idx(kp[k] >> 16, lane)] = (unsigned short)((kp[k] & 0xFFFFu) + 1);
-      __syncwarp();
-      for (unsigned b = lane; b < nbins; b += 32) {
-        uint4 *row = reinterpret_cast<uint4 *>(mat + b * 32);
-        unsigned run = 0;
-#pragma unroll
-        for (int cq = 0; cq < 4; ++cq) {
-          uint4 q = row[cq ^ ((b >> 1) & 3u)];
-          unsigned *w4 = reinterpret_cast<unsigned *>(&q);
-#pragma unroll
-          for (int x = 0; x < 4; ++x) {
-            const unsigned wv = w4[x], a = wv & 0xFFFFu, bb = wv >> 16;
-            w4[x] = run | ((run + a) << 16);
-            run += a + bb;
-          }
-          row[cq ^ ((b >> 1) & 3u)] = q;
-        }
-        myt[b] = (unsigned short)run;
-      }
-      __syncwarp();
-#pragma unroll
-      for (int k = 0; k < kPerLane; ++k)
-        if ((kp[k] >> 16) != kNoKey) kp[k] += mat[mat_idx(kp[k] >> 16, lane)];
-    }
-    k1_publish(wsum, first, last, has, viol, kept);
-    __syncthreads();  // B1: summaries + bin totals published; every raw slot consumed
-    if (warp == 0) k1_tile_summary(p, t, wsum);
-    if (is_win) {
-      const unsigned total = k1_bin_bases(p, tile, wt, myb);
 #pragma unroll
       for (int k = 0; k < kPerLane; ++k) {
         const unsigned key = kp[k] >> 16;
-        if (key != kNoKey) sbuf[myb[key] + (kp[k] & 0xFFFFu)] = e[k];
+        if (key != kNoKey) {
+          unsigned char *ctr = rows + key * 48 + lane;
+          const unsigned r = *ctr;
+          *ctr = (unsigned char)(r + 1);
+          kp[k] |= r;
+        }
       }
-      __syncthreads();  // B2: the tile is bin-sorted in shared memory
-      const uint4 *s4 = reinterpret_cast<const uint4 *>(sbuf);
-      uint4 *d4 = reinterpret_cast<uint4 *>(p.stage + (size_t)tile * kTileS);
-      for (unsigned q = threadIdx.x; q < (total + 1) / 2; q += kK1Threads) d4[q] = s4[q];
+      __syncwarp();
+      for (unsigned b = lane; b < nbins; b += 32) {  // one bin row per lane: byte-SIMD prefix
+        uint4 *row = reinterpret_cast<uint4 *>(rows + b * 48);
+        const uint4 q0 = row[0], q1 = row[1];
+        unsigned w[8] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w};
+        unsigned base[8];
+        unsigned run = 0;
+#pragma unroll
+        for (int x = 0; x < 8; ++x) {
+          const unsigned incl = w[x] * 0x01010101u;  // byte j = counts of lanes 4x .. 4x+j (<= 64)
+          base[x] = run;
+          run += incl >> 24;
+          w[x] = incl - w[x];
+        }
+        row[0] = make_uint4(w[0], w[1], w[2], w[3]);
+        row[1] = make_uint4(w[4], w[5], w[6], w[7]);
+        row[2] = make_uint4(base[0] | (base[1] << 16), base[2] | (base[3] << 16), base[4] | (base[5] << 16),
+                            base[6] | (base[7] << 16));
+        myt[b] = (unsigned short)run;
+      }
+      __syncwarp();
+      const unsigned short *rows16 = reinterpret_cast<const unsigned short *>(rows);
+#pragma unroll
+      for (int k = 0; k < kPerLane; ++k) {
+        const unsigned key = kp[k] >> 16;
+        if (key != kNoKey) kp[k] += rows[key * 48 + lane] + rows16[key * 24 + 16 + (lane >> 2)];
+      }
+      __syncwarp();  // the slot is free again
     }
-    __syncthreads();  // B3: shared buffers free for the next tile
+    PTM(3);
+    // the next tile's records stream into the slot while this tile is published and written out
+    cp_async_wait_all();
+    __syncwarp();
+    if (nxt < n_tiles) prefetch_raw(dsm[par ^ 1]);
+    cp_async_commit();
+    k1_publish(wsum[par], first, last, has, viol, kept);
+    __syncthreads();  // B1 (the only CTA barrier per tile): summaries + bin totals of this tile
+    PTM(4);
+    if (warp == 0) k1_tile_summary(p, t, wsum[par]);
+    if (is_win) {
+      k1_bin_bases(p, tile, wt, myb);
+      unsigned long long *dst = p.stage + (size_t)tile * kTileS;
+#pragma unroll
+      for (int k = 0; k < kPerLane; ++k) {
+        const unsigned key = kp[k] >> 16;
+        if (key != kNoKey) dst[myb[key] + (kp[k] & 0xFFFFu)] = e[k];
+      }
+    }
+    PTM(5);
   }
+  cp_async_wait_all();
 }
 
 __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
@@ -1420,7 +1537,7 @@ void launch_regions(const Params &p, cudaStream_t st) {
 void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
   const unsigned nr = p.W + 2;
   const unsigned blocks = nr < 4096 ? nr : 4096;
-  if (p.n_tiles_s) k_fill_tile_regions<<<blocks, 64, 0, st>>>(p.rts, const_cast<uint32_t *>(p.tile_reg_s), nr);
+  if (p.n_tiles_s) k_fill_tile_desc<<<blocks, 64, 0, st>>>(p);
   if (p.n_tiles_e) k_fill_tile_regions<<<blocks, 64, 0, st>>>(p.rte, const_cast<uint32_t *>(p.tile_reg_e), nr);
 }
 
