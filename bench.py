@@ -40,29 +40,51 @@ def _peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    """SM clocks + throttle reasons sampled DURING the timed region (NVML every 10 ms; nvidia-smi
+    fallback).  Reasons follow nvidia-smi's clocks_event_reasons names."""
 
-    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+    REASONS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+               "hw_power_brake_slowdown": 0x80, "sw_power_cap": 0x4}
 
-    def __init__(self, index: int):
+    def __init__(self, index: int, period: float = 0.01):
         self.index = index
-        self.rows = []
+        self.period = period
+        self.rows = []  # (sm_mhz, max_mhz, reason_mask)
         self._stop = threading.Event()
         self._t = None
+        self._nvml = None
+        try:
+            import pynvml
+
+            pynvml.nvmlInit()
+            self._nvml = pynvml
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(index)
+        except Exception:
+            self._nvml = None
+
+    def _sample(self):
+        if self._nvml is not None:
+            n = self._nvml
+            sm = n.nvmlDeviceGetClockInfo(self._h, n.NVML_CLOCK_SM)
+            mx = n.nvmlDeviceGetMaxClockInfo(self._h, n.NVML_CLOCK_SM)
+            rs = n.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+            return float(sm), float(mx), int(rs)
+        q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.sw_power_cap,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.hw_thermal_slowdown")
+        out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}", "--format=csv,noheader,nounits"],
+                             capture_output=True, text=True, timeout=5).stdout
+        p = [x.strip() for x in out.strip().split(",")]
+        bits = (0x8, 0x4, 0x20, 0x40)
+        mask = sum(b for b, v in zip(bits, p[2:6]) if v == "Active")
+        return float(p[0]), float(p[1]), mask
 
     def _run(self):
         while not self._stop.is_set():
             try:
-                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
-                parts = [x.strip() for x in out.stdout.strip().split(",")]
-                if len(parts) >= 7:
-                    self.rows.append(parts)
+                self.rows.append(self._sample())
             except Exception:
                 pass
-            self._stop.wait(0.2)
+            self._stop.wait(self.period)
 
     def __enter__(self):
         self._t = threading.Thread(target=self._run, daemon=True)
@@ -75,14 +97,11 @@ class ClockSampler:
 
     def summary(self):
         if not self.rows:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
-        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in self.rows for i in range(4) if "Active" in r[3 + i]
-                          and "Not" not in r[3 + i]})
-        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows)}
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [r[0] for r in self.rows]
+        reasons = sorted({k for r in self.rows for k, bit in self.REASONS.items() if r[2] & bit})
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": max(r[1] for r in self.rows), "reasons": reasons,
+                "samples": len(self.rows), "source": "nvml" if self._nvml is not None else "nvidia-smi"}
 
 
 # ---------------------------------------------------------------------------------------------
@@ -205,7 +224,10 @@ def run_native(args):
     # correctness guard on the timed configuration: every record accounted for
     S = res["summary"]
     assert int(S["n_samples"].sum() + S["n_events"].sum() + S["n_dropped"].sum()) == n_rec * world
+    from paper_conf_micro_mosallaeii024_b200 import _native
+
     mon.profile(True)
+    n_launch0 = _native.lib().rtm_kernel_launches()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         if dist:
@@ -221,6 +243,7 @@ def run_native(args):
         if dist:
             dist.barrier()
     ms = ev0.elapsed_time(ev1)
+    n_launches = int(_native.lib().rtm_kernel_launches() - n_launch0)
     prof = mon.profile_read()
     mon.profile(False)
     if dist:
@@ -263,24 +286,27 @@ def run_native(args):
         if dist:
             dist.destroy_process_group()
         return
-    # ---- roofline of the dominant kernel (largest share of the step)
+    # ---- roofline of the dominant kernel: largest share of the step among the kernels on the
+    # critical (main) stream; k_events runs on a side stream overlapped with the partition + fold
     peaks = _peaks()
     hbm = float(peaks.get("hbm_gbs", 6650.0))
-    dom = max((k for k in prof if prof[k]["launches"]), key=lambda k: prof[k]["total_ms"])
-    d = prof[dom]
-    hbm_kernel = "k_partition"
-    hk = prof[hbm_kernel]
-    achieved_gbs = (hk["algo_bytes"] / hk["launches"]) / (hk["total_ms"] / hk["launches"] / 1e3) / 1e9
     step_ms = ms / args.steps
     shares = {k: round(prof[k]["total_ms"] / args.steps / step_ms, 4) for k in prof if prof[k]["launches"]}
-    launches = sum(prof[k]["launches"] for k in prof)
+    main_stream = [k for k in prof if prof[k]["launches"] and prof[k]["algo_bytes"] and k != "k_events"]
+    dom = max(main_stream, key=lambda k: prof[k]["total_ms"])
+    dk = prof[dom]
+    achieved_gbs = (dk["algo_bytes"] / dk["launches"]) / (dk["total_ms"] / dk["launches"] / 1e3) / 1e9
     traffic = None
-    tp = os.path.join(ROOT, "profiles", "r01_partition_traffic.json")
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get("bytes_per_launch")
+            allt = json.load(open(tp)).get("all", {})
+            traffic = next((v for k, v in allt.items() if k == dom or k.startswith(dom + "_")), None)
         except Exception:
             traffic = None
+    per_kernel = {k: {"achieved_gbs": round((prof[k]["algo_bytes"] / prof[k]["launches"]) /
+                                            (prof[k]["total_ms"] / prof[k]["launches"] / 1e3) / 1e9, 1),
+                      "share": shares[k]} for k in main_stream}
     path_gbs = 16.0 * n_rec / (step_ms / 1e3) / 1e9
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
@@ -296,14 +322,15 @@ def run_native(args):
                    "n_buffers": int(len(owner)), "records_per_gpu": n_rec, "windows": W, "k": wl.k,
                    "hang_windows": wl.hang_windows, "l2": "inputs (1.6 GB/GPU) larger than L2; no flush",
                    "parallelism": f"owner-component shards x{world}" if world > 1 else "single GPU"},
-        "roofline": {"bound": "hbm", "kernel": hbm_kernel, "achieved": achieved_gbs, "peak": hbm, "unit": "GB/s",
-                     "frac": achieved_gbs / hbm, "traffic": traffic, "peak_source": "MEASURED_PEAKS.json hbm_gbs",
-                     "path_achieved": path_gbs, "path_frac": path_gbs / hbm,
-                     "dominant_kernel": dom, "dominant_share": shares.get(dom)},
+        "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved_gbs, "peak": hbm, "unit": "GB/s",
+                     "frac": achieved_gbs / hbm, "traffic": traffic,
+                     "algo_bytes_per_launch": dk["algo_bytes"] / dk["launches"],
+                     "peak_source": "MEASURED_PEAKS.json hbm_gbs (burst copy)", "share": shares.get(dom),
+                     "path_achieved": path_gbs, "path_frac": path_gbs / hbm, "per_kernel": per_kernel},
         "kernel_share": shares,
         "cpu_baseline": cpu,
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 16 * n_rec, "d2h_bytes_per_step": d2h},
-        "gpu_launches": launches,
+        "gpu_launches": n_launches,
         "clocks": clk.summary(),
         "wall_s_timed": t_wall,
     }
@@ -315,7 +342,7 @@ def run_native(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -189,6 +189,9 @@ rtm_status rtm_profile_read(rtm_ctx *ctx, rtm_kernel_time *out, uint32_t cap, ui
 const char *rtm_status_str(rtm_status s);
 /* Build identification string ("librtm sm_100a ..."). */
 const char *rtm_version(void);
+/* Kernel launches issued by this library in this process so far (all contexts, all streams).
+ * Monotone; callers take differences around a region to count the kernels it launched. */
+uint64_t rtm_kernel_launches(void);
 
 #ifdef __cplusplus
 }

@@ -52,7 +52,8 @@ class KernelTime(ctypes.Structure):
 # every symbol include/rtm.h declares (checked by tests/test_abi.py)
 EXPORTS = ("rtm_create", "rtm_destroy", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers",
            "rtm_progress", "rtm_hang_check", "rtm_buffer_stats", "rtm_window_results", "rtm_window_reduce_local",
-           "rtm_merge", "rtm_profile", "rtm_profile_read", "rtm_status_str", "rtm_version")
+           "rtm_merge", "rtm_profile", "rtm_profile_read", "rtm_status_str", "rtm_version",
+           "rtm_kernel_launches")
 
 _lib = None
 
@@ -90,6 +91,8 @@ def lib():
     L.rtm_status_str.restype = ctypes.c_char_p
     L.rtm_version.argtypes = []
     L.rtm_version.restype = ctypes.c_char_p
+    L.rtm_kernel_launches.argtypes = []
+    L.rtm_kernel_launches.restype = ctypes.c_uint64
     _lib = L
     return L
 

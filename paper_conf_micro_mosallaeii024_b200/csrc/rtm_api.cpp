@@ -385,8 +385,10 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   launch_events(p, c->st2);
   if (c->prof) prof_end_on(c, c->st2);
   CK(cudaEventRecord(c->ev_join, c->st2));
-  LAUNCH(KT_PARTITION, (uint64_t)ns * 16, launch_partition(p, c->n_sms, c->st));
-  LAUNCH(KT_FOLD, 0, launch_fold(p, c->n_sms, c->st));
+  // algorithmic bytes: partition = 16 B record in + 8 B compacted entry out per
+  // sample; fold = the 8 B entry per sample
+  LAUNCH(KT_PARTITION, (uint64_t)ns * 24, launch_partition(p, c->n_sms, c->st));
+  LAUNCH(KT_FOLD, (uint64_t)ns * 8, launch_fold(p, c->n_sms, c->st));
   CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
   LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
   LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
@@ -483,6 +485,8 @@ const char *rtm_status_str(rtm_status s) {
 }
 
 const char *rtm_version(void) { return "librtm 0.1 sm_100a (window-snapshot reducer)"; }
+
+uint64_t rtm_kernel_launches(void) { return (uint64_t)kernel_launches(); }
 
 rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   if (!cfg || !out) return RTM_E_INVALID;

@@ -137,6 +137,7 @@ void launch_progress(const Params &p, cudaStream_t st);
 uint64_t pack_bytes(const Params &p);
 void launch_pack(const Params &p, void *pack, cudaStream_t st);
 void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStream_t st);
+unsigned long long kernel_launches();  // kernels launched by this library in this process
 void configure_kernels_once();  // opt-in shared-memory limits, once per device
 size_t fold_smem_bytes();
 size_t partition_smem_bytes(uint32_t nbins, uint32_t nb);

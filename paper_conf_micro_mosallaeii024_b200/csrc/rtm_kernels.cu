@@ -7,6 +7,8 @@
 
 #include <type_traits>
 
+#include <atomic>
+
 #include "rtm_internal.h"
 
 namespace rtm {
@@ -1510,6 +1512,10 @@ __global__ void k_merge_tables(Params p, const unsigned char *g, unsigned world,
 // ============================================================================================
 // launchers
 // ============================================================================================
+std::atomic<unsigned long long> g_kernel_launches{0};
+inline void count_launch() { g_kernel_launches.fetch_add(1, std::memory_order_relaxed); }
+unsigned long long kernel_launches() { return g_kernel_launches.load(std::memory_order_relaxed); }
+
 size_t fold_smem_bytes() { return sizeof(FoldSmem) * kFoldWarps; }
 size_t partition_smem_bytes(uint32_t nbins, uint32_t nb) {
   return nbins <= kLmMaxBins ? k1_smem_lm(nbins, nb) : k1_smem_mx(nbins);
@@ -1525,20 +1531,20 @@ void launch_split(const Params &p, bool samples, long long *outB, cudaStream_t s
   const unsigned warps = p.W + 1;
   const unsigned threads = 128;
   const unsigned blocks = (warps * 32 + threads - 1) / threads;
-  if (samples) k_split<true><<<blocks, threads, 0, st>>>(p, outB);
-  else k_split<false><<<blocks, threads, 0, st>>>(p, outB);
+  if (samples) { k_split<true><<<blocks, threads, 0, st>>>(p, outB); count_launch(); }
+  else { k_split<false><<<blocks, threads, 0, st>>>(p, outB); count_launch(); }
 }
 
 void launch_regions(const Params &p, cudaStream_t st) {
-  k_regions<<<1, 1024, 0, st>>>(const_cast<long long *>(p.Bs), p.ns, p.W, const_cast<uint32_t *>(p.rts), kTileS);
-  k_regions<<<1, 1024, 0, st>>>(const_cast<long long *>(p.Be), p.ne, p.W, const_cast<uint32_t *>(p.rte), kTileE);
+  { k_regions<<<1, 1024, 0, st>>>(const_cast<long long *>(p.Bs), p.ns, p.W, const_cast<uint32_t *>(p.rts), kTileS); count_launch(); }
+  { k_regions<<<1, 1024, 0, st>>>(const_cast<long long *>(p.Be), p.ne, p.W, const_cast<uint32_t *>(p.rte), kTileE); count_launch(); }
 }
 
 void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
   const unsigned nr = p.W + 2;
   const unsigned blocks = nr < 4096 ? nr : 4096;
-  if (p.n_tiles_s) k_fill_tile_desc<<<blocks, 64, 0, st>>>(p);
-  if (p.n_tiles_e) k_fill_tile_regions<<<blocks, 64, 0, st>>>(p.rte, const_cast<uint32_t *>(p.tile_reg_e), nr);
+  if (p.n_tiles_s) { k_fill_tile_desc<<<blocks, 64, 0, st>>>(p); count_launch(); }
+  if (p.n_tiles_e) { k_fill_tile_regions<<<blocks, 64, 0, st>>>(p.rte, const_cast<uint32_t *>(p.tile_reg_e), nr); count_launch(); }
 }
 
 void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
@@ -1550,16 +1556,16 @@ void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
     if (per_sm < 1) per_sm = 1;
     unsigned grid = (unsigned)(n_sms * per_sm);
     if (grid > p.n_tiles_s) grid = p.n_tiles_s;
-    k_partition_lm<<<grid, kK1Threads, sm, st>>>(p);
+    { k_partition_lm<<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
   } else {
-    k_partition_mx<<<p.n_tiles_s, kK1Threads, sm, st>>>(p);
+    { k_partition_mx<<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
   }
 }
 
 void launch_events(const Params &p, cudaStream_t st) {
   if (!p.n_tiles_e) return;
   const size_t sm = (size_t)2 * p.nk * 4 + (p.ncw <= 2048 ? (size_t)p.ncw * 4 : 0);
-  k_events<<<p.n_tiles_e, kK3Threads, sm, st>>>(p);
+  { k_events<<<p.n_tiles_e, kK3Threads, sm, st>>>(p); count_launch(); }
 }
 
 void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
@@ -1572,28 +1578,28 @@ void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
   const unsigned need = (units + kFoldWarps - 1) / kFoldWarps;
   if (grid > need) grid = need;
   if (grid == 0) grid = 1;
-  k_fold<<<grid, kFoldWarps * 32, sm, st>>>(p);
+  { k_fold<<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
 }
 
 void launch_order_check(const Params &p, cudaStream_t st) {
-  if (p.n_tiles_s) k_order_check<<<1, 1024, 0, st>>>(p.smeta, p.n_tiles_s, p.rts + p.W + 2, p.status, 1u);
-  if (p.n_tiles_e) k_order_check<<<1, 1024, 0, st>>>(p.emeta, p.n_tiles_e, p.rte + p.W + 2, p.status, 2u);
+  if (p.n_tiles_s) { k_order_check<<<1, 1024, 0, st>>>(p.smeta, p.n_tiles_s, p.rts + p.W + 2, p.status, 1u); count_launch(); }
+  if (p.n_tiles_e) { k_order_check<<<1, 1024, 0, st>>>(p.emeta, p.n_tiles_e, p.rte + p.W + 2, p.status, 2u); count_launch(); }
 }
 
 void launch_topk(const Params &p, cudaStream_t st) {
-  if (p.n_elig == p.nb) k_topk<true><<<p.W, kTopkThreads, topk_smem_bytes(p.nb), st>>>(p);
-  else k_topk<false><<<p.W, kTopkThreads, topk_smem_bytes(p.n_elig), st>>>(p);
+  if (p.n_elig == p.nb) { k_topk<true><<<p.W, kTopkThreads, topk_smem_bytes(p.nb), st>>>(p); count_launch(); }
+  else { k_topk<false><<<p.W, kTopkThreads, topk_smem_bytes(p.n_elig), st>>>(p); count_launch(); }
 }
 
 void launch_hang(const Params &p, cudaStream_t st) {
   const unsigned threads = 256;
   const size_t n = (size_t)p.W * p.ncw + p.nc;
-  k_hang<<<(unsigned)((n + threads - 1) / threads), threads, 0, st>>>(p);
+  { k_hang<<<(unsigned)((n + threads - 1) / threads), threads, 0, st>>>(p); count_launch(); }
 }
 
 void launch_progress(const Params &p, cudaStream_t st) {
   const unsigned comp_blocks = (p.nc + 255) / 256 < 256 ? (p.nc + 255) / 256 : 256;
-  k_progress<<<p.nk + comp_blocks, 256, 0, st>>>(p);
+  { k_progress<<<p.nk + comp_blocks, 256, 0, st>>>(p); count_launch(); }
 }
 
 uint64_t pack_bytes(const Params &p) { return pack_layout(p).total; }
@@ -1632,8 +1638,8 @@ void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStr
   while (P < world * p.k) P <<= 1;
   const size_t sm = (size_t)P * 16;
   if (sm > 48 * 1024) cudaFuncSetAttribute(k_merge_windows, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-  k_merge_windows<<<p.W, 256, sm, st>>>(p, static_cast<const unsigned char *>(gathered), world, stride);
-  k_merge_tables<<<256, 256, 0, st>>>(p, static_cast<const unsigned char *>(gathered), world, stride);
+  { k_merge_windows<<<p.W, 256, sm, st>>>(p, static_cast<const unsigned char *>(gathered), world, stride); count_launch(); }
+  { k_merge_tables<<<256, 256, 0, st>>>(p, static_cast<const unsigned char *>(gathered), world, stride); count_launch(); }
 }
 
 }  // namespace rtm

@@ -86,3 +86,13 @@ def test_product_never_touches_the_oracle():
                 src = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in src and "from oracle" not in src, f
                 assert "liboracle" not in src and "oracle.h" not in src, f
+
+
+def test_kernel_launch_counter_is_monotone_without_gpu():
+    """rtm_kernel_launches needs no device: it only reads the library's launch counter."""
+    from paper_conf_micro_mosallaeii024_b200 import _native
+
+    L = _native.lib()
+    a = L.rtm_kernel_launches()
+    b = L.rtm_kernel_launches()
+    assert b >= a >= 0

@@ -1,6 +1,7 @@
 """Summarise an ncu launch list (CSV) and a --set full report into markdown for profiles/."""
 import csv
 import json
+import os
 import subprocess
 import sys
 
@@ -50,6 +51,6 @@ for row in r[2:]:
 lines.append("")
 lines.append("Units row: " + ", ".join(f"{w}={r[1][H.index(w)]}" for w in want if w in H))
 open(out_md, "w").write("\n".join(lines) + "\n")
-json.dump({"kernel": "k_partition", "bytes_per_launch": traffic.get("k_partition"), "all": traffic, "source": rep},
-          open(out_md.replace("_summary.md", "_partition_traffic.json"), "w"), indent=1)
+json.dump({"what": "dram__bytes_read.sum + dram__bytes_write.sum per launch (ncu --set full, C2)", "all": traffic,
+           "source": rep, "tag": tag}, open(os.path.join(os.path.dirname(out_md), "traffic.json"), "w"), indent=1)
 print("\n".join(lines))
