@@ -841,6 +841,7 @@ struct FoldSmem {
   unsigned n[kBin];                // kept samples this window (0: untouched, other fields stale)
   unsigned seg_end[32];            // flattened segment table of the current tile group
   unsigned long long seg_ptr[32];
+  unsigned char owner[kBin];       // duplicate detection: last lane that wrote each buffer slot
 };
 
 // One chunk of <= 32 consecutive records (ingest order) of one (window, bin) unit.  Records of
@@ -854,9 +855,19 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
   const unsigned lid = (unsigned)(e & (kBin - 1));
   const unsigned lvl = (unsigned)(e >> 8) & 0xFFFFu;
   const unsigned long long off = e >> 24;
-  const unsigned am = __ballot_sync(kFull, act);
-  const unsigned mb = match_bits<kBinLog>(lid);  // all lanes (ballots are collective)
-  const unsigned peers = act ? (mb & am) : (1u << lane);
+  // Peers = lanes holding the same buffer.  Most lanes hold a buffer no other lane of the chunk
+  // holds, and __match_any_sync costs ~2 cycles of SM throughput per DISTINCT key in the warp
+  // (tools/microbench.cu), so duplicates are found first through a shared-memory slot per
+  // buffer (a lane whose write lost has a peer and tells the winner), and only duplicate lanes
+  // present their real key to the match; the rest share one sentinel key.
+  if (act) S.owner[lid] = (unsigned char)lane;
+  __syncwarp();
+  const unsigned win = act ? S.owner[lid] : (unsigned)lane;
+  const bool lost = win != (unsigned)lane;
+  const unsigned told = __reduce_or_sync(kFull, lost ? (1u << win) : 0u);
+  const bool dup = lost | ((told >> lane) & 1u);
+  const unsigned mk = __match_any_sync(kFull, dup ? lid : 0xFFFFFFFFu);
+  const unsigned peers = dup ? mk : (1u << lane);
   const unsigned lower = peers & lt;
   const int pred = lower ? 31 - __clz(lower) : lane;
   const unsigned rank = __popc(lower);
@@ -901,7 +912,7 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
   __syncwarp();
 }
 
-__global__ void __launch_bounds__(kFoldWarps * 32) k_fold(Params p) {
+__global__ void __launch_bounds__(kFoldWarps * 32, 6) k_fold(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   FoldSmem &S = reinterpret_cast<FoldSmem *>(smem)[threadIdx.x >> 5];
   const int lane = threadIdx.x & 31;

@@ -64,6 +64,23 @@ __global__ void k_popc_alu(unsigned *out, unsigned seed) {
   out[blockIdx.x * blockDim.x + threadIdx.x] = acc;
 }
 
+// MATCH restricted to a few lanes holding few distinct keys (the fold's duplicate lanes)
+template <int ACTIVE_EVERY, int NKEYS>
+__global__ void k_match_sparse(unsigned *out, unsigned seed) {
+  unsigned x = seed ^ threadIdx.x, acc = 0;
+  const unsigned lane = threadIdx.x & 31;
+  const unsigned mask = __ballot_sync(0xFFFFFFFFu, lane % ACTIVE_EVERY == 0);
+  if (lane % ACTIVE_EVERY == 0) {
+#pragma unroll 8
+    for (int i = 0; i < ITERS; ++i) {
+      unsigned key = (x >> 3) % NKEYS;
+      acc += __match_any_sync(mask, key);
+      x = x * 1664525u + 1013904223u;
+    }
+  }
+  out[blockIdx.x * blockDim.x + threadIdx.x] = acc;
+}
+
 template <int BITS>
 __device__ __forceinline__ unsigned match_ballot(unsigned key) {
   unsigned m = 0xFFFFFFFFu;
@@ -127,6 +144,11 @@ int main() {
     run("match_ball9", k_match_ballot9, w, 1);
     run("match_any", k_match, w, 1);
     run("match_dep", k_match_dep, w, 1);
+    run("m_all_2k", k_match_sparse<1, 2>, w, 1);
+    run("m_all_8k", k_match_sparse<1, 8>, w, 1);
+    run("m_8lane_2k", k_match_sparse<4, 2>, w, 1);
+    run("m_4lane_2k", k_match_sparse<8, 2>, w, 1);
+    run("m_4lane_4k", k_match_sparse<8, 4>, w, 1);
     run("ballot", k_ballot, w, 1);
     run("shfl_idx", k_shfl, w, 1);
     run("sts_u8", k_sts8, w, 1);
