@@ -12,6 +12,7 @@ uses PyTorch for device memory, streams and ``torch.distributed`` plumbing.
 from __future__ import annotations
 
 import ctypes
+from collections.abc import Mapping
 
 import numpy as np
 
@@ -124,7 +125,7 @@ class Monitor:
             N.check(N.lib().rtm_window_reduce(self._h, t_end.ctypes.data, W, summ.ctypes.data), "rtm_window_reduce")
         self._keep = []
         self.W = W
-        return self.results(W)
+        return LazyResults(self, W, summ)
 
     def results(self, W=None):
         """All per-window results of the last batch (one rtm_window_results call)."""
@@ -195,6 +196,32 @@ class Monitor:
 
 
 _cudart = None
+
+
+class LazyResults(Mapping):
+    """The mapping Monitor.window_reduce returns: "summary" is filled by the call itself; the
+    other per-window arrays ("topk", "topk_n", "progress") are copied out of the library on first
+    access (one rtm_window_results call), so a caller that only needs the summaries pays no host
+    copy of the top-k / progress tables.  Valid until the next window_reduce."""
+
+    _KEYS = ("summary", "topk", "topk_n", "progress")
+
+    def __init__(self, mon, W, summary):
+        self._mon, self._W = mon, W
+        self._d = {"summary": summary}
+
+    def __getitem__(self, key):
+        if key not in self._KEYS:
+            raise KeyError(key)
+        if key not in self._d:
+            self._d.update(self._mon.results(self._W))
+        return self._d[key]
+
+    def __iter__(self):
+        return iter(self._KEYS)
+
+    def __len__(self):
+        return len(self._KEYS)
 
 
 def _copy_from_ptr(dst_tensor, src_ptr: int, nbytes: int):

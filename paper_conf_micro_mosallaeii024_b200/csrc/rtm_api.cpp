@@ -62,16 +62,17 @@ struct rtm_ctx {
   DevBuf s_own, e_own;              // internal concatenation
   uint64_t s_own_n = 0, e_own_n = 0;
   // per-call workspaces
-  DevBuf T, Bs, Be, rts, rte, treg_s, treg_e, tdesc, soff, stage, smeta, emeta, lastlvl, win, kdelta, cdelta, active,
-      anyfull, hung, unit_ctr, status, topk, topk_n, prog, bstat, comps, pack, gathered;
+  DevBuf T, Bs, Be, rts, rte, treg_s, treg_e, tdesc, soff, stage, smeta, emeta, lastlvl, res, kdelta, cdelta, active,
+      anyfull, hung, unit_ctr, bstat, comps, pack, gathered;
   Pinned h_small, h_res;
   // results of the last call
   bool have = false;
   uint32_t W = 0;
   std::vector<rtm_window_summary> sum;
-  std::vector<unsigned long long> topk_h;
-  std::vector<uint32_t> topk_n_h;
-  std::vector<rtm_progress_entry> prog_h;
+  // results of the last call: views into the pinned host buffer h_res (valid until the next call)
+  const unsigned long long *topk_h = nullptr;
+  const uint32_t *topk_n_h = nullptr;
+  const rtm_progress_entry *prog_h = nullptr;
   std::vector<int64_t> t_end_h;
   // profiling
   bool prof = false;
@@ -213,15 +214,17 @@ void free_buf(DevBuf &b) {
 }
 
 rtm_status zero_state(rtm_ctx *c) {
-  CK(cudaMemsetAsync(c->carry[0].p, 0, (size_t)c->nb * 2, c->st));
-  CK(cudaMemsetAsync(c->carry[1].p, 0, (size_t)c->nb * 2, c->st));
-  CK(cudaMemsetAsync(c->run[0].p, 0, (size_t)c->nc * 4, c->st));
-  CK(cudaMemsetAsync(c->run[1].p, 0, (size_t)c->nc * 4, c->st));
-  CK(cudaMemsetAsync(c->kstart.p, 0, (size_t)c->nk * 8, c->st));
-  CK(cudaMemsetAsync(c->kend.p, 0, (size_t)c->nk * 8, c->st));
-  CK(cudaMemsetAsync(c->cstart.p, 0, (size_t)c->nc * 8, c->st));
-  CK(cudaMemsetAsync(c->cend.p, 0, (size_t)c->nc * 8, c->st));
-  CK(cudaStreamSynchronize(c->st));
+  ClearList cl;  // stream-ordered: the next call's kernels see the cleared state
+  cl.add(c->carry[0].p, (size_t)c->nb * 2);
+  cl.add(c->carry[1].p, (size_t)c->nb * 2);
+  cl.add(c->run[0].p, (size_t)c->nc * 4);
+  cl.add(c->run[1].p, (size_t)c->nc * 4);
+  cl.add(c->kstart.p, (size_t)c->nk * 8);
+  cl.add(c->kend.p, (size_t)c->nk * 8);
+  cl.add(c->cstart.p, (size_t)c->nc * 8);
+  cl.add(c->cend.p, (size_t)c->nc * 8);
+  launch_clear(cl, c->st);
+  CK(cudaGetLastError());
   c->cur = 0;
   c->t_prev = c->t0;
   c->have = false;
@@ -265,6 +268,31 @@ rtm_status append(rtm_ctx *c, std::vector<Chunk> &dev, DevBuf &own, uint64_t &ow
 
 // The local (per-rank) part of a reduce call.  On success the device result arrays hold this
 // rank's per-window results for n_windows windows.
+// Per-call results, one device buffer and one pinned host buffer of the same layout (a single
+// D2H copy per call): window fields | top-k | progress | top-k counts | status.
+struct ResLayout {
+  size_t win, topk, prog, topk_n, status, bytes;
+};
+ResLayout res_layout(const rtm_ctx *c, uint32_t W) {
+  ResLayout L;
+  L.win = 0;
+  L.topk = L.win + (size_t)kWinFields * W * 8;
+  L.prog = L.topk + (size_t)W * c->k * 8;
+  L.topk_n = L.prog + (size_t)W * c->nk * 5 * 8;
+  L.status = L.topk_n + (((size_t)W * 4 + 15) & ~(size_t)15);
+  L.bytes = L.status + 16;
+  return L;
+}
+void set_result_ptrs(rtm_ctx *c, uint32_t W, Params &p) {
+  const ResLayout L = res_layout(c, W);
+  char *d = (char *)c->res.p;
+  p.win = (unsigned long long *)(d + L.win);
+  p.topk = (unsigned long long *)(d + L.topk);
+  p.prog = (long long *)(d + L.prog);
+  p.topk_n = (uint32_t *)(d + L.topk_n);
+  p.status = (uint32_t *)(d + L.status);
+}
+
 rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p) {
   if (c->sticky) return (rtm_status)c->sticky;
   if (!t_end || W == 0) return RTM_E_INVALID;
@@ -330,44 +358,45 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   if (c->flags.cap < Wn * c->nbins * 4) {
     if ((s = ensure(c, c->flags, Wn * c->nbins * 4, true))) return s;
   }
-  if ((s = ensure(c, c->win, (size_t)kWinFields * Wn * 8))) return s;
+  if ((s = ensure(c, c->res, res_layout(c, W).bytes))) return s;
   if ((s = ensure(c, c->kdelta, Wn * c->nk * 2 * 4))) return s;
   if ((s = ensure(c, c->cdelta, (size_t)c->nc * 2 * 8))) return s;
   if ((s = ensure(c, c->active, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->anyfull, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->hung, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->unit_ctr, 8))) return s;
-  if ((s = ensure(c, c->status, 8))) return s;
-  if ((s = ensure(c, c->topk, Wn * c->k * 8))) return s;
-  if ((s = ensure(c, c->topk_n, Wn * 4))) return s;
-  if ((s = ensure(c, c->prog, Wn * c->nk * 5 * 8))) return s;
   if ((s = ensure(c, c->bstat, (size_t)c->nb * sizeof(rtm_buffer_stat)))) return s;
   if ((s = ensure(c, c->comps, (size_t)c->nc * sizeof(rtm_component_tasks)))) return s;
 
-  CK(cudaMemsetAsync(c->win.p, 0, (size_t)kWinFields * Wn * 8, c->st));
-  CK(cudaMemsetAsync(c->kdelta.p, 0, Wn * c->nk * 2 * 4, c->st));
-  CK(cudaMemsetAsync(c->cdelta.p, 0, (size_t)c->nc * 2 * 8, c->st));
-  CK(cudaMemsetAsync(c->active.p, 0, Wn * c->ncw * 4, c->st));
-  CK(cudaMemsetAsync(c->anyfull.p, 0, Wn * c->ncw * 4, c->st));
-  CK(cudaMemsetAsync(c->unit_ctr.p, 0, 8, c->st));
-  CK(cudaMemsetAsync(c->status.p, 0, 8, c->st));
+  {
+    const ResLayout L = res_layout(c, W);
+    ClearList cl;
+    cl.add(c->res.p, (size_t)kWinFields * Wn * 8);
+    cl.add((char *)c->res.p + L.status, 16);
+    cl.add(c->kdelta.p, Wn * c->nk * 2 * 4);
+    cl.add(c->cdelta.p, (size_t)c->nc * 2 * 8);
+    cl.add(c->active.p, Wn * c->ncw * 4);
+    cl.add(c->anyfull.p, Wn * c->ncw * 4);
+    cl.add(c->unit_ctr.p, 8);
+    launch_clear(cl, c->st);
+  }
 
   p.tdesc = (TileDesc *)c->tdesc.p; p.tile_reg_s = (const uint32_t *)c->treg_s.p; p.tile_reg_e = (const uint32_t *)c->treg_e.p;
   p.n_tiles_s = nts; p.n_tiles_e = nte;
   p.soff = (uint16_t *)c->soff.p; p.stage = (unsigned long long *)c->stage.p;
   p.smeta = (TileMeta *)c->smeta.p; p.emeta = (TileMeta *)c->emeta.p;
   p.lastlvl = (uint16_t *)c->lastlvl.p; p.flags = (uint32_t *)c->flags.p;
-  p.win = (unsigned long long *)c->win.p; p.kdelta = (uint32_t *)c->kdelta.p;
+  set_result_ptrs(c, W, p);
+  p.kdelta = (uint32_t *)c->kdelta.p;
   p.cdelta = (unsigned long long *)c->cdelta.p; p.active = (uint32_t *)c->active.p;
   p.anyfull = (uint32_t *)c->anyfull.p; p.hung = (uint32_t *)c->hung.p;
-  p.unit_ctr = (uint32_t *)c->unit_ctr.p; p.status = (uint32_t *)c->status.p;
+  p.unit_ctr = (uint32_t *)c->unit_ctr.p;
   p.carry_in = (const uint16_t *)c->carry[c->cur].p; p.carry_out = (uint16_t *)c->carry[c->cur ^ 1].p;
   p.run = (const uint32_t *)c->run[c->cur].p;
   p.run_out = (uint32_t *)c->run[c->cur ^ 1].p;
   p.kstart = (long long *)c->kstart.p; p.kend = (long long *)c->kend.p;
   p.cstart = (long long *)c->cstart.p; p.cend = (long long *)c->cend.p;
-  p.topk = (unsigned long long *)c->topk.p; p.topk_n = (uint32_t *)c->topk_n.p;
-  p.prog = (long long *)c->prog.p; p.bstat = (rtm_buffer_stat *)c->bstat.p;
+  p.bstat = (rtm_buffer_stat *)c->bstat.p;
   p.comps = (rtm_component_tasks *)c->comps.p;
 
 #ifdef RTM_PHASE_TIMING
@@ -412,20 +441,18 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
 // D2H of the per-window results and bookkeeping after a (local or merged) reduce.
 rtm_status finish(rtm_ctx *c, const int64_t *t_end, uint32_t W, rtm_window_summary *out) {
   const size_t Wn = W;
-  const size_t bytes = (size_t)kWinFields * Wn * 8 + Wn * c->k * 8 + Wn * 4 + Wn * c->nk * 5 * 8 + 16;
+  const ResLayout L = res_layout(c, W);
+  const size_t bytes = L.bytes;
   rtm_status s;
   if ((s = ensure_pinned(c, c->h_res, bytes))) return s;
   char *h = (char *)c->h_res.p;
-  unsigned long long *hwin = (unsigned long long *)h;
-  unsigned long long *htopk = hwin + kWinFields * Wn;
-  long long *hprog = (long long *)(htopk + Wn * c->k);
-  uint32_t *htopk_n = (uint32_t *)(hprog + Wn * c->nk * 5);
-  uint32_t *hstatus = htopk_n + Wn;
-  CK(cudaMemcpyAsync(hwin, c->win.p, (size_t)kWinFields * Wn * 8, cudaMemcpyDeviceToHost, c->st));
-  CK(cudaMemcpyAsync(htopk, c->topk.p, Wn * c->k * 8, cudaMemcpyDeviceToHost, c->st));
-  CK(cudaMemcpyAsync(hprog, c->prog.p, Wn * c->nk * 5 * 8, cudaMemcpyDeviceToHost, c->st));
-  CK(cudaMemcpyAsync(htopk_n, c->topk_n.p, Wn * 4, cudaMemcpyDeviceToHost, c->st));
-  CK(cudaMemcpyAsync(hstatus, c->status.p, 4, cudaMemcpyDeviceToHost, c->st));
+  unsigned long long *hwin = (unsigned long long *)(h + L.win);
+  unsigned long long *htopk = (unsigned long long *)(h + L.topk);
+  long long *hprog = (long long *)(h + L.prog);
+  uint32_t *htopk_n = (uint32_t *)(h + L.topk_n);
+  uint32_t *hstatus = (uint32_t *)(h + L.status);
+  // one copy: the device results buffer has the same layout (res_layout)
+  CK(cudaMemcpyAsync(h, c->res.p, bytes, cudaMemcpyDeviceToHost, c->st));
   CK(cudaStreamSynchronize(c->st));
   prof_collect(c);
   if (*hstatus & 4u) {  // look-back wait timed out: internal error, never expected
@@ -449,10 +476,9 @@ rtm_status finish(rtm_ctx *c, const int64_t *t_end, uint32_t W, rtm_window_summa
     S.n_touched = (uint32_t)hwin[WF_TOUCHED * Wn + w];
     S.n_hung = (uint32_t)hwin[WF_HUNG * Wn + w];
   }
-  c->topk_h.assign(htopk, htopk + Wn * c->k);
-  c->topk_n_h.assign(htopk_n, htopk_n + Wn);
-  c->prog_h.resize(Wn * c->nk);
-  memcpy(c->prog_h.data(), hprog, Wn * c->nk * 5 * 8);
+  c->topk_h = htopk;
+  c->topk_n_h = htopk_n;
+  c->prog_h = reinterpret_cast<const rtm_progress_entry *>(hprog);
   if (out) memcpy(out, c->sum.data(), Wn * sizeof(rtm_window_summary));
   c->t_prev = t_end[W - 1];
   c->cur ^= 1;
@@ -579,8 +605,8 @@ void rtm_destroy(rtm_ctx *c) {
                     &c->kstart, &c->rcp, &c->elig_ids,
                     &c->kend, &c->cstart, &c->cend, &c->flags, &c->s_own, &c->e_own, &c->T, &c->Bs, &c->Be,
                     &c->rts, &c->rte, &c->treg_s, &c->treg_e, &c->tdesc, &c->soff, &c->stage, &c->smeta, &c->emeta,
-                    &c->lastlvl, &c->win, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
-                    &c->unit_ctr, &c->status, &c->topk, &c->topk_n, &c->prog, &c->bstat, &c->comps, &c->pack,
+                    &c->lastlvl, &c->res, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
+                    &c->unit_ctr, &c->bstat, &c->comps, &c->pack,
                     &c->gathered};
   for (DevBuf *b : bufs) free_buf(*b);
   if (c->h_small.p) cudaFreeHost(c->h_small.p);
@@ -668,10 +694,9 @@ rtm_status rtm_merge(rtm_ctx *c, const void *gathered, uint32_t world, rtm_windo
   p.nb = c->nb; p.nc = c->nc; p.nk = c->nk; p.nbins = c->nbins; p.ncw = c->ncw; p.k = c->k;
   p.rank_mode = c->rank_mode; p.W = W;
   p.ktotal = (const int64_t *)c->ktotal.p; p.rcp = (const unsigned long long *)c->rcp.p;
-  p.win = (unsigned long long *)c->win.p; p.topk = (unsigned long long *)c->topk.p;
-  p.topk_n = (uint32_t *)c->topk_n.p; p.prog = (long long *)c->prog.p; p.hung = (uint32_t *)c->hung.p;
+  set_result_ptrs(c, W, p);
+  p.hung = (uint32_t *)c->hung.p;
   p.comps = (rtm_component_tasks *)c->comps.p; p.bstat = (rtm_buffer_stat *)c->bstat.p;
-  p.status = (uint32_t *)c->status.p;
   LAUNCH(KT_MERGE, 0, launch_merge(p, gathered, world, c->st));
   CK(cudaGetLastError());
   std::vector<int64_t> te = c->t_end_h;
@@ -701,11 +726,11 @@ rtm_status rtm_window_results(rtm_ctx *c, uint32_t first, uint32_t count, rtm_wi
   if (!c->have) return RTM_E_STATE;
   if ((uint64_t)first + count > c->W) return RTM_E_INVALID;
   if (summaries) memcpy(summaries, c->sum.data() + first, (size_t)count * sizeof(rtm_window_summary));
-  if (topk_n) memcpy(topk_n, c->topk_n_h.data() + first, (size_t)count * 4);
+  if (topk_n) memcpy(topk_n, c->topk_n_h + first, (size_t)count * 4);
   if (bars)
-    memcpy(bars, c->prog_h.data() + (size_t)first * c->nk, (size_t)count * c->nk * sizeof(rtm_progress_entry));
+    memcpy(bars, c->prog_h + (size_t)first * c->nk, (size_t)count * c->nk * sizeof(rtm_progress_entry));
   if (topk) {
-    const unsigned long long *src = c->topk_h.data() + (size_t)first * c->k;
+    const unsigned long long *src = c->topk_h + (size_t)first * c->k;
     for (uint32_t w = 0; w < count; ++w) {
       const uint32_t n = c->topk_n_h[first + w];
       rtm_topk_entry *o = topk + (size_t)w * c->k;
@@ -726,7 +751,7 @@ rtm_status rtm_progress(rtm_ctx *c, uint32_t window, rtm_progress_entry *bars, r
   if (!c->have) return RTM_E_STATE;
   if (window >= c->W) return RTM_E_INVALID;
   if (comps && window != c->W - 1) return RTM_E_INVALID;
-  memcpy(bars, c->prog_h.data() + (size_t)window * c->nk, (size_t)c->nk * sizeof(rtm_progress_entry));
+  memcpy(bars, c->prog_h + (size_t)window * c->nk, (size_t)c->nk * sizeof(rtm_progress_entry));
   if (comps) {
     CK(cudaSetDevice(c->device));
     CK(cudaMemcpyAsync(comps, c->comps.p, (size_t)c->nc * sizeof(rtm_component_tasks), cudaMemcpyDeviceToHost,

@@ -138,6 +138,22 @@ uint64_t pack_bytes(const Params &p);
 void launch_pack(const Params &p, void *pack, cudaStream_t st);
 void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStream_t st);
 unsigned long long kernel_launches();  // kernels launched by this library in this process
+
+// Device ranges zeroed by ONE kernel launch (replaces per-buffer cudaMemsetAsync calls).
+struct ClearList {
+  static constexpr int kMax = 12;
+  void *ptr[kMax];
+  unsigned long long bytes[kMax];
+  int n = 0;
+  void add(void *p, size_t b) {
+    if (p && b && n < kMax) {
+      ptr[n] = p;
+      bytes[n] = b;
+      ++n;
+    }
+  }
+};
+void launch_clear(const ClearList &cl, cudaStream_t st);
 void configure_kernels_once();  // opt-in shared-memory limits, once per device
 size_t fold_smem_bytes();
 size_t partition_smem_bytes(uint32_t nbins, uint32_t nb);

@@ -1523,9 +1523,34 @@ __global__ void k_merge_tables(Params p, const unsigned char *g, unsigned world,
 // ============================================================================================
 // launchers
 // ============================================================================================
+// zero every range of the list: 16-byte stores over each range's 16-byte-aligned body, bytes
+// for the ends (ranges come from cudaMalloc'd buffers and may have any length)
+__global__ void k_clear(ClearList cl) {
+  const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (size_t)gridDim.x * blockDim.x;
+  for (int r = 0; r < cl.n; ++r) {
+    unsigned char *b = static_cast<unsigned char *>(cl.ptr[r]);
+    const size_t n = cl.bytes[r];
+    const size_t head = (16 - ((uintptr_t)b & 15)) & 15;
+    const size_t h = head < n ? head : n;
+    const size_t body = (n - h) / 16;
+    if (tid < h) b[tid] = 0;
+    uint4 *b4 = reinterpret_cast<uint4 *>(b + h);
+    for (size_t i = tid; i < body; i += nth) b4[i] = make_uint4(0, 0, 0, 0);
+    for (size_t i = h + body * 16 + tid; i < n; i += nth) b[i] = 0;
+  }
+}
+
 std::atomic<unsigned long long> g_kernel_launches{0};
 inline void count_launch() { g_kernel_launches.fetch_add(1, std::memory_order_relaxed); }
 unsigned long long kernel_launches() { return g_kernel_launches.load(std::memory_order_relaxed); }
+
+void launch_clear(const ClearList &cl, cudaStream_t st) {
+  if (!cl.n) return;
+  unsigned long long mx = 0;
+  for (int r = 0; r < cl.n; ++r) mx = cl.bytes[r] > mx ? cl.bytes[r] : mx;
+  const unsigned blocks = (unsigned)((mx / 16 + 255) / 256 + 1);
+  { k_clear<<<blocks < 1184 ? blocks : 1184, 256, 0, st>>>(cl); count_launch(); }
+}
 
 size_t fold_smem_bytes() { return sizeof(FoldSmem) * kFoldWarps; }
 size_t partition_smem_bytes(uint32_t nbins, uint32_t nb) {
