@@ -1177,29 +1177,79 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     const unsigned b = id_of(i);
     return fullness_key(lv[b], __ldg(p.cap + b), p.rank_mode, p.rcp);
   };
-  if (keys_in_smem)
-    for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) {
-      const unsigned b = id_of(i);
-      keys[i] = fullness_key(lv[b], __ldg(p.cap + b), p.rank_mode, p.rcp);
+  if (keys_in_smem) {
+    if (ALL && (p.nb & 7u) == 0) {  // 8 consecutive buffers per thread: 16-byte level / capacity loads
+      const uint4 *lv4 = reinterpret_cast<const uint4 *>(lv);
+      const uint4 *cp4 = reinterpret_cast<const uint4 *>(p.cap);
+      uint4 *k4 = reinterpret_cast<uint4 *>(keys);
+#pragma unroll 2
+      for (unsigned g = threadIdx.x; g < ne / 8; g += blockDim.x) {
+        const uint4 L = lv4[g], C = __ldg(cp4 + g);
+        const unsigned lw[4] = {L.x, L.y, L.z, L.w}, cw[4] = {C.x, C.y, C.z, C.w};
+        unsigned kk[8];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          kk[2 * q] = fullness_key(lw[q] & 0xFFFFu, cw[q] & 0xFFFFu, p.rank_mode, p.rcp);
+          kk[2 * q + 1] = fullness_key(lw[q] >> 16, cw[q] >> 16, p.rank_mode, p.rcp);
+        }
+        k4[2 * g] = make_uint4(kk[0], kk[1], kk[2], kk[3]);
+        k4[2 * g + 1] = make_uint4(kk[4], kk[5], kk[6], kk[7]);
+      }
+    } else {
+      for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) {
+        const unsigned b = id_of(i);
+        keys[i] = fullness_key(lv[b], __ldg(p.cap + b), p.rank_mode, p.rcp);
+      }
     }
+  }
   const unsigned keff = p.k < ne ? p.k : ne;
   if (keff == 0) {
     if (threadIdx.x == 0) p.topk_n[w] = 0;
     return;
   }
+  // Shortcut: when the largest key is held by >= k buffers (e.g. >= k buffers are 100 % full, the
+  // bottleneck picture of L197-L199), the answer is the k lowest ids holding it: tau = max key.
+  __shared__ unsigned s_max, s_cnt_max;
+  if (threadIdx.x == 0) s_max = 0, s_cnt_max = 0;
+  __syncthreads();
+  {
+    unsigned m = 0;
+    for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) m = max(m, key_at(i));
+    m = __reduce_max_sync(kFull, m);
+    if ((threadIdx.x & 31) == 0) atomicMax(&s_max, m);
+    __syncthreads();
+    const unsigned M = s_max;
+    unsigned c = 0;
+    for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) c += key_at(i) == M;
+    c = __reduce_add_sync(kFull, c);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(&s_cnt_max, c);
+    __syncthreads();
+  }
+  const bool top_tie = s_cnt_max >= keff;
   // MSB radix select.  After the first digit only candidates (top byte >= the selected digit,
   // at most k + the selected bucket) can matter: they are compacted in id order when they fit,
   // so the remaining passes and the selection scan ~1k keys instead of every buffer.
-  unsigned prefix = 0, mask = 0, need = keff;
+  unsigned prefix = top_tie ? s_max : 0u, mask = 0, need = keff;
   unsigned n_it = ne;  // iteration space: all keys, or the candidate list
   bool use_c = false;
-  for (int d = 3; d >= 0; --d) {
+  for (int d = top_tie ? -1 : 3; d >= 0; --d) {
     for (unsigned i = threadIdx.x; i < 8 * 256; i += blockDim.x) hist[i] = 0;
     __syncthreads();
     unsigned *myh = hist + (warp & 7) * 256;
-    for (unsigned j = threadIdx.x; j < n_it; j += blockDim.x) {
-      const unsigned k = key_at(use_c ? cand[j] : j);
-      if ((k & mask) == prefix) atomicAdd(&myh[(k >> (8 * d)) & 255u], 1u);
+    // warp-aggregated increments: many keys share a digit (empty / full buffers), and same-address
+    // shared atomics serialise; __match_any_sync costs ~2 cycles per distinct digit in the warp
+    const unsigned lane = threadIdx.x & 31;
+    for (unsigned j0 = threadIdx.x - lane; j0 < n_it; j0 += blockDim.x) {
+      const unsigned j = j0 + lane;
+      bool ok = false;
+      unsigned dg = 0;
+      if (j < n_it) {
+        const unsigned k = key_at(use_c ? cand[j] : j);
+        ok = (k & mask) == prefix;
+        dg = (k >> (8 * d)) & 255u;
+      }
+      const unsigned peers = __match_any_sync(kFull, ok ? dg : 0xFFFFFFFFu);
+      if (ok && lane == (unsigned)__ffs(peers) - 1) atomicAdd(&myh[dg], (unsigned)__popc(peers));
     }
     __syncthreads();
     if (threadIdx.x < 256) {
