@@ -280,3 +280,27 @@ def test_c2_full_size_parity():
                           s[idx])
     ref = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw).reduce(s, e, wl.t_end())
     assert_same(got, ref, mon)
+
+
+@pytest.mark.parametrize("n_top", [0, 10, 63, 64, 65, 200])
+@pytest.mark.parametrize("at_cap", [True, False])
+def test_topk_paths_top_tie_and_radix(n_top, at_cap):
+    """k=64 over 3000 buffers where exactly n_top buffers share the largest fullness (100 % full, or
+    7/8 with everything else lower): n_top >= k takes the top-tie shortcut, fewer takes the radix
+    select; both must match the oracle's sort (ties by buffer id)."""
+    rng = np.random.default_rng(77 + n_top + 1000 * at_cap)
+    nb = 3000
+    caps = rng.choice(np.array([4, 8, 16, 128, 1024], np.uint16), nb)
+    top = rng.choice(nb, n_top, replace=False)
+    caps[top] = 8
+    lv = np.minimum(rng.integers(0, 1024, nb), caps // 2).astype(np.uint16)  # <= 50 % full
+    lv[top] = 8 if at_cap else 7
+    s = sample_array([(i, b, int(lv[b]), int(caps[b])) for i, b in enumerate(rng.permutation(nb))])
+    owner = (np.arange(nb) // 4).astype(np.uint32)
+    kw = dict(t0=0, hang_windows=4, k=64, rank_mode=0)
+    orc, mon = _pair(owner, caps, np.ones(2, np.int64), int(owner[-1]) + 1, **kw)
+    ref = orc.reduce(s, event_array([]), [nb + 10])
+    mon.ingest(_dev(s), None)
+    got = mon.window_reduce([nb + 10])
+    assert int(got["topk_n"][0]) == int(ref["topk_n"][0]) == 64
+    assert np.array_equal(got["topk"][0], ref["topk"][0])
