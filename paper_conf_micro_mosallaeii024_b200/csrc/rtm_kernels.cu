@@ -834,15 +834,25 @@ __global__ void __launch_bounds__(kK3Threads) k_events(Params p) {
 // L_in from the nearest earlier window with a resolved level (decoupled look-back), finalizes
 // and resolves its own untouched cells.
 // ============================================================================================
+// Per-buffer fold state, one 16-byte record so a chain head / tail moves it with ONE shared
+// access: D (x, y), last | max << 16 (z), min | n16 << 16 (w).  last == 0xFFFF (never a valid
+// level: capacity 65535 is reserved) marks a buffer untouched in the window; the sample count is
+// hi[] * 65536 + n16 (hi[] low 16 bits, touched only when n16 wraps).  The offset of the first
+// sample in the window is ts0 | (hi >> 16) << 32 (hi bits only for windows >= 2^32 ticks).  6.5 KB
+// per warp: 8 CTAs of 4 warps per SM.
 struct FoldSmem {
-  unsigned long long D[kBin];      // sum_i (l_i - l_{i-1}) * (t_end - ts_i), l_{-1} = 0
-  unsigned long long ts0[kBin];    // offset of the first kept sample in the window
-  unsigned long long cml[kBin];    // cur | max << 16 | min << 32   (levels seen this window)
-  unsigned n[kBin];                // kept samples this window (0: untouched, other fields stale)
+  uint4 st[kBin];
+  unsigned ts0[kBin];              // offset of the first kept sample in the window, low 32 bits
+  unsigned hi[kBin];               // n_hi | ts0_hi << 16
   unsigned seg_end[32];            // flattened segment table of the current tile group
-  unsigned long long seg_ptr[32];
+  unsigned seg_base[32];           // staging index of each segment, minus its flattened start
   unsigned char owner[kBin];       // duplicate detection: last lane that wrote each buffer slot
 };
+constexpr unsigned kUntouchedZ = 0xFFFFFFFFu;  // st.z of an untouched buffer
+__device__ __forceinline__ bool st_touched(const uint4 &v) { return (v.z & 0xFFFFu) != 0xFFFFu; }
+__device__ __forceinline__ unsigned long long st_D(const uint4 &v) {
+  return ((unsigned long long)v.y << 32) | v.x;
+}
 
 // One chunk of <= 32 consecutive records (ingest order) of one (window, bin) unit.  Records of
 // the same buffer (peers, found with __match_any_sync) form a chain in lane order: each record's
@@ -873,13 +883,10 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
   const unsigned rank = __popc(lower);
   const bool tail = (peers >> lane) == 1u;
   const unsigned plv = __shfl_sync(kFull, lvl, pred);
-  unsigned c0 = 0;
-  unsigned long long st = 0;
-  if (act && (!lower || tail)) {  // chain heads need the state's level, tails update the state
-    c0 = S.n[lid];
-    st = S.cml[lid];
-  }
-  const unsigned prev = lower ? plv : (c0 ? (unsigned)(st & 0xFFFFu) : 0u);
+  uint4 sv = make_uint4(0, 0, kUntouchedZ, 0);
+  if (act && (!lower || tail)) sv = S.st[lid];  // chain heads need the level, tails the state
+  const bool c0 = st_touched(sv);
+  const unsigned prev = lower ? plv : (c0 ? (sv.z & 0xFFFFu) : 0u);
   const unsigned long long contrib =
       act ? (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off)) : 0ull;
   unsigned long long sum = contrib;
@@ -898,21 +905,26 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
   if (act && tail) {
     unsigned hi = mm >> 16, lo = mm & 0xFFFFu;
     unsigned long long d = sum;
+    unsigned n16 = rank + 1;
     if (c0) {
-      hi = max(hi, (unsigned)(st >> 16) & 0xFFFFu);
-      lo = min(lo, (unsigned)(st >> 32) & 0xFFFFu);
-      d += S.D[lid];
+      hi = max(hi, sv.z >> 16);
+      lo = min(lo, sv.w & 0xFFFFu);
+      d += st_D(sv);
+      n16 += sv.w >> 16;
+      if (n16 > 0xFFFFu) {  // rare: more than 65535 samples of one buffer in one window
+        S.hi[lid] += 1;
+        n16 -= 0x10000u;
+      }
     } else {
-      S.ts0[lid] = off0;
+      S.ts0[lid] = (unsigned)off0;
+      if (off0 >> 32) S.hi[lid] += (unsigned)(off0 >> 32) << 16;  // windows >= 2^32 ticks only
     }
-    S.D[lid] = d;
-    S.n[lid] = c0 + rank + 1;
-    S.cml[lid] = (unsigned long long)lvl | ((unsigned long long)hi << 16) | ((unsigned long long)lo << 32);
+    S.st[lid] = make_uint4((unsigned)d, (unsigned)(d >> 32), lvl | (hi << 16), lo | (n16 << 16));
   }
   __syncwarp();
 }
 
-__global__ void __launch_bounds__(kFoldWarps * 32, 6) k_fold(Params p) {
+__global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   FoldSmem &S = reinterpret_cast<FoldSmem *>(smem)[threadIdx.x >> 5];
   const int lane = threadIdx.x & 31;
@@ -928,7 +940,10 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 6) k_fold(Params p) {
     const unsigned long long Wlen = (unsigned long long)(te - tb);
     const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
 #pragma unroll
-    for (int i = 0; i < kBin / 32; ++i) S.n[lane + 32 * i] = 0;
+    for (int i = 0; i < kBin / 32; ++i) {
+      S.st[lane + 32 * i] = make_uint4(0, 0, kUntouchedZ, 0);
+      S.hi[lane + 32 * i] = 0;
+    }
     __syncwarp();
     // ---- phase 1: the (tile, bin) segments of window w, flattened into one stream of chunks
     for (unsigned tg = t_lo; tg < t_hi; tg += 32) {
@@ -947,14 +962,13 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 6) k_fold(Params p) {
       const unsigned total = __shfl_sync(kFull, pre, 31);
       // per-warp segment table: end (inclusive prefix) and the staging address of each segment
       S.seg_end[lane] = pre;
-      S.seg_ptr[lane] = (unsigned long long)(p.stage + (size_t)(tg + lane) * kTileS + seg_lo) -
-                        (unsigned long long)(pre - seg_len) * 8ull;
+      S.seg_base[lane] = (tg + lane) * (unsigned)kTileS + seg_lo - (pre - seg_len);
       __syncwarp();
       unsigned sgi = 0;  // this lane's current segment (cursor), advanced without warp collectives
       auto fetch = [&](unsigned g) -> unsigned long long {
         if (g >= total) return 0ull;
         while (g >= S.seg_end[sgi]) ++sgi;
-        return __ldcg(reinterpret_cast<const unsigned long long *>(S.seg_ptr[sgi]) + g);
+        return __ldcg(p.stage + (S.seg_base[sgi] + g));
       };
       // 4-deep software pipeline: staging reads are DRAM/L2 round trips
       unsigned long long e0 = fetch(lane), e1 = fetch(32 + lane), e2 = fetch(64 + lane), e3 = fetch(96 + lane);
@@ -973,7 +987,7 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 6) k_fold(Params p) {
 #pragma unroll
     for (int i = 0; i < kBin / 32; ++i) {
       const unsigned l = lane + 32 * i, b = b_base + l;
-      if (b < p.nb) lw[b] = S.n[l] ? (uint16_t)(S.cml[l] & 0xFFFFu) : kSent;
+      if (b < p.nb) lw[b] = (uint16_t)(S.st[l].z & 0xFFFFu);  // 0xFFFF == kSent: untouched
     }
     __threadfence();
     __syncwarp();
@@ -1028,16 +1042,17 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 6) k_fold(Params p) {
       const unsigned l = lane + 32 * i, b = b_base + l;
       if (b >= p.nb) continue;
       const unsigned L = lin[i];
-      const unsigned cnt = S.n[l];
+      const uint4 sv = S.st[l];
+      const unsigned hw = S.hi[l];
+      const unsigned cnt = st_touched(sv) ? ((hw & 0xFFFFu) << 16) + (sv.w >> 16) : 0u;
       unsigned long long I;
       unsigned mx, mn, last;
       if (cnt) {
-        const unsigned long long st = S.cml[l];
-        const unsigned hi = (unsigned)(st >> 16) & 0xFFFFu, lo = (unsigned)(st >> 32) & 0xFFFFu;
-        I = (unsigned long long)L * S.ts0[l] + S.D[l];
+        const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
+        I = (unsigned long long)L * (((unsigned long long)(hw >> 16) << 32) | S.ts0[l]) + st_D(sv);
         mx = hi > L ? hi : L;
         mn = lo < L ? lo : L;
-        last = (unsigned)(st & 0xFFFFu);
+        last = sv.z & 0xFFFFu;
       } else {
         I = (unsigned long long)L * Wlen;
         mx = mn = last = L;
