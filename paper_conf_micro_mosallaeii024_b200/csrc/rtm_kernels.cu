@@ -860,6 +860,7 @@ __device__ __forceinline__ unsigned long long st_D(const uint4 &v) {
 // Contributions are computed in parallel; the group's sum / max / min travel down the chain in
 // `maxrank` shuffle steps and only the chain's last lane updates the shared state, so every
 // state update in a chunk touches a distinct buffer.
+template <bool NAR>
 __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, bool act, unsigned long long e,
                                            unsigned long long Wlen) {
   const unsigned lid = (unsigned)(e & (kBin - 1));
@@ -887,8 +888,11 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
   if (act && (!lower || tail)) sv = S.st[lid];  // chain heads need the level, tails the state
   const bool c0 = st_touched(sv);
   const unsigned prev = lower ? plv : (c0 ? (sv.z & 0xFFFFu) : 0u);
+  // NAR: windows shorter than 2^32 ticks, (t_end - ts) fits 32 bits: one wide multiply
   const unsigned long long contrib =
-      act ? (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off)) : 0ull;
+      !act ? 0ull
+      : NAR ? (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(unsigned)(Wlen - off))
+            : (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off));
   unsigned long long sum = contrib;
   unsigned mm = (lvl << 16) | lvl;  // max << 16 | min over the chain so far
   const unsigned maxrank = __reduce_max_sync(kFull, rank);
@@ -917,13 +921,14 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
       }
     } else {
       S.ts0[lid] = (unsigned)off0;
-      if (off0 >> 32) S.hi[lid] += (unsigned)(off0 >> 32) << 16;  // windows >= 2^32 ticks only
+      if (!NAR && (off0 >> 32)) S.hi[lid] += (unsigned)(off0 >> 32) << 16;  // windows >= 2^32 ticks
     }
     S.st[lid] = make_uint4((unsigned)d, (unsigned)(d >> 32), lvl | (hi << 16), lo | (n16 << 16));
   }
   __syncwarp();
 }
 
+template <bool NAR>
 __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   FoldSmem &S = reinterpret_cast<FoldSmem *>(smem)[threadIdx.x >> 5];
@@ -960,21 +965,23 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
         if (lane >= o) pre += y;
       }
       const unsigned total = __shfl_sync(kFull, pre, 31);
-      // per-warp segment table: end (inclusive prefix) and the staging address of each segment
+      // per-warp segment table: end (inclusive prefix) and the staging index of each segment
+      // minus its flattened start
       S.seg_end[lane] = pre;
       S.seg_base[lane] = (tg + lane) * (unsigned)kTileS + seg_lo - (pre - seg_len);
       __syncwarp();
       unsigned sgi = 0;  // this lane's current segment (cursor), advanced without warp collectives
-      auto fetch = [&](unsigned g) -> unsigned long long {
+      auto fetch = [&](unsigned c) -> unsigned long long {
+        const unsigned g = c + lane;
         if (g >= total) return 0ull;
         while (g >= S.seg_end[sgi]) ++sgi;
         return __ldcg(p.stage + (S.seg_base[sgi] + g));
       };
       // 4-deep software pipeline: staging reads are DRAM/L2 round trips
-      unsigned long long e0 = fetch(lane), e1 = fetch(32 + lane), e2 = fetch(64 + lane), e3 = fetch(96 + lane);
+      unsigned long long e0 = fetch(0), e1 = fetch(32), e2 = fetch(64), e3 = fetch(96);
       for (unsigned c = 0; c < total; c += 32) {
-        const unsigned long long en = fetch(c + 128 + lane);
-        fold_chunk(S, lane, lt, c + lane < total, e0, Wlen);
+        const unsigned long long en = fetch(c + 128);
+        fold_chunk<NAR>(S, lane, lt, c + lane < total, e0, Wlen);
         e0 = e1;
         e1 = e2;
         e2 = e3;
@@ -1672,14 +1679,15 @@ void launch_events(const Params &p, cudaStream_t st) {
 void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
   const size_t sm = fold_smem_bytes();
   int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fold, kFoldWarps * 32, sm);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fold<true>, kFoldWarps * 32, sm);
   if (per_sm < 1) per_sm = 1;
   unsigned grid = (unsigned)(n_sms * per_sm);
   const unsigned units = p.W * p.nbins;
   const unsigned need = (units + kFoldWarps - 1) / kFoldWarps;
   if (grid > need) grid = need;
   if (grid == 0) grid = 1;
-  { k_fold<<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  if (p.narrow) { k_fold<true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else { k_fold<false><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
 }
 
 void launch_order_check(const Params &p, cudaStream_t st) {
@@ -1717,7 +1725,8 @@ void configure_kernels_once() {
   cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
   cudaFuncSetAttribute(k_topk<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)topk_smem_bytes(kTopkSmemKeys));
-  cudaFuncSetAttribute(k_fold, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
+  cudaFuncSetAttribute(k_fold<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
+  cudaFuncSetAttribute(k_fold<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
   cudaGetLastError();
 }
 
