@@ -335,8 +335,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.s = (const rtm_level_sample *)sp; p.ns = ns;
   p.e = (const rtm_task_event *)ep; p.ne = ne;
 
-  LAUNCH(KT_SPLIT, 0, launch_split(p, true, (long long *)c->Bs.p + 1, c->st));
-  LAUNCH(KT_SPLIT, 0, launch_split(p, false, (long long *)c->Be.p + 1, c->st));
+  LAUNCH(KT_SPLIT, 0, launch_split(p, (long long *)c->Bs.p + 1, (long long *)c->Be.p + 1, c->st));
   p.Bs = (const long long *)c->Bs.p; p.Be = (const long long *)c->Be.p;
   p.rts = (const uint32_t *)c->rts.p; p.rte = (const uint32_t *)c->rte.p;
   launch_regions(p, c->st);  // region tile tables on the device: no host round trip

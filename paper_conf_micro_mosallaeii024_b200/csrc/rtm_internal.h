@@ -123,7 +123,7 @@ struct Params {
 };
 
 // launchers (rtm_kernels.cu); all asynchronous on `st`
-void launch_split(const Params &p, bool samples, long long *outB, cudaStream_t st);
+void launch_split(const Params &p, long long *outBs, long long *outBe, cudaStream_t st);
 void launch_regions(const Params &p, cudaStream_t st);
 void launch_fill_tile_regions(const Params &p, cudaStream_t st);
 void launch_partition(const Params &p, int n_sms, cudaStream_t st);

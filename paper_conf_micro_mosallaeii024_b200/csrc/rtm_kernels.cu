@@ -129,10 +129,8 @@ __device__ unsigned block_excl_scan(unsigned v, unsigned *scratch /*[32]*/, unsi
 // per boundary, 33-ary search with 32 probes per step, then a linear warp scan.
 // ============================================================================================
 template <bool SAMPLES>
-__global__ void k_split(Params p, long long *outB) {
-  const unsigned q = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+__device__ __forceinline__ void split_one(const Params &p, unsigned q, long long *outB) {
   const int lane = threadIdx.x & 31;
-  if (q > p.W) return;
   const long long T = p.T[q];
   const unsigned long long N = SAMPLES ? p.ns : p.ne;
   const int4 *recs = SAMPLES ? reinterpret_cast<const int4 *>(p.s) : reinterpret_cast<const int4 *>(p.e);
@@ -178,11 +176,17 @@ __global__ void k_split(Params p, long long *outB) {
   if (lane == 0) outB[q] = (long long)ans;
 }
 
+// Both streams in one launch: warps 0..W split the samples, warps W+1..2W+1 the events.
+__global__ void k_split(Params p, long long *outBs, long long *outBe) {
+  const unsigned q = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;  // warp-uniform
+  if (q <= p.W) split_one<true>(p, q, outBs);
+  else if (q <= 2 * p.W + 1) split_one<false>(p, q - (p.W + 1), outBe);
+}
+
 // Region boundaries -> tile table on the device (no host round trip): B[0] = 0, B[W+2] = N, the
 // split positions made monotone (only an unsorted stream can break that; it is reported by the
 // order check), rt[r] = first tile of region r, rt[W+2] = number of tiles.  One CTA.
-__global__ void __launch_bounds__(1024) k_regions(long long *B, unsigned long long N, uint32_t W, uint32_t *rt,
-                                                   int tile) {
+__device__ __forceinline__ void regions_one(long long *B, unsigned long long N, uint32_t W, uint32_t *rt, int tile) {
   __shared__ long long wmax[32];
   __shared__ unsigned wsum[32];
   __shared__ long long carry_m;
@@ -230,10 +234,23 @@ __global__ void __launch_bounds__(1024) k_regions(long long *B, unsigned long lo
   }
 }
 
-// sample tiles: region id + descriptor (start, bounds, size, window) per tile
-__global__ void k_fill_tile_desc(Params p) {
-  const uint32_t nr = p.W + 2;
-  for (uint32_t r = blockIdx.x; r < nr; r += gridDim.x) {
+// CTA 0: sample regions, CTA 1: event regions.
+__global__ void __launch_bounds__(1024) k_regions(Params p, long long *Bs, long long *Be, uint32_t *rts, uint32_t *rte) {
+  if (blockIdx.x == 0) regions_one(Bs, p.ns, p.W, rts, kTileS);
+  else regions_one(Be, p.ne, p.W, rte, kTileE);
+}
+
+// first half of the grid: sample tiles (region id + descriptor: start, bounds, size, window);
+// second half: event tiles (region id)
+__global__ void k_fill_tiles(Params p) {
+  const uint32_t nr = p.W + 2, half = gridDim.x / 2;
+  if (blockIdx.x >= half) {
+    for (uint32_t r = blockIdx.x - half; r < nr; r += half)
+      for (uint32_t t = p.rte[r] + threadIdx.x; t < p.rte[r + 1]; t += blockDim.x)
+        const_cast<uint32_t *>(p.tile_reg_e)[t] = r;
+    return;
+  }
+  for (uint32_t r = blockIdx.x; r < nr; r += half) {
     const Region g = region_of(p, r);
     const long long lo = g.lo_ts;
     const unsigned long long wlen =
@@ -255,10 +272,6 @@ __global__ void k_fill_tile_desc(Params p) {
   }
 }
 
-__global__ void k_fill_tile_regions(const uint32_t *rt, uint32_t *tile_reg, uint32_t n_regions) {
-  for (uint32_t r = blockIdx.x; r < n_regions; r += gridDim.x)
-    for (uint32_t t = rt[r] + threadIdx.x; t < rt[r + 1]; t += blockDim.x) tile_reg[t] = r;
-}
 
 // ============================================================================================
 // K1: sample partition.  A tile is <= 4096 samples of ONE region, handled by one CTA of 8 warps;
@@ -1110,52 +1123,35 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
 }
 
 // ============================================================================================
-// K4: cross-tile order check (single CTA).  Tile t violates the contract if its own flag is set
-// or its first field-valid ts is below the max ts of all earlier tiles.
+// K4: cross-tile order check.  Every tile has its in-tile verdict (flag bit 1: range / order
+// inside the tile) and the offsets of its first / last field-valid record.  The field-valid
+// stream is non-decreasing iff every tile passes its own check and starts at or after the last
+// field-valid record of the nearest earlier tile that has one, so each tile is checked
+// independently (one thread per tile; the back-scan over tiles without valid records is
+// normally zero steps).  Sample tiles first, then event tiles, in one launch.
 // ============================================================================================
-__global__ void __launch_bounds__(1024) k_order_check(const TileMeta *meta, unsigned n_max, const uint32_t *n_dev,
-                                                       unsigned *status, unsigned bit) {
-  const unsigned n = *n_dev < n_max ? *n_dev : n_max;
-  __shared__ long long wmax[32];
-  __shared__ long long carry_s;
-  __shared__ unsigned bad_s;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  if (threadIdx.x == 0) { carry_s = kTsMin; bad_s = 0; }
-  __syncthreads();
-  for (unsigned base = 0; base < n; base += blockDim.x) {
-    const unsigned t = base + threadIdx.x;
-    TileMeta m;
-    m.flags = 0; m.first_ts = 0; m.last_ts = kTsMin;
-    if (t < n) m = meta[t];
-    const bool has = m.flags & 1u;
-    long long x = has ? m.last_ts : kTsMin;  // inclusive max-scan
-    for (int o = 1; o < 32; o <<= 1) {
-      long long y = shfl_ll(x, lane >= o ? lane - o : lane);
-      if (lane >= o && y > x) x = y;
-    }
-    if (lane == 31) wmax[warp] = x;
-    __syncthreads();
-    if (warp == 0) {
-      long long s = wmax[lane];
-      for (int o = 1; o < 32; o <<= 1) {
-        long long y = shfl_ll(s, lane >= o ? lane - o : lane);
-        if (lane >= o && y > s) s = y;
+__global__ void k_order_check(Params p) {
+  const unsigned ns = p.rts[p.W + 2] < p.n_tiles_s ? p.rts[p.W + 2] : p.n_tiles_s;
+  const unsigned ne = p.rte[p.W + 2] < p.n_tiles_e ? p.rte[p.W + 2] : p.n_tiles_e;
+  unsigned bad = 0;
+  for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < ns + ne; i += gridDim.x * blockDim.x) {
+    const bool smp = i < ns;
+    const TileMeta *meta = smp ? p.smeta : p.emeta;
+    const unsigned t = smp ? i : i - ns;
+    const TileMeta m = meta[t];
+    bool b = (m.flags & 2u) != 0;
+    if ((m.flags & 1u) && !b)
+      for (unsigned j = t; j-- > 0;) {
+        const TileMeta q = meta[j];
+        if (q.flags & 1u) {
+          b = m.first_ts < q.last_ts;
+          break;
+        }
       }
-      wmax[lane] = s;
-    }
-    __syncthreads();
-    long long before = carry_s;
-    const long long wprev = warp ? wmax[warp - 1] : kTsMin;
-    if (wprev > before) before = wprev;
-    long long xin = shfl_ll(x, lane ? lane - 1 : 0);
-    if (lane && xin > before) before = xin;
-    bool bad = (m.flags & 2u) || (has && m.first_ts < before);
-    if (__any_sync(kFull, bad) && lane == 0) atomicOr(&bad_s, 1u);
-    __syncthreads();
-    if (threadIdx.x == 0 && wmax[31] > carry_s) carry_s = wmax[31];
-    __syncthreads();
+    if (b) bad |= smp ? 1u : 2u;
   }
-  if (threadIdx.x == 0 && bad_s) atomicOr(status, bit);
+  bad = __reduce_or_sync(kFull, bad);
+  if ((threadIdx.x & 31) == 0 && bad) atomicOr(p.status, bad);
 }
 
 // ============================================================================================
@@ -1635,24 +1631,20 @@ size_t topk_smem_bytes(uint32_t nb) {
   return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8 + kTopkCand * 4;
 }
 
-void launch_split(const Params &p, bool samples, long long *outB, cudaStream_t st) {
-  const unsigned warps = p.W + 1;
+void launch_split(const Params &p, long long *outBs, long long *outBe, cudaStream_t st) {
+  const unsigned warps = 2 * (p.W + 1);
   const unsigned threads = 128;
   const unsigned blocks = (warps * 32 + threads - 1) / threads;
-  if (samples) { k_split<true><<<blocks, threads, 0, st>>>(p, outB); count_launch(); }
-  else { k_split<false><<<blocks, threads, 0, st>>>(p, outB); count_launch(); }
+  { k_split<<<blocks, threads, 0, st>>>(p, outBs, outBe); count_launch(); }
 }
-
 void launch_regions(const Params &p, cudaStream_t st) {
-  { k_regions<<<1, 1024, 0, st>>>(const_cast<long long *>(p.Bs), p.ns, p.W, const_cast<uint32_t *>(p.rts), kTileS); count_launch(); }
-  { k_regions<<<1, 1024, 0, st>>>(const_cast<long long *>(p.Be), p.ne, p.W, const_cast<uint32_t *>(p.rte), kTileE); count_launch(); }
+  { k_regions<<<2, 1024, 0, st>>>(p, const_cast<long long *>(p.Bs), const_cast<long long *>(p.Be),
+                                   const_cast<uint32_t *>(p.rts), const_cast<uint32_t *>(p.rte)); count_launch(); }
 }
-
 void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
   const unsigned nr = p.W + 2;
-  const unsigned blocks = nr < 4096 ? nr : 4096;
-  if (p.n_tiles_s) { k_fill_tile_desc<<<blocks, 64, 0, st>>>(p); count_launch(); }
-  if (p.n_tiles_e) { k_fill_tile_regions<<<blocks, 64, 0, st>>>(p.rte, const_cast<uint32_t *>(p.tile_reg_e), nr); count_launch(); }
+  const unsigned blocks = nr < 2048 ? nr : 2048;
+  { k_fill_tiles<<<2 * blocks, 64, 0, st>>>(p); count_launch(); }
 }
 
 void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
@@ -1691,8 +1683,11 @@ void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
 }
 
 void launch_order_check(const Params &p, cudaStream_t st) {
-  if (p.n_tiles_s) { k_order_check<<<1, 1024, 0, st>>>(p.smeta, p.n_tiles_s, p.rts + p.W + 2, p.status, 1u); count_launch(); }
-  if (p.n_tiles_e) { k_order_check<<<1, 1024, 0, st>>>(p.emeta, p.n_tiles_e, p.rte + p.W + 2, p.status, 2u); count_launch(); }
+  const unsigned n = p.n_tiles_s + p.n_tiles_e;  // upper bound; the kernel reads the device counts
+  if (!n) return;
+  unsigned blocks = (n + 255) / 256;
+  blocks = blocks < 1184 ? blocks : 1184;
+  { k_order_check<<<blocks, 256, 0, st>>>(p); count_launch(); }
 }
 
 void launch_topk(const Params &p, cudaStream_t st) {

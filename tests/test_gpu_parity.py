@@ -304,3 +304,38 @@ def test_topk_paths_top_tie_and_radix(n_top, at_cap):
     got = mon.window_reduce([nb + 10])
     assert int(got["topk_n"][0]) == int(ref["topk_n"][0]) == 64
     assert np.array_equal(got["topk"][0], ref["topk"][0])
+
+
+@pytest.mark.parametrize("disorder", [False, True])
+@pytest.mark.parametrize("stream", ["samples", "events"])
+def test_order_check_across_tiles_with_invalid_gap(disorder, stream):
+    """The cross-tile order check compares each tile with the nearest EARLIER tile that has a
+    field-valid record: here three 4096-record tiles, the middle one entirely field-invalid, and
+    (disorder) the third starting below the first tile's last ts.  Oracle and GPU must agree."""
+    nb, n = 8, 4096
+    owner = np.zeros(nb, np.uint32)
+    cap = np.full(nb, 4, np.uint16)
+    ts = np.concatenate([np.arange(n), np.full(n, 5000), np.arange(n) + (n - 10 if disorder else n)])
+    if stream == "samples":
+        rows = [(int(t), i % nb, 1, 4) for i, t in enumerate(ts)]
+        for i in range(n, 2 * n):
+            rows[i] = (int(ts[i]), nb + 3, 1, 4)  # buffer id out of range: field-invalid
+        s, e = sample_array(rows), event_array([])
+    else:
+        rows = [(int(t), i, 0 | (0 << 20) | ((i & 1) << 31)) for i, t in enumerate(ts)]
+        for i in range(n, 2 * n):
+            rows[i] = (int(ts[i]), i, 7)  # component 7 >= n_components: field-invalid
+        s, e = sample_array([]), event_array(rows)
+    kw = dict(t0=0, hang_windows=2, k=4)
+    orc, mon = _pair(owner, cap, np.full(1, 10 ** 6, np.int64), 1, **kw)
+    ends = [3 * n + 100]
+    ref = orc.reduce(s, e, ends)
+    mon.ingest(_dev(s) if len(s) else None, _dev(e) if len(e) else None)
+    if disorder:
+        assert ref["rc"] == -4
+        with pytest.raises(RTMError) as ei:
+            mon.window_reduce(ends)
+        assert ei.value.code == N.RTM_E_ORDER
+    else:
+        assert ref["rc"] == 0
+        assert_same(mon.window_reduce(ends), ref, mon)
