@@ -1195,54 +1195,58 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     const unsigned b = id_of(i);
     return fullness_key(lv[b], __ldg(p.cap + b), p.rank_mode, p.rcp);
   };
-  if (keys_in_smem) {
-    if (ALL && (p.nb & 7u) == 0) {  // 8 consecutive buffers per thread: 16-byte level / capacity loads
-      const uint4 *lv4 = reinterpret_cast<const uint4 *>(lv);
-      const uint4 *cp4 = reinterpret_cast<const uint4 *>(p.cap);
-      uint4 *k4 = reinterpret_cast<uint4 *>(keys);
+  // keys (shared memory when they fit) and, in the same pass, the largest key and how many
+  // buffers hold it (per thread, then per warp, then per CTA)
+  __shared__ unsigned s_max, s_cnt_max;
+  if (threadIdx.x == 0) s_max = 0, s_cnt_max = 0;
+  unsigned tm = 0, tc = 0;
+  auto track = [&](unsigned k) {
+    if (k > tm) tm = k, tc = 0;
+    tc += (k == tm);
+  };
+  if (keys_in_smem && ALL && (p.nb & 7u) == 0) {  // 8 consecutive buffers per thread: 16-B loads
+    const uint4 *lv4 = reinterpret_cast<const uint4 *>(lv);
+    const uint4 *cp4 = reinterpret_cast<const uint4 *>(p.cap);
+    uint4 *k4 = reinterpret_cast<uint4 *>(keys);
 #pragma unroll 2
-      for (unsigned g = threadIdx.x; g < ne / 8; g += blockDim.x) {
-        const uint4 L = lv4[g], C = __ldg(cp4 + g);
-        const unsigned lw[4] = {L.x, L.y, L.z, L.w}, cw[4] = {C.x, C.y, C.z, C.w};
-        unsigned kk[8];
+    for (unsigned g = threadIdx.x; g < ne / 8; g += blockDim.x) {
+      const uint4 L = lv4[g], C = __ldg(cp4 + g);
+      const unsigned lw[4] = {L.x, L.y, L.z, L.w}, cw[4] = {C.x, C.y, C.z, C.w};
+      unsigned kk[8];
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          kk[2 * q] = fullness_key(lw[q] & 0xFFFFu, cw[q] & 0xFFFFu, p.rank_mode, p.rcp);
-          kk[2 * q + 1] = fullness_key(lw[q] >> 16, cw[q] >> 16, p.rank_mode, p.rcp);
-        }
-        k4[2 * g] = make_uint4(kk[0], kk[1], kk[2], kk[3]);
-        k4[2 * g + 1] = make_uint4(kk[4], kk[5], kk[6], kk[7]);
+      for (int q = 0; q < 4; ++q) {
+        kk[2 * q] = fullness_key(lw[q] & 0xFFFFu, cw[q] & 0xFFFFu, p.rank_mode, p.rcp);
+        kk[2 * q + 1] = fullness_key(lw[q] >> 16, cw[q] >> 16, p.rank_mode, p.rcp);
       }
-    } else {
-      for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) {
-        const unsigned b = id_of(i);
-        keys[i] = fullness_key(lv[b], __ldg(p.cap + b), p.rank_mode, p.rcp);
-      }
+#pragma unroll
+      for (int q = 0; q < 8; ++q) track(kk[q]);
+      k4[2 * g] = make_uint4(kk[0], kk[1], kk[2], kk[3]);
+      k4[2 * g + 1] = make_uint4(kk[4], kk[5], kk[6], kk[7]);
+    }
+  } else {
+    for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) {
+      const unsigned b = id_of(i);
+      const unsigned k = fullness_key(lv[b], __ldg(p.cap + b), p.rank_mode, p.rcp);
+      if (keys_in_smem) keys[i] = k;
+      track(k);
     }
   }
   const unsigned keff = p.k < ne ? p.k : ne;
+  {
+    const unsigned wm = __reduce_max_sync(kFull, tm);
+    const unsigned wc = __reduce_add_sync(kFull, tm == wm ? tc : 0u);
+    __syncthreads();
+    if ((threadIdx.x & 31) == 0) atomicMax(&s_max, wm);
+    __syncthreads();
+    if ((threadIdx.x & 31) == 0 && wm == s_max && wc) atomicAdd(&s_cnt_max, wc);
+    __syncthreads();
+  }
   if (keff == 0) {
     if (threadIdx.x == 0) p.topk_n[w] = 0;
     return;
   }
   // Shortcut: when the largest key is held by >= k buffers (e.g. >= k buffers are 100 % full, the
   // bottleneck picture of L197-L199), the answer is the k lowest ids holding it: tau = max key.
-  __shared__ unsigned s_max, s_cnt_max;
-  if (threadIdx.x == 0) s_max = 0, s_cnt_max = 0;
-  __syncthreads();
-  {
-    unsigned m = 0;
-    for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) m = max(m, key_at(i));
-    m = __reduce_max_sync(kFull, m);
-    if ((threadIdx.x & 31) == 0) atomicMax(&s_max, m);
-    __syncthreads();
-    const unsigned M = s_max;
-    unsigned c = 0;
-    for (unsigned i = threadIdx.x; i < ne; i += blockDim.x) c += key_at(i) == M;
-    c = __reduce_add_sync(kFull, c);
-    if ((threadIdx.x & 31) == 0 && c) atomicAdd(&s_cnt_max, c);
-    __syncthreads();
-  }
   const bool top_tie = s_cnt_max >= keff;
   // MSB radix select.  After the first digit only candidates (top byte >= the selected digit,
   // at most k + the selected bucket) can matter: they are compacted in id order when they fit,
