@@ -1335,9 +1335,10 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     }
   }
   __syncthreads();
-  // bitonic sort descending over the next power of two >= keff
+  // bitonic sort descending over the next power of two >= keff (top tie: the winners share one
+  // key and were written in id order, so they are already sorted)
   unsigned P = 1;
-  while (P < keff) P <<= 1;
+  while (!top_tie && P < keff) P <<= 1;
   for (unsigned i = keff + threadIdx.x; i < P; i += blockDim.x) sel[i] = 0ull;
   __syncthreads();
   for (unsigned size = 2; size <= P; size <<= 1) {
