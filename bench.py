@@ -156,26 +156,22 @@ def run_reference(args):
 
 
 # ---------------------------------------------------------------------------------------------
-def weak_registry(wl, world):
-    """Registry of the N-times larger system: rank r's local buffer l -> global id (comp-major)."""
+def weak_registry(wl, rank, world):
+    """Rank `rank`'s shard of the N-times larger system, as a RANK-LOCAL registry: its own
+    C2-sized buffer set (dense local ids, include/rtm.h buffer_global_id) with the global id of
+    every local buffer and the global owning component.  Global layout: component-major, global
+    component = local component * N + rank (owner-component sharding)."""
     import gen
 
-    nbl = wl.n_buffers
-    owner, cap, tot = gen.registry(wl)  # local shapes; capacity depends on (seed, local id)
+    wr = wl.scaled(wl.name, seed=wl.seed + 1000 * rank) if world > 1 else wl
+    owner, cap, tot = gen.registry(wr)
     if world == 1:
-        return owner, cap, tot
-    gb = np.arange(nbl * world, dtype=np.int64)
-    gc = gb // 4
-    r = gc % world
-    lc = gc // world
-    lb = lc * 4 + gb % 4
-    caps = np.empty(nbl * world, np.uint16)
-    for rr in range(world):
-        wr = wl.scaled(wl.name, seed=wl.seed + 1000 * rr)
-        _, cr, _ = gen.registry(wr)
-        m = r == rr
-        caps[m] = cr[lb[m]]
-    return gc.astype(np.uint32), caps, tot * world
+        return wr, owner, cap, tot, None
+    bpc = wl.buffers_per_comp
+    lb = np.arange(wl.n_buffers, dtype=np.int64)
+    gcomp = (lb // bpc) * world + rank
+    gid = (gcomp * bpc + lb % bpc).astype(np.uint32)
+    return wr, gcomp.astype(np.uint32), cap, tot * world, gid
 
 
 def run_native(args):
@@ -194,23 +190,21 @@ def run_native(args):
 
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     wl = gen.C2
-    wr = wl.scaled(wl.name, seed=wl.seed + 1000 * rank) if world > 1 else wl
-    owner, cap, tot = weak_registry(wl, world)
-    nc = (len(owner) + 3) // 4
-    owned = None
-    if world > 1:
-        owned = (np.arange(nc) % world == rank).astype(np.uint8)
+    wr, owner, cap, tot, gid = weak_registry(wl, rank, world)
+    nc = wl.n_components * world
     dev = torch.device("cuda", local)
     ds = torch.empty(wl.n_samples * 16, dtype=torch.uint8, device=dev)
     de = torch.empty(wl.n_events * 16, dtype=torch.uint8, device=dev)
     st = torch.cuda.current_stream(dev).cuda_stream
     gen.fill_device("samples", wr, ds.data_ptr(), 0, wl.n_samples, st)
     gen.fill_device("events", wr, de.data_ptr(), 0, wl.n_events, st)
-    if world > 1:
-        gen.remap_weak(wr, ds.data_ptr(), wl.n_samples, de.data_ptr(), wl.n_events, rank, world, st)
+    if world > 1:  # samples keep their rank-local buffer ids; events name global components
+        gen.remap_weak(wr, ds.data_ptr(), 0, de.data_ptr(), wl.n_events, rank, world, st)
     torch.cuda.synchronize()
+    extra = {} if gid is None else dict(buffer_global_id=gid, n_global_buffers=wl.n_buffers * world,
+                                        pack_buffers=wl.n_buffers)
     mon = Monitor(owner, cap, tot, n_components=nc, t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k, device=local,
-                  rank=rank, world=world, owned_components=owned)
+                  rank=rank, world=world, **extra)
     t_end = wl.t_end()
     n_rec = wl.n_samples + wl.n_events
 
@@ -319,7 +313,7 @@ def run_native(args):
         "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
         "data": "synthetic",
         "config": {"workload": wl.description + (f" (x{world} shards, weak scaling)" if world > 1 else ""),
-                   "n_buffers": int(len(owner)), "records_per_gpu": n_rec, "windows": W, "k": wl.k,
+                   "n_buffers": int(wl.n_buffers * world), "records_per_gpu": n_rec, "windows": W, "k": wl.k,
                    "hang_windows": wl.hang_windows, "l2": "inputs (1.6 GB/GPU) larger than L2; no flush",
                    "parallelism": f"owner-component shards x{world}" if world > 1 else "single GPU"},
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved_gbs, "peak": hbm, "unit": "GB/s",

@@ -104,6 +104,16 @@ typedef struct {
   rtm_allgather_fn allgather;       /* required when world > 1                                 */
   void *allgather_user;
   void *stream;                     /* cudaStream_t to run on (NULL = the legacy default)      */
+  /* Rank-local buffer numbering (owner sharding without a global registry on every rank):
+   * when buffer_global_id is set, this context registers only its own buffers as a dense local
+   * numbering 0..n_buffers-1, records carry LOCAL buffer ids, and every result reports GLOBAL
+   * ids: top-k entries, the digest's buffer id, and the per-buffer table (indexed by global id,
+   * n_global_buffers entries).  Global ids must be strictly increasing in the local id, so ties
+   * broken by local id agree with ties by global id.  pack_buffers (world > 1) = the largest
+   * n_buffers over the ranks (equal-size exchange packs); 0 means n_buffers.                   */
+  const uint32_t *buffer_global_id; /* host [n_buffers] or NULL (ids are global)               */
+  uint32_t n_global_buffers;        /* > every global id; 0 when buffer_global_id is NULL       */
+  uint32_t pack_buffers;
 } rtm_config;
 
 /* ---- per-window outputs --------------------------------------------------------------------- */
@@ -167,7 +177,8 @@ rtm_status rtm_topk_buffers(rtm_ctx *ctx, uint32_t window, rtm_topk_entry *out, 
 rtm_status rtm_progress(rtm_ctx *ctx, uint32_t window, rtm_progress_entry *bars, rtm_component_tasks *comps);
 /* Hang-flagged component ids of `window`, ascending.  Writes min(cap, n) ids; *n_hung = n. */
 rtm_status rtm_hang_check(rtm_ctx *ctx, uint32_t window, uint32_t *comp_ids, uint32_t cap, uint32_t *n_hung);
-/* Full per-buffer table of the last window of the batch for buffers [first, first+count). */
+/* Full per-buffer table of the last window of the batch for buffers [first, first+count)
+ * (global ids when the context uses a rank-local numbering; buffers of no rank read as zero). */
 rtm_status rtm_buffer_stats(rtm_ctx *ctx, uint32_t first, uint32_t count, rtm_buffer_stat *out);
 
 /* Bulk form of the three accessors above for windows [first, first+count) of the last batch:

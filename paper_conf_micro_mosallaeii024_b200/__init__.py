@@ -58,7 +58,8 @@ class Monitor:
 
     def __init__(self, buffer_owner, buffer_capacity, kernel_total, *, n_components: int, t0: int = 0,
                  hang_windows: int = 8, k: int = 64, rank_mode: int = RTM_RANK_PERCENT, device: int = 0,
-                 rank: int = 0, world: int = 1, owned_components=None, stream=None, process_group=None):
+                 rank: int = 0, world: int = 1, owned_components=None, stream=None, process_group=None,
+                 buffer_global_id=None, n_global_buffers: int = 0, pack_buffers: int = 0):
         import torch
 
         if not torch.cuda.is_available():
@@ -81,6 +82,12 @@ class Monitor:
         cfg.owned_components = None if self._owned is None else self._owned.ctypes.data
         cfg.allgather = N.ALLGATHER_FN()  # the binding runs the exchange itself (two-phase API)
         cfg.stream = self._stream.cuda_stream
+        # rank-local buffer numbering (include/rtm.h): records carry local ids, results global ids
+        self._gid = None if buffer_global_id is None else np.ascontiguousarray(buffer_global_id, dtype=np.uint32)
+        cfg.buffer_global_id = None if self._gid is None else self._gid.ctypes.data
+        cfg.n_global_buffers = int(n_global_buffers)
+        cfg.pack_buffers = int(pack_buffers)
+        self.n_table = int(n_global_buffers) if self._gid is not None else self.n_buffers
         h = ctypes.c_void_p()
         N.check(N.lib().rtm_create(ctypes.byref(cfg), ctypes.byref(h)), "rtm_create")
         self._h = h
@@ -179,7 +186,7 @@ class Monitor:
 
     def buffer_stats(self, first: int = 0, count: int | None = None):
         if count is None:
-            count = self.n_buffers - first
+            count = self.n_table - first  # global ids with a rank-local numbering
         out = np.zeros(count, BSTAT_DTYPE)
         N.check(N.lib().rtm_buffer_stats(self._h, first, count, out.ctypes.data), "rtm_buffer_stats")
         return out

@@ -41,6 +41,8 @@ class Config(ctypes.Structure):
         ("rank_mode", ctypes.c_int32), ("device", ctypes.c_int32), ("rank", ctypes.c_int32),
         ("world", ctypes.c_int32), ("owned_components", ctypes.c_void_p), ("allgather", ALLGATHER_FN),
         ("allgather_user", ctypes.c_void_p), ("stream", ctypes.c_void_p),
+        ("buffer_global_id", ctypes.c_void_p), ("n_global_buffers", ctypes.c_uint32),
+        ("pack_buffers", ctypes.c_uint32),
     ]
 
 

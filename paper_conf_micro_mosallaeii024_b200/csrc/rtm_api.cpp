@@ -49,6 +49,8 @@ struct rtm_ctx {
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   int n_sms;
   DevBuf cap, owner, elig, ktotal, rcp, elig_ids;
+  DevBuf gid, bstat_g;      // rank-local numbering: global id per local buffer, table by global id
+  uint32_t n_global = 0, pack_nb = 0;
   uint32_t n_elig = 0;
   // persistent state
   DevBuf carry[2];
@@ -396,6 +398,8 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.kstart = (long long *)c->kstart.p; p.kend = (long long *)c->kend.p;
   p.cstart = (long long *)c->cstart.p; p.cend = (long long *)c->cend.p;
   p.bstat = (rtm_buffer_stat *)c->bstat.p;
+  p.gid = (const uint32_t *)c->gid.p; p.n_global = c->n_global; p.pack_nb = c->pack_nb;
+  p.bstat_g = (rtm_buffer_stat *)c->bstat_g.p;
   p.comps = (rtm_component_tasks *)c->comps.p;
 
 #ifdef RTM_PHASE_TIMING
@@ -526,6 +530,12 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   for (uint32_t b = 0; b < cfg->n_buffers; ++b)
     if (cfg->buffer_capacity[b] == 0 || cfg->buffer_capacity[b] == 0xFFFFu || cfg->buffer_owner[b] >= cfg->n_components)
       return RTM_E_INVALID;
+  if (cfg->buffer_global_id) {  // strictly increasing global ids below n_global_buffers
+    for (uint32_t b = 0; b < cfg->n_buffers; ++b)
+      if (cfg->buffer_global_id[b] >= cfg->n_global_buffers || (b && cfg->buffer_global_id[b] <= cfg->buffer_global_id[b - 1]))
+        return RTM_E_INVALID;
+  }
+  if (cfg->pack_buffers && cfg->pack_buffers < cfg->n_buffers) return RTM_E_INVALID;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || cfg->device < 0 || cfg->device >= ndev) {
     cudaGetLastError();
@@ -545,6 +555,8 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   c->world = cfg->world;
   c->t0 = cfg->t0;
   c->t_prev = cfg->t0;
+  c->n_global = cfg->buffer_global_id ? cfg->n_global_buffers : 0;
+  c->pack_nb = cfg->pack_buffers ? cfg->pack_buffers : cfg->n_buffers;
   c->allgather = cfg->allgather;
   c->allgather_user = cfg->allgather_user;
   c->st = (cudaStream_t)cfg->stream;
@@ -591,6 +603,16 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
     cudaGetLastError();
     return fail(RTM_E_CUDA);
   }
+  if (cfg->buffer_global_id) {
+    if ((s = ensure(c, c->gid, (size_t)c->nb * 4)) ||
+        (s = ensure(c, c->bstat_g, (size_t)c->n_global * sizeof(rtm_buffer_stat))))
+      return fail(s);
+    if (cudaMemcpy(c->gid.p, cfg->buffer_global_id, (size_t)c->nb * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemset(c->bstat_g.p, 0, (size_t)c->n_global * sizeof(rtm_buffer_stat)) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(RTM_E_CUDA);
+    }
+  }
   if ((s = zero_state(c))) return fail(s);
   *out = c;
   return RTM_OK;
@@ -601,7 +623,7 @@ void rtm_destroy(rtm_ctx *c) {
   cudaSetDevice(c->device);
   cudaStreamSynchronize(c->st);
   DevBuf *bufs[] = {&c->cap, &c->owner, &c->elig, &c->ktotal, &c->carry[0], &c->carry[1], &c->run[0], &c->run[1],
-                    &c->kstart, &c->rcp, &c->elig_ids,
+                    &c->kstart, &c->rcp, &c->elig_ids, &c->gid, &c->bstat_g,
                     &c->kend, &c->cstart, &c->cend, &c->flags, &c->s_own, &c->e_own, &c->T, &c->Bs, &c->Be,
                     &c->rts, &c->rte, &c->treg_s, &c->treg_e, &c->tdesc, &c->soff, &c->stage, &c->smeta, &c->emeta,
                     &c->lastlvl, &c->res, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
@@ -658,6 +680,8 @@ rtm_status rtm_window_reduce(rtm_ctx *c, const int64_t *t_end, uint32_t n_window
     }
     LAUNCH(KT_MERGE, 0, launch_merge(p, c->gathered.p, c->world, c->st));
     CK(cudaGetLastError());
+  } else if (c->gid.p) {
+    launch_scatter_bstat(p, c->st);
   }
   return finish(c, t_end, n_windows, out);
 }
@@ -696,6 +720,8 @@ rtm_status rtm_merge(rtm_ctx *c, const void *gathered, uint32_t world, rtm_windo
   set_result_ptrs(c, W, p);
   p.hung = (uint32_t *)c->hung.p;
   p.comps = (rtm_component_tasks *)c->comps.p; p.bstat = (rtm_buffer_stat *)c->bstat.p;
+  p.gid = (const uint32_t *)c->gid.p; p.n_global = c->n_global; p.pack_nb = c->pack_nb;
+  p.bstat_g = (rtm_buffer_stat *)c->bstat_g.p;
   LAUNCH(KT_MERGE, 0, launch_merge(p, gathered, world, c->st));
   CK(cudaGetLastError());
   std::vector<int64_t> te = c->t_end_h;
@@ -790,10 +816,12 @@ rtm_status rtm_buffer_stats(rtm_ctx *c, uint32_t first, uint32_t count, rtm_buff
   if (!c || (count && !out)) return RTM_E_INVALID;
   if (c->sticky) return (rtm_status)c->sticky;
   if (!c->have) return RTM_E_STATE;
-  if ((uint64_t)first + count > c->nb) return RTM_E_INVALID;
+  const bool by_gid = c->gid.p != nullptr;
+  if ((uint64_t)first + count > (by_gid ? c->n_global : c->nb)) return RTM_E_INVALID;
   if (!count) return RTM_OK;
   CK(cudaSetDevice(c->device));
-  CK(cudaMemcpyAsync(out, (rtm_buffer_stat *)c->bstat.p + first, (size_t)count * sizeof(rtm_buffer_stat),
+  CK(cudaMemcpyAsync(out, (rtm_buffer_stat *)(by_gid ? c->bstat_g.p : c->bstat.p) + first,
+                     (size_t)count * sizeof(rtm_buffer_stat),
                      cudaMemcpyDeviceToHost, c->st));
   CK(cudaStreamSynchronize(c->st));
   for (uint32_t i = 0; i < count; ++i) out[i].reserved = 0;

@@ -76,6 +76,9 @@ struct Params {
   const int64_t *ktotal;
   const unsigned long long *rcp;  // [65536] floor(2^48 / c) (exact fullness key, K5)
   const uint32_t *elig_ids;  // [n_elig] ascending ids of ranked buffers
+  const uint32_t *gid;       // [nb] global buffer id (rank-local numbering) or nullptr
+  uint32_t n_global;         // global id space (per-buffer table size) when gid is set
+  uint32_t pack_nb;          // per-buffer entries in an exchange pack
   uint32_t n_elig;
   // call
   uint32_t W;                // windows in the call
@@ -117,7 +120,8 @@ struct Params {
   unsigned long long *topk;  // [W * k] packed (id | level<<32 | cap<<48)
   uint32_t *topk_n;          // [W]
   long long *prog;           // [W * nk * 5]
-  rtm_buffer_stat *bstat;    // [nb]
+  rtm_buffer_stat *bstat;    // [nb] last window, local ids
+  rtm_buffer_stat *bstat_g;  // [n_global] merged / scattered table by global id (gid set)
   rtm_component_tasks *comps;// [nc]
   unsigned long long *dbg;   // phase-timing scratch (RTM_PHASE_TIMING builds only)
 };
@@ -137,6 +141,7 @@ void launch_progress(const Params &p, cudaStream_t st);
 uint64_t pack_bytes(const Params &p);
 void launch_pack(const Params &p, void *pack, cudaStream_t st);
 void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStream_t st);
+void launch_scatter_bstat(const Params &p, cudaStream_t st);  // gid set, world == 1
 unsigned long long kernel_launches();  // kernels launched by this library in this process
 
 // Device ranges zeroed by ONE kernel launch (replaces per-buffer cudaMemsetAsync calls).

@@ -1085,8 +1085,9 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
       }
       if (cnt) {
         // digest term: odd-constant products of (I, n|b, levels), XOR, one fmix64
+        const unsigned bid = p.gid ? __ldg(p.gid + b) : b;  // the digest names buffers by global id
         unsigned long long h = (I * 0x9E3779B97F4A7C15ULL) ^
-                               ((((unsigned long long)cnt << 32) | b) * 0xC2B2AE3D27D4EB4FULL) ^
+                               ((((unsigned long long)cnt << 32) | bid) * 0xC2B2AE3D27D4EB4FULL) ^
                                (((unsigned long long)last | ((unsigned long long)mx << 16) |
                                  ((unsigned long long)mn << 32) | ((unsigned long long)capb << 48)) *
                                 0x165667B19E3779F9ULL);
@@ -1358,7 +1359,8 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     unsigned long long out = 0xFFFFFFFFull;  // buffer_id 0xFFFFFFFF, level 0, cap 0
     if (i < keff) {
       unsigned b = 0xFFFFFFFFu - (unsigned)(sel[i] & 0xFFFFFFFFu);
-      out = (unsigned long long)b | ((unsigned long long)lv[b] << 32) | ((unsigned long long)__ldg(p.cap + b) << 48);
+      out = (unsigned long long)(p.gid ? __ldg(p.gid + b) : b) | ((unsigned long long)lv[b] << 32) |
+            ((unsigned long long)__ldg(p.cap + b) << 48);
     }
     p.topk[(size_t)w * p.k + i] = out;
   }
@@ -1463,10 +1465,11 @@ __global__ void __launch_bounds__(256) k_progress(Params p) {
 // ============================================================================================
 // Multi-rank merge (world > 1).  Pack layout per rank (bytes, 8-aligned sections):
 //   win [kWinFields][W] u64 | topk [W][k] u64 | topk_n [W] u32 (padded) | prog [W][nk][5] i64 |
-//   hung [W][ncw] u32 (padded) | comps [nc] (3 x i64) | bstat [nb] (32 B; reserved = owned)
+//   hung [W][ncw] u32 (padded) | comps [nc] (3 x i64) | bstat [pack_nb] (32 B; reserved = owned) |
+//   gids [pack_nb] u32 (rank-local numbering only: the global id of each bstat entry, ~0 = pad)
 // ============================================================================================
 struct PackLayout {
-  size_t win, topk, topk_n, prog, hung, comps, bstat, total;
+  size_t win, topk, topk_n, prog, hung, comps, bstat, gids, total;
 };
 __host__ __device__ inline size_t align8(size_t x) { return (x + 7) & ~(size_t)7; }
 __host__ __device__ inline PackLayout pack_layout(const Params &p) {
@@ -1478,7 +1481,8 @@ __host__ __device__ inline PackLayout pack_layout(const Params &p) {
   L.prog = o; o += align8((size_t)p.W * p.nk * 5 * 8);
   L.hung = o; o += align8((size_t)p.W * p.ncw * 4);
   L.comps = o; o += align8((size_t)p.nc * sizeof(rtm_component_tasks));
-  L.bstat = o; o += align8((size_t)p.nb * sizeof(rtm_buffer_stat));
+  L.bstat = o; o += align8((size_t)p.pack_nb * sizeof(rtm_buffer_stat));
+  L.gids = o; o += p.gid ? align8((size_t)p.pack_nb * 4) : 0;
   L.total = o;
   return L;
 }
@@ -1581,6 +1585,14 @@ __global__ void k_merge_tables(Params p, const unsigned char *g, unsigned world,
     t.in_flight = t.started - t.finished;
     p.comps[c] = t;
   }
+  if (p.gid) {  // rank-local numbering: scatter every rank's entries to their global ids
+    for (size_t q = tid; q < (size_t)world * p.pack_nb; q += nth) {
+      const unsigned r = (unsigned)(q / p.pack_nb), i = (unsigned)(q % p.pack_nb);
+      const unsigned gb = reinterpret_cast<const unsigned *>(g + stride * r + L.gids)[i];
+      if (gb < p.n_global) p.bstat_g[gb] = reinterpret_cast<const rtm_buffer_stat *>(g + stride * r + L.bstat)[i];
+    }
+    return;
+  }
   for (size_t b = tid; b < p.nb; b += nth) {
     rtm_buffer_stat pick = reinterpret_cast<const rtm_buffer_stat *>(g + L.bstat)[b];
     for (unsigned r = 0; r < world; ++r) {
@@ -1589,6 +1601,12 @@ __global__ void k_merge_tables(Params p, const unsigned char *g, unsigned world,
     }
     p.bstat[b] = pick;
   }
+}
+
+// world == 1 with a rank-local numbering: the table by global id
+__global__ void k_scatter_bstat(Params p) {
+  for (size_t b = (size_t)blockIdx.x * blockDim.x + threadIdx.x; b < p.nb; b += (size_t)gridDim.x * blockDim.x)
+    p.bstat_g[__ldg(p.gid + b)] = p.bstat[b];
 }
 
 }  // namespace
@@ -1740,6 +1758,18 @@ void launch_pack(const Params &p, void *pack, cudaStream_t st) {
   cudaMemcpyAsync(d + L.hung, p.hung, (size_t)p.W * p.ncw * 4, cudaMemcpyDeviceToDevice, st);
   cudaMemcpyAsync(d + L.comps, p.comps, (size_t)p.nc * sizeof(rtm_component_tasks), cudaMemcpyDeviceToDevice, st);
   cudaMemcpyAsync(d + L.bstat, p.bstat, (size_t)p.nb * sizeof(rtm_buffer_stat), cudaMemcpyDeviceToDevice, st);
+  if (p.pack_nb > p.nb)
+    cudaMemsetAsync(d + L.bstat + (size_t)p.nb * sizeof(rtm_buffer_stat), 0,
+                    (size_t)(p.pack_nb - p.nb) * sizeof(rtm_buffer_stat), st);
+  if (p.gid) {
+    cudaMemcpyAsync(d + L.gids, p.gid, (size_t)p.nb * 4, cudaMemcpyDeviceToDevice, st);
+    if (p.pack_nb > p.nb) cudaMemsetAsync(d + L.gids + (size_t)p.nb * 4, 0xFF, (size_t)(p.pack_nb - p.nb) * 4, st);
+  }
+}
+
+void launch_scatter_bstat(const Params &p, cudaStream_t st) {
+  const unsigned blocks = (p.nb + 255) / 256;
+  { k_scatter_bstat<<<blocks < 1184 ? blocks : 1184, 256, 0, st>>>(p); count_launch(); }
 }
 
 void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStream_t st) {

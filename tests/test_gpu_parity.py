@@ -339,3 +339,61 @@ def test_order_check_across_tiles_with_invalid_gap(disorder, stream):
     else:
         assert ref["rc"] == 0
         assert_same(mon.window_reduce(ends), ref, mon)
+
+
+def test_rank_local_numbering_shards_merge_equals_whole():
+    """Owner sharding with RANK-LOCAL buffer numbering (include/rtm.h buffer_global_id): each
+    shard registers only its own buffers (dense local ids, records remapped to them), results
+    carry global ids; the merged top-k, digests, progress, hang flags and the per-buffer table
+    (by global id) must equal the whole-trace oracle."""
+    import ctypes
+
+    from paper_conf_micro_mosallaeii024_b200 import _copy_from_ptr
+
+    wl = gen.C1.scaled("C1-lshard", n_samples=200_000, n_events=20_000, n_windows=6)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    ref = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw).reduce(gen.samples(wl), gen.events(wl),
+                                                                                   wl.t_end())
+    G = 3
+    gids = [np.nonzero(owner % G == r)[0].astype(np.uint32) for r in range(G)]
+    pack_nb = max(len(g) for g in gids)
+    mons, packs = [], []
+    ends = np.ascontiguousarray(wl.t_end())
+    for r in range(G):
+        gid = gids[r]
+        m = Monitor(owner[gid], cap[gid], tot, n_components=wl.n_components, rank=r, world=G,
+                    buffer_global_id=gid, n_global_buffers=len(owner), pack_buffers=pack_nb, **kw)
+        s = gen.samples(wl, shard=(G, r)).copy()
+        loc = np.searchsorted(gid, s["buffer_id"])
+        ok = (loc < len(gid)) & (gid[np.minimum(loc, len(gid) - 1)] == s["buffer_id"])
+        s["buffer_id"] = np.where(ok, loc, 0xFFFFFFF0).astype(np.uint32)
+        m.ingest(_dev(s), _dev(gen.events(wl, shard=(G, r))))
+        pack, nbytes = ctypes.c_void_p(), ctypes.c_uint64()
+        N.check(N.lib().rtm_window_reduce_local(m._h, ends.ctypes.data, len(ends), ctypes.byref(pack),
+                                                ctypes.byref(nbytes)), "local")
+        t = torch.empty(int(nbytes.value), dtype=torch.uint8, device="cuda")
+        _copy_from_ptr(t, pack.value, int(nbytes.value))
+        torch.cuda.synchronize()
+        mons.append(m)
+        packs.append(t)
+    assert len({int(t.numel()) for t in packs}) == 1  # equal-size packs (pack_buffers)
+    gathered = torch.cat(packs)
+    for m in mons:
+        summ = np.zeros(wl.n_windows, N.SUMMARY_DTYPE)
+        N.check(N.lib().rtm_merge(m._h, gathered.data_ptr(), G, summ.ctypes.data), "merge")
+        m.W = wl.n_windows
+        got = m.results()
+        assert np.array_equal(got["summary"], summ)
+        assert_same(got, ref, m)
+
+
+def test_rank_local_numbering_rejects_unsorted_ids():
+    owner = np.zeros(3, np.uint32)
+    cap = np.full(3, 4, np.uint16)
+    with pytest.raises(RTMError):
+        Monitor(owner, cap, np.ones(1, np.int64), n_components=1, buffer_global_id=np.array([5, 3, 9], np.uint32),
+                n_global_buffers=10)
+    with pytest.raises(RTMError):
+        Monitor(owner, cap, np.ones(1, np.int64), n_components=1, buffer_global_id=np.array([1, 3, 10], np.uint32),
+                n_global_buffers=10)
