@@ -183,12 +183,18 @@ def run_native(args):
     world = args.gpus
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("RTM_BENCH_BACKEND", "nccl") != "nccl":  # plumbing checks: ranks may share a GPU
+        local %= torch.cuda.device_count()
     torch.cuda.set_device(local)
     dist = None
     if world > 1:
         import torch.distributed as dist
 
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("RTM_BENCH_BACKEND", "nccl")  # gloo: ranks sharing one GPU (plumbing checks)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     wl = gen.C2
     wr, owner, cap, tot, gid = weak_registry(wl, rank, world)
     nc = wl.n_components * world
@@ -241,7 +247,7 @@ def run_native(args):
     prof = mon.profile_read()
     mon.profile(False)
     if dist:
-        t = torch.tensor([ms], device=dev)
+        t = torch.tensor([ms], device=dev if dist.get_backend() == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
     value = n_rec * world * args.steps / (ms / 1e3)
@@ -269,7 +275,7 @@ def run_native(args):
     torch.cuda.synchronize()
     te = time.perf_counter() - te
     if dist:
-        t = torch.tensor([te], device=dev)
+        t = torch.tensor([te], device=dev if dist.get_backend() == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         te = float(t.item())
     e2e_value = n_rec * world * e2e_steps / te

@@ -38,6 +38,8 @@ def allgather_packs(send, world: int, group=None):
     import torch
     import torch.distributed as dist
 
+    if send.is_cuda and dist.get_backend(group) == "gloo":  # gloo: stage through host memory
+        return allgather_packs(send.cpu(), world, group).to(send.device)
     recv = torch.empty(world * send.numel(), dtype=send.dtype, device=send.device)
     try:
         dist.all_gather_into_tensor(recv, send, group=group)
