@@ -397,3 +397,18 @@ def test_rank_local_numbering_rejects_unsorted_ids():
     with pytest.raises(RTMError):
         Monitor(owner, cap, np.ones(1, np.int64), n_components=1, buffer_global_id=np.array([1, 3, 10], np.uint32),
                 n_global_buffers=10)
+
+
+@pytest.mark.parametrize("n_buffers", [32768, 33000, 81920, 262144])
+def test_many_bins_partition_paths(n_buffers):
+    """n_bins <= 128 takes the lane-major partition, more bins the match-based fallback
+    (k_partition_mx): both must agree with the oracle (C3-like buffer counts, short trace)."""
+    wl = gen.C1.scaled("C1-bins", n_samples=400_000, n_events=40_000, n_buffers=n_buffers, n_windows=5)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    s, e = gen.samples(wl), gen.events(wl)
+    ref = orc.reduce(s, e, wl.t_end())
+    mon.ingest(_dev(s), _dev(e))
+    got = mon.window_reduce(wl.t_end())
+    assert_same(got, ref, mon)
