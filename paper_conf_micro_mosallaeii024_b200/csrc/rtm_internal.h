@@ -109,7 +109,7 @@ struct Params {
   uint32_t *active;          // [W * ncw]
   uint32_t *anyfull;         // [W * ncw]
   uint32_t *hung;            // [W * ncw]
-  uint32_t *unit_ctr;
+  uint32_t *unit_ctr;        // [0] fold units dequeued, [1] partition tiles claimed
   uint32_t *status;          // bit0 sample order, bit1 event order
   const uint16_t *carry_in;  // [nb]
   uint16_t *carry_out;       // [nb]

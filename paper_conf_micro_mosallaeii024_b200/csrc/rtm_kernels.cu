@@ -515,7 +515,20 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   // exclusive in-word prefixes) + 8 u16 word bases
   unsigned char *rows = reinterpret_cast<unsigned char *>(raw);
   for (unsigned i = threadIdx.x; i < p.nb; i += kK1Threads) capS[i] = __ldg(p.cap + i);
+  // Tiles are claimed dynamically (p.unit_ctr[1]) so a CTA that starts late - the side-stream
+  // event kernel holds SMs at first - simply takes fewer tiles.  Claims run two ahead:
+  // ring[i & 3] is iteration i's tile, written by thread 0 in iteration i - 2 and read after
+  // the barrier of iteration i - 1.
+  __shared__ unsigned ring[4];
   const unsigned n_tiles = p.rts[p.W + 2];
+  auto claim = [&]() -> unsigned {
+    const unsigned t = atomicAdd(p.unit_ctr + 1, 1u);
+    return t < n_tiles ? t : ~0u;
+  };
+  if (threadIdx.x == 0) {
+    ring[0] = claim();
+    ring[1] = ring[0] != ~0u ? claim() : ~0u;
+  }
   const int sub0 = warp * kSub;
   // async prefetch of a tile (descriptor already in dsm[slot]): this warp's 512 raw records,
   // record i to the 16-byte slot 16(i>>4) + ((i&15) ^ ((i>>4)&7))
@@ -528,8 +541,9 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
       if (i < m) cp_async16(raw + ((i & ~15) | ((i & 15) ^ ((i >> 4) & 7))), src + i);
     }
   };
-  unsigned tile = blockIdx.x;
-  if (tile < n_tiles) {
+  __syncthreads();  // capacity table, ring[0..1]
+  unsigned tile = ring[0];
+  if (tile != ~0u) {
     if (lane < 3) cp_async16(reinterpret_cast<int4 *>(dsm) + lane, reinterpret_cast<const int4 *>(p.tdesc + tile) + lane);
     cp_async_commit();
     cp_async_wait_all();
@@ -537,17 +551,17 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     prefetch_raw(dsm[0]);
   }
   cp_async_commit();
-  __syncthreads();  // capacity table
   long long pt_ = clock64();
   (void)pt_;
-  for (unsigned par = 0; tile < n_tiles; tile += gridDim.x, par ^= 1) {
-    const unsigned nxt = tile + gridDim.x;
+  for (unsigned it = 0, par = 0; tile != ~0u; ++it, par ^= 1) {
+    const unsigned nxt = ring[(it + 1) & 3];
+    if (threadIdx.x == 0) ring[(it + 2) & 3] = nxt != ~0u ? claim() : ~0u;
     const K1Tile t = k1_tile_from(dsm[par], tile);
     const bool is_win = t.g.window >= 0;
     unsigned short *wt = wt2 + (size_t)par * (vb / 2);
     unsigned short *myt = wt + (size_t)warp * nbins;
     __syncwarp();  // dsm[par] read by every lane before it is reused
-    if (nxt < n_tiles && lane < 3)
+    if (nxt != ~0u && lane < 3)
       cp_async16(reinterpret_cast<int4 *>(dsm + (par ^ 1)) + lane, reinterpret_cast<const int4 *>(p.tdesc + nxt) + lane);
     cp_async_commit();
     cp_async_wait_1();  // this tile's raw records (the descriptor group may still be in flight)
@@ -621,7 +635,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     // the next tile's records stream into the slot while this tile is published and written out
     cp_async_wait_all();
     __syncwarp();
-    if (nxt < n_tiles) prefetch_raw(dsm[par ^ 1]);
+    if (nxt != ~0u) prefetch_raw(dsm[par ^ 1]);
     cp_async_commit();
     k1_publish(wsum[par], first, last, has, viol, kept);
     __syncthreads();  // B1 (the only CTA barrier per tile): summaries + bin totals of this tile
@@ -637,6 +651,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
       }
     }
     PTM(5);
+    tile = nxt;
   }
   cp_async_wait_all();
 }
