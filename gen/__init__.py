@@ -45,8 +45,19 @@ class GenParams(ctypes.Structure):
         ("invalid_ppm", ctypes.c_uint32),
         ("shard_world", ctypes.c_uint32),
         ("shard_rank", ctypes.c_uint32),
-        ("reserved", ctypes.c_uint32),
+        ("zipf_n", ctypes.c_uint32),
+        ("zipf_cdf", ctypes.c_uint64),
+        ("zipf_a", ctypes.c_uint32),
+        ("zipf_b", ctypes.c_uint32),
+        ("dl_fill_ts", ctypes.c_int64 * 2),
+        ("dl_quiet_ts", ctypes.c_int64 * 2),
+        ("dl_comp", ctypes.c_uint32 * 4),
+        ("dl_sink", ctypes.c_uint32),
+        ("n_dl_stages", ctypes.c_uint32),
     ]
+
+
+assert ctypes.sizeof(GenParams) == 160
 
 
 @dataclass
@@ -68,6 +79,14 @@ class Workload:
     invalid_ppm: int = 0
     rank_mode: int = 0  # 0 percent, 1 size
     description: str = ""
+    # C4: Zipf exponent over buffer ranks (0 = uniform ids); ranks scattered by an affine map
+    zipf_s: float = 0.0
+    zipf_a: int = 0x9E3779B1 % (1 << 20) | 1
+    zipf_b: int = 12345
+    # C3: injected circular wait, per stage (window where the components go quiet, components);
+    # their buffers are held full from `deadlock_lead` windows earlier
+    deadlock: tuple = ()
+    deadlock_lead: int = 3
 
     @property
     def n_components(self) -> int:
@@ -104,7 +123,51 @@ class Workload:
         p.invalid_ppm = self.invalid_ppm
         p.shard_world = shard_world
         p.shard_rank = shard_rank
+        if self.zipf_s > 0:
+            import math
+            a = self.zipf_a % self.n_buffers or 1
+            while math.gcd(a, self.n_buffers) != 1:  # bijection on [0, n)
+                a += 1
+            p.zipf_n = self.n_buffers
+            p.zipf_a = a
+            p.zipf_b = self.zipf_b % self.n_buffers
+        if self.deadlock:
+            assert len(self.deadlock) <= 2
+            p.n_dl_stages = len(self.deadlock)
+            p.dl_sink = self.n_components - 1
+            for s, (w_d, comps) in enumerate(self.deadlock):
+                p.dl_quiet_ts[s] = self.t_begin(w_d)
+                p.dl_fill_ts[s] = self.t_begin(max(0, w_d - self.deadlock_lead))
+                p.dl_comp[2 * s] = comps[0]
+                p.dl_comp[2 * s + 1] = comps[1]
         return p
+
+    def t_begin(self, w: int) -> int:
+        """Begin of window w (= end of window w-1; t0 for w = 0)."""
+        return self.t0 + (w * self.ticks) // self.n_windows
+
+    def index_at(self, kind: str, T: int) -> int:
+        """First stream index whose ts >= T (ts_i = t0 + (i * mul) >> 32 is non-decreasing)."""
+        p = self.params()
+        mul = p.ts_mul_s if kind == "samples" else p.ts_mul_e
+        n = self.n_samples if kind == "samples" else self.n_events
+        d = T - self.t0
+        if d <= 0:
+            return 0
+        return min(n, -(-(d << 32) // mul))
+
+    def zipf_table(self) -> np.ndarray:
+        """u64 inverse-CDF thresholds of Zipf(s) over ranks 0..n-1 (P(rank r) ~ (r+1)^-s): a draw
+        u < 2^64 maps to the first r with u < cdf[r].  Built once on the host in fp64 (input data,
+        identical for the host and device generators); last entry 2^64-1."""
+        n = self.n_buffers
+        w = np.arange(1, n + 1, dtype=np.float64) ** (-self.zipf_s)
+        c = np.cumsum(w)
+        c /= c[-1]
+        t = np.minimum(np.floor(c * 2.0**64), 2.0**64 - 2048).astype(np.uint64)
+        t = np.maximum.accumulate(t)
+        t[-1] = np.uint64(0xFFFFFFFFFFFFFFFF)
+        return t
 
     def t_end(self, first: int = 0, count: int | None = None) -> np.ndarray:
         """Window ends: t_end[w] = t0 + (w+1)*T // n_windows (half-open windows)."""
@@ -126,9 +189,27 @@ C1 = Workload("C1-tiny", 1_000_000, 100_000, 1000, 4, 10, 16, 8, seed=1,
 C1_INVALID = C1.scaled("C1-invalid", invalid_ppm=10_000)
 C2 = Workload("C2-1gpu", 90_000_000, 10_000_000, 20480, 8, 1000, 64, 8, seed=2,
               description="MGPUSim-shaped 1-GPU run: ~20k buffers, 100M records, 1k windows, k=64")
-C3 = Workload("C3-4gpu", 900_000_000, 100_000_000, 81920, 32, 10000, 64, 16, seed=3,
-              description="MGPUSim-shaped 4-GPU run: ~80k buffers, 1B records, 10k windows")
-CONFIGS = {w.name: w for w in (C1, C1_INVALID, C2, C3)}
+# C3: 4 simulated GPUs x 20480 components; the injected circular wait sits on simulated GPU 2
+# (components 10240..15359): an "L2 local storage" / "L2 write buffer" pair goes quiet at window
+# 6000 and the upstream L1 / DRAM-controller pair it backs up at window 6005 (case study 2,
+# PAPER.md L217, L229).  H = 32: the smallest power of two at which the injection-free trace
+# flags nothing (tools/calibrate_h.py).
+C3_DEADLOCK = ((6000, (11240, 11243)), (6005, (11236, 11250)))
+C3 = Workload("C3-4gpu", 900_000_000, 100_000_000, 81920, 32, 10000, 64, 32, seed=3, deadlock=C3_DEADLOCK,
+              description="MGPUSim-shaped 4-GPU run: ~80k buffers, 1B records, 10k windows, injected "
+                          "circular-full-buffer deadlock")
+C3_CLEAN = C3.scaled("C3-clean", deadlock=())
+# C3 shape at 1/100 of the records (same buffers, components, deadlock pair): oracle in seconds
+C3_SMALL = C3.scaled("C3-small", n_samples=9_000_000, n_events=1_000_000, n_windows=100,
+                     deadlock=((60, (11240, 11243)), (65, (11236, 11250))))
+# C4: 1M buffers, Zipf(0.99) hot spots (YCSB-style exponent; BASELINE.json gives none), k = 1024
+C4 = Workload("C4-skewed", 1_800_000_000, 200_000_000, 1 << 20, 64, 2000, 1024, 16, seed=4, zipf_s=0.99,
+              description="skewed trace: 1M buffers, Zipf-distributed buffer_id hot spots, 2B records, top-k=1024")
+C4_SMALL = C4.scaled("C4-small", n_samples=18_000_000, n_events=2_000_000, n_windows=20)
+# C5: recorded for the next round (1M windows needs the sparse-window path)
+C5 = Workload("C5-long", 7_200_000_000, 800_000_000, 327680, 128, 1_000_000, 64, 256, seed=5,
+              description="long run: 16 simulated GPUs, ~320k buffers, 8B records in 1M windows")
+CONFIGS = {w.name: w for w in (C1, C1_INVALID, C2, C3, C3_CLEAN, C3_SMALL, C4, C4_SMALL, C5)}
 
 
 # ---------------------------------------------------------------------------------------
@@ -163,6 +244,10 @@ def samples(wl: Workload, start: int = 0, count: int | None = None, shard=(1, 0)
         count = wl.n_samples - start
     out = np.empty(count, dtype=SAMPLE_DTYPE)
     p = wl.params(*shard)
+    tab = None
+    if p.zipf_n:
+        tab = _zipf_host(wl)
+        p.zipf_cdf = tab.ctypes.data
     n = host_lib().gen_fill_samples(ctypes.byref(p), start, count, out.ctypes.data)
     return out[:n]
 
@@ -204,13 +289,45 @@ def device_lib():
         lib.gen_cuda_remap_weak.argtypes = [P, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint64,
                                             ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p]
         lib.gen_cuda_remap_weak.restype = ctypes.c_int
+        lib.gen_cuda_upload.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.POINTER(ctypes.c_void_p)]
+        lib.gen_cuda_upload.restype = ctypes.c_int
         _dev = lib
     return _dev
+
+
+_ZIPF_HOST: dict = {}
+_ZIPF_DEV: dict = {}
+
+
+def _zipf_key(wl):
+    return (wl.n_buffers, wl.zipf_s)
+
+
+def _zipf_host(wl):
+    k = _zipf_key(wl)
+    if k not in _ZIPF_HOST:
+        _ZIPF_HOST[k] = wl.zipf_table()
+    return _ZIPF_HOST[k]
+
+
+def _zipf_dev(wl):
+    """Device copy of the Zipf table (process lifetime; input data for the device generator)."""
+    k = _zipf_key(wl)
+    if k not in _ZIPF_DEV:
+        t = _zipf_host(wl)
+        ptr = ctypes.c_void_p()
+        err = device_lib().gen_cuda_upload(t.ctypes.data, t.nbytes, ctypes.byref(ptr))
+        if err != 0:
+            raise RuntimeError(f"gen_cuda_upload failed: cudaError {err}")
+        _ZIPF_DEV[k] = ptr.value
+    return _ZIPF_DEV[k]
 
 
 def fill_device(kind: str, wl: Workload, ptr: int, start: int, count: int, stream: int = 0) -> None:
     """Write records [start, start+count) of the (unsharded) trace into device memory at ptr."""
     p = wl.params()
+    if p.zipf_n and kind == "samples":
+        p.zipf_cdf = _zipf_dev(wl)
     fn = device_lib().gen_cuda_fill_samples if kind == "samples" else device_lib().gen_cuda_fill_events
     err = fn(ctypes.byref(p), start, count, ctypes.c_void_p(ptr), ctypes.c_void_p(stream))
     if err != 0:

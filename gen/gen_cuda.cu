@@ -85,4 +85,15 @@ int gen_cuda_remap_weak(const rtm_gen_params *p, void *s, uint64_t ns, void *e, 
   return (int)cudaGetLastError();
 }
 
+// Copy a host table (e.g. the Zipf thresholds) into a new device allocation (kept for the process).
+int gen_cuda_upload(const void *host, uint64_t bytes, void **out) {
+  void *d = nullptr;
+  cudaError_t e = cudaMalloc(&d, bytes ? bytes : 1);
+  if (e != cudaSuccess) return (int)e;
+  e = cudaMemcpy(d, host, bytes, cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) return (int)e;
+  *out = d;
+  return 0;
+}
+
 }  // extern "C"

@@ -59,7 +59,18 @@ typedef struct {
   uint32_t invalid_ppm;       /* corrupted records per million (0 = clean trace)     */
   uint32_t shard_world;       /* >1: keep only records whose owner comp % world == rank */
   uint32_t shard_rank;
-  uint32_t reserved;
+  uint32_t zipf_n;            /* >0: buffer ids drawn by Zipf rank (C4), see gen_buffer_id    */
+  uint64_t zipf_cdf;          /* address of u64 thresholds[zipf_n] (host or device memory,
+                                 matching the fill), increasing, last = UINT64_MAX             */
+  uint32_t zipf_a;            /* id = (rank * zipf_a + zipf_b) mod n_buffers (zipf_a coprime) */
+  uint32_t zipf_b;
+  int64_t dl_fill_ts[2];      /* deadlock stage s (C3): from dl_fill_ts[s] on, every sample of a
+                                 buffer owned by dl_comp[2s], dl_comp[2s+1] is at capacity       */
+  int64_t dl_quiet_ts[2];     /* ... and from dl_quiet_ts[s] on, their task events are
+                                 redirected to component dl_sink (the stuck tasks stay in flight) */
+  uint32_t dl_comp[4];
+  uint32_t dl_sink;
+  uint32_t n_dl_stages;       /* 0: no injection */
 } rtm_gen_params;
 
 /* ---- counter-based RNG: splitmix64 (Steele, Lea, Flood 2014) ---------------------- */
@@ -116,10 +127,32 @@ GEN_HD uint32_t gen_task_kernel(const rtm_gen_params *p, uint64_t task) {
   return k < p->n_kernels ? (uint32_t)k : p->n_kernels - 1;
 }
 
+/* Buffer of sample i: uniform (Lemire), or Zipf over ranks by inverse CDF (binary search for
+   the first threshold above u), ranks scattered over ids by an affine bijection (C4 hot spots
+   land in unrelated components). */
+GEN_HD uint32_t gen_buffer_id(const rtm_gen_params *p, uint64_t i) {
+  uint64_t u = gen_u(p, GEN_S_BUF, i);
+  if (!p->zipf_n) return gen_below(u, p->n_buffers);
+  const uint64_t *cdf = (const uint64_t *)(uintptr_t)p->zipf_cdf;
+  uint32_t lo = 0, hi = p->zipf_n - 1u; /* answer in [lo, hi] */
+  while (lo < hi) {
+    uint32_t mid = lo + (hi - lo) / 2u;
+    if (u < cdf[mid]) hi = mid;
+    else lo = mid + 1u;
+  }
+  return (uint32_t)(((uint64_t)lo * p->zipf_a + p->zipf_b) % p->n_buffers);
+}
+/* deadlock stage (0-based) of component c, or -1 */
+GEN_HD int gen_dl_stage(const rtm_gen_params *p, uint32_t c) {
+  for (uint32_t s = 0; s < p->n_dl_stages && s < 2u; ++s)
+    if (c == p->dl_comp[2u * s] || c == p->dl_comp[2u * s + 1u]) return (int)s;
+  return -1;
+}
+
 /* Level sample at stream index i (clean or, with invalid_ppm, possibly corrupted). */
 GEN_HD gen_sample_rec gen_sample(const rtm_gen_params *p, uint64_t i) {
   gen_sample_rec r;
-  uint32_t b = gen_below(gen_u(p, GEN_S_BUF, i), p->n_buffers);
+  uint32_t b = gen_buffer_id(p, i);
   uint16_t cap = gen_capacity(p, b);
   uint32_t cls = gen_class(p, b);
   uint64_t u1 = gen_u(p, GEN_S_L1, i), u2 = gen_u(p, GEN_S_L2, i);
@@ -133,6 +166,10 @@ GEN_HD gen_sample_rec gen_sample(const rtm_gen_params *p, uint64_t i) {
     lvl = (u1 % 10u) != 0u ? cap : cap - 1u;
   }
   r.ts = p->t0 + (int64_t)gen_mulshr32(i, p->ts_mul_s);
+  if (p->n_dl_stages) { /* injected circular wait: the stage's buffers back up and stay full */
+    int s = gen_dl_stage(p, gen_owner(p, b));
+    if (s >= 0 && r.ts >= p->dl_fill_ts[s]) lvl = cap;
+  }
   r.buffer_id = b;
   r.level = (uint16_t)lvl;
   r.capacity = cap;
@@ -172,6 +209,10 @@ GEN_HD gen_event_rec gen_event(const rtm_gen_params *p, uint64_t j) {
     }
   }
   r.ts = p->t0 + (int64_t)gen_mulshr32(j, p->ts_mul_e);
+  if (p->n_dl_stages) { /* a deadlocked component neither starts nor finishes tasks */
+    int s = gen_dl_stage(p, comp);
+    if (s >= 0 && r.ts >= p->dl_quiet_ts[s]) comp = p->dl_sink;
+  }
   r.task_id = (uint32_t)task;
   r.meta = (comp & 0xFFFFFu) | ((kern & 0x7FFu) << 20) | (kind << 31);
   if (comp > 0xFFFFFu) r.meta = 0xFFFFFu | ((kern & 0x7FFu) << 20) | (kind << 31);

@@ -96,7 +96,7 @@ class Oracle:
     def reset(self):
         lib().orc_reset(self._h)
 
-    def reduce(self, samples, events, t_end, *, want_hung=True, want_all_stats=False):
+    def reduce(self, samples, events, t_end, *, want_hung=True, want_all_stats=False, want_topk=True):
         samples = np.ascontiguousarray(samples)
         events = np.ascontiguousarray(events)
         t_end = np.ascontiguousarray(t_end, dtype=np.int64)
@@ -112,7 +112,8 @@ class Oracle:
             "all_stats": np.zeros((W, self.n_buffers), BSTAT_DTYPE) if want_all_stats else None,
         }
         rc = lib().orc_reduce(self._h, _ptr(samples), len(samples), _ptr(events), len(events), _ptr(t_end), W,
-                              _ptr(out["summary"]), _ptr(out["topk"]), _ptr(out["topk_n"]), _ptr(out["progress"]),
+                              _ptr(out["summary"]), _ptr(out["topk"]) if want_topk else None,
+                              _ptr(out["topk_n"]) if want_topk else None, _ptr(out["progress"]),
                               _ptr(out["hung"]), _ptr(out["stats"]), _ptr(out["comps"]), _ptr(out["all_stats"]))
         out["rc"] = rc
         return out

@@ -430,3 +430,89 @@ def test_gpu_fullness_key_reciprocal_formula_is_exact():
     for c in (65533, 65534, 40961, 32768, 32769):
         for l in (0, 1, c // 2, c - 2, c - 1):
             assert gpu_key(l, c) == (l << 32) // c
+
+
+# ---------------------------------------------------------------------------------------------
+# C3 (injected circular wait) and C4 (Zipf skew) shapes, oracle side
+def _oracle_for(wl, **kw):
+    owner, cap, tot = gen.registry(wl)
+    args = dict(t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k)
+    args.update(kw)
+    return oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **args)
+
+
+def test_c3_small_injected_deadlock_is_flagged_and_nothing_else():
+    """Case study 2 (L217, L229) at C3's shape: the injected pair is flagged from w_d + H - 1 on
+    (at most `deadlock_lead` windows earlier if it happened to fall silent while its buffers were
+    already held full), the upstream pair it backs up 5 windows later; the same trace without the
+    injection flags nothing at this H (the calibration of H)."""
+    wl = gen.C3_SMALL
+    s, e = gen.samples(wl), gen.events(wl)
+    r = _oracle_for(wl).reduce(s, e, wl.t_end(), want_topk=False)
+    assert r["rc"] == 0
+    hung = [set(np.nonzero(h)[0].tolist()) for h in r["hung"]]
+    H, lead = wl.hang_windows, wl.deadlock_lead
+    injected = set()
+    for w_d, cs in wl.deadlock:
+        for c in cs:
+            injected.add(c)
+            first = next(w for w in range(wl.n_windows) if c in hung[w])
+            assert w_d + H - 1 - lead <= first <= w_d + H - 1
+            assert all(c in hung[w] for w in range(w_d + H - 1, wl.n_windows))
+    assert set().union(*hung) == injected
+    clean = wl.scaled("C3-small-clean", deadlock=())
+    rc = _oracle_for(clean).reduce(gen.samples(clean), gen.events(clean), clean.t_end(), want_topk=False)
+    assert rc["hung"].sum() == 0
+    # the injected components' stuck tasks stay in flight: no START / END after w_d
+    w_d, (a, b) = wl.deadlock[0]
+    comp = e["meta"] & 0xFFFFF
+    assert not np.any(np.isin(comp[e["ts"] >= wl.t_begin(w_d)], [a, b]))
+
+
+def test_c3_small_streamed_batches_equal_one_call():
+    """The oracle context carries state across calls: streaming the trace in window batches (the
+    way the large GPU parity tests drive it) gives the one-call results."""
+    wl = gen.C3_SMALL.scaled("C3-batch", n_samples=2_000_000, n_events=200_000, n_windows=40,
+                             deadlock=((20, (11240, 11243)),), hang_windows=4)
+    s, e = gen.samples(wl), gen.events(wl)
+    one = _oracle_for(wl).reduce(s, e, wl.t_end())
+    orc = _oracle_for(wl)
+    for w0 in range(0, wl.n_windows, 7):
+        w1 = min(wl.n_windows, w0 + 7)
+        sl = slice(wl.index_at("samples", wl.t_begin(w0)), wl.index_at("samples", wl.t_begin(w1)))
+        el = slice(wl.index_at("events", wl.t_begin(w0)), wl.index_at("events", wl.t_begin(w1)))
+        r = orc.reduce(s[sl], e[el], wl.t_end()[w0:w1])
+        assert np.array_equal(r["summary"], one["summary"][w0:w1])
+        assert np.array_equal(r["topk"], one["topk"][w0:w1])
+        assert np.array_equal(r["progress"], one["progress"][w0:w1])
+        assert np.array_equal(r["hung"], one["hung"][w0:w1])
+    assert np.array_equal(r["stats"], one["stats"])
+
+
+def test_zipf_generator_shape():
+    """C4's buffer ids: Zipf(0.99) rank frequencies (top-1 share = 1 / H_{n,s}), scattered by a
+    bijection over the id space."""
+    wl = gen.C4_SMALL
+    s = gen.samples(wl, 0, 1_000_000)
+    cnt = np.bincount(s["buffer_id"], minlength=wl.n_buffers)
+    r = np.arange(1, wl.n_buffers + 1, dtype=np.float64)
+    p1 = 1.0 / np.sum(r ** -wl.zipf_s)
+    top = np.sort(cnt)[::-1]
+    assert abs(top[0] / len(s) - p1) < 5 * np.sqrt(p1 / len(s))
+    assert abs(top[1] / len(s) - p1 / 2 ** wl.zipf_s) < 5 * np.sqrt(p1 / len(s))
+    t = wl.zipf_table()
+    assert np.all(np.diff(t.astype(np.float64)) >= 0) and t[-1] == np.uint64(2**64 - 1)
+    p = wl.params()
+    ids = (np.arange(wl.n_buffers, dtype=np.uint64) * p.zipf_a + p.zipf_b) % wl.n_buffers
+    assert len(np.unique(ids)) == wl.n_buffers
+
+
+def test_c4_small_oracle_topk_matches_fraction_sort():
+    """k = 1024 under skew: the oracle's top-k of the last window equals an exact Fraction sort."""
+    wl = gen.C4_SMALL.scaled("C4-tiny", n_samples=2_000_000, n_events=200_000, n_windows=3,
+                             n_buffers=1 << 16)
+    s, e = gen.samples(wl), gen.events(wl)
+    r = _oracle_for(wl).reduce(s, e, wl.t_end())
+    st = r["stats"]
+    order = sorted(range(wl.n_buffers), key=lambda b: (-Fraction(int(st["last"][b]), int(st["capacity"][b])), b))
+    assert r["topk"][-1]["buffer_id"].tolist() == order[:wl.k]
