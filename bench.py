@@ -195,7 +195,7 @@ def run_native(args):
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         else:
             dist.init_process_group(backend)
-    wl = gen.C2
+    wl = gen.CONFIGS[args.config]
     wr, owner, cap, tot, gid = weak_registry(wl, rank, world)
     nc = wl.n_components * world
     dev = torch.device("cuda", local)
@@ -253,6 +253,22 @@ def run_native(args):
     value = n_rec * world * args.steps / (ms / 1e3)
 
     # ---- e2e through the same C-ABI with HOST buffers (pinned), results read back each step
+    e2e_value = None
+    if 16 * n_rec <= (8 << 30) and not args.no_e2e:
+        e2e_value = run_e2e(args, mon, ds, de, wl, t_end, n_rec, world, dist, dev)
+    W = wl.n_windows
+    d2h = W * (8 * 6 + wl.k * 8 + 4 + wl.n_kernels * 40 + 4)
+    rank_done = rank != 0
+    if rank_done:
+        if dist:
+            dist.destroy_process_group()
+        return
+    return finish(args, wl, world, ms, prof, n_rec, value, e2e_value, d2h, n_launches, clk, t_wall, dist)
+
+
+def run_e2e(args, mon, ds, de, wl, t_end, n_rec, world, dist, dev):
+    import torch
+
     hs = torch.empty(wl.n_samples * 16, dtype=torch.uint8, pin_memory=True)
     he = torch.empty(wl.n_events * 16, dtype=torch.uint8, pin_memory=True)
     hs.copy_(ds)
@@ -278,14 +294,11 @@ def run_native(args):
         t = torch.tensor([te], device=dev if dist.get_backend() == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         te = float(t.item())
-    e2e_value = n_rec * world * e2e_steps / te
-    W = wl.n_windows
-    d2h = W * (8 * 6 + wl.k * 8 + 4 + wl.n_kernels * 40 + 4)
+    return n_rec * world * e2e_steps / te
 
-    if rank != 0:
-        if dist:
-            dist.destroy_process_group()
-        return
+
+def finish(args, wl, world, ms, prof, n_rec, value, e2e_value, d2h, n_launches, clk, t_wall, dist):
+    W = wl.n_windows
     # ---- roofline of the dominant kernel: largest share of the step among the kernels on the
     # critical (main) stream; k_events runs on a side stream overlapped with the partition + fold
     peaks = _peaks()
@@ -298,7 +311,7 @@ def run_native(args):
     achieved_gbs = (dk["algo_bytes"] / dk["launches"]) / (dk["total_ms"] / dk["launches"] / 1e3) / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tp):
+    if os.path.exists(tp) and args.config == "C2-1gpu":  # traffic.json holds the C2 capture
         try:
             allt = json.load(open(tp)).get("all", {})
             traffic = next((v for k, v in allt.items() if k == dom or k.startswith(dom + "_")), None)
@@ -313,14 +326,15 @@ def run_native(args):
         n_win = int(os.environ.get("RTM_CPU_WINDOWS", "40"))
         recs, dt = cpu_reference_step(wl, n_win)
         cpu = {"value": recs / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"first {n_win} of {W} C2 windows ({recs} records), single-threaded C oracle"}
+               "sample": f"first {n_win} of {W} {wl.name} windows ({recs} records), single-threaded C oracle"}
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
         "data": "synthetic",
         "config": {"workload": wl.description + (f" (x{world} shards, weak scaling)" if world > 1 else ""),
                    "n_buffers": int(wl.n_buffers * world), "records_per_gpu": n_rec, "windows": W, "k": wl.k,
-                   "hang_windows": wl.hang_windows, "l2": "inputs (1.6 GB/GPU) larger than L2; no flush",
+                   "hang_windows": wl.hang_windows,
+                   "l2": f"inputs ({16 * n_rec / 1e9:.1f} GB/GPU) larger than L2; no flush",
                    "parallelism": f"owner-component shards x{world}" if world > 1 else "single GPU"},
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved_gbs, "peak": hbm, "unit": "GB/s",
                      "frac": achieved_gbs / hbm, "traffic": traffic,
@@ -329,7 +343,8 @@ def run_native(args):
                      "path_achieved": path_gbs, "path_frac": path_gbs / hbm, "per_kernel": per_kernel},
         "kernel_share": shares,
         "cpu_baseline": cpu,
-        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 16 * n_rec, "d2h_bytes_per_step": d2h},
+        "e2e": ({"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 16 * n_rec, "d2h_bytes_per_step": d2h}
+                if e2e_value is not None else None),
         "gpu_launches": n_launches,
         "clocks": clk.summary(),
         "wall_s_timed": t_wall,
@@ -346,6 +361,10 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--config", default="C2-1gpu",
+                    help="workload (gen.CONFIGS); the bench line is C2-1gpu, the others are parity configs "
+                         "measured for profiles/")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -192,18 +192,20 @@ C2 = Workload("C2-1gpu", 90_000_000, 10_000_000, 20480, 8, 1000, 64, 8, seed=2,
 # C3: 4 simulated GPUs x 20480 components; the injected circular wait sits on simulated GPU 2
 # (components 10240..15359): an "L2 local storage" / "L2 write buffer" pair goes quiet at window
 # 6000 and the upstream L1 / DRAM-controller pair it backs up at window 6005 (case study 2,
-# PAPER.md L217, L229).  H = 32: the smallest power of two at which the injection-free trace
-# flags nothing (tools/calibrate_h.py).
+# PAPER.md L217, L229).  H = 40: the smallest of {32, 40, 48, 56, 64} at which the injection-free
+# trace flags nothing (tools/calibrate_h.py: 6 components at H = 32, none from 40 on).
 C3_DEADLOCK = ((6000, (11240, 11243)), (6005, (11236, 11250)))
-C3 = Workload("C3-4gpu", 900_000_000, 100_000_000, 81920, 32, 10000, 64, 32, seed=3, deadlock=C3_DEADLOCK,
+C3 = Workload("C3-4gpu", 900_000_000, 100_000_000, 81920, 32, 10000, 64, 40, seed=3, deadlock=C3_DEADLOCK,
               description="MGPUSim-shaped 4-GPU run: ~80k buffers, 1B records, 10k windows, injected "
                           "circular-full-buffer deadlock")
 C3_CLEAN = C3.scaled("C3-clean", deadlock=())
 # C3 shape at 1/100 of the records (same buffers, components, deadlock pair): oracle in seconds
 C3_SMALL = C3.scaled("C3-small", n_samples=9_000_000, n_events=1_000_000, n_windows=100,
-                     deadlock=((60, (11240, 11243)), (65, (11236, 11250))))
-# C4: 1M buffers, Zipf(0.99) hot spots (YCSB-style exponent; BASELINE.json gives none), k = 1024
-C4 = Workload("C4-skewed", 1_800_000_000, 200_000_000, 1 << 20, 64, 2000, 1024, 16, seed=4, zipf_s=0.99,
+                     deadlock=((40, (11240, 11243)), (45, (11236, 11250))))
+# C4: 1M buffers, Zipf(0.99) hot spots (YCSB-style exponent; BASELINE.json gives none), k = 1024.
+# H = 96: the smallest of {16, 32, 48, 64, 96} at which the trace flags nothing (cold buffers held
+# full between rare samples in quiet components; tools/calibrate_h.py: 593 at 32, 1 at 64, 0 at 96)
+C4 = Workload("C4-skewed", 1_800_000_000, 200_000_000, 1 << 20, 64, 2000, 1024, 96, seed=4, zipf_s=0.99,
               description="skewed trace: 1M buffers, Zipf-distributed buffer_id hot spots, 2B records, top-k=1024")
 C4_SMALL = C4.scaled("C4-small", n_samples=18_000_000, n_events=2_000_000, n_windows=20)
 # C5: recorded for the next round (1M windows needs the sparse-window path)
