@@ -50,6 +50,7 @@ struct rtm_ctx {
   int n_sms;
   DevBuf cap, owner, elig, ktotal, rcp, elig_ids;
   DevBuf gid, bstat_g;      // rank-local numbering: global id per local buffer, table by global id
+  DevBuf tkscr;             // per-slice top-k candidates (few-window calls)
   uint32_t n_global = 0, pack_nb = 0;
   uint32_t n_elig = 0;
   // persistent state
@@ -367,6 +368,11 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   if ((s = ensure(c, c->hung, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->unit_ctr, 8))) return s;
   if ((s = ensure(c, c->bstat, (size_t)c->nb * sizeof(rtm_buffer_stat)))) return s;
+  p.tk_slices = topk_slices(c->nb, c->k, W, c->n_sms, c->n_elig == c->nb, &p.tk_slice_len);
+  if (p.tk_slices > 1) {
+    if ((s = ensure(c, c->tkscr, (size_t)W * p.tk_slices * c->k * 8))) return s;
+    p.tk_scratch = (unsigned long long *)c->tkscr.p;
+  }
   if ((s = ensure(c, c->comps, (size_t)c->nc * sizeof(rtm_component_tasks)))) return s;
 
   {

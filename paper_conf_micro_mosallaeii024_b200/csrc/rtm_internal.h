@@ -119,6 +119,9 @@ struct Params {
   long long *cstart, *cend;  // [nc] cumulative
   unsigned long long *topk;  // [W * k] packed (id | level<<32 | cap<<48)
   uint32_t *topk_n;          // [W]
+  uint32_t tk_slices;        // top-k slices per window (> 1: few windows, K5 runs per id slice)
+  uint32_t tk_slice_len;     // buffers per slice (multiple of 8)
+  unsigned long long *tk_scratch;  // [W * tk_slices * k] per-slice candidates (key32 << 32 | ~id)
   long long *prog;           // [W * nk * 5]
   rtm_buffer_stat *bstat;    // [nb] last window, local ids
   rtm_buffer_stat *bstat_g;  // [n_global] merged / scattered table by global id (gid set)
@@ -135,6 +138,8 @@ void launch_events(const Params &p, cudaStream_t st);
 void launch_fold(const Params &p, int n_sms, cudaStream_t st);
 void launch_order_check(const Params &p, cudaStream_t st);
 void launch_topk(const Params &p, cudaStream_t st);
+// slices per window for K5 (1 = one CTA per window); sets *slice_len
+uint32_t topk_slices(uint32_t nb, uint32_t k, uint32_t W, int n_sms, bool all, uint32_t *slice_len);
 void launch_hang(const Params &p, cudaStream_t st);
 void launch_progress(const Params &p, cudaStream_t st);
 // multi-rank exchange

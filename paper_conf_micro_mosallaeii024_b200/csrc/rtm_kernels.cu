@@ -7,6 +7,7 @@
 
 #include <type_traits>
 
+#include <algorithm>
 #include <atomic>
 
 #include "rtm_internal.h"
@@ -1194,10 +1195,10 @@ __device__ __forceinline__ unsigned fullness_key(unsigned l, unsigned c, int mod
 template <bool ALL>
 __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
-  const unsigned ne = ALL ? p.nb : p.n_elig;  // ranked buffers (ids ascending)
-  const bool keys_in_smem = ne <= kTopkSmemKeys;
+  const unsigned key_cap = ALL ? p.tk_slice_len : p.n_elig;  // keys one CTA ranks at most
+  const bool keys_in_smem = key_cap <= kTopkSmemKeys;
   unsigned *keys = reinterpret_cast<unsigned *>(smem);                                  // [ne] or none
-  unsigned *hist = keys + (keys_in_smem ? ((ne + 1) & ~1u) : 0);                        // [8][256]
+  unsigned *hist = keys + (keys_in_smem ? ((key_cap + 1) & ~1u) : 0);                        // [8][256]
   unsigned long long *sel = reinterpret_cast<unsigned long long *>(hist + 8 * 256);     // [1024]
   unsigned *cand = reinterpret_cast<unsigned *>(sel + 1024);                             // [kTopkCand]
   __shared__ unsigned scan_scratch[32];
@@ -1205,7 +1206,12 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
   const unsigned w = blockIdx.x;
   const uint16_t *lv = p.lastlvl + (size_t)w * p.nb;
   const int warp = threadIdx.x >> 5;
-  auto id_of = [&](unsigned i) -> unsigned { return ALL ? i : __ldg(p.elig_ids + i); };
+  // few windows (streaming): the buffers of a window are split into id slices, one CTA each;
+  // every slice keeps its own top-k candidates and k_topk_merge ranks their union (exact: the
+  // global top-k is contained in the union of the slices' top-k)
+  const unsigned slo = ALL ? blockIdx.y * p.tk_slice_len : 0u;
+  const unsigned ne = ALL ? min(p.nb - slo, p.tk_slice_len) : p.n_elig;  // ranked buffers (ids ascending)
+  auto id_of = [&](unsigned i) -> unsigned { return ALL ? slo + i : __ldg(p.elig_ids + i); };
   auto key_at = [&](unsigned i) -> unsigned {
     if (keys_in_smem) return keys[i];
     const unsigned b = id_of(i);
@@ -1221,8 +1227,8 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     tc += (k == tm);
   };
   if (keys_in_smem && ALL && (p.nb & 7u) == 0) {  // 8 consecutive buffers per thread: 16-B loads
-    const uint4 *lv4 = reinterpret_cast<const uint4 *>(lv);
-    const uint4 *cp4 = reinterpret_cast<const uint4 *>(p.cap);
+    const uint4 *lv4 = reinterpret_cast<const uint4 *>(lv + slo);  // slices start at multiples of 8
+    const uint4 *cp4 = reinterpret_cast<const uint4 *>(p.cap + slo);
     uint4 *k4 = reinterpret_cast<uint4 *>(keys);
 #pragma unroll 2
     for (unsigned g = threadIdx.x; g < ne / 8; g += blockDim.x) {
@@ -1257,8 +1263,12 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     if ((threadIdx.x & 31) == 0 && wm == s_max && wc) atomicAdd(&s_cnt_max, wc);
     __syncthreads();
   }
+  const bool sliced = ALL && p.tk_slices > 1;
+  unsigned long long *scr = sliced ? p.tk_scratch + ((size_t)w * p.tk_slices + blockIdx.y) * p.k : nullptr;
   if (keff == 0) {
-    if (threadIdx.x == 0) p.topk_n[w] = 0;
+    if (threadIdx.x == 0 && !sliced) p.topk_n[w] = 0;
+    if (sliced)
+      for (unsigned i = threadIdx.x; i < p.k; i += blockDim.x) scr[i] = 0ull;
     return;
   }
   // Shortcut: when the largest key is held by >= k buffers (e.g. >= k buffers are 100 % full, the
@@ -1351,6 +1361,10 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     }
   }
   __syncthreads();
+  if (sliced) {  // this slice's candidates (unsorted); k_topk_merge ranks the union
+    for (unsigned i = threadIdx.x; i < p.k; i += blockDim.x) scr[i] = i < keff ? sel[i] : 0ull;
+    return;
+  }
   // bitonic sort descending over the next power of two >= keff (top tie: the winners share one
   // key and were written in id order, so they are already sorted)
   unsigned P = 1;
@@ -1374,6 +1388,45 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     unsigned long long out = 0xFFFFFFFFull;  // buffer_id 0xFFFFFFFF, level 0, cap 0
     if (i < keff) {
       unsigned b = 0xFFFFFFFFu - (unsigned)(sel[i] & 0xFFFFFFFFu);
+      out = (unsigned long long)(p.gid ? __ldg(p.gid + b) : b) | ((unsigned long long)lv[b] << 32) |
+            ((unsigned long long)__ldg(p.cap + b) << 48);
+    }
+    p.topk[(size_t)w * p.k + i] = out;
+  }
+  if (threadIdx.x == 0) p.topk_n[w] = keff;
+}
+
+// One CTA per window: the union of the slices' candidates (composite key32 << 32 | ~id, padding
+// 0 ranks last) bitonic-sorted descending; the first min(k, nb) are the window's top-k.
+constexpr unsigned kTopkMergeMax = 4096;
+__global__ void __launch_bounds__(1024) k_topk_merge(Params p) {
+  __shared__ unsigned long long v[kTopkMergeMax];
+  const unsigned w = blockIdx.x;
+  const unsigned n = p.tk_slices * p.k;
+  unsigned P = 1;
+  while (P < n) P <<= 1;
+  const unsigned long long *src = p.tk_scratch + (size_t)w * n;
+  for (unsigned i = threadIdx.x; i < P; i += blockDim.x) v[i] = i < n ? src[i] : 0ull;
+  __syncthreads();
+  for (unsigned size = 2; size <= P; size <<= 1) {
+    for (unsigned stride = size >> 1; stride > 0; stride >>= 1) {
+      for (unsigned i = threadIdx.x; i < P; i += blockDim.x) {
+        const unsigned jx = i ^ stride;
+        if (jx > i) {
+          const bool desc = (i & size) == 0;
+          const unsigned long long a = v[i], b = v[jx];
+          if ((a < b) == desc) { v[i] = b; v[jx] = a; }
+        }
+      }
+      __syncthreads();
+    }
+  }
+  const unsigned keff = p.k < p.nb ? p.k : p.nb;
+  const uint16_t *lv = p.lastlvl + (size_t)w * p.nb;
+  for (unsigned i = threadIdx.x; i < p.k; i += blockDim.x) {
+    unsigned long long out = 0xFFFFFFFFull;  // buffer_id 0xFFFFFFFF, level 0, cap 0
+    if (i < keff) {
+      const unsigned b = 0xFFFFFFFFu - (unsigned)(v[i] & 0xFFFFFFFFu);
       out = (unsigned long long)(p.gid ? __ldg(p.gid + b) : b) | ((unsigned long long)lv[b] << 32) |
             ((unsigned long long)__ldg(p.cap + b) << 48);
     }
@@ -1728,7 +1781,26 @@ void launch_order_check(const Params &p, cudaStream_t st) {
   { k_order_check<<<blocks, 256, 0, st>>>(p); count_launch(); }
 }
 
+uint32_t topk_slices(uint32_t nb, uint32_t k, uint32_t W, int n_sms, bool all, uint32_t *slice_len) {
+  uint32_t P = 1;
+  if (all && (nb & 7u) == 0 && W < (uint32_t)n_sms) {
+    P = (2u * (uint32_t)n_sms + W - 1) / W;
+    P = std::min(P, nb / 2048u);
+    P = std::min(P, std::max(2u, 1024u / k));  // merge sorts <= max(1024, 2k) candidates
+    if (P < 2) P = 1;
+  }
+  uint32_t L = P > 1 ? (((nb + P - 1) / P + 7) & ~7u) : nb;
+  if (P > 1) P = (nb + L - 1) / L;
+  *slice_len = L;
+  return P;
+}
+
 void launch_topk(const Params &p, cudaStream_t st) {
+  if (p.n_elig == p.nb && p.tk_slices > 1) {
+    { k_topk<true><<<dim3(p.W, p.tk_slices), kTopkThreads, topk_smem_bytes(p.tk_slice_len), st>>>(p); count_launch(); }
+    { k_topk_merge<<<p.W, 1024, 0, st>>>(p); count_launch(); }
+    return;
+  }
   if (p.n_elig == p.nb) { k_topk<true><<<p.W, kTopkThreads, topk_smem_bytes(p.nb), st>>>(p); count_launch(); }
   else { k_topk<false><<<p.W, kTopkThreads, topk_smem_bytes(p.n_elig), st>>>(p); count_launch(); }
 }

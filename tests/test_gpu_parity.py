@@ -412,3 +412,28 @@ def test_many_bins_partition_paths(n_buffers):
     mon.ingest(_dev(s), _dev(e))
     got = mon.window_reduce(wl.t_end())
     assert_same(got, ref, mon)
+
+
+@pytest.mark.parametrize("n_buffers,k,calls", [(20480, 64, (1, 1, 3, 37, 1)), (65536, 1024, (1, 2)),
+                                                (16384, 16, (5, 1)), (20482, 64, (1, 2))])
+def test_topk_slices_few_window_calls(n_buffers, k, calls):
+    """Calls with fewer windows than SMs split each window's buffers into id slices (one top-k
+    CTA per slice, then a merge of the slices' candidates); every call must still equal the
+    oracle's full sort (n_buffers not a multiple of 8 takes the one-CTA path)."""
+    n_win = sum(calls)
+    wl = gen.C1.scaled("C1-slices", n_samples=600_000, n_events=60_000, n_buffers=n_buffers, n_windows=n_win, k=k)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=k)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    s, e = gen.samples(wl), gen.events(wl)
+    t_end = wl.t_end()
+    w0 = 0
+    for m in calls:
+        w1 = w0 + m
+        sl = slice(wl.index_at("samples", wl.t_begin(w0)), wl.index_at("samples", wl.t_begin(w1)))
+        el = slice(wl.index_at("events", wl.t_begin(w0)), wl.index_at("events", wl.t_begin(w1)))
+        ref = orc.reduce(s[sl], e[el], t_end[w0:w1])
+        mon.ingest(_dev(s[sl]), _dev(e[el]))
+        got = mon.window_reduce(t_end[w0:w1])
+        assert_same(got, ref, mon)
+        w0 = w1

@@ -51,7 +51,19 @@ for w in range(W):
         recs += (s1 - s0) + (e1 - e0)
     assert int(res["summary"]["n_dropped"][0]) == 0
 lat = np.array(lat) * 1e6
+# per-kernel device time of a call (CUDA events around each launch, library profiler)
+mon.profile(True)
+n_prof = min(200, W)
+mon.reset()
+for w in range(n_prof):
+    s0, s1 = wl.index_at("samples", wl.t_begin(w)), wl.index_at("samples", wl.t_begin(w + 1))
+    e0, e1 = wl.index_at("events", wl.t_begin(w)), wl.index_at("events", wl.t_begin(w + 1))
+    mon.ingest(ds[s0 * 16:s1 * 16], de[e0 * 16:e1 * 16])
+    mon.window_reduce(t_end[w:w + 1])
+prof = {k: round(v["total_ms"] * 1e3 / n_prof, 2) for k, v in mon.profile_read().items() if v["launches"]}
+mon.profile(False)
 print(json.dumps({"what": "per-window snapshot latency, one window per call (streaming)", "config": wl.name,
                   "n_buffers": wl.n_buffers, "windows": args.windows, "records_per_window": recs / args.windows,
                   "p50_us": float(np.percentile(lat, 50)), "p99_us": float(np.percentile(lat, 99)),
-                  "mean_us": float(lat.mean()), "records_per_s": recs / (lat.sum() / 1e6)}))
+                  "mean_us": float(lat.mean()), "records_per_s": recs / (lat.sum() / 1e6),
+                  "kernel_us_per_call": prof}))
