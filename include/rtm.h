@@ -193,6 +193,28 @@ rtm_status rtm_window_reduce_local(rtm_ctx *ctx, const int64_t *t_end, uint32_t 
                                    const void **pack, uint64_t *pack_bytes);
 rtm_status rtm_merge(rtm_ctx *ctx, const void *gathered, uint32_t world, rtm_window_summary *out);
 
+/* ---- Value monitor (§IV-C.3, Fig. 2 F) ----------
+ * The dashboard plots "up to five values" over time and keeps "the last 300 data points"
+ * (L175, L179).  Here a watched buffer's value per window is its rtm_buffer_stat of that window
+ * (last / max / min level, integral, mean occupancy): every window of every reduce appends one
+ * point per watched buffer to that buffer's ring of the last RTM_WATCH_POINTS windows.  The
+ * points are produced by the fold kernel in the same pass as the snapshot (no extra pass over
+ * the records) and copied back with the call's results.  With world > 1 a ring fills on the
+ * rank that owns the buffer; the other ranks' rings for it stay empty. */
+enum { RTM_WATCH_MAX = 5, RTM_WATCH_POINTS = 300 };
+typedef struct {
+  int64_t t_end;                    /* end of the window the point describes                  */
+  rtm_buffer_stat stat;             /* that window's statistics of the watched buffer         */
+} rtm_watch_point;                  /* 40 B */
+/* Replace the watched set by buffer_ids[0..n) (n <= RTM_WATCH_MAX, distinct, < n_buffers;
+ * global ids with a rank-local numbering) and clear every ring; n = 0 stops watching.
+ * RTM_E_INVALID (no state change) for n > RTM_WATCH_MAX, duplicates or out-of-range ids. */
+rtm_status rtm_watch(rtm_ctx *ctx, const uint32_t *buffer_ids, uint32_t n);
+/* The ring of watched slot `slot` (order given to rtm_watch), oldest point first:
+ * out[RTM_WATCH_POINTS] (host) receives min(points so far, RTM_WATCH_POINTS) points,
+ * *n_out that count.  RTM_E_INVALID for slot >= the watched count. */
+rtm_status rtm_watch_series(rtm_ctx *ctx, uint32_t slot, rtm_watch_point *out, uint32_t *n_out);
+
 /* Per-kernel CUDA-event timing on the context stream (off by default). */
 rtm_status rtm_profile(rtm_ctx *ctx, int32_t enable);
 rtm_status rtm_profile_read(rtm_ctx *ctx, rtm_kernel_time *out, uint32_t cap, uint32_t *n);

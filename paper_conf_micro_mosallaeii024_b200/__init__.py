@@ -191,6 +191,18 @@ class Monitor:
         N.check(N.lib().rtm_buffer_stats(self._h, first, count, out.ctypes.data), "rtm_buffer_stats")
         return out
 
+    def watch(self, buffer_ids):
+        """Value monitor: watch up to 5 buffers; clears the rings."""
+        ids = np.ascontiguousarray(buffer_ids, dtype=np.uint32)
+        N.check(N.lib().rtm_watch(self._h, ids.ctypes.data if len(ids) else None, len(ids)), "rtm_watch")
+
+    def watch_series(self, slot: int):
+        """Points of watched slot `slot` (last <= 300 windows, oldest first): t_end + window stats."""
+        out = np.zeros(N.RTM_WATCH_POINTS, N.WATCH_DTYPE)
+        n = ctypes.c_uint32()
+        N.check(N.lib().rtm_watch_series(self._h, slot, out.ctypes.data, ctypes.byref(n)), "rtm_watch_series")
+        return out[: n.value]
+
     def profile(self, enable: bool = True):
         N.check(N.lib().rtm_profile(self._h, 1 if enable else 0), "rtm_profile")
 

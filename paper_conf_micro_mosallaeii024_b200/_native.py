@@ -30,6 +30,11 @@ COMP_DTYPE = np.dtype([("started", "<i8"), ("finished", "<i8"), ("in_flight", "<
 BSTAT_DTYPE = np.dtype([("integral", "<i8"), ("last", "<u2"), ("max", "<u2"), ("min", "<u2"), ("capacity", "<u2"),
                         ("n_samples", "<u4"), ("reserved", "<u4"), ("mean_occ", "<f8")])
 
+WATCH_DTYPE = np.dtype([("t_end", "<i8"), ("integral", "<i8"), ("last", "<u2"), ("max", "<u2"), ("min", "<u2"),
+                        ("capacity", "<u2"), ("n_samples", "<u4"), ("reserved", "<u4"), ("mean_occ", "<f8")])
+assert WATCH_DTYPE.itemsize == 40
+RTM_WATCH_MAX, RTM_WATCH_POINTS = 5, 300
+
 ALLGATHER_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64)
 
 
@@ -55,7 +60,7 @@ class KernelTime(ctypes.Structure):
 EXPORTS = ("rtm_create", "rtm_destroy", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers",
            "rtm_progress", "rtm_hang_check", "rtm_buffer_stats", "rtm_window_results", "rtm_window_reduce_local",
            "rtm_merge", "rtm_profile", "rtm_profile_read", "rtm_status_str", "rtm_version",
-           "rtm_kernel_launches")
+           "rtm_kernel_launches", "rtm_watch", "rtm_watch_series")
 
 _lib = None
 
@@ -85,7 +90,9 @@ def lib():
     L.rtm_merge.argtypes = [vp, vp, u32, vp]
     L.rtm_profile.argtypes = [vp, i32]
     L.rtm_profile_read.argtypes = [vp, vp, u32, P(u32)]
-    for fn in ("rtm_create", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers", "rtm_progress",
+    L.rtm_watch.argtypes = [vp, vp, u32]
+    L.rtm_watch_series.argtypes = [vp, u32, vp, P(u32)]
+    for fn in ("rtm_watch", "rtm_watch_series", "rtm_create", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers", "rtm_progress",
                "rtm_hang_check", "rtm_buffer_stats", "rtm_window_reduce_local", "rtm_merge", "rtm_profile",
                "rtm_profile_read", "rtm_window_results"):
         getattr(L, fn).restype = ctypes.c_int

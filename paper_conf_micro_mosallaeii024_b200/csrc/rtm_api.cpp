@@ -51,6 +51,12 @@ struct rtm_ctx {
   DevBuf cap, owner, elig, ktotal, rcp, elig_ids;
   DevBuf gid, bstat_g;      // rank-local numbering: global id per local buffer, table by global id
   DevBuf tkscr;             // per-slice top-k candidates (few-window calls)
+  // value monitor: watched ids (as given), their local ids (~0: not on this rank), rings
+  std::vector<uint32_t> gid_h;  // host copy of the global ids (rank-local numbering)
+  uint32_t n_watch = 0;
+  uint32_t watch_ids[RTM_WATCH_MAX] = {0}, watch_local[RTM_WATCH_MAX] = {0};
+  std::vector<rtm_watch_point> ring[RTM_WATCH_MAX];
+  uint32_t ring_head[RTM_WATCH_MAX] = {0}, ring_n[RTM_WATCH_MAX] = {0};
   uint32_t n_global = 0, pack_nb = 0;
   uint32_t n_elig = 0;
   // persistent state
@@ -274,7 +280,7 @@ rtm_status append(rtm_ctx *c, std::vector<Chunk> &dev, DevBuf &own, uint64_t &ow
 // Per-call results, one device buffer and one pinned host buffer of the same layout (a single
 // D2H copy per call): window fields | top-k | progress | top-k counts | status.
 struct ResLayout {
-  size_t win, topk, prog, topk_n, status, bytes;
+  size_t win, topk, prog, topk_n, status, watch, bytes;
 };
 ResLayout res_layout(const rtm_ctx *c, uint32_t W) {
   ResLayout L;
@@ -283,7 +289,8 @@ ResLayout res_layout(const rtm_ctx *c, uint32_t W) {
   L.prog = L.topk + (size_t)W * c->k * 8;
   L.topk_n = L.prog + (size_t)W * c->nk * 5 * 8;
   L.status = L.topk_n + (((size_t)W * 4 + 15) & ~(size_t)15);
-  L.bytes = L.status + 16;
+  L.watch = L.status + 16;  // value monitor points, only while buffers are watched
+  L.bytes = L.watch + (c->n_watch ? (size_t)W * RTM_WATCH_MAX * sizeof(rtm_buffer_stat) : 0);
   return L;
 }
 void set_result_ptrs(rtm_ctx *c, uint32_t W, Params &p) {
@@ -294,6 +301,9 @@ void set_result_ptrs(rtm_ctx *c, uint32_t W, Params &p) {
   p.prog = (long long *)(d + L.prog);
   p.topk_n = (uint32_t *)(d + L.topk_n);
   p.status = (uint32_t *)(d + L.status);
+  p.n_watch = c->n_watch;
+  for (uint32_t q = 0; q < RTM_WATCH_MAX; ++q) p.watch[q] = q < c->n_watch ? c->watch_local[q] : 0xFFFFFFFFu;
+  p.wstat = (rtm_buffer_stat *)(d + L.watch);
 }
 
 rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p) {
@@ -485,6 +495,21 @@ rtm_status finish(rtm_ctx *c, const int64_t *t_end, uint32_t W, rtm_window_summa
     S.n_touched = (uint32_t)hwin[WF_TOUCHED * Wn + w];
     S.n_hung = (uint32_t)hwin[WF_HUNG * Wn + w];
   }
+  if (c->n_watch) {  // value monitor: append this batch's points to the rings
+    const rtm_buffer_stat *hw = (const rtm_buffer_stat *)(h + L.watch);
+    for (uint32_t q = 0; q < c->n_watch; ++q) {
+      if (c->watch_local[q] == 0xFFFFFFFFu) continue;
+      std::vector<rtm_watch_point> &r = c->ring[q];
+      if (r.size() != RTM_WATCH_POINTS) r.assign(RTM_WATCH_POINTS, rtm_watch_point());
+      for (uint32_t w = 0; w < W; ++w) {
+        rtm_watch_point &pt = r[(c->ring_head[q] + c->ring_n[q]) % RTM_WATCH_POINTS];
+        pt.t_end = t_end[w];
+        pt.stat = hw[(size_t)w * RTM_WATCH_MAX + q];
+        if (c->ring_n[q] < RTM_WATCH_POINTS) ++c->ring_n[q];
+        else c->ring_head[q] = (c->ring_head[q] + 1) % RTM_WATCH_POINTS;
+      }
+    }
+  }
   c->topk_h = htopk;
   c->topk_n_h = htopk_n;
   c->prog_h = reinterpret_cast<const rtm_progress_entry *>(hprog);
@@ -562,6 +587,7 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   c->t0 = cfg->t0;
   c->t_prev = cfg->t0;
   c->n_global = cfg->buffer_global_id ? cfg->n_global_buffers : 0;
+  if (cfg->buffer_global_id) c->gid_h.assign(cfg->buffer_global_id, cfg->buffer_global_id + c->nb);
   c->pack_nb = cfg->pack_buffers ? cfg->pack_buffers : cfg->n_buffers;
   c->allgather = cfg->allgather;
   c->allgather_user = cfg->allgather_user;
@@ -652,7 +678,38 @@ rtm_status rtm_reset(rtm_ctx *c) {
   cudaStreamSynchronize(c->st);
   cudaGetLastError();
   c->sticky = 0;
+  for (uint32_t q = 0; q < RTM_WATCH_MAX; ++q) c->ring_head[q] = c->ring_n[q] = 0;
   return zero_state(c);
+}
+
+rtm_status rtm_watch(rtm_ctx *c, const uint32_t *ids, uint32_t n) {
+  if (!c || n > RTM_WATCH_MAX || (n && !ids)) return RTM_E_INVALID;
+  const uint32_t space = c->gid.p ? c->n_global : c->nb;
+  for (uint32_t q = 0; q < n; ++q) {
+    if (ids[q] >= space) return RTM_E_INVALID;
+    for (uint32_t r = 0; r < q; ++r)
+      if (ids[r] == ids[q]) return RTM_E_INVALID;
+  }
+  for (uint32_t q = 0; q < n; ++q) {
+    uint32_t loc = ids[q];
+    if (c->gid.p) {  // rank-local numbering: the local buffer with this global id, if any
+      auto it = std::lower_bound(c->gid_h.begin(), c->gid_h.end(), ids[q]);
+      loc = (it != c->gid_h.end() && *it == ids[q]) ? (uint32_t)(it - c->gid_h.begin()) : 0xFFFFFFFFu;
+    }
+    c->watch_ids[q] = ids[q];
+    c->watch_local[q] = loc;
+  }
+  c->n_watch = n;
+  for (uint32_t q = 0; q < RTM_WATCH_MAX; ++q) c->ring_head[q] = c->ring_n[q] = 0;
+  return RTM_OK;
+}
+
+rtm_status rtm_watch_series(rtm_ctx *c, uint32_t slot, rtm_watch_point *out, uint32_t *n_out) {
+  if (!c || !out || !n_out || slot >= c->n_watch) return RTM_E_INVALID;
+  const uint32_t n = c->ring_n[slot];
+  for (uint32_t i = 0; i < n; ++i) out[i] = c->ring[slot][(c->ring_head[slot] + i) % RTM_WATCH_POINTS];
+  *n_out = n;
+  return RTM_OK;
 }
 
 rtm_status rtm_ingest(rtm_ctx *c, const rtm_level_sample *samples, uint64_t n_samples, const rtm_task_event *events,

@@ -126,6 +126,9 @@ struct Params {
   rtm_buffer_stat *bstat;    // [nb] last window, local ids
   rtm_buffer_stat *bstat_g;  // [n_global] merged / scattered table by global id (gid set)
   rtm_component_tasks *comps;// [nc]
+  uint32_t n_watch;          // value monitor: watched local buffer ids (0xFFFFFFFF: not on this rank)
+  uint32_t watch[RTM_WATCH_MAX];
+  rtm_buffer_stat *wstat;    // [W * RTM_WATCH_MAX] per-window statistics of the watched buffers
   unsigned long long *dbg;   // phase-timing scratch (RTM_PHASE_TIMING builds only)
 };
 

@@ -1115,7 +1115,10 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
         dig += h;
         ++touched;
       }
-      if (last_window) {
+      int wq = -1;  // value monitor slot of b (at most RTM_WATCH_MAX compares, usually none)
+      for (unsigned q = 0; q < p.n_watch; ++q)
+        if (p.watch[q] == b) wq = (int)q;
+      if (last_window || wq >= 0) {
         rtm_buffer_stat st;
         st.integral = (int64_t)I;
         st.last = (uint16_t)last;
@@ -1125,8 +1128,11 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
         st.n_samples = cnt;
         st.reserved = __ldg(p.elig + b);
         st.mean_occ = Wlen ? __ddiv_rn((double)(long long)I, (double)((long long)capb * (long long)Wlen)) : 0.0;
-        p.bstat[b] = st;
-        p.carry_out[b] = (uint16_t)last;
+        if (wq >= 0) p.wstat[(size_t)w * RTM_WATCH_MAX + wq] = st;
+        if (last_window) {
+          p.bstat[b] = st;
+          p.carry_out[b] = (uint16_t)last;
+        }
       }
     }
     dig = warp_sum(dig);

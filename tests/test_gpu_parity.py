@@ -437,3 +437,46 @@ def test_topk_slices_few_window_calls(n_buffers, k, calls):
         got = mon.window_reduce(t_end[w0:w1])
         assert_same(got, ref, mon)
         w0 = w1
+
+
+def test_value_monitor_rings_last_300_windows():
+    """Value monitor (up to 5 values, the last 300 points): 5 watched buffers
+    over 400 windows in 40 calls; each ring holds the last 300 windows' statistics of its
+    buffer, equal to the oracle's per-window table; invalid watch sets are rejected."""
+    wl = gen.C1.scaled("C1-watch", n_samples=400_000, n_events=40_000, n_windows=400)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    ids = [0, 7, 999, 500, 123]
+    with pytest.raises(RTMError):
+        mon.watch(list(range(6)))
+    with pytest.raises(RTMError):
+        mon.watch([3, 3])
+    with pytest.raises(RTMError):
+        mon.watch([wl.n_buffers])
+    mon.watch(ids)
+    s, e = gen.samples(wl), gen.events(wl)
+    t_end = wl.t_end()
+    ref_rows = []
+    for w0 in range(0, wl.n_windows, 10):
+        w1 = w0 + 10
+        sl = slice(wl.index_at("samples", wl.t_begin(w0)), wl.index_at("samples", wl.t_begin(w1)))
+        el = slice(wl.index_at("events", wl.t_begin(w0)), wl.index_at("events", wl.t_begin(w1)))
+        ref = orc.reduce(s[sl], e[el], t_end[w0:w1], want_all_stats=True)
+        ref_rows.append(ref["all_stats"])
+        mon.ingest(_dev(s[sl]), _dev(e[el]))
+        mon.window_reduce(t_end[w0:w1])
+        if w0 == 0:
+            assert len(mon.watch_series(0)) == 10
+    A = np.concatenate(ref_rows)  # [400, n_buffers]
+    for q, b in enumerate(ids):
+        ser = mon.watch_series(q)
+        assert len(ser) == 300
+        assert np.array_equal(ser["t_end"], t_end[100:])
+        for f in ("integral", "last", "max", "min", "capacity", "n_samples", "mean_occ"):
+            assert np.array_equal(ser[f], A[100:, b][f]), (b, f)
+    mon.reset()
+    assert len(mon.watch_series(0)) == 0
+    mon.watch([])
+    with pytest.raises(RTMError):
+        mon.watch_series(0)
