@@ -57,6 +57,8 @@ def lib():
         L.orc_digest_term.restype = u64
         L.orc_merge_topk.argtypes = [vp, vp, u32, u32, u32, ctypes.c_int32, vp, vp]
         L.orc_merge_topk.restype = ctypes.c_int
+        L.orc_persistence.argtypes = [vp, vp]
+        L.orc_persistence.restype = None
         _lib = L
     return _lib
 
@@ -95,6 +97,12 @@ class Oracle:
 
     def reset(self):
         lib().orc_reset(self._h)
+
+    def persistence(self):
+        """Per buffer: windows (since create / reset) in which it was in the top-k list."""
+        out = np.zeros(self.n_buffers, np.uint32)
+        lib().orc_persistence(self._h, out.ctypes.data)
+        return out
 
     def reduce(self, samples, events, t_end, *, want_hung=True, want_all_stats=False, want_topk=True):
         samples = np.ascontiguousarray(samples)

@@ -153,6 +153,9 @@ class Brute:
             elig = [b for b in range(self.nb) if self.owned[self.owner[b]]]
             if self.mode == 0:
                 order = sorted(elig, key=lambda b: (-Fraction(self.lvl[b], self.cap[b]), b))
+            elif self.mode == 2:  # the window's mean occupancy: tick-loop integral / (cap * W)
+                order = sorted(elig, key=lambda b: (-(Fraction(stats[b]["integral"], self.cap[b] * (te - tp))
+                                                      if te > tp else Fraction(0)), b))
             else:
                 order = sorted(elig, key=lambda b: (-self.lvl[b], b))
             top = [(b, self.lvl[b], self.cap[b]) for b in order[: self.k]]

@@ -25,6 +25,7 @@ struct orc_ctx {
   uint16_t *lvl;       /* level of every buffer at the end of the last reduced window */
   int64_t *c_started, *c_ended, *k_started, *k_ended;
   uint32_t *run;       /* consecutive windows with cond_c true */
+  uint32_t *persist;   /* per buffer: windows in which it was in the top-k list */
   int sticky;
 };
 
@@ -77,6 +78,7 @@ orc_ctx *orc_create(const orc_config *cfg) {
   c->k_started = (int64_t *)malloc(sizeof(int64_t) * c->nk);
   c->k_ended = (int64_t *)malloc(sizeof(int64_t) * c->nk);
   c->run = (uint32_t *)malloc(sizeof(uint32_t) * c->nc);
+  c->persist = (uint32_t *)malloc(sizeof(uint32_t) * (c->nb ? c->nb : 1));
   orc_reset(c);
   return c;
 }
@@ -89,13 +91,14 @@ void orc_reset(orc_ctx *c) {
   memset(c->k_started, 0, sizeof(int64_t) * c->nk);
   memset(c->k_ended, 0, sizeof(int64_t) * c->nk);
   memset(c->run, 0, sizeof(uint32_t) * c->nc);
+  memset(c->persist, 0, sizeof(uint32_t) * c->nb);
   c->sticky = 0;
 }
 
 void orc_destroy(orc_ctx *c) {
   if (!c) return;
   free(c->owner); free(c->cap); free(c->ktotal); free(c->owned); free(c->lvl);
-  free(c->c_started); free(c->c_ended); free(c->k_started); free(c->k_ended); free(c->run);
+  free(c->c_started); free(c->c_ended); free(c->k_started); free(c->k_ended); free(c->run); free(c->persist);
   free(c);
 }
 
@@ -112,10 +115,19 @@ static uint32_t window_of(const int64_t *t_end, uint32_t W, int64_t ts) {
 /* Bottleneck Analyzer order: fullness percentage (or element count),
  * descending; equal fullness -> buffer_id ascending.  Ratios compared exactly by
  * cross-multiplication: a.l/a.c > b.l/b.c  <=>  a.l*b.c > b.l*a.c. */
-typedef struct { uint32_t id; uint16_t l, c; } rank_item;
+typedef struct { uint32_t id; uint16_t l, c; uint64_t I; } rank_item;
 static int cmp_percent(const void *pa, const void *pb) {
   const rank_item *a = (const rank_item *)pa, *b = (const rank_item *)pb;
   uint64_t x = (uint64_t)a->l * b->c, y = (uint64_t)b->l * a->c;
+  if (x != y) return x > y ? -1 : 1;
+  return a->id < b->id ? -1 : (a->id > b->id ? 1 : 0);
+}
+/* Persistence ranking ("repeatedly at the top", L173, L197-L199): the
+ * window's time-weighted mean occupancy I / (cap * W), descending; within one window W is
+ * common, so I_a/c_a > I_b/c_b  <=>  I_a*c_b > I_b*c_a (128-bit products, exact). */
+static int cmp_mean(const void *pa, const void *pb) {
+  const rank_item *a = (const rank_item *)pa, *b = (const rank_item *)pb;
+  unsigned __int128 x = (unsigned __int128)a->I * b->c, y = (unsigned __int128)b->I * a->c;
   if (x != y) return x > y ? -1 : 1;
   return a->id < b->id ? -1 : (a->id > b->id ? 1 : 0);
 }
@@ -300,9 +312,12 @@ int orc_reduce(orc_ctx *c, const orc_sample *s, uint64_t ns, const orc_event *e,
     if (topk || topk_n) {
       uint32_t m = 0;
       for (uint32_t b = 0; b < nb; ++b)
-        if (c->owned[c->owner[b]]) { items[m].id = b; items[m].l = c->lvl[b]; items[m].c = c->cap[b]; ++m; }
-      qsort(items, m, sizeof(rank_item), c->rank_mode == 1 ? cmp_size : cmp_percent);
+        if (c->owned[c->owner[b]]) {
+          items[m].id = b; items[m].l = c->lvl[b]; items[m].c = c->cap[b]; items[m].I = I[b]; ++m;
+        }
+      qsort(items, m, sizeof(rank_item), c->rank_mode == 1 ? cmp_size : c->rank_mode == 2 ? cmp_mean : cmp_percent);
       uint32_t kk = c->k < m ? c->k : m;
+      for (uint32_t i = 0; i < kk; ++i) c->persist[items[i].id]++;
       if (topk_n) topk_n[w] = kk;
       if (topk)
         for (uint32_t i = 0; i < c->k; ++i) {
@@ -359,4 +374,9 @@ int orc_merge_topk(const orc_topk *const *shard_topk, const uint32_t *const *sha
   }
   free(items);
   return 0;
+}
+
+/* Windows-in-top-k counter of every buffer since create / reset. */
+void orc_persistence(const orc_ctx *c, uint32_t *out) {
+  for (uint32_t b = 0; b < c->nb; ++b) out[b] = c->persist[b];
 }

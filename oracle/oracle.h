@@ -34,7 +34,7 @@ typedef struct {
   int64_t t0;
   uint32_t hang_windows;           /* H >= 1 */
   uint32_t k;
-  int32_t rank_mode;               /* 0 percent, 1 size */
+  int32_t rank_mode;               /* 0 percent, 1 size, 2 window mean occupancy */
   const uint8_t *owned;            /* [n_components] nullable: shard ownership, restricts ranking */
 } orc_config;
 
@@ -57,6 +57,7 @@ typedef struct { int64_t started, finished, in_flight; } orc_comp;
 typedef struct orc_ctx orc_ctx;
 
 orc_ctx *orc_create(const orc_config *cfg);
+void orc_persistence(const orc_ctx *c, uint32_t *out); /* [n_buffers] windows in the top-k */
 void orc_destroy(orc_ctx *c);
 void orc_reset(orc_ctx *c);
 

@@ -516,3 +516,58 @@ def test_c4_small_oracle_topk_matches_fraction_sort():
     st = r["stats"]
     order = sorted(range(wl.n_buffers), key=lambda b: (-Fraction(int(st["last"][b]), int(st["capacity"][b])), b))
     assert r["topk"][-1]["buffer_id"].tolist() == order[:wl.k]
+
+
+# ---------------------------------------------------------------------------------------------
+# Persistence ranking: rank mode 2 = the window's time-weighted mean
+# occupancy; windows-in-top-k counter
+@pytest.mark.parametrize("seed", range(40))
+def test_mean_occupancy_ranking_and_persistence_match_brute_force(seed):
+    """Against brute.py's tick-loop integral ranked with exact Fractions I / (cap * W), and the
+    persistence counter against counting the brute force's top-k lists."""
+    rng = np.random.default_rng(5000 + seed)
+    case = random_tiny_case(rng)
+    case["mode"] = 2
+    kw = dict(t0=case["t0"], hang_windows=case["H"], k=case["k"], rank_mode=2)
+    orc = oracle.Oracle(case["owner"], case["caps"], case["totals"], n_components=case["nc"], **kw)
+    br = brute.Brute(case["owner"], case["caps"], case["totals"], case["nc"], **kw)
+    counts = np.zeros(case["nb"], np.uint32)
+    for srows, erows, ends in case["calls"]:
+        o = orc.reduce(sample_array(srows), event_array(erows), ends, want_all_stats=True)
+        b = br.reduce(srows, erows, ends)
+        _compare(o, b, case["nb"], case["nk"], case["nc"])
+        for bw in b:
+            for bid, _, _ in bw["topk"]:
+                counts[bid] += 1
+    assert np.array_equal(orc.persistence(), counts)
+
+
+def test_mean_ranking_closed_forms():
+    """(i) A window without samples holds every level constant, so mean occupancy = level / cap
+    exactly and the mean ranking equals the Percent ranking (Fig. 3 table as levels).
+    (ii) Worked example E1 (integral 46 of 80 -> 0.575) ranks below a buffer full the whole
+    window (1.0) and above one at 1/4 all window (0.25), ties by id."""
+    rows = [ln.split() for ln in open(os.path.join(GOLDEN, "fig3_buffers.txt")) if ln.strip() and not ln.startswith("#")]
+    lvls = [int(r[1]) for r in rows]
+    caps = np.array([int(r[2]) for r in rows], np.uint16)
+    n = len(rows)
+    owner = np.arange(n, dtype=np.uint32)
+    fill = sample_array([(0, b, lvls[b], int(caps[b])) for b in range(n)])
+    tops = {}
+    for mode in (0, 2):
+        orc = oracle.Oracle(owner, caps, np.ones(1, np.int64), n_components=n, t0=0, hang_windows=4, k=n,
+                            rank_mode=mode)
+        orc.reduce(fill, event_array([]), [1])
+        r = orc.reduce(sample_array([]), event_array([]), [11])  # no samples: levels constant
+        tops[mode] = r["topk"][0]["buffer_id"].tolist()
+    assert tops[2] == tops[0]
+    # (ii): buffers 0 (E1), 1 (full all window), 2 (2 of 8 all window), 3 (same as 1, higher id)
+    caps = np.array([8, 4, 8, 4], np.uint16)
+    orc = oracle.Oracle(np.arange(4, dtype=np.uint32), caps, np.ones(1, np.int64), n_components=4, t0=-10,
+                        hang_windows=4, k=4, rank_mode=2)
+    orc.reduce(sample_array([(-1, 0, 2, 8), (-1, 1, 4, 4), (-1, 2, 2, 8), (-1, 3, 4, 4)]), event_array([]), [0])
+    r = orc.reduce(sample_array([(3, 0, 5, 8), (3, 0, 4, 8), (7, 0, 8, 8)]), event_array([]), [10],
+                   want_all_stats=True)
+    assert int(r["all_stats"][0][0]["integral"]) == 46
+    assert r["topk"][0]["buffer_id"].tolist() == [1, 3, 0, 2]
+    assert orc.persistence().tolist() == [2, 2, 2, 2]
