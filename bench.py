@@ -210,7 +210,7 @@ def run_native(args):
     extra = {} if gid is None else dict(buffer_global_id=gid, n_global_buffers=wl.n_buffers * world,
                                         pack_buffers=wl.n_buffers)
     mon = Monitor(owner, cap, tot, n_components=nc, t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k, device=local,
-                  rank=rank, world=world, **extra)
+                  rank=rank, world=world, rank_mode=args.rank_mode, **extra)
     t_end = wl.t_end()
     n_rec = wl.n_samples + wl.n_events
 
@@ -333,7 +333,7 @@ def finish(args, wl, world, ms, prof, n_rec, value, e2e_value, d2h, n_launches, 
         "data": "synthetic",
         "config": {"workload": wl.description + (f" (x{world} shards, weak scaling)" if world > 1 else ""),
                    "n_buffers": int(wl.n_buffers * world), "records_per_gpu": n_rec, "windows": W, "k": wl.k,
-                   "hang_windows": wl.hang_windows,
+                   "hang_windows": wl.hang_windows, "rank_mode": args.rank_mode,
                    "l2": f"inputs ({16 * n_rec / 1e9:.1f} GB/GPU) larger than L2; no flush",
                    "parallelism": f"owner-component shards x{world}" if world > 1 else "single GPU"},
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved_gbs, "peak": hbm, "unit": "GB/s",
@@ -362,6 +362,7 @@ def main():
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--rank-mode", type=int, default=0, help="0 percent (bench line), 1 size, 2 mean occupancy")
     ap.add_argument("--config", default="C2-1gpu",
                     help="workload (gen.CONFIGS); the bench line is C2-1gpu, the others are parity configs "
                          "measured for profiles/")

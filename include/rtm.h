@@ -51,7 +51,12 @@ typedef enum {
 
 enum { RTM_MEM_HOST = 0, RTM_MEM_DEVICE = 1 };
 /* "sort the buffers by their fullness percentage or by the number of elements" */
-enum { RTM_RANK_PERCENT = 0, RTM_RANK_SIZE = 1 };
+enum { RTM_RANK_PERCENT = 0, RTM_RANK_SIZE = 1,
+       /* persistence ranking (a buffer "repeatedly at the top of the list"
+        * is the bottleneck, L173, L197-L199): the window's time-weighted mean occupancy
+        * integral / (capacity * window length), descending, ties by buffer_id.  world == 1 only;
+        * every window of a call must be shorter than 2^32 ticks (else RTM_E_INVALID). */
+       RTM_RANK_MEAN = 2 };
 
 /* ---- trace records (16 B each, little-endian, naturally aligned) --------------------------
  * rtm_level_sample: buffer `buffer_id` holds `level` elements of `capacity` from tick ts on
@@ -192,6 +197,12 @@ rtm_status rtm_window_results(rtm_ctx *ctx, uint32_t first, uint32_t count, rtm_
 rtm_status rtm_window_reduce_local(rtm_ctx *ctx, const int64_t *t_end, uint32_t n_windows,
                                    const void **pack, uint64_t *pack_bytes);
 rtm_status rtm_merge(rtm_ctx *ctx, const void *gathered, uint32_t world, rtm_window_summary *out);
+
+/* Windows-in-top-k counter (persistence): for buffers [first,
+ * first+count) (global ids with a rank-local numbering), the number of windows since create /
+ * reset in which the buffer was in the window's top-k list (the merged list when world > 1).
+ * out (host) holds count entries. */
+rtm_status rtm_topk_persistence(rtm_ctx *ctx, uint32_t first, uint32_t count, uint32_t *out);
 
 /* ---- Value monitor (§IV-C.3, Fig. 2 F) ----------
  * The dashboard plots "up to five values" over time and keeps "the last 300 data points"

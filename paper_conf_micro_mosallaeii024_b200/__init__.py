@@ -17,11 +17,12 @@ from collections.abc import Mapping
 import numpy as np
 
 from . import _native as N
-from ._native import (BSTAT_DTYPE, COMP_DTYPE, EVENT_DTYPE, PROGRESS_DTYPE, RTM_RANK_PERCENT, RTM_RANK_SIZE,
+from ._native import (BSTAT_DTYPE, COMP_DTYPE, EVENT_DTYPE, PROGRESS_DTYPE, RTM_RANK_MEAN, RTM_RANK_PERCENT,
+                      RTM_RANK_SIZE,
                       SAMPLE_DTYPE, SUMMARY_DTYPE, TOPK_DTYPE, RTMError)
 
 __all__ = ["Monitor", "RTMError", "SAMPLE_DTYPE", "EVENT_DTYPE", "SUMMARY_DTYPE", "TOPK_DTYPE", "PROGRESS_DTYPE",
-           "COMP_DTYPE", "BSTAT_DTYPE", "RTM_RANK_PERCENT", "RTM_RANK_SIZE", "version"]
+           "COMP_DTYPE", "BSTAT_DTYPE", "RTM_RANK_PERCENT", "RTM_RANK_SIZE", "RTM_RANK_MEAN", "version"]
 
 N.lib()  # fail at import time if the native library is missing
 
@@ -189,6 +190,14 @@ class Monitor:
             count = self.n_table - first  # global ids with a rank-local numbering
         out = np.zeros(count, BSTAT_DTYPE)
         N.check(N.lib().rtm_buffer_stats(self._h, first, count, out.ctypes.data), "rtm_buffer_stats")
+        return out
+
+    def topk_persistence(self, first: int = 0, count: int | None = None):
+        """Windows-in-top-k counter per buffer since create / reset (persistence, L173, L197-L199)."""
+        if count is None:
+            count = self.n_table - first
+        out = np.zeros(count, np.uint32)
+        N.check(N.lib().rtm_topk_persistence(self._h, first, count, out.ctypes.data), "rtm_topk_persistence")
         return out
 
     def watch(self, buffer_ids):

@@ -16,7 +16,7 @@ LIB_PATH = os.environ.get("RTM_LIB_PATH") or os.path.join(HERE, "librtm.so")  # 
 RTM_OK, RTM_E_INVALID, RTM_E_CUDA, RTM_E_COMM, RTM_E_ORDER, RTM_E_TOO_SMALL, RTM_E_STATE, RTM_E_NOMEM = (
     0, -1, -2, -3, -4, -5, -6, -7)
 RTM_MEM_HOST, RTM_MEM_DEVICE = 0, 1
-RTM_RANK_PERCENT, RTM_RANK_SIZE = 0, 1
+RTM_RANK_PERCENT, RTM_RANK_SIZE, RTM_RANK_MEAN = 0, 1, 2
 
 # record and result layouts (include/rtm.h)
 SAMPLE_DTYPE = np.dtype([("ts", "<i8"), ("buffer_id", "<u4"), ("level", "<u2"), ("capacity", "<u2")])
@@ -60,7 +60,7 @@ class KernelTime(ctypes.Structure):
 EXPORTS = ("rtm_create", "rtm_destroy", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers",
            "rtm_progress", "rtm_hang_check", "rtm_buffer_stats", "rtm_window_results", "rtm_window_reduce_local",
            "rtm_merge", "rtm_profile", "rtm_profile_read", "rtm_status_str", "rtm_version",
-           "rtm_kernel_launches", "rtm_watch", "rtm_watch_series")
+           "rtm_kernel_launches", "rtm_watch", "rtm_watch_series", "rtm_topk_persistence")
 
 _lib = None
 
@@ -91,8 +91,9 @@ def lib():
     L.rtm_profile.argtypes = [vp, i32]
     L.rtm_profile_read.argtypes = [vp, vp, u32, P(u32)]
     L.rtm_watch.argtypes = [vp, vp, u32]
+    L.rtm_topk_persistence.argtypes = [vp, u32, u32, vp]
     L.rtm_watch_series.argtypes = [vp, u32, vp, P(u32)]
-    for fn in ("rtm_watch", "rtm_watch_series", "rtm_create", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers", "rtm_progress",
+    for fn in ("rtm_watch", "rtm_watch_series", "rtm_topk_persistence", "rtm_create", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers", "rtm_progress",
                "rtm_hang_check", "rtm_buffer_stats", "rtm_window_reduce_local", "rtm_merge", "rtm_profile",
                "rtm_profile_read", "rtm_window_results"):
         getattr(L, fn).restype = ctypes.c_int

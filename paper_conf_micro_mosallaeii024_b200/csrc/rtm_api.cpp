@@ -51,6 +51,8 @@ struct rtm_ctx {
   DevBuf cap, owner, elig, ktotal, rcp, elig_ids;
   DevBuf gid, bstat_g;      // rank-local numbering: global id per local buffer, table by global id
   DevBuf tkscr;             // per-slice top-k candidates (few-window calls)
+  DevBuf mkey, rcp64;       // rank mode MEAN: per-(window, buffer) order keys, floor(2^64 / c)
+  DevBuf persist;           // windows-in-top-k counter per buffer (id space)
   // value monitor: watched ids (as given), their local ids (~0: not on this rank), rings
   std::vector<uint32_t> gid_h;  // host copy of the global ids (rank-local numbering)
   uint32_t n_watch = 0;
@@ -232,6 +234,7 @@ rtm_status zero_state(rtm_ctx *c) {
   cl.add(c->kend.p, (size_t)c->nk * 8);
   cl.add(c->cstart.p, (size_t)c->nc * 8);
   cl.add(c->cend.p, (size_t)c->nc * 8);
+  cl.add(c->persist.p, (size_t)(c->n_global ? c->n_global : c->nb) * 4);
   launch_clear(cl, c->st);
   CK(cudaGetLastError());
   c->cur = 0;
@@ -344,6 +347,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.narrow = 1;
   for (uint32_t w = 0; w < W; ++w)
     if (t_end[w] - (w ? t_end[w - 1] : c->t_prev) >= ((int64_t)1 << 32)) p.narrow = 0;
+  if (c->rank_mode == RTM_RANK_MEAN && !p.narrow) return RTM_E_INVALID;  // before any launch
   p.T = (const long long *)c->T.p;
   p.s = (const rtm_level_sample *)sp; p.ns = ns;
   p.e = (const rtm_task_event *)ep; p.ne = ne;
@@ -378,7 +382,14 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   if ((s = ensure(c, c->hung, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->unit_ctr, 8))) return s;
   if ((s = ensure(c, c->bstat, (size_t)c->nb * sizeof(rtm_buffer_stat)))) return s;
-  p.tk_slices = topk_slices(c->nb, c->k, W, c->n_sms, c->n_elig == c->nb, &p.tk_slice_len);
+  if (c->rank_mode == RTM_RANK_MEAN) {  // order keys (windows shorter than 2^32 ticks, checked above)
+    if ((s = ensure(c, c->mkey, Wn * c->nb * 8))) return s;
+    p.mkey = (unsigned long long *)c->mkey.p;
+    p.rcp64 = (const unsigned long long *)c->rcp64.p;
+  }
+  p.persist = (uint32_t *)c->persist.p;
+  p.tk_slices = topk_slices(c->nb, c->k, W, c->n_sms, c->n_elig == c->nb && c->rank_mode != RTM_RANK_MEAN,
+                            &p.tk_slice_len);
   if (p.tk_slices > 1) {
     if ((s = ensure(c, c->tkscr, (size_t)W * p.tk_slices * c->k * 8))) return s;
     p.tk_scratch = (unsigned long long *)c->tkscr.p;
@@ -440,6 +451,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
   LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
   LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
+  if (c->world == 1) launch_persist(p, c->st);  // world > 1: counted from the merged lists
   LAUNCH(KT_HANG, 0, launch_hang(p, c->st));
   LAUNCH(KT_PROGRESS, 0, launch_progress(p, c->st));
   CK(cudaGetLastError());
@@ -555,7 +567,9 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   if (cfg->n_components == 0 || cfg->n_components > (1u << 20)) return RTM_E_INVALID;
   if (cfg->n_kernels == 0 || cfg->n_kernels > 2048) return RTM_E_INVALID;
   if (cfg->k == 0 || cfg->k > 1024 || cfg->hang_windows == 0) return RTM_E_INVALID;
-  if (cfg->rank_mode != RTM_RANK_PERCENT && cfg->rank_mode != RTM_RANK_SIZE) return RTM_E_INVALID;
+  if (cfg->rank_mode != RTM_RANK_PERCENT && cfg->rank_mode != RTM_RANK_SIZE && cfg->rank_mode != RTM_RANK_MEAN)
+    return RTM_E_INVALID;
+  if (cfg->rank_mode == RTM_RANK_MEAN && cfg->world > 1) return RTM_E_INVALID;
   if (!cfg->buffer_owner || !cfg->buffer_capacity || !cfg->kernel_total) return RTM_E_INVALID;
   if (cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world) return RTM_E_INVALID;
   for (uint32_t b = 0; b < cfg->n_buffers; ++b)
@@ -611,8 +625,18 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
       (s = ensure(c, c->kstart, (size_t)c->nk * 8)) ||
       (s = ensure(c, c->kend, (size_t)c->nk * 8)) || (s = ensure(c, c->cstart, (size_t)c->nc * 8)) ||
       (s = ensure(c, c->cend, (size_t)c->nc * 8)) || (s = ensure(c, c->rcp, (size_t)65536 * 8)) ||
-      (s = ensure(c, c->elig_ids, (size_t)c->nb * 4)))
+      (s = ensure(c, c->elig_ids, (size_t)c->nb * 4)) ||
+      (s = ensure(c, c->persist, (size_t)(c->n_global ? c->n_global : c->nb) * 4)))
     return fail(s);
+  if (c->rank_mode == RTM_RANK_MEAN) {
+    if ((s = ensure(c, c->rcp64, (size_t)65536 * 8))) return fail(s);
+    std::vector<unsigned long long> r64(65536, 0);
+    for (uint32_t cc = 2; cc < 65536; ++cc) r64[cc] = (unsigned long long)(((unsigned __int128)1 << 64) / cc);
+    if (cudaMemcpy(c->rcp64.p, r64.data(), 65536 * 8, cudaMemcpyHostToDevice) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(RTM_E_CUDA);
+    }
+  }
   std::vector<uint8_t> elig(c->nb);
   std::vector<uint32_t> elig_ids;
   for (uint32_t b = 0; b < c->nb; ++b) {
@@ -682,6 +706,18 @@ rtm_status rtm_reset(rtm_ctx *c) {
   return zero_state(c);
 }
 
+rtm_status rtm_topk_persistence(rtm_ctx *c, uint32_t first, uint32_t count, uint32_t *out) {
+  if (!c || (count && !out)) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  const uint32_t space = c->n_global ? c->n_global : c->nb;
+  if ((uint64_t)first + count > space) return RTM_E_INVALID;
+  if (!count) return RTM_OK;
+  CK(cudaSetDevice(c->device));
+  CK(cudaMemcpyAsync(out, (const uint32_t *)c->persist.p + first, (size_t)count * 4, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  return RTM_OK;
+}
+
 rtm_status rtm_watch(rtm_ctx *c, const uint32_t *ids, uint32_t n) {
   if (!c || n > RTM_WATCH_MAX || (n && !ids)) return RTM_E_INVALID;
   const uint32_t space = c->gid.p ? c->n_global : c->nb;
@@ -742,6 +778,7 @@ rtm_status rtm_window_reduce(rtm_ctx *c, const int64_t *t_end, uint32_t n_window
       return RTM_E_COMM;
     }
     LAUNCH(KT_MERGE, 0, launch_merge(p, c->gathered.p, c->world, c->st));
+    launch_persist(p, c->st);
     CK(cudaGetLastError());
   } else if (c->gid.p) {
     launch_scatter_bstat(p, c->st);
@@ -785,7 +822,9 @@ rtm_status rtm_merge(rtm_ctx *c, const void *gathered, uint32_t world, rtm_windo
   p.comps = (rtm_component_tasks *)c->comps.p; p.bstat = (rtm_buffer_stat *)c->bstat.p;
   p.gid = (const uint32_t *)c->gid.p; p.n_global = c->n_global; p.pack_nb = c->pack_nb;
   p.bstat_g = (rtm_buffer_stat *)c->bstat_g.p;
+  p.persist = (uint32_t *)c->persist.p;
   LAUNCH(KT_MERGE, 0, launch_merge(p, gathered, world, c->st));
+  launch_persist(p, c->st);
   CK(cudaGetLastError());
   std::vector<int64_t> te = c->t_end_h;
   return finish(c, te.data(), W, out);

@@ -126,6 +126,9 @@ struct Params {
   rtm_buffer_stat *bstat;    // [nb] last window, local ids
   rtm_buffer_stat *bstat_g;  // [n_global] merged / scattered table by global id (gid set)
   rtm_component_tasks *comps;// [nc]
+  unsigned long long *mkey;  // [W * nb] rank mode MEAN: floor(integral * 2^32 / cap) (exact order key)
+  const unsigned long long *rcp64;  // [65536] floor(2^64 / c) (c >= 2)
+  uint32_t *persist;         // [id space] windows in the top-k list
   uint32_t n_watch;          // value monitor: watched local buffer ids (0xFFFFFFFF: not on this rank)
   uint32_t watch[RTM_WATCH_MAX];
   rtm_buffer_stat *wstat;    // [W * RTM_WATCH_MAX] per-window statistics of the watched buffers
@@ -145,6 +148,7 @@ void launch_topk(const Params &p, cudaStream_t st);
 uint32_t topk_slices(uint32_t nb, uint32_t k, uint32_t W, int n_sms, bool all, uint32_t *slice_len);
 void launch_hang(const Params &p, cudaStream_t st);
 void launch_progress(const Params &p, cudaStream_t st);
+void launch_persist(const Params &p, cudaStream_t st);
 // multi-rank exchange
 uint64_t pack_bytes(const Params &p);
 void launch_pack(const Params &p, void *pack, cudaStream_t st);

@@ -852,6 +852,23 @@ __global__ void __launch_bounds__(kK3Threads) k_events(Params p) {
       if (abits[i]) atomicOr(p.active + (size_t)g.window * p.ncw + i, abits[i]);
 }
 
+// Persistence ranking key (rank mode MEAN): floor(I * 2^32 / c), exact.  Within a window the
+// mean occupancy I / (c * W) orders like I / c; distinct ratios I1/c1 != I2/c2 differ by at least
+// 1/(c1 c2) >= 2^-32 * 1.00003, so the floors differ: the key is exactly order-preserving.  Needs
+// I / c < 2^32 (I <= c * W, windows shorter than 2^32 ticks).  m = floor(2^64 / c): q0 =
+// floor(I m / 2^64) is floor(I / c) or one less (the error I eps / 2^64 < 1); one remainder test.
+__device__ __forceinline__ unsigned long long mean_key(unsigned long long I, unsigned c,
+                                                       const unsigned long long *rcp64) {
+  if (c <= 1) return I << 32;
+  const unsigned long long m = __ldg(rcp64 + c);
+  unsigned long long q = __umul64hi(I, m), r = I - q * c;
+  if (r >= c) ++q, r -= c;
+  const unsigned long long x = r << 32;  // r < c <= 65535
+  unsigned long long lo = __umul64hi(x, m);
+  if (x - lo * c >= c) ++lo;
+  return (q << 32) | lo;
+}
+
 // ============================================================================================
 // K2: fold.  One warp per (window, bin) unit; units are dequeued in window-major order, so a
 // unit only ever waits on units dequeued before it (forward progress).  Phase 1 folds the
@@ -1095,6 +1112,7 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
         lw[b] = (uint16_t)L;  // resolve the untouched cell
       }
       const unsigned capb = __ldg(p.cap + b);
+      if (p.mkey) p.mkey[(size_t)w * p.nb + b] = mean_key(I, capb, p.rcp64);
       if (mn == capb) {
         const unsigned c = __ldg(p.owner + b);
         atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
@@ -1439,6 +1457,140 @@ __global__ void __launch_bounds__(1024) k_topk_merge(Params p) {
     p.topk[(size_t)w * p.k + i] = out;
   }
   if (threadIdx.x == 0) p.topk_n[w] = keff;
+}
+
+// K5 for rank mode MEAN: one CTA per window over the 64-bit keys of the fold (mean_key).  MSB
+// radix select over 8 x 8-bit digits (keys read from L2; windows shorter than 2^32 ticks leave the
+// top bytes zero, one pass each); as soon as the keys at or above the selected prefix fit the
+// candidate list they are compacted in id order and the remaining digits scan only them.  Keys >
+// tau are taken, then the first `need` keys == tau in id order; the k winners are bitonic-sorted by
+// (key desc, id asc).
+constexpr int kT64Threads = 512;
+constexpr unsigned kT64Cand = 8192;
+__global__ void __launch_bounds__(kT64Threads) k_topk64(Params p) {
+  __shared__ unsigned hist[256];
+  __shared__ unsigned scan_scratch[32];
+  __shared__ unsigned s_digit, s_need, s_ncand, s_ngt;
+  __shared__ unsigned cand[kT64Cand];
+  __shared__ unsigned long long selk[1024];
+  __shared__ unsigned seli[1024];
+  const unsigned w = blockIdx.x, ne = p.nb, lane = threadIdx.x & 31;
+  const unsigned long long *key = p.mkey + (size_t)w * p.nb;
+  const unsigned keff = p.k < ne ? p.k : ne;
+  unsigned long long prefix = 0, mask = 0;
+  unsigned need = keff, n_it = ne;
+  bool use_c = false;
+  for (int d = 7; d >= 0; --d) {
+    for (unsigned i = threadIdx.x; i < 256; i += blockDim.x) hist[i] = 0;
+    __syncthreads();
+    for (unsigned j0 = threadIdx.x - lane; j0 < n_it; j0 += blockDim.x) {
+      const unsigned j = j0 + lane;
+      bool ok = false;
+      unsigned dg = 0;
+      if (j < n_it) {
+        const unsigned long long k = __ldcg(key + (use_c ? cand[j] : j));
+        ok = (k & mask) == prefix;
+        dg = (unsigned)(k >> (8 * d)) & 255u;
+      }
+      const unsigned peers = __match_any_sync(kFull, ok ? dg : 0xFFFFFFFFu);
+      if (ok && lane == (unsigned)__ffs(peers) - 1) atomicAdd(&hist[dg], (unsigned)__popc(peers));
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned cum = 0;
+      int x = 255;
+      for (; x > 0; --x) {
+        if (cum + hist[x] >= need) break;
+        cum += hist[x];
+      }
+      s_digit = (unsigned)x;
+      s_need = need - cum;
+      s_ncand = (keff - need) + cum + hist[x];  // keys at or above the new prefix
+    }
+    __syncthreads();
+    prefix |= (unsigned long long)s_digit << (8 * d);
+    mask |= 255ull << (8 * d);
+    if (!use_c && d > 0 && s_ncand <= kT64Cand) {  // compact keys >= the prefix, id order
+      const unsigned long long lim = prefix >> (8 * d);
+      const unsigned chunk = (ne + blockDim.x - 1) / blockDim.x, c0 = threadIdx.x * chunk;
+      unsigned cnt = 0;
+      for (unsigned i = c0; i < c0 + chunk && i < ne; ++i) cnt += (__ldcg(key + i) >> (8 * d)) >= lim;
+      unsigned pos = block_excl_scan(cnt, scan_scratch, nullptr);
+      for (unsigned i = c0; i < c0 + chunk && i < ne; ++i)
+        if ((__ldcg(key + i) >> (8 * d)) >= lim) cand[pos++] = i;
+      n_it = s_ncand;
+      use_c = true;
+    }
+    need = s_need;
+    __syncthreads();
+  }
+  const unsigned long long tau = prefix;
+  if (threadIdx.x == 0) s_ngt = 0;
+  __syncthreads();
+  const unsigned chunk = (n_it + blockDim.x - 1) / blockDim.x, c0 = threadIdx.x * chunk;
+  unsigned ceq = 0;
+  for (unsigned j = c0; j < c0 + chunk && j < n_it; ++j) {
+    const unsigned i = use_c ? cand[j] : j;
+    const unsigned long long k = __ldcg(key + i);
+    if (k > tau) {
+      const unsigned slot = atomicAdd(&s_ngt, 1u);
+      selk[slot] = k;
+      seli[slot] = i;
+    }
+    ceq += (k == tau);
+  }
+  unsigned rank = block_excl_scan(ceq, scan_scratch, nullptr);
+  const unsigned ngt = s_ngt;
+  for (unsigned j = c0; j < c0 + chunk && j < n_it && rank < need; ++j) {
+    const unsigned i = use_c ? cand[j] : j;
+    if (__ldcg(key + i) == tau) {
+      selk[ngt + rank] = tau;
+      seli[ngt + rank] = i;
+      ++rank;
+    }
+  }
+  __syncthreads();
+  unsigned P = 1;
+  while (P < keff) P <<= 1;
+  for (unsigned i = keff + threadIdx.x; i < P; i += blockDim.x) selk[i] = 0ull, seli[i] = 0xFFFFFFFFu;
+  __syncthreads();
+  for (unsigned size = 2; size <= P; size <<= 1) {  // (key desc, id asc)
+    for (unsigned stride = size >> 1; stride > 0; stride >>= 1) {
+      for (unsigned i = threadIdx.x; i < P; i += blockDim.x) {
+        const unsigned jx = i ^ stride;
+        if (jx > i) {
+          const bool desc = (i & size) == 0;
+          const unsigned long long a = selk[i], b = selk[jx];
+          const unsigned ia = seli[i], ib = seli[jx];
+          const bool a_before_b = a > b || (a == b && ia < ib);
+          if (a_before_b != desc) {
+            selk[i] = b; selk[jx] = a;
+            seli[i] = ib; seli[jx] = ia;
+          }
+        }
+      }
+      __syncthreads();
+    }
+  }
+  const uint16_t *lv = p.lastlvl + (size_t)w * p.nb;
+  for (unsigned i = threadIdx.x; i < p.k; i += blockDim.x) {
+    unsigned long long out = 0xFFFFFFFFull;
+    if (i < keff) {
+      const unsigned b = seli[i];
+      out = (unsigned long long)(p.gid ? __ldg(p.gid + b) : b) | ((unsigned long long)lv[b] << 32) |
+            ((unsigned long long)__ldg(p.cap + b) << 48);
+    }
+    p.topk[(size_t)w * p.k + i] = out;
+  }
+  if (threadIdx.x == 0) p.topk_n[w] = keff;
+}
+
+// Windows-in-top-k counter: one thread per (window, rank) of the call's (merged) lists.
+__global__ void k_persist(Params p) {
+  const size_t t = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= (size_t)p.W * p.k) return;
+  const unsigned w = (unsigned)(t / p.k), i = (unsigned)(t % p.k);
+  if (i < p.topk_n[w]) atomicAdd(p.persist + (unsigned)(p.topk[t] & 0xFFFFFFFFull), 1u);
 }
 
 // ============================================================================================
@@ -1802,6 +1954,10 @@ uint32_t topk_slices(uint32_t nb, uint32_t k, uint32_t W, int n_sms, bool all, u
 }
 
 void launch_topk(const Params &p, cudaStream_t st) {
+  if (p.mkey) {  // rank mode MEAN
+    { k_topk64<<<p.W, kT64Threads, 0, st>>>(p); count_launch(); }
+    return;
+  }
   if (p.n_elig == p.nb && p.tk_slices > 1) {
     { k_topk<true><<<dim3(p.W, p.tk_slices), kTopkThreads, topk_smem_bytes(p.tk_slice_len), st>>>(p); count_launch(); }
     { k_topk_merge<<<p.W, 1024, 0, st>>>(p); count_launch(); }
@@ -1809,6 +1965,12 @@ void launch_topk(const Params &p, cudaStream_t st) {
   }
   if (p.n_elig == p.nb) { k_topk<true><<<p.W, kTopkThreads, topk_smem_bytes(p.nb), st>>>(p); count_launch(); }
   else { k_topk<false><<<p.W, kTopkThreads, topk_smem_bytes(p.n_elig), st>>>(p); count_launch(); }
+}
+
+void launch_persist(const Params &p, cudaStream_t st) {
+  const size_t n = (size_t)p.W * p.k;
+  if (!n || !p.persist) return;
+  { k_persist<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(p); count_launch(); }
 }
 
 void launch_hang(const Params &p, cudaStream_t st) {

@@ -480,3 +480,47 @@ def test_value_monitor_rings_last_300_windows():
     mon.watch([])
     with pytest.raises(RTMError):
         mon.watch_series(0)
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_mean_ranking_random_tiny_traces(seed):
+    """Rank mode MEAN (persistence ranking): random tiny traces, GPU vs oracle, plus the
+    windows-in-top-k counter after every call."""
+    rng = np.random.default_rng(7000 + seed)
+    case = random_tiny_case(rng)
+    kw = dict(t0=case["t0"], hang_windows=case["H"], k=case["k"], rank_mode=2)
+    orc, mon = _pair(case["owner"], case["caps"], case["totals"], case["nc"], **kw)
+    for srows, erows, ends in case["calls"]:
+        ref = orc.reduce(sample_array(srows), event_array(erows), ends)
+        mon.ingest(sample_array(srows), event_array(erows))
+        got = mon.window_reduce(np.array(ends, np.int64))
+        assert_same(got, ref, mon, comps=False)
+        assert np.array_equal(mon.topk_persistence(), orc.persistence())
+
+
+@pytest.mark.parametrize("mode", [0, 1, 2])
+def test_ranking_modes_c1_and_persistence(mode):
+    """C1 (1M samples, 1000 buffers, 10 windows) in every rank mode: top-k lists and the
+    persistence counter equal the oracle's."""
+    wl = gen.C1
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k, rank_mode=mode)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    s, e = gen.samples(wl), gen.events(wl)
+    for lo, hi in ((0, 4), (4, 5), (5, 10)):
+        sl = slice(wl.index_at("samples", wl.t_begin(lo)), wl.index_at("samples", wl.t_begin(hi)))
+        el = slice(wl.index_at("events", wl.t_begin(lo)), wl.index_at("events", wl.t_begin(hi)))
+        ref = orc.reduce(s[sl], e[el], wl.t_end()[lo:hi])
+        mon.ingest(_dev(s[sl]), _dev(e[el]))
+        got = mon.window_reduce(wl.t_end()[lo:hi])
+        assert_same(got, ref, mon)
+    assert np.array_equal(mon.topk_persistence(), orc.persistence())
+
+
+def test_mean_mode_rejects_long_windows():
+    owner, cap = np.zeros(2, np.uint32), np.array([4, 8], np.uint16)
+    mon = Monitor(owner, cap, np.ones(1, np.int64), n_components=1, t0=0, k=2, rank_mode=2)
+    with pytest.raises(RTMError):
+        mon.window_reduce(np.array([1 << 33], np.int64))
+    got = mon.window_reduce(np.array([10], np.int64))  # state unchanged: the next call works
+    assert int(got["summary"]["t_begin"][0]) == 0
