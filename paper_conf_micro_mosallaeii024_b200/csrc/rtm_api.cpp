@@ -437,34 +437,21 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
 #endif
   launch_fill_tile_regions(p, c->st);
   // task events are independent of the sample path: run them on a side stream, overlapped with
-  // the partition and the fold, and join before the kernels that read their outputs
-  static int ev_mode = -1;
-  if (ev_mode < 0) { const char *e = getenv("RTM_EV"); ev_mode = e ? atoi(e) : 0; }
-  auto fork_events = [&]() -> rtm_status {
-    CK(cudaEventRecord(c->ev_fork, c->st));
-    CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
-    if (c->prof) prof_begin_on(c, KT_EVENTS, (uint64_t)ne * 16, c->st2);
-    launch_events(p, c->st2);
-    if (c->prof) prof_end_on(c, c->st2);
-    CK(cudaEventRecord(c->ev_join, c->st2));
-    return RTM_OK;
-  };
-  if (ev_mode == 0 && (s = fork_events())) return s;
+  // the partition and the fold, and join before the kernels that read their outputs (placing
+  // them after the partition or overlapping the top-k instead measured the same step time)
+  CK(cudaEventRecord(c->ev_fork, c->st));
+  CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
+  if (c->prof) prof_begin_on(c, KT_EVENTS, (uint64_t)ne * 16, c->st2);
+  launch_events(p, c->st2);
+  if (c->prof) prof_end_on(c, c->st2);
+  CK(cudaEventRecord(c->ev_join, c->st2));
   // algorithmic bytes: partition = 16 B record in + 8 B compacted entry out per
   // sample; fold = the 8 B entry per sample
   LAUNCH(KT_PARTITION, (uint64_t)ns * 24, launch_partition(p, c->n_sms, c->st));
-  if (ev_mode == 1 && (s = fork_events())) return s;
   LAUNCH(KT_FOLD, (uint64_t)ns * 8, launch_fold(p, c->n_sms, c->st));
-  if (ev_mode == 2) {  // events overlap the top-k (which does not read them)
-    if ((s = fork_events())) return s;
-    LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
-    CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
-    LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
-  } else {
-    CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
-    LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
-    LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
-  }
+  CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
+  LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
+  LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
   if (c->world == 1) launch_persist(p, c->st);  // world > 1: counted from the merged lists
   LAUNCH(KT_HANG, 0, launch_hang(p, c->st));
   LAUNCH(KT_PROGRESS, 0, launch_progress(p, c->st));
