@@ -59,6 +59,11 @@ def lib():
         L.orc_merge_topk.restype = ctypes.c_int
         L.orc_persistence.argtypes = [vp, vp]
         L.orc_persistence.restype = None
+        L.orc_bar_create.argtypes = [vp, ctypes.c_int64, ctypes.POINTER(u32)]
+        L.orc_bar_update.argtypes = [vp, u32, ctypes.c_int64]
+        L.orc_bar_destroy.argtypes = [vp, u32]
+        for fn in ("orc_bar_create", "orc_bar_update", "orc_bar_destroy"):
+            getattr(L, fn).restype = ctypes.c_int
         _lib = L
     return _lib
 
@@ -97,6 +102,20 @@ class Oracle:
 
     def reset(self):
         lib().orc_reset(self._h)
+
+    def bar_create(self, total):
+        i = ctypes.c_uint32()
+        if lib().orc_bar_create(self._h, int(total), ctypes.byref(i)) != 0:
+            raise ValueError("no free progress bar id")
+        return i.value
+
+    def bar_update(self, bar, total):
+        if lib().orc_bar_update(self._h, int(bar), int(total)) != 0:
+            raise ValueError("progress bar not live")
+
+    def bar_destroy(self, bar):
+        if lib().orc_bar_destroy(self._h, int(bar)) != 0:
+            raise ValueError("progress bar not live")
 
     def persistence(self):
         """Per buffer: windows (since create / reset) in which it was in the top-k list."""

@@ -55,6 +55,23 @@ class Brute:
         self.cs, self.ce = [0] * self.nc, [0] * self.nc
         self.ks, self.ke = [0] * self.nk, [0] * self.nk
         self.run = [0] * self.nc
+        self.live = [1] * self.nk
+
+    # progress bar registry (Create / Update / DestroyProgressBar)
+    def bar_create(self, total):
+        k = self.live.index(0)  # lowest free id (ValueError if none)
+        self.live[k], self.total[k], self.ks[k], self.ke[k] = 1, int(total), 0, 0
+        return k
+
+    def bar_update(self, k, total):
+        if not self.live[k]:
+            raise ValueError("not live")
+        self.total[k] = int(total)
+
+    def bar_destroy(self, k):
+        if not self.live[k]:
+            raise ValueError("not live")
+        self.live[k] = 0
 
     # field validity (DESIGN.md §2 "ingest")
     def _sample_valid(self, r):
@@ -63,7 +80,8 @@ class Brute:
 
     def _event_valid(self, r):
         ts, task, meta = r
-        return (meta & 0xFFFFF) < self.nc and ((meta >> 20) & 0x7FF) < self.nk
+        kern = (meta >> 20) & 0x7FF
+        return (meta & 0xFFFFF) < self.nc and kern < self.nk and self.live[kern] == 1
 
     def reduce(self, samples, events, t_end):
         """samples: list of (ts, buffer_id, level, capacity); events: list of (ts, task_id, meta)."""
@@ -149,6 +167,7 @@ class Brute:
                 active[c] = 1
             progress = [dict(total=self.total[k], started=self.ks[k], finished=self.ke[k],
                              in_flight=self.ks[k] - self.ke[k], not_started=self.total[k] - self.ks[k])
+                        if self.live[k] else dict(total=0, started=0, finished=0, in_flight=0, not_started=0)
                         for k in range(self.nk)]
             elig = [b for b in range(self.nb) if self.owned[self.owner[b]]]
             if self.mode == 0:

@@ -26,6 +26,8 @@ struct orc_ctx {
   int64_t *c_started, *c_ended, *k_started, *k_ended;
   uint32_t *run;       /* consecutive windows with cond_c true */
   uint32_t *persist;   /* per buffer: windows in which it was in the top-k list */
+  uint8_t *live;       /* progress bar id in use (Create/DestroyProgressBar, L99) */
+  int64_t *ktotal0;    /* bar totals as registered at create (restored by reset) */
   int sticky;
 };
 
@@ -79,6 +81,9 @@ orc_ctx *orc_create(const orc_config *cfg) {
   c->k_ended = (int64_t *)malloc(sizeof(int64_t) * c->nk);
   c->run = (uint32_t *)malloc(sizeof(uint32_t) * c->nc);
   c->persist = (uint32_t *)malloc(sizeof(uint32_t) * (c->nb ? c->nb : 1));
+  c->live = (uint8_t *)malloc(c->nk ? c->nk : 1);
+  c->ktotal0 = (int64_t *)malloc(sizeof(int64_t) * (c->nk ? c->nk : 1));
+  memcpy(c->ktotal0, cfg->kernel_total, sizeof(int64_t) * c->nk);
   orc_reset(c);
   return c;
 }
@@ -92,6 +97,8 @@ void orc_reset(orc_ctx *c) {
   memset(c->k_ended, 0, sizeof(int64_t) * c->nk);
   memset(c->run, 0, sizeof(uint32_t) * c->nc);
   memset(c->persist, 0, sizeof(uint32_t) * c->nb);
+  memset(c->live, 1, c->nk); /* every registered bar is live */
+  memcpy(c->ktotal, c->ktotal0, sizeof(int64_t) * c->nk);
   c->sticky = 0;
 }
 
@@ -99,6 +106,7 @@ void orc_destroy(orc_ctx *c) {
   if (!c) return;
   free(c->owner); free(c->cap); free(c->ktotal); free(c->owned); free(c->lvl);
   free(c->c_started); free(c->c_ended); free(c->k_started); free(c->k_ended); free(c->run); free(c->persist);
+  free(c->live); free(c->ktotal0);
   free(c);
 }
 
@@ -153,7 +161,7 @@ static int classify(int is_sample, const void *recs, uint64_t n, const orc_ctx *
       ts = s[i].ts;
     } else {
       uint32_t comp = e[i].meta & 0xFFFFFu, kern = (e[i].meta >> 20) & 0x7FFu;
-      valid = comp < c->nc && kern < c->nk;
+      valid = comp < c->nc && kern < c->nk && c->live[kern]; /* a destroyed bar takes no events */
       ts = e[i].ts;
     }
     if (valid) {
@@ -301,6 +309,7 @@ int orc_reduce(orc_ctx *c, const orc_sample *s, uint64_t ns, const orc_event *e,
     if (prog)
       for (uint32_t k = 0; k < nk; ++k) {
         orc_progress *P = &prog[(uint64_t)w * nk + k];
+        if (!c->live[k]) { memset(P, 0, sizeof(*P)); continue; } /* free bar id: all zero */
         P->total = c->ktotal[k];
         P->started = c->k_started[k];
         P->finished = c->k_ended[k];
@@ -379,4 +388,30 @@ int orc_merge_topk(const orc_topk *const *shard_topk, const uint32_t *const *sha
 /* Windows-in-top-k counter of every buffer since create / reset. */
 void orc_persistence(const orc_ctx *c, uint32_t *out) {
   for (uint32_t b = 0; b < c->nb; ++b) out[b] = c->persist[b];
+}
+
+/* Progress bar registry (CreateProgressBar / UpdateProgressBar / DestroyProgressBar, L99, L131):
+ * create takes the lowest free id and starts its counts at zero; update sets the total; destroy
+ * frees the id (events naming a free id are field-invalid).  Return 0, or -1 (no free id /
+ * id not live / out of range). */
+int orc_bar_create(orc_ctx *c, int64_t total, uint32_t *id) {
+  for (uint32_t k = 0; k < c->nk; ++k)
+    if (!c->live[k]) {
+      c->live[k] = 1;
+      c->ktotal[k] = total;
+      c->k_started[k] = c->k_ended[k] = 0;
+      *id = k;
+      return 0;
+    }
+  return -1;
+}
+int orc_bar_update(orc_ctx *c, uint32_t id, int64_t total) {
+  if (id >= c->nk || !c->live[id]) return -1;
+  c->ktotal[id] = total;
+  return 0;
+}
+int orc_bar_destroy(orc_ctx *c, uint32_t id) {
+  if (id >= c->nk || !c->live[id]) return -1;
+  c->live[id] = 0;
+  return 0;
 }

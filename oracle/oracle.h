@@ -58,6 +58,9 @@ typedef struct orc_ctx orc_ctx;
 
 orc_ctx *orc_create(const orc_config *cfg);
 void orc_persistence(const orc_ctx *c, uint32_t *out); /* [n_buffers] windows in the top-k */
+int orc_bar_create(orc_ctx *c, int64_t total, uint32_t *id);
+int orc_bar_update(orc_ctx *c, uint32_t id, int64_t total);
+int orc_bar_destroy(orc_ctx *c, uint32_t id);
 void orc_destroy(orc_ctx *c);
 void orc_reset(orc_ctx *c);
 

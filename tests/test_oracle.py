@@ -571,3 +571,69 @@ def test_mean_ranking_closed_forms():
     assert int(r["all_stats"][0][0]["integral"]) == 46
     assert r["topk"][0]["buffer_id"].tolist() == [1, 3, 0, 2]
     assert orc.persistence().tolist() == [2, 2, 2, 2]
+
+
+# ---------------------------------------------------------------------------------------------
+# Dynamic progress bars (Create/Update/DestroyProgressBar, L99, L131)
+def _bar_ops(rng, nk):
+    """A random sequence of registry operations (as (op, arg) tuples) applied between calls."""
+    ops = []
+    for _ in range(int(rng.integers(0, 4))):
+        u = rng.random()
+        if u < 0.4:
+            ops.append(("destroy", int(rng.integers(0, nk))))
+        elif u < 0.7:
+            ops.append(("create", int(rng.integers(0, 20))))
+        else:
+            ops.append(("update", (int(rng.integers(0, nk)), int(rng.integers(0, 20)))))
+    return ops
+
+
+def _apply(ctx, op, arg):
+    """Apply one registry op; returns the result or 'err' (both sides must agree)."""
+    try:
+        if op == "create":
+            return ctx.bar_create(arg)
+        if op == "update":
+            return ctx.bar_update(*arg)
+        return ctx.bar_destroy(arg)
+    except Exception:
+        return "err"
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_dynamic_progress_bars_match_brute_force(seed):
+    """Bars created / updated / destroyed between calls: a destroyed id takes no events (they are
+    dropped and counted), reads all-zero, and a re-created id starts from zero with its new total;
+    the oracle equals brute.py on random tiny traces."""
+    rng = np.random.default_rng(9000 + seed)
+    case = random_tiny_case(rng)
+    kw = dict(t0=case["t0"], hang_windows=case["H"], k=case["k"], rank_mode=case["mode"])
+    orc = oracle.Oracle(case["owner"], case["caps"], case["totals"], n_components=case["nc"], **kw)
+    br = brute.Brute(case["owner"], case["caps"], case["totals"], case["nc"], **kw)
+    for srows, erows, ends in case["calls"]:
+        for op, arg in _bar_ops(rng, case["nk"]):
+            assert _apply(orc, op, arg) == _apply(br, op, arg)
+        o = orc.reduce(sample_array(srows), event_array(erows), ends, want_all_stats=True)
+        b = br.reduce(srows, erows, ends)
+        _compare(o, b, case["nb"], case["nk"], case["nc"])
+
+
+def test_dynamic_progress_bars_worked_example():
+    """Bar 1 destroyed: its 2 events are dropped and it reads zero; re-created with total 5 it
+    counts only later events (L131: finished / executing / not started)."""
+    owner, cap = np.zeros(1, np.uint32), np.array([4], np.uint16)
+    orc = oracle.Oracle(owner, cap, np.array([3, 4], np.int64), n_components=1, t0=0, k=1)
+    ev = lambda rows: event_array([(t, i, pack_meta(0, kern, kind)) for t, i, kern, kind in rows])  # noqa: E731
+    r = orc.reduce(sample_array([]), ev([(1, 0, 0, 0), (2, 1, 1, 0), (3, 1, 1, 1)]), [10])
+    assert list(r["progress"][0][1].tolist()) == [4, 1, 1, 0, 3]
+    orc.bar_destroy(1)
+    r = orc.reduce(sample_array([]), ev([(11, 2, 1, 0), (12, 3, 1, 0), (13, 0, 0, 1)]), [20])
+    assert int(r["summary"]["n_dropped"][0]) == 2 and int(r["summary"]["n_events"][0]) == 1
+    assert list(r["progress"][0][1].tolist()) == [0, 0, 0, 0, 0]
+    assert list(r["progress"][0][0].tolist()) == [3, 1, 1, 0, 2]
+    assert orc.bar_create(5) == 1
+    r = orc.reduce(sample_array([]), ev([(21, 4, 1, 0)]), [30])
+    assert list(r["progress"][0][1].tolist()) == [5, 1, 0, 1, 4]
+    with pytest.raises(ValueError):
+        orc.bar_create(1)  # both ids live
