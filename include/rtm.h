@@ -64,7 +64,8 @@ enum { RTM_RANK_PERCENT = 0, RTM_RANK_SIZE = 1,
  * rtm_task_event: START or END of one task (e.g. a thread block of a GPU kernel, L91, L131).
  *   meta = component_id (bits 0..19) | kernel_id (bits 20..30) | kind (bit 31: 0 START, 1 END)
  * Field-valid sample: buffer_id < n_buffers, capacity == registered capacity, level <= capacity.
- * Field-valid event:  component_id < n_components, kernel_id < n_kernels.
+ * Field-valid event:  component_id < n_components, kernel_id < n_kernels, bar kernel_id live
+ *   (rtm_bar_destroy frees an id; every registered bar starts live).
  * Ordering contract: within the records pending at one rtm_window_reduce call, the ts of
  * field-valid samples is non-decreasing in ingest order, and likewise for field-valid events
  * (reading R15).  A violation makes the call fail with RTM_E_ORDER (sticky).       */
@@ -197,6 +198,21 @@ rtm_status rtm_window_results(rtm_ctx *ctx, uint32_t first, uint32_t count, rtm_
 rtm_status rtm_window_reduce_local(rtm_ctx *ctx, const int64_t *t_end, uint32_t n_windows,
                                    const void **pack, uint64_t *pack_bytes);
 rtm_status rtm_merge(rtm_ctx *ctx, const void *gathered, uint32_t world, rtm_window_summary *out);
+
+/* ---- Progress bar registry (CreateProgressBar / UpdateProgressBar / DestroyProgressBar, PAPER.md
+ * L99; progress bars L131).  Bar ids are the kernel_id field of task
+ * events, 0 <= id < n_kernels; every bar registered at rtm_create starts live.  Calls take
+ * effect at the next rtm_window_reduce (stream-ordered); with world > 1 every rank must make the
+ * same calls.
+ * rtm_bar_create: the lowest free id becomes live with `total` tasks and zero counts; *bar_id
+ *   receives it.  RTM_E_TOO_SMALL (no state change) when all n_kernels ids are live.
+ * rtm_bar_update: set a live bar's total (not_started = total - started).
+ * rtm_bar_destroy: free a live id.  Task events naming a free id are field-invalid (dropped and
+ *   counted) until it is created again; its progress entry reads all zero.
+ * RTM_E_INVALID (no state change) for an id that is out of range or not live. */
+rtm_status rtm_bar_create(rtm_ctx *ctx, int64_t total, uint32_t *bar_id);
+rtm_status rtm_bar_update(rtm_ctx *ctx, uint32_t bar_id, int64_t total);
+rtm_status rtm_bar_destroy(rtm_ctx *ctx, uint32_t bar_id);
 
 /* Windows-in-top-k counter (persistence): for buffers [first,
  * first+count) (global ids with a rank-local numbering), the number of windows since create /

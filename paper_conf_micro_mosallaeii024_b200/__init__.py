@@ -192,6 +192,18 @@ class Monitor:
         N.check(N.lib().rtm_buffer_stats(self._h, first, count, out.ctypes.data), "rtm_buffer_stats")
         return out
 
+    # progress bar registry (Create / Update / DestroyProgressBar)
+    def bar_create(self, total: int) -> int:
+        i = ctypes.c_uint32()
+        N.check(N.lib().rtm_bar_create(self._h, int(total), ctypes.byref(i)), "rtm_bar_create")
+        return i.value
+
+    def bar_update(self, bar: int, total: int) -> None:
+        N.check(N.lib().rtm_bar_update(self._h, int(bar), int(total)), "rtm_bar_update")
+
+    def bar_destroy(self, bar: int) -> None:
+        N.check(N.lib().rtm_bar_destroy(self._h, int(bar)), "rtm_bar_destroy")
+
     def topk_persistence(self, first: int = 0, count: int | None = None):
         """Windows-in-top-k counter per buffer since create / reset (persistence, L173, L197-L199)."""
         if count is None:

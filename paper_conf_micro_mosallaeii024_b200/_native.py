@@ -60,7 +60,8 @@ class KernelTime(ctypes.Structure):
 EXPORTS = ("rtm_create", "rtm_destroy", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers",
            "rtm_progress", "rtm_hang_check", "rtm_buffer_stats", "rtm_window_results", "rtm_window_reduce_local",
            "rtm_merge", "rtm_profile", "rtm_profile_read", "rtm_status_str", "rtm_version",
-           "rtm_kernel_launches", "rtm_watch", "rtm_watch_series", "rtm_topk_persistence")
+           "rtm_kernel_launches", "rtm_watch", "rtm_watch_series", "rtm_topk_persistence",
+           "rtm_bar_create", "rtm_bar_update", "rtm_bar_destroy")
 
 _lib = None
 
@@ -92,8 +93,12 @@ def lib():
     L.rtm_profile_read.argtypes = [vp, vp, u32, P(u32)]
     L.rtm_watch.argtypes = [vp, vp, u32]
     L.rtm_topk_persistence.argtypes = [vp, u32, u32, vp]
+    L.rtm_bar_create.argtypes = [vp, ctypes.c_int64, P(u32)]
+    L.rtm_bar_update.argtypes = [vp, u32, ctypes.c_int64]
+    L.rtm_bar_destroy.argtypes = [vp, u32]
     L.rtm_watch_series.argtypes = [vp, u32, vp, P(u32)]
-    for fn in ("rtm_watch", "rtm_watch_series", "rtm_topk_persistence", "rtm_create", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers", "rtm_progress",
+    for fn in ("rtm_watch", "rtm_watch_series", "rtm_topk_persistence", "rtm_bar_create", "rtm_bar_update",
+               "rtm_bar_destroy", "rtm_create", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers", "rtm_progress",
                "rtm_hang_check", "rtm_buffer_stats", "rtm_window_reduce_local", "rtm_merge", "rtm_profile",
                "rtm_profile_read", "rtm_window_results"):
         getattr(L, fn).restype = ctypes.c_int

@@ -53,6 +53,9 @@ struct rtm_ctx {
   DevBuf tkscr;             // per-slice top-k candidates (few-window calls)
   DevBuf mkey, rcp64;       // rank mode MEAN: per-(window, buffer) order keys, floor(2^64 / c)
   DevBuf persist;           // windows-in-top-k counter per buffer (id space)
+  DevBuf klive;             // progress bar ids in use
+  std::vector<uint8_t> klive_h;
+  std::vector<int64_t> ktotal0;  // bar totals registered at create (restored by reset)
   // value monitor: watched ids (as given), their local ids (~0: not on this rank), rings
   std::vector<uint32_t> gid_h;  // host copy of the global ids (rank-local numbering)
   uint32_t n_watch = 0;
@@ -237,6 +240,10 @@ rtm_status zero_state(rtm_ctx *c) {
   cl.add(c->persist.p, (size_t)(c->n_global ? c->n_global : c->nb) * 4);
   launch_clear(cl, c->st);
   CK(cudaGetLastError());
+  c->klive_h.assign(c->nk, 1);  // every registered bar live, registered totals
+  CK(cudaMemcpyAsync(c->klive.p, c->klive_h.data(), c->nk, cudaMemcpyHostToDevice, c->st));
+  CK(cudaMemcpyAsync(c->ktotal.p, c->ktotal0.data(), (size_t)c->nk * 8, cudaMemcpyHostToDevice, c->st));
+  CK(cudaStreamSynchronize(c->st));  // pageable sources
   c->cur = 0;
   c->t_prev = c->t0;
   c->have = false;
@@ -342,6 +349,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.rank_mode = c->rank_mode; p.H = c->H;
   p.cap = (const uint16_t *)c->cap.p; p.owner = (const uint32_t *)c->owner.p;
   p.elig = (const uint8_t *)c->elig.p; p.ktotal = (const int64_t *)c->ktotal.p;
+  p.klive = (const uint8_t *)c->klive.p;
   p.rcp = (const unsigned long long *)c->rcp.p; p.elig_ids = (const uint32_t *)c->elig_ids.p; p.n_elig = c->n_elig;
   p.W = W; p.epoch = c->epoch;
   p.narrow = 1;
@@ -627,8 +635,10 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
       (s = ensure(c, c->kend, (size_t)c->nk * 8)) || (s = ensure(c, c->cstart, (size_t)c->nc * 8)) ||
       (s = ensure(c, c->cend, (size_t)c->nc * 8)) || (s = ensure(c, c->rcp, (size_t)65536 * 8)) ||
       (s = ensure(c, c->elig_ids, (size_t)c->nb * 4)) ||
-      (s = ensure(c, c->persist, (size_t)(c->n_global ? c->n_global : c->nb) * 4)))
+      (s = ensure(c, c->persist, (size_t)(c->n_global ? c->n_global : c->nb) * 4)) ||
+      (s = ensure(c, c->klive, (size_t)c->nk)))
     return fail(s);
+  c->ktotal0.assign(cfg->kernel_total, cfg->kernel_total + c->nk);
   if (c->rank_mode == RTM_RANK_MEAN) {
     if ((s = ensure(c, c->rcp64, (size_t)65536 * 8))) return fail(s);
     std::vector<unsigned long long> r64(65536, 0);
@@ -705,6 +715,45 @@ rtm_status rtm_reset(rtm_ctx *c) {
   c->sticky = 0;
   for (uint32_t q = 0; q < RTM_WATCH_MAX; ++q) c->ring_head[q] = c->ring_n[q] = 0;
   return zero_state(c);
+}
+
+rtm_status rtm_bar_create(rtm_ctx *c, int64_t total, uint32_t *bar_id) {
+  if (!c || !bar_id) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  uint32_t k = 0;
+  while (k < c->nk && c->klive_h[k]) ++k;
+  if (k == c->nk) return RTM_E_TOO_SMALL;
+  CK(cudaSetDevice(c->device));
+  const int64_t zero = 0;
+  const uint8_t one = 1;
+  CK(cudaMemcpyAsync((int64_t *)c->ktotal.p + k, &total, 8, cudaMemcpyHostToDevice, c->st));
+  CK(cudaMemcpyAsync((int64_t *)c->kstart.p + k, &zero, 8, cudaMemcpyHostToDevice, c->st));
+  CK(cudaMemcpyAsync((int64_t *)c->kend.p + k, &zero, 8, cudaMemcpyHostToDevice, c->st));
+  CK(cudaMemcpyAsync((uint8_t *)c->klive.p + k, &one, 1, cudaMemcpyHostToDevice, c->st));
+  CK(cudaStreamSynchronize(c->st));  // pageable stack sources
+  c->klive_h[k] = 1;
+  *bar_id = k;
+  return RTM_OK;
+}
+
+rtm_status rtm_bar_update(rtm_ctx *c, uint32_t bar_id, int64_t total) {
+  if (!c || bar_id >= c->nk || !c->klive_h[bar_id]) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  CK(cudaSetDevice(c->device));
+  CK(cudaMemcpyAsync((int64_t *)c->ktotal.p + bar_id, &total, 8, cudaMemcpyHostToDevice, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  return RTM_OK;
+}
+
+rtm_status rtm_bar_destroy(rtm_ctx *c, uint32_t bar_id) {
+  if (!c || bar_id >= c->nk || !c->klive_h[bar_id]) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  CK(cudaSetDevice(c->device));
+  const uint8_t zero = 0;
+  CK(cudaMemcpyAsync((uint8_t *)c->klive.p + bar_id, &zero, 1, cudaMemcpyHostToDevice, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  c->klive_h[bar_id] = 0;
+  return RTM_OK;
 }
 
 rtm_status rtm_topk_persistence(rtm_ctx *c, uint32_t first, uint32_t count, uint32_t *out) {

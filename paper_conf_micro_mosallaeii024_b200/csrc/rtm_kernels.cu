@@ -75,7 +75,8 @@ __device__ __forceinline__ bool sample_valid(const Params &p, const int4 &v) {
 }
 __device__ __forceinline__ bool event_valid(const Params &p, const int4 &v) {
   unsigned meta = (unsigned)v.w;
-  return (meta & 0xFFFFFu) < p.nc && ((meta >> 20) & 0x7FFu) < p.nk;
+  const unsigned kern = (meta >> 20) & 0x7FFu;
+  return (meta & 0xFFFFFu) < p.nc && kern < p.nk && __ldg(p.klive + kern);
 }
 
 // region r of a call: 0 head (ts < t_begin), 1..W window r-1, W+1 tail (ts >= t_end[W-1])
@@ -1647,7 +1648,8 @@ __global__ void __launch_bounds__(256) k_progress(Params p) {
   const unsigned k = blockIdx.x;
   if (k < p.nk) {
     long long s = p.kstart[k], e = p.kend[k];
-    const long long total = p.ktotal[k];
+    const bool live = p.klive[k] != 0;  // a free bar id reads all zero (its counts stay zero)
+    const long long total = live ? p.ktotal[k] : 0;
     for (unsigned base = 0; base < p.W; base += blockDim.x) {
       const unsigned w = base + threadIdx.x;
       unsigned ds = 0, de = 0;
@@ -1662,10 +1664,10 @@ __global__ void __launch_bounds__(256) k_progress(Params p) {
         long long S = s + xs + ds, E = e + xe + de;
         long long *o = p.prog + ((size_t)w * p.nk + k) * 5;
         o[0] = total;
-        o[1] = S;
-        o[2] = E;
-        o[3] = S - E;
-        o[4] = total - S;
+        o[1] = live ? S : 0;
+        o[2] = live ? E : 0;
+        o[3] = live ? S - E : 0;
+        o[4] = live ? total - S : 0;
       }
       s += ts_;
       e += te_;

@@ -524,3 +524,52 @@ def test_mean_mode_rejects_long_windows():
         mon.window_reduce(np.array([1 << 33], np.int64))
     got = mon.window_reduce(np.array([10], np.int64))  # state unchanged: the next call works
     assert int(got["summary"]["t_begin"][0]) == 0
+
+
+@pytest.mark.parametrize("seed", range(25))
+def test_dynamic_progress_bars_random(seed):
+    """Bars created / updated / destroyed between calls: GPU vs oracle on random
+    tiny traces, including the dropped events of destroyed ids and zero entries."""
+    from tests.test_oracle import _apply, _bar_ops
+    rng = np.random.default_rng(9000 + seed)
+    case = random_tiny_case(rng)
+    kw = dict(t0=case["t0"], hang_windows=case["H"], k=case["k"], rank_mode=case["mode"])
+    orc, mon = _pair(case["owner"], case["caps"], case["totals"], case["nc"], **kw)
+    for srows, erows, ends in case["calls"]:
+        for op, arg in _bar_ops(rng, case["nk"]):
+            assert _apply(orc, op, arg) == _apply(mon, op, arg)
+        ref = orc.reduce(sample_array(srows), event_array(erows), ends)
+        mon.ingest(sample_array(srows), event_array(erows))
+        got = mon.window_reduce(np.array(ends, np.int64))
+        assert_same(got, ref, mon)
+
+
+def test_dynamic_progress_bars_c1_kernels_retired():
+    """C1 with its 4 kernel bars: after window 4 bar 0 is destroyed (its remaining thread blocks
+    become invalid records) and re-created for a new kernel with another total; the GPU matches
+    the oracle on every window, and rtm_reset restores the registry."""
+    wl = gen.C1
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    s, e = gen.samples(wl), gen.events(wl)
+    for lo, hi in ((0, 4), (4, 7), (7, 10)):
+        if lo == 4:
+            for x in (orc, mon):
+                x.bar_destroy(0)
+                x.bar_update(3, 12345)
+        if lo == 7:
+            assert orc.bar_create(777) == mon.bar_create(777) == 0
+        sl = slice(wl.index_at("samples", wl.t_begin(lo)), wl.index_at("samples", wl.t_begin(hi)))
+        el = slice(wl.index_at("events", wl.t_begin(lo)), wl.index_at("events", wl.t_begin(hi)))
+        ref = orc.reduce(s[sl], e[el], wl.t_end()[lo:hi])
+        mon.ingest(_dev(s[sl]), _dev(e[el]))
+        got = mon.window_reduce(wl.t_end()[lo:hi])
+        assert_same(got, ref, mon)
+    with pytest.raises(RTMError):
+        mon.bar_create(1)  # every id live again
+    mon.reset()
+    orc.reset()
+    ref = orc.reduce(s[:1000], e[:100], wl.t_end()[:1])
+    mon.ingest(_dev(s[:1000]), _dev(e[:100]))
+    assert_same(mon.window_reduce(wl.t_end()[:1]), ref, mon)
