@@ -32,7 +32,8 @@ class _Config(ctypes.Structure):
     _fields_ = [("n_buffers", ctypes.c_uint32), ("n_components", ctypes.c_uint32), ("n_kernels", ctypes.c_uint32),
                 ("buffer_owner", ctypes.c_void_p), ("buffer_capacity", ctypes.c_void_p),
                 ("kernel_total", ctypes.c_void_p), ("t0", ctypes.c_int64), ("hang_windows", ctypes.c_uint32),
-                ("k", ctypes.c_uint32), ("rank_mode", ctypes.c_int32), ("owned", ctypes.c_void_p)]
+                ("k", ctypes.c_uint32), ("rank_mode", ctypes.c_int32), ("owned", ctypes.c_void_p),
+                ("hang_mode", ctypes.c_int32)]
 
 
 _lib = None
@@ -76,7 +77,7 @@ class Oracle:
     """Stateful oracle context (mirrors rtm_create / rtm_window_reduce semantics)."""
 
     def __init__(self, owner, capacity, kernel_total, *, n_components=None, t0=0, hang_windows=8, k=16, rank_mode=0,
-                 owned=None):
+                 owned=None, hang_mode=0):
         self.owner = np.ascontiguousarray(owner, dtype=np.uint32)
         self.capacity = np.ascontiguousarray(capacity, dtype=np.uint16)
         self.kernel_total = np.ascontiguousarray(kernel_total, dtype=np.int64)
@@ -88,7 +89,7 @@ class Oracle:
         self.k = k
         self.owned = None if owned is None else np.ascontiguousarray(owned, dtype=np.uint8)
         cfg = _Config(self.n_buffers, self.n_components, self.n_kernels, _ptr(self.owner), _ptr(self.capacity),
-                      _ptr(self.kernel_total), t0, hang_windows, k, rank_mode, _ptr(self.owned))
+                      _ptr(self.kernel_total), t0, hang_windows, k, rank_mode, _ptr(self.owned), hang_mode)
         self._h = lib().orc_create(ctypes.byref(cfg))
         if not self._h:
             raise ValueError("orc_create rejected the configuration")

@@ -43,12 +43,12 @@ class OrderError(Exception):
 
 class Brute:
     def __init__(self, owner, capacity, kernel_total, n_components, *, t0=0, hang_windows=8, k=16, rank_mode=0,
-                 owned=None):
+                 owned=None, hang_mode=0):
         self.owner = [int(x) for x in owner]
         self.cap = [int(x) for x in capacity]
         self.total = [int(x) for x in kernel_total]
         self.nb, self.nc, self.nk = len(self.owner), int(n_components), len(self.total)
-        self.H, self.k, self.mode = hang_windows, k, rank_mode
+        self.H, self.k, self.mode, self.hang_mode = hang_windows, k, rank_mode, hang_mode
         self.owned = [1] * self.nc if owned is None else [int(x) for x in owned]
         self.t_prev = t0
         self.lvl = [0] * self.nb
@@ -180,7 +180,9 @@ class Brute:
             top = [(b, self.lvl[b], self.cap[b]) for b in order[: self.k]]
             hung = []
             for c in range(self.nc):
-                anyfull = any(stats[b]["min"] == self.cap[b] for b in range(self.nb) if self.owner[b] == c)
+                held = (lambda b: stats[b]["min"] >= 1) if self.hang_mode == 1 else \
+                    (lambda b: stats[b]["min"] == self.cap[b])
+                anyfull = any(held(b) for b in range(self.nb) if self.owner[b] == c)
                 cond = anyfull and not active[c]
                 self.run[c] = self.run[c] + 1 if cond else 0
                 if self.run[c] >= self.H:
@@ -190,3 +192,30 @@ class Brute:
                             topk=top, progress=progress, hung=hung, stats=stats))
         self.t_prev = t_end[-1]
         return out
+
+
+def hang_roots(flagged, src, dst):
+    """Root causes among hang-flagged components:
+    with the links restricted to flagged components ("c sends to d"), c is a root iff every
+    flagged component reachable from c can reach c back (c lies in a sink strongly-connected
+    component: a circular wait, or a stuck component with no flagged successor).  Brute-force
+    reachability, ascending ids."""
+    F = set(int(x) for x in flagged)
+    succ = {c: [] for c in F}
+    for a, b in zip(src, dst):
+        a, b = int(a), int(b)
+        if a in F and b in F:
+            succ[a].append(b)
+
+    def reach(c):
+        seen, todo = {c}, [c]
+        while todo:
+            x = todo.pop()
+            for y in succ[x]:
+                if y not in seen:
+                    seen.add(y)
+                    todo.append(y)
+        return seen
+
+    R = {c: reach(c) for c in F}
+    return sorted(c for c in F if all(c in R[d] for d in R[c]))

@@ -20,7 +20,7 @@ struct orc_ctx {
   int64_t *ktotal;
   uint8_t *owned;
   uint32_t H, k;
-  int32_t rank_mode;
+  int32_t rank_mode, hang_mode;
   int64_t t0, t_prev;
   uint16_t *lvl;       /* level of every buffer at the end of the last reduced window */
   int64_t *c_started, *c_ended, *k_started, *k_ended;
@@ -73,6 +73,7 @@ orc_ctx *orc_create(const orc_config *cfg) {
   c->H = cfg->hang_windows;
   c->k = cfg->k;
   c->rank_mode = cfg->rank_mode;
+  c->hang_mode = cfg->hang_mode;
   c->t0 = cfg->t0;
   c->lvl = (uint16_t *)malloc(sizeof(uint16_t) * c->nb);
   c->c_started = (int64_t *)malloc(sizeof(int64_t) * c->nc);
@@ -274,7 +275,9 @@ int orc_reduce(orc_ctx *c, const orc_sample *s, uint64_t ns, const orc_event *e,
     uint32_t touched = 0;
     for (uint32_t b = 0; b < nb; ++b) {
       I[b] += (uint64_t)L[b] * (uint64_t)(te - t[b]);
-      full[b] = (mn[b] == c->cap[b]); /* full for the whole window, carry-in included */
+      /* held for the whole window, carry-in included: full (R9) or, in the paper's looser
+       * reading, non-empty ("any content in a buffer", L229) */
+      full[b] = c->hang_mode == 1 ? (mn[b] >= 1) : (mn[b] == c->cap[b]);
       c->lvl[b] = L[b];
       if (cnt[b] > 0) {
         touched++;

@@ -36,6 +36,7 @@ typedef struct {
   uint32_t k;
   int32_t rank_mode;               /* 0 percent, 1 size, 2 window mean occupancy */
   const uint8_t *owned;            /* [n_components] nullable: shard ownership, restricts ranking */
+  int32_t hang_mode;               /* 0: a buffer full all window; 1: non-empty all window (L229) */
 } orc_config;
 
 typedef struct {

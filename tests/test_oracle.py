@@ -637,3 +637,42 @@ def test_dynamic_progress_bars_worked_example():
     assert list(r["progress"][0][1].tolist()) == [5, 1, 0, 1, 4]
     with pytest.raises(ValueError):
         orc.bar_create(1)  # both ids live
+
+
+# ---------------------------------------------------------------------------------------------
+# Looser hang criterion and root causes
+def test_hang_roots_case_study_2_and_chain():
+    """Case study 2 (L217, L229, L235): L1 (0) and the DRAM controller (3) back up behind the L2
+    write buffer (2) <-> local storage (1) circular wait: roots {1, 2}.  Fig. 4's chain A -> B ->
+    C -> D (L161) with B and C stuck: C is the root (B waits on it); with D stuck too, D is."""
+    src, dst = [0, 3, 2, 1, 0], [2, 1, 1, 2, 4]
+    assert brute.hang_roots([0, 1, 2, 3], src, dst) == [1, 2]
+    assert brute.hang_roots([0, 3], src, dst) == [0, 3]  # nothing flagged downstream of them
+    chain_s, chain_d = [0, 1, 2], [1, 2, 3]
+    assert brute.hang_roots([1, 2], chain_s, chain_d) == [2]
+    assert brute.hang_roots([1, 2, 3], chain_s, chain_d) == [3]
+    assert brute.hang_roots([], chain_s, chain_d) == []
+
+
+def test_nonempty_hang_mode_matches_brute_force_and_flags_back_pressure():
+    """RTM_HANG_NONEMPTY ("any content in a buffer", L229) against brute.py on random tiny traces;
+    and on the constructed deadlock it also flags the backed-up components earlier than the full
+    criterion does (a non-empty buffer is enough)."""
+    for seed in range(30):
+        rng = np.random.default_rng(11000 + seed)
+        case = random_tiny_case(rng)
+        kw = dict(t0=case["t0"], hang_windows=case["H"], k=case["k"], rank_mode=case["mode"], hang_mode=1)
+        orc = oracle.Oracle(case["owner"], case["caps"], case["totals"], n_components=case["nc"], **kw)
+        br = brute.Brute(case["owner"], case["caps"], case["totals"], case["nc"], **kw)
+        for srows, erows, ends in case["calls"]:
+            o = orc.reduce(sample_array(srows), event_array(erows), ends, want_all_stats=True)
+            _compare(o, br.reduce(srows, erows, ends), case["nb"], case["nk"], case["nc"])
+    # one buffer at 1 of 4 (non-empty, not full) in a silent component: window 0 starts empty (the
+    # carry-in 0 counts), windows 1 and 2 are non-empty throughout: flagged at window 2 (H = 2)
+    orc = oracle.Oracle(np.zeros(1, np.uint32), np.array([4], np.uint16), np.ones(1, np.int64), n_components=1,
+                        t0=0, hang_windows=2, k=1, hang_mode=1)
+    r = orc.reduce(sample_array([(0, 0, 1, 4)]), event_array([]), [10, 20, 30])
+    assert r["hung"][:, 0].tolist() == [0, 0, 1]
+    full = oracle.Oracle(np.zeros(1, np.uint32), np.array([4], np.uint16), np.ones(1, np.int64), n_components=1,
+                         t0=0, hang_windows=2, k=1, hang_mode=0)
+    assert full.reduce(sample_array([(0, 0, 1, 4)]), event_array([]), [10, 20, 30])["hung"].sum() == 0
