@@ -50,6 +50,14 @@ typedef enum {
 } rtm_status;
 
 enum { RTM_MEM_HOST = 0, RTM_MEM_DEVICE = 1 };
+/* Which buffers count toward the hang condition (a component with such a buffer for the whole
+ * window and no task event, H windows in a row, is flagged):
+ * RTM_HANG_FULL: a buffer at capacity the whole window (R9, the default);
+ * RTM_HANG_NONEMPTY: a buffer non-empty the whole window — the paper's own, looser sign: "if
+ *   there is any content in a buffer, we know the buffer owner cannot proceed" (L229; SURVEY.md
+ *   §8(f) row 4).  It also flags components backed up behind the stuck one (back-pressure,
+ *   L229); rtm_hang_roots separates those given the component connection graph. */
+enum { RTM_HANG_FULL = 0, RTM_HANG_NONEMPTY = 1 };
 /* "sort the buffers by their fullness percentage or by the number of elements" */
 enum { RTM_RANK_PERCENT = 0, RTM_RANK_SIZE = 1,
        /* persistence ranking (a buffer "repeatedly at the top of the list"
@@ -120,6 +128,7 @@ typedef struct {
   const uint32_t *buffer_global_id; /* host [n_buffers] or NULL (ids are global)               */
   uint32_t n_global_buffers;        /* > every global id; 0 when buffer_global_id is NULL       */
   uint32_t pack_buffers;
+  int32_t hang_mode;                /* RTM_HANG_FULL (0, default) or RTM_HANG_NONEMPTY          */
 } rtm_config;
 
 /* ---- per-window outputs --------------------------------------------------------------------- */
@@ -183,6 +192,20 @@ rtm_status rtm_topk_buffers(rtm_ctx *ctx, uint32_t window, rtm_topk_entry *out, 
 rtm_status rtm_progress(rtm_ctx *ctx, uint32_t window, rtm_progress_entry *bars, rtm_component_tasks *comps);
 /* Hang-flagged component ids of `window`, ascending.  Writes min(cap, n) ids; *n_hung = n. */
 rtm_status rtm_hang_check(rtm_ctx *ctx, uint32_t window, uint32_t *comp_ids, uint32_t cap, uint32_t *n_hung);
+/* Hang root causes (L229-L235, L342-L344).  The paper finds the stuck
+ * components by hand: flagged components may only be backed up behind the real culprit
+ * ("caused by buffer backpressure", L229; "L1 cache and DRAM controllers cannot make progress
+ * because they cannot send messages to L2 caches", L235) and names a graph of component
+ * connections as the missing view (L342-L344).  Given that graph:
+ * rtm_set_links: n_links directed links, component src[i] sends to component dst[i] (host
+ *   arrays; replaces the previous graph; ids < n_components, else RTM_E_INVALID).
+ * rtm_hang_roots: among the components flagged in `window` (last batch), the members of the
+ *   sink strongly-connected components of the links restricted to flagged components: a
+ *   circular wait (case study 2, L217) or a stuck component whose successors are not flagged;
+ *   components flagged only because they wait on one of those are left out.  Ascending ids;
+ *   writes min(cap, n) ids, *n_roots = n.  Computed on the host from the window's flagged set. */
+rtm_status rtm_set_links(rtm_ctx *ctx, const uint32_t *src, const uint32_t *dst, uint32_t n_links);
+rtm_status rtm_hang_roots(rtm_ctx *ctx, uint32_t window, uint32_t *comp_ids, uint32_t cap, uint32_t *n_roots);
 /* Full per-buffer table of the last window of the batch for buffers [first, first+count)
  * (global ids when the context uses a rank-local numbering; buffers of no rank read as zero). */
 rtm_status rtm_buffer_stats(rtm_ctx *ctx, uint32_t first, uint32_t count, rtm_buffer_stat *out);

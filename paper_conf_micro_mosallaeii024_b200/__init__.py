@@ -60,7 +60,7 @@ class Monitor:
     def __init__(self, buffer_owner, buffer_capacity, kernel_total, *, n_components: int, t0: int = 0,
                  hang_windows: int = 8, k: int = 64, rank_mode: int = RTM_RANK_PERCENT, device: int = 0,
                  rank: int = 0, world: int = 1, owned_components=None, stream=None, process_group=None,
-                 buffer_global_id=None, n_global_buffers: int = 0, pack_buffers: int = 0):
+                 buffer_global_id=None, n_global_buffers: int = 0, pack_buffers: int = 0, hang_mode: int = 0):
         import torch
 
         if not torch.cuda.is_available():
@@ -88,6 +88,7 @@ class Monitor:
         cfg.buffer_global_id = None if self._gid is None else self._gid.ctypes.data
         cfg.n_global_buffers = int(n_global_buffers)
         cfg.pack_buffers = int(pack_buffers)
+        cfg.hang_mode = int(hang_mode)
         self.n_table = int(n_global_buffers) if self._gid is not None else self.n_buffers
         h = ctypes.c_void_p()
         N.check(N.lib().rtm_create(ctypes.byref(cfg), ctypes.byref(h)), "rtm_create")
@@ -184,6 +185,23 @@ class Monitor:
         N.check(N.lib().rtm_hang_check(self._h, window, ids.ctypes.data, len(ids), ctypes.byref(n)),
                 "rtm_hang_check")
         return ids[: n.value]
+
+    def set_links(self, src, dst):
+        """Component connection graph (component src[i] sends to dst[i]) for hang_roots."""
+        a = np.ascontiguousarray(src, dtype=np.uint32)
+        b = np.ascontiguousarray(dst, dtype=np.uint32)
+        if a.shape != b.shape:
+            raise ValueError("src and dst must have the same length")
+        N.check(N.lib().rtm_set_links(self._h, a.ctypes.data if len(a) else None, b.ctypes.data if len(b) else None,
+                                      len(a)), "rtm_set_links")
+
+    def hang_roots(self, window: int):
+        """Root causes among the window's flagged components (sink SCCs of the flagged links)."""
+        cap = self.n_components
+        out = np.zeros(max(1, cap), np.uint32)
+        n = ctypes.c_uint32()
+        N.check(N.lib().rtm_hang_roots(self._h, window, out.ctypes.data, cap, ctypes.byref(n)), "rtm_hang_roots")
+        return out[: n.value].copy()
 
     def buffer_stats(self, first: int = 0, count: int | None = None):
         if count is None:

@@ -47,7 +47,7 @@ class Config(ctypes.Structure):
         ("world", ctypes.c_int32), ("owned_components", ctypes.c_void_p), ("allgather", ALLGATHER_FN),
         ("allgather_user", ctypes.c_void_p), ("stream", ctypes.c_void_p),
         ("buffer_global_id", ctypes.c_void_p), ("n_global_buffers", ctypes.c_uint32),
-        ("pack_buffers", ctypes.c_uint32),
+        ("pack_buffers", ctypes.c_uint32), ("hang_mode", ctypes.c_int32),
     ]
 
 
@@ -61,7 +61,7 @@ EXPORTS = ("rtm_create", "rtm_destroy", "rtm_reset", "rtm_ingest", "rtm_window_r
            "rtm_progress", "rtm_hang_check", "rtm_buffer_stats", "rtm_window_results", "rtm_window_reduce_local",
            "rtm_merge", "rtm_profile", "rtm_profile_read", "rtm_status_str", "rtm_version",
            "rtm_kernel_launches", "rtm_watch", "rtm_watch_series", "rtm_topk_persistence",
-           "rtm_bar_create", "rtm_bar_update", "rtm_bar_destroy")
+           "rtm_bar_create", "rtm_bar_update", "rtm_bar_destroy", "rtm_set_links", "rtm_hang_roots")
 
 _lib = None
 
@@ -96,9 +96,11 @@ def lib():
     L.rtm_bar_create.argtypes = [vp, ctypes.c_int64, P(u32)]
     L.rtm_bar_update.argtypes = [vp, u32, ctypes.c_int64]
     L.rtm_bar_destroy.argtypes = [vp, u32]
+    L.rtm_set_links.argtypes = [vp, vp, vp, u32]
+    L.rtm_hang_roots.argtypes = [vp, u32, vp, u32, P(u32)]
     L.rtm_watch_series.argtypes = [vp, u32, vp, P(u32)]
     for fn in ("rtm_watch", "rtm_watch_series", "rtm_topk_persistence", "rtm_bar_create", "rtm_bar_update",
-               "rtm_bar_destroy", "rtm_create", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers", "rtm_progress",
+               "rtm_bar_destroy", "rtm_set_links", "rtm_hang_roots", "rtm_create", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers", "rtm_progress",
                "rtm_hang_check", "rtm_buffer_stats", "rtm_window_reduce_local", "rtm_merge", "rtm_profile",
                "rtm_profile_read", "rtm_window_results"):
         getattr(L, fn).restype = ctypes.c_int

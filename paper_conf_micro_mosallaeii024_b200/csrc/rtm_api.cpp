@@ -40,7 +40,7 @@ const char *kKernelNames[KT_N] = {"k_split", "k_partition", "k_events", "k_fold"
 struct rtm_ctx {
   // registry
   uint32_t nb, nc, nk, nbins, ncw, k, H;
-  int32_t rank_mode, device, rank, world;
+  int32_t rank_mode, device, rank, world, hang_mode;
   int64_t t0;
   rtm_allgather_fn allgather;
   void *allgather_user;
@@ -56,6 +56,8 @@ struct rtm_ctx {
   DevBuf klive;             // progress bar ids in use
   std::vector<uint8_t> klive_h;
   std::vector<int64_t> ktotal0;  // bar totals registered at create (restored by reset)
+  bool bars_dirty = true;        // registry changed since create / the last reset
+  std::vector<uint32_t> link_off, link_dst;  // component connection graph (CSR by source)
   // value monitor: watched ids (as given), their local ids (~0: not on this rank), rings
   std::vector<uint32_t> gid_h;  // host copy of the global ids (rank-local numbering)
   uint32_t n_watch = 0;
@@ -240,10 +242,13 @@ rtm_status zero_state(rtm_ctx *c) {
   cl.add(c->persist.p, (size_t)(c->n_global ? c->n_global : c->nb) * 4);
   launch_clear(cl, c->st);
   CK(cudaGetLastError());
-  c->klive_h.assign(c->nk, 1);  // every registered bar live, registered totals
-  CK(cudaMemcpyAsync(c->klive.p, c->klive_h.data(), c->nk, cudaMemcpyHostToDevice, c->st));
-  CK(cudaMemcpyAsync(c->ktotal.p, c->ktotal0.data(), (size_t)c->nk * 8, cudaMemcpyHostToDevice, c->st));
-  CK(cudaStreamSynchronize(c->st));  // pageable sources
+  if (c->bars_dirty) {  // every registered bar live with its registered total (only after changes:
+    c->klive_h.assign(c->nk, 1);  // reset sits inside streaming loops, keep it free of host syncs)
+    CK(cudaMemcpyAsync(c->klive.p, c->klive_h.data(), c->nk, cudaMemcpyHostToDevice, c->st));
+    CK(cudaMemcpyAsync(c->ktotal.p, c->ktotal0.data(), (size_t)c->nk * 8, cudaMemcpyHostToDevice, c->st));
+    CK(cudaStreamSynchronize(c->st));  // pageable sources
+    c->bars_dirty = false;
+  }
   c->cur = 0;
   c->t_prev = c->t0;
   c->have = false;
@@ -346,10 +351,11 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
 
   memset(&p, 0, sizeof(p));
   p.nb = c->nb; p.nc = c->nc; p.nk = c->nk; p.nbins = c->nbins; p.ncw = c->ncw; p.k = c->k;
-  p.rank_mode = c->rank_mode; p.H = c->H;
+  p.rank_mode = c->rank_mode; p.H = c->H; p.hang_mode = c->hang_mode;
   p.cap = (const uint16_t *)c->cap.p; p.owner = (const uint32_t *)c->owner.p;
   p.elig = (const uint8_t *)c->elig.p; p.ktotal = (const int64_t *)c->ktotal.p;
   p.klive = (const uint8_t *)c->klive.p;
+  p.all_live = std::find(c->klive_h.begin(), c->klive_h.end(), (uint8_t)0) == c->klive_h.end();
   p.rcp = (const unsigned long long *)c->rcp.p; p.elig_ids = (const uint32_t *)c->elig_ids.p; p.n_elig = c->n_elig;
   p.W = W; p.epoch = c->epoch;
   p.narrow = 1;
@@ -579,6 +585,7 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   if (cfg->rank_mode != RTM_RANK_PERCENT && cfg->rank_mode != RTM_RANK_SIZE && cfg->rank_mode != RTM_RANK_MEAN)
     return RTM_E_INVALID;
   if (cfg->rank_mode == RTM_RANK_MEAN && cfg->world > 1) return RTM_E_INVALID;
+  if (cfg->hang_mode != RTM_HANG_FULL && cfg->hang_mode != RTM_HANG_NONEMPTY) return RTM_E_INVALID;
   if (!cfg->buffer_owner || !cfg->buffer_capacity || !cfg->kernel_total) return RTM_E_INVALID;
   if (cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world) return RTM_E_INVALID;
   for (uint32_t b = 0; b < cfg->n_buffers; ++b)
@@ -604,6 +611,7 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   c->k = cfg->k;
   c->H = cfg->hang_windows;
   c->rank_mode = cfg->rank_mode;
+  c->hang_mode = cfg->hang_mode;
   c->device = cfg->device;
   c->rank = cfg->rank;
   c->world = cfg->world;
@@ -732,6 +740,7 @@ rtm_status rtm_bar_create(rtm_ctx *c, int64_t total, uint32_t *bar_id) {
   CK(cudaMemcpyAsync((uint8_t *)c->klive.p + k, &one, 1, cudaMemcpyHostToDevice, c->st));
   CK(cudaStreamSynchronize(c->st));  // pageable stack sources
   c->klive_h[k] = 1;
+  c->bars_dirty = true;
   *bar_id = k;
   return RTM_OK;
 }
@@ -742,6 +751,7 @@ rtm_status rtm_bar_update(rtm_ctx *c, uint32_t bar_id, int64_t total) {
   CK(cudaSetDevice(c->device));
   CK(cudaMemcpyAsync((int64_t *)c->ktotal.p + bar_id, &total, 8, cudaMemcpyHostToDevice, c->st));
   CK(cudaStreamSynchronize(c->st));
+  c->bars_dirty = true;
   return RTM_OK;
 }
 
@@ -753,6 +763,7 @@ rtm_status rtm_bar_destroy(rtm_ctx *c, uint32_t bar_id) {
   CK(cudaMemcpyAsync((uint8_t *)c->klive.p + bar_id, &zero, 1, cudaMemcpyHostToDevice, c->st));
   CK(cudaStreamSynchronize(c->st));
   c->klive_h[bar_id] = 0;
+  c->bars_dirty = true;
   return RTM_OK;
 }
 
@@ -938,29 +949,123 @@ rtm_status rtm_progress(rtm_ctx *c, uint32_t window, rtm_progress_entry *bars, r
   return RTM_OK;
 }
 
-rtm_status rtm_hang_check(rtm_ctx *c, uint32_t window, uint32_t *comp_ids, uint32_t cap, uint32_t *n_hung) {
-  if (!c || !n_hung || (cap && !comp_ids)) return RTM_E_INVALID;
-  if (c->sticky) return (rtm_status)c->sticky;
-  if (!c->have) return RTM_E_STATE;
-  if (window >= c->W) return RTM_E_INVALID;
+// flagged component ids of `window` of the last batch, ascending
+static rtm_status hung_list(rtm_ctx *c, uint32_t window, std::vector<uint32_t> &ids) {
   std::vector<uint32_t> bits(c->ncw);
   CK(cudaSetDevice(c->device));
   CK(cudaMemcpyAsync(bits.data(), (uint32_t *)c->hung.p + (size_t)window * c->ncw, (size_t)c->ncw * 4,
                      cudaMemcpyDeviceToHost, c->st));
   CK(cudaStreamSynchronize(c->st));
-  uint32_t n = 0;
+  ids.clear();
   for (uint32_t q = 0; q < c->ncw; ++q) {
     uint32_t x = bits[q];
     while (x) {
       const int bpos = __builtin_ctz(x);
       x &= x - 1;
       const uint32_t comp = q * 32 + bpos;
-      if (comp >= c->nc) continue;
-      if (n < cap) comp_ids[n] = comp;
-      ++n;
+      if (comp < c->nc) ids.push_back(comp);
     }
   }
-  *n_hung = n;
+  return RTM_OK;
+}
+
+rtm_status rtm_hang_check(rtm_ctx *c, uint32_t window, uint32_t *comp_ids, uint32_t cap, uint32_t *n_hung) {
+  if (!c || !n_hung || (cap && !comp_ids)) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (!c->have) return RTM_E_STATE;
+  if (window >= c->W) return RTM_E_INVALID;
+  std::vector<uint32_t> ids;
+  rtm_status s = hung_list(c, window, ids);
+  if (s) return s;
+  for (size_t i = 0; i < ids.size() && i < cap; ++i) comp_ids[i] = ids[i];
+  *n_hung = (uint32_t)ids.size();
+  return RTM_OK;
+}
+
+rtm_status rtm_set_links(rtm_ctx *c, const uint32_t *src, const uint32_t *dst, uint32_t n_links) {
+  if (!c || (n_links && (!src || !dst))) return RTM_E_INVALID;
+  for (uint32_t i = 0; i < n_links; ++i)
+    if (src[i] >= c->nc || dst[i] >= c->nc) return RTM_E_INVALID;
+  c->link_off.assign((size_t)c->nc + 1, 0);
+  for (uint32_t i = 0; i < n_links; ++i) ++c->link_off[src[i] + 1];
+  for (uint32_t q = 0; q < c->nc; ++q) c->link_off[q + 1] += c->link_off[q];
+  c->link_dst.assign(n_links, 0);
+  std::vector<uint32_t> fill(c->link_off.begin(), c->link_off.end() - 1);
+  for (uint32_t i = 0; i < n_links; ++i) c->link_dst[fill[src[i]]++] = dst[i];
+  return RTM_OK;
+}
+
+// Sink strongly-connected components of the links among the flagged set (iterative Tarjan).
+rtm_status rtm_hang_roots(rtm_ctx *c, uint32_t window, uint32_t *comp_ids, uint32_t cap, uint32_t *n_roots) {
+  if (!c || !n_roots || (cap && !comp_ids)) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (!c->have) return RTM_E_STATE;
+  if (window >= c->W) return RTM_E_INVALID;
+  std::vector<uint32_t> F;
+  rtm_status s = hung_list(c, window, F);
+  if (s) return s;
+  const size_t m = F.size();
+  auto local = [&](uint32_t comp) -> int64_t {  // index in F (sorted) or -1
+    auto it = std::lower_bound(F.begin(), F.end(), comp);
+    return (it != F.end() && *it == comp) ? (int64_t)(it - F.begin()) : -1;
+  };
+  std::vector<std::vector<uint32_t>> adj(m);  // links restricted to flagged components
+  if (!c->link_off.empty())
+    for (size_t i = 0; i < m; ++i)
+      for (uint32_t e = c->link_off[F[i]]; e < c->link_off[F[i] + 1]; ++e) {
+        const int64_t j = local(c->link_dst[e]);
+        if (j >= 0) adj[i].push_back((uint32_t)j);
+      }
+  const uint32_t kNone = 0xFFFFFFFFu;
+  std::vector<uint32_t> idx(m, kNone), low(m, 0), comp(m, kNone), stk;
+  std::vector<uint8_t> on(m, 0);
+  uint32_t counter = 0, n_scc = 0;
+  std::vector<std::pair<uint32_t, uint32_t>> call;  // (node, next edge)
+  for (size_t r = 0; r < m; ++r) {
+    if (idx[r] != kNone) continue;
+    call.push_back({(uint32_t)r, 0});
+    while (!call.empty()) {
+      const uint32_t v = call.back().first;
+      uint32_t &ei = call.back().second;
+      if (ei == 0 && idx[v] == kNone) {
+        idx[v] = low[v] = counter++;
+        stk.push_back(v);
+        on[v] = 1;
+      }
+      if (ei < adj[v].size()) {
+        const uint32_t w = adj[v][ei++];
+        if (idx[w] == kNone) call.push_back({w, 0});
+        else if (on[w]) low[v] = std::min(low[v], idx[w]);
+        continue;
+      }
+      if (low[v] == idx[v]) {  // v roots an SCC
+        uint32_t x;
+        do {
+          x = stk.back();
+          stk.pop_back();
+          on[x] = 0;
+          comp[x] = n_scc;
+        } while (x != v);
+        ++n_scc;
+      }
+      call.pop_back();
+      if (!call.empty()) {
+        const uint32_t u = call.back().first;
+        low[u] = std::min(low[u], low[v]);
+      }
+    }
+  }
+  std::vector<uint8_t> sink(n_scc, 1);  // an SCC with a link to another SCC is not a sink
+  for (size_t i = 0; i < m; ++i)
+    for (uint32_t j : adj[i])
+      if (comp[j] != comp[i]) sink[comp[i]] = 0;
+  uint32_t n = 0;
+  for (size_t i = 0; i < m; ++i)
+    if (sink[comp[i]]) {
+      if (n < cap) comp_ids[n] = F[i];
+      ++n;
+    }
+  *n_roots = n;
   return RTM_OK;
 }
 

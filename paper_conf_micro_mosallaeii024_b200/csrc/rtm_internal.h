@@ -70,11 +70,13 @@ struct Params {
   uint32_t nb, nc, nk, nbins, ncw, k;
   int32_t rank_mode;
   uint32_t H;
+  int32_t hang_mode;         // RTM_HANG_FULL / RTM_HANG_NONEMPTY
   const uint16_t *cap;
   const uint32_t *owner;
   const uint8_t *elig;       // [nb] 1 if buffer ranks on this rank
   const int64_t *ktotal;
   const uint8_t *klive;      // [nk] progress bar id in use (rtm_bar_create / rtm_bar_destroy)
+  int32_t all_live;          // every bar id live: event validity skips the klive lookup
   const unsigned long long *rcp;  // [65536] floor(2^48 / c) (exact fullness key, K5)
   const uint32_t *elig_ids;  // [n_elig] ascending ids of ranked buffers
   const uint32_t *gid;       // [nb] global buffer id (rank-local numbering) or nullptr

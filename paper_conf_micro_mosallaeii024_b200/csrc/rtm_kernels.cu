@@ -76,7 +76,7 @@ __device__ __forceinline__ bool sample_valid(const Params &p, const int4 &v) {
 __device__ __forceinline__ bool event_valid(const Params &p, const int4 &v) {
   unsigned meta = (unsigned)v.w;
   const unsigned kern = (meta >> 20) & 0x7FFu;
-  return (meta & 0xFFFFFu) < p.nc && kern < p.nk && __ldg(p.klive + kern);
+  return (meta & 0xFFFFFu) < p.nc && kern < p.nk && (p.all_live || __ldg(p.klive + kern));
 }
 
 // region r of a call: 0 head (ts < t_begin), 1..W window r-1, W+1 tail (ts >= t_end[W-1])
@@ -1114,7 +1114,7 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
       }
       const unsigned capb = __ldg(p.cap + b);
       if (p.mkey) p.mkey[(size_t)w * p.nb + b] = mean_key(I, capb, p.rcp64);
-      if (mn == capb) {
+      if (p.hang_mode == RTM_HANG_NONEMPTY ? mn >= 1u : mn == capb) {  // held the whole window
         const unsigned c = __ldg(p.owner + b);
         atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
       }

@@ -573,3 +573,50 @@ def test_dynamic_progress_bars_c1_kernels_retired():
     ref = orc.reduce(s[:1000], e[:100], wl.t_end()[:1])
     mon.ingest(_dev(s[:1000]), _dev(e[:100]))
     assert_same(mon.window_reduce(wl.t_end()[:1]), ref, mon)
+
+
+@pytest.mark.parametrize("hang_mode", [0, 1])
+def test_case_study_deadlock_roots(hang_mode):
+    """Case study 2 with the component connection graph (L1 -> L2 write buffer <-> local storage
+    <- DRAM controller, CU -> L1): the GPU's flags equal the oracle's in both hang modes, and the
+    root causes are the circular wait {1, 2} — the backed-up L1 and DRAM controller are not."""
+    from oracle import brute
+    from tests.test_oracle import _deadlock_trace
+
+    caps, S, E = _deadlock_trace()
+    owner = np.arange(5, dtype=np.uint32)
+    kw = dict(t0=0, hang_windows=2, k=5, hang_mode=hang_mode)
+    orc, mon = _pair(owner, np.array(caps, np.uint16), np.array([100], np.int64), 5, **kw)
+    src, dst = [0, 2, 1, 3, 4], [2, 1, 2, 1, 0]
+    mon.set_links(src, dst)
+    ends = [100 * (w + 1) for w in range(6)]
+    ref = orc.reduce(sample_array(S), event_array(E), ends)
+    mon.ingest(_dev(sample_array(S)), _dev(event_array(E)))
+    got = mon.window_reduce(ends)
+    assert_same(got, ref, mon)
+    for w in range(6):
+        flagged = np.nonzero(ref["hung"][w])[0]
+        assert mon.hang_roots(w).tolist() == brute.hang_roots(flagged, src, dst), w
+    assert mon.hang_roots(5).tolist() == [1, 2]
+
+
+@pytest.mark.parametrize("seed", range(20))
+def test_nonempty_hang_mode_and_roots_random(seed):
+    """RTM_HANG_NONEMPTY on random tiny traces with random connection graphs: flags equal the
+    oracle's, root causes equal the brute-force reachability definition on them."""
+    from oracle import brute
+
+    rng = np.random.default_rng(12000 + seed)
+    case = random_tiny_case(rng)
+    kw = dict(t0=case["t0"], hang_windows=case["H"], k=case["k"], rank_mode=case["mode"], hang_mode=1)
+    orc, mon = _pair(case["owner"], case["caps"], case["totals"], case["nc"], **kw)
+    nl = int(rng.integers(0, 3 * case["nc"]))
+    src, dst = rng.integers(0, case["nc"], nl), rng.integers(0, case["nc"], nl)
+    mon.set_links(src, dst)
+    for srows, erows, ends in case["calls"]:
+        ref = orc.reduce(sample_array(srows), event_array(erows), ends)
+        mon.ingest(sample_array(srows), event_array(erows))
+        got = mon.window_reduce(np.array(ends, np.int64))
+        assert_same(got, ref, mon)
+        for w in range(len(ends)):
+            assert mon.hang_roots(w).tolist() == brute.hang_roots(np.nonzero(ref["hung"][w])[0], src, dst)
