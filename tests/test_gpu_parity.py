@@ -620,3 +620,47 @@ def test_nonempty_hang_mode_and_roots_random(seed):
         assert_same(got, ref, mon)
         for w in range(len(ends)):
             assert mon.hang_roots(w).tolist() == brute.hang_roots(np.nonzero(ref["hung"][w])[0], src, dst)
+
+
+def test_limits_max_sizes_wide_windows_and_hot_buffer():
+    """Registry and record limits in one trace: 2^20 components, 2048 progress bars, k = 1024,
+    capacities 1 .. 65534 with levels up to 65534, windows of 2^33 and ~2^39 ticks next to 0- and
+    5-tick ones (the 64-bit offset paths), and one buffer with more than 65535 samples in a
+    window (the per-window sample counter's wide path); t0 far below zero."""
+    rng = np.random.default_rng(31337)
+    nb, nc, nk = 3000, 1 << 20, 2048
+    owner = ((np.arange(nb, dtype=np.int64) * 349) % nc).astype(np.uint32)
+    cap = rng.choice([1, 2, 8, 1024, 65534], size=nb).astype(np.uint16)
+    t0 = -(1 << 41)
+    lens = [1 << 33, 5, 0, (1 << 39) + 12345, 1000]
+    ends = list(np.cumsum([t0] + lens)[1:].astype(np.int64))
+    n = 300_000
+    ts = np.sort(rng.integers(t0, ends[-1], n))
+    b = rng.integers(0, nb, n).astype(np.uint32)
+    hot = (ts >= ends[2]) & (ts < ends[3]) & (rng.random(n) < 0.6)  # > 65535 samples in window 3
+    b[hot] = 7
+    lvl = (rng.random(n) * (cap[b].astype(np.float64) + 1)).astype(np.int64)
+    lvl = np.minimum(lvl, cap[b]).astype(np.uint16)
+    s = np.zeros(n, gen.SAMPLE_DTYPE)
+    s["ts"], s["buffer_id"], s["level"], s["capacity"] = ts, b, lvl, cap[b]
+    ne = 50_000
+    ets = np.sort(rng.integers(t0, ends[-1], ne))
+    comp = rng.integers(0, nc, ne).astype(np.uint32)
+    kern = rng.integers(0, nk, ne).astype(np.uint32)
+    kind = rng.integers(0, 2, ne).astype(np.uint32)
+    e = np.zeros(ne, gen.EVENT_DTYPE)
+    e["ts"], e["task_id"], e["meta"] = ets, np.arange(ne), comp | (kern << 20) | (kind << 31)
+    tot = rng.integers(0, 100, nk).astype(np.int64)
+    assert int(hot.sum()) > 65535
+    for mode in (0, 2):
+        if mode == 2:  # mean-occupancy keys need windows < 2^32 ticks: those calls are rejected
+            mon = Monitor(owner, cap, tot, n_components=nc, t0=t0, hang_windows=2, k=1024, rank_mode=2)
+            with pytest.raises(RTMError):
+                mon.window_reduce(np.array(ends, np.int64))
+            continue
+        orc, mon = _pair(owner, cap, tot, nc, t0=t0, hang_windows=2, k=1024, rank_mode=mode)
+        ref = orc.reduce(s, e, np.array(ends, np.int64))
+        assert ref["rc"] == 0
+        mon.ingest(_dev(s), _dev(e))
+        got = mon.window_reduce(np.array(ends, np.int64))
+        assert_same(got, ref, mon)  # window 3's digest covers the hot buffer's > 65535-sample count
