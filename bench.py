@@ -314,7 +314,7 @@ def finish(args, wl, world, ms, prof, n_rec, value, e2e_value, d2h, n_launches, 
     if os.path.exists(tp) and args.config == "C2-1gpu":  # traffic.json holds the C2 capture
         try:
             allt = json.load(open(tp)).get("all", {})
-            traffic = next((v for k, v in allt.items() if k == dom or k.startswith(dom + "_")), None)
+            traffic = next((v for k, v in allt.items() if k == dom or k.startswith((dom + "_", dom + "<"))), None)
         except Exception:
             traffic = None
     per_kernel = {k: {"achieved_gbs": round((prof[k]["algo_bytes"] / prof[k]["launches"]) /
