@@ -394,7 +394,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   if ((s = ensure(c, c->active, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->anyfull, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->hung, Wn * c->ncw * 4))) return s;
-  if ((s = ensure(c, c->unit_ctr, 8))) return s;
+  if ((s = ensure(c, c->unit_ctr, 16))) return s;
   if ((s = ensure(c, c->bstat, (size_t)c->nb * sizeof(rtm_buffer_stat)))) return s;
   if (c->rank_mode == RTM_RANK_MEAN) {  // order keys (windows shorter than 2^32 ticks, checked above)
     if ((s = ensure(c, c->mkey, Wn * c->nb * 8))) return s;
@@ -419,7 +419,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     cl.add(c->cdelta.p, (size_t)c->nc * 2 * 8);
     cl.add(c->active.p, Wn * c->ncw * 4);
     cl.add(c->anyfull.p, Wn * c->ncw * 4);
-    cl.add(c->unit_ctr.p, 8);
+    cl.add(c->unit_ctr.p, 16);
     launch_clear(cl, c->st);
   }
 
@@ -450,20 +450,25 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.dbg = dbg;
 #endif
   launch_fill_tile_regions(p, c->st);
-  // task events are independent of the sample path: run them on a side stream, overlapped with
-  // the partition and the fold, and join before the kernels that read their outputs (placing
-  // them after the partition or overlapping the top-k instead measured the same step time)
-  CK(cudaEventRecord(c->ev_fork, c->st));
-  CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
-  if (c->prof) prof_begin_on(c, KT_EVENTS, (uint64_t)ne * 16, c->st2);
-  launch_events(p, c->st2);
-  if (c->prof) prof_end_on(c, c->st2);
-  CK(cudaEventRecord(c->ev_join, c->st2));
+  // Task events are independent of the sample path.  Lane-major partition path: the persistent
+  // partition kernel runs the event tiles after its sample tiles (claimed dynamically), so no
+  // concurrent kernel competes with the issue-bound fold.  Otherwise: a side stream, overlapped
+  // with the partition and the fold, joined before the kernels that read the event outputs.
+  p.fuse_events = partition_fuses_events(p.nbins, nts) ? 1 : 0;
+  if (!p.fuse_events) {
+    CK(cudaEventRecord(c->ev_fork, c->st));
+    CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
+    if (c->prof) prof_begin_on(c, KT_EVENTS, (uint64_t)ne * 16, c->st2);
+    launch_events(p, c->st2);
+    if (c->prof) prof_end_on(c, c->st2);
+    CK(cudaEventRecord(c->ev_join, c->st2));
+  }
   // algorithmic bytes: partition = 16 B record in + 8 B compacted entry out per
-  // sample; fold = the 8 B entry per sample
-  LAUNCH(KT_PARTITION, (uint64_t)ns * 24, launch_partition(p, c->n_sms, c->st));
+  // sample (+ 16 B per task event when the event tiles run inside it); fold = the 8 B entry
+  LAUNCH(KT_PARTITION, (uint64_t)ns * 24 + (p.fuse_events ? (uint64_t)ne * 16 : 0),
+         launch_partition(p, c->n_sms, c->st));
   LAUNCH(KT_FOLD, (uint64_t)ns * 8, launch_fold(p, c->n_sms, c->st));
-  CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
+  if (!p.fuse_events) CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
   LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
   LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
   if (c->world == 1) launch_persist(p, c->st);  // world > 1: counted from the merged lists

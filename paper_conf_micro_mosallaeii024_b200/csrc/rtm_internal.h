@@ -112,7 +112,8 @@ struct Params {
   uint32_t *active;          // [W * ncw]
   uint32_t *anyfull;         // [W * ncw]
   uint32_t *hung;            // [W * ncw]
-  uint32_t *unit_ctr;        // [0] fold units dequeued, [1] partition tiles claimed
+  uint32_t *unit_ctr;        // [0] fold units dequeued, [1] partition tiles, [2] fused event tiles claimed
+  int32_t fuse_events;       // the persistent partition also runs the event tiles (K3 in K1)
   uint32_t *status;          // bit0 sample order, bit1 event order
   const uint16_t *carry_in;  // [nb]
   uint16_t *carry_out;       // [nb]
@@ -144,6 +145,7 @@ void launch_regions(const Params &p, cudaStream_t st);
 void launch_fill_tile_regions(const Params &p, cudaStream_t st);
 void launch_partition(const Params &p, int n_sms, cudaStream_t st);
 void launch_events(const Params &p, cudaStream_t st);
+bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s);  // lane-major partition path
 void launch_fold(const Params &p, int n_sms, cudaStream_t st);
 void launch_order_check(const Params &p, cudaStream_t st);
 void launch_topk(const Params &p, cudaStream_t st);

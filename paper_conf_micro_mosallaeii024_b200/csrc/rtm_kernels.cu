@@ -276,6 +276,124 @@ __global__ void k_fill_tiles(Params p) {
 
 
 // ============================================================================================
+// K3: task events.  One CTA per tile of <= 4096 events of one region: validate, order-check,
+// per-(window, kernel) START/END counts, per-(window, component) activity bits and per-call
+// per-component START/END deltas (progress bars, L131; "task counts stop changing", L227).
+// ============================================================================================
+// One event tile, by a whole CTA of kK3Threads (also run inside the persistent partition kernel,
+// after its sample tiles: smem = the CTA's dynamic shared memory, >= events_smem_bytes).
+__device__ __forceinline__ void events_tile(const Params &p, unsigned tile, unsigned char *smem) {
+  unsigned *khist = reinterpret_cast<unsigned *>(smem);  // [nk*2]
+  unsigned *abits = khist + 2 * p.nk;                     // [ncw] if smem_bits
+  __shared__ long long wfirst[8], wlast[8];
+  __shared__ unsigned whas[8], wviol[8], wkept[8];
+  const bool smem_bits = p.ncw <= 2048;
+
+  const unsigned r = p.tile_reg_e[tile];
+  const long long start = p.Be[r] + (long long)(tile - p.rte[r]) * kTileE;
+  long long endp = p.Be[r + 1];
+  if (endp > start + kTileE) endp = start + kTileE;
+  const int n = (int)(endp - start);
+  const Region g = region_of(p, r);
+  const bool is_win = g.window >= 0;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const unsigned lt = lanemask_lt();
+  if (is_win) {
+    for (unsigned i = threadIdx.x; i < 2 * p.nk; i += blockDim.x) khist[i] = 0;
+    if (smem_bits)
+      for (unsigned i = threadIdx.x; i < p.ncw; i += blockDim.x) abits[i] = 0;
+  }
+  __syncthreads();
+  const int4 *src = reinterpret_cast<const int4 *>(p.e) + start;
+  long long carry = kTsMin, first = kTsMax;
+  bool has = false, viol = false;
+  unsigned kept = 0;
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    int4 v[8];
+#pragma unroll
+    for (int jj = 0; jj < 8; ++jj) {
+      int i = warp * 512 + (h * 8 + jj) * 32 + lane;
+      v[jj] = i < n ? ld_stream(src + i) : make_int4(0, 0, 0, 0);
+    }
+#pragma unroll
+    for (int jj = 0; jj < 8; ++jj) {
+      const int i = warp * 512 + (h * 8 + jj) * 32 + lane;
+      const bool valid = i < n && event_valid(p, v[jj]);
+      const long long ts = rec_ts(v[jj]);
+      const unsigned vm = __ballot_sync(kFull, valid);
+      const unsigned lower = vm & lt;
+      const long long prev = shfl_ll(ts, lower ? 31 - __clz(lower) : lane);
+      if (valid && ((lower ? prev : carry) > ts || ts < g.lo_ts || ts >= g.hi_ts)) viol = true;
+      if (vm) {
+        if (!has) first = shfl_ll(ts, __ffs(vm) - 1);
+        has = true;
+        carry = shfl_ll(ts, 31 - __clz(vm));
+      }
+      const bool keep = valid && is_win;
+      kept += keep;
+      const unsigned meta = (unsigned)v[jj].w;
+      const unsigned comp = meta & 0xFFFFFu, kern = (meta >> 20) & 0x7FFu, kind = meta >> 31;
+      const unsigned kk = keep ? kern * 2 + kind : 0xFFFFFFFFu;
+      const unsigned peers = __match_any_sync(kFull, kk);
+      if (keep && lane == __ffs(peers) - 1) atomicAdd(&khist[kk], (unsigned)__popc(peers));
+      if (keep) {
+        if (smem_bits) atomicOr(&abits[comp >> 5], 1u << (comp & 31));
+        else atomicOr(p.active + (size_t)g.window * p.ncw + (comp >> 5), 1u << (comp & 31));
+        atomicAdd(p.cdelta + 2 * comp + kind, 1ull);
+      }
+    }
+  }
+  kept = warp_sum(kept);
+  const bool wv = __any_sync(kFull, viol);
+  if (lane == 0) {
+    wfirst[warp] = first;
+    wlast[warp] = carry;
+    whas[warp] = has;
+    wviol[warp] = wv;
+    wkept[warp] = kept;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    long long run = kTsMin, tf = 0;
+    bool th = false, tv = false;
+    unsigned tk = 0;
+    for (int w = 0; w < 8; ++w) {
+      tk += wkept[w];
+      tv |= wviol[w] != 0;
+      if (whas[w]) {
+        if (wfirst[w] < run) tv = true;
+        if (!th) tf = wfirst[w];
+        th = true;
+        run = wlast[w];
+      }
+    }
+    TileMeta m;
+    m.first_ts = tf;
+    m.last_ts = run;
+    m.flags = (th ? 1u : 0u) | (tv ? 2u : 0u);
+    m.pad = 0;
+    p.emeta[tile] = m;
+    if ((unsigned)n > tk) atomicAdd(p.win + WF_DROPPED * p.W + g.charge, (unsigned long long)(n - tk));
+    if (tk) atomicAdd(p.win + WF_EVENTS * p.W + g.window, (unsigned long long)tk);
+  }
+  if (is_win) {
+    for (unsigned i = threadIdx.x; i < 2 * p.nk; i += blockDim.x)
+      if (khist[i]) atomicAdd(p.kdelta + ((size_t)g.window * p.nk) * 2 + i, khist[i]);
+    if (smem_bits)
+      for (unsigned i = threadIdx.x; i < p.ncw; i += blockDim.x)
+        if (abits[i]) atomicOr(p.active + (size_t)g.window * p.ncw + i, abits[i]);
+  }
+  __syncthreads();  // shared memory free for the next tile
+}
+
+__global__ void __launch_bounds__(kK3Threads) k_events(Params p) {
+  if (blockIdx.x >= p.rte[p.W + 2]) return;  // grid sized by an upper bound
+  extern __shared__ __align__(16) unsigned char smem[];
+  events_tile(p, blockIdx.x, smem);
+}
+
+// ============================================================================================
 // K1: sample partition.  A tile is <= 4096 samples of ONE region, handled by one CTA of 8 warps;
 // warp w owns the sub-tile [512w, 512w + 512).  Per sample: field validity, range + order check
 // against the previous field-valid sample, and a stable multisplit by bin (buffer_id >> 8).  Kept
@@ -656,6 +774,18 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     tile = nxt;
   }
   cp_async_wait_all();
+  if (p.fuse_events) {  // then task-event tiles, claimed dynamically (K3 fused into K1): the event
+    __shared__ unsigned s_et;  // work fills the partition's tail instead of competing with the fold
+    const unsigned n_e = p.rte[p.W + 2];
+    __syncthreads();  // every warp is done with the raw slots: they hold the event tile's counters
+    for (;;) {
+      if (threadIdx.x == 0) s_et = atomicAdd(p.unit_ctr + 2, 1u);
+      __syncthreads();
+      const unsigned et = s_et;
+      if (et >= n_e) break;
+      events_tile(p, et, smem);  // ends with a CTA barrier
+    }
+  }
 }
 
 __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
@@ -742,116 +872,6 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
   for (unsigned q = threadIdx.x; q < (total + 1) / 2; q += kK1Threads) d4[q] = s4[q];
 }
 
-// ============================================================================================
-// K3: task events.  One CTA per tile of <= 4096 events of one region: validate, order-check,
-// per-(window, kernel) START/END counts, per-(window, component) activity bits and per-call
-// per-component START/END deltas (progress bars, L131; "task counts stop changing", L227).
-// ============================================================================================
-__global__ void __launch_bounds__(kK3Threads) k_events(Params p) {
-  if (blockIdx.x >= p.rte[p.W + 2]) return;  // grid sized by an upper bound
-  extern __shared__ __align__(16) unsigned char smem[];
-  unsigned *khist = reinterpret_cast<unsigned *>(smem);  // [nk*2]
-  unsigned *abits = khist + 2 * p.nk;                     // [ncw] if smem_bits
-  __shared__ long long wfirst[8], wlast[8];
-  __shared__ unsigned whas[8], wviol[8], wkept[8];
-  const bool smem_bits = p.ncw <= 2048;
-
-  const unsigned tile = blockIdx.x;
-  const unsigned r = p.tile_reg_e[tile];
-  const long long start = p.Be[r] + (long long)(tile - p.rte[r]) * kTileE;
-  long long endp = p.Be[r + 1];
-  if (endp > start + kTileE) endp = start + kTileE;
-  const int n = (int)(endp - start);
-  const Region g = region_of(p, r);
-  const bool is_win = g.window >= 0;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const unsigned lt = lanemask_lt();
-  if (is_win) {
-    for (unsigned i = threadIdx.x; i < 2 * p.nk; i += blockDim.x) khist[i] = 0;
-    if (smem_bits)
-      for (unsigned i = threadIdx.x; i < p.ncw; i += blockDim.x) abits[i] = 0;
-  }
-  __syncthreads();
-  const int4 *src = reinterpret_cast<const int4 *>(p.e) + start;
-  long long carry = kTsMin, first = kTsMax;
-  bool has = false, viol = false;
-  unsigned kept = 0;
-#pragma unroll
-  for (int h = 0; h < 2; ++h) {
-    int4 v[8];
-#pragma unroll
-    for (int jj = 0; jj < 8; ++jj) {
-      int i = warp * 512 + (h * 8 + jj) * 32 + lane;
-      v[jj] = i < n ? ld_stream(src + i) : make_int4(0, 0, 0, 0);
-    }
-#pragma unroll
-    for (int jj = 0; jj < 8; ++jj) {
-      const int i = warp * 512 + (h * 8 + jj) * 32 + lane;
-      const bool valid = i < n && event_valid(p, v[jj]);
-      const long long ts = rec_ts(v[jj]);
-      const unsigned vm = __ballot_sync(kFull, valid);
-      const unsigned lower = vm & lt;
-      const long long prev = shfl_ll(ts, lower ? 31 - __clz(lower) : lane);
-      if (valid && ((lower ? prev : carry) > ts || ts < g.lo_ts || ts >= g.hi_ts)) viol = true;
-      if (vm) {
-        if (!has) first = shfl_ll(ts, __ffs(vm) - 1);
-        has = true;
-        carry = shfl_ll(ts, 31 - __clz(vm));
-      }
-      const bool keep = valid && is_win;
-      kept += keep;
-      const unsigned meta = (unsigned)v[jj].w;
-      const unsigned comp = meta & 0xFFFFFu, kern = (meta >> 20) & 0x7FFu, kind = meta >> 31;
-      const unsigned kk = keep ? kern * 2 + kind : 0xFFFFFFFFu;
-      const unsigned peers = __match_any_sync(kFull, kk);
-      if (keep && lane == __ffs(peers) - 1) atomicAdd(&khist[kk], (unsigned)__popc(peers));
-      if (keep) {
-        if (smem_bits) atomicOr(&abits[comp >> 5], 1u << (comp & 31));
-        else atomicOr(p.active + (size_t)g.window * p.ncw + (comp >> 5), 1u << (comp & 31));
-        atomicAdd(p.cdelta + 2 * comp + kind, 1ull);
-      }
-    }
-  }
-  kept = warp_sum(kept);
-  const bool wv = __any_sync(kFull, viol);
-  if (lane == 0) {
-    wfirst[warp] = first;
-    wlast[warp] = carry;
-    whas[warp] = has;
-    wviol[warp] = wv;
-    wkept[warp] = kept;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    long long run = kTsMin, tf = 0;
-    bool th = false, tv = false;
-    unsigned tk = 0;
-    for (int w = 0; w < 8; ++w) {
-      tk += wkept[w];
-      tv |= wviol[w] != 0;
-      if (whas[w]) {
-        if (wfirst[w] < run) tv = true;
-        if (!th) tf = wfirst[w];
-        th = true;
-        run = wlast[w];
-      }
-    }
-    TileMeta m;
-    m.first_ts = tf;
-    m.last_ts = run;
-    m.flags = (th ? 1u : 0u) | (tv ? 2u : 0u);
-    m.pad = 0;
-    p.emeta[tile] = m;
-    if ((unsigned)n > tk) atomicAdd(p.win + WF_DROPPED * p.W + g.charge, (unsigned long long)(n - tk));
-    if (tk) atomicAdd(p.win + WF_EVENTS * p.W + g.window, (unsigned long long)tk);
-  }
-  if (!is_win) return;
-  for (unsigned i = threadIdx.x; i < 2 * p.nk; i += blockDim.x)
-    if (khist[i]) atomicAdd(p.kdelta + ((size_t)g.window * p.nk) * 2 + i, khist[i]);
-  if (smem_bits)
-    for (unsigned i = threadIdx.x; i < p.ncw; i += blockDim.x)
-      if (abits[i]) atomicOr(p.active + (size_t)g.window * p.ncw + i, abits[i]);
-}
 
 // Persistence ranking key (rank mode MEAN): floor(I * 2^32 / c), exact.  Within a window the
 // mean occupancy I / (c * W) orders like I / c; distinct ratios I1/c1 != I2/c2 differ by at least
@@ -1898,6 +1918,8 @@ void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
   { k_fill_tiles<<<2 * blocks, 64, 0, st>>>(p); count_launch(); }
 }
 
+bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s) { return n_tiles_s && nbins <= kLmMaxBins; }
+
 void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   if (!p.n_tiles_s) return;
   const size_t sm = partition_smem_bytes(p.nbins, p.nb);
@@ -1906,7 +1928,8 @@ void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm, kK1Threads, sm);
     if (per_sm < 1) per_sm = 1;
     unsigned grid = (unsigned)(n_sms * per_sm);
-    if (grid > p.n_tiles_s) grid = p.n_tiles_s;
+    const unsigned work = p.n_tiles_s + (p.fuse_events ? p.n_tiles_e : 0u);
+    if (grid > work) grid = work;
     { k_partition_lm<<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
   } else {
     { k_partition_mx<<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
