@@ -208,8 +208,11 @@ C3_SMALL = C3.scaled("C3-small", n_samples=9_000_000, n_events=1_000_000, n_wind
 C4 = Workload("C4-skewed", 1_800_000_000, 200_000_000, 1 << 20, 64, 2000, 1024, 96, seed=4, zipf_s=0.99,
               description="skewed trace: 1M buffers, Zipf-distributed buffer_id hot spots, 2B records, top-k=1024")
 C4_SMALL = C4.scaled("C4-small", n_samples=18_000_000, n_events=2_000_000, n_windows=20)
-# C5: recorded for the next round (1M windows needs the sparse-window path)
-C5 = Workload("C5-long", 7_200_000_000, 800_000_000, 327680, 128, 1_000_000, 64, 256, seed=5,
+# C5: streamed in batches of windows at full size (tools/c5_full.py).  H = 2048: a component sees
+# ~0.01 task events per window (800 events over 81920 components), so quiet gaps of a few hundred
+# windows are normal; P(gap >= H) = exp(-H/102) over ~8e8 gaps needs H ~ 2000 to flag nothing.
+# Measured: H = 256 flags ~850 components per window; H = 2048 one component in 2282 of 1M windows.
+C5 = Workload("C5-long", 7_200_000_000, 800_000_000, 327680, 128, 1_000_000, 64, 2048, seed=5,
               description="long run: 16 simulated GPUs, ~320k buffers, 8B records in 1M windows")
 CONFIGS = {w.name: w for w in (C1, C1_INVALID, C2, C3, C3_CLEAN, C3_SMALL, C4, C4_SMALL, C5)}
 

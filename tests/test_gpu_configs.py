@@ -142,7 +142,8 @@ def test_c4_full_size_parity():
 def test_c5_first_windows_parity():
     """BASELINE configs[4] (16 simulated GPUs, 327680 buffers, 1M windows of ~8k records): its
     first 1000 windows (8M records) in one call, every window checked.  The full 1M-window run
-    needs the sparse-window path, so only this slice is a parity case."""
+    (128 GB, streamed in 1000 calls) is `tools/c5_full.py` against a range-parallel oracle
+    (~10 min on 15 cores; profiles/r01_c5_full.json)."""
     wl = gen.C5
     n_win = 1000
     ns = wl.index_at("samples", wl.t_begin(n_win))
