@@ -455,6 +455,8 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   // concurrent kernel competes with the issue-bound fold.  Otherwise: a side stream, overlapped
   // with the partition and the fold, joined before the kernels that read the event outputs.
   p.fuse_events = partition_fuses_events(p.nbins, nts) ? 1 : 0;
+  static const int xp = getenv("RTM_XP") ? atoi(getenv("RTM_XP")) : 0;
+  p.xp = xp;
   if (!p.fuse_events) {
     CK(cudaEventRecord(c->ev_fork, c->st));
     CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));

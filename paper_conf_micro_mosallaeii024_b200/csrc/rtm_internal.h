@@ -114,6 +114,7 @@ struct Params {
   uint32_t *hung;            // [W * ncw]
   uint32_t *unit_ctr;        // [0] fold units dequeued, [1] partition tiles, [2] fused event tiles claimed
   int32_t fuse_events;       // the persistent partition also runs the event tiles (K3 in K1)
+  int32_t xp;                // experiment switch (env RTM_XP, bit mask; A/B runs only, 0 = product path)
   uint32_t *status;          // bit0 sample order, bit1 event order
   const uint16_t *carry_in;  // [nb]
   uint16_t *carry_out;       // [nb]
