@@ -911,7 +911,6 @@ struct FoldSmem {
   uint4 st[kBin];
   unsigned ts0[kBin];              // offset of the first kept sample in the window, low 32 bits
   unsigned hi[kBin];               // n_hi | ts0_hi << 16
-  unsigned seg_end[32];            // flattened segment table of the current tile group
   unsigned seg_base[32];           // staging index of each segment, minus its flattened start
   unsigned char owner[kBin];       // duplicate detection: last lane that wrote each buffer slot
 };
@@ -1032,16 +1031,23 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
         if (lane >= o) pre += y;
       }
       const unsigned total = __shfl_sync(kFull, pre, 31);
-      // per-warp segment table: end (inclusive prefix) and the staging index of each segment
-      // minus its flattened start
-      S.seg_end[lane] = pre;
-      S.seg_base[lane] = (tg + lane) * (unsigned)kTileS + seg_lo - (pre - seg_len);
+      // per-warp table of the NON-EMPTY segments (compacted, so their ends are strictly
+      // increasing): staging index of each segment minus its flattened start.  The segment of
+      // flattened position g is the number of segment ends <= g: per 32-position chunk, one
+      // OR-reduction marks the ends inside the chunk and each lane counts the marks at or below it.
+      const unsigned nonempty = __ballot_sync(kFull, seg_len != 0);
+      if (seg_len) S.seg_base[__popc(nonempty & lt)] = (tg + lane) * (unsigned)kTileS + seg_lo - (pre - seg_len);
+      const unsigned my_end = seg_len ? pre : 0xFFFFFFFFu;
+      const unsigned le = (2u << lane) - 1u;  // lanes <= this one
       __syncwarp();
-      unsigned sgi = 0;  // this lane's current segment (cursor), advanced without warp collectives
+      unsigned seg_before = 0;  // segments ending at or before the current chunk's first position
       auto fetch = [&](unsigned c) -> unsigned long long {
+        const unsigned x = my_end - c;
+        const unsigned ends = __reduce_or_sync(kFull, x < 32u ? 1u << x : 0u);
+        const unsigned sgi = seg_before + __popc(ends & le);
+        seg_before += __popc(ends);
         const unsigned g = c + lane;
         if (g >= total) return 0ull;
-        while (g >= S.seg_end[sgi]) ++sgi;
         return __ldcg(p.stage + (S.seg_base[sgi] + g));
       };
       // 4-deep software pipeline: staging reads are DRAM/L2 round trips
