@@ -618,6 +618,12 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
   } while (0)
 #endif
 
+// STAGED: after the tile's barrier the warps permute their entries into the first half of the raw
+// staging (shared memory), a second barrier, then warps 0-3 copy the tile out with coalesced
+// 16-byte stores and only then prefetch their next raw records (named barrier among themselves);
+// warps 4-7 prefetch early as in the direct variant.  Direct: every lane stores its entries
+// straight to global memory (8-byte stores scattered over the tile's bins).
+template <bool STAGED>
 __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ K1WarpSum wsum[2][kK1Warps];
@@ -755,13 +761,38 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     // the next tile's records stream into the slot while this tile is published and written out
     cp_async_wait_all();
     __syncwarp();
-    if (nxt != ~0u) prefetch_raw(dsm[par ^ 1]);
-    cp_async_commit();
+    const bool early = !STAGED || warp >= kK1Warps / 2;  // slots outside the staged half
+    if (early) {
+      if (nxt != ~0u) prefetch_raw(dsm[par ^ 1]);
+      cp_async_commit();
+    }
     k1_publish(wsum[par], first, last, has, viol, kept);
     __syncthreads();  // B1 (the only CTA barrier per tile): summaries + bin totals of this tile
     PTM(4);
     if (warp == 0) k1_tile_summary(p, t, wsum[par]);
-    if (is_win) {
+    if (STAGED) {
+      unsigned total = 0;
+      if (is_win) {
+        total = k1_bin_bases(p, tile, wt, myb);
+        unsigned long long *sst = reinterpret_cast<unsigned long long *>(smem);
+#pragma unroll
+        for (int k = 0; k < kPerLane; ++k) {
+          const unsigned key = kp[k] >> 16;
+          if (key != kNoKey) sst[myb[key] + (kp[k] & 0xFFFFu)] = e[k];
+        }
+      }
+      __syncthreads();  // B2: the tile's entries are in bin order in shared memory
+      if (!early) {
+        if (is_win) {
+          const uint4 *s4 = reinterpret_cast<const uint4 *>(smem);
+          uint4 *d4 = reinterpret_cast<uint4 *>(p.stage + (size_t)tile * kTileS);
+          for (unsigned q = threadIdx.x; q < (total + 1) / 2; q += kK1Threads / 2) d4[q] = s4[q];
+        }
+        asm volatile("bar.sync 1, %0;" ::"n"(kK1Threads / 2) : "memory");  // staged half read out
+        if (nxt != ~0u) prefetch_raw(dsm[par ^ 1]);
+        cp_async_commit();
+      }
+    } else if (is_win) {
       k1_bin_bases(p, tile, wt, myb);
       unsigned long long *dst = p.stage + (size_t)tile * kTileS;
 #pragma unroll
@@ -1931,12 +1962,13 @@ void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   const size_t sm = partition_smem_bytes(p.nbins, p.nb);
   if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM (capacity table loaded once)
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm, kK1Threads, sm);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm<false>, kK1Threads, sm);
     if (per_sm < 1) per_sm = 1;
     unsigned grid = (unsigned)(n_sms * per_sm);
     const unsigned work = p.n_tiles_s + (p.fuse_events ? p.n_tiles_e : 0u);
     if (grid > work) grid = work;
-    { k_partition_lm<<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
+    if (p.xp & 4) { k_partition_lm<false><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }  // A/B: direct
+    else { k_partition_lm<true><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
   } else {
     { k_partition_mx<<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
   }
@@ -2023,7 +2055,9 @@ void configure_kernels_once() {
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 128 || done[dev]) return;
   done[dev] = true;
-  cudaFuncSetAttribute(k_partition_lm, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  cudaFuncSetAttribute(k_partition_lm<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       (int)k1_smem_lm(kLmMaxBins, kLmMaxBins * kBin));
+  cudaFuncSetAttribute(k_partition_lm<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)k1_smem_lm(kLmMaxBins, kLmMaxBins * kBin));
   cudaFuncSetAttribute(k_partition_mx, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
   cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
