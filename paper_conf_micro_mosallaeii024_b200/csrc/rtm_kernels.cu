@@ -1100,7 +1100,9 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
       const unsigned l = lane + 32 * i, b = b_base + l;
       if (b < p.nb) lw[b] = (uint16_t)(S.st[l].z & 0xFFFFu);  // 0xFFFF == kSent: untouched
     }
-    __threadfence();
+    // No per-lane fence: bar.warp.sync orders every lane's lastlvl stores before lane 0's
+    // st.release.gpu, and release is cumulative (PTX memory model), so a reader that acquires the
+    // flag sees them (measured: fold -2 %, the fence was 3.7 % of its stall samples).
     __syncwarp();
     if (lane == 0) st_release_u32(p.flags + (size_t)w * p.nbins + bin, p.epoch);
     // ---- phase 2: carry-in by look-back, finalize
