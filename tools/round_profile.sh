@@ -11,5 +11,5 @@ timeout 900 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/b
 timeout 600 $NCU --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv \
   python tools/prof_step.py --warmup 1 --steps 1 > gpurun_out/ncu_launches.log 2>&1; echo "launches rc=$?"
 timeout 1500 $NCU --set full --clock-control none --import-source on -k regex:"k_partition|k_fold|k_topk|k_events" \
-  -s 4 -c 4 -f -o gpurun_out/prof_full python tools/prof_step.py --warmup 1 --steps 1 > gpurun_out/ncu_full.log 2>&1; echo "full rc=$?"
+  -s 3 -c 3 -f -o gpurun_out/prof_full python tools/prof_step.py --warmup 1 --steps 1 > gpurun_out/ncu_full.log 2>&1; echo "full rc=$?"
 ls -la gpurun_out/
