@@ -769,7 +769,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     k1_publish(wsum[par], first, last, has, viol, kept);
     __syncthreads();  // B1 (the only CTA barrier per tile): summaries + bin totals of this tile
     PTM(4);
-    if (warp == 0) k1_tile_summary(p, t, wsum[par]);
+    if (!STAGED && warp == 0) k1_tile_summary(p, t, wsum[par]);
     if (STAGED) {
       unsigned total = 0;
       if (is_win) {
@@ -782,6 +782,9 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
         }
       }
       __syncthreads();  // B2: the tile's entries are in bin order in shared memory
+      // the tile summary (serial, latency-bound) by the last warp, which is otherwise idle until
+      // the next tile: wsum[par] is rewritten only after the next tile's barrier
+      if (warp == kK1Warps - 1) k1_tile_summary(p, t, wsum[par]);
       if (!early) {
         if (is_win) {
           const uint4 *s4 = reinterpret_cast<const uint4 *>(smem);
