@@ -1304,6 +1304,54 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     const unsigned b = id_of(i);
     return fullness_key(lv[b], __ldg(p.cap + b), p.rank_mode, p.rcp);
   };
+  const unsigned keff = p.k < ne ? p.k : ne;
+  const bool sliced = ALL && p.tk_slices > 1;
+  unsigned long long *scr = sliced ? p.tk_scratch + ((size_t)w * p.tk_slices + blockIdx.y) * p.k : nullptr;
+  if (keff == 0) {
+    if (threadIdx.x == 0 && !sliced) p.topk_n[w] = 0;
+    if (sliced)
+      for (unsigned i = threadIdx.x; i < p.k; i += blockDim.x) scr[i] = 0ull;
+    return;
+  }
+  // Full-prefix shortcut (Percent mode): a 100 %-full buffer has the largest possible key
+  // (0xFFFFFFFF), so if the k lowest ids holding it are found while scanning in id order, they
+  // ARE the top-k (ties by id) and the rest of the window is never read.  In the bottleneck
+  // picture (L197-L199) that is a short prefix of the ids; otherwise the scan reaches the end
+  // and the general path below runs.
+  __shared__ unsigned s_full;
+  bool fast = false;
+  if (p.rank_mode == RTM_RANK_PERCENT) {
+    const bool vec = ALL && (p.nb & 7u) == 0;  // 8 consecutive buffers per thread (16-B loads)
+    const unsigned per = vec ? 8u : 1u, step = blockDim.x * per;
+    unsigned found = 0;
+    for (unsigned base = 0; base < ne && found < keff; base += step) {
+      const unsigned i0 = base + threadIdx.x * per;
+      unsigned fm = 0;  // bit q: buffer i0 + q is 100 % full
+      if (vec) {
+        if (i0 < ne) {
+          const uint4 L = reinterpret_cast<const uint4 *>(lv + slo)[i0 / 8];
+          const uint4 C = __ldg(reinterpret_cast<const uint4 *>(p.cap + slo) + i0 / 8);
+          const unsigned lw[4] = {L.x, L.y, L.z, L.w}, cw[4] = {C.x, C.y, C.z, C.w};
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            fm |= ((lw[q] & 0xFFFFu) >= (cw[q] & 0xFFFFu) ? 1u : 0u) << (2 * q);
+            fm |= ((lw[q] >> 16) >= (cw[q] >> 16) ? 1u : 0u) << (2 * q + 1);
+          }
+        }
+      } else if (i0 < ne) {
+        const unsigned b = id_of(i0);
+        fm = lv[b] >= __ldg(p.cap + b) ? 1u : 0u;
+      }
+      unsigned tot;
+      unsigned pos = found + block_excl_scan(__popc(fm), scan_scratch, &tot);
+      for (unsigned x = fm; x && pos < keff; x &= x - 1, ++pos)
+        sel[pos] = (0xFFFFFFFFull << 32) | (0xFFFFFFFFu - id_of(i0 + __ffs(x) - 1));
+      found += tot;
+    }
+    fast = found >= keff;
+  }
+  bool top_tie = fast;  // winners share one key and were written in id order
+  if (!fast) {
   // keys (shared memory when they fit) and, in the same pass, the largest key and how many
   // buffers hold it (per thread, then per warp, then per CTA)
   __shared__ unsigned s_max, s_cnt_max;
@@ -1340,7 +1388,6 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
       track(k);
     }
   }
-  const unsigned keff = p.k < ne ? p.k : ne;
   {
     const unsigned wm = __reduce_max_sync(kFull, tm);
     const unsigned wc = __reduce_add_sync(kFull, tm == wm ? tc : 0u);
@@ -1350,17 +1397,9 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     if ((threadIdx.x & 31) == 0 && wm == s_max && wc) atomicAdd(&s_cnt_max, wc);
     __syncthreads();
   }
-  const bool sliced = ALL && p.tk_slices > 1;
-  unsigned long long *scr = sliced ? p.tk_scratch + ((size_t)w * p.tk_slices + blockIdx.y) * p.k : nullptr;
-  if (keff == 0) {
-    if (threadIdx.x == 0 && !sliced) p.topk_n[w] = 0;
-    if (sliced)
-      for (unsigned i = threadIdx.x; i < p.k; i += blockDim.x) scr[i] = 0ull;
-    return;
-  }
-  // Shortcut: when the largest key is held by >= k buffers (e.g. >= k buffers are 100 % full, the
-  // bottleneck picture of L197-L199), the answer is the k lowest ids holding it: tau = max key.
-  const bool top_tie = s_cnt_max >= keff;
+  // Shortcut: when the largest key is held by >= k buffers, the answer is the k lowest ids
+  // holding it: tau = max key.
+  top_tie = s_cnt_max >= keff;
   // MSB radix select.  After the first digit only candidates (top byte >= the selected digit,
   // at most k + the selected bucket) can matter: they are compacted in id order when they fit,
   // so the remaining passes and the selection scan ~1k keys instead of every buffer.
@@ -1447,6 +1486,7 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
       ++rank;
     }
   }
+  }  // general path
   __syncthreads();
   if (sliced) {  // this slice's candidates (unsorted); k_topk_merge ranks the union
     for (unsigned i = threadIdx.x; i < p.k; i += blockDim.x) scr[i] = i < keff ? sel[i] : 0ull;
