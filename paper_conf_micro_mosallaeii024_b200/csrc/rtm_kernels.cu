@@ -1711,6 +1711,7 @@ __device__ __forceinline__ unsigned hang_cond(const Params &p, unsigned j, unsig
 __global__ void k_hang(Params p) {
   const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
   const size_t nflag = (size_t)p.W * p.ncw;
+  const size_t nflag_w = (nflag + 31) & ~(size_t)31;  // warp-aligned start of the run part
   if (tid < nflag) {
     const unsigned w = (unsigned)(tid / p.ncw), q = (unsigned)(tid % p.ncw);
     const long long first = (long long)w - (long long)p.H + 1;
@@ -1728,16 +1729,37 @@ __global__ void k_hang(Params p) {
     if (q == p.ncw - 1 && (p.nc & 31)) acc &= (1u << (p.nc & 31)) - 1u;
     p.hung[(size_t)w * p.ncw + q] = acc;
     if (acc) atomicAdd(p.win + WF_HUNG * p.W + w, (unsigned long long)__popc(acc));
-  } else if (tid < nflag + p.nc) {
-    const unsigned c = (unsigned)(tid - nflag), q = c >> 5, bit = c & 31;
+  } else if (tid >= nflag_w && tid < nflag_w + (size_t)p.ncw * 32) {
+    // carried run length for the next call: one warp per 32-component word, lane = component.
+    // Windows are taken 32 at a time from the last one backwards (lane l: window W-1-32g-l); one
+    // ballot per component marks the windows where its condition fails, the first such lane ends
+    // its run.  A run through every window of the call continues the carried run.
+    const unsigned q = (unsigned)((tid - nflag_w) >> 5), lane = threadIdx.x & 31, c = q * 32 + lane;
     unsigned r = 0;
-    long long j = (long long)p.W - 1;
-    for (; j >= 0; --j) {
-      if ((hang_cond(p, (unsigned)j, q) >> bit) & 1u) ++r;
-      else break;
+    bool done = false;
+    for (unsigned g = 0; __any_sync(kFull, !done); ++g) {
+      const long long j = (long long)p.W - 1 - 32ll * g - lane;
+      const unsigned word = j >= 0 ? hang_cond(p, (unsigned)j, q) : 0xFFFFFFFFu;
+      unsigned zeros = 0;  // this lane's component: windows of the group where cond fails
+#pragma unroll 4
+      for (unsigned b = 0; b < 32; ++b) {
+        const unsigned m = __ballot_sync(kFull, j >= 0 && !((word >> b) & 1u));
+        if (lane == b) zeros = m;
+      }
+      if (!done) {
+        const long long left = (long long)p.W - 32ll * g;  // windows of the call not yet scanned
+        if (zeros) {
+          r += __ffs(zeros) - 1;
+          done = true;
+        } else if (left <= 32) {
+          r += (unsigned)left + (c < p.nc ? p.run[c] : 0u);
+          done = true;
+        } else {
+          r += 32;
+        }
+      }
     }
-    if (j < 0) r += p.run[c];
-    p.run_out[c] = r;
+    if (c < p.nc) p.run_out[c] = r;
   }
 }
 
@@ -2083,7 +2105,7 @@ void launch_persist(const Params &p, cudaStream_t st) {
 
 void launch_hang(const Params &p, cudaStream_t st) {
   const unsigned threads = 256;
-  const size_t n = (size_t)p.W * p.ncw + p.nc;
+  const size_t n = (((size_t)p.W * p.ncw + 31) & ~(size_t)31) + (size_t)p.ncw * 32;
   { k_hang<<<(unsigned)((n + threads - 1) / threads), threads, 0, st>>>(p); count_launch(); }
 }
 

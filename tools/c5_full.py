@@ -57,6 +57,8 @@ def gpu_pass(wl, n_windows, batch, sampled, checkpoints):
 
     owner, cap, tot = gen.registry(wl)
     mon = Monitor(owner, cap, tot, n_components=wl.n_components, t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k)
+    if os.environ.get("C5_PROFILE"):
+        mon.profile(True)
     max_s = max(ranges(wl, a, b)[1] - ranges(wl, a, b)[0] for a, b in [(0, batch), (n_windows - batch, n_windows)])
     max_e = max(ranges(wl, a, b)[3] - ranges(wl, a, b)[2] for a, b in [(0, batch), (n_windows - batch, n_windows)])
     ds = torch.empty((max_s + 4096) * 16, dtype=torch.uint8, device="cuda")
@@ -97,6 +99,8 @@ def gpu_pass(wl, n_windows, batch, sampled, checkpoints):
                 hung[w] = mon.hang_check(w - w0)
     stats = mon.buffer_stats()
     summ = np.concatenate(summ)
+    if os.environ.get("C5_PROFILE"):
+        print(json.dumps({k: round(v["total_ms"], 2) for k, v in mon.profile_read().items() if v["launches"]}))
     out = {
         "records": n_rec, "windows": n_windows, "batch": batch, "calls": len(prog_h),
         "reduce_wall_s": t_reduce, "reduce_device_s": dev_ms / 1e3, "gen_s": t_gen,
