@@ -137,7 +137,7 @@ __device__ __forceinline__ void split_one(const Params &p, unsigned q, long long
   const unsigned long long N = SAMPLES ? p.ns : p.ne;
   const int4 *recs = SAMPLES ? reinterpret_cast<const int4 *>(p.s) : reinterpret_cast<const int4 *>(p.e);
   unsigned long long lo = 0, hi = N;
-  while (hi - lo > 1024) {
+  while (hi - lo > 64) {  // then <= 2 dependent rounds of the final scan
     unsigned long long span = hi - lo;
     unsigned long long qq = lo + span * (unsigned long long)(lane + 1) / 33ull;
     int state = 0;  // 0 unknown, 1 valid with ts < T, 2 valid with ts >= T
@@ -1534,7 +1534,12 @@ __global__ void __launch_bounds__(1024) k_topk_merge(Params p) {
   while (P < n) P <<= 1;
   const unsigned long long *src = p.tk_scratch + (size_t)w * n;
   for (unsigned i = threadIdx.x; i < P; i += blockDim.x) v[i] = i < n ? src[i] : 0ull;
-  __syncthreads();
+  // slice 0 holds the lowest ids: if all its k candidates are 100 % full (the largest key) they
+  // are the answer, already in id order (full-prefix shortcut of k_topk) - no sort
+  bool full0 = true;
+  for (unsigned i = threadIdx.x; i < (p.k < p.nb ? p.k : p.nb); i += blockDim.x)
+    full0 &= (src[i] >> 32) == 0xFFFFFFFFull;
+  if (__syncthreads_and(full0)) P = 1;
   for (unsigned size = 2; size <= P; size <<= 1) {
     for (unsigned stride = size >> 1; stride > 0; stride >>= 1) {
       for (unsigned i = threadIdx.x; i < P; i += blockDim.x) {
