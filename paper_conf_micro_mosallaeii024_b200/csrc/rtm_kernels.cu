@@ -822,6 +822,42 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   }
 }
 
+// After B1, the whole CTA: bins in rows of blockDim.x (thread = bin, conflict-free); each bin's
+// CTA base from one block scan per row, then every warp's base for the bin (earlier warps'
+// counts added) written to wb[warp][bin] and the CTA base to the tile's soff row.  O(n_bins) per
+// tile in total, instead of every warp scanning every bin (O(8 n_bins)): the cost that dominates
+// the many-bin partition.  Ends with a CTA barrier; returns the tile's kept total.
+__device__ __forceinline__ unsigned k1_bin_bases_cta(const Params &p, unsigned tile, const unsigned short *wt,
+                                                     unsigned short *wb, unsigned *scratch) {
+  const unsigned nbins = p.nbins;
+  uint16_t *offs = p.soff + (size_t)tile * (nbins + 1);
+  unsigned carry = 0;
+  for (unsigned row = 0; row < nbins; row += blockDim.x) {
+    const unsigned b = row + threadIdx.x;
+    unsigned cnt[kK1Warps], T = 0;
+#pragma unroll
+    for (int w2 = 0; w2 < kK1Warps; ++w2) {
+      cnt[w2] = b < nbins ? wt[(size_t)w2 * nbins + b] : 0u;
+      T += cnt[w2];
+    }
+    unsigned tot;
+    const unsigned base = carry + block_excl_scan(T, scratch, &tot);
+    if (b < nbins) {
+      offs[b] = (uint16_t)base;
+      unsigned run = base;
+#pragma unroll
+      for (int w2 = 0; w2 < kK1Warps; ++w2) {
+        wb[(size_t)w2 * nbins + b] = (unsigned short)run;
+        run += cnt[w2];
+      }
+    }
+    carry += tot;
+  }
+  if (threadIdx.x == 0) offs[nbins] = (uint16_t)carry;
+  __syncthreads();
+  return carry;
+}
+
 __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ K1WarpSum wsum[kK1Warps];
@@ -894,7 +930,9 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
   __syncthreads();  // B1
   if (warp == 0) k1_tile_summary(p, t, wsum);
   if (!is_win) return;
-  const unsigned total = k1_bin_bases(p, tile, wt, myb);
+  __shared__ unsigned bb_scratch[32];
+  const unsigned total = (p.xp & 32) ? k1_bin_bases(p, tile, wt, myb)  // A/B: per-warp bases
+                                     : k1_bin_bases_cta(p, tile, wt, wb, bb_scratch);
 #pragma unroll
   for (int k = 0; k < kPerLane; ++k) {
     const unsigned key = kp[k] >> 16;
@@ -1318,7 +1356,6 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
   // ARE the top-k (ties by id) and the rest of the window is never read.  In the bottleneck
   // picture (L197-L199) that is a short prefix of the ids; otherwise the scan reaches the end
   // and the general path below runs.
-  __shared__ unsigned s_full;
   bool fast = false;
   if (p.rank_mode == RTM_RANK_PERCENT) {
     const bool vec = ALL && (p.nb & 7u) == 0;  // 8 consecutive buffers per thread (16-B loads)
