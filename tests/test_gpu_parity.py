@@ -306,6 +306,53 @@ def test_topk_paths_top_tie_and_radix(n_top, at_cap):
     assert np.array_equal(got["topk"][0], ref["topk"][0])
 
 
+@pytest.mark.parametrize("placement", ["slice0", "later_slices", "split_k_minus_1", "kth_at_slice_end",
+                                       "none", "scattered"])
+@pytest.mark.parametrize("n_windows", [1, 200])
+def test_topk_full_prefix_shortcut(placement, n_windows):
+    """Percent-mode top-k scans ids in order for 100 %-full buffers and stops at k (DESIGN.md §4
+    K5); with few windows the buffers are split into id slices and the merge takes slice 0's list
+    when all its k candidates are full.  Full buffers are placed so that the scan succeeds in
+    slice 0, only in later slices, misses by one, ends exactly at a slice boundary, never
+    succeeds, or is scattered; every window must equal the oracle's full sort."""
+    rng = np.random.default_rng(hash(placement) % 1000 + n_windows)
+    nb, k = 20480, 64
+    caps = rng.choice(np.array([4, 8, 16, 128, 1024], np.uint16), nb)
+    if placement == "slice0":
+        full = rng.choice(1024, 100, replace=False)
+    elif placement == "later_slices":
+        full = 8192 + rng.choice(8192, 100, replace=False)
+    elif placement == "split_k_minus_1":
+        full = np.concatenate([rng.choice(1024, k - 1, replace=False), [nb - 1]])
+    elif placement == "kth_at_slice_end":
+        full = np.concatenate([rng.choice(2047, k - 1, replace=False), [2047]])
+    elif placement == "none":
+        full = np.array([], np.int64)
+    else:
+        full = rng.choice(nb, 300, replace=False)
+    lv = np.minimum(rng.integers(0, 1024, nb), caps - 1).astype(np.uint16)
+    lv[full] = caps[full]
+    rows = []
+    for w in range(n_windows):  # every window re-samples a random subset; fulls stay full
+        ids = rng.choice(nb, nb // 4 if w else nb, replace=False)
+        lvw = lv.copy()
+        if w:
+            lvw[ids] = np.where(np.isin(ids, full), caps[ids], np.minimum(rng.integers(0, 1024, len(ids)), caps[ids] - 1))
+            lv = lvw
+        rows += [(w * 100000 + i, int(b), int(lvw[b]), int(caps[b])) for i, b in enumerate(ids)]
+    s = sample_array(rows)
+    owner = (np.arange(nb) // 4).astype(np.uint32)
+    kw = dict(t0=0, hang_windows=4, k=k, rank_mode=0)
+    orc, mon = _pair(owner, caps, np.ones(2, np.int64), int(owner[-1]) + 1, **kw)
+    t_end = [(w + 1) * 100000 for w in range(n_windows)]
+    ref = orc.reduce(s, event_array([]), t_end)
+    mon.ingest(_dev(s), None)
+    got = mon.window_reduce(t_end)
+    assert np.array_equal(got["topk_n"], ref["topk_n"])
+    for w in range(n_windows):
+        assert np.array_equal(got["topk"][w], ref["topk"][w]), w
+
+
 @pytest.mark.parametrize("disorder", [False, True])
 @pytest.mark.parametrize("stream", ["samples", "events"])
 def test_order_check_across_tiles_with_invalid_gap(disorder, stream):
