@@ -472,8 +472,9 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   LAUNCH(KT_FOLD, (uint64_t)ns * 8, launch_fold(p, c->n_sms, c->st));
   if (!p.fuse_events) CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
   LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
+  p.persist_inline = c->world == 1 && p.persist;  // world > 1: counted from the merged lists
   LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
-  if (c->world == 1) launch_persist(p, c->st);  // world > 1: counted from the merged lists
+  p.persist_inline = 0;
   LAUNCH(KT_HANG, 0, launch_hang(p, c->st));
   LAUNCH(KT_PROGRESS, 0, launch_progress(p, c->st));
   CK(cudaGetLastError());

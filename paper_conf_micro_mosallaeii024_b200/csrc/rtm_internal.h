@@ -134,6 +134,7 @@ struct Params {
   unsigned long long *mkey;  // [W * nb] rank mode MEAN: floor(integral * 2^32 / cap) (exact order key)
   const unsigned long long *rcp64;  // [65536] floor(2^64 / c) (c >= 2)
   uint32_t *persist;         // [id space] windows in the top-k list
+  int32_t persist_inline;    // world == 1: the top-k kernels count their own winners (no k_persist)
   uint32_t n_watch;          // value monitor: watched local buffer ids (0xFFFFFFFF: not on this rank)
   uint32_t watch[RTM_WATCH_MAX];
   rtm_buffer_stat *wstat;    // [W * RTM_WATCH_MAX] per-window statistics of the watched buffers

@@ -1554,6 +1554,7 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
       unsigned b = 0xFFFFFFFFu - (unsigned)(sel[i] & 0xFFFFFFFFu);
       out = (unsigned long long)(p.gid ? __ldg(p.gid + b) : b) | ((unsigned long long)lv[b] << 32) |
             ((unsigned long long)__ldg(p.cap + b) << 48);
+      if (p.persist_inline) atomicAdd(p.persist + (unsigned)(out & 0xFFFFFFFFull), 1u);  // k_persist fused
     }
     p.topk[(size_t)w * p.k + i] = out;
   }
@@ -1598,6 +1599,7 @@ __global__ void __launch_bounds__(1024) k_topk_merge(Params p) {
       const unsigned b = 0xFFFFFFFFu - (unsigned)(v[i] & 0xFFFFFFFFu);
       out = (unsigned long long)(p.gid ? __ldg(p.gid + b) : b) | ((unsigned long long)lv[b] << 32) |
             ((unsigned long long)__ldg(p.cap + b) << 48);
+      if (p.persist_inline) atomicAdd(p.persist + (unsigned)(out & 0xFFFFFFFFull), 1u);  // k_persist fused
     }
     p.topk[(size_t)w * p.k + i] = out;
   }
@@ -1724,6 +1726,7 @@ __global__ void __launch_bounds__(kT64Threads) k_topk64(Params p) {
       const unsigned b = seli[i];
       out = (unsigned long long)(p.gid ? __ldg(p.gid + b) : b) | ((unsigned long long)lv[b] << 32) |
             ((unsigned long long)__ldg(p.cap + b) << 48);
+      if (p.persist_inline) atomicAdd(p.persist + (unsigned)(out & 0xFFFFFFFFull), 1u);  // k_persist fused
     }
     p.topk[(size_t)w * p.k + i] = out;
   }
