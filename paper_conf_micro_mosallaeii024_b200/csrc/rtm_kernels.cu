@@ -1753,11 +1753,77 @@ __device__ __forceinline__ unsigned hang_cond(const Params &p, unsigned j, unsig
   return __ldg(p.anyfull + i) & ~__ldg(p.active + i);
 }
 
+// Long H (> kHangShortH): the per-(window, word) AND loop costs O(run length) per thread and
+// runs are long when components stay quiet (C5: H = 2048), so one thread per word computes the
+// sliding-window AND over H windows in two passes (van Herk / Gil-Werman): prefix ANDs inside
+// blocks of H windows forward, suffix ANDs backward; the range [w-H+1, w] is suffix(w-H+1) &
+// prefix(w).  Windows w < H-1 reach before the call: prefix(w) (= AND over 0..w) and the carried
+// run must cover the rest.
+constexpr unsigned kHangShortH = 64;
+__host__ __device__ constexpr size_t hang_flag_threads(uint32_t W, uint32_t ncw, uint32_t H) {
+  return H > kHangShortH ? (size_t)ncw : (size_t)W * ncw;
+}
+
 __global__ void k_hang(Params p) {
   const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const size_t nflag = (size_t)p.W * p.ncw;
+  const bool lng = p.H > kHangShortH;
+  const size_t nflag = hang_flag_threads(p.W, p.ncw, p.H);
   const size_t nflag_w = (nflag + 31) & ~(size_t)31;  // warp-aligned start of the run part
-  if (tid < nflag) {
+  if (lng && tid < nflag) {
+    const unsigned q = (unsigned)tid, H = p.H, W = p.W;
+    const unsigned vmask = (q == p.ncw - 1 && (p.nc & 31)) ? (1u << (p.nc & 31)) - 1u : 0xFFFFFFFFu;
+    // window from which each component's carried run completes H (windows w < H-1 only)
+    unsigned first_ok[32];
+#pragma unroll
+    for (int b = 0; b < 32; ++b) {
+      const unsigned cc = q * 32 + b;
+      const unsigned r = cc < p.nc ? p.run[cc] : 0u;
+      first_ok[b] = r >= H - 1 ? 0u : H - 1 - r;
+    }
+    unsigned acc = 0;
+    constexpr unsigned kB = 8;  // cond words loaded per batch (independent loads in flight)
+    for (unsigned w0 = 0; w0 < W; w0 += kB) {  // forward: prefix AND inside blocks of H windows
+      unsigned cb[kB];
+#pragma unroll
+      for (unsigned i = 0; i < kB; ++i) cb[i] = w0 + i < W ? hang_cond(p, w0 + i, q) : 0u;
+#pragma unroll
+      for (unsigned i = 0; i < kB; ++i) {
+        const unsigned w = w0 + i;
+        if (w >= W) break;
+        acc = (w % H == 0) ? cb[i] : (acc & cb[i]);
+        unsigned out = acc;
+        if (w + 1 < H) {  // final here: needs the carried run (run_in >= H - (w+1))
+          unsigned elig = 0;
+          for (unsigned x = acc; x; x &= x - 1) {
+            const unsigned b = __ffs(x) - 1;
+            if (w >= first_ok[b]) elig |= 1u << b;
+          }
+          out = acc & elig & vmask;
+          if (out) atomicAdd(p.win + WF_HUNG * p.W + w, (unsigned long long)__popc(out));
+        }
+        p.hung[(size_t)w * p.ncw + q] = out;  // w >= H-1: prefix(w), finished by the backward pass
+      }
+    }
+    unsigned suf = 0;
+    // backward: suffix AND inside blocks; only needed when some window of the call is >= H-1
+    for (long long s0 = (long long)W - 1; W >= H && s0 >= 0; s0 -= kB) {
+      unsigned cb[kB];
+#pragma unroll
+      for (unsigned i = 0; i < kB; ++i) cb[i] = s0 - (long long)i >= 0 ? hang_cond(p, (unsigned)(s0 - i), q) : 0u;
+#pragma unroll
+      for (unsigned i = 0; i < kB; ++i) {
+        const long long s = s0 - (long long)i;
+        if (s < 0) break;
+        suf = ((unsigned long long)s % H == H - 1 || s == (long long)W - 1) ? cb[i] : (suf & cb[i]);
+        const unsigned long long w = (unsigned long long)s + H - 1;
+        if (w < W) {
+          const unsigned f = suf & p.hung[(size_t)w * p.ncw + q] & vmask;
+          p.hung[(size_t)w * p.ncw + q] = f;
+          if (f) atomicAdd(p.win + WF_HUNG * p.W + w, (unsigned long long)__popc(f));
+        }
+      }
+    }
+  } else if (!lng && tid < nflag) {
     const unsigned w = (unsigned)(tid / p.ncw), q = (unsigned)(tid % p.ncw);
     const long long first = (long long)w - (long long)p.H + 1;
     unsigned acc = 0xFFFFFFFFu;
@@ -2150,7 +2216,7 @@ void launch_persist(const Params &p, cudaStream_t st) {
 
 void launch_hang(const Params &p, cudaStream_t st) {
   const unsigned threads = 256;
-  const size_t n = (((size_t)p.W * p.ncw + 31) & ~(size_t)31) + (size_t)p.ncw * 32;
+  const size_t n = ((hang_flag_threads(p.W, p.ncw, p.H) + 31) & ~(size_t)31) + (size_t)p.ncw * 32;
   { k_hang<<<(unsigned)((n + threads - 1) / threads), threads, 0, st>>>(p); count_launch(); }
 }
 

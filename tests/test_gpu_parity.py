@@ -353,6 +353,32 @@ def test_topk_full_prefix_shortcut(placement, n_windows):
         assert np.array_equal(got["topk"][w], ref["topk"][w]), w
 
 
+@pytest.mark.parametrize("H", [65, 100, 160])
+def test_long_hang_window_across_calls(H):
+    """H above the per-(window, word) AND loop's range takes the two-pass sliding-window AND
+    (DESIGN.md §4 K6); quiet components (few events) and held-full buffers make long runs that
+    cross call boundaries, so windows w < H-1 of every call depend on the carried run.  Flags and
+    n_hung of every window must equal the oracle's."""
+    wl = gen.C1.scaled("C1-longH", n_samples=300_000, n_events=3_000, n_windows=600, hang_windows=H)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=H, k=wl.k)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    s, e = gen.samples(wl), gen.events(wl)
+    t_end = wl.t_end()
+    w0, total_hung = 0, 0
+    for m in (50, 1, 120, 7, 300, 122):
+        w1 = w0 + m
+        sl = slice(wl.index_at("samples", wl.t_begin(w0)), wl.index_at("samples", wl.t_begin(w1)))
+        el = slice(wl.index_at("events", wl.t_begin(w0)), wl.index_at("events", wl.t_begin(w1)))
+        ref = orc.reduce(s[sl], e[el], t_end[w0:w1])
+        mon.ingest(_dev(s[sl]), _dev(e[el]))
+        got = mon.window_reduce(t_end[w0:w1])
+        assert_same(got, ref, mon, stats=False, comps=False)
+        total_hung += int(ref["summary"]["n_hung"].sum())
+        w0 = w1
+    assert w0 == wl.n_windows and total_hung > 0  # the long-run path was exercised
+
+
 @pytest.mark.parametrize("disorder", [False, True])
 @pytest.mark.parametrize("stream", ["samples", "events"])
 def test_order_check_across_tiles_with_invalid_gap(disorder, stream):
