@@ -1123,16 +1123,19 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
         if (g >= total) return 0ull;
         return __ldcg(p.stage + (S.seg_base[sgi] + g));
       };
-      // 4-deep software pipeline: staging reads are DRAM/L2 round trips
-      unsigned long long e0 = fetch(0), e1 = fetch(32), e2 = fetch(64), e3 = fetch(96);
+#if defined(RTM_FOLD_DEPTH1)
+      for (unsigned c = 0; c < total; c += 32) fold_chunk<NAR>(S, lane, lt, c + lane < total, fetch(c), Wlen);
+#else
+      // 2-deep software pipeline over the staging reads (measured on C2: depth 2 709 us, 3 715 us,
+      // 4 719 us, 6 727 us - deeper costs registers the chunk logic needs)
+      unsigned long long e0 = fetch(0), e1 = fetch(32);
       for (unsigned c = 0; c < total; c += 32) {
-        const unsigned long long en = fetch(c + 128);
+        const unsigned long long en = fetch(c + 64);
         fold_chunk<NAR>(S, lane, lt, c + lane < total, e0, Wlen);
         e0 = e1;
-        e1 = e2;
-        e2 = e3;
-        e3 = en;
+        e1 = en;
       }
+#endif
     }
     // ---- publish this window's last levels (kSent: untouched) and the phase-1 flag
     const unsigned b_base = bin * kBin;
