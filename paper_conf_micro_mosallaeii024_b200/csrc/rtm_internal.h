@@ -30,7 +30,10 @@ constexpr int kTileS = 4096;                // samples per partition tile
 constexpr int kTileE = 4096;                // events per event tile
 constexpr int kK1Threads = 256;             // 8 warps x 512-sample sub-tiles
 constexpr int kK3Threads = 256;
-constexpr int kFoldWarps = 4;               // warps per fold CTA
+#ifndef RTM_FOLD_WARPS
+#define RTM_FOLD_WARPS 4
+#endif
+constexpr int kFoldWarps = RTM_FOLD_WARPS;  // warps per fold CTA (compile-time A/B override)
 constexpr uint16_t kSent = 0xFFFFu;         // "no kept sample in this window" marker
 constexpr uint32_t kMaxBins = 4096;         // n_buffers <= 2^20 (fallback partition smem 160 KB)
 constexpr uint32_t kTopkSmemKeys = 40960;   // keys held in shared memory by the top-k kernel

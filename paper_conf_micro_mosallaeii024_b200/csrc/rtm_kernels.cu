@@ -1068,7 +1068,7 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
 }
 
 template <bool NAR>
-__global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
+__global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   FoldSmem &S = reinterpret_cast<FoldSmem *>(smem)[threadIdx.x >> 5];
   const int lane = threadIdx.x & 31;
@@ -1123,11 +1123,8 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
         if (g >= total) return 0ull;
         return __ldcg(p.stage + (S.seg_base[sgi] + g));
       };
-#if defined(RTM_FOLD_DEPTH1)
-      for (unsigned c = 0; c < total; c += 32) fold_chunk<NAR>(S, lane, lt, c + lane < total, fetch(c), Wlen);
-#else
       // 2-deep software pipeline over the staging reads (measured on C2: depth 2 709 us, 3 715 us,
-      // 4 719 us, 6 727 us - deeper costs registers the chunk logic needs)
+      // 4 719 us, 6 727 us - deeper costs registers the chunk logic needs; depth 1: 863 us)
       unsigned long long e0 = fetch(0), e1 = fetch(32);
       for (unsigned c = 0; c < total; c += 32) {
         const unsigned long long en = fetch(c + 64);
@@ -1135,7 +1132,6 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 8) k_fold(Params p) {
         e0 = e1;
         e1 = en;
       }
-#endif
     }
     // ---- publish this window's last levels (kSent: untouched) and the phase-1 flag
     const unsigned b_base = bin * kBin;
