@@ -1067,7 +1067,11 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
   __syncwarp();
 }
 
-template <bool NAR>
+// SPARSE (few samples per unit: C3-C5 shapes): many of a unit's 256 buffers are untouched in
+// several consecutive windows, so the look-back walks several windows; it takes them two at a time
+// (both flags waited for by two lanes, both rows loaded before either is used), halving the
+// dependent round trips.  A separate instantiation: the dense (C2) code is unchanged.
+template <bool NAR, bool SPARSE = false>
 __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   FoldSmem &S = reinterpret_cast<FoldSmem *>(smem)[threadIdx.x >> 5];
@@ -1163,8 +1167,9 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
         need = 0;
         break;
       }
-      if (lane == 0) {
-        const unsigned *f = p.flags + (size_t)j * p.nbins + bin;
+      const int pair = (SPARSE && j >= 1) ? 1 : 0;  // windows j and j-1 in one step
+      if (lane <= (unsigned)pair) {
+        const unsigned *f = p.flags + (size_t)(j - lane) * p.nbins + bin;
         unsigned spins = 0;
         while (ld_acquire_u32(f) != p.epoch) {
           __nanosleep(64);
@@ -1176,17 +1181,40 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
       }
       __syncwarp();
       const unsigned short *lj = p.lastlvl + (size_t)j * p.nb + b_base + lane;
+      if constexpr (SPARSE) {
+        unsigned short v0[kBin / 32], v1[kBin / 32];
 #pragma unroll
-      for (int i = 0; i < kBin / 32; ++i) {
-        if (need & (1u << i)) {
-          const unsigned short v = ld_relaxed_u16(lj + 32 * i);
-          if (v != kSent) {
-            lin[i] = v;
-            need &= ~(1u << i);
+        for (int i = 0; i < kBin / 32; ++i) {
+          v0[i] = v1[i] = kSent;
+          if (need & (1u << i)) {
+            v0[i] = ld_relaxed_u16(lj + 32 * i);
+            if (pair) v1[i] = ld_relaxed_u16(lj - p.nb + 32 * i);
           }
         }
+#pragma unroll
+        for (int i = 0; i < kBin / 32; ++i) {
+          if (need & (1u << i)) {
+            const unsigned short v = v0[i] != kSent ? v0[i] : v1[i];
+            if (v != kSent) {
+              lin[i] = v;
+              need &= ~(1u << i);
+            }
+          }
+        }
+        j -= 1 + pair;
+      } else {
+#pragma unroll
+        for (int i = 0; i < kBin / 32; ++i) {
+          if (need & (1u << i)) {
+            const unsigned short v = ld_relaxed_u16(lj + 32 * i);
+            if (v != kSent) {
+              lin[i] = v;
+              need &= ~(1u << i);
+            }
+          }
+        }
+        --j;
       }
-      --j;
     }
     unsigned long long dig = 0;
     unsigned touched = 0;
@@ -2168,7 +2196,11 @@ void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
   const unsigned need = (units + kFoldWarps - 1) / kFoldWarps;
   if (grid > need) grid = need;
   if (grid == 0) grid = 1;
-  if (p.narrow) { k_fold<true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  // sparse units: fewer than 512 kept samples per (window, bin) on average (RTM_XP=512: dense)
+  const bool sparse = !(p.xp & 512) && p.ns < (uint64_t)512 * units;
+  if (p.narrow && sparse) { k_fold<true, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else if (p.narrow) { k_fold<true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else if (sparse) { k_fold<false, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else { k_fold<false><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
 }
 
@@ -2243,6 +2275,8 @@ void configure_kernels_once() {
                        (int)topk_smem_bytes(kTopkSmemKeys));
   cudaFuncSetAttribute(k_fold<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
   cudaFuncSetAttribute(k_fold<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
+  cudaFuncSetAttribute(k_fold<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
+  cudaFuncSetAttribute(k_fold<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
   cudaGetLastError();
 }
 
