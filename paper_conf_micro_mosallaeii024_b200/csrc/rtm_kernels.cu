@@ -1068,9 +1068,9 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
 }
 
 // SPARSE (few samples per unit: C3-C5 shapes): many of a unit's 256 buffers are untouched in
-// several consecutive windows, so the look-back walks several windows; it takes them two at a time
-// (both flags waited for by two lanes, both rows loaded before either is used), halving the
-// dependent round trips.  A separate instantiation: the dense (C2) code is unchanged.
+// several consecutive windows, so the look-back walks several windows; it takes RTM_LB_STEP of
+// them per step (their flags waited for by as many lanes, all rows loaded before any is used),
+// dividing the dependent round trips.  A separate instantiation: the dense (C2) code is unchanged.
 template <bool NAR, bool SPARSE = false>
 __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -1167,7 +1167,12 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
         need = 0;
         break;
       }
-      const int pair = (SPARSE && j >= 1) ? 1 : 0;  // windows j and j-1 in one step
+#ifndef RTM_LB_STEP
+#define RTM_LB_STEP 3  // measured (C3 fold / C5 fold per 20k windows): 2 -> 15.6 / 67.5 ms, 3 -> 14.7 / 60.5, 4 spills: 19.2 / 87.8
+#endif
+      constexpr int kStep = SPARSE ? RTM_LB_STEP : 1;  // windows per look-back step
+      const int nwin = j + 1 < kStep ? j + 1 : kStep;   // windows j .. j - nwin + 1
+      const int pair = nwin - 1;
       if (lane <= (unsigned)pair) {
         const unsigned *f = p.flags + (size_t)(j - lane) * p.nbins + bin;
         unsigned spins = 0;
@@ -1182,26 +1187,28 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
       __syncwarp();
       const unsigned short *lj = p.lastlvl + (size_t)j * p.nb + b_base + lane;
       if constexpr (SPARSE) {
-        unsigned short v0[kBin / 32], v1[kBin / 32];
+        unsigned short v[kStep][kBin / 32];
 #pragma unroll
-        for (int i = 0; i < kBin / 32; ++i) {
-          v0[i] = v1[i] = kSent;
-          if (need & (1u << i)) {
-            v0[i] = ld_relaxed_u16(lj + 32 * i);
-            if (pair) v1[i] = ld_relaxed_u16(lj - p.nb + 32 * i);
+        for (int d = 0; d < kStep; ++d)
+#pragma unroll
+          for (int i = 0; i < kBin / 32; ++i) {
+            v[d][i] = kSent;
+            if (d < nwin && (need & (1u << i))) v[d][i] = ld_relaxed_u16(lj - (size_t)d * p.nb + 32 * i);
           }
-        }
 #pragma unroll
         for (int i = 0; i < kBin / 32; ++i) {
           if (need & (1u << i)) {
-            const unsigned short v = v0[i] != kSent ? v0[i] : v1[i];
-            if (v != kSent) {
-              lin[i] = v;
+            unsigned short x = kSent;
+#pragma unroll
+            for (int d = kStep - 1; d >= 0; --d)
+              if (v[d][i] != kSent) x = v[d][i];  // the most recent window holding a level wins
+            if (x != kSent) {
+              lin[i] = x;
               need &= ~(1u << i);
             }
           }
         }
-        j -= 1 + pair;
+        j -= nwin;
       } else {
 #pragma unroll
         for (int i = 0; i < kBin / 32; ++i) {
