@@ -1170,7 +1170,10 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
 #ifndef RTM_LB_STEP
 #define RTM_LB_STEP 3  // measured (C3 fold / C5 fold per 20k windows): 2 -> 15.6 / 67.5 ms, 3 -> 14.7 / 60.5, 4 spills: 19.2 / 87.8
 #endif
-      constexpr int kStep = SPARSE ? RTM_LB_STEP : 1;  // windows per look-back step
+#ifndef RTM_LB_STEP_DENSE
+#define RTM_LB_STEP_DENSE 1  // C2: 3 windows per step 704 us, 2 (spills) 727 us, 1 705 us - kept simple
+#endif
+      constexpr int kStep = SPARSE ? RTM_LB_STEP : RTM_LB_STEP_DENSE;  // windows per look-back step
       const int nwin = j + 1 < kStep ? j + 1 : kStep;   // windows j .. j - nwin + 1
       const int pair = nwin - 1;
       if (lane <= (unsigned)pair) {
@@ -1186,7 +1189,7 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
       }
       __syncwarp();
       const unsigned short *lj = p.lastlvl + (size_t)j * p.nb + b_base + lane;
-      if constexpr (SPARSE) {
+      if constexpr (kStep > 1) {
         unsigned short v[kStep][kBin / 32];
 #pragma unroll
         for (int d = 0; d < kStep; ++d)
