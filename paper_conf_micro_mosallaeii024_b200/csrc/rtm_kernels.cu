@@ -1916,7 +1916,7 @@ __global__ void k_hang(Params p) {
 // K7: progress bars (L131): per kernel, cumulative START/END over windows (block scan), and
 // the per-component cumulative counts for the last window.
 // ============================================================================================
-__global__ void __launch_bounds__(256) k_progress(Params p) {
+__global__ void __launch_bounds__(1024) k_progress(Params p) {
   __shared__ unsigned scan_scratch[32];
   const unsigned k = blockIdx.x;
   if (k < p.nk) {
@@ -2263,8 +2263,9 @@ void launch_hang(const Params &p, cudaStream_t st) {
 }
 
 void launch_progress(const Params &p, cudaStream_t st) {
-  const unsigned comp_blocks = (p.nc + 255) / 256 < 256 ? (p.nc + 255) / 256 : 256;
-  { k_progress<<<p.nk + comp_blocks, 256, 0, st>>>(p); count_launch(); }
+  // 1024 threads: one block scan covers up to 1024 windows per kernel bar (4 rounds at 256)
+  const unsigned comp_blocks = (p.nc + 1023) / 1024 < 256 ? (p.nc + 1023) / 1024 : 256;
+  { k_progress<<<p.nk + comp_blocks, 1024, 0, st>>>(p); count_launch(); }
 }
 
 uint64_t pack_bytes(const Params &p) { return pack_layout(p).total; }
