@@ -62,8 +62,10 @@ enum { RTM_HANG_FULL = 0, RTM_HANG_NONEMPTY = 1 };
 enum { RTM_RANK_PERCENT = 0, RTM_RANK_SIZE = 1,
        /* persistence ranking (a buffer "repeatedly at the top of the list"
         * is the bottleneck, L173, L197-L199): the window's time-weighted mean occupancy
-        * integral / (capacity * window length), descending, ties by buffer_id.  world == 1 only;
-        * every window of a call must be shorter than 2^32 ticks (else RTM_E_INVALID). */
+        * integral / (capacity * window length), descending, ties by buffer_id.  Every window of a
+        * call must be shorter than 2^32 ticks (else RTM_E_INVALID).  world > 1: each rank ranks its
+        * owned buffers and the exchange pack carries the 64-bit order key of every candidate, so
+        * the merge ranks the union exactly. */
        RTM_RANK_MEAN = 2 };
 
 /* ---- trace records (16 B each, little-endian, naturally aligned) --------------------------
@@ -110,7 +112,7 @@ typedef struct {
   int64_t t0;                       /* begin of the first window                               */
   uint32_t hang_windows;            /* H >= 1: consecutive windows before a hang is flagged    */
   uint32_t k;                       /* top-k computed for every window, 1 .. 1024              */
-  int32_t rank_mode;                /* RTM_RANK_PERCENT or RTM_RANK_SIZE                       */
+  int32_t rank_mode;                /* RTM_RANK_PERCENT, RTM_RANK_SIZE or RTM_RANK_MEAN        */
   int32_t device;                   /* CUDA device ordinal                                     */
   int32_t rank, world;              /* world == 1: single GPU; else this context is one shard  */
   const uint8_t *owned_components;  /* host [n_components] or NULL (= all): components whose

@@ -52,6 +52,7 @@ struct rtm_ctx {
   DevBuf gid, bstat_g;      // rank-local numbering: global id per local buffer, table by global id
   DevBuf tkscr;             // per-slice top-k candidates (few-window calls)
   DevBuf mkey, rcp64;       // rank mode MEAN: per-(window, buffer) order keys, floor(2^64 / c)
+  DevBuf tkey;              // rank mode MEAN, world > 1: the local top-k's order keys (exchange pack)
   DevBuf persist;           // windows-in-top-k counter per buffer (id space)
   DevBuf klive;             // progress bar ids in use
   std::vector<uint8_t> klive_h;
@@ -400,6 +401,10 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     if ((s = ensure(c, c->mkey, Wn * c->nb * 8))) return s;
     p.mkey = (unsigned long long *)c->mkey.p;
     p.rcp64 = (const unsigned long long *)c->rcp64.p;
+    if (c->world > 1) {  // the merge ranks the ranks' candidates by these keys
+      if ((s = ensure(c, c->tkey, Wn * c->k * 8))) return s;
+      p.tkey = (unsigned long long *)c->tkey.p;
+    }
   }
   p.persist = (uint32_t *)c->persist.p;
   p.tk_slices = topk_slices(c->nb, c->k, W, c->n_sms, c->n_elig == c->nb && c->rank_mode != RTM_RANK_MEAN,
@@ -592,7 +597,6 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   if (cfg->k == 0 || cfg->k > 1024 || cfg->hang_windows == 0) return RTM_E_INVALID;
   if (cfg->rank_mode != RTM_RANK_PERCENT && cfg->rank_mode != RTM_RANK_SIZE && cfg->rank_mode != RTM_RANK_MEAN)
     return RTM_E_INVALID;
-  if (cfg->rank_mode == RTM_RANK_MEAN && cfg->world > 1) return RTM_E_INVALID;
   if (cfg->hang_mode != RTM_HANG_FULL && cfg->hang_mode != RTM_HANG_NONEMPTY) return RTM_E_INVALID;
   if (!cfg->buffer_owner || !cfg->buffer_capacity || !cfg->kernel_total) return RTM_E_INVALID;
   if (cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world) return RTM_E_INVALID;
@@ -711,7 +715,7 @@ void rtm_destroy(rtm_ctx *c) {
                     &c->rts, &c->rte, &c->treg_s, &c->treg_e, &c->tdesc, &c->soff, &c->stage, &c->smeta, &c->emeta,
                     &c->lastlvl, &c->res, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
                     &c->unit_ctr, &c->bstat, &c->comps, &c->pack,
-                    &c->gathered};
+                    &c->gathered, &c->tkscr, &c->mkey, &c->rcp64, &c->tkey, &c->persist, &c->klive};
   for (DevBuf *b : bufs) free_buf(*b);
   if (c->h_small.p) cudaFreeHost(c->h_small.p);
   if (c->h_res.p) cudaFreeHost(c->h_res.p);

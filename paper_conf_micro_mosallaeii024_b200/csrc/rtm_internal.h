@@ -136,6 +136,7 @@ struct Params {
   rtm_component_tasks *comps;// [nc]
   unsigned long long *mkey;  // [W * nb] rank mode MEAN: floor(integral * 2^32 / cap) (exact order key)
   const unsigned long long *rcp64;  // [65536] floor(2^64 / c) (c >= 2)
+  unsigned long long *tkey;  // [W * k] MEAN, world > 1: order keys of the local top-k (exchange pack)
   uint32_t *persist;         // [id space] windows in the top-k list
   int32_t persist_inline;    // world == 1: the top-k kernels count their own winners (no k_persist)
   uint32_t n_watch;          // value monitor: watched local buffer ids (0xFFFFFFFF: not on this rank)

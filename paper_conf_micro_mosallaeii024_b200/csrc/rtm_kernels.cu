@@ -1659,8 +1659,11 @@ __global__ void __launch_bounds__(kT64Threads) k_topk64(Params p) {
   __shared__ unsigned cand[kT64Cand];
   __shared__ unsigned long long selk[1024];
   __shared__ unsigned seli[1024];
-  const unsigned w = blockIdx.x, ne = p.nb, lane = threadIdx.x & 31;
-  const unsigned long long *key = p.mkey + (size_t)w * p.nb;
+  // candidates: the eligible buffers (owned components; all when n_elig == nb), indexed in id order
+  const bool sub = p.n_elig < p.nb;
+  const unsigned w = blockIdx.x, ne = sub ? p.n_elig : p.nb, lane = threadIdx.x & 31;
+  const unsigned long long *keyw = p.mkey + (size_t)w * p.nb;
+  auto K = [&](unsigned i) { return __ldcg(keyw + (sub ? __ldg(p.elig_ids + i) : i)); };
   const unsigned keff = p.k < ne ? p.k : ne;
   unsigned long long prefix = 0, mask = 0;
   unsigned need = keff, n_it = ne;
@@ -1673,7 +1676,7 @@ __global__ void __launch_bounds__(kT64Threads) k_topk64(Params p) {
       bool ok = false;
       unsigned dg = 0;
       if (j < n_it) {
-        const unsigned long long k = __ldcg(key + (use_c ? cand[j] : j));
+        const unsigned long long k = K(use_c ? cand[j] : j);
         ok = (k & mask) == prefix;
         dg = (unsigned)(k >> (8 * d)) & 255u;
       }
@@ -1699,10 +1702,10 @@ __global__ void __launch_bounds__(kT64Threads) k_topk64(Params p) {
       const unsigned long long lim = prefix >> (8 * d);
       const unsigned chunk = (ne + blockDim.x - 1) / blockDim.x, c0 = threadIdx.x * chunk;
       unsigned cnt = 0;
-      for (unsigned i = c0; i < c0 + chunk && i < ne; ++i) cnt += (__ldcg(key + i) >> (8 * d)) >= lim;
+      for (unsigned i = c0; i < c0 + chunk && i < ne; ++i) cnt += (K(i) >> (8 * d)) >= lim;
       unsigned pos = block_excl_scan(cnt, scan_scratch, nullptr);
       for (unsigned i = c0; i < c0 + chunk && i < ne; ++i)
-        if ((__ldcg(key + i) >> (8 * d)) >= lim) cand[pos++] = i;
+        if ((K(i) >> (8 * d)) >= lim) cand[pos++] = i;
       n_it = s_ncand;
       use_c = true;
     }
@@ -1716,7 +1719,7 @@ __global__ void __launch_bounds__(kT64Threads) k_topk64(Params p) {
   unsigned ceq = 0;
   for (unsigned j = c0; j < c0 + chunk && j < n_it; ++j) {
     const unsigned i = use_c ? cand[j] : j;
-    const unsigned long long k = __ldcg(key + i);
+    const unsigned long long k = K(i);
     if (k > tau) {
       const unsigned slot = atomicAdd(&s_ngt, 1u);
       selk[slot] = k;
@@ -1728,7 +1731,7 @@ __global__ void __launch_bounds__(kT64Threads) k_topk64(Params p) {
   const unsigned ngt = s_ngt;
   for (unsigned j = c0; j < c0 + chunk && j < n_it && rank < need; ++j) {
     const unsigned i = use_c ? cand[j] : j;
-    if (__ldcg(key + i) == tau) {
+    if (K(i) == tau) {
       selk[ngt + rank] = tau;
       seli[ngt + rank] = i;
       ++rank;
@@ -1761,12 +1764,13 @@ __global__ void __launch_bounds__(kT64Threads) k_topk64(Params p) {
   for (unsigned i = threadIdx.x; i < p.k; i += blockDim.x) {
     unsigned long long out = 0xFFFFFFFFull;
     if (i < keff) {
-      const unsigned b = seli[i];
+      const unsigned b = sub ? __ldg(p.elig_ids + seli[i]) : seli[i];
       out = (unsigned long long)(p.gid ? __ldg(p.gid + b) : b) | ((unsigned long long)lv[b] << 32) |
             ((unsigned long long)__ldg(p.cap + b) << 48);
       if (p.persist_inline) atomicAdd(p.persist + (unsigned)(out & 0xFFFFFFFFull), 1u);  // k_persist fused
     }
     p.topk[(size_t)w * p.k + i] = out;
+    if (p.tkey) p.tkey[(size_t)w * p.k + i] = i < keff ? selk[i] : 0ull;  // world > 1: for the merge
   }
   if (threadIdx.x == 0) p.topk_n[w] = keff;
 }
@@ -1967,10 +1971,11 @@ __global__ void __launch_bounds__(1024) k_progress(Params p) {
 // Multi-rank merge (world > 1).  Pack layout per rank (bytes, 8-aligned sections):
 //   win [kWinFields][W] u64 | topk [W][k] u64 | topk_n [W] u32 (padded) | prog [W][nk][5] i64 |
 //   hung [W][ncw] u32 (padded) | comps [nc] (3 x i64) | bstat [pack_nb] (32 B; reserved = owned) |
-//   gids [pack_nb] u32 (rank-local numbering only: the global id of each bstat entry, ~0 = pad)
+//   gids [pack_nb] u32 (rank-local numbering only: the global id of each bstat entry, ~0 = pad) |
+//   tkey [W][k] u64 (rank mode MEAN only: the order key of each top-k entry, mean_key)
 // ============================================================================================
 struct PackLayout {
-  size_t win, topk, topk_n, prog, hung, comps, bstat, gids, total;
+  size_t win, topk, topk_n, prog, hung, comps, bstat, gids, tkey, total;
 };
 __host__ __device__ inline size_t align8(size_t x) { return (x + 7) & ~(size_t)7; }
 __host__ __device__ inline PackLayout pack_layout(const Params &p) {
@@ -1984,6 +1989,7 @@ __host__ __device__ inline PackLayout pack_layout(const Params &p) {
   L.comps = o; o += align8((size_t)p.nc * sizeof(rtm_component_tasks));
   L.bstat = o; o += align8((size_t)p.pack_nb * sizeof(rtm_buffer_stat));
   L.gids = o; o += p.gid ? align8((size_t)p.pack_nb * 4) : 0;
+  L.tkey = o; o += p.rank_mode == RTM_RANK_MEAN ? (size_t)p.W * p.k * 8 : 0;
   L.total = o;
   return L;
 }
@@ -1995,7 +2001,10 @@ __device__ __forceinline__ unsigned long long topk_composite(unsigned long long 
   return ((unsigned long long)fullness_key(l, c, mode, rcp) << 32) | (0xFFFFFFFFu - b);
 }
 
-// one CTA per window: merge world x k candidates; sums of scalar fields; progress sums; hang OR
+// one CTA per window: merge world x k candidates; sums of scalar fields; progress sums; hang OR.
+// Candidates rank by (key, sec) descending: PERCENT / SIZE key = fullness32 << 32 | ~id, sec = 0;
+// MEAN key = the 64-bit mean_key from the pack, sec = ~id.  Padding (0, 0) ranks last: a real
+// candidate has key >= 1 (PERCENT / SIZE) or sec >= 1 (MEAN, ids < 2^32 - 1).
 __global__ void __launch_bounds__(256) k_merge_windows(Params p, const unsigned char *g, unsigned world,
                                                        size_t stride) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -2006,19 +2015,28 @@ __global__ void __launch_bounds__(256) k_merge_windows(Params p, const unsigned 
   unsigned P = 1;
   while (P < nc_all) P <<= 1;
   unsigned long long *full_ent = cand + P;  // [P] entries aligned with cand
+  unsigned *sec = reinterpret_cast<unsigned *>(full_ent + P);  // [P] tie-break word (MEAN: ~id)
+  const bool mean = p.rank_mode == RTM_RANK_MEAN;
   for (unsigned i = threadIdx.x; i < P; i += blockDim.x) {
     unsigned long long key = 0, en = 0;
+    unsigned sc = 0;
     if (i < nc_all) {
       const unsigned r = i / p.k, s = i % p.k;
       const unsigned char *base = g + stride * r;
       const unsigned n = reinterpret_cast<const unsigned *>(base + L.topk_n)[w];
       if (s < n) {
         en = reinterpret_cast<const unsigned long long *>(base + L.topk)[(size_t)w * p.k + s];
-        key = topk_composite(en, p.rank_mode, p.rcp);
+        if (mean) {
+          key = reinterpret_cast<const unsigned long long *>(base + L.tkey)[(size_t)w * p.k + s];
+          sc = 0xFFFFFFFFu - (unsigned)(en & 0xFFFFFFFFull);
+        } else {
+          key = topk_composite(en, p.rank_mode, p.rcp);
+        }
       }
     }
     cand[i] = key;
     full_ent[i] = en;
+    sec[i] = sc;
   }
   __syncthreads();
   for (unsigned size = 2; size <= P; size <<= 1) {
@@ -2028,8 +2046,10 @@ __global__ void __launch_bounds__(256) k_merge_windows(Params p, const unsigned 
         if (jx > i) {
           bool desc = (i & size) == 0;
           unsigned long long a = cand[i], b = cand[jx];
-          if ((a < b) == desc) {
+          const unsigned sa = sec[i], sb = sec[jx];
+          if ((a < b || (a == b && sa < sb)) == desc) {
             cand[i] = b; cand[jx] = a;
+            sec[i] = sb; sec[jx] = sa;
             unsigned long long t = full_ent[i]; full_ent[i] = full_ent[jx]; full_ent[jx] = t;
           }
         }
@@ -2308,6 +2328,10 @@ void launch_pack(const Params &p, void *pack, cudaStream_t st) {
     cudaMemcpyAsync(d + L.gids, p.gid, (size_t)p.nb * 4, cudaMemcpyDeviceToDevice, st);
     if (p.pack_nb > p.nb) cudaMemsetAsync(d + L.gids + (size_t)p.nb * 4, 0xFF, (size_t)(p.pack_nb - p.nb) * 4, st);
   }
+  if (p.rank_mode == RTM_RANK_MEAN) {
+    if (p.tkey) cudaMemcpyAsync(d + L.tkey, p.tkey, (size_t)p.W * p.k * 8, cudaMemcpyDeviceToDevice, st);
+    else cudaMemsetAsync(d + L.tkey, 0, (size_t)p.W * p.k * 8, st);
+  }
 }
 
 void launch_scatter_bstat(const Params &p, cudaStream_t st) {
@@ -2319,7 +2343,7 @@ void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStr
   const size_t stride = pack_layout(p).total;
   unsigned P = 1;
   while (P < world * p.k) P <<= 1;
-  const size_t sm = (size_t)P * 16;
+  const size_t sm = (size_t)P * 20;  // cand + full_ent (u64) + sec (u32)
   if (sm > 48 * 1024) cudaFuncSetAttribute(k_merge_windows, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
   { k_merge_windows<<<p.W, 256, sm, st>>>(p, static_cast<const unsigned char *>(gathered), world, stride); count_launch(); }
   { k_merge_tables<<<256, 256, 0, st>>>(p, static_cast<const unsigned char *>(gathered), world, stride); count_launch(); }

@@ -222,15 +222,20 @@ def test_case_study_deadlock_on_gpu():
     assert [list(mon.hang_check(w)) for w in range(6)] == [[], [], [], [], [1, 2], [0, 1, 2, 3]]
 
 
-def test_virtual_shards_merge_equals_whole():
-    """Three shard contexts on one GPU (owner-component sharding) + the library's merge kernels."""
+SHARD_RANKINGS = [(0, None), (1, None), (2, None), (2, 512)]  # (rank_mode, k); k=512 > owned per rank
+
+
+@pytest.mark.parametrize("mode,k", SHARD_RANKINGS)
+def test_virtual_shards_merge_equals_whole(mode, k):
+    """Three shard contexts on one GPU (owner-component sharding) + the library's merge kernels, in
+    every rank mode (MEAN: the packs carry the 64-bit order keys, include/rtm.h RTM_RANK_MEAN)."""
     import ctypes
 
     from paper_conf_micro_mosallaeii024_b200 import _copy_from_ptr
 
     wl = gen.C1.scaled("C1-vshard", n_samples=200_000, n_events=20_000, n_windows=6)
     owner, cap, tot = gen.registry(wl)
-    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    kw = dict(t0=wl.t0, hang_windows=2, k=k or wl.k, rank_mode=mode)
     ref = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw).reduce(gen.samples(wl), gen.events(wl),
                                                                                    wl.t_end())
     G = 3
@@ -414,7 +419,8 @@ def test_order_check_across_tiles_with_invalid_gap(disorder, stream):
         assert_same(mon.window_reduce(ends), ref, mon)
 
 
-def test_rank_local_numbering_shards_merge_equals_whole():
+@pytest.mark.parametrize("mode,k", SHARD_RANKINGS)
+def test_rank_local_numbering_shards_merge_equals_whole(mode, k):
     """Owner sharding with RANK-LOCAL buffer numbering (include/rtm.h buffer_global_id): each
     shard registers only its own buffers (dense local ids, records remapped to them), results
     carry global ids; the merged top-k, digests, progress, hang flags and the per-buffer table
@@ -425,7 +431,7 @@ def test_rank_local_numbering_shards_merge_equals_whole():
 
     wl = gen.C1.scaled("C1-lshard", n_samples=200_000, n_events=20_000, n_windows=6)
     owner, cap, tot = gen.registry(wl)
-    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    kw = dict(t0=wl.t0, hang_windows=2, k=k or wl.k, rank_mode=mode)
     ref = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw).reduce(gen.samples(wl), gen.events(wl),
                                                                                    wl.t_end())
     G = 3

@@ -405,6 +405,28 @@ def test_shard_merge_equals_whole():
     assert np.array_equal(hung, whole["hung"])
 
 
+def test_shard_topk_mean_decomposes():
+    """Rank mode MEAN at world > 1: the merge ranks the union of the shards' lists by
+    their exchanged order keys, which is exact iff, in every window, each shard's list is the prefix
+    of the whole-trace ranking restricted to that shard's owned buffers (then the whole top-k lies
+    in the union, in the same relative order).  Checked on the oracle alone, no keys needed."""
+    wl = gen.C1.scaled("C1-shard-mean", n_samples=200_000, n_events=20_000, n_windows=6)
+    owner, cap, tot = gen.registry(wl)
+    for k in (wl.k, 512):
+        kw = dict(n_components=wl.n_components, t0=wl.t0, hang_windows=2, k=k, rank_mode=2)
+        whole = oracle.Oracle(owner, cap, tot, **kw).reduce(gen.samples(wl), gen.events(wl), wl.t_end())
+        for r in range(3):
+            owned = (np.arange(wl.n_components) % 3 == r).astype(np.uint8)
+            sh = oracle.Oracle(owner, cap, tot, owned=owned, **kw).reduce(gen.samples(wl, shard=(3, r)),
+                                                                           gen.events(wl, shard=(3, r)), wl.t_end())
+            n_owned = int(owned[owner].sum())
+            for w in range(wl.n_windows):
+                ids = [int(x) for x in sh["topk"][w]["buffer_id"][: sh["topk_n"][w]]]
+                assert len(ids) == min(k, n_owned) and all(owned[owner[b]] for b in ids)
+                mine = [int(b) for b in whole["topk"][w]["buffer_id"][: whole["topk_n"][w]] if owned[owner[b]]]
+                assert ids[: len(mine)] == mine  # the whole list's owned part is this shard's prefix
+
+
 def test_gpu_fullness_key_reciprocal_formula_is_exact():
     """The CUDA top-k computes floor(l*2^32/c) as q0 = (l*m)>>16, m = floor(2^48/c), plus one
     remainder fix-up (DESIGN.md §4 K5).  Emulated here exhaustively for small caps and on random
