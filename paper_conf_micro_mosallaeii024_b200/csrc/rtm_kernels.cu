@@ -39,6 +39,11 @@ __device__ __forceinline__ unsigned ld_acquire_u32(const unsigned *p) {
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ unsigned ld_relaxed_u32(const unsigned *p) {
+  unsigned v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
 __device__ __forceinline__ void st_release_u32(unsigned *p, unsigned v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -1179,13 +1184,20 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
       if (lane <= (unsigned)pair) {
         const unsigned *f = p.flags + (size_t)(j - lane) * p.nbins + bin;
         unsigned spins = 0;
-        while (ld_acquire_u32(f) != p.epoch) {
+#ifndef RTM_SPIN_RELAXED
+#define RTM_SPIN_RELAXED 1
+#endif
+        // ld.acquire.gpu compiles to a strong load + CCTL.IVALL (the whole L1 invalidated) per
+        // poll: spin relaxed, then ONE acquire of the flag (epochs are never overwritten within a
+        // call, so it reads the published value and synchronizes with its release)
+        while ((RTM_SPIN_RELAXED ? ld_relaxed_u32(f) : ld_acquire_u32(f)) != p.epoch) {
           __nanosleep(64);
           if (++spins > (1u << 25)) {  // ~seconds: never expected; fail loudly instead of hanging
             atomicOr(p.status, 4u);
             break;
           }
         }
+        if (RTM_SPIN_RELAXED) (void)ld_acquire_u32(f);
       }
       __syncwarp();
       const unsigned short *lj = p.lastlvl + (size_t)j * p.nb + b_base + lane;
