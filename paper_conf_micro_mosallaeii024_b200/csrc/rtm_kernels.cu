@@ -1019,6 +1019,41 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
   const unsigned win = act ? S.owner[lid] : (unsigned)lane;
   const bool lost = win != (unsigned)lane;
   const unsigned told = __reduce_or_sync(kFull, lost ? (1u << win) : 0u);
+#ifndef RTM_FOLD_NODUP_FAST
+#define RTM_FOLD_NODUP_FAST 1
+#endif
+  // the buffer state update of a chain tail (sum / mm / count over the chain, head's offset)
+  auto update = [&](const uint4 &sv, bool c0, unsigned long long d, unsigned mm, unsigned n16,
+                    unsigned long long off0) {
+    unsigned hi = mm >> 16, lo = mm & 0xFFFFu;
+    if (c0) {
+      hi = max(hi, sv.z >> 16);
+      lo = min(lo, sv.w & 0xFFFFu);
+      d += st_D(sv);
+      n16 += sv.w >> 16;
+      if (n16 > 0xFFFFu) {  // rare: more than 65535 samples of one buffer in one window
+        S.hi[lid] += 1;
+        n16 -= 0x10000u;
+      }
+    } else {
+      S.ts0[lid] = (unsigned)off0;
+      if (!NAR && (off0 >> 32)) S.hi[lid] += (unsigned)(off0 >> 32) << 16;  // windows >= 2^32 ticks
+    }
+    S.st[lid] = make_uint4((unsigned)d, (unsigned)(d >> 32), lvl | (hi << 16), lo | (n16 << 16));
+  };
+  if (RTM_FOLD_NODUP_FAST && told == 0) {  // warp-uniform: every buffer of the chunk is distinct
+    if (act) {  // each lane is its buffer's whole chain: no match, no chain propagation
+      const uint4 sv = S.st[lid];
+      const bool c0 = st_touched(sv);
+      const unsigned prev = c0 ? (sv.z & 0xFFFFu) : 0u;
+      const unsigned long long contrib =
+          NAR ? (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(unsigned)(Wlen - off))
+              : (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off));
+      update(sv, c0, contrib, (lvl << 16) | lvl, 1u, off);
+    }
+    __syncwarp();
+    return;
+  }
   const bool dup = lost | ((told >> lane) & 1u);
   const unsigned mk = __match_any_sync(kFull, dup ? lid : 0xFFFFFFFFu);
   const unsigned peers = dup ? mk : (1u << lane);
@@ -1050,25 +1085,7 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
     }
   }
   const unsigned long long off0 = __shfl_sync(kFull, off, __ffs(peers) - 1);  // chain head's offset
-  if (act && tail) {
-    unsigned hi = mm >> 16, lo = mm & 0xFFFFu;
-    unsigned long long d = sum;
-    unsigned n16 = rank + 1;
-    if (c0) {
-      hi = max(hi, sv.z >> 16);
-      lo = min(lo, sv.w & 0xFFFFu);
-      d += st_D(sv);
-      n16 += sv.w >> 16;
-      if (n16 > 0xFFFFu) {  // rare: more than 65535 samples of one buffer in one window
-        S.hi[lid] += 1;
-        n16 -= 0x10000u;
-      }
-    } else {
-      S.ts0[lid] = (unsigned)off0;
-      if (!NAR && (off0 >> 32)) S.hi[lid] += (unsigned)(off0 >> 32) << 16;  // windows >= 2^32 ticks
-    }
-    S.st[lid] = make_uint4((unsigned)d, (unsigned)(d >> 32), lvl | (hi << 16), lo | (n16 << 16));
-  }
+  if (act && tail) update(sv, c0, sum, mm, rank + 1, off0);
   __syncwarp();
 }
 

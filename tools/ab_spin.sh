@@ -1,4 +1,5 @@
-B=paper_conf_micro_mosallaeii024_b200/librtm_b.so
+# A/B of a compile-time variant: default librtm.so (A) vs librtm_b.so (B): GPU parity on A, C2 bench lines alternating, one C3 line each
+B=${1:-paper_conf_micro_mosallaeii024_b200/librtm_b.so}
 timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -p no:cacheprovider -k "not full" 2>&1 | tail -1
 for i in 1 2 3; do
   for v in A B; do
