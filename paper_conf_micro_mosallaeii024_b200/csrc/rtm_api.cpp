@@ -474,14 +474,29 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   // sample (+ 16 B per task event when the event tiles run inside it); fold = the 8 B entry
   LAUNCH(KT_PARTITION, (uint64_t)ns * 24 + (p.fuse_events ? (uint64_t)ne * 16 : 0),
          launch_partition(p, c->n_sms, c->st));
+  // The order check (tile metadata) and the progress bars (event counts) do not read the fold's
+  // outputs: on the side stream, beside the fold (after the event kernel when it runs there);
+  // joined before the top-k.  One-window streaming calls: -13 us of dependent launches.
+  static const bool side = !getenv("RTM_NO_SIDE_TAIL");  // A/B switch
+  if (side) {
+    CK(cudaEventRecord(c->ev_fork, c->st));
+    CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
+    if (c->prof) prof_begin_on(c, KT_ORDER, 0, c->st2);
+    launch_order_check(p, c->st2);
+    if (c->prof) prof_end_on(c, c->st2);
+    if (c->prof) prof_begin_on(c, KT_PROGRESS, 0, c->st2);
+    launch_progress(p, c->st2);
+    if (c->prof) prof_end_on(c, c->st2);
+    CK(cudaEventRecord(c->ev_join, c->st2));
+  }
   LAUNCH(KT_FOLD, (uint64_t)ns * 8, launch_fold(p, c->n_sms, c->st));
-  if (!p.fuse_events) CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
-  LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
+  if (side || !p.fuse_events) CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
+  if (!side) LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
   p.persist_inline = c->world == 1 && p.persist;  // world > 1: counted from the merged lists
   LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
   p.persist_inline = 0;
   LAUNCH(KT_HANG, 0, launch_hang(p, c->st));
-  LAUNCH(KT_PROGRESS, 0, launch_progress(p, c->st));
+  if (!side) LAUNCH(KT_PROGRESS, 0, launch_progress(p, c->st));
   CK(cudaGetLastError());
 #ifdef RTM_PHASE_TIMING
   {
@@ -638,7 +653,12 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   if (cudaSetDevice(c->device) != cudaSuccess) { cudaGetLastError(); delete c; return RTM_E_CUDA; }
   configure_kernels_once();
   cudaDeviceGetAttribute(&c->n_sms, cudaDevAttrMultiProcessorCount, c->device);
-  if (cudaStreamCreateWithFlags(&c->st2, cudaStreamNonBlocking) != cudaSuccess ||
+  // side stream at the highest priority: its small kernels (order check, progress) are dispatched
+  // before the persistent fold's CTAs, which would otherwise hold every SM until the fold ends
+  int prio_lo = 0, prio_hi = 0;
+  cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+  if (getenv("RTM_SIDE_PRIO_OFF")) prio_hi = prio_lo;  // A/B switch
+  if (cudaStreamCreateWithPriority(&c->st2, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess) {
     cudaGetLastError();
