@@ -492,10 +492,23 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   LAUNCH(KT_FOLD, (uint64_t)ns * 8, launch_fold(p, c->n_sms, c->st));
   if (side || !p.fuse_events) CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
   if (!side) LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
+  // the hang flags (fold's anyfull + event activity bits) and the top-k (fold's last levels) are
+  // independent: the hang kernel on the side stream beside the top-k (the waits above are already
+  // enqueued, so the fork / join events can be recorded again)
+  static const bool side_hang = !getenv("RTM_NO_SIDE_HANG");  // A/B switch
+  if (side_hang) {
+    CK(cudaEventRecord(c->ev_fork, c->st));
+    CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
+    if (c->prof) prof_begin_on(c, KT_HANG, 0, c->st2);
+    launch_hang(p, c->st2);
+    if (c->prof) prof_end_on(c, c->st2);
+    CK(cudaEventRecord(c->ev_join, c->st2));
+  }
   p.persist_inline = c->world == 1 && p.persist;  // world > 1: counted from the merged lists
   LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
   p.persist_inline = 0;
-  LAUNCH(KT_HANG, 0, launch_hang(p, c->st));
+  if (side_hang) CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
+  else LAUNCH(KT_HANG, 0, launch_hang(p, c->st));
   if (!side) LAUNCH(KT_PROGRESS, 0, launch_progress(p, c->st));
   CK(cudaGetLastError());
 #ifdef RTM_PHASE_TIMING
