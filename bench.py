@@ -344,7 +344,7 @@ def finish(args, wl, world, ms, prof, n_rec, value, e2e_value, d2h, n_launches, 
         "kernel_share": shares,
         # side-stream kernels: their event interval runs from the partition's end until they get SM
         # slots beside the persistent fold (k_order_check, k_progress), or overlaps the partition
-        "side_stream": [k for k in ("k_events", "k_order_check", "k_progress") if k in shares],
+        "side_stream": [k for k in ("k_events", "k_order_check", "k_progress", "k_hang") if k in shares],
         "cpu_baseline": cpu,
         "e2e": ({"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 16 * n_rec, "d2h_bytes_per_step": d2h}
                 if e2e_value is not None else None),
