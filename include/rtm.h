@@ -219,7 +219,11 @@ rtm_status rtm_window_results(rtm_ctx *ctx, uint32_t first, uint32_t count, rtm_
 
 /* Two-phase form of rtm_window_reduce for callers that run the exchange themselves:
  * reduce_local computes this rank's results and packs them; *pack / *pack_bytes give the
- * device buffer to all-gather; rtm_merge consumes world*pack_bytes gathered bytes (device). */
+ * device buffer to all-gather; rtm_merge consumes world*pack_bytes gathered bytes (device).
+ * The pack is owned by the context and valid until its next reduce call; its size depends on
+ * n_windows, k, the pack size in buffers and the rank mode (MEAN adds each candidate's 64-bit
+ * order key), so every rank must use the same configuration.  Errors: RTM_E_INVALID (null
+ * arguments), RTM_E_STATE (rtm_merge without a preceding reduce_local), the reduce's own. */
 rtm_status rtm_window_reduce_local(rtm_ctx *ctx, const int64_t *t_end, uint32_t n_windows,
                                    const void **pack, uint64_t *pack_bytes);
 rtm_status rtm_merge(rtm_ctx *ctx, const void *gathered, uint32_t world, rtm_window_summary *out);
