@@ -103,7 +103,7 @@ typedef int (*rtm_allgather_fn)(void *user, const void *send, void *recv, uint64
 
 /* ---- configuration (≈ RegisterComponent + CreateProgressBar) ------------------ */
 typedef struct {
-  uint32_t n_buffers;               /* 1 .. 2^31-1                                             */
+  uint32_t n_buffers;               /* 1 .. 2^20 (1048576; larger: RTM_E_INVALID)              */
   uint32_t n_components;            /* 1 .. 2^20                                               */
   uint32_t n_kernels;               /* progress bars, 1 .. 2048                                */
   const uint32_t *buffer_owner;     /* host [n_buffers]: owning component id                   */
@@ -114,7 +114,8 @@ typedef struct {
   uint32_t k;                       /* top-k computed for every window, 1 .. 1024              */
   int32_t rank_mode;                /* RTM_RANK_PERCENT, RTM_RANK_SIZE or RTM_RANK_MEAN        */
   int32_t device;                   /* CUDA device ordinal                                     */
-  int32_t rank, world;              /* world == 1: single GPU; else this context is one shard  */
+  int32_t rank, world;              /* world == 1: single GPU; else this context is one shard;
+                                       world * k <= 8192 (merge candidates in shared memory)   */
   const uint8_t *owned_components;  /* host [n_components] or NULL (= all): components whose
                                        buffers and events this rank holds (ranking restricted) */
   rtm_allgather_fn allgather;       /* required when world > 1                                 */
@@ -222,8 +223,11 @@ rtm_status rtm_window_results(rtm_ctx *ctx, uint32_t first, uint32_t count, rtm_
  * device buffer to all-gather; rtm_merge consumes world*pack_bytes gathered bytes (device).
  * The pack is owned by the context and valid until its next reduce call; its size depends on
  * n_windows, k, the pack size in buffers and the rank mode (MEAN adds each candidate's 64-bit
- * order key), so every rank must use the same configuration.  Errors: RTM_E_INVALID (null
- * arguments), RTM_E_STATE (rtm_merge without a preceding reduce_local), the reduce's own. */
+ * order key), so every rank must use the same configuration.  Between a successful
+ * reduce_local and its rtm_merge the context is merge-pending: another reduce (local or not)
+ * and rtm_watch return RTM_E_STATE (no state change); rtm_reset clears the pending merge and
+ * the call's effects.  Errors: RTM_E_INVALID (null arguments), RTM_E_STATE (rtm_merge without
+ * a preceding reduce_local, or a second reduce while merge-pending), the reduce's own. */
 rtm_status rtm_window_reduce_local(rtm_ctx *ctx, const int64_t *t_end, uint32_t n_windows,
                                    const void **pack, uint64_t *pack_bytes);
 rtm_status rtm_merge(rtm_ctx *ctx, const void *gathered, uint32_t world, rtm_window_summary *out);
@@ -264,7 +268,8 @@ typedef struct {
 } rtm_watch_point;                  /* 40 B */
 /* Replace the watched set by buffer_ids[0..n) (n <= RTM_WATCH_MAX, distinct, < n_buffers;
  * global ids with a rank-local numbering) and clear every ring; n = 0 stops watching.
- * RTM_E_INVALID (no state change) for n > RTM_WATCH_MAX, duplicates or out-of-range ids. */
+ * RTM_E_INVALID (no state change) for n > RTM_WATCH_MAX, duplicates or out-of-range ids;
+ * RTM_E_STATE while a merge is pending (rtm_window_reduce_local without rtm_merge). */
 rtm_status rtm_watch(rtm_ctx *ctx, const uint32_t *buffer_ids, uint32_t n);
 /* The ring of watched slot `slot` (order given to rtm_watch), oldest point first:
  * out[RTM_WATCH_POINTS] (host) receives min(points so far, RTM_WATCH_POINTS) points,

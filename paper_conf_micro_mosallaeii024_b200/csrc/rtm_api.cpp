@@ -61,6 +61,7 @@ struct rtm_ctx {
   std::vector<uint32_t> link_off, link_dst;  // component connection graph (CSR by source)
   // value monitor: watched ids (as given), their local ids (~0: not on this rank), rings
   std::vector<uint32_t> gid_h;  // host copy of the global ids (rank-local numbering)
+  std::vector<uint8_t> elig_h;  // host copy of elig (buffer owned by this rank)
   uint32_t n_watch = 0;
   uint32_t watch_ids[RTM_WATCH_MAX] = {0}, watch_local[RTM_WATCH_MAX] = {0};
   std::vector<rtm_watch_point> ring[RTM_WATCH_MAX];
@@ -71,7 +72,8 @@ struct rtm_ctx {
   DevBuf carry[2];
   int cur = 0;
   DevBuf run[2], kstart, kend, cstart, cend, flags;
-  uint32_t epoch = 1;
+  uint32_t epoch = 1;        // look-back flag value of the current / last call (never 0)
+  bool merge_pending = false;  // rtm_window_reduce_local done, rtm_merge not yet
   int64_t t_prev;
   int sticky = 0;
   // pending stream
@@ -253,6 +255,7 @@ rtm_status zero_state(rtm_ctx *c) {
   c->cur = 0;
   c->t_prev = c->t0;
   c->have = false;
+  c->merge_pending = false;
   c->W = 0;
   c->s_dev.clear();
   c->e_dev.clear();
@@ -324,6 +327,7 @@ void set_result_ptrs(rtm_ctx *c, uint32_t W, Params &p) {
 
 rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p) {
   if (c->sticky) return (rtm_status)c->sticky;
+  if (c->merge_pending) return RTM_E_STATE;  // the previous local reduce awaits rtm_merge
   if (!t_end || W == 0) return RTM_E_INVALID;
   if (t_end[0] < c->t_prev) return RTM_E_INVALID;
   if (t_end[0] - c->t_prev >= kMaxWindowLen) return RTM_E_INVALID;
@@ -358,6 +362,10 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.klive = (const uint8_t *)c->klive.p;
   p.all_live = std::find(c->klive_h.begin(), c->klive_h.end(), (uint8_t)0) == c->klive_h.end();
   p.rcp = (const unsigned long long *)c->rcp.p; p.elig_ids = (const uint32_t *)c->elig_ids.p; p.n_elig = c->n_elig;
+  // A fresh look-back epoch for every call, taken before any kernel runs: a call that failed
+  // after its fold published flags (order error, exchange error) must not leave flags that
+  // the next call would read as already published.
+  c->epoch = c->epoch == 0xFFFFFFFFu ? 1u : c->epoch + 1u;
   p.W = W; p.epoch = c->epoch;
   p.narrow = 1;
   for (uint32_t w = 0; w < W; ++w)
@@ -460,8 +468,6 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   // concurrent kernel competes with the issue-bound fold.  Otherwise: a side stream, overlapped
   // with the partition and the fold, joined before the kernels that read the event outputs.
   p.fuse_events = partition_fuses_events(p.nbins, nts) ? 1 : 0;
-  static const int xp = getenv("RTM_XP") ? atoi(getenv("RTM_XP")) : 0;
-  p.xp = xp;
   if (!p.fuse_events) {
     CK(cudaEventRecord(c->ev_fork, c->st));
     CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
@@ -477,7 +483,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   // The order check (tile metadata) and the progress bars (event counts) do not read the fold's
   // outputs: on the side stream, beside the fold (after the event kernel when it runs there);
   // joined before the top-k.  One-window streaming calls: -13 us of dependent launches.
-  static const bool side = !getenv("RTM_NO_SIDE_TAIL");  // A/B switch
+  constexpr bool side = true;  // measured: C2 step 1.575 -> 1.556 ms
   if (side) {
     CK(cudaEventRecord(c->ev_fork, c->st));
     CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
@@ -495,7 +501,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   // the hang flags (fold's anyfull + event activity bits) and the top-k (fold's last levels) are
   // independent: the hang kernel on the side stream beside the top-k (the waits above are already
   // enqueued, so the fork / join events can be recorded again)
-  static const bool side_hang = !getenv("RTM_NO_SIDE_HANG");  // A/B switch
+  constexpr bool side_hang = true;  // measured: C2 step 1.559 -> 1.552 ms
   if (side_hang) {
     CK(cudaEventRecord(c->ev_fork, c->st));
     CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
@@ -584,7 +590,7 @@ rtm_status finish(rtm_ctx *c, const int64_t *t_end, uint32_t W, rtm_window_summa
   if (out) memcpy(out, c->sum.data(), Wn * sizeof(rtm_window_summary));
   c->t_prev = t_end[W - 1];
   c->cur ^= 1;
-  c->epoch = c->epoch == 0xFFFFFFFFu ? 1u : c->epoch + 1u;
+  c->merge_pending = false;
   c->have = true;
   c->W = W;
   c->s_dev.clear();
@@ -637,6 +643,7 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
         return RTM_E_INVALID;
   }
   if (cfg->pack_buffers && cfg->pack_buffers < cfg->n_buffers) return RTM_E_INVALID;
+  if (cfg->world > 1 && !merge_fits(cfg->world, cfg->k)) return RTM_E_INVALID;  // merge candidates in smem
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || cfg->device < 0 || cfg->device >= ndev) {
     cudaGetLastError();
@@ -670,7 +677,6 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   // before the persistent fold's CTAs, which would otherwise hold every SM until the fold ends
   int prio_lo = 0, prio_hi = 0;
   cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
-  if (getenv("RTM_SIDE_PRIO_OFF")) prio_hi = prio_lo;  // A/B switch
   if (cudaStreamCreateWithPriority(&c->st2, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess) {
@@ -708,6 +714,7 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
     if (elig[b]) elig_ids.push_back(b);
   }
   c->n_elig = (uint32_t)elig_ids.size();
+  c->elig_h = elig;
   std::vector<unsigned long long> rcp(65536, 0);
   for (uint32_t cc = 2; cc < 65536; ++cc) rcp[cc] = (1ull << 48) / cc;  // c == 1: only l == 0 < c
   if (cudaMemcpy(c->rcp.p, rcp.data(), 65536 * 8, cudaMemcpyHostToDevice) != cudaSuccess ||
@@ -826,6 +833,7 @@ rtm_status rtm_topk_persistence(rtm_ctx *c, uint32_t first, uint32_t count, uint
 
 rtm_status rtm_watch(rtm_ctx *c, const uint32_t *ids, uint32_t n) {
   if (!c || n > RTM_WATCH_MAX || (n && !ids)) return RTM_E_INVALID;
+  if (c->merge_pending) return RTM_E_STATE;  // the pending merge copies results in the frozen layout
   const uint32_t space = c->gid.p ? c->n_global : c->nb;
   for (uint32_t q = 0; q < n; ++q) {
     if (ids[q] >= space) return RTM_E_INVALID;
@@ -834,6 +842,7 @@ rtm_status rtm_watch(rtm_ctx *c, const uint32_t *ids, uint32_t n) {
   }
   for (uint32_t q = 0; q < n; ++q) {
     uint32_t loc = ids[q];
+    if (!c->gid.p && !c->elig_h.empty() && !c->elig_h[loc]) loc = 0xFFFFFFFFu;  // owned by another rank
     if (c->gid.p) {  // rank-local numbering: the local buffer with this global id, if any
       auto it = std::lower_bound(c->gid_h.begin(), c->gid_h.end(), ids[q]);
       loc = (it != c->gid_h.end() && *it == ids[q]) ? (uint32_t)(it - c->gid_h.begin()) : 0xFFFFFFFFu;
@@ -905,17 +914,19 @@ rtm_status rtm_window_reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t n_
   CK(cudaStreamSynchronize(c->st));
   *pack = c->pack.p;
   *pack_bytes_out = pb;
-  // remember the call for rtm_merge
+  // remember the call for rtm_merge; no other reduce (and no rtm_watch, which would change the
+  // results layout) until it runs
   c->t_end_h.assign(t_end, t_end + n_windows);
   c->W = n_windows;
   c->have = false;
+  c->merge_pending = true;
   return RTM_OK;
 }
 
 rtm_status rtm_merge(rtm_ctx *c, const void *gathered, uint32_t world, rtm_window_summary *out) {
   if (!c || !gathered || world == 0) return RTM_E_INVALID;
   if (c->sticky) return (rtm_status)c->sticky;
-  if (c->t_end_h.empty() || c->have) return RTM_E_STATE;
+  if (!c->merge_pending || c->t_end_h.empty() || c->have) return RTM_E_STATE;
   CK(cudaSetDevice(c->device));
   const uint32_t W = (uint32_t)c->t_end_h.size();
   Params p;

@@ -117,7 +117,6 @@ struct Params {
   uint32_t *hung;            // [W * ncw]
   uint32_t *unit_ctr;        // [0] fold units dequeued, [1] partition tiles, [2] fused event tiles claimed
   int32_t fuse_events;       // the persistent partition also runs the event tiles (K3 in K1)
-  int32_t xp;                // experiment switch (env RTM_XP, bit mask; A/B runs only, 0 = product path)
   uint32_t *status;          // bit0 sample order, bit1 event order
   const uint16_t *carry_in;  // [nb]
   uint16_t *carry_out;       // [nb]
@@ -164,6 +163,7 @@ void launch_persist(const Params &p, cudaStream_t st);
 uint64_t pack_bytes(const Params &p);
 void launch_pack(const Params &p, void *pack, cudaStream_t st);
 void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStream_t st);
+bool merge_fits(uint32_t world, uint32_t k);  // world * k candidates fit the merge's shared memory
 void launch_scatter_bstat(const Params &p, cudaStream_t st);  // gid set, world == 1
 unsigned long long kernel_launches();  // kernels launched by this library in this process
 

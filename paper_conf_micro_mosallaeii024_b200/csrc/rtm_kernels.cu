@@ -623,12 +623,11 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
   } while (0)
 #endif
 
-// STAGED: after the tile's barrier the warps permute their entries into the first half of the raw
-// staging (shared memory), a second barrier, then warps 0-3 copy the tile out with coalesced
-// 16-byte stores and only then prefetch their next raw records (named barrier among themselves);
-// warps 4-7 prefetch early as in the direct variant.  Direct: every lane stores its entries
-// straight to global memory (8-byte stores scattered over the tile's bins).
-template <bool STAGED>
+// After the tile's barrier the warps permute their entries into the first half of the raw staging
+// (shared memory), a second barrier, then warps 0-3 copy the tile out with coalesced 16-byte stores
+// and only then prefetch their next raw records (named barrier among themselves); warps 4-7
+// prefetch before the first barrier (measured 813 -> 692 us on C2 against direct 8-byte scatter
+// stores from every lane, which touched 32 sectors per store instruction).
 __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ K1WarpSum wsum[2][kK1Warps];
@@ -766,7 +765,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     // the next tile's records stream into the slot while this tile is published and written out
     cp_async_wait_all();
     __syncwarp();
-    const bool early = !STAGED || warp >= kK1Warps / 2;  // slots outside the staged half
+    const bool early = warp >= kK1Warps / 2;  // slots outside the staged half
     if (early) {
       if (nxt != ~0u) prefetch_raw(dsm[par ^ 1]);
       cp_async_commit();
@@ -774,8 +773,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     k1_publish(wsum[par], first, last, has, viol, kept);
     __syncthreads();  // B1 (the only CTA barrier per tile): summaries + bin totals of this tile
     PTM(4);
-    if (!STAGED && warp == 0) k1_tile_summary(p, t, wsum[par]);
-    if (STAGED) {
+    {
       unsigned total = 0;
       if (is_win) {
         total = k1_bin_bases(p, tile, wt, myb);
@@ -799,14 +797,6 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
         asm volatile("bar.sync 1, %0;" ::"n"(kK1Threads / 2) : "memory");  // staged half read out
         if (nxt != ~0u) prefetch_raw(dsm[par ^ 1]);
         cp_async_commit();
-      }
-    } else if (is_win) {
-      k1_bin_bases(p, tile, wt, myb);
-      unsigned long long *dst = p.stage + (size_t)tile * kTileS;
-#pragma unroll
-      for (int k = 0; k < kPerLane; ++k) {
-        const unsigned key = kp[k] >> 16;
-        if (key != kNoKey) dst[myb[key] + (kp[k] & 0xFFFFu)] = e[k];
       }
     }
     PTM(5);
@@ -936,8 +926,7 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
   if (warp == 0) k1_tile_summary(p, t, wsum);
   if (!is_win) return;
   __shared__ unsigned bb_scratch[32];
-  const unsigned total = (p.xp & 32) ? k1_bin_bases(p, tile, wt, myb)  // A/B: per-warp bases
-                                     : k1_bin_bases_cta(p, tile, wt, wb, bb_scratch);
+  const unsigned total = k1_bin_bases_cta(p, tile, wt, wb, bb_scratch);
 #pragma unroll
   for (int k = 0; k < kPerLane; ++k) {
     const unsigned key = kp[k] >> 16;
@@ -1469,7 +1458,7 @@ __global__ void __launch_bounds__(kTopkThreads) k_topk(Params p) {
     const uint4 *lv4 = reinterpret_cast<const uint4 *>(lv + slo);  // slices start at multiples of 8
     const uint4 *cp4 = reinterpret_cast<const uint4 *>(p.cap + slo);
     uint4 *k4 = reinterpret_cast<uint4 *>(keys);
-#pragma unroll 2
+#pragma unroll 1  // unroll 2 spilled 12 B (ptxas) at the 128-register cap of 512 threads
     for (unsigned g = threadIdx.x; g < ne / 8; g += blockDim.x) {
       const uint4 L = lv4[g], C = __ldg(cp4 + g);
       const unsigned lw[4] = {L.x, L.y, L.z, L.w}, cw[4] = {C.x, C.y, C.z, C.w};
@@ -2227,13 +2216,12 @@ void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   const size_t sm = partition_smem_bytes(p.nbins, p.nb);
   if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM (capacity table loaded once)
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm<false>, kK1Threads, sm);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm, kK1Threads, sm);
     if (per_sm < 1) per_sm = 1;
     unsigned grid = (unsigned)(n_sms * per_sm);
     const unsigned work = p.n_tiles_s + (p.fuse_events ? p.n_tiles_e : 0u);
     if (grid > work) grid = work;
-    if (p.xp & 4) { k_partition_lm<false><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }  // A/B: direct
-    else { k_partition_lm<true><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
+    { k_partition_lm<<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
   } else {
     { k_partition_mx<<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
   }
@@ -2255,8 +2243,8 @@ void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
   const unsigned need = (units + kFoldWarps - 1) / kFoldWarps;
   if (grid > need) grid = need;
   if (grid == 0) grid = 1;
-  // sparse units: fewer than 512 kept samples per (window, bin) on average (RTM_XP=512: dense)
-  const bool sparse = !(p.xp & 512) && p.ns < (uint64_t)512 * units;
+  // sparse units: fewer than 512 kept samples per (window, bin) on average
+  const bool sparse = p.ns < (uint64_t)512 * units;
   if (p.narrow && sparse) { k_fold<true, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else if (p.narrow) { k_fold<true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else if (sparse) { k_fold<false, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
@@ -2325,9 +2313,7 @@ void configure_kernels_once() {
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 128 || done[dev]) return;
   done[dev] = true;
-  cudaFuncSetAttribute(k_partition_lm<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                       (int)k1_smem_lm(kLmMaxBins, kLmMaxBins * kBin));
-  cudaFuncSetAttribute(k_partition_lm<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  cudaFuncSetAttribute(k_partition_lm, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)k1_smem_lm(kLmMaxBins, kLmMaxBins * kBin));
   cudaFuncSetAttribute(k_partition_mx, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
   cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
@@ -2366,6 +2352,13 @@ void launch_pack(const Params &p, void *pack, cudaStream_t st) {
 void launch_scatter_bstat(const Params &p, cudaStream_t st) {
   const unsigned blocks = (p.nb + 255) / 256;
   { k_scatter_bstat<<<blocks < 1184 ? blocks : 1184, 256, 0, st>>>(p); count_launch(); }
+}
+
+// k_merge_windows holds next_pow2(world * k) candidates of 20 B in shared memory (opt-in 227 KB)
+bool merge_fits(uint32_t world, uint32_t k) {
+  uint64_t P = 1;
+  while (P < (uint64_t)world * k) P <<= 1;
+  return P * 20 <= 227ull * 1024;
 }
 
 void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStream_t st) {

@@ -41,11 +41,12 @@ def _host_slice(dev, lo, hi, dtype):
     return dev[lo * 16:hi * 16].cpu().numpy().view(dtype)
 
 
-def run_config(wl, *, batch, topk_windows=None):
+def run_config(wl, *, batch, topk_windows=None, rank_mode=0):
     """GPU: one call over all windows.  Oracle: batches of `batch` windows.  Returns the
-    per-window hang lists of the oracle for property checks."""
+    per-window hang lists of the oracle for property checks.  When every window's top-k is
+    compared, the windows-in-top-k counter (persistence) is compared too."""
     owner, cap, tot = gen.registry(wl)
-    kw = dict(t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k)
+    kw = dict(t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k, rank_mode=rank_mode)
     ds, de = _device_trace(wl)
     # the device generator writes the same records as the host one (spot check)
     idx = np.random.default_rng(1).integers(0, wl.n_samples, 2048)
@@ -60,6 +61,7 @@ def run_config(wl, *, batch, topk_windows=None):
     stats = mon.buffer_stats()
     _, comps = mon.progress(wl.n_windows - 1, comps=True)
     ghung = [mon.hang_check(w) for w in range(wl.n_windows)]
+    gpersist = mon.topk_persistence()
     del mon
 
     orc = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw)
@@ -93,6 +95,8 @@ def run_config(wl, *, batch, topk_windows=None):
             assert np.array_equal(stats["mean_occ"], rs["mean_occ"])
             for f in ("started", "finished", "in_flight"):
                 assert np.array_equal(comps[f], ref["comps"][f]), f
+    if topk_windows is None:
+        assert np.array_equal(gpersist, orc.persistence())
     return hung_ref
 
 
@@ -117,9 +121,11 @@ def test_c3_small_deadlock_parity():
     check_deadlock_flags(gen.C3_SMALL, hung)
 
 
-def test_c4_small_zipf_parity():
-    wl = gen.C4_SMALL
-    run_config(wl, batch=5)
+@pytest.mark.parametrize("rank_mode", [0, 1, 2])
+def test_c4_small_zipf_parity(rank_mode):
+    """C4's shape (2^20 buffers, Zipf 0.99, k = 1024) in every rank mode: MEAN ranks 1M 64-bit
+    order keys per window (k_topk64's uncompacted large-n path)."""
+    run_config(gen.C4_SMALL, batch=5, rank_mode=rank_mode)
 
 
 @pytest.mark.slow

@@ -2,7 +2,9 @@
 (gloo: the one-GPU box has no second device for NCCL, both ranks share cuda:0), owner-component
 sharding, `Monitor.window_reduce` = rtm_window_reduce_local -> all_gather of the packs -> rtm_merge.
 Every rank's merged results must equal the whole-trace oracle, in rank modes
-PERCENT and MEAN (the pack carries MEAN's 64-bit order keys)."""
+PERCENT and MEAN (the pack carries MEAN's 64-bit order keys), across two calls with a progress bar
+destroyed and another updated in between; the windows-in-top-k counter and the value monitor's
+rings (filled on the owning rank only) are compared too."""
 from __future__ import annotations
 
 import os
@@ -45,14 +47,42 @@ def _worker(rank, world, port, mode, result_path):
         wl = gen.C1.scaled("C1-dist", n_samples=200_000, n_events=20_000, n_windows=6)
         owner, cap, tot = gen.registry(wl)
         kw = dict(t0=wl.t0, hang_windows=2, k=wl.k, rank_mode=mode)
-        ref = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw).reduce(
-            gen.samples(wl), gen.events(wl), wl.t_end())
+        orc = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw)
         owned = (np.arange(wl.n_components) % world == rank).astype(np.uint8)
         mon = Monitor(owner, cap, tot, n_components=wl.n_components, rank=rank, world=world,
                       owned_components=owned, **kw)
-        mon.ingest(_dev(gen.samples(wl, shard=(world, rank))), _dev(gen.events(wl, shard=(world, rank))))
-        mon.window_reduce(wl.t_end())
-        assert_same(mon.results(), ref, mon)
+        watched = [0, 5, 17, 998]  # owners 0, 1, 4, 249: both ranks own some
+        mon.watch(watched)
+        s_all, e_all = gen.samples(wl), gen.events(wl)
+        s_sh, e_sh = gen.samples(wl, shard=(world, rank)), gen.events(wl, shard=(world, rank))
+        t_end = wl.t_end()
+        rows = []
+        for lo, hi in ((0, 2), (2, 6)):
+            if lo == 2:  # dynamic progress bars between calls, the same on every rank
+                for x in (orc, mon):
+                    x.bar_destroy(0)
+                    x.bar_update(1, 4321)
+            sl = slice(wl.index_at("samples", wl.t_begin(lo)), wl.index_at("samples", wl.t_begin(hi)))
+            el = slice(wl.index_at("events", wl.t_begin(lo)), wl.index_at("events", wl.t_begin(hi)))
+            ref = orc.reduce(s_all[sl], e_all[el], t_end[lo:hi], want_all_stats=True)
+            rows.append(ref["all_stats"])
+            ss = s_sh[(s_sh["ts"] >= wl.t_begin(lo)) & (s_sh["ts"] < wl.t_begin(hi))]
+            es = e_sh[(e_sh["ts"] >= wl.t_begin(lo)) & (e_sh["ts"] < wl.t_begin(hi))]
+            mon.ingest(_dev(ss), _dev(es))
+            mon.window_reduce(t_end[lo:hi])
+            assert_same(mon.results(), ref, mon)
+        # windows-in-top-k counter, counted from the merged lists
+        assert np.array_equal(mon.topk_persistence(), orc.persistence())
+        # value monitor: the owner's ring equals the oracle's per-window table, others stay empty
+        A = np.concatenate(rows)
+        for q, b in enumerate(watched):
+            ser = mon.watch_series(q)
+            if owned[owner[b]]:
+                assert np.array_equal(ser["t_end"], t_end), b
+                for f in ("integral", "last", "max", "min", "capacity", "n_samples", "mean_occ"):
+                    assert np.array_equal(ser[f], A[:, b][f]), (b, f)
+            else:
+                assert len(ser) == 0, b
         msg = "ok"
         dist.destroy_process_group()
     except Exception:  # noqa: BLE001 - reported through the result file

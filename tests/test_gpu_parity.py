@@ -236,8 +236,8 @@ def test_virtual_shards_merge_equals_whole(mode, k):
     wl = gen.C1.scaled("C1-vshard", n_samples=200_000, n_events=20_000, n_windows=6)
     owner, cap, tot = gen.registry(wl)
     kw = dict(t0=wl.t0, hang_windows=2, k=k or wl.k, rank_mode=mode)
-    ref = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw).reduce(gen.samples(wl), gen.events(wl),
-                                                                                   wl.t_end())
+    orc = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw)
+    ref = orc.reduce(gen.samples(wl), gen.events(wl), wl.t_end())
     G = 3
     mons, packs = [], []
     for r in range(G):
@@ -261,11 +261,15 @@ def test_virtual_shards_merge_equals_whole(mode, k):
         got = m.results()
         assert np.array_equal(got["summary"], summ)
         assert_same(got, ref, m)
+        assert np.array_equal(m.topk_persistence(), orc.persistence())  # counted from the merged lists
 
 
 @pytest.mark.slow
-def test_c2_full_size_parity():
-    """BASELINE configs[1] at full size, in the launch configuration bench.py times."""
+@pytest.mark.parametrize("rank_mode", [0, 1, 2])
+def test_c2_full_size_parity(rank_mode):
+    """BASELINE configs[1] at full size, in the launch configuration bench.py times, in every
+    rank mode (PERCENT is the bench's; SIZE and MEAN rank the same 20480 buffers by level and by
+    64-bit mean-occupancy keys); the persistence counter too."""
     wl = gen.C2
     owner, cap, tot = gen.registry(wl)
     ds = torch.empty(wl.n_samples * 16, dtype=torch.uint8, device="cuda")
@@ -273,7 +277,7 @@ def test_c2_full_size_parity():
     gen.fill_device("samples", wl, ds.data_ptr(), 0, wl.n_samples)
     gen.fill_device("events", wl, de.data_ptr(), 0, wl.n_events)
     torch.cuda.synchronize()
-    kw = dict(t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k)
+    kw = dict(t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k, rank_mode=rank_mode)
     mon = Monitor(owner, cap, tot, n_components=wl.n_components, **kw)
     mon.ingest(ds, de)
     got = mon.window_reduce(wl.t_end())
@@ -283,8 +287,10 @@ def test_c2_full_size_parity():
     idx = np.random.default_rng(0).integers(0, wl.n_samples, 4096)
     assert np.array_equal(ds.view(-1, 16)[torch.from_numpy(idx).cuda()].cpu().numpy().view(gen.SAMPLE_DTYPE).ravel(),
                           s[idx])
-    ref = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw).reduce(s, e, wl.t_end())
+    orc = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw)
+    ref = orc.reduce(s, e, wl.t_end())
     assert_same(got, ref, mon)
+    assert np.array_equal(mon.topk_persistence(), orc.persistence())
 
 
 @pytest.mark.parametrize("n_top", [0, 10, 63, 64, 65, 200])
@@ -432,8 +438,8 @@ def test_rank_local_numbering_shards_merge_equals_whole(mode, k):
     wl = gen.C1.scaled("C1-lshard", n_samples=200_000, n_events=20_000, n_windows=6)
     owner, cap, tot = gen.registry(wl)
     kw = dict(t0=wl.t0, hang_windows=2, k=k or wl.k, rank_mode=mode)
-    ref = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw).reduce(gen.samples(wl), gen.events(wl),
-                                                                                   wl.t_end())
+    orc = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw)
+    ref = orc.reduce(gen.samples(wl), gen.events(wl), wl.t_end())
     G = 3
     gids = [np.nonzero(owner % G == r)[0].astype(np.uint32) for r in range(G)]
     pack_nb = max(len(g) for g in gids)
@@ -465,6 +471,7 @@ def test_rank_local_numbering_shards_merge_equals_whole(mode, k):
         got = m.results()
         assert np.array_equal(got["summary"], summ)
         assert_same(got, ref, m)
+        assert np.array_equal(m.topk_persistence(), orc.persistence())  # counted from the merged lists
 
 
 def test_rank_local_numbering_rejects_unsorted_ids():
@@ -743,3 +750,72 @@ def test_limits_max_sizes_wide_windows_and_hot_buffer():
         mon.ingest(_dev(s), _dev(e))
         got = mon.window_reduce(np.array(ends, np.int64))
         assert_same(got, ref, mon)  # window 3's digest covers the hot buffer's > 65535-sample count
+
+
+def test_order_error_then_reset_then_multiwindow_lookback():
+    """A multi-window call that fails with RTM_E_ORDER has already run its fold (which publishes
+    look-back flags); after rtm_reset the next multi-window call must not read those flags as
+    published (every call takes a fresh look-back epoch): its results equal the oracle's."""
+    wl = gen.C1.scaled("C1-epoch", n_samples=400_000, n_events=40_000, n_windows=8)
+    owner, cap, tot = gen.registry(wl)
+    s, e = gen.samples(wl), gen.events(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    bad = s.copy()
+    j = len(bad) - 10  # one inversion near the end: every window's fold still runs
+    bad[j], bad[j + 1] = bad[j + 1].copy(), bad[j].copy()
+    bad["ts"][j] += 3
+    mon.ingest(_dev(bad), _dev(e))
+    with pytest.raises(RTMError) as ei:
+        mon.window_reduce(wl.t_end())
+    assert ei.value.code == N.RTM_E_ORDER
+    mon.reset()
+    for _ in range(2):  # the same multi-window call twice from a reset state
+        ref = orc.reduce(s, e, wl.t_end())
+        mon.ingest(_dev(s), _dev(e))
+        assert_same(mon.window_reduce(wl.t_end()), ref, mon)
+        mon.reset()
+        orc.reset()
+
+
+def test_merge_pending_state_and_world_k_limit():
+    """rtm_window_reduce_local leaves the context merge-pending: a second reduce and rtm_watch
+    return RTM_E_STATE (no state change) until rtm_merge; rtm_reset clears it.  rtm_create
+    rejects world * k above what the merge holds in shared memory."""
+    import ctypes
+
+    from paper_conf_micro_mosallaeii024_b200 import _copy_from_ptr
+
+    wl = gen.C1.scaled("C1-pending", n_samples=50_000, n_events=5_000, n_windows=3)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    with pytest.raises(RTMError) as ei:
+        Monitor(owner, cap, tot, n_components=wl.n_components, rank=0, world=16, k=1024,
+                owned_components=np.ones(wl.n_components, np.uint8), t0=wl.t0)
+    assert ei.value.code == N.RTM_E_INVALID
+    orc = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw)
+    ref = orc.reduce(gen.samples(wl), gen.events(wl), wl.t_end())
+    m = Monitor(owner, cap, tot, n_components=wl.n_components, rank=0, world=1, **kw)
+    ends = np.ascontiguousarray(wl.t_end())
+    for attempt in range(2):
+        m.ingest(_dev(gen.samples(wl)), _dev(gen.events(wl)))
+        pack, nbytes = ctypes.c_void_p(), ctypes.c_uint64()
+        N.check(N.lib().rtm_window_reduce_local(m._h, ends.ctypes.data, len(ends), ctypes.byref(pack),
+                                                ctypes.byref(nbytes)), "local")
+        rc = N.lib().rtm_window_reduce_local(m._h, ends.ctypes.data, len(ends), ctypes.byref(pack),
+                                             ctypes.byref(nbytes))
+        assert rc == N.RTM_E_STATE
+        with pytest.raises(RTMError) as ei:
+            m.watch([1])
+        assert ei.value.code == N.RTM_E_STATE
+        if attempt == 0:  # abandon the exchange: reset clears the pending merge
+            m.reset()
+            continue
+        t = torch.empty(int(nbytes.value), dtype=torch.uint8, device="cuda")
+        _copy_from_ptr(t, pack.value, int(nbytes.value))
+        torch.cuda.synchronize()
+        summ = np.zeros(wl.n_windows, N.SUMMARY_DTYPE)
+        N.check(N.lib().rtm_merge(m._h, t.data_ptr(), 1, summ.ctypes.data), "merge")
+        m.W = wl.n_windows
+        assert_same(m.results(), ref, m)
+    assert N.lib().rtm_merge(m._h, t.data_ptr(), 1, summ.ctypes.data) == N.RTM_E_STATE
