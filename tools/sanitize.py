@@ -1,0 +1,67 @@
+"""Workload for compute-sanitizer (SURVEY.md §4 "Sanitizers", §5): a C1-shaped trace through the
+C-ABI in the launch configurations the tests use — one multi-window call (partition, fold with
+look-back, top-k, hang, progress), single-window calls (top-k slices + merge), rank modes SIZE and
+MEAN, invalid records — every result compared with the oracle so a silent corruption also fails.
+
+    compute-sanitizer --tool memcheck python tools/sanitize.py [--small]
+"""
+from __future__ import annotations
+
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import gen  # noqa: E402
+import oracle  # noqa: E402
+from paper_conf_micro_mosallaeii024_b200 import Monitor  # noqa: E402
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a).view(np.uint8)).cuda()
+
+
+def check(got, ref, n_windows):
+    for f in ("n_samples", "n_events", "n_dropped", "digest", "n_touched", "n_hung"):
+        assert np.array_equal(got["summary"][f], ref["summary"][f]), f
+    for w in range(n_windows):
+        n = int(ref["topk_n"][w])
+        assert np.array_equal(got["topk"][w][:n], ref["topk"][w][:n]), w
+    for f in ("started", "finished", "in_flight"):
+        assert np.array_equal(got["progress"][f], ref["progress"][f]), f
+
+
+def main():
+    small = "--small" in sys.argv
+    ns = 60_000 if small else 300_000
+    base = gen.C1_INVALID.scaled("C1-sanitize", n_samples=ns, n_events=ns // 10, n_windows=6)
+    owner, cap, tot = gen.registry(base)
+    s, e = gen.samples(base), gen.events(base)
+    t_end = base.t_end()
+    for mode in (0, 1, 2):
+        kw = dict(t0=base.t0, hang_windows=2, k=base.k, rank_mode=mode)
+        orc = oracle.Oracle(owner, cap, tot, n_components=base.n_components, **kw)
+        mon = Monitor(owner, cap, tot, n_components=base.n_components, **kw)
+        # one multi-window call, then one window per call
+        ref = orc.reduce(s, e, t_end[:4])
+        lo_s, lo_e = base.index_at("samples", base.t_begin(4)), base.index_at("events", base.t_begin(4))
+        mon.ingest(_dev(s[:lo_s]), _dev(e[:lo_e]))
+        check(mon.window_reduce(t_end[:4]), ref, 4)
+        for w in (4, 5):
+            hs, he = base.index_at("samples", base.t_begin(w + 1)), base.index_at("events", base.t_begin(w + 1))
+            ref = orc.reduce(s[lo_s:hs], e[lo_e:he], t_end[w:w + 1])
+            mon.ingest(_dev(s[lo_s:hs]), _dev(e[lo_e:he]))
+            check(mon.window_reduce(t_end[w:w + 1]), ref, 1)
+            lo_s, lo_e = hs, he
+        mon.buffer_stats()
+        mon.close()
+    print("sanitize workload OK")
+
+
+if __name__ == "__main__":
+    main()
