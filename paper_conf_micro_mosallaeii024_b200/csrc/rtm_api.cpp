@@ -934,6 +934,7 @@ rtm_status rtm_merge(rtm_ctx *c, const void *gathered, uint32_t world, rtm_windo
   p.nb = c->nb; p.nc = c->nc; p.nk = c->nk; p.nbins = c->nbins; p.ncw = c->ncw; p.k = c->k;
   p.rank_mode = c->rank_mode; p.W = W;
   p.ktotal = (const int64_t *)c->ktotal.p; p.rcp = (const unsigned long long *)c->rcp.p;
+  p.klive = (const uint8_t *)c->klive.p;
   set_result_ptrs(c, W, p);
   p.hung = (uint32_t *)c->hung.p;
   p.comps = (rtm_component_tasks *)c->comps.p; p.bstat = (rtm_buffer_stat *)c->bstat.p;

@@ -1078,76 +1078,16 @@ __device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, b
   __syncwarp();
 }
 
-// SPARSE (few samples per unit: C3-C5 shapes): many of a unit's 256 buffers are untouched in
-// several consecutive windows, so the look-back walks several windows; it takes RTM_LB_STEP of
-// them per step (their flags waited for by as many lanes, all rows loaded before any is used),
-// dividing the dependent round trips.  A separate instantiation: the dense (C2) code is unchanged.
-template <bool NAR, bool SPARSE = false>
-__global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Params p) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  FoldSmem &S = reinterpret_cast<FoldSmem *>(smem)[threadIdx.x >> 5];
-  const int lane = threadIdx.x & 31;
-  const unsigned lt = lanemask_lt();
-  const unsigned n_units = p.W * p.nbins;
-  for (;;) {
-    unsigned u = 0;
-    if (lane == 0) u = atomicAdd(p.unit_ctr, 1u);
-    u = __shfl_sync(kFull, u, 0);
-    if (u >= n_units) break;
-    const unsigned w = u / p.nbins, bin = u % p.nbins;
-    const long long tb = p.T[w], te = p.T[w + 1];
-    const unsigned long long Wlen = (unsigned long long)(te - tb);
-    const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
-#pragma unroll
-    for (int i = 0; i < kBin / 32; ++i) {
-      S.st[lane + 32 * i] = make_uint4(0, 0, kUntouchedZ, 0);
-      S.hi[lane + 32 * i] = 0;
-    }
-    __syncwarp();
-    // ---- phase 1: the (tile, bin) segments of window w, flattened into one stream of chunks
-    for (unsigned tg = t_lo; tg < t_hi; tg += 32) {
-      unsigned seg_lo = 0, seg_len = 0;
-      if (tg + lane < t_hi) {
-        const uint16_t *o = p.soff + (size_t)(tg + lane) * (p.nbins + 1) + bin;
-        seg_lo = __ldg(o);
-        seg_len = (unsigned)__ldg(o + 1) - seg_lo;
-      }
-      unsigned pre = seg_len;  // inclusive prefix of segment lengths over lanes
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const unsigned y = __shfl_up_sync(kFull, pre, o);
-        if (lane >= o) pre += y;
-      }
-      const unsigned total = __shfl_sync(kFull, pre, 31);
-      // per-warp table of the NON-EMPTY segments (compacted, so their ends are strictly
-      // increasing): staging index of each segment minus its flattened start.  The segment of
-      // flattened position g is the number of segment ends <= g: per 32-position chunk, one
-      // OR-reduction marks the ends inside the chunk and each lane counts the marks at or below it.
-      const unsigned nonempty = __ballot_sync(kFull, seg_len != 0);
-      if (seg_len) S.seg_base[__popc(nonempty & lt)] = (tg + lane) * (unsigned)kTileS + seg_lo - (pre - seg_len);
-      const unsigned my_end = seg_len ? pre : 0xFFFFFFFFu;
-      const unsigned le = (2u << lane) - 1u;  // lanes <= this one
-      __syncwarp();
-      unsigned seg_before = 0;  // segments ending at or before the current chunk's first position
-      auto fetch = [&](unsigned c) -> unsigned long long {
-        const unsigned x = my_end - c;
-        const unsigned ends = __reduce_or_sync(kFull, x < 32u ? 1u << x : 0u);
-        const unsigned sgi = seg_before + __popc(ends & le);
-        seg_before += __popc(ends);
-        const unsigned g = c + lane;
-        if (g >= total) return 0ull;
-        return __ldcg(p.stage + (S.seg_base[sgi] + g));
-      };
-      // 2-deep software pipeline over the staging reads (measured on C2: depth 2 709 us, 3 715 us,
-      // 4 719 us, 6 727 us - deeper costs registers the chunk logic needs; depth 1: 863 us)
-      unsigned long long e0 = fetch(0), e1 = fetch(32);
-      for (unsigned c = 0; c < total; c += 32) {
-        const unsigned long long en = fetch(c + 64);
-        fold_chunk<NAR>(S, lane, lt, c + lane < total, e0, Wlen);
-        e0 = e1;
-        e1 = en;
-      }
-    }
+// Phase 2 of a fold unit (window w, bin), shared by both fold kernels: publish the window's last
+// levels (kSent: untouched) and the phase-1 flag, resolve the carry-in L_in by decoupled
+// look-back over earlier windows' published levels, finalize (integral, max / min with the
+// carry-in, full bits, digest, mean-occupancy keys, watched buffers, the last window's table).
+// S holds the unit's per-buffer phase-1 state: st (D, last | max << 16, min | n16 << 16), hi
+// (n_hi | ts0_hi << 16) and ts0 (offset of the buffer's first kept sample in the window).
+template <bool NAR, bool SPARSE, typename FS>
+__device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, unsigned bin,
+                                            unsigned long long Wlen, int lane) {
+  {
     // ---- publish this window's last levels (kSent: untouched) and the phase-1 flag
     const unsigned b_base = bin * kBin;
     uint16_t *lw = p.lastlvl + (size_t)w * p.nb;
@@ -1317,6 +1257,80 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
       if (touched) atomicAdd(p.win + WF_TOUCHED * p.W + w, (unsigned long long)touched);
     }
     __syncwarp();
+  }
+}
+
+// SPARSE (few samples per unit: C3-C5 shapes): many of a unit's 256 buffers are untouched in
+// several consecutive windows, so the look-back walks several windows; it takes RTM_LB_STEP of
+// them per step (their flags waited for by as many lanes, all rows loaded before any is used),
+// dividing the dependent round trips.  A separate instantiation: the dense (C2) code is unchanged.
+template <bool NAR, bool SPARSE = false>
+__global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Params p) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  FoldSmem &S = reinterpret_cast<FoldSmem *>(smem)[threadIdx.x >> 5];
+  const int lane = threadIdx.x & 31;
+  const unsigned lt = lanemask_lt();
+  const unsigned n_units = p.W * p.nbins;
+  for (;;) {
+    unsigned u = 0;
+    if (lane == 0) u = atomicAdd(p.unit_ctr, 1u);
+    u = __shfl_sync(kFull, u, 0);
+    if (u >= n_units) break;
+    const unsigned w = u / p.nbins, bin = u % p.nbins;
+    const long long tb = p.T[w], te = p.T[w + 1];
+    const unsigned long long Wlen = (unsigned long long)(te - tb);
+    const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
+#pragma unroll
+    for (int i = 0; i < kBin / 32; ++i) {
+      S.st[lane + 32 * i] = make_uint4(0, 0, kUntouchedZ, 0);
+      S.hi[lane + 32 * i] = 0;
+    }
+    __syncwarp();
+    // ---- phase 1: the (tile, bin) segments of window w, flattened into one stream of chunks
+    for (unsigned tg = t_lo; tg < t_hi; tg += 32) {
+      unsigned seg_lo = 0, seg_len = 0;
+      if (tg + lane < t_hi) {
+        const uint16_t *o = p.soff + (size_t)(tg + lane) * (p.nbins + 1) + bin;
+        seg_lo = __ldg(o);
+        seg_len = (unsigned)__ldg(o + 1) - seg_lo;
+      }
+      unsigned pre = seg_len;  // inclusive prefix of segment lengths over lanes
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned y = __shfl_up_sync(kFull, pre, o);
+        if (lane >= o) pre += y;
+      }
+      const unsigned total = __shfl_sync(kFull, pre, 31);
+      // per-warp table of the NON-EMPTY segments (compacted, so their ends are strictly
+      // increasing): staging index of each segment minus its flattened start.  The segment of
+      // flattened position g is the number of segment ends <= g: per 32-position chunk, one
+      // OR-reduction marks the ends inside the chunk and each lane counts the marks at or below it.
+      const unsigned nonempty = __ballot_sync(kFull, seg_len != 0);
+      if (seg_len) S.seg_base[__popc(nonempty & lt)] = (tg + lane) * (unsigned)kTileS + seg_lo - (pre - seg_len);
+      const unsigned my_end = seg_len ? pre : 0xFFFFFFFFu;
+      const unsigned le = (2u << lane) - 1u;  // lanes <= this one
+      __syncwarp();
+      unsigned seg_before = 0;  // segments ending at or before the current chunk's first position
+      auto fetch = [&](unsigned c) -> unsigned long long {
+        const unsigned x = my_end - c;
+        const unsigned ends = __reduce_or_sync(kFull, x < 32u ? 1u << x : 0u);
+        const unsigned sgi = seg_before + __popc(ends & le);
+        seg_before += __popc(ends);
+        const unsigned g = c + lane;
+        if (g >= total) return 0ull;
+        return __ldcg(p.stage + (S.seg_base[sgi] + g));
+      };
+      // 2-deep software pipeline over the staging reads (measured on C2: depth 2 709 us, 3 715 us,
+      // 4 719 us, 6 727 us - deeper costs registers the chunk logic needs; depth 1: 863 us)
+      unsigned long long e0 = fetch(0), e1 = fetch(32);
+      for (unsigned c = 0; c < total; c += 32) {
+        const unsigned long long en = fetch(c + 64);
+        fold_chunk<NAR>(S, lane, lt, c + lane < total, e0, Wlen);
+        e0 = e1;
+        e1 = en;
+      }
+    }
+    fold_finish<NAR, SPARSE>(p, S, w, bin, Wlen, lane);
   }
 }
 
@@ -2101,7 +2115,8 @@ __global__ void __launch_bounds__(256) k_merge_windows(Params p, const unsigned 
       E += o[2];
     }
     long long *o = p.prog + ((size_t)w * p.nk + k) * 5;
-    const long long total = p.ktotal[k];
+    const bool live = p.klive[k] != 0;  // a destroyed bar reads all zero (rtm_bar_destroy)
+    const long long total = live ? p.ktotal[k] : 0;
     o[0] = total; o[1] = S; o[2] = E; o[3] = S - E; o[4] = total - S;
   }
   for (unsigned q = threadIdx.x; q < p.ncw; q += blockDim.x) {

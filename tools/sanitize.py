@@ -48,8 +48,8 @@ def main():
         orc = oracle.Oracle(owner, cap, tot, n_components=base.n_components, **kw)
         mon = Monitor(owner, cap, tot, n_components=base.n_components, **kw)
         # one multi-window call, then one window per call
-        ref = orc.reduce(s, e, t_end[:4])
         lo_s, lo_e = base.index_at("samples", base.t_begin(4)), base.index_at("events", base.t_begin(4))
+        ref = orc.reduce(s[:lo_s], e[:lo_e], t_end[:4])
         mon.ingest(_dev(s[:lo_s]), _dev(e[:lo_e]))
         check(mon.window_reduce(t_end[:4]), ref, 4)
         for w in (4, 5):
