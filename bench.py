@@ -128,6 +128,77 @@ def cpu_reference_step(wl, n_windows_sample: int):
     return recs, dt
 
 
+def host_info():
+    """nproc, CPU model and RAM of the box the baseline ran on."""
+    model = None
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    ram = None
+    try:
+        for ln in open("/proc/meminfo"):
+            if ln.startswith("MemTotal"):
+                ram = round(int(ln.split()[1]) / 1024 / 1024, 1)
+                break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model, "ram_gib": ram}
+
+
+def _shard_worker(args):
+    """One shard of the sharded oracle baseline: owner components c % P == r."""
+    wl_name, n_win, P, r, barrier = args
+    import gen
+    import oracle
+
+    wl = gen.CONFIGS[wl_name]
+    ends = wl.t_end()[:n_win]
+    t_hi = int(ends[-1])
+    ns = min(wl.n_samples, int((t_hi - wl.t0) * wl.samples_per_tick) + 4)
+    ne = min(wl.n_events, int((t_hi - wl.t0) * wl.n_events // max(1, wl.ticks)) + 4)
+    s, e = gen.samples(wl, 0, ns, shard=(P, r)), gen.events(wl, 0, ne, shard=(P, r))
+    owner, cap, tot = gen.registry(wl)
+    owned = (np.arange(wl.n_components) % P == r).astype(np.uint8)
+    orc = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, t0=wl.t0, hang_windows=wl.hang_windows,
+                        k=wl.k, owned=owned)
+    barrier.wait()  # every shard starts together: the parallel run shares the host's memory system
+    t0 = time.perf_counter()
+    out = orc.reduce(s, e, ends, want_hung=False)
+    dt = time.perf_counter() - t0
+    assert out["rc"] == 0
+    return dt, out
+
+
+def cpu_sharded_step(wl, n_win, P):
+    """The oracle as it stands on P = nproc host processes, one component shard each (owner
+    sharding), plus the merge of their per-window results (top-k lists, counters):
+    SURVEY.md §8(d)(ii).  Time = the slowest shard's reduce + the merge."""
+    import multiprocessing as mp
+
+    import oracle
+
+    ctx = mp.get_context("fork")
+    with ctx.Manager() as m:
+        barrier = m.Barrier(P)
+        with ctx.Pool(P) as pool:
+            res = pool.map(_shard_worker, [(wl.name, n_win, P, r, barrier) for r in range(P)])
+    dts = [r[0] for r in res]
+    outs = [r[1] for r in res]
+    t0 = time.perf_counter()
+    top, top_n = oracle.merge_topk(outs, wl.k)
+    tot = {f: sum(o["summary"][f].astype(np.uint64) for o in outs)
+           for f in ("n_samples", "n_events", "n_dropped", "digest", "n_touched")}
+    prog = {f: sum(o["progress"][f] for o in outs) for f in ("started", "finished")}
+    dt_merge = time.perf_counter() - t0
+    del top, top_n, prog
+    recs = int(tot["n_samples"].sum() + tot["n_events"].sum() + tot["n_dropped"].sum())
+    return recs, max(dts) + dt_merge
+
+
 def run_reference(args):
     """--impl reference: the CPU oracle timed on the host cores, same metric/config (rank 0 only)."""
     import gen
@@ -226,7 +297,6 @@ def run_native(args):
     assert int(S["n_samples"].sum() + S["n_events"].sum() + S["n_dropped"].sum()) == n_rec * world
     from paper_conf_micro_mosallaeii024_b200 import _native
 
-    mon.profile(True)
     n_launch0 = _native.lib().rtm_kernel_launches()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
@@ -244,6 +314,14 @@ def run_native(args):
             dist.barrier()
     ms = ev0.elapsed_time(ev1)
     n_launches = int(_native.lib().rtm_kernel_launches() - n_launch0)
+    # per-kernel CUDA-event times: a separate pass of the same K steps (not the timed region)
+    mon.profile(True)
+    ev0.record()
+    for _ in range(args.steps):
+        step()
+    ev1.record()
+    torch.cuda.synchronize()
+    prof_ms = ev0.elapsed_time(ev1)
     prof = mon.profile_read()
     mon.profile(False)
     if dist:
@@ -253,9 +331,9 @@ def run_native(args):
     value = n_rec * world * args.steps / (ms / 1e3)
 
     # ---- e2e through the same C-ABI with HOST buffers (pinned), results read back each step
-    e2e_value = None
+    e2e_value, e2e_steps = None, 0
     if 16 * n_rec <= (8 << 30) and not args.no_e2e:
-        e2e_value = run_e2e(args, mon, ds, de, wl, t_end, n_rec, world, dist, dev)
+        e2e_value, e2e_steps = run_e2e(args, mon, ds, de, wl, t_end, n_rec, world, dist, dev)
     W = wl.n_windows
     d2h = W * (8 * 6 + wl.k * 8 + 4 + wl.n_kernels * 40 + 4)
     rank_done = rank != 0
@@ -263,7 +341,8 @@ def run_native(args):
         if dist:
             dist.destroy_process_group()
         return
-    return finish(args, wl, world, ms, prof, n_rec, value, e2e_value, d2h, n_launches, clk, t_wall, dist)
+    return finish(args, wl, world, ms, prof, prof_ms, n_rec, value, e2e_value, e2e_steps, d2h, n_launches, clk,
+                  t_wall, dist)
 
 
 def run_e2e(args, mon, ds, de, wl, t_end, n_rec, world, dist, dev):
@@ -274,7 +353,7 @@ def run_e2e(args, mon, ds, de, wl, t_end, n_rec, world, dist, dev):
     hs.copy_(ds)
     he.copy_(de)
     torch.cuda.synchronize()
-    e2e_steps = max(1, min(3, args.steps))
+    e2e_steps = max(1, min(10, args.steps))  # ~30 ms per step (the H2D of 1.6 GB)
 
     def step_host():
         mon.reset()
@@ -294,19 +373,28 @@ def run_e2e(args, mon, ds, de, wl, t_end, n_rec, world, dist, dev):
         t = torch.tensor([te], device=dev if dist.get_backend() == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         te = float(t.item())
-    return n_rec * world * e2e_steps / te
+    return n_rec * world * e2e_steps / te, e2e_steps
 
 
-def finish(args, wl, world, ms, prof, n_rec, value, e2e_value, d2h, n_launches, clk, t_wall, dist):
+NOMINAL_HBM_GBS = 8000.0  # B200 HBM3e nominal (SURVEY.md §8(d) reports both denominators)
+
+
+def finish(args, wl, world, ms, prof, prof_ms, n_rec, value, e2e_value, e2e_steps, d2h, n_launches, clk, t_wall,
+           dist):
     W = wl.n_windows
-    # ---- roofline of the dominant kernel: largest share of the step among the kernels on the
-    # critical (main) stream; k_events runs on a side stream overlapped with the partition + fold
+    # ---- roofline: algorithmic bytes = 16 B per record, read once.  They are
+    # charged to the kernel that reads the records (k_partition; it also runs the task-event tiles
+    # on the lane-major path); the fold reads only the 8-B staging entries (not algorithmic: they
+    # show up in `traffic`).  The per-kernel numbers come from a separate profiled pass of the same
+    # K steps (CUDA events around every launch, rtm_profile), so the timed region above carries no
+    # profiling events.
     peaks = _peaks()
     hbm = float(peaks.get("hbm_gbs", 6650.0))
     step_ms = ms / args.steps
-    shares = {k: round(prof[k]["total_ms"] / args.steps / step_ms, 4) for k in prof if prof[k]["launches"]}
-    main_stream = [k for k in prof if prof[k]["launches"] and prof[k]["algo_bytes"] and k != "k_events"]
-    dom = max(main_stream, key=lambda k: prof[k]["total_ms"])
+    pstep_ms = prof_ms / args.steps
+    shares = {k: round(prof[k]["total_ms"] / args.steps / pstep_ms, 4) for k in prof if prof[k]["launches"]}
+    algo = [k for k in prof if prof[k]["launches"] and prof[k]["algo_bytes"]]
+    dom = max(algo, key=lambda k: prof[k]["total_ms"])
     dk = prof[dom]
     achieved_gbs = (dk["algo_bytes"] / dk["launches"]) / (dk["total_ms"] / dk["launches"] / 1e3) / 1e9
     traffic = None
@@ -317,16 +405,31 @@ def finish(args, wl, world, ms, prof, n_rec, value, e2e_value, d2h, n_launches, 
             traffic = next((v for k, v in allt.items() if k == dom or k.startswith((dom + "_", dom + "<"))), None)
         except Exception:
             traffic = None
-    per_kernel = {k: {"achieved_gbs": round((prof[k]["algo_bytes"] / prof[k]["launches"]) /
-                                            (prof[k]["total_ms"] / prof[k]["launches"] / 1e3) / 1e9, 1),
-                      "share": shares[k]} for k in main_stream}
+    per_kernel = {k: {"ms_per_step": round(prof[k]["total_ms"] / args.steps, 4), "share": shares[k],
+                      "algo_bytes_per_launch": prof[k]["algo_bytes"] / prof[k]["launches"],
+                      "achieved_gbs": (round((prof[k]["algo_bytes"] / prof[k]["launches"]) /
+                                             (prof[k]["total_ms"] / prof[k]["launches"] / 1e3) / 1e9, 1)
+                                       if prof[k]["algo_bytes"] else None)}
+                  for k in prof if prof[k]["launches"]}
     path_gbs = 16.0 * n_rec / (step_ms / 1e3) / 1e9
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         n_win = int(os.environ.get("RTM_CPU_WINDOWS", "40"))
         recs, dt = cpu_reference_step(wl, n_win)
+        info = host_info()
         cpu = {"value": recs / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"first {n_win} of {W} {wl.name} windows ({recs} records), single-threaded C oracle"}
+               "sample": f"first {n_win} of {W} {wl.name} windows ({recs} records), single-threaded C oracle",
+               "host": info}
+        P = info["nproc"] or 1
+        if P > 1 and not args.no_cpu_sharded:
+            # every shard process generates the sample's records and keeps its own (~1.6 MB of
+            # records per C2 window per process): bound the host memory to ~8 GB in total
+            n_win_p = int(os.environ.get("RTM_CPU_WINDOWS_SHARDED", str(max(5, min(W, 10 * n_win, 5000 // P)))))
+            recs_p, dt_p = cpu_sharded_step(wl, n_win_p, P)
+            cpu["sharded"] = {"value": recs_p / dt_p, "unit": UNIT, "cores": P, "kind": "oracle",
+                              "sample": f"first {n_win_p} of {W} {wl.name} windows ({recs_p} records) on {P} "
+                                        "processes, one owner-component shard each, + the merge "
+                                        "(slowest shard's reduce + merge time)"}
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
@@ -337,16 +440,25 @@ def finish(args, wl, world, ms, prof, n_rec, value, e2e_value, d2h, n_launches, 
                    "l2": f"inputs ({16 * n_rec / 1e9:.1f} GB/GPU) larger than L2; no flush",
                    "parallelism": f"owner-component shards x{world}" if world > 1 else "single GPU"},
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved_gbs, "peak": hbm, "unit": "GB/s",
-                     "frac": achieved_gbs / hbm, "traffic": traffic,
+                     "frac": achieved_gbs / hbm, "frac_nominal": achieved_gbs / NOMINAL_HBM_GBS, "traffic": traffic,
                      "algo_bytes_per_launch": dk["algo_bytes"] / dk["launches"],
-                     "peak_source": "MEASURED_PEAKS.json hbm_gbs (burst copy)", "share": shares.get(dom),
-                     "path_achieved": path_gbs, "path_frac": path_gbs / hbm, "per_kernel": per_kernel},
+                     "algo_bytes_rule": "16 B per record read (SURVEY.md §8(d)); staging entries are not algorithmic",
+                     "peak_source": "MEASURED_PEAKS.json hbm_gbs (burst copy)", "nominal_peak": NOMINAL_HBM_GBS,
+                     "share": shares.get(dom),
+                     "path_achieved": path_gbs, "path_frac": path_gbs / hbm,
+                     "path_frac_nominal": path_gbs / NOMINAL_HBM_GBS},
+        "kernels": per_kernel,
         "kernel_share": shares,
+        "kernel_timing": f"separate profiled pass of {args.steps} steps ({pstep_ms:.4f} ms/step with events); "
+                         "the timed region carries no profiling events",
         # side-stream kernels: their event interval runs from the partition's end until they get SM
         # slots beside the persistent fold (k_order_check, k_progress), or overlaps the partition
         "side_stream": [k for k in ("k_events", "k_order_check", "k_progress", "k_hang") if k in shares],
         "cpu_baseline": cpu,
-        "e2e": ({"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 16 * n_rec, "d2h_bytes_per_step": d2h}
+        "e2e": ({"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 16 * n_rec, "d2h_bytes_per_step": d2h,
+                 "steps": e2e_steps,
+                 "note": "pinned host trace -> device inside every step: bound by the host link "
+                         "(16 B/record over PCIe/C2C), not by the kernels"}
                 if e2e_value is not None else None),
         "gpu_launches": n_launches,
         "clocks": clk.summary(),
@@ -365,6 +477,7 @@ def main():
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-sharded", action="store_true", help="skip the nproc-process oracle baseline")
     ap.add_argument("--rank-mode", type=int, default=0, help="0 percent (bench line), 1 size, 2 mean occupancy")
     ap.add_argument("--config", default="C2-1gpu",
                     help="workload (gen.CONFIGS); the bench line is C2-1gpu, the others are parity configs "

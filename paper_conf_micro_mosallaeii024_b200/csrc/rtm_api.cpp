@@ -476,9 +476,10 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     if (c->prof) prof_end_on(c, c->st2);
     CK(cudaEventRecord(c->ev_join, c->st2));
   }
-  // algorithmic bytes: partition = 16 B record in + 8 B compacted entry out per
-  // sample (+ 16 B per task event when the event tiles run inside it); fold = the 8 B entry
-  LAUNCH(KT_PARTITION, (uint64_t)ns * 24 + (p.fuse_events ? (uint64_t)ne * 16 : 0),
+  // algorithmic bytes: 16 B per record, read once - charged to
+  // the kernel that reads the records (the partition, + the event tiles it runs when fused); the
+  // 8-B staging entries between partition and fold are not algorithmic (ncu traffic shows them)
+  LAUNCH(KT_PARTITION, (uint64_t)ns * 16 + (p.fuse_events ? (uint64_t)ne * 16 : 0),
          launch_partition(p, c->n_sms, c->st));
   // The order check (tile metadata) and the progress bars (event counts) do not read the fold's
   // outputs: on the side stream, beside the fold (after the event kernel when it runs there);
@@ -495,7 +496,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     if (c->prof) prof_end_on(c, c->st2);
     CK(cudaEventRecord(c->ev_join, c->st2));
   }
-  LAUNCH(KT_FOLD, (uint64_t)ns * 8, launch_fold(p, c->n_sms, c->st));
+  LAUNCH(KT_FOLD, 0, launch_fold(p, c->n_sms, c->st));
   if (side || !p.fuse_events) CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
   if (!side) LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
   // the hang flags (fold's anyfull + event activity bits) and the top-k (fold's last levels) are
