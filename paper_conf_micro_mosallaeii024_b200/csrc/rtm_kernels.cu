@@ -73,6 +73,25 @@ __device__ __forceinline__ unsigned match_bits(unsigned key) {
   return m;
 }
 
+// Runtime bit count (uniform across the warp): keys < 2^bits, bits <= 13 (unrolled; the bits
+// above `bits` are skipped by a uniform branch).
+__device__ __forceinline__ unsigned match_bits_n(unsigned key, unsigned bits) {
+  unsigned m = kFull;
+#pragma unroll
+  for (unsigned k = 0; k < 13; ++k) {
+    if (k < bits) {
+      const unsigned b = __ballot_sync(kFull, (key >> k) & 1u);
+      m &= ((key >> k) & 1u) ? b : ~b;
+    }
+  }
+  return m;
+}
+__host__ __device__ __forceinline__ unsigned bits_for(unsigned n_values) {  // smallest b: n_values <= 2^b
+  unsigned b = 0;
+  while (b < 31 && (1u << b) < n_values) ++b;
+  return b;
+}
+
 // field validity (include/rtm.h)
 __device__ __forceinline__ bool sample_valid(const Params &p, const int4 &v) {
   unsigned b = (unsigned)v.z, lvl = (unsigned)v.w & 0xFFFFu, c = (unsigned)v.w >> 16;
@@ -303,6 +322,7 @@ __device__ __forceinline__ void events_tile(const Params &p, unsigned tile, unsi
   const bool is_win = g.window >= 0;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
+  const unsigned kb = bits_for(2 * p.nk + 1);  // (kernel, kind) keys and the sentinel
   if (is_win) {
     for (unsigned i = threadIdx.x; i < 2 * p.nk; i += blockDim.x) khist[i] = 0;
     if (smem_bits)
@@ -339,8 +359,8 @@ __device__ __forceinline__ void events_tile(const Params &p, unsigned tile, unsi
       kept += keep;
       const unsigned meta = (unsigned)v[jj].w;
       const unsigned comp = meta & 0xFFFFFu, kern = (meta >> 20) & 0x7FFu, kind = meta >> 31;
-      const unsigned kk = keep ? kern * 2 + kind : 0xFFFFFFFFu;
-      const unsigned peers = __match_any_sync(kFull, kk);
+      const unsigned kk = keep ? kern * 2 + kind : 2 * p.nk;  // sentinel 2 nk for dropped events
+      const unsigned peers = match_bits_n(kk, kb);
       if (keep && lane == __ffs(peers) - 1) atomicAdd(&khist[kk], (unsigned)__popc(peers));
       if (keep) {
         if (smem_bits) atomicOr(&abits[comp >> 5], 1u << (comp & 31));
@@ -870,6 +890,7 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
   const bool is_win = t.g.window >= 0;
   const int sub0 = warp * kSub;
   const int4 *src = reinterpret_cast<const int4 *>(p.s) + t.start + sub0;
+  const unsigned kb = bits_for(nbins + 1);  // bin keys and the sentinel nbins
   if (is_win)
     for (unsigned q = lane; q < nbins; q += 32) myt[q] = 0;
   __syncwarp();
@@ -910,7 +931,9 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
       const unsigned key = keep ? (b >> kBinLog) : kNoKey;
       unsigned pos = 0;
       if (is_win) {  // CTA-uniform
-        const unsigned peers = __match_any_sync(kFull, key);
+        // peers by one ballot per key bit (the sentinel maps to nbins): __match_any_sync costs ~2
+        // cycles of SM throughput per distinct key, and 320-4096 bins give ~30 distinct keys per warp
+        const unsigned peers = match_bits_n(keep ? key : nbins, kb);
         const unsigned basec = keep ? myt[key] : 0u;
         __syncwarp();
         if (keep && lane == __ffs(peers) - 1) myt[key] = (unsigned short)(basec + __popc(peers));
