@@ -40,6 +40,7 @@ const char *kKernelNames[KT_N] = {"k_split", "k_partition", "k_events", "k_fold"
 struct rtm_ctx {
   // registry
   uint32_t nb, nc, nk, nbins, ncw, k, H;
+  int32_t bin_log = 8;
   int32_t rank_mode, device, rank, world, hang_mode;
   int64_t t0;
   rtm_allgather_fn allgather;
@@ -330,9 +331,10 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   if (c->merge_pending) return RTM_E_STATE;  // the previous local reduce awaits rtm_merge
   if (!t_end || W == 0) return RTM_E_INVALID;
   if (t_end[0] < c->t_prev) return RTM_E_INVALID;
-  if (t_end[0] - c->t_prev >= kMaxWindowLen) return RTM_E_INVALID;
+  const int64_t max_wlen = max_window_len(c->bin_log);
+  if (t_end[0] - c->t_prev >= max_wlen) return RTM_E_INVALID;
   for (uint32_t w = 1; w < W; ++w)
-    if (t_end[w] < t_end[w - 1] || t_end[w] - t_end[w - 1] >= kMaxWindowLen) return RTM_E_INVALID;
+    if (t_end[w] < t_end[w - 1] || t_end[w] - t_end[w - 1] >= max_wlen) return RTM_E_INVALID;
   CK(cudaSetDevice(c->device));
 
   const void *sp, *ep;
@@ -356,6 +358,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
 
   memset(&p, 0, sizeof(p));
   p.nb = c->nb; p.nc = c->nc; p.nk = c->nk; p.nbins = c->nbins; p.ncw = c->ncw; p.k = c->k;
+  p.bin_log = c->bin_log;
   p.rank_mode = c->rank_mode; p.H = c->H; p.hang_mode = c->hang_mode;
   p.cap = (const uint16_t *)c->cap.p; p.owner = (const uint32_t *)c->owner.p;
   p.elig = (const uint8_t *)c->elig.p; p.ktotal = (const int64_t *)c->ktotal.p;
@@ -654,7 +657,10 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   c->nb = cfg->n_buffers;
   c->nc = cfg->n_components;
   c->nk = cfg->n_kernels;
-  c->nbins = (c->nb + kBin - 1) / kBin;
+  // 256 buffers per bin; 512 when that keeps the bins within the lane-major partition's 170 (nb
+  // 43521 .. 87040, e.g. C3's 81920: otherwise 320 bins take the match-based fallback)
+  c->bin_log = (c->nb > 170u * 256u && c->nb <= 170u * 512u) ? 9 : 8;
+  c->nbins = (c->nb + (1u << c->bin_log) - 1) >> c->bin_log;
   c->ncw = (c->nc + 31) / 32;
   c->k = cfg->k;
   c->H = cfg->hang_windows;

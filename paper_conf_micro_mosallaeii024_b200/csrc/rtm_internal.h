@@ -24,8 +24,7 @@
 
 namespace rtm {
 
-constexpr int kBinLog = 8;                  // 256 buffers per bin
-constexpr int kBin = 1 << kBinLog;
+constexpr int kBin = 256;                   // buffers per bin (bin_log 8); bin_log 9: 512
 constexpr int kTileS = 4096;                // samples per partition tile
 constexpr int kTileE = 4096;                // events per event tile
 constexpr int kK1Threads = 256;             // 8 warps x 512-sample sub-tiles
@@ -37,7 +36,8 @@ constexpr int kFoldWarps = RTM_FOLD_WARPS;  // warps per fold CTA (compile-time 
 constexpr uint16_t kSent = 0xFFFFu;         // "no kept sample in this window" marker
 constexpr uint32_t kMaxBins = 4096;         // n_buffers <= 2^20 (fallback partition smem 160 KB)
 constexpr uint32_t kTopkSmemKeys = 40960;   // keys held in shared memory by the top-k kernel
-constexpr int64_t kMaxWindowLen = (int64_t)1 << 40;  // ts offset field of a staging entry
+// ts offset field of a staging entry: 48 - bin_log bits (entry = off << (16 + bin_log) | level << bin_log | lid)
+inline int64_t max_window_len(int bin_log) { return (int64_t)1 << (48 - bin_log); }
 
 // per-window scalar accumulators, SoA [kWinFields][W] u64
 enum { WF_SAMPLES = 0, WF_EVENTS, WF_DROPPED, WF_DIGEST, WF_TOUCHED, WF_HUNG, kWinFields };
@@ -71,6 +71,7 @@ struct KernelTimer {
 struct Params {
   // registry
   uint32_t nb, nc, nk, nbins, ncw, k;
+  int32_t bin_log;           // buffers per bin = 2^bin_log (8 or 9)
   int32_t rank_mode;
   uint32_t H;
   int32_t hang_mode;         // RTM_HANG_FULL / RTM_HANG_NONEMPTY
@@ -183,7 +184,7 @@ struct ClearList {
 };
 void launch_clear(const ClearList &cl, cudaStream_t st);
 void configure_kernels_once();  // opt-in shared-memory limits, once per device
-size_t fold_smem_bytes();
+size_t fold_smem_bytes(int bin_log);
 size_t partition_smem_bytes(uint32_t nbins, uint32_t nb);
 size_t topk_smem_bytes(uint32_t nb);
 

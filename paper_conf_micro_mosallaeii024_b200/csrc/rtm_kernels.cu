@@ -442,7 +442,7 @@ constexpr int kSub = kTileS / (kK1Threads / 32);  // 512 samples per warp
 constexpr int kPerLane = kSub / 32;               // 16
 constexpr int kK1Warps = kK1Threads / 32;         // 8
 constexpr unsigned kNoKey = 0xFFFFu;
-constexpr uint32_t kLmMaxBins = 128;              // count rows (nbins x 48 B) fit the raw slot; cap <= 64 KB
+constexpr uint32_t kLmMaxBins = 170;              // count rows (nbins x 48 B) fit the 8 KB raw slot
 static_assert(kPerLane == 16, "lane-major swizzle assumes 16 records per lane");
 static_assert((size_t)kLmMaxBins * 48 <= (size_t)kSub * 16, "count rows must fit the raw slot");
 
@@ -456,9 +456,9 @@ __host__ __device__ constexpr size_t k1_vec_bytes(uint32_t nbins) { return k1_al
 // dynamic shared memory.  lm: raw 16 B x 4096 | wt x 2 (tile parity) | wb | tile descriptors
 // (8 warps x 2) | cap[nb];  mx: sbuf 8 B x 4096 | wt | wb
 // (wt: 8 x nbins u16 bin totals / live counters, wb: 8 x nbins u16 bin bases)
-__host__ __device__ constexpr size_t k1_smem_lm(uint32_t nbins, uint32_t nb) {
+__host__ __device__ constexpr size_t k1_smem_lm(uint32_t nbins, uint32_t nb, bool caps = true) {
   return (size_t)kTileS * 16 + 3 * k1_vec_bytes(nbins) + (size_t)kK1Warps * 2 * sizeof(TileDesc) +
-         k1_align16((size_t)nb * 2);
+         (caps ? k1_align16((size_t)nb * 2) : 0);
 }
 __host__ __device__ constexpr size_t k1_smem_mx(uint32_t nbins) { return (size_t)kTileS * 8 + 2 * k1_vec_bytes(nbins); }
 
@@ -577,7 +577,7 @@ __device__ __forceinline__ void k1_publish(K1WarpSum *wsum, unsigned long long f
 // One lane's 16 consecutive records: field check, running min / max of the field-valid offsets
 // (an inversion inside the lane shows up as an offset below the running max), entries, keys.
 // NAR: windows shorter than 2^32 ticks, so offsets are compared and packed in 32 bits.
-template <bool NAR>
+template <bool NAR, int BL, bool CAPS>
 __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool is_win, const int4 *raw,
                                         const unsigned short *capS, int sub0, unsigned long long (&e)[kPerLane],
                                         unsigned (&kp)[kPerLane], unsigned long long &first,
@@ -591,11 +591,18 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
     const int i = lane * kPerLane + k;
     const int4 v = raw[lane * kPerLane + (k ^ (lane & 7))];
     const unsigned b = (unsigned)v.z, lvl = (unsigned)v.w & 0xFFFFu, c = (unsigned)v.w >> 16;
-    const unsigned capb = capS[b < p.nb ? b : 0u];
+    const unsigned capb = CAPS ? capS[b < p.nb ? b : 0u] : (unsigned)__ldg(p.cap + (b < p.nb ? b : 0u));
     const bool valid = (sub0 + i < t.n) & (b < p.nb) & (c == capb) & (lvl <= c);
     const unsigned long long off = (unsigned long long)(rec_ts(v) - t.lo);
     hv |= valid;
-    if (NAR) {
+    if (NAR && BL != 8) {  // (o << (16 + BL)) | (level << BL) | (buffer_id & (2^BL - 1)), o < 2^32
+      const unsigned o = (unsigned)off;
+      bad |= valid & (o < mx);
+      mx = max(mx, valid ? o : 0u);
+      mn = min(mn, valid ? o : ~0u);
+      hiacc |= valid ? (unsigned)(off >> 32) : 0u;
+      e[k] = ((unsigned long long)o << (16 + BL)) | ((unsigned long long)lvl << BL) | (b & ((1u << BL) - 1u));
+    } else if (NAR) {
       const unsigned o = (unsigned)off;
       bad |= valid & (o < mx);
       mx = max(mx, valid ? o : 0u);
@@ -608,11 +615,11 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
       bad |= valid & (off < mx64);
       mx64 = max(mx64, valid ? off : 0ull);
       mn64 = min(mn64, valid ? off : ~0ull);
-      e[k] = (off << 24) | ((unsigned long long)lvl << 8) | (b & (kBin - 1));
+      e[k] = (off << (16 + BL)) | ((unsigned long long)lvl << BL) | (b & ((1u << BL) - 1u));
     }
     const bool keep = valid & is_win;
     kept += keep;
-    kp[k] = (keep ? (b >> kBinLog) : kNoKey) << 16;
+    kp[k] = (keep ? (b >> BL) : kNoKey) << 16;
   }
   if (NAR) {
     bad |= hv & ((hiacc != 0u) | ((unsigned long long)mx >= t.wlen));
@@ -648,6 +655,7 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
 // and only then prefetch their next raw records (named barrier among themselves); warps 4-7
 // prefetch before the first barrier (measured 813 -> 692 us on C2 against direct 8-byte scatter
 // stores from every lane, which touched 32 sectors per store instruction).
+template <int BL, bool CAPS>
 __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ K1WarpSum wsum[2][kK1Warps];
@@ -664,7 +672,8 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   // after the scan the slot holds the count rows: 48 B per bin = 32 u8 lane counters (later the
   // exclusive in-word prefixes) + 8 u16 word bases
   unsigned char *rows = reinterpret_cast<unsigned char *>(raw);
-  for (unsigned i = threadIdx.x; i < p.nb; i += kK1Threads) capS[i] = __ldg(p.cap + i);
+  if (CAPS)  // the capacity table in shared memory (the field check gathers it per sample)
+    for (unsigned i = threadIdx.x; i < p.nb; i += kK1Threads) capS[i] = __ldg(p.cap + i);
   // Tiles are claimed dynamically (p.unit_ctr[1]) so a CTA that starts late - the side-stream
   // event kernel holds SMs at first - simply takes fewer tiles.  Claims run two ahead:
   // ring[i & 3] is iteration i's tile, written by thread 0 in iteration i - 2 and read after
@@ -723,8 +732,8 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     unsigned long long first, last;
     bool has, viol;
     unsigned kept = 0;
-    if (p.narrow && is_win) lm_scan<true>(p, t, is_win, raw, capS, sub0, e, kp, first, last, has, viol, kept);
-    else lm_scan<false>(p, t, is_win, raw, capS, sub0, e, kp, first, last, has, viol, kept);
+    if (p.narrow && is_win) lm_scan<true, BL, CAPS>(p, t, is_win, raw, capS, sub0, e, kp, first, last, has, viol, kept);
+    else lm_scan<false, BL, CAPS>(p, t, is_win, raw, capS, sub0, e, kp, first, last, has, viol, kept);
     {  // order across lanes: my first vs the last of the nearest earlier lane with a valid record
       const unsigned hm = __ballot_sync(kFull, has);
       const unsigned lower = hm & lt;
@@ -928,7 +937,7 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
       }
       const bool keep = valid & is_win;
       kept += keep;
-      const unsigned key = keep ? (b >> kBinLog) : kNoKey;
+      const unsigned key = keep ? (b >> 8) : kNoKey;  // the fallback runs with 256-buffer bins
       unsigned pos = 0;
       if (is_win) {  // CTA-uniform
         // peers by one ballot per key bit (the sentinel maps to nbins): __match_any_sync costs ~2
@@ -941,7 +950,7 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
         pos = basec + __popc(peers & lt);
       }
       kp[j] = (key << 16) | pos;
-      e[j] = (off << 24) | ((unsigned long long)lvl << 8) | (b & (kBin - 1));
+      e[j] = (off << 24) | ((unsigned long long)lvl << 8) | (b & 255u);
     }
   }
   k1_publish(wsum, first, last, has, viol, kept);
@@ -996,12 +1005,14 @@ __device__ __forceinline__ unsigned long long mean_key(unsigned long long I, uns
 // hi[] * 65536 + n16 (hi[] low 16 bits, touched only when n16 wraps).  The offset of the first
 // sample in the window is ts0 | (hi >> 16) << 32 (hi bits only for windows >= 2^32 ticks).  6.5 KB
 // per warp: 8 CTAs of 4 warps per SM.
+template <int BL>
 struct FoldSmem {
-  uint4 st[kBin];
-  unsigned ts0[kBin];              // offset of the first kept sample in the window, low 32 bits
-  unsigned hi[kBin];               // n_hi | ts0_hi << 16
+  static constexpr int kB = 1 << BL;
+  uint4 st[kB];
+  unsigned ts0[kB];                // offset of the first kept sample in the window, low 32 bits
+  unsigned hi[kB];                 // n_hi | ts0_hi << 16
   unsigned seg_base[32];           // staging index of each segment, minus its flattened start
-  unsigned char owner[kBin];       // duplicate detection: last lane that wrote each buffer slot
+  unsigned char owner[kB];         // duplicate detection: last lane that wrote each buffer slot
 };
 constexpr unsigned kUntouchedZ = 0xFFFFFFFFu;  // st.z of an untouched buffer
 __device__ __forceinline__ bool st_touched(const uint4 &v) { return (v.z & 0xFFFFu) != 0xFFFFu; }
@@ -1015,12 +1026,12 @@ __device__ __forceinline__ unsigned long long st_D(const uint4 &v) {
 // Contributions are computed in parallel; the group's sum / max / min travel down the chain in
 // `maxrank` shuffle steps and only the chain's last lane updates the shared state, so every
 // state update in a chunk touches a distinct buffer.
-template <bool NAR>
-__device__ __forceinline__ void fold_chunk(FoldSmem &S, int lane, unsigned lt, bool act, unsigned long long e,
+template <bool NAR, int BL>
+__device__ __forceinline__ void fold_chunk(FoldSmem<BL> &S, int lane, unsigned lt, bool act, unsigned long long e,
                                            unsigned long long Wlen) {
-  const unsigned lid = (unsigned)(e & (kBin - 1));
-  const unsigned lvl = (unsigned)(e >> 8) & 0xFFFFu;
-  const unsigned long long off = e >> 24;
+  const unsigned lid = (unsigned)(e & ((1u << BL) - 1u));
+  const unsigned lvl = (unsigned)(e >> BL) & 0xFFFFu;
+  const unsigned long long off = e >> (16 + BL);
   // Peers = lanes holding the same buffer.  Most lanes hold a buffer no other lane of the chunk
   // holds, and __match_any_sync costs ~2 cycles of SM throughput per DISTINCT key in the warp
   // (tools/microbench.cu), so duplicates are found first through a shared-memory slot per
@@ -1112,10 +1123,10 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
                                             unsigned long long Wlen, int lane) {
   {
     // ---- publish this window's last levels (kSent: untouched) and the phase-1 flag
-    const unsigned b_base = bin * kBin;
+    const unsigned b_base = bin * FS::kB;
     uint16_t *lw = p.lastlvl + (size_t)w * p.nb;
 #pragma unroll
-    for (int i = 0; i < kBin / 32; ++i) {
+    for (int i = 0; i < FS::kB / 32; ++i) {
       const unsigned l = lane + 32 * i, b = b_base + l;
       if (b < p.nb) lw[b] = (uint16_t)(S.st[l].z & 0xFFFFu);  // 0xFFFF == kSent: untouched
     }
@@ -1125,10 +1136,10 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
     __syncwarp();
     if (lane == 0) st_release_u32(p.flags + (size_t)w * p.nbins + bin, p.epoch);
     // ---- phase 2: carry-in by look-back, finalize
-    unsigned short lin[kBin / 32];
+    unsigned short lin[FS::kB / 32];
     unsigned need = 0;
 #pragma unroll
-    for (int i = 0; i < kBin / 32; ++i) {
+    for (int i = 0; i < FS::kB / 32; ++i) {
       lin[i] = 0;
       if (b_base + lane + 32 * i < p.nb) need |= 1u << i;
     }
@@ -1136,7 +1147,7 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
     while (__any_sync(kFull, need != 0)) {
       if (j < 0) {
 #pragma unroll
-        for (int i = 0; i < kBin / 32; ++i)
+        for (int i = 0; i < FS::kB / 32; ++i)
           if (need & (1u << i)) lin[i] = __ldg(p.carry_in + b_base + lane + 32 * i);
         need = 0;
         break;
@@ -1171,16 +1182,16 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
       __syncwarp();
       const unsigned short *lj = p.lastlvl + (size_t)j * p.nb + b_base + lane;
       if constexpr (kStep > 1) {
-        unsigned short v[kStep][kBin / 32];
+        unsigned short v[kStep][FS::kB / 32];
 #pragma unroll
         for (int d = 0; d < kStep; ++d)
 #pragma unroll
-          for (int i = 0; i < kBin / 32; ++i) {
+          for (int i = 0; i < FS::kB / 32; ++i) {
             v[d][i] = kSent;
             if (d < nwin && (need & (1u << i))) v[d][i] = ld_relaxed_u16(lj - (size_t)d * p.nb + 32 * i);
           }
 #pragma unroll
-        for (int i = 0; i < kBin / 32; ++i) {
+        for (int i = 0; i < FS::kB / 32; ++i) {
           if (need & (1u << i)) {
             unsigned short x = kSent;
 #pragma unroll
@@ -1195,7 +1206,7 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
         j -= nwin;
       } else {
 #pragma unroll
-        for (int i = 0; i < kBin / 32; ++i) {
+        for (int i = 0; i < FS::kB / 32; ++i) {
           if (need & (1u << i)) {
             const unsigned short v = ld_relaxed_u16(lj + 32 * i);
             if (v != kSent) {
@@ -1211,7 +1222,7 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
     unsigned touched = 0;
     const bool last_window = (w == p.W - 1);
 #pragma unroll
-    for (int i = 0; i < kBin / 32; ++i) {
+    for (int i = 0; i < FS::kB / 32; ++i) {
       const unsigned l = lane + 32 * i, b = b_base + l;
       if (b >= p.nb) continue;
       const unsigned L = lin[i];
@@ -1287,10 +1298,11 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
 // several consecutive windows, so the look-back walks several windows; it takes RTM_LB_STEP of
 // them per step (their flags waited for by as many lanes, all rows loaded before any is used),
 // dividing the dependent round trips.  A separate instantiation: the dense (C2) code is unchanged.
-template <bool NAR, bool SPARSE = false>
-__global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Params p) {
+template <bool NAR, bool SPARSE, int BL>
+__global__ void __launch_bounds__(kFoldWarps * 32, (BL == 8 ? 32 : 16) / kFoldWarps) k_fold(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
-  FoldSmem &S = reinterpret_cast<FoldSmem *>(smem)[threadIdx.x >> 5];
+  using FS = FoldSmem<BL>;
+  FS &S = reinterpret_cast<FS *>(smem)[threadIdx.x >> 5];
   const int lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
   const unsigned n_units = p.W * p.nbins;
@@ -1304,7 +1316,7 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
     const unsigned long long Wlen = (unsigned long long)(te - tb);
     const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
 #pragma unroll
-    for (int i = 0; i < kBin / 32; ++i) {
+    for (int i = 0; i < FS::kB / 32; ++i) {
       S.st[lane + 32 * i] = make_uint4(0, 0, kUntouchedZ, 0);
       S.hi[lane + 32 * i] = 0;
     }
@@ -1348,7 +1360,7 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
       unsigned long long e0 = fetch(0), e1 = fetch(32);
       for (unsigned c = 0; c < total; c += 32) {
         const unsigned long long en = fetch(c + 64);
-        fold_chunk<NAR>(S, lane, lt, c + lane < total, e0, Wlen);
+        fold_chunk<NAR, BL>(S, lane, lt, c + lane < total, e0, Wlen);
         e0 = e1;
         e1 = en;
       }
@@ -2220,13 +2232,17 @@ void launch_clear(const ClearList &cl, cudaStream_t st) {
   { k_clear<<<blocks < 1184 ? blocks : 1184, 256, 0, st>>>(cl); count_launch(); }
 }
 
-size_t fold_smem_bytes() { return sizeof(FoldSmem) * kFoldWarps; }
+size_t fold_smem_bytes(int bin_log) {
+  return (bin_log == 9 ? sizeof(FoldSmem<9>) : sizeof(FoldSmem<8>)) * kFoldWarps;
+}
+// lane-major partition: the capacity table in shared memory when two CTAs still fit per SM
+bool partition_caps_smem(uint32_t nbins, uint32_t nb) { return k1_smem_lm(nbins, nb, true) + 1024 <= 113 * 1024; }
 size_t partition_smem_bytes(uint32_t nbins, uint32_t nb) {
-  return nbins <= kLmMaxBins ? k1_smem_lm(nbins, nb) : k1_smem_mx(nbins);
+  return nbins <= kLmMaxBins ? k1_smem_lm(nbins, nb, partition_caps_smem(nbins, nb)) : k1_smem_mx(nbins);
 }
 static_assert(2 * (k1_smem_lm(80, 20480) + 1024 + 512) <= 228 * 1024, "C2-sized partition CTAs must fit 2 per SM");
-static_assert(k1_smem_lm(kLmMaxBins, kLmMaxBins * kBin) <= 227 * 1024 && k1_smem_mx(kMaxBins) <= 227 * 1024,
-              "partition shared memory exceeds the 227 KB opt-in limit");
+static_assert(k1_smem_lm(kLmMaxBins, 0, false) <= 113 * 1024 && k1_smem_mx(kMaxBins) <= 227 * 1024,
+              "partition shared memory exceeds the opt-in limit");
 size_t topk_smem_bytes(uint32_t nb) {
   return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8 + kTopkCand * 4;
 }
@@ -2249,17 +2265,29 @@ void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
 
 bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s) { return n_tiles_s && nbins <= kLmMaxBins; }
 
+template <int BL, bool CAPS>
+void launch_partition_lm(const Params &p, int n_sms, size_t sm, cudaStream_t st) {
+  int per_sm = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm<BL, CAPS>, kK1Threads, sm);
+  if (per_sm < 1) per_sm = 1;
+  unsigned grid = (unsigned)(n_sms * per_sm);
+  const unsigned work = p.n_tiles_s + (p.fuse_events ? p.n_tiles_e : 0u);
+  if (grid > work) grid = work;
+  { k_partition_lm<BL, CAPS><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
+}
+
 void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   if (!p.n_tiles_s) return;
   const size_t sm = partition_smem_bytes(p.nbins, p.nb);
-  if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM (capacity table loaded once)
-    int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm, kK1Threads, sm);
-    if (per_sm < 1) per_sm = 1;
-    unsigned grid = (unsigned)(n_sms * per_sm);
-    const unsigned work = p.n_tiles_s + (p.fuse_events ? p.n_tiles_e : 0u);
-    if (grid > work) grid = work;
-    { k_partition_lm<<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
+  if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM
+    const bool caps = partition_caps_smem(p.nbins, p.nb);
+    if (p.bin_log == 9) {
+      if (caps) launch_partition_lm<9, true>(p, n_sms, sm, st);
+      else launch_partition_lm<9, false>(p, n_sms, sm, st);
+    } else {
+      if (caps) launch_partition_lm<8, true>(p, n_sms, sm, st);
+      else launch_partition_lm<8, false>(p, n_sms, sm, st);
+    }
   } else {
     { k_partition_mx<<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
   }
@@ -2271,10 +2299,11 @@ void launch_events(const Params &p, cudaStream_t st) {
   { k_events<<<p.n_tiles_e, kK3Threads, sm, st>>>(p); count_launch(); }
 }
 
-void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
-  const size_t sm = fold_smem_bytes();
+template <int BL>
+void launch_fold_bl(const Params &p, int n_sms, cudaStream_t st) {
+  const size_t sm = fold_smem_bytes(BL);
   int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fold<true>, kFoldWarps * 32, sm);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fold<true, false, BL>, kFoldWarps * 32, sm);
   if (per_sm < 1) per_sm = 1;
   unsigned grid = (unsigned)(n_sms * per_sm);
   const unsigned units = p.W * p.nbins;
@@ -2283,10 +2312,15 @@ void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
   if (grid == 0) grid = 1;
   // sparse units: fewer than 512 kept samples per (window, bin) on average
   const bool sparse = p.ns < (uint64_t)512 * units;
-  if (p.narrow && sparse) { k_fold<true, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
-  else if (p.narrow) { k_fold<true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
-  else if (sparse) { k_fold<false, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
-  else { k_fold<false><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  if (p.narrow && sparse) { k_fold<true, true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else if (p.narrow) { k_fold<true, false, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else if (sparse) { k_fold<false, true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else { k_fold<false, false, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+}
+
+void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
+  if (p.bin_log == 9) launch_fold_bl<9>(p, n_sms, st);
+  else launch_fold_bl<8>(p, n_sms, st);
 }
 
 void launch_order_check(const Params &p, cudaStream_t st) {
@@ -2351,16 +2385,21 @@ void configure_kernels_once() {
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 128 || done[dev]) return;
   done[dev] = true;
-  cudaFuncSetAttribute(k_partition_lm, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                       (int)k1_smem_lm(kLmMaxBins, kLmMaxBins * kBin));
+  const int lm_caps = (int)k1_smem_lm(kLmMaxBins, 113 * 512, true);  // <= 113 KB by partition_caps_smem
+  const int lm_glob = (int)k1_smem_lm(kLmMaxBins, 0, false);
+  cudaFuncSetAttribute(k_partition_lm<8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  cudaFuncSetAttribute(k_partition_lm<9, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<9, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
   cudaFuncSetAttribute(k_partition_mx, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
   cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
   cudaFuncSetAttribute(k_topk<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)topk_smem_bytes(kTopkSmemKeys));
-  cudaFuncSetAttribute(k_fold<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
-  cudaFuncSetAttribute(k_fold<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
-  cudaFuncSetAttribute(k_fold<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
-  cudaFuncSetAttribute(k_fold<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes());
+#define RTM_FOLD_ATTR(NAR_, SP_, BL_) \
+  cudaFuncSetAttribute(k_fold<NAR_, SP_, BL_>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes(BL_))
+  RTM_FOLD_ATTR(true, false, 8); RTM_FOLD_ATTR(false, false, 8); RTM_FOLD_ATTR(true, true, 8); RTM_FOLD_ATTR(false, true, 8);
+  RTM_FOLD_ATTR(true, false, 9); RTM_FOLD_ATTR(false, false, 9); RTM_FOLD_ATTR(true, true, 9); RTM_FOLD_ATTR(false, true, 9);
+#undef RTM_FOLD_ATTR
   cudaGetLastError();
 }
 
