@@ -132,6 +132,9 @@ typedef struct {
   uint32_t n_global_buffers;        /* > every global id; 0 when buffer_global_id is NULL       */
   uint32_t pack_buffers;
   int32_t hang_mode;                /* RTM_HANG_FULL (0, default) or RTM_HANG_NONEMPTY          */
+  int32_t allgather_on_stream;      /* world > 1: nonzero = `allgather` enqueues the collective on
+                                       `stream` (e.g. NCCL) and may return before it completes; the
+                                       library then never synchronises the host around it      */
 } rtm_config;
 
 /* ---- per-window outputs --------------------------------------------------------------------- */
@@ -187,7 +190,12 @@ rtm_status rtm_ingest(rtm_ctx *ctx, const rtm_level_sample *samples, uint64_t n_
  * t_end (collective); all ranks then return identical merged results. */
 rtm_status rtm_window_reduce(rtm_ctx *ctx, const int64_t *t_end, uint32_t n_windows, rtm_window_summary *out);
 
-/* Results of the most recent rtm_window_reduce; `window` indexes its batch. */
+/* Results of the most recent rtm_window_reduce; `window` indexes its batch.
+ * world > 1: the per-window results above (summaries, top-k, progress bars) are merged by every
+ * reduce.  The per-buffer table, the per-component totals and the hang lists are exchanged only
+ * on demand (rtm_sync_tables, or rtm_tables_local + rtm_tables_merge): until then
+ * rtm_buffer_stats, rtm_progress with comps, and rtm_hang_check / rtm_hang_roots of a window
+ * whose merged n_hung is nonzero return RTM_E_STATE (windows with n_hung == 0 answer empty). */
 /* Bottleneck Analyzer list (L173): min(k, eligible buffers) entries, most occupied first,
  * ties by buffer_id ascending.  out holds k entries. */
 rtm_status rtm_topk_buffers(rtm_ctx *ctx, uint32_t window, rtm_topk_entry *out, uint32_t *n_out);
@@ -222,7 +230,8 @@ rtm_status rtm_window_results(rtm_ctx *ctx, uint32_t first, uint32_t count, rtm_
 /* Two-phase form of rtm_window_reduce for callers that run the exchange themselves:
  * reduce_local computes this rank's results and packs them; *pack / *pack_bytes give the
  * device buffer to all-gather; rtm_merge consumes world*pack_bytes gathered bytes (device).
- * The pack is owned by the context and valid until its next reduce call; its size depends on
+ * The pack is owned by the context and valid until its next reduce call, and complete in the
+ * context stream's order (consume it on that stream, or synchronise first); its size depends on
  * n_windows, k, the pack size in buffers and the rank mode (MEAN adds each candidate's 64-bit
  * order key), so every rank must use the same configuration.  Between a successful
  * reduce_local and its rtm_merge the context is merge-pending: another reduce (local or not)
@@ -232,6 +241,20 @@ rtm_status rtm_window_results(rtm_ctx *ctx, uint32_t first, uint32_t count, rtm_
 rtm_status rtm_window_reduce_local(rtm_ctx *ctx, const int64_t *t_end, uint32_t n_windows,
                                    const void **pack, uint64_t *pack_bytes);
 rtm_status rtm_merge(rtm_ctx *ctx, const void *gathered, uint32_t world, rtm_window_summary *out);
+
+/* Bytes of the per-call exchange pack (world > 1): kWinFields x 8 + k x 8 (+ k x 8 in rank mode
+ * MEAN) + 4 + n_kernels x 8 per window; a pure function, no context. */
+uint64_t rtm_exchange_bytes(uint32_t n_windows, uint32_t k, uint32_t n_kernels, int32_t rank_mode);
+
+/* On-demand exchange of the last call's tables (world > 1, collective: every rank calls it
+ * after the same reduce).  rtm_sync_tables runs it through the config's allgather callback;
+ * rtm_tables_local / rtm_tables_merge are its two-phase form: *pack (device, owned by the
+ * context, complete in the context stream's order) holds this rank's per-component totals,
+ * per-buffer table of the last window and per-window hang bitmaps; rtm_tables_merge consumes
+ * world * bytes gathered bytes (device, rank-major).  RTM_E_STATE before the first reduce. */
+rtm_status rtm_sync_tables(rtm_ctx *ctx);
+rtm_status rtm_tables_local(rtm_ctx *ctx, const void **pack, uint64_t *bytes);
+rtm_status rtm_tables_merge(rtm_ctx *ctx, const void *gathered, uint32_t world);
 
 /* ---- Progress bar registry (CreateProgressBar / UpdateProgressBar / DestroyProgressBar, PAPER.md
  * L99; progress bars L131).  Bar ids are the kernel_id field of task

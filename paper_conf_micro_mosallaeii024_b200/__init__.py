@@ -95,6 +95,8 @@ class Monitor:
         self._h = h
         self._keep = []
         self.W = 0
+        self._synced = True
+        self._n_hung = np.zeros(0, np.uint32)
 
     # ------------------------------------------------------------------------------------------
     def close(self):
@@ -130,6 +132,7 @@ class Monitor:
         summ = np.zeros(W, SUMMARY_DTYPE)
         if self.world > 1:
             self._reduce_distributed(t_end, summ)
+            self._synced = False
         else:
             N.check(N.lib().rtm_window_reduce(self._h, t_end.ctypes.data, W, summ.ctypes.data), "rtm_window_reduce")
         self._keep = []
@@ -157,13 +160,43 @@ class Monitor:
         nbytes = ctypes.c_uint64()
         N.check(N.lib().rtm_window_reduce_local(self._h, t_end.ctypes.data, len(t_end), ctypes.byref(pack),
                                                 ctypes.byref(nbytes)), "rtm_window_reduce_local")
-        n = int(nbytes.value)
-        dev = torch.device("cuda", self.device)
-        send = torch.empty(n, dtype=torch.uint8, device=dev)
-        _copy_from_ptr(send, pack.value, n)
-        recv = allgather_packs(send, self.world, self._pg)
-        torch.cuda.current_stream(dev).synchronize()
+        recv = self._exchange(pack.value, int(nbytes.value))
         N.check(N.lib().rtm_merge(self._h, recv.data_ptr(), self.world, summ.ctypes.data), "rtm_merge")
+
+    def _exchange(self, ptr: int, n: int):
+        """All-gather a library pack (device, complete in the Monitor stream's order).  NCCL: the
+        copy, the collective and the library's next kernels are ordered on that stream - no host
+        synchronisation; gloo stages through host memory (synchronous)."""
+        import torch
+
+        from .dist import allgather_packs
+
+        dev = torch.device("cuda", self.device)
+        with torch.cuda.stream(self._stream):
+            send = torch.empty(n, dtype=torch.uint8, device=dev)
+            _copy_from_ptr(send, ptr, n)
+            recv = allgather_packs(send, self.world, self._pg)
+        return recv
+
+    def sync_tables(self):
+        """world > 1: exchange the last call's per-buffer table, per-component totals and hang
+        lists (collective: every rank calls it after the same reduce).  The accessors that need
+        them call it on first use after a reduce."""
+        if self.world <= 1 or self._synced:
+            return
+        pack = ctypes.c_void_p()
+        nbytes = ctypes.c_uint64()
+        N.check(N.lib().rtm_tables_local(self._h, ctypes.byref(pack), ctypes.byref(nbytes)), "rtm_tables_local")
+        recv = self._exchange(pack.value, int(nbytes.value))
+        N.check(N.lib().rtm_tables_merge(self._h, recv.data_ptr(), self.world), "rtm_tables_merge")
+        self._synced = True
+
+    def _n_hung_at(self, window: int) -> int:
+        """Merged flagged count of `window` of the last batch (identical on every rank)."""
+        out = np.zeros(1, SUMMARY_DTYPE)
+        N.check(N.lib().rtm_window_results(self._h, window, 1, out.ctypes.data, None, None, None),
+                "rtm_window_results")
+        return int(out["n_hung"][0])
 
     def topk(self, window: int):
         out = np.zeros(self.k, TOPK_DTYPE)
@@ -173,12 +206,16 @@ class Monitor:
 
     def progress(self, window: int, comps: bool = False):
         bars = np.zeros(self.n_kernels, PROGRESS_DTYPE)
+        if comps:
+            self.sync_tables()
         cs = np.zeros(self.n_components, COMP_DTYPE) if comps else None
         N.check(N.lib().rtm_progress(self._h, window, bars.ctypes.data, None if cs is None else cs.ctypes.data),
                 "rtm_progress")
         return (bars, cs) if comps else bars
 
     def hang_check(self, window: int):
+        if self.world > 1 and self._n_hung_at(window):
+            self.sync_tables()
         n = ctypes.c_uint32()
         N.check(N.lib().rtm_hang_check(self._h, window, None, 0, ctypes.byref(n)), "rtm_hang_check")
         ids = np.zeros(max(1, n.value), np.uint32)
@@ -197,6 +234,8 @@ class Monitor:
 
     def hang_roots(self, window: int):
         """Root causes among the window's flagged components (sink SCCs of the flagged links)."""
+        if self.world > 1 and self._n_hung_at(window):
+            self.sync_tables()
         cap = self.n_components
         out = np.zeros(max(1, cap), np.uint32)
         n = ctypes.c_uint32()
@@ -206,6 +245,7 @@ class Monitor:
     def buffer_stats(self, first: int = 0, count: int | None = None):
         if count is None:
             count = self.n_table - first  # global ids with a rank-local numbering
+        self.sync_tables()
         out = np.zeros(count, BSTAT_DTYPE)
         N.check(N.lib().rtm_buffer_stats(self._h, first, count, out.ctypes.data), "rtm_buffer_stats")
         return out

@@ -48,6 +48,7 @@ class Config(ctypes.Structure):
         ("allgather_user", ctypes.c_void_p), ("stream", ctypes.c_void_p),
         ("buffer_global_id", ctypes.c_void_p), ("n_global_buffers", ctypes.c_uint32),
         ("pack_buffers", ctypes.c_uint32), ("hang_mode", ctypes.c_int32),
+        ("allgather_on_stream", ctypes.c_int32),
     ]
 
 
@@ -61,7 +62,8 @@ EXPORTS = ("rtm_create", "rtm_destroy", "rtm_reset", "rtm_ingest", "rtm_window_r
            "rtm_progress", "rtm_hang_check", "rtm_buffer_stats", "rtm_window_results", "rtm_window_reduce_local",
            "rtm_merge", "rtm_profile", "rtm_profile_read", "rtm_status_str", "rtm_version",
            "rtm_kernel_launches", "rtm_watch", "rtm_watch_series", "rtm_topk_persistence",
-           "rtm_bar_create", "rtm_bar_update", "rtm_bar_destroy", "rtm_set_links", "rtm_hang_roots")
+           "rtm_bar_create", "rtm_bar_update", "rtm_bar_destroy", "rtm_set_links", "rtm_hang_roots",
+           "rtm_exchange_bytes", "rtm_sync_tables", "rtm_tables_local", "rtm_tables_merge")
 
 _lib = None
 
@@ -99,10 +101,13 @@ def lib():
     L.rtm_set_links.argtypes = [vp, vp, vp, u32]
     L.rtm_hang_roots.argtypes = [vp, u32, vp, u32, P(u32)]
     L.rtm_watch_series.argtypes = [vp, u32, vp, P(u32)]
+    L.rtm_sync_tables.argtypes = [vp]
+    L.rtm_tables_local.argtypes = [vp, P(vp), P(u64)]
+    L.rtm_tables_merge.argtypes = [vp, vp, u32]
     for fn in ("rtm_watch", "rtm_watch_series", "rtm_topk_persistence", "rtm_bar_create", "rtm_bar_update",
                "rtm_bar_destroy", "rtm_set_links", "rtm_hang_roots", "rtm_create", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers", "rtm_progress",
                "rtm_hang_check", "rtm_buffer_stats", "rtm_window_reduce_local", "rtm_merge", "rtm_profile",
-               "rtm_profile_read", "rtm_window_results"):
+               "rtm_profile_read", "rtm_window_results", "rtm_sync_tables", "rtm_tables_local", "rtm_tables_merge"):
         getattr(L, fn).restype = ctypes.c_int
     L.rtm_status_str.argtypes = [ctypes.c_int]
     L.rtm_status_str.restype = ctypes.c_char_p
@@ -110,6 +115,8 @@ def lib():
     L.rtm_version.restype = ctypes.c_char_p
     L.rtm_kernel_launches.argtypes = []
     L.rtm_kernel_launches.restype = ctypes.c_uint64
+    L.rtm_exchange_bytes.argtypes = [u32, u32, u32, i32]
+    L.rtm_exchange_bytes.restype = ctypes.c_uint64
     _lib = L
     return L
 

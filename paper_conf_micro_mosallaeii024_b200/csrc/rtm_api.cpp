@@ -75,6 +75,10 @@ struct rtm_ctx {
   DevBuf run[2], kstart, kend, cstart, cend, flags;
   uint32_t epoch = 1;        // look-back flag value of the current / last call (never 0)
   bool merge_pending = false;  // rtm_window_reduce_local done, rtm_merge not yet
+  bool tables_synced = true;   // world > 1: the last call's tables exchanged (rtm_tables_merge)
+  bool ag_on_stream = false;   // the allgather callback is stream-ordered on `st` (no host sync)
+  DevBuf gcum;                 // world > 1: merged cumulative START / END per bar [nk][2] i64
+  DevBuf tpack, tgathered;     // on-demand tables exchange
   int64_t t_prev;
   int sticky = 0;
   // pending stream
@@ -244,6 +248,7 @@ rtm_status zero_state(rtm_ctx *c) {
   cl.add(c->cstart.p, (size_t)c->nc * 8);
   cl.add(c->cend.p, (size_t)c->nc * 8);
   cl.add(c->persist.p, (size_t)(c->n_global ? c->n_global : c->nb) * 4);
+  cl.add(c->gcum.p, (size_t)c->nk * 16);
   launch_clear(cl, c->st);
   CK(cudaGetLastError());
   if (c->bars_dirty) {  // every registered bar live with its registered total (only after changes:
@@ -257,6 +262,7 @@ rtm_status zero_state(rtm_ctx *c) {
   c->t_prev = c->t0;
   c->have = false;
   c->merge_pending = false;
+  c->tables_synced = true;
   c->W = 0;
   c->s_dev.clear();
   c->e_dev.clear();
@@ -676,6 +682,7 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   c->pack_nb = cfg->pack_buffers ? cfg->pack_buffers : cfg->n_buffers;
   c->allgather = cfg->allgather;
   c->allgather_user = cfg->allgather_user;
+  c->ag_on_stream = cfg->allgather_on_stream != 0;
   c->st = (cudaStream_t)cfg->stream;
   if (cudaSetDevice(c->device) != cudaSuccess) { cudaGetLastError(); delete c; return RTM_E_CUDA; }
   configure_kernels_once();
@@ -702,7 +709,7 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
       (s = ensure(c, c->cend, (size_t)c->nc * 8)) || (s = ensure(c, c->rcp, (size_t)65536 * 8)) ||
       (s = ensure(c, c->elig_ids, (size_t)c->nb * 4)) ||
       (s = ensure(c, c->persist, (size_t)(c->n_global ? c->n_global : c->nb) * 4)) ||
-      (s = ensure(c, c->klive, (size_t)c->nk)))
+      (s = ensure(c, c->klive, (size_t)c->nk)) || (s = ensure(c, c->gcum, (size_t)c->nk * 16)))
     return fail(s);
   c->ktotal0.assign(cfg->kernel_total, cfg->kernel_total + c->nk);
   if (c->rank_mode == RTM_RANK_MEAN) {
@@ -762,7 +769,8 @@ void rtm_destroy(rtm_ctx *c) {
                     &c->rts, &c->rte, &c->treg_s, &c->treg_e, &c->tdesc, &c->soff, &c->stage, &c->smeta, &c->emeta,
                     &c->lastlvl, &c->res, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
                     &c->unit_ctr, &c->bstat, &c->comps, &c->pack,
-                    &c->gathered, &c->tkscr, &c->mkey, &c->rcp64, &c->tkey, &c->persist, &c->klive};
+                    &c->gathered, &c->tkscr, &c->mkey, &c->rcp64, &c->tkey, &c->persist, &c->klive,
+                    &c->gcum, &c->tpack, &c->tgathered};
   for (DevBuf *b : bufs) free_buf(*b);
   if (c->h_small.p) cudaFreeHost(c->h_small.p);
   if (c->h_res.p) cudaFreeHost(c->h_res.p);
@@ -796,6 +804,8 @@ rtm_status rtm_bar_create(rtm_ctx *c, int64_t total, uint32_t *bar_id) {
   CK(cudaMemcpyAsync((int64_t *)c->ktotal.p + k, &total, 8, cudaMemcpyHostToDevice, c->st));
   CK(cudaMemcpyAsync((int64_t *)c->kstart.p + k, &zero, 8, cudaMemcpyHostToDevice, c->st));
   CK(cudaMemcpyAsync((int64_t *)c->kend.p + k, &zero, 8, cudaMemcpyHostToDevice, c->st));
+  CK(cudaMemcpyAsync((int64_t *)c->gcum.p + 2 * k, &zero, 8, cudaMemcpyHostToDevice, c->st));
+  CK(cudaMemcpyAsync((int64_t *)c->gcum.p + 2 * k + 1, &zero, 8, cudaMemcpyHostToDevice, c->st));
   CK(cudaMemcpyAsync((uint8_t *)c->klive.p + k, &one, 1, cudaMemcpyHostToDevice, c->st));
   CK(cudaStreamSynchronize(c->st));  // pageable stack sources
   c->klive_h[k] = 1;
@@ -894,14 +904,15 @@ rtm_status rtm_window_reduce(rtm_ctx *c, const int64_t *t_end, uint32_t n_window
     if ((s = ensure(c, c->pack, pb))) return s;
     if ((s = ensure(c, c->gathered, pb * c->world))) return s;
     launch_pack(p, c->pack.p, c->st);
-    CK(cudaStreamSynchronize(c->st));
+    if (!c->ag_on_stream) CK(cudaStreamSynchronize(c->st));  // else the callback orders itself on st
     if (c->allgather(c->allgather_user, c->pack.p, c->gathered.p, pb) != 0) {
       c->sticky = RTM_E_COMM;
       return RTM_E_COMM;
     }
-    LAUNCH(KT_MERGE, 0, launch_merge(p, c->gathered.p, c->world, c->st));
+    LAUNCH(KT_MERGE, 0, launch_merge(p, c->gathered.p, c->world, (long long *)c->gcum.p, c->st));
     launch_persist(p, c->st);
     CK(cudaGetLastError());
+    c->tables_synced = false;
   } else if (c->gid.p) {
     launch_scatter_bstat(p, c->st);
   }
@@ -917,8 +928,7 @@ rtm_status rtm_window_reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t n_
   const uint64_t pb = pack_bytes(p);
   if ((s = ensure(c, c->pack, pb))) return s;
   launch_pack(p, c->pack.p, c->st);
-  CK(cudaGetLastError());
-  CK(cudaStreamSynchronize(c->st));
+  CK(cudaGetLastError());  // the pack is complete in the context stream's order (no host sync)
   *pack = c->pack.p;
   *pack_bytes_out = pb;
   // remember the call for rtm_merge; no other reduce (and no rtm_watch, which would change the
@@ -948,11 +958,75 @@ rtm_status rtm_merge(rtm_ctx *c, const void *gathered, uint32_t world, rtm_windo
   p.gid = (const uint32_t *)c->gid.p; p.n_global = c->n_global; p.pack_nb = c->pack_nb;
   p.bstat_g = (rtm_buffer_stat *)c->bstat_g.p;
   p.persist = (uint32_t *)c->persist.p;
-  LAUNCH(KT_MERGE, 0, launch_merge(p, gathered, world, c->st));
+  LAUNCH(KT_MERGE, 0, launch_merge(p, gathered, world, (long long *)c->gcum.p, c->st));
   launch_persist(p, c->st);
   CK(cudaGetLastError());
+  c->tables_synced = c->world <= 1;
   std::vector<int64_t> te = c->t_end_h;
   return finish(c, te.data(), W, out);
+}
+
+// Params of the last call's tables (the on-demand exchange)
+static Params table_params(rtm_ctx *c) {
+  Params p;
+  memset(&p, 0, sizeof(p));
+  p.nb = c->nb; p.nc = c->nc; p.nk = c->nk; p.nbins = c->nbins; p.ncw = c->ncw; p.k = c->k;
+  p.W = c->W;
+  p.hung = (uint32_t *)c->hung.p;
+  p.comps = (rtm_component_tasks *)c->comps.p; p.bstat = (rtm_buffer_stat *)c->bstat.p;
+  p.cstart = (long long *)c->cstart.p; p.cend = (long long *)c->cend.p;
+  p.gid = (const uint32_t *)c->gid.p; p.n_global = c->n_global; p.pack_nb = c->pack_nb;
+  p.bstat_g = (rtm_buffer_stat *)c->bstat_g.p;
+  return p;
+}
+
+rtm_status rtm_tables_local(rtm_ctx *c, const void **pack, uint64_t *bytes) {
+  if (!c || !pack || !bytes) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (!c->have) return RTM_E_STATE;
+  CK(cudaSetDevice(c->device));
+  const Params p = table_params(c);
+  const uint64_t tb = tables_bytes(p);
+  rtm_status s;
+  if ((s = ensure(c, c->tpack, tb))) return s;
+  launch_pack_tables(p, c->tpack.p, c->st);
+  CK(cudaGetLastError());  // complete in the context stream's order
+  *pack = c->tpack.p;
+  *bytes = tb;
+  return RTM_OK;
+}
+
+rtm_status rtm_tables_merge(rtm_ctx *c, const void *gathered, uint32_t world) {
+  if (!c || !gathered || world == 0) return RTM_E_INVALID;
+  if (c->sticky) return (rtm_status)c->sticky;
+  if (!c->have) return RTM_E_STATE;
+  CK(cudaSetDevice(c->device));
+  const Params p = table_params(c);
+  launch_merge_tables(p, gathered, world, c->st);
+  CK(cudaGetLastError());
+  c->tables_synced = true;
+  return RTM_OK;
+}
+
+rtm_status rtm_sync_tables(rtm_ctx *c) {
+  if (!c) return RTM_E_INVALID;
+  if (c->world > 1 && !c->allgather) return RTM_E_INVALID;
+  if (c->world <= 1 || c->tables_synced) return c->sticky ? (rtm_status)c->sticky : (c->have ? RTM_OK : RTM_E_STATE);
+  const void *pk;
+  uint64_t tb;
+  rtm_status s = rtm_tables_local(c, &pk, &tb);
+  if (s) return s;
+  if ((s = ensure(c, c->tgathered, tb * c->world))) return s;
+  if (!c->ag_on_stream) CK(cudaStreamSynchronize(c->st));
+  if (c->allgather(c->allgather_user, pk, c->tgathered.p, tb) != 0) {
+    c->sticky = RTM_E_COMM;
+    return RTM_E_COMM;
+  }
+  return rtm_tables_merge(c, c->tgathered.p, c->world);
+}
+
+uint64_t rtm_exchange_bytes(uint32_t n_windows, uint32_t k, uint32_t n_kernels, int32_t rank_mode) {
+  return exchange_bytes(n_windows, k, n_kernels, rank_mode);
 }
 
 rtm_status rtm_topk_buffers(rtm_ctx *c, uint32_t window, rtm_topk_entry *out, uint32_t *n_out) {
@@ -1003,6 +1077,7 @@ rtm_status rtm_progress(rtm_ctx *c, uint32_t window, rtm_progress_entry *bars, r
   if (!c->have) return RTM_E_STATE;
   if (window >= c->W) return RTM_E_INVALID;
   if (comps && window != c->W - 1) return RTM_E_INVALID;
+  if (comps && !c->tables_synced) return RTM_E_STATE;  // world > 1: rtm_sync_tables first
   memcpy(bars, c->prog_h + (size_t)window * c->nk, (size_t)c->nk * sizeof(rtm_progress_entry));
   if (comps) {
     CK(cudaSetDevice(c->device));
@@ -1038,6 +1113,13 @@ rtm_status rtm_hang_check(rtm_ctx *c, uint32_t window, uint32_t *comp_ids, uint3
   if (c->sticky) return (rtm_status)c->sticky;
   if (!c->have) return RTM_E_STATE;
   if (window >= c->W) return RTM_E_INVALID;
+  if (!c->tables_synced) {  // world > 1: the merged count is known; the list needs the tables
+    if (c->sum[window].n_hung == 0) {
+      *n_hung = 0;
+      return RTM_OK;
+    }
+    return RTM_E_STATE;
+  }
   std::vector<uint32_t> ids;
   rtm_status s = hung_list(c, window, ids);
   if (s) return s;
@@ -1065,6 +1147,13 @@ rtm_status rtm_hang_roots(rtm_ctx *c, uint32_t window, uint32_t *comp_ids, uint3
   if (c->sticky) return (rtm_status)c->sticky;
   if (!c->have) return RTM_E_STATE;
   if (window >= c->W) return RTM_E_INVALID;
+  if (!c->tables_synced) {
+    if (c->sum[window].n_hung == 0) {
+      *n_roots = 0;
+      return RTM_OK;
+    }
+    return RTM_E_STATE;
+  }
   std::vector<uint32_t> F;
   rtm_status s = hung_list(c, window, F);
   if (s) return s;
@@ -1139,6 +1228,7 @@ rtm_status rtm_buffer_stats(rtm_ctx *c, uint32_t first, uint32_t count, rtm_buff
   if (!c->have) return RTM_E_STATE;
   const bool by_gid = c->gid.p != nullptr;
   if ((uint64_t)first + count > (by_gid ? c->n_global : c->nb)) return RTM_E_INVALID;
+  if (!c->tables_synced) return RTM_E_STATE;  // world > 1: rtm_sync_tables first
   if (!count) return RTM_OK;
   CK(cudaSetDevice(c->device));
   CK(cudaMemcpyAsync(out, (rtm_buffer_stat *)(by_gid ? c->bstat_g.p : c->bstat.p) + first,

@@ -163,7 +163,11 @@ void launch_persist(const Params &p, cudaStream_t st);
 // multi-rank exchange
 uint64_t pack_bytes(const Params &p);
 void launch_pack(const Params &p, void *pack, cudaStream_t st);
-void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStream_t st);
+void launch_merge(const Params &p, const void *gathered, uint32_t world, long long *gcum, cudaStream_t st);
+uint64_t exchange_bytes(uint32_t W, uint32_t k, uint32_t nk, int rank_mode);  // per-call pack size
+uint64_t tables_bytes(const Params &p);
+void launch_pack_tables(const Params &p, void *pack, cudaStream_t st);
+void launch_merge_tables(const Params &p, const void *gathered, uint32_t world, cudaStream_t st);
 bool merge_fits(uint32_t world, uint32_t k);  // world * k candidates fit the merge's shared memory
 void launch_scatter_bstat(const Params &p, cudaStream_t st);  // gid set, world == 1
 unsigned long long kernel_launches();  // kernels launched by this library in this process

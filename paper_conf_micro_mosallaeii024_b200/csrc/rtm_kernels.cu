@@ -73,25 +73,6 @@ __device__ __forceinline__ unsigned match_bits(unsigned key) {
   return m;
 }
 
-// Runtime bit count (uniform across the warp): keys < 2^bits, bits <= 13 (unrolled; the bits
-// above `bits` are skipped by a uniform branch).
-__device__ __forceinline__ unsigned match_bits_n(unsigned key, unsigned bits) {
-  unsigned m = kFull;
-#pragma unroll
-  for (unsigned k = 0; k < 13; ++k) {
-    if (k < bits) {
-      const unsigned b = __ballot_sync(kFull, (key >> k) & 1u);
-      m &= ((key >> k) & 1u) ? b : ~b;
-    }
-  }
-  return m;
-}
-__host__ __device__ __forceinline__ unsigned bits_for(unsigned n_values) {  // smallest b: n_values <= 2^b
-  unsigned b = 0;
-  while (b < 31 && (1u << b) < n_values) ++b;
-  return b;
-}
-
 // field validity (include/rtm.h)
 __device__ __forceinline__ bool sample_valid(const Params &p, const int4 &v) {
   unsigned b = (unsigned)v.z, lvl = (unsigned)v.w & 0xFFFFu, c = (unsigned)v.w >> 16;
@@ -322,7 +303,6 @@ __device__ __forceinline__ void events_tile(const Params &p, unsigned tile, unsi
   const bool is_win = g.window >= 0;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
-  const unsigned kb = bits_for(2 * p.nk + 1);  // (kernel, kind) keys and the sentinel
   if (is_win) {
     for (unsigned i = threadIdx.x; i < 2 * p.nk; i += blockDim.x) khist[i] = 0;
     if (smem_bits)
@@ -359,8 +339,8 @@ __device__ __forceinline__ void events_tile(const Params &p, unsigned tile, unsi
       kept += keep;
       const unsigned meta = (unsigned)v[jj].w;
       const unsigned comp = meta & 0xFFFFFu, kern = (meta >> 20) & 0x7FFu, kind = meta >> 31;
-      const unsigned kk = keep ? kern * 2 + kind : 2 * p.nk;  // sentinel 2 nk for dropped events
-      const unsigned peers = match_bits_n(kk, kb);
+      const unsigned kk = keep ? kern * 2 + kind : 0xFFFFFFFFu;
+      const unsigned peers = __match_any_sync(kFull, kk);
       if (keep && lane == __ffs(peers) - 1) atomicAdd(&khist[kk], (unsigned)__popc(peers));
       if (keep) {
         if (smem_bits) atomicOr(&abits[comp >> 5], 1u << (comp & 31));
@@ -899,7 +879,6 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
   const bool is_win = t.g.window >= 0;
   const int sub0 = warp * kSub;
   const int4 *src = reinterpret_cast<const int4 *>(p.s) + t.start + sub0;
-  const unsigned kb = bits_for(nbins + 1);  // bin keys and the sentinel nbins
   if (is_win)
     for (unsigned q = lane; q < nbins; q += 32) myt[q] = 0;
   __syncwarp();
@@ -940,9 +919,8 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
       const unsigned key = keep ? (b >> 8) : kNoKey;  // the fallback runs with 256-buffer bins
       unsigned pos = 0;
       if (is_win) {  // CTA-uniform
-        // peers by one ballot per key bit (the sentinel maps to nbins): __match_any_sync costs ~2
-        // cycles of SM throughput per distinct key, and 320-4096 bins give ~30 distinct keys per warp
-        const unsigned peers = match_bits_n(keep ? key : nbins, kb);
+        // (per-bit ballots instead of MATCH measured equal on C3 / C4: the fallback is latency-bound)
+        const unsigned peers = __match_any_sync(kFull, key);
         const unsigned basec = keep ? myt[key] : 0u;
         __syncwarp();
         if (keep && lane == __ffs(peers) - 1) myt[key] = (unsigned short)(basec + __popc(peers));
@@ -2041,22 +2019,45 @@ __global__ void __launch_bounds__(1024) k_progress(Params p) {
 //   gids [pack_nb] u32 (rank-local numbering only: the global id of each bstat entry, ~0 = pad) |
 //   tkey [W][k] u64 (rank mode MEAN only: the order key of each top-k entry, mean_key)
 // ============================================================================================
+// Per-call exchange pack (world > 1): only what the per-window merged results need.
+//   win   [kWinFields][W] u64   counters and digest (sums over ranks)
+//   topk  [W][k] u64            local top-k entries (id | level << 32 | cap << 48)
+//   topk_n[W] u32
+//   kd    [W][nk][2] u32        this rank's START / END events per window and bar (the merge
+//                               sums them and carries the merged cumulative counts across calls)
+//   tkey  [W][k] u64            rank mode MEAN: each candidate's 64-bit order key
+// The per-buffer table, per-component totals and hang bitmaps are NOT in it: they are exchanged on
+// demand (rtm_tables_local / rtm_tables_merge / rtm_sync_tables).
 struct PackLayout {
-  size_t win, topk, topk_n, prog, hung, comps, bstat, gids, tkey, total;
+  size_t win, topk, topk_n, kd, tkey, total;
 };
 __host__ __device__ inline size_t align8(size_t x) { return (x + 7) & ~(size_t)7; }
-__host__ __device__ inline PackLayout pack_layout(const Params &p) {
+__host__ __device__ inline PackLayout pack_layout_for(uint32_t W, uint32_t k, uint32_t nk, int rank_mode) {
   PackLayout L;
   size_t o = 0;
-  L.win = o; o += align8((size_t)kWinFields * p.W * 8);
-  L.topk = o; o += align8((size_t)p.W * p.k * 8);
-  L.topk_n = o; o += align8((size_t)p.W * 4);
-  L.prog = o; o += align8((size_t)p.W * p.nk * 5 * 8);
-  L.hung = o; o += align8((size_t)p.W * p.ncw * 4);
-  L.comps = o; o += align8((size_t)p.nc * sizeof(rtm_component_tasks));
+  L.win = o; o += align8((size_t)kWinFields * W * 8);
+  L.topk = o; o += align8((size_t)W * k * 8);
+  L.topk_n = o; o += align8((size_t)W * 4);
+  L.kd = o; o += align8((size_t)W * nk * 2 * 4);
+  L.tkey = o; o += rank_mode == RTM_RANK_MEAN ? (size_t)W * k * 8 : 0;
+  L.total = o;
+  return L;
+}
+__host__ __device__ inline PackLayout pack_layout(const Params &p) { return pack_layout_for(p.W, p.k, p.nk, p.rank_mode); }
+
+// On-demand tables pack (the last call's state): per-component START / END totals, the
+// per-buffer table of the last window (with global ids under a rank-local numbering) and the
+// per-window hang bitmaps.
+struct TablesLayout {
+  size_t comps, bstat, gids, hung, total;
+};
+__host__ __device__ inline TablesLayout tables_layout(const Params &p) {
+  TablesLayout L;
+  size_t o = 0;
+  L.comps = o; o += align8((size_t)p.nc * 16);
   L.bstat = o; o += align8((size_t)p.pack_nb * sizeof(rtm_buffer_stat));
   L.gids = o; o += p.gid ? align8((size_t)p.pack_nb * 4) : 0;
-  L.tkey = o; o += p.rank_mode == RTM_RANK_MEAN ? (size_t)p.W * p.k * 8 : 0;
+  L.hung = o; o += align8((size_t)p.W * p.ncw * 4);
   L.total = o;
   return L;
 }
@@ -2141,38 +2142,67 @@ __global__ void __launch_bounds__(256) k_merge_windows(Params p, const unsigned 
       s += reinterpret_cast<const unsigned long long *>(g + stride * r + L.win)[(size_t)threadIdx.x * p.W + w];
     p.win[(size_t)threadIdx.x * p.W + w] = s;
   }
-  // progress: sum of per-rank cumulative START / END
-  for (unsigned k = threadIdx.x; k < p.nk; k += blockDim.x) {
-    long long S = 0, E = 0;
-    for (unsigned r = 0; r < world; ++r) {
-      const long long *o = reinterpret_cast<const long long *>(g + stride * r + L.prog) + ((size_t)w * p.nk + k) * 5;
-      S += o[1];
-      E += o[2];
+}
+
+// Merged progress bars (L131): one CTA per bar; the bar's START / END deltas summed over ranks,
+// prefix-summed over the call's windows on top of the merged cumulative counts of earlier calls
+// (gcum, identical on every rank), which are then advanced.
+__global__ void __launch_bounds__(1024) k_merge_progress(Params p, const unsigned char *g, unsigned world,
+                                                         size_t stride, long long *gcum) {
+  __shared__ unsigned scan_scratch[32];
+  const PackLayout L = pack_layout(p);
+  const unsigned k = blockIdx.x;
+  long long s = gcum[2 * k], e = gcum[2 * k + 1];
+  const bool live = p.klive[k] != 0;  // a destroyed bar reads all zero (rtm_bar_destroy)
+  const long long total = live ? p.ktotal[k] : 0;
+  for (unsigned base = 0; base < p.W; base += blockDim.x) {
+    const unsigned w = base + threadIdx.x;
+    unsigned ds = 0, de = 0;
+    if (w < p.W)
+      for (unsigned r = 0; r < world; ++r) {
+        const unsigned *kd = reinterpret_cast<const unsigned *>(g + stride * r + L.kd) + ((size_t)w * p.nk + k) * 2;
+        ds += kd[0];
+        de += kd[1];
+      }
+    unsigned ts_, te_;
+    const unsigned xs = block_excl_scan(ds, scan_scratch, &ts_);
+    const unsigned xe = block_excl_scan(de, scan_scratch, &te_);
+    if (w < p.W) {
+      const long long S = s + xs + ds, E = e + xe + de;
+      long long *o = p.prog + ((size_t)w * p.nk + k) * 5;
+      o[0] = total;
+      o[1] = live ? S : 0;
+      o[2] = live ? E : 0;
+      o[3] = live ? S - E : 0;
+      o[4] = live ? total - S : 0;
     }
-    long long *o = p.prog + ((size_t)w * p.nk + k) * 5;
-    const bool live = p.klive[k] != 0;  // a destroyed bar reads all zero (rtm_bar_destroy)
-    const long long total = live ? p.ktotal[k] : 0;
-    o[0] = total; o[1] = S; o[2] = E; o[3] = S - E; o[4] = total - S;
+    s += ts_;
+    e += te_;
   }
-  for (unsigned q = threadIdx.x; q < p.ncw; q += blockDim.x) {
-    unsigned x = 0;
-    for (unsigned r = 0; r < world; ++r) x |= reinterpret_cast<const unsigned *>(g + stride * r + L.hung)[(size_t)w * p.ncw + q];
-    p.hung[(size_t)w * p.ncw + q] = x;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    gcum[2 * k] = s;
+    gcum[2 * k + 1] = e;
   }
 }
 
 __global__ void k_merge_tables(Params p, const unsigned char *g, unsigned world, size_t stride) {
-  const PackLayout L = pack_layout(p);
+  const TablesLayout L = tables_layout(p);
   const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (size_t)gridDim.x * blockDim.x;
   for (size_t c = tid; c < p.nc; c += nth) {
     rtm_component_tasks t = {0, 0, 0};
     for (unsigned r = 0; r < world; ++r) {
-      const rtm_component_tasks x = reinterpret_cast<const rtm_component_tasks *>(g + stride * r + L.comps)[c];
-      t.started += x.started;
-      t.finished += x.finished;
+      const long long *x = reinterpret_cast<const long long *>(g + stride * r + L.comps) + 2 * c;
+      t.started += x[0];
+      t.finished += x[1];
     }
     t.in_flight = t.started - t.finished;
     p.comps[c] = t;
+  }
+  for (size_t q = tid; q < (size_t)p.W * p.ncw; q += nth) {  // hang flags: OR over ranks
+    unsigned x = 0;
+    for (unsigned r = 0; r < world; ++r) x |= reinterpret_cast<const unsigned *>(g + stride * r + L.hung)[q];
+    p.hung[q] = x;
   }
   if (p.gid) {  // rank-local numbering: scatter every rank's entries to their global ids
     for (size_t q = tid; q < (size_t)world * p.pack_nb; q += nth) {
@@ -2189,6 +2219,17 @@ __global__ void k_merge_tables(Params p, const unsigned char *g, unsigned world,
       if (x.reserved) { pick = x; break; }
     }
     p.bstat[b] = pick;
+  }
+}
+
+// this rank's tables pack
+__global__ void k_pack_tables(Params p, unsigned char *d) {
+  const TablesLayout L = tables_layout(p);
+  const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (size_t)gridDim.x * blockDim.x;
+  for (size_t c = tid; c < p.nc; c += nth) {
+    long long *x = reinterpret_cast<long long *>(d + L.comps) + 2 * c;
+    x[0] = p.cstart[c];
+    x[1] = p.cend[c];
   }
 }
 
@@ -2378,6 +2419,9 @@ void launch_progress(const Params &p, cudaStream_t st) {
 }
 
 uint64_t pack_bytes(const Params &p) { return pack_layout(p).total; }
+uint64_t exchange_bytes(uint32_t W, uint32_t k, uint32_t nk, int rank_mode) {
+  return pack_layout_for(W, k, nk, rank_mode).total;
+}
 
 void configure_kernels_once() {
   static bool done[128] = {false};
@@ -2409,9 +2453,19 @@ void launch_pack(const Params &p, void *pack, cudaStream_t st) {
   cudaMemcpyAsync(d + L.win, p.win, (size_t)kWinFields * p.W * 8, cudaMemcpyDeviceToDevice, st);
   cudaMemcpyAsync(d + L.topk, p.topk, (size_t)p.W * p.k * 8, cudaMemcpyDeviceToDevice, st);
   cudaMemcpyAsync(d + L.topk_n, p.topk_n, (size_t)p.W * 4, cudaMemcpyDeviceToDevice, st);
-  cudaMemcpyAsync(d + L.prog, p.prog, (size_t)p.W * p.nk * 5 * 8, cudaMemcpyDeviceToDevice, st);
-  cudaMemcpyAsync(d + L.hung, p.hung, (size_t)p.W * p.ncw * 4, cudaMemcpyDeviceToDevice, st);
-  cudaMemcpyAsync(d + L.comps, p.comps, (size_t)p.nc * sizeof(rtm_component_tasks), cudaMemcpyDeviceToDevice, st);
+  cudaMemcpyAsync(d + L.kd, p.kdelta, (size_t)p.W * p.nk * 2 * 4, cudaMemcpyDeviceToDevice, st);
+  if (p.rank_mode == RTM_RANK_MEAN) {
+    if (p.tkey) cudaMemcpyAsync(d + L.tkey, p.tkey, (size_t)p.W * p.k * 8, cudaMemcpyDeviceToDevice, st);
+    else cudaMemsetAsync(d + L.tkey, 0, (size_t)p.W * p.k * 8, st);
+  }
+}
+
+uint64_t tables_bytes(const Params &p) { return tables_layout(p).total; }
+
+void launch_pack_tables(const Params &p, void *pack, cudaStream_t st) {
+  const TablesLayout L = tables_layout(p);
+  unsigned char *d = static_cast<unsigned char *>(pack);
+  { k_pack_tables<<<p.nc / 256 + 1 < 1184 ? p.nc / 256 + 1 : 1184, 256, 0, st>>>(p, d); count_launch(); }
   cudaMemcpyAsync(d + L.bstat, p.bstat, (size_t)p.nb * sizeof(rtm_buffer_stat), cudaMemcpyDeviceToDevice, st);
   if (p.pack_nb > p.nb)
     cudaMemsetAsync(d + L.bstat + (size_t)p.nb * sizeof(rtm_buffer_stat), 0,
@@ -2420,10 +2474,12 @@ void launch_pack(const Params &p, void *pack, cudaStream_t st) {
     cudaMemcpyAsync(d + L.gids, p.gid, (size_t)p.nb * 4, cudaMemcpyDeviceToDevice, st);
     if (p.pack_nb > p.nb) cudaMemsetAsync(d + L.gids + (size_t)p.nb * 4, 0xFF, (size_t)(p.pack_nb - p.nb) * 4, st);
   }
-  if (p.rank_mode == RTM_RANK_MEAN) {
-    if (p.tkey) cudaMemcpyAsync(d + L.tkey, p.tkey, (size_t)p.W * p.k * 8, cudaMemcpyDeviceToDevice, st);
-    else cudaMemsetAsync(d + L.tkey, 0, (size_t)p.W * p.k * 8, st);
-  }
+  cudaMemcpyAsync(d + L.hung, p.hung, (size_t)p.W * p.ncw * 4, cudaMemcpyDeviceToDevice, st);
+}
+
+void launch_merge_tables(const Params &p, const void *gathered, uint32_t world, cudaStream_t st) {
+  { k_merge_tables<<<256, 256, 0, st>>>(p, static_cast<const unsigned char *>(gathered), world,
+                                        tables_layout(p).total); count_launch(); }
 }
 
 void launch_scatter_bstat(const Params &p, cudaStream_t st) {
@@ -2438,14 +2494,14 @@ bool merge_fits(uint32_t world, uint32_t k) {
   return P * 20 <= 227ull * 1024;
 }
 
-void launch_merge(const Params &p, const void *gathered, uint32_t world, cudaStream_t st) {
+void launch_merge(const Params &p, const void *gathered, uint32_t world, long long *gcum, cudaStream_t st) {
   const size_t stride = pack_layout(p).total;
   unsigned P = 1;
   while (P < world * p.k) P <<= 1;
   const size_t sm = (size_t)P * 20;  // cand + full_ent (u64) + sec (u32)
   if (sm > 48 * 1024) cudaFuncSetAttribute(k_merge_windows, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
   { k_merge_windows<<<p.W, 256, sm, st>>>(p, static_cast<const unsigned char *>(gathered), world, stride); count_launch(); }
-  { k_merge_tables<<<256, 256, 0, st>>>(p, static_cast<const unsigned char *>(gathered), world, stride); count_launch(); }
+  { k_merge_progress<<<p.nk, 1024, 0, st>>>(p, static_cast<const unsigned char *>(gathered), world, stride, gcum); count_launch(); }
 }
 
 }  // namespace rtm

@@ -222,6 +222,37 @@ def test_case_study_deadlock_on_gpu():
     assert [list(mon.hang_check(w)) for w in range(6)] == [[], [], [], [], [1, 2], [0, 1, 2, 3]]
 
 
+def _merge_shards(mons, packs, n_windows):
+    """The exchange of the two-phase API for shard contexts on one GPU: every shard merges the
+    concatenated per-call packs (rtm_merge), then the on-demand tables (rtm_tables_local /
+    rtm_tables_merge).  Returns each shard's merged results."""
+    import ctypes
+
+    from paper_conf_micro_mosallaeii024_b200 import _copy_from_ptr
+
+    G = len(mons)
+    gathered = torch.cat(packs)
+    outs = []
+    for m in mons:
+        summ = np.zeros(n_windows, N.SUMMARY_DTYPE)
+        N.check(N.lib().rtm_merge(m._h, gathered.data_ptr(), G, summ.ctypes.data), "merge")
+        m.W = n_windows
+        outs.append((m.results(), summ))
+    tabs = []
+    for m in mons:
+        pack, nbytes = ctypes.c_void_p(), ctypes.c_uint64()
+        N.check(N.lib().rtm_tables_local(m._h, ctypes.byref(pack), ctypes.byref(nbytes)), "tables_local")
+        t = torch.empty(int(nbytes.value), dtype=torch.uint8, device="cuda")
+        _copy_from_ptr(t, pack.value, int(nbytes.value))
+        tabs.append(t)
+    torch.cuda.synchronize()
+    tg = torch.cat(tabs)
+    for m in mons:
+        N.check(N.lib().rtm_tables_merge(m._h, tg.data_ptr(), G), "tables_merge")
+        m._synced = True
+    return outs
+
+
 SHARD_RANKINGS = [(0, None), (1, None), (2, None), (2, 512)]  # (rank_mode, k); k=512 > owned per rank
 
 
@@ -253,12 +284,7 @@ def test_virtual_shards_merge_equals_whole(mode, k):
         torch.cuda.synchronize()
         mons.append(m)
         packs.append(t)
-    gathered = torch.cat(packs)
-    for m in mons:
-        summ = np.zeros(wl.n_windows, N.SUMMARY_DTYPE)
-        N.check(N.lib().rtm_merge(m._h, gathered.data_ptr(), G, summ.ctypes.data), "merge")
-        m.W = wl.n_windows
-        got = m.results()
+    for m, (got, summ) in zip(mons, _merge_shards(mons, packs, wl.n_windows)):
         assert np.array_equal(got["summary"], summ)
         assert_same(got, ref, m)
         assert np.array_equal(m.topk_persistence(), orc.persistence())  # counted from the merged lists
@@ -463,12 +489,7 @@ def test_rank_local_numbering_shards_merge_equals_whole(mode, k):
         mons.append(m)
         packs.append(t)
     assert len({int(t.numel()) for t in packs}) == 1  # equal-size packs (pack_buffers)
-    gathered = torch.cat(packs)
-    for m in mons:
-        summ = np.zeros(wl.n_windows, N.SUMMARY_DTYPE)
-        N.check(N.lib().rtm_merge(m._h, gathered.data_ptr(), G, summ.ctypes.data), "merge")
-        m.W = wl.n_windows
-        got = m.results()
+    for m, (got, summ) in zip(mons, _merge_shards(mons, packs, wl.n_windows)):
         assert np.array_equal(got["summary"], summ)
         assert_same(got, ref, m)
         assert np.array_equal(m.topk_persistence(), orc.persistence())  # counted from the merged lists
