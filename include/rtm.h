@@ -182,8 +182,8 @@ rtm_status rtm_ingest(rtm_ctx *ctx, const rtm_level_sample *samples, uint64_t n_
 
 /* THE HOT PATH.  Reduce all pending records over n_windows consecutive windows
  * [t_prev, t_end[0]), [t_end[0], t_end[1]), ... (t_end host array, non-decreasing,
- * t_end[0] >= t_prev, each window shorter than 2^40 ticks - 2^39 when 43520 < n_buffers <=
- * 87040, where bins of 512 buffers are used; else RTM_E_INVALID, no state change).  Records outside
+ * t_end[0] >= t_prev, each window shorter than 2^40 ticks, else RTM_E_INVALID with no state
+ * change).  Records outside
  * [t_prev, t_end[n-1]) are dropped and counted, not carried.  Blocks until the per-window
  * summaries, top-k lists and progress bars are on the host; `out` (host, nullable)
  * receives n_windows summaries.  With world > 1 every rank must call it with the same

@@ -663,9 +663,14 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
   c->nb = cfg->n_buffers;
   c->nc = cfg->n_components;
   c->nk = cfg->n_kernels;
-  // 256 buffers per bin; 512 when that keeps the bins within the lane-major partition's 170 (nb
-  // 43521 .. 87040, e.g. C3's 81920: otherwise 320 bins take the match-based fallback)
-  c->bin_log = (c->nb > 170u * 256u && c->nb <= 170u * 512u) ? 9 : 8;
+  // 256 buffers per bin; 128 for large registries (131073 .. 524288 buffers, e.g. C5's 327680):
+  // very sparse windows are folded by one warp per bin walking the windows in order, and halving
+  // the bin doubles the warps (the partition fallback takes up to 4096 bins)
+  c->bin_log = (c->nb > 131072u && c->nb <= kMaxBins * 128u) ? 7 : 8;
+#ifdef RTM_FORCE_BIN_LOG  // compile-time A/B builds only (tools/build_variant.sh)
+  c->bin_log = RTM_FORCE_BIN_LOG;
+  if (c->nb > kMaxBins * (1u << c->bin_log)) c->bin_log = 8;
+#endif
   c->nbins = (c->nb + (1u << c->bin_log) - 1) >> c->bin_log;
   c->ncw = (c->nc + 31) / 32;
   c->k = cfg->k;

@@ -37,7 +37,7 @@ constexpr uint16_t kSent = 0xFFFFu;         // "no kept sample in this window" m
 constexpr uint32_t kMaxBins = 4096;         // n_buffers <= 2^20 (fallback partition smem 160 KB)
 constexpr uint32_t kTopkSmemKeys = 40960;   // keys held in shared memory by the top-k kernel
 // ts offset field of a staging entry: 48 - bin_log bits (entry = off << (16 + bin_log) | level << bin_log | lid)
-inline int64_t max_window_len(int bin_log) { return (int64_t)1 << (48 - bin_log); }
+inline int64_t max_window_len(int bin_log) { return (int64_t)1 << (bin_log >= 8 ? 40 : 48 - bin_log > 40 ? 40 : 48 - bin_log); }
 
 // per-window scalar accumulators, SoA [kWinFields][W] u64
 enum { WF_SAMPLES = 0, WF_EVENTS, WF_DROPPED, WF_DIGEST, WF_TOUCHED, WF_HUNG, kWinFields };
@@ -71,7 +71,7 @@ struct KernelTimer {
 struct Params {
   // registry
   uint32_t nb, nc, nk, nbins, ncw, k;
-  int32_t bin_log;           // buffers per bin = 2^bin_log (8 or 9)
+  int32_t bin_log;           // buffers per bin = 2^bin_log (8, or 7 for large registries)
   int32_t rank_mode;
   uint32_t H;
   int32_t hang_mode;         // RTM_HANG_FULL / RTM_HANG_NONEMPTY

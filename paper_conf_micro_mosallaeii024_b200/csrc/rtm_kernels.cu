@@ -575,14 +575,7 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
     const bool valid = (sub0 + i < t.n) & (b < p.nb) & (c == capb) & (lvl <= c);
     const unsigned long long off = (unsigned long long)(rec_ts(v) - t.lo);
     hv |= valid;
-    if (NAR && BL != 8) {  // (o << (16 + BL)) | (level << BL) | (buffer_id & (2^BL - 1)), o < 2^32
-      const unsigned o = (unsigned)off;
-      bad |= valid & (o < mx);
-      mx = max(mx, valid ? o : 0u);
-      mn = min(mn, valid ? o : ~0u);
-      hiacc |= valid ? (unsigned)(off >> 32) : 0u;
-      e[k] = ((unsigned long long)o << (16 + BL)) | ((unsigned long long)lvl << BL) | (b & ((1u << BL) - 1u));
-    } else if (NAR) {
+    if (NAR) {
       const unsigned o = (unsigned)off;
       bad |= valid & (o < mx);
       mx = max(mx, valid ? o : 0u);
@@ -637,6 +630,7 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
 // stores from every lane, which touched 32 sectors per store instruction).
 template <int BL, bool CAPS>
 __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
+  static_assert(BL == 8, "lane-major entries pack the buffer id in one byte");
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ K1WarpSum wsum[2][kK1Warps];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -862,6 +856,7 @@ __device__ __forceinline__ unsigned k1_bin_bases_cta(const Params &p, unsigned t
   return carry;
 }
 
+template <int BL>
 __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ K1WarpSum wsum[kK1Warps];
@@ -916,7 +911,7 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
       }
       const bool keep = valid & is_win;
       kept += keep;
-      const unsigned key = keep ? (b >> 8) : kNoKey;  // the fallback runs with 256-buffer bins
+      const unsigned key = keep ? (b >> BL) : kNoKey;
       unsigned pos = 0;
       if (is_win) {  // CTA-uniform
         // (per-bit ballots instead of MATCH measured equal on C3 / C4: the fallback is latency-bound)
@@ -928,7 +923,7 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
         pos = basec + __popc(peers & lt);
       }
       kp[j] = (key << 16) | pos;
-      e[j] = (off << 24) | ((unsigned long long)lvl << 8) | (b & 255u);
+      e[j] = (off << (16 + BL)) | ((unsigned long long)lvl << BL) | (b & ((1u << BL) - 1u));
     }
   }
   k1_publish(wsum, first, last, has, viol, kept);
@@ -1198,30 +1193,35 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
     }
     unsigned long long dig = 0;
     unsigned touched = 0;
-    const bool last_window = (w == p.W - 1);
-#pragma unroll
-    for (int i = 0; i < FS::kB / 32; ++i) {
-      const unsigned l = lane + 32 * i, b = b_base + l;
-      if (b >= p.nb) continue;
-      const unsigned L = lin[i];
+    // the window's statistics of buffer slot i (carry-in L_in = lin[i] resolved above)
+    auto stat_of = [&](int i, unsigned long long &I, unsigned &mx, unsigned &mn, unsigned &last) -> unsigned {
+      const unsigned l = lane + 32 * i, L = lin[i];
       const uint4 sv = S.st[l];
       const unsigned hw = S.hi[l];
-      const unsigned cnt = st_touched(sv) ? ((hw & 0xFFFFu) << 16) + (sv.w >> 16) : 0u;
-      unsigned long long I;
-      unsigned mx, mn, last;
-      if (cnt) {
+      if (st_touched(sv)) {
         const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
         I = (unsigned long long)L * (((unsigned long long)(hw >> 16) << 32) | S.ts0[l]) + st_D(sv);
         mx = hi > L ? hi : L;
         mn = lo < L ? lo : L;
         last = sv.z & 0xFFFFu;
-      } else {
-        I = (unsigned long long)L * Wlen;
-        mx = mn = last = L;
-        lw[b] = (uint16_t)L;  // resolve the untouched cell
+        return ((hw & 0xFFFFu) << 16) + (sv.w >> 16);
       }
-      const unsigned capb = __ldg(p.cap + b);
-      if (p.mkey) p.mkey[(size_t)w * p.nb + b] = mean_key(I, capb, p.rcp64);
+      I = (unsigned long long)L * Wlen;
+      mx = mn = last = L;
+      return 0u;
+    };
+    const unsigned nb = p.nb;
+    const unsigned short *capp = p.cap;
+#pragma unroll
+    for (int i = 0; i < FS::kB / 32; ++i) {
+      const unsigned b = b_base + lane + 32 * i;
+      if (b >= nb) continue;
+      unsigned long long I;
+      unsigned mx, mn, last;
+      const unsigned cnt = stat_of(i, I, mx, mn, last);
+      if (!cnt) lw[b] = (uint16_t)last;  // resolve the untouched cell
+      const unsigned capb = __ldg(capp + b);
+      if (p.mkey) p.mkey[(size_t)w * nb + b] = mean_key(I, capb, p.rcp64);
       if (p.hang_mode == RTM_HANG_NONEMPTY ? mn >= 1u : mn == capb) {  // held the whole window
         const unsigned c = __ldg(p.owner + b);
         atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
@@ -1242,10 +1242,23 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
         dig += h;
         ++touched;
       }
-      int wq = -1;  // value monitor slot of b (at most RTM_WATCH_MAX compares, usually none)
-      for (unsigned q = 0; q < p.n_watch; ++q)
-        if (p.watch[q] == b) wq = (int)q;
-      if (last_window || wq >= 0) {
+    }
+    // rare, uniform: the call's last window (per-buffer table, next call's carry) and the value
+    // monitor's watched buffers - a second pass, so the loop above stays small
+    const bool last_window = (w == p.W - 1);
+    if (last_window || p.n_watch) {
+#pragma unroll
+      for (int i = 0; i < FS::kB / 32; ++i) {
+        const unsigned b = b_base + lane + 32 * i;
+        if (b >= nb) continue;
+        int wq = -1;  // value monitor slot of b (at most RTM_WATCH_MAX compares)
+        for (unsigned q = 0; q < p.n_watch; ++q)
+          if (p.watch[q] == b) wq = (int)q;
+        if (!last_window && wq < 0) continue;
+        unsigned long long I;
+        unsigned mx, mn, last;
+        const unsigned cnt = stat_of(i, I, mx, mn, last);
+        const unsigned capb = __ldg(capp + b);
         rtm_buffer_stat st;
         st.integral = (int64_t)I;
         st.last = (uint16_t)last;
@@ -1272,33 +1285,13 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
   }
 }
 
-// SPARSE (few samples per unit: C3-C5 shapes): many of a unit's 256 buffers are untouched in
-// several consecutive windows, so the look-back walks several windows; it takes RTM_LB_STEP of
-// them per step (their flags waited for by as many lanes, all rows loaded before any is used),
-// dividing the dependent round trips.  A separate instantiation: the dense (C2) code is unchanged.
-template <bool NAR, bool SPARSE, int BL>
-__global__ void __launch_bounds__(kFoldWarps * 32, (BL == 8 ? 32 : 16) / kFoldWarps) k_fold(Params p) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  using FS = FoldSmem<BL>;
-  FS &S = reinterpret_cast<FS *>(smem)[threadIdx.x >> 5];
-  const int lane = threadIdx.x & 31;
-  const unsigned lt = lanemask_lt();
-  const unsigned n_units = p.W * p.nbins;
-  for (;;) {
-    unsigned u = 0;
-    if (lane == 0) u = atomicAdd(p.unit_ctr, 1u);
-    u = __shfl_sync(kFull, u, 0);
-    if (u >= n_units) break;
-    const unsigned w = u / p.nbins, bin = u % p.nbins;
-    const long long tb = p.T[w], te = p.T[w + 1];
-    const unsigned long long Wlen = (unsigned long long)(te - tb);
-    const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
-#pragma unroll
-    for (int i = 0; i < FS::kB / 32; ++i) {
-      S.st[lane + 32 * i] = make_uint4(0, 0, kUntouchedZ, 0);
-      S.hi[lane + 32 * i] = 0;
-    }
-    __syncwarp();
+// Phase 1 of a fold unit (window w, bin): the (tile, bin) segments of window w flattened into one
+// stream of 32-sample chunks, each folded by fold_chunk into S (carry-in left symbolic).
+template <bool NAR, int BL>
+__device__ __forceinline__ void fold_phase1(const Params &p, FoldSmem<BL> &S, unsigned w, unsigned bin,
+                                            unsigned long long Wlen, int lane, unsigned lt) {
+  const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
+  {
     // ---- phase 1: the (tile, bin) segments of window w, flattened into one stream of chunks
     for (unsigned tg = t_lo; tg < t_hi; tg += 32) {
       unsigned seg_lo = 0, seg_len = 0;
@@ -1343,7 +1336,232 @@ __global__ void __launch_bounds__(kFoldWarps * 32, (BL == 8 ? 32 : 16) / kFoldWa
         e1 = en;
       }
     }
+  }
+}
+
+// SPARSE (few samples per unit: C3-C5 shapes): many of a unit's 256 buffers are untouched in
+// several consecutive windows, so the look-back walks several windows; it takes RTM_LB_STEP of
+// them per step (their flags waited for by as many lanes, all rows loaded before any is used),
+// dividing the dependent round trips.  A separate instantiation: the dense (C2) code is unchanged.
+template <bool NAR, bool SPARSE, int BL>
+__global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Params p) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  using FS = FoldSmem<BL>;
+  FS &S = reinterpret_cast<FS *>(smem)[threadIdx.x >> 5];
+  const int lane = threadIdx.x & 31;
+  const unsigned lt = lanemask_lt();
+  const unsigned n_units = p.W * p.nbins;
+  for (;;) {
+    unsigned u = 0;
+    if (lane == 0) u = atomicAdd(p.unit_ctr, 1u);
+    u = __shfl_sync(kFull, u, 0);
+    if (u >= n_units) break;
+    const unsigned w = u / p.nbins, bin = u % p.nbins;
+    const long long tb = p.T[w], te = p.T[w + 1];
+    const unsigned long long Wlen = (unsigned long long)(te - tb);
+#pragma unroll
+    for (int i = 0; i < FS::kB / 32; ++i) {
+      S.st[lane + 32 * i] = make_uint4(0, 0, kUntouchedZ, 0);
+      S.hi[lane + 32 * i] = 0;
+    }
+    __syncwarp();
+    fold_phase1<NAR, BL>(p, S, w, bin, Wlen, lane, lt);
     fold_finish<NAR, SPARSE>(p, S, w, bin, Wlen, lane);
+  }
+}
+
+// ============================================================================================
+// K2 for very sparse calls (C5: ~0.02 kept samples per buffer and window): one warp per bin
+// walks ALL windows of the call in order, so every buffer's carry-in is known when its window is
+// finalized (no published rows to look back through) and the per-window work is proportional to
+// the window's records, not to the bin's 256 buffers:
+//   - the window's samples are folded by fold_phase1 (as in k_fold);
+//   - only touched buffers are finalized (integral, max / min with the carry-in, digest, count),
+//     their carried level advanced and their state reset;
+//   - every buffer still gets its cell of the window's last-level row (the top-k ranks all
+//     buffers) and its held-full bit (hang, R9), from the carried level when untouched.
+// Lane l owns buffers l + 32 i (i < 8) of the bin; their capacities and owners stay in registers
+// for the whole call, their carried levels in shared memory.  Rank mode MEAN (a 64-bit key per
+// buffer and window) keeps the windowed k_fold.
+// ============================================================================================
+template <int BL>
+struct FoldSeqSmem {
+  static constexpr int kB = 1 << BL, kPer = kB / 32;
+  FoldSmem<BL> f;
+  unsigned short lvl[kB];   // carried level of every buffer of the bin
+  unsigned short list[kB];  // the window's touched buffers (compacted)
+  unsigned short capS[kB];  // capacities and owners of the bin (the touched finalize reads them)
+  unsigned ownS[kB];
+  unsigned tmask[kPer];     // the window's touched buffers (bit lid)
+};
+
+template <bool NAR, int BL>
+__global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  using QS = FoldSeqSmem<BL>;
+  constexpr int kB = QS::kB, kPer = QS::kPer;
+  QS &Q = reinterpret_cast<QS *>(smem)[threadIdx.x >> 5];
+  FoldSmem<BL> &S = Q.f;
+  const int lane = threadIdx.x & 31;
+  const unsigned lt = lanemask_lt();
+  const bool nonempty_mode = p.hang_mode == RTM_HANG_NONEMPTY;
+  for (;;) {
+    unsigned bin = 0;
+    if (lane == 0) bin = atomicAdd(p.unit_ctr, 1u);
+    bin = __shfl_sync(kFull, bin, 0);
+    if (bin >= p.nbins) break;
+    const unsigned b_base = bin * (unsigned)kB;
+    // this lane's contiguous buffers kPer lane .. kPer lane + kPer - 1 (row stores, held-full bits)
+    const unsigned c0 = b_base + kPer * lane;
+    const bool vec = (p.nb & (kPer - 1)) == 0;  // aligned row segments
+    unsigned capv[kPer], ownv[kPer];
+#pragma unroll
+    for (int j = 0; j < kPer; ++j) {
+      const unsigned b = c0 + j;
+      capv[j] = b < p.nb ? __ldg(p.cap + b) : 0xFFFFu;
+      ownv[j] = b < p.nb ? __ldg(p.owner + b) : 0;
+    }
+#pragma unroll
+    for (int i = 0; i < kPer; ++i) {
+      const unsigned l = lane + 32 * i, b = b_base + l;
+      S.st[l] = make_uint4(0, 0, kUntouchedZ, 0);
+      S.hi[l] = 0;
+      Q.lvl[l] = b < p.nb ? __ldg(p.carry_in + b) : 0;
+      Q.capS[l] = b < p.nb ? __ldg(p.cap + b) : 0xFFFFu;
+      Q.ownS[l] = b < p.nb ? __ldg(p.owner + b) : 0;
+    }
+    __syncwarp();
+    for (unsigned w = 0; w < p.W; ++w) {
+      const long long tb = p.T[w], te = p.T[w + 1];
+      const unsigned long long Wlen = (unsigned long long)(te - tb);
+      const bool last_window = (w == p.W - 1);
+      fold_phase1<NAR, BL>(p, S, w, bin, Wlen, lane, lt);
+      __syncwarp();
+      // ---- compact the touched buffers (owner-strided scan of the state)
+      unsigned nt = 0;
+#pragma unroll
+      for (int i = 0; i < kPer; ++i) {
+        const bool t = st_touched(S.st[lane + 32 * i]);
+        const unsigned m = __ballot_sync(kFull, t);
+        if (t) Q.list[nt + __popc(m & lt)] = (unsigned short)(lane + 32 * i);
+        if (lane == 0) Q.tmask[i] = m;
+        nt += __popc(m);
+      }
+      __syncwarp();
+      // ---- finalize the touched buffers, 32 at a time
+      unsigned long long dig = 0;
+      for (unsigned q0 = 0; q0 < nt; q0 += 32) {
+        const unsigned q = q0 + lane;
+        if (q < nt) {
+          const unsigned l = Q.list[q], b = b_base + l;
+          const unsigned L = Q.lvl[l];
+          const uint4 sv = S.st[l];
+          const unsigned hw = S.hi[l];
+          const unsigned cnt = ((hw & 0xFFFFu) << 16) + (sv.w >> 16);
+          const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
+          const unsigned long long I =
+              (unsigned long long)L * (((unsigned long long)(hw >> 16) << 32) | S.ts0[l]) + st_D(sv);
+          const unsigned mx = hi > L ? hi : L, mn = lo < L ? lo : L, last = sv.z & 0xFFFFu;
+          const unsigned capb = Q.capS[l];
+          const unsigned bid = p.gid ? __ldg(p.gid + b) : b;
+          unsigned long long h = (I * 0x9E3779B97F4A7C15ULL) ^
+                                 ((((unsigned long long)cnt << 32) | bid) * 0xC2B2AE3D27D4EB4FULL) ^
+                                 (((unsigned long long)last | ((unsigned long long)mx << 16) |
+                                   ((unsigned long long)mn << 32) | ((unsigned long long)capb << 48)) *
+                                  0x165667B19E3779F9ULL);
+          h ^= h >> 30;
+          h *= 0xbf58476d1ce4e5b9ULL;
+          h ^= h >> 27;
+          h *= 0x94d049bb133111ebULL;
+          h ^= h >> 31;
+          dig += h;
+          if (nonempty_mode ? mn >= 1u : mn == capb) {  // held the whole window
+            const unsigned c = Q.ownS[l];
+            atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
+          }
+          if (last_window || p.n_watch) {  // rare: the call's table, the value monitor
+            int wq = -1;
+            for (unsigned k2 = 0; k2 < p.n_watch; ++k2)
+              if (p.watch[k2] == b) wq = (int)k2;
+            if (last_window || wq >= 0) {
+              rtm_buffer_stat st;
+              st.integral = (int64_t)I;
+              st.last = (uint16_t)last;
+              st.max = (uint16_t)mx;
+              st.min = (uint16_t)mn;
+              st.capacity = (uint16_t)capb;
+              st.n_samples = cnt;
+              st.reserved = __ldg(p.elig + b);
+              st.mean_occ = Wlen ? __ddiv_rn((double)(long long)I, (double)((long long)capb * (long long)Wlen)) : 0.0;
+              if (wq >= 0) p.wstat[(size_t)w * RTM_WATCH_MAX + wq] = st;
+              if (last_window) {
+                p.bstat[b] = st;
+                p.carry_out[b] = (uint16_t)last;
+              }
+            }
+          }
+          Q.lvl[l] = (unsigned short)last;
+          S.st[l] = make_uint4(0, 0, kUntouchedZ, 0);
+          S.hi[l] = 0;
+        }
+      }
+      __syncwarp();
+      // ---- the window's last-level row (every buffer) and the untouched buffers' held-full bits
+      uint16_t *lw = p.lastlvl + (size_t)w * p.nb;
+      unsigned lvw[kPer / 2];  // levels of c0 .. c0 + kPer - 1, two per word
+      if constexpr (kPer == 8) {
+        const uint4 v = reinterpret_cast<const uint4 *>(Q.lvl)[lane];
+        lvw[0] = v.x; lvw[1] = v.y; lvw[2] = v.z; lvw[3] = v.w;
+        if (vec && c0 < p.nb) reinterpret_cast<uint4 *>(lw + b_base)[lane] = v;
+      } else {
+        const uint2 v = reinterpret_cast<const uint2 *>(Q.lvl)[lane];
+        lvw[0] = v.x; lvw[1] = v.y;
+        if (vec && c0 < p.nb) reinterpret_cast<uint2 *>(lw + b_base)[lane] = v;
+      }
+      if (!vec) {
+#pragma unroll
+        for (int j = 0; j < kPer; ++j)
+          if (c0 + j < p.nb) lw[c0 + j] = (uint16_t)(lvw[j >> 1] >> (16 * (j & 1)));
+      }
+      const unsigned tb8 = (Q.tmask[(kPer * lane) >> 5] >> ((kPer * lane) & 31)) & ((1u << kPer) - 1u);
+#pragma unroll
+      for (int j = 0; j < kPer; ++j) {
+        const unsigned L = (lvw[j >> 1] >> (16 * (j & 1))) & 0xFFFFu;
+        if (!((tb8 >> j) & 1u) && c0 + j < p.nb && (nonempty_mode ? L >= 1u : L == capv[j]))
+          atomicOr(p.anyfull + (size_t)w * p.ncw + (ownv[j] >> 5), 1u << (ownv[j] & 31));
+      }
+      if (last_window || p.n_watch) {  // rare: untouched buffers' statistics
+#pragma unroll
+        for (int j = 0; j < kPer; ++j) {
+          const unsigned b = c0 + j;
+          if (b >= p.nb || ((tb8 >> j) & 1u)) continue;
+          int wq = -1;
+          for (unsigned k2 = 0; k2 < p.n_watch; ++k2)
+            if (p.watch[k2] == b) wq = (int)k2;
+          if (!last_window && wq < 0) continue;
+          const unsigned L = Q.lvl[kPer * lane + j];
+          rtm_buffer_stat st;
+          st.integral = (int64_t)((unsigned long long)L * Wlen);
+          st.last = st.max = st.min = (uint16_t)L;
+          st.capacity = (uint16_t)capv[j];
+          st.n_samples = 0;
+          st.reserved = __ldg(p.elig + b);
+          st.mean_occ = Wlen ? __ddiv_rn((double)(long long)((unsigned long long)L * Wlen),
+                                         (double)((long long)capv[j] * (long long)Wlen)) : 0.0;
+          if (wq >= 0) p.wstat[(size_t)w * RTM_WATCH_MAX + wq] = st;
+          if (last_window) {
+            p.bstat[b] = st;
+            p.carry_out[b] = (uint16_t)L;
+          }
+        }
+      }
+      dig = warp_sum(dig);
+      if (lane == 0) {
+        if (dig) atomicAdd(p.win + WF_DIGEST * p.W + w, dig);
+        if (nt) atomicAdd(p.win + WF_TOUCHED * p.W + w, (unsigned long long)nt);
+      }
+      __syncwarp();
+    }
   }
 }
 
@@ -2274,7 +2492,7 @@ void launch_clear(const ClearList &cl, cudaStream_t st) {
 }
 
 size_t fold_smem_bytes(int bin_log) {
-  return (bin_log == 9 ? sizeof(FoldSmem<9>) : sizeof(FoldSmem<8>)) * kFoldWarps;
+  return (bin_log == 7 ? sizeof(FoldSmem<7>) : sizeof(FoldSmem<8>)) * kFoldWarps;
 }
 // lane-major partition: the capacity table in shared memory when two CTAs still fit per SM
 bool partition_caps_smem(uint32_t nbins, uint32_t nb) { return k1_smem_lm(nbins, nb, true) + 1024 <= 113 * 1024; }
@@ -2321,16 +2539,12 @@ void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   if (!p.n_tiles_s) return;
   const size_t sm = partition_smem_bytes(p.nbins, p.nb);
   if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM
-    const bool caps = partition_caps_smem(p.nbins, p.nb);
-    if (p.bin_log == 9) {
-      if (caps) launch_partition_lm<9, true>(p, n_sms, sm, st);
-      else launch_partition_lm<9, false>(p, n_sms, sm, st);
-    } else {
-      if (caps) launch_partition_lm<8, true>(p, n_sms, sm, st);
-      else launch_partition_lm<8, false>(p, n_sms, sm, st);
-    }
+    // bin_log 8 here: bin_log 7 is only chosen for > 131072 buffers (> 170 bins)
+    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true>(p, n_sms, sm, st);
+    else launch_partition_lm<8, false>(p, n_sms, sm, st);
   } else {
-    { k_partition_mx<<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
+    if (p.bin_log == 7) { k_partition_mx<7><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
+    else { k_partition_mx<8><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
   }
 }
 
@@ -2351,16 +2565,40 @@ void launch_fold_bl(const Params &p, int n_sms, cudaStream_t st) {
   const unsigned need = (units + kFoldWarps - 1) / kFoldWarps;
   if (grid > need) grid = need;
   if (grid == 0) grid = 1;
-  // sparse units: fewer than 512 kept samples per (window, bin) on average
-  const bool sparse = p.ns < (uint64_t)512 * units;
+  // sparse: fewer than 2 samples per buffer and window on average (C3-C5 shapes), so many of a
+  // unit's buffers are untouched and the look-back walks several windows
+  const bool sparse = p.ns < 2ull * p.nb * p.W;
   if (p.narrow && sparse) { k_fold<true, true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else if (p.narrow) { k_fold<true, false, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else if (sparse) { k_fold<false, true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else { k_fold<false, false, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
 }
 
+// very sparse calls: fewer than 1 kept sample per 8 buffer-windows (C5 ~ 1 in 45); PERCENT / SIZE
+bool fold_sequential(const Params &p) {
+  return !p.mkey && p.W > 1 && (unsigned long long)p.ns * 8ull < (unsigned long long)p.nb * p.W;
+}
+
+template <int BL>
+void launch_fold_seq(const Params &p, int n_sms, cudaStream_t st) {
+  const size_t sm = sizeof(FoldSeqSmem<BL>) * kFoldWarps;
+  int per_sm = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fold_seq<true, BL>, kFoldWarps * 32, sm);
+  if (per_sm < 1) per_sm = 1;
+  unsigned grid = (unsigned)(n_sms * per_sm);
+  const unsigned need = (p.nbins + kFoldWarps - 1) / kFoldWarps;
+  if (grid > need) grid = need;
+  if (p.narrow) { k_fold_seq<true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else { k_fold_seq<false, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+}
+
 void launch_fold(const Params &p, int n_sms, cudaStream_t st) {
-  if (p.bin_log == 9) launch_fold_bl<9>(p, n_sms, st);
+  if (fold_sequential(p)) {
+    if (p.bin_log == 7) launch_fold_seq<7>(p, n_sms, st);
+    else launch_fold_seq<8>(p, n_sms, st);
+    return;
+  }
+  if (p.bin_log == 7) launch_fold_bl<7>(p, n_sms, st);
   else launch_fold_bl<8>(p, n_sms, st);
 }
 
@@ -2433,17 +2671,20 @@ void configure_kernels_once() {
   const int lm_glob = (int)k1_smem_lm(kLmMaxBins, 0, false);
   cudaFuncSetAttribute(k_partition_lm<8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
   cudaFuncSetAttribute(k_partition_lm<8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
-  cudaFuncSetAttribute(k_partition_lm<9, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
-  cudaFuncSetAttribute(k_partition_lm<9, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
-  cudaFuncSetAttribute(k_partition_mx, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
+  cudaFuncSetAttribute(k_partition_mx<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
+  cudaFuncSetAttribute(k_partition_mx<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
   cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
   cudaFuncSetAttribute(k_topk<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)topk_smem_bytes(kTopkSmemKeys));
 #define RTM_FOLD_ATTR(NAR_, SP_, BL_) \
   cudaFuncSetAttribute(k_fold<NAR_, SP_, BL_>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes(BL_))
   RTM_FOLD_ATTR(true, false, 8); RTM_FOLD_ATTR(false, false, 8); RTM_FOLD_ATTR(true, true, 8); RTM_FOLD_ATTR(false, true, 8);
-  RTM_FOLD_ATTR(true, false, 9); RTM_FOLD_ATTR(false, false, 9); RTM_FOLD_ATTR(true, true, 9); RTM_FOLD_ATTR(false, true, 9);
+  RTM_FOLD_ATTR(true, false, 7); RTM_FOLD_ATTR(false, false, 7); RTM_FOLD_ATTR(true, true, 7); RTM_FOLD_ATTR(false, true, 7);
 #undef RTM_FOLD_ATTR
+  cudaFuncSetAttribute(k_fold_seq<true, 7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<7>) * kFoldWarps));
+  cudaFuncSetAttribute(k_fold_seq<false, 7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<7>) * kFoldWarps));
+  cudaFuncSetAttribute(k_fold_seq<true, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<8>) * kFoldWarps));
+  cudaFuncSetAttribute(k_fold_seq<false, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<8>) * kFoldWarps));
   cudaGetLastError();
 }
 

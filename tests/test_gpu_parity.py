@@ -840,3 +840,41 @@ def test_merge_pending_state_and_world_k_limit():
         m.W = wl.n_windows
         assert_same(m.results(), ref, m)
     assert N.lib().rtm_merge(m._h, t.data_ptr(), 1, summ.ctypes.data) == N.RTM_E_STATE
+
+
+@pytest.mark.parametrize("hang_mode", [0, 1])
+def test_very_sparse_calls_sequential_fold(hang_mode):
+    """Calls with fewer than one kept sample per 8 buffer-windows (C5's shape: ~1 in 45) take the
+    sequential fold (one warp per bin walks the call's windows, only touched buffers finalized).
+    40 000 buffers, 900 windows in calls of 1, 299 and 600 windows, 0.02-0.05 samples per
+    buffer-window, H small enough to flag components, watched buffers: every window's summary,
+    top-k, progress, hang list, the last window's table and the value-monitor rings equal the
+    oracle's."""
+    wl = gen.C5.scaled("C5-seq", n_samples=1_200_000, n_events=120_000, n_buffers=40_000, n_windows=900,
+                       hang_windows=6)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=6, k=wl.k, hang_mode=hang_mode)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    watched = [0, 12345, 39999]
+    mon.watch(watched)
+    s, e = gen.samples(wl), gen.events(wl)
+    t_end = wl.t_end()
+    rows, w0, flagged = [], 0, 0
+    for m in (1, 299, 600):
+        w1 = w0 + m
+        sl = slice(wl.index_at("samples", wl.t_begin(w0)), wl.index_at("samples", wl.t_begin(w1)))
+        el = slice(wl.index_at("events", wl.t_begin(w0)), wl.index_at("events", wl.t_begin(w1)))
+        assert (sl.stop - sl.start) * 8 < wl.n_buffers * m or m == 1  # the sequential path (W > 1)
+        ref = orc.reduce(s[sl], e[el], t_end[w0:w1], want_all_stats=True)
+        rows.append(ref["all_stats"])
+        mon.ingest(_dev(s[sl]), _dev(e[el]))
+        got = mon.window_reduce(t_end[w0:w1])
+        assert_same(got, ref, mon)
+        flagged += int(ref["summary"]["n_hung"].sum())
+        w0 = w1
+    assert flagged > 0
+    A = np.concatenate(rows)
+    for q, b in enumerate(watched):
+        ser = mon.watch_series(q)
+        for f in ("integral", "last", "max", "min", "capacity", "n_samples", "mean_occ"):
+            assert np.array_equal(ser[f], A[-300:, b][f]), (b, f)
