@@ -1431,137 +1431,222 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
       Q.ownS[l] = b < p.nb ? __ldg(p.owner + b) : 0;
     }
     __syncwarp();
-    for (unsigned w = 0; w < p.W; ++w) {
-      const long long tb = p.T[w], te = p.T[w + 1];
-      const unsigned long long Wlen = (unsigned long long)(te - tb);
+    // finalize of window w (its samples are folded into S): touched buffers, the last-level row,
+    // held-full bits, the window's digest and touched count
+    auto finalize = [&](unsigned w, unsigned long long Wlen) {
       const bool last_window = (w == p.W - 1);
-      fold_phase1<NAR, BL>(p, S, w, bin, Wlen, lane, lt);
-      __syncwarp();
-      // ---- compact the touched buffers (owner-strided scan of the state)
-      unsigned nt = 0;
+        // ---- compact the touched buffers (owner-strided scan of the state)
+        unsigned nt = 0;
 #pragma unroll
-      for (int i = 0; i < kPer; ++i) {
-        const bool t = st_touched(S.st[lane + 32 * i]);
-        const unsigned m = __ballot_sync(kFull, t);
-        if (t) Q.list[nt + __popc(m & lt)] = (unsigned short)(lane + 32 * i);
-        if (lane == 0) Q.tmask[i] = m;
-        nt += __popc(m);
-      }
-      __syncwarp();
-      // ---- finalize the touched buffers, 32 at a time
-      unsigned long long dig = 0;
-      for (unsigned q0 = 0; q0 < nt; q0 += 32) {
-        const unsigned q = q0 + lane;
-        if (q < nt) {
-          const unsigned l = Q.list[q], b = b_base + l;
-          const unsigned L = Q.lvl[l];
-          const uint4 sv = S.st[l];
-          const unsigned hw = S.hi[l];
-          const unsigned cnt = ((hw & 0xFFFFu) << 16) + (sv.w >> 16);
-          const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
-          const unsigned long long I =
-              (unsigned long long)L * (((unsigned long long)(hw >> 16) << 32) | S.ts0[l]) + st_D(sv);
-          const unsigned mx = hi > L ? hi : L, mn = lo < L ? lo : L, last = sv.z & 0xFFFFu;
-          const unsigned capb = Q.capS[l];
-          const unsigned bid = p.gid ? __ldg(p.gid + b) : b;
-          unsigned long long h = (I * 0x9E3779B97F4A7C15ULL) ^
-                                 ((((unsigned long long)cnt << 32) | bid) * 0xC2B2AE3D27D4EB4FULL) ^
-                                 (((unsigned long long)last | ((unsigned long long)mx << 16) |
-                                   ((unsigned long long)mn << 32) | ((unsigned long long)capb << 48)) *
-                                  0x165667B19E3779F9ULL);
-          h ^= h >> 30;
-          h *= 0xbf58476d1ce4e5b9ULL;
-          h ^= h >> 27;
-          h *= 0x94d049bb133111ebULL;
-          h ^= h >> 31;
-          dig += h;
-          if (nonempty_mode ? mn >= 1u : mn == capb) {  // held the whole window
-            const unsigned c = Q.ownS[l];
-            atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
+        for (int i = 0; i < kPer; ++i) {
+          const bool t = st_touched(S.st[lane + 32 * i]);
+          const unsigned m = __ballot_sync(kFull, t);
+          if (t) Q.list[nt + __popc(m & lt)] = (unsigned short)(lane + 32 * i);
+          if (lane == 0) Q.tmask[i] = m;
+          nt += __popc(m);
+        }
+        __syncwarp();
+        // ---- finalize the touched buffers, 32 at a time
+        unsigned long long dig = 0;
+        for (unsigned q0 = 0; q0 < nt; q0 += 32) {
+          const unsigned q = q0 + lane;
+          if (q < nt) {
+            const unsigned l = Q.list[q], b = b_base + l;
+            const unsigned L = Q.lvl[l];
+            const uint4 sv = S.st[l];
+            const unsigned hw = S.hi[l];
+            const unsigned cnt = ((hw & 0xFFFFu) << 16) + (sv.w >> 16);
+            const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
+            const unsigned long long I =
+                (unsigned long long)L * (((unsigned long long)(hw >> 16) << 32) | S.ts0[l]) + st_D(sv);
+            const unsigned mx = hi > L ? hi : L, mn = lo < L ? lo : L, last = sv.z & 0xFFFFu;
+            const unsigned capb = Q.capS[l];
+            const unsigned bid = p.gid ? __ldg(p.gid + b) : b;
+            unsigned long long h = (I * 0x9E3779B97F4A7C15ULL) ^
+                                   ((((unsigned long long)cnt << 32) | bid) * 0xC2B2AE3D27D4EB4FULL) ^
+                                   (((unsigned long long)last | ((unsigned long long)mx << 16) |
+                                     ((unsigned long long)mn << 32) | ((unsigned long long)capb << 48)) *
+                                    0x165667B19E3779F9ULL);
+            h ^= h >> 30;
+            h *= 0xbf58476d1ce4e5b9ULL;
+            h ^= h >> 27;
+            h *= 0x94d049bb133111ebULL;
+            h ^= h >> 31;
+            dig += h;
+            if (nonempty_mode ? mn >= 1u : mn == capb) {  // held the whole window
+              const unsigned c = Q.ownS[l];
+              atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
+            }
+            if (last_window || p.n_watch) {  // rare: the call's table, the value monitor
+              int wq = -1;
+              for (unsigned k2 = 0; k2 < p.n_watch; ++k2)
+                if (p.watch[k2] == b) wq = (int)k2;
+              if (last_window || wq >= 0) {
+                rtm_buffer_stat st;
+                st.integral = (int64_t)I;
+                st.last = (uint16_t)last;
+                st.max = (uint16_t)mx;
+                st.min = (uint16_t)mn;
+                st.capacity = (uint16_t)capb;
+                st.n_samples = cnt;
+                st.reserved = __ldg(p.elig + b);
+                st.mean_occ = Wlen ? __ddiv_rn((double)(long long)I, (double)((long long)capb * (long long)Wlen)) : 0.0;
+                if (wq >= 0) p.wstat[(size_t)w * RTM_WATCH_MAX + wq] = st;
+                if (last_window) {
+                  p.bstat[b] = st;
+                  p.carry_out[b] = (uint16_t)last;
+                }
+              }
+            }
+            Q.lvl[l] = (unsigned short)last;
+            S.st[l] = make_uint4(0, 0, kUntouchedZ, 0);
+            S.hi[l] = 0;
           }
-          if (last_window || p.n_watch) {  // rare: the call's table, the value monitor
+        }
+        __syncwarp();
+        // ---- the window's last-level row (every buffer) and the untouched buffers' held-full bits
+        uint16_t *lw = p.lastlvl + (size_t)w * p.nb;
+        unsigned lvw[kPer / 2];  // levels of c0 .. c0 + kPer - 1, two per word
+        if constexpr (kPer == 8) {
+          const uint4 v = reinterpret_cast<const uint4 *>(Q.lvl)[lane];
+          lvw[0] = v.x; lvw[1] = v.y; lvw[2] = v.z; lvw[3] = v.w;
+          if (vec && c0 < p.nb) reinterpret_cast<uint4 *>(lw + b_base)[lane] = v;
+        } else {
+          const uint2 v = reinterpret_cast<const uint2 *>(Q.lvl)[lane];
+          lvw[0] = v.x; lvw[1] = v.y;
+          if (vec && c0 < p.nb) reinterpret_cast<uint2 *>(lw + b_base)[lane] = v;
+        }
+        if (!vec) {
+#pragma unroll
+          for (int j = 0; j < kPer; ++j)
+            if (c0 + j < p.nb) lw[c0 + j] = (uint16_t)(lvw[j >> 1] >> (16 * (j & 1)));
+        }
+        const unsigned tb8 = (Q.tmask[(kPer * lane) >> 5] >> ((kPer * lane) & 31)) & ((1u << kPer) - 1u);
+        // untouched buffers held full (non-empty) by their carried level (fullm, kept current by
+        // the touched finalize); the touched ones were decided above from their window minimum
+#pragma unroll
+        for (int j = 0; j < kPer; ++j) {
+          const unsigned L = (lvw[j >> 1] >> (16 * (j & 1))) & 0xFFFFu;
+          if (!((tb8 >> j) & 1u) && c0 + j < p.nb && (nonempty_mode ? L >= 1u : L == capv[j]))
+            atomicOr(p.anyfull + (size_t)w * p.ncw + (ownv[j] >> 5), 1u << (ownv[j] & 31));
+        }
+        if (last_window || p.n_watch) {  // rare: untouched buffers' statistics
+#pragma unroll
+          for (int j = 0; j < kPer; ++j) {
+            const unsigned b = c0 + j;
+            if (b >= p.nb || ((tb8 >> j) & 1u)) continue;
             int wq = -1;
             for (unsigned k2 = 0; k2 < p.n_watch; ++k2)
               if (p.watch[k2] == b) wq = (int)k2;
-            if (last_window || wq >= 0) {
-              rtm_buffer_stat st;
-              st.integral = (int64_t)I;
-              st.last = (uint16_t)last;
-              st.max = (uint16_t)mx;
-              st.min = (uint16_t)mn;
-              st.capacity = (uint16_t)capb;
-              st.n_samples = cnt;
-              st.reserved = __ldg(p.elig + b);
-              st.mean_occ = Wlen ? __ddiv_rn((double)(long long)I, (double)((long long)capb * (long long)Wlen)) : 0.0;
-              if (wq >= 0) p.wstat[(size_t)w * RTM_WATCH_MAX + wq] = st;
-              if (last_window) {
-                p.bstat[b] = st;
-                p.carry_out[b] = (uint16_t)last;
-              }
+            if (!last_window && wq < 0) continue;
+            const unsigned L = Q.lvl[kPer * lane + j];
+            rtm_buffer_stat st;
+            st.integral = (int64_t)((unsigned long long)L * Wlen);
+            st.last = st.max = st.min = (uint16_t)L;
+            st.capacity = (uint16_t)capv[j];
+            st.n_samples = 0;
+            st.reserved = __ldg(p.elig + b);
+            st.mean_occ = Wlen ? __ddiv_rn((double)(long long)((unsigned long long)L * Wlen),
+                                           (double)((long long)capv[j] * (long long)Wlen)) : 0.0;
+            if (wq >= 0) p.wstat[(size_t)w * RTM_WATCH_MAX + wq] = st;
+            if (last_window) {
+              p.bstat[b] = st;
+              p.carry_out[b] = (uint16_t)L;
             }
           }
-          Q.lvl[l] = (unsigned short)last;
-          S.st[l] = make_uint4(0, 0, kUntouchedZ, 0);
-          S.hi[l] = 0;
         }
-      }
-      __syncwarp();
-      // ---- the window's last-level row (every buffer) and the untouched buffers' held-full bits
-      uint16_t *lw = p.lastlvl + (size_t)w * p.nb;
-      unsigned lvw[kPer / 2];  // levels of c0 .. c0 + kPer - 1, two per word
-      if constexpr (kPer == 8) {
-        const uint4 v = reinterpret_cast<const uint4 *>(Q.lvl)[lane];
-        lvw[0] = v.x; lvw[1] = v.y; lvw[2] = v.z; lvw[3] = v.w;
-        if (vec && c0 < p.nb) reinterpret_cast<uint4 *>(lw + b_base)[lane] = v;
-      } else {
-        const uint2 v = reinterpret_cast<const uint2 *>(Q.lvl)[lane];
-        lvw[0] = v.x; lvw[1] = v.y;
-        if (vec && c0 < p.nb) reinterpret_cast<uint2 *>(lw + b_base)[lane] = v;
-      }
-      if (!vec) {
+        dig = warp_sum(dig);
+        if (lane == 0) {
+          if (dig) atomicAdd(p.win + WF_DIGEST * p.W + w, dig);
+          if (nt) atomicAdd(p.win + WF_TOUCHED * p.W + w, (unsigned long long)nt);
+        }
+        __syncwarp();
+    };
+    // Software pipeline over the windows: while window w's staging entries and window w+1's
+    // segment offsets are in flight, window w-1 is finalized (a window's chain of dependent
+    // loads - tile range, segment offsets, entries - would otherwise stall the warp every window).
+    // Fast path: a window's segments for this bin span <= 32 tiles; else fold_phase1.
+    unsigned n_tlo = p.rts[1], n_thi = p.rts[2];
+    unsigned n_lo = 0, n_len = 0;
+    bool n_ok = n_thi - n_tlo <= 32u;
+    if (n_ok && n_tlo + lane < n_thi) {
+      const uint16_t *o = p.soff + (size_t)(n_tlo + lane) * (p.nbins + 1) + bin;
+      n_lo = __ldg(o);
+      n_len = (unsigned)__ldg(o + 1) - n_lo;
+    }
+    bool pend = false;
+    unsigned pw = 0;
+    unsigned long long pWlen = 0;
+    for (unsigned w = 0; w < p.W; ++w) {
+      const long long tb = p.T[w], te = p.T[w + 1];
+      const unsigned long long Wlen = (unsigned long long)(te - tb);
+      if (n_ok) {
+        const unsigned t_lo = n_tlo, seg_lo = n_lo, seg_len = n_len;
+        // flatten window w's segments (one group of <= 32 tiles)
+        unsigned pre = seg_len;
 #pragma unroll
-        for (int j = 0; j < kPer; ++j)
-          if (c0 + j < p.nb) lw[c0 + j] = (uint16_t)(lvw[j >> 1] >> (16 * (j & 1)));
-      }
-      const unsigned tb8 = (Q.tmask[(kPer * lane) >> 5] >> ((kPer * lane) & 31)) & ((1u << kPer) - 1u);
-#pragma unroll
-      for (int j = 0; j < kPer; ++j) {
-        const unsigned L = (lvw[j >> 1] >> (16 * (j & 1))) & 0xFFFFu;
-        if (!((tb8 >> j) & 1u) && c0 + j < p.nb && (nonempty_mode ? L >= 1u : L == capv[j]))
-          atomicOr(p.anyfull + (size_t)w * p.ncw + (ownv[j] >> 5), 1u << (ownv[j] & 31));
-      }
-      if (last_window || p.n_watch) {  // rare: untouched buffers' statistics
-#pragma unroll
-        for (int j = 0; j < kPer; ++j) {
-          const unsigned b = c0 + j;
-          if (b >= p.nb || ((tb8 >> j) & 1u)) continue;
-          int wq = -1;
-          for (unsigned k2 = 0; k2 < p.n_watch; ++k2)
-            if (p.watch[k2] == b) wq = (int)k2;
-          if (!last_window && wq < 0) continue;
-          const unsigned L = Q.lvl[kPer * lane + j];
-          rtm_buffer_stat st;
-          st.integral = (int64_t)((unsigned long long)L * Wlen);
-          st.last = st.max = st.min = (uint16_t)L;
-          st.capacity = (uint16_t)capv[j];
-          st.n_samples = 0;
-          st.reserved = __ldg(p.elig + b);
-          st.mean_occ = Wlen ? __ddiv_rn((double)(long long)((unsigned long long)L * Wlen),
-                                         (double)((long long)capv[j] * (long long)Wlen)) : 0.0;
-          if (wq >= 0) p.wstat[(size_t)w * RTM_WATCH_MAX + wq] = st;
-          if (last_window) {
-            p.bstat[b] = st;
-            p.carry_out[b] = (uint16_t)L;
+        for (int o = 1; o < 32; o <<= 1) {
+          const unsigned y = __shfl_up_sync(kFull, pre, o);
+          if (lane >= o) pre += y;
+        }
+        const unsigned total = __shfl_sync(kFull, pre, 31);
+        const unsigned nonempty = __ballot_sync(kFull, seg_len != 0);
+        if (seg_len) S.seg_base[__popc(nonempty & lt)] = (t_lo + lane) * (unsigned)kTileS + seg_lo - (pre - seg_len);
+        const unsigned my_end = seg_len ? pre : 0xFFFFFFFFu;
+        const unsigned le = (2u << lane) - 1u;
+        __syncwarp();
+        unsigned seg_before = 0;
+        auto fetch = [&](unsigned c) -> unsigned long long {
+          const unsigned x = my_end - c;
+          const unsigned ends = __reduce_or_sync(kFull, x < 32u ? 1u << x : 0u);
+          const unsigned sgi = seg_before + __popc(ends & le);
+          seg_before += __popc(ends);
+          const unsigned g = c + lane;
+          if (g >= total) return 0ull;
+          return __ldcg(p.stage + (S.seg_base[sgi] + g));
+        };
+        unsigned long long e0 = fetch(0), e1 = total > 32u ? fetch(32) : 0ull;  // usually one chunk
+        // next window's tile range and this lane's segment (in flight during the finalize)
+        if (w + 1 < p.W) {
+          n_tlo = n_thi;
+          n_thi = p.rts[w + 3];
+          n_ok = n_thi - n_tlo <= 32u;
+          n_lo = n_len = 0;
+          if (n_ok && n_tlo + lane < n_thi) {
+            const uint16_t *o = p.soff + (size_t)(n_tlo + lane) * (p.nbins + 1) + bin;
+            n_lo = __ldg(o);
+            n_len = (unsigned)__ldg(o + 1) - n_lo;
+          }
+        }
+        if (pend) finalize(pw, pWlen);
+        for (unsigned c = 0; c < total; c += 32) {
+          const unsigned long long en = c + 64 < total ? fetch(c + 64) : 0ull;
+          fold_chunk<NAR, BL>(S, lane, lt, c + lane < total, e0, Wlen);
+          e0 = e1;
+          e1 = en;
+        }
+        __syncwarp();
+      } else {  // many tiles in one window: the general phase 1, no overlap
+        if (pend) finalize(pw, pWlen);
+        fold_phase1<NAR, BL>(p, S, w, bin, Wlen, lane, lt);
+        __syncwarp();
+        if (w + 1 < p.W) {
+          n_tlo = p.rts[w + 2];
+          n_thi = p.rts[w + 3];
+          n_ok = n_thi - n_tlo <= 32u;
+          n_lo = n_len = 0;
+          if (n_ok && n_tlo + lane < n_thi) {
+            const uint16_t *o = p.soff + (size_t)(n_tlo + lane) * (p.nbins + 1) + bin;
+            n_lo = __ldg(o);
+            n_len = (unsigned)__ldg(o + 1) - n_lo;
           }
         }
       }
-      dig = warp_sum(dig);
-      if (lane == 0) {
-        if (dig) atomicAdd(p.win + WF_DIGEST * p.W + w, dig);
-        if (nt) atomicAdd(p.win + WF_TOUCHED * p.W + w, (unsigned long long)nt);
-      }
-      __syncwarp();
+      pend = true;
+      pw = w;
+      pWlen = Wlen;
     }
+    if (pend) finalize(pw, pWlen);
   }
 }
 
