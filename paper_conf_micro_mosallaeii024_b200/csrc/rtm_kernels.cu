@@ -1522,8 +1522,8 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
             if (c0 + j < p.nb) lw[c0 + j] = (uint16_t)(lvw[j >> 1] >> (16 * (j & 1)));
         }
         const unsigned tb8 = (Q.tmask[(kPer * lane) >> 5] >> ((kPer * lane) & 31)) & ((1u << kPer) - 1u);
-        // untouched buffers held full (non-empty) by their carried level (fullm, kept current by
-        // the touched finalize); the touched ones were decided above from their window minimum
+        // untouched buffers held full (non-empty) by their carried level; the touched ones were
+        // decided above from their window minimum
 #pragma unroll
         for (int j = 0; j < kPer; ++j) {
           const unsigned L = (lvw[j >> 1] >> (16 * (j & 1))) & 0xFFFFu;
