@@ -441,6 +441,8 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     cl.add(c->cdelta.p, (size_t)c->nc * 2 * 8);
     cl.add(c->active.p, Wn * c->ncw * 4);
     cl.add(c->anyfull.p, Wn * c->ncw * 4);
+    // long H, call shorter than H: the hang kernel stops at the first window its prefix AND empties
+    if (c->H > 64 && W < c->H) cl.add(c->hung.p, Wn * c->ncw * 4);
     cl.add(c->unit_ctr.p, 16);
     launch_clear(cl, c->st);
   }

@@ -2150,8 +2150,47 @@ __device__ __forceinline__ unsigned hang_cond(const Params &p, unsigned j, unsig
 // prefix(w).  Windows w < H-1 reach before the call: prefix(w) (= AND over 0..w) and the carried
 // run must cover the rest.
 constexpr unsigned kHangShortH = 64;
+// calls shorter than H with a long H (C5: 1000-window calls, H = 2048) take k_hang_prefix
+__host__ __device__ constexpr bool hang_prefix_path(uint32_t W, uint32_t H) { return H > kHangShortH && W < H; }
 __host__ __device__ constexpr size_t hang_flag_threads(uint32_t W, uint32_t ncw, uint32_t H) {
-  return H > kHangShortH ? (size_t)ncw : (size_t)W * ncw;
+  return hang_prefix_path(W, H) ? 0 : H > kHangShortH ? (size_t)ncw : (size_t)W * ncw;
+}
+
+// Long H and a call shorter than H: every window w of the call is flagged iff the condition held
+// in windows 0..w of the call (a prefix AND) and the carried run covers the rest (run_in >= H-1-w).
+// One warp per 32-component word, lane = window inside a group of 32: the prefix AND is a warp
+// scan, the carried-run test a per-bit threshold (first window at which the bit may be flagged).
+__global__ void __launch_bounds__(256) k_hang_prefix(Params p) {
+  const unsigned q = (unsigned)(((size_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5), lane = threadIdx.x & 31;
+  if (q >= p.ncw) return;  // warp-uniform
+  const unsigned H = p.H, W = p.W;
+  const unsigned vmask = (q == p.ncw - 1 && (p.nc & 31)) ? (1u << (p.nc & 31)) - 1u : 0xFFFFFFFFu;
+  // lane b: the first window of the call at which component q*32+b may be flagged
+  const unsigned cc = q * 32 + lane;
+  const unsigned r = cc < p.nc ? p.run[cc] : 0u;
+  const unsigned first_ok_lane = r >= H - 1 ? 0u : H - 1 - r;
+  unsigned acc = 0xFFFFFFFFu;  // AND of the condition over the windows before this group
+  for (unsigned w0 = 0; w0 < W && __any_sync(kFull, acc != 0); w0 += 32) {
+    const unsigned w = w0 + lane;
+    unsigned x = w < W ? hang_cond(p, w, q) : 0xFFFFFFFFu;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {  // inclusive prefix AND over the group's windows
+      const unsigned y = __shfl_up_sync(kFull, x, o);
+      if (lane >= (unsigned)o) x &= y;
+    }
+    x &= acc;
+    acc = __shfl_sync(kFull, x, 31);
+    // bits whose carried run already covers window w (thresholds gathered from their lanes)
+    unsigned elig = 0;
+#pragma unroll
+    for (int b = 0; b < 32; ++b) elig |= (w >= (unsigned)__shfl_sync(kFull, first_ok_lane, b) ? 1u : 0u) << b;
+    const unsigned out = x & elig & vmask;
+    if (w < W) {
+      p.hung[(size_t)w * p.ncw + q] = out;
+      if (out) atomicAdd(p.win + WF_HUNG * p.W + w, (unsigned long long)__popc(out));
+    }
+  }
+  // windows after the prefix AND emptied: nothing flagged (hung rows are cleared per call)
 }
 
 __global__ void k_hang(Params p) {
@@ -2731,6 +2770,10 @@ void launch_persist(const Params &p, cudaStream_t st) {
 
 void launch_hang(const Params &p, cudaStream_t st) {
   const unsigned threads = 256;
+  if (hang_prefix_path(p.W, p.H)) {
+    const size_t nt = (size_t)p.ncw * 32;
+    { k_hang_prefix<<<(unsigned)((nt + threads - 1) / threads), threads, 0, st>>>(p); count_launch(); }
+  }
   const size_t n = ((hang_flag_threads(p.W, p.ncw, p.H) + 31) & ~(size_t)31) + (size_t)p.ncw * 32;
   { k_hang<<<(unsigned)((n + threads - 1) / threads), threads, 0, st>>>(p); count_launch(); }
 }
