@@ -40,13 +40,13 @@ def _peaks():
 
 
 class ClockSampler:
-    """SM clocks + throttle reasons sampled DURING the timed region (NVML every 10 ms; nvidia-smi
+    """SM clocks + throttle reasons sampled DURING the timed region (NVML every 2 ms; nvidia-smi
     fallback).  Reasons follow nvidia-smi's clocks_event_reasons names."""
 
     REASONS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
                "hw_power_brake_slowdown": 0x80, "sw_power_cap": 0x4}
 
-    def __init__(self, index: int, period: float = 0.01):
+    def __init__(self, index: int, period: float = 0.002):
         self.index = index
         self.period = period
         self.rows = []  # (sm_mhz, max_mhz, reason_mask)
