@@ -878,3 +878,34 @@ def test_very_sparse_calls_sequential_fold(hang_mode):
         ser = mon.watch_series(q)
         for f in ("integral", "last", "max", "min", "capacity", "n_samples", "mean_occ"):
             assert np.array_equal(ser[f], A[-300:, b][f]), (b, f)
+
+
+def test_large_registry_bins_of_128_dense_and_sparse_calls():
+    """Registries of 131073 .. 524288 buffers use bins of 128 buffers (C5's 327680): the fallback
+    partition with 128-buffer bins and every fold path on them - a dense call (>= 2 samples per
+    buffer-window: windowed chain fold), a sparse one (look-back over 3 windows per step) and a
+    very sparse one (sequential fold) - against the oracle."""
+    wl = gen.C1.scaled("C1-bl7", n_samples=3_600_000, n_events=360_000, n_buffers=140_000, n_windows=40)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    s, e = gen.samples(wl), gen.events(wl)
+    t_end = wl.t_end()
+    calls = ([int(t_end[3])], [int(x) for x in t_end[4:8]])  # 2.6 and 0.64 samples per buffer-window
+    w0 = 0
+    for ends in calls:
+        w1 = w0 + (4 if len(ends) == 1 else len(ends))
+        sl = slice(wl.index_at("samples", wl.t_begin(w0)), wl.index_at("samples", wl.t_begin(w1)))
+        el = slice(wl.index_at("events", wl.t_begin(w0)), wl.index_at("events", wl.t_begin(w1)))
+        ref = orc.reduce(s[sl], e[el], ends)
+        mon.ingest(_dev(s[sl]), _dev(e[el]))
+        assert_same(mon.window_reduce(ends), ref, mon)
+        w0 = w1
+    t_end = t_end[:8]
+    # a very sparse call: few records over many windows
+    ends = [int(t_end[-1]) + 1000 * (i + 1) for i in range(40)]
+    few = sample_array([(int(t_end[-1]) + 37 * i, (i * 7919) % wl.n_buffers, 1, int(cap[(i * 7919) % wl.n_buffers]))
+                        for i in range(500)])
+    ref = orc.reduce(few, event_array([]), ends)
+    mon.ingest(_dev(few), None)
+    assert_same(mon.window_reduce(ends), ref, mon)
