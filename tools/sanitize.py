@@ -60,6 +60,25 @@ def main():
             lo_s, lo_e = hs, he
         mon.buffer_stats()
         mon.close()
+    # a very sparse call (sequential fold) with a long H (prefix hang kernel), 128-buffer bins
+    nb = 140_000
+    owner2 = (np.arange(nb) // 4).astype(np.uint32)
+    cap2 = np.full(nb, 8, np.uint16)
+    tot2 = np.full(2, 100, np.int64)
+    rng = np.random.default_rng(7)
+    m = 4000 if small else 20_000
+    ts = np.sort(rng.integers(0, 200_000, m))
+    sp = np.zeros(m, gen.SAMPLE_DTYPE)
+    sp["ts"], sp["buffer_id"] = ts, rng.integers(0, nb, m)
+    sp["level"], sp["capacity"] = rng.integers(0, 9, m), 8
+    ends = np.arange(1, 201, dtype=np.int64) * 1000
+    kw = dict(t0=0, hang_windows=300, k=16)
+    orc = oracle.Oracle(owner2, cap2, tot2, n_components=nb // 4, **kw)
+    mon = Monitor(owner2, cap2, tot2, n_components=nb // 4, **kw)
+    ref = orc.reduce(sp, np.zeros(0, gen.EVENT_DTYPE), ends)
+    mon.ingest(_dev(sp), None)
+    check(mon.window_reduce(ends), ref, len(ends))
+    mon.close()
     print("sanitize workload OK")
 
 
