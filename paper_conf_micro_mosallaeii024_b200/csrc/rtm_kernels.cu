@@ -423,7 +423,6 @@ constexpr int kPerLane = kSub / 32;               // 16
 constexpr int kK1Warps = kK1Threads / 32;         // 8
 constexpr unsigned kNoKey = 0xFFFFu;
 constexpr uint32_t kLmMaxBins = 170;              // count rows (nbins x 48 B) fit the 8 KB raw slot
-constexpr uint32_t kLmMaxBinsX = 340;             // rows in their own region (one CTA per SM)
 static_assert(kPerLane == 16, "lane-major swizzle assumes 16 records per lane");
 static_assert((size_t)kLmMaxBins * 48 <= (size_t)kSub * 16, "count rows must fit the raw slot");
 
@@ -437,10 +436,9 @@ __host__ __device__ constexpr size_t k1_vec_bytes(uint32_t nbins) { return k1_al
 // dynamic shared memory.  lm: raw 16 B x 4096 | wt x 2 (tile parity) | wb | tile descriptors
 // (8 warps x 2) | cap[nb];  mx: sbuf 8 B x 4096 | wt | wb
 // (wt: 8 x nbins u16 bin totals / live counters, wb: 8 x nbins u16 bin bases)
-__host__ __device__ constexpr size_t k1_rows_stride(uint32_t nbins) { return k1_align16((size_t)nbins * 48); }
-__host__ __device__ constexpr size_t k1_smem_lm(uint32_t nbins, uint32_t nb, bool caps = true, bool xr = false) {
+__host__ __device__ constexpr size_t k1_smem_lm(uint32_t nbins, uint32_t nb, bool caps = true) {
   return (size_t)kTileS * 16 + 3 * k1_vec_bytes(nbins) + (size_t)kK1Warps * 2 * sizeof(TileDesc) +
-         (caps ? k1_align16((size_t)nb * 2) : 0) + (xr ? (size_t)kK1Warps * k1_rows_stride(nbins) : 0);
+         (caps ? k1_align16((size_t)nb * 2) : 0);
 }
 __host__ __device__ constexpr size_t k1_smem_mx(uint32_t nbins) { return (size_t)kTileS * 8 + 2 * k1_vec_bytes(nbins); }
 
@@ -630,7 +628,7 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
 // and only then prefetch their next raw records (named barrier among themselves); warps 4-7
 // prefetch before the first barrier (measured 813 -> 692 us on C2 against direct 8-byte scatter
 // stores from every lane, which touched 32 sectors per store instruction).
-template <int BL, bool CAPS, bool XR>
+template <int BL, bool CAPS>
 __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   static_assert(BL == 8, "lane-major entries pack the buffer id in one byte");
   extern __shared__ __align__(16) unsigned char smem[];
@@ -646,10 +644,8 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   unsigned short *capS = reinterpret_cast<unsigned short *>(tail + 3 * vb + (size_t)kK1Warps * 2 * sizeof(TileDesc));
   int4 *raw = reinterpret_cast<int4 *>(smem) + warp * kSub;  // this warp's slot
   // after the scan the slot holds the count rows: 48 B per bin = 32 u8 lane counters (later the
-  // exclusive in-word prefixes) + 8 u16 word bases; XR (171..340 bins): rows in their own region
-  unsigned char *rows = XR ? tail + 3 * vb + (size_t)kK1Warps * 2 * sizeof(TileDesc) +
-                                 (CAPS ? k1_align16((size_t)p.nb * 2) : 0) + (size_t)warp * k1_rows_stride(nbins)
-                           : reinterpret_cast<unsigned char *>(raw);
+  // exclusive in-word prefixes) + 8 u16 word bases
+  unsigned char *rows = reinterpret_cast<unsigned char *>(raw);
   if (CAPS)  // the capacity table in shared memory (the field check gathers it per sample)
     for (unsigned i = threadIdx.x; i < p.nb; i += kK1Threads) capS[i] = __ldg(p.cap + i);
   // Tiles are claimed dynamically (p.unit_ctr[1]) so a CTA that starts late - the side-stream
@@ -2625,13 +2621,10 @@ size_t fold_smem_bytes(int bin_log) {
 // lane-major partition: the capacity table in shared memory when two CTAs still fit per SM
 bool partition_caps_smem(uint32_t nbins, uint32_t nb) { return k1_smem_lm(nbins, nb, true) + 1024 <= 113 * 1024; }
 size_t partition_smem_bytes(uint32_t nbins, uint32_t nb) {
-  return nbins <= kLmMaxBins    ? k1_smem_lm(nbins, nb, partition_caps_smem(nbins, nb))
-         : nbins <= kLmMaxBinsX ? k1_smem_lm(nbins, nb, false, true)
-                                : k1_smem_mx(nbins);
+  return nbins <= kLmMaxBins ? k1_smem_lm(nbins, nb, partition_caps_smem(nbins, nb)) : k1_smem_mx(nbins);
 }
 static_assert(2 * (k1_smem_lm(80, 20480) + 1024 + 512) <= 228 * 1024, "C2-sized partition CTAs must fit 2 per SM");
-static_assert(k1_smem_lm(kLmMaxBins, 0, false) <= 113 * 1024 && k1_smem_mx(kMaxBins) <= 227 * 1024 &&
-                  k1_smem_lm(kLmMaxBinsX, 0, false, true) <= 227 * 1024,
+static_assert(k1_smem_lm(kLmMaxBins, 0, false) <= 113 * 1024 && k1_smem_mx(kMaxBins) <= 227 * 1024,
               "partition shared memory exceeds the opt-in limit");
 size_t topk_smem_bytes(uint32_t nb) {
   return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8 + kTopkCand * 4;
@@ -2653,17 +2646,17 @@ void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
   { k_fill_tiles<<<2 * blocks, 64, 0, st>>>(p); count_launch(); }
 }
 
-bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s) { return n_tiles_s && nbins <= kLmMaxBinsX; }
+bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s) { return n_tiles_s && nbins <= kLmMaxBins; }
 
-template <int BL, bool CAPS, bool XR>
+template <int BL, bool CAPS>
 void launch_partition_lm(const Params &p, int n_sms, size_t sm, cudaStream_t st) {
   int per_sm = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm<BL, CAPS, XR>, kK1Threads, sm);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm<BL, CAPS>, kK1Threads, sm);
   if (per_sm < 1) per_sm = 1;
   unsigned grid = (unsigned)(n_sms * per_sm);
   const unsigned work = p.n_tiles_s + (p.fuse_events ? p.n_tiles_e : 0u);
   if (grid > work) grid = work;
-  { k_partition_lm<BL, CAPS, XR><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
+  { k_partition_lm<BL, CAPS><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
 }
 
 void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
@@ -2671,10 +2664,8 @@ void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   const size_t sm = partition_smem_bytes(p.nbins, p.nb);
   if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM
     // bin_log 8 here: bin_log 7 is only chosen for > 131072 buffers (> 170 bins)
-    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, false>(p, n_sms, sm, st);
-    else launch_partition_lm<8, false, false>(p, n_sms, sm, st);
-  } else if (p.nbins <= kLmMaxBinsX && p.bin_log == 8) {  // rows in their own region: one CTA / SM
-    launch_partition_lm<8, false, true>(p, n_sms, sm, st);
+    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true>(p, n_sms, sm, st);
+    else launch_partition_lm<8, false>(p, n_sms, sm, st);
   } else {
     if (p.bin_log == 7) { k_partition_mx<7><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
     else { k_partition_mx<8><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
@@ -2806,10 +2797,8 @@ void configure_kernels_once() {
   done[dev] = true;
   const int lm_caps = (int)k1_smem_lm(kLmMaxBins, 113 * 512, true);  // <= 113 KB by partition_caps_smem
   const int lm_glob = (int)k1_smem_lm(kLmMaxBins, 0, false);
-  cudaFuncSetAttribute(k_partition_lm<8, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
-  cudaFuncSetAttribute(k_partition_lm<8, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
-  cudaFuncSetAttribute(k_partition_lm<8, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                       (int)k1_smem_lm(kLmMaxBinsX, 0, false, true));
+  cudaFuncSetAttribute(k_partition_lm<8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
   cudaFuncSetAttribute(k_partition_mx<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
   cudaFuncSetAttribute(k_partition_mx<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
   cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
