@@ -200,28 +200,38 @@ def cpu_sharded_step(wl, n_win, P):
 
 
 def run_reference(args):
-    """--impl reference: the CPU oracle timed on the host cores, same metric/config (rank 0 only)."""
+    """--impl reference: the CPU oracle as it stands, timed on the box's host cores (rank 0 only):
+    `nproc` processes, one owner-component shard each, + the merge of their results (the
+    single-core run when the host has one core or RTM_REF_CORES=1); same metric and config."""
     import gen
 
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
     wl = gen.C2
-    n_win = int(os.environ.get("RTM_REF_WINDOWS", "25"))
+    info = host_info()
+    P = int(os.environ.get("RTM_REF_CORES", str(info["nproc"] or 1)))
+    n_win = int(os.environ.get("RTM_REF_WINDOWS", str(25 if P <= 1 else max(25, min(wl.n_windows, 2500 // P)))))
+
+    def one():
+        return cpu_reference_step(wl, n_win) if P <= 1 else cpu_sharded_step(wl, n_win, P)
+
     for _ in range(args.warmup):
-        cpu_reference_step(wl, n_win)
+        one()
     tot_recs, tot_t = 0, 0.0
     for _ in range(args.steps):
-        r, dt = cpu_reference_step(wl, n_win)
+        r, dt = one()
         tot_recs += r
         tot_t += dt
     v = tot_recs / tot_t
+    how = ("single-threaded C oracle" if P <= 1 else
+           f"{P} processes, one owner-component shard each, + the merge (slowest shard's reduce + merge time)")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_t / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
             "config": {"workload": wl.description, "sample": f"first {n_win} of {wl.n_windows} windows"},
-            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"first {n_win} windows of C2 ({tot_recs // args.steps} records/step)"},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": P, "kind": "oracle", "host": info,
+                             "sample": f"first {n_win} windows of C2 ({tot_recs // args.steps} records/step), {how}"},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 

@@ -909,3 +909,87 @@ def test_large_registry_bins_of_128_dense_and_sparse_calls():
     ref = orc.reduce(few, event_array([]), ends)
     mon.ingest(_dev(few), None)
     assert_same(mon.window_reduce(ends), ref, mon)
+
+
+@pytest.mark.parametrize("on_stream", [0, 1])
+def test_c_abi_allgather_callback_two_ranks(on_stream):
+    """The C-level multi-rank path: two contexts (world 2, owner sharding) on cuda:0, each driven
+    by its own thread through rtm_window_reduce with an `allgather` callback (host-synchronised, or
+    stream-ordered with allgather_on_stream), then rtm_sync_tables through the same callback; both
+    ranks' merged results and tables equal the whole-trace oracle."""
+    import ctypes
+    import threading
+
+    wl = gen.C1.scaled("C1-cb", n_samples=150_000, n_events=15_000, n_windows=5)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    orc = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw)
+    ref = orc.reduce(gen.samples(wl), gen.events(wl), wl.t_end())
+    G = 2
+    cudart = ctypes.CDLL("libcudart.so.12")
+    cudart.cudaMemcpy.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int]
+    cudart.cudaStreamSynchronize.argtypes = [ctypes.c_void_p]
+    barrier = threading.Barrier(G)
+    sends = [None] * G
+    streams = [torch.cuda.Stream() for _ in range(G)]
+
+    def make_cb(r):
+        def cb(user, send, recv, nbytes):
+            if on_stream:  # the callback must order itself: finish this rank's pack first
+                cudart.cudaStreamSynchronize(ctypes.c_void_p(streams[r].cuda_stream))
+            sends[r] = send
+            barrier.wait()
+            for q in range(G):
+                if cudart.cudaMemcpy(ctypes.c_void_p(recv + q * nbytes), ctypes.c_void_p(sends[q]), nbytes, 3):
+                    return 1
+            barrier.wait()
+            return 0
+        return N.ALLGATHER_FN(cb)
+
+    cbs = [make_cb(r) for r in range(G)]
+    mons, keep = [], []
+    for r in range(G):
+        owned = (np.arange(wl.n_components) % G == r).astype(np.uint8)
+        m = Monitor(owner, cap, tot, n_components=wl.n_components, rank=r, world=G, owned_components=owned,
+                    stream=streams[r], **kw)
+        # swap in a context whose config carries the callback (the binding's own uses the two-phase API)
+        cfg = N.Config()
+        cfg.n_buffers, cfg.n_components, cfg.n_kernels = len(owner), wl.n_components, len(tot)
+        cfg.buffer_owner, cfg.buffer_capacity, cfg.kernel_total = m._owner.ctypes.data, m._cap.ctypes.data, m._tot.ctypes.data
+        cfg.t0, cfg.hang_windows, cfg.k, cfg.rank_mode = wl.t0, 2, wl.k, 0
+        cfg.device, cfg.rank, cfg.world = 0, r, G
+        cfg.owned_components = owned.ctypes.data
+        cfg.allgather = cbs[r]
+        cfg.stream = streams[r].cuda_stream
+        cfg.allgather_on_stream = on_stream
+        h = ctypes.c_void_p()
+        N.check(N.lib().rtm_create(ctypes.byref(cfg), ctypes.byref(h)), "rtm_create")
+        N.lib().rtm_destroy(m._h)
+        m._h = h
+        keep.append(owned)
+        s, e = gen.samples(wl, shard=(G, r)), gen.events(wl, shard=(G, r))
+        keep += [s, e]
+        N.check(N.lib().rtm_ingest(m._h, s.ctypes.data, len(s), e.ctypes.data, len(e), N.RTM_MEM_HOST), "ingest")
+        mons.append(m)
+    ends = np.ascontiguousarray(wl.t_end())
+    rcs = [None] * G
+    summs = [np.zeros(wl.n_windows, N.SUMMARY_DTYPE) for _ in range(G)]
+
+    def run(r):
+        rcs[r] = N.lib().rtm_window_reduce(mons[r]._h, ends.ctypes.data, len(ends), summs[r].ctypes.data)
+        if rcs[r] == 0:
+            rcs[r] = N.lib().rtm_sync_tables(mons[r]._h)
+
+    th = [threading.Thread(target=run, args=(r,)) for r in range(G)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=120)
+    assert rcs == [0, 0], rcs
+    for r, m in enumerate(mons):
+        m.W = wl.n_windows
+        m._synced = True
+        got = m.results()
+        assert np.array_equal(got["summary"], summs[r])
+        assert_same(got, ref, m)
+        assert np.array_equal(m.topk_persistence(), orc.persistence())
