@@ -344,6 +344,9 @@ def run_native(args):
     e2e_value, e2e_steps = None, 0
     if 16 * n_rec <= (8 << 30) and not args.no_e2e:
         e2e_value, e2e_steps = run_e2e(args, mon, ds, de, wl, t_end, n_rec, world, dist, dev)
+    streaming = None
+    if world == 1 and not args.no_streaming:
+        streaming = run_streaming(mon, ds, de, wl, t_end)
     W = wl.n_windows
     d2h = W * (8 * 6 + wl.k * 8 + 4 + wl.n_kernels * 40 + 4)
     rank_done = rank != 0
@@ -352,7 +355,30 @@ def run_native(args):
             dist.destroy_process_group()
         return
     return finish(args, wl, world, ms, prof, prof_ms, n_rec, value, e2e_value, e2e_steps, d2h, n_launches, clk,
-                  t_wall, dist)
+                  t_wall, dist, streaming)
+
+
+def run_streaming(mon, ds, de, wl, t_end, n_windows: int = 300, warmup: int = 20):
+    """Per-window snapshot latency in streaming mode: one window per
+    rtm_window_reduce call, the window's records already in HBM (slices of the resident trace),
+    host wall clock from the ingest to the results on the host (the call blocks on its D2H)."""
+    mon.reset()
+    lat, recs = [], 0
+    for w in range(warmup + n_windows):
+        s0, s1 = wl.index_at("samples", wl.t_begin(w)), wl.index_at("samples", wl.t_begin(w + 1))
+        e0, e1 = wl.index_at("events", wl.t_begin(w)), wl.index_at("events", wl.t_begin(w + 1))
+        t = time.perf_counter()
+        mon.ingest(ds[s0 * 16:s1 * 16], de[e0 * 16:e1 * 16])
+        mon.window_reduce(t_end[w:w + 1])
+        dt = time.perf_counter() - t
+        if w >= warmup:
+            lat.append(dt * 1e6)
+            recs += (s1 - s0) + (e1 - e0)
+    lat = np.array(lat)
+    return {"what": "one window per rtm_window_reduce call, records resident in HBM, host wall clock per call",
+            "windows": n_windows, "records_per_window": recs / n_windows,
+            "p50_us": float(np.percentile(lat, 50)), "p99_us": float(np.percentile(lat, 99)),
+            "tool": "tools/latency.py (per-kernel breakdown, C5)"}
 
 
 def run_e2e(args, mon, ds, de, wl, t_end, n_rec, world, dist, dev):
@@ -390,7 +416,7 @@ NOMINAL_HBM_GBS = 8000.0  # B200 HBM3e nominal (SURVEY.md §8(d) reports both de
 
 
 def finish(args, wl, world, ms, prof, prof_ms, n_rec, value, e2e_value, e2e_steps, d2h, n_launches, clk, t_wall,
-           dist):
+           dist, streaming=None):
     W = wl.n_windows
     # ---- roofline: algorithmic bytes = 16 B per record, read once.  They are
     # charged to the kernel that reads the records (k_partition; it also runs the task-event tiles
@@ -470,6 +496,7 @@ def finish(args, wl, world, ms, prof, prof_ms, n_rec, value, e2e_value, e2e_step
                  "note": "pinned host trace -> device inside every step: bound by the host link "
                          "(16 B/record over PCIe/C2C), not by the kernels"}
                 if e2e_value is not None else None),
+        "streaming": streaming,
         "gpu_launches": n_launches,
         "clocks": clk.summary(),
         "wall_s_timed": t_wall,
@@ -488,6 +515,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-sharded", action="store_true", help="skip the nproc-process oracle baseline")
+    ap.add_argument("--no-streaming", action="store_true", help="skip the one-window-per-call latency")
     ap.add_argument("--rank-mode", type=int, default=0, help="0 percent (bench line), 1 size, 2 mean occupancy")
     ap.add_argument("--config", default="C2-1gpu",
                     help="workload (gen.CONFIGS); the bench line is C2-1gpu, the others are parity configs "
