@@ -32,7 +32,7 @@ struct Chunk {
 };
 
 enum KernelId { KT_SPLIT, KT_PARTITION, KT_EVENTS, KT_FOLD, KT_ORDER, KT_TOPK, KT_HANG, KT_PROGRESS, KT_MERGE, KT_N };
-const char *kKernelNames[KT_N] = {"k_split", "k_partition", "k_events", "k_fold", "k_order_check",
+const char *kKernelNames[KT_N] = {"k_prep", "k_partition", "k_events", "k_fold", "k_order_check",
                                   "k_topk", "k_hang", "k_progress", "k_merge"};
 
 }  // namespace
@@ -384,11 +384,8 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.s = (const rtm_level_sample *)sp; p.ns = ns;
   p.e = (const rtm_task_event *)ep; p.ne = ne;
 
-  LAUNCH(KT_SPLIT, 0, launch_split(p, (long long *)c->Bs.p + 1, (long long *)c->Be.p + 1, c->st));
   p.Bs = (const long long *)c->Bs.p; p.Be = (const long long *)c->Be.p;
   p.rts = (const uint32_t *)c->rts.p; p.rte = (const uint32_t *)c->rte.p;
-  launch_regions(p, c->st);  // region tile tables on the device: no host round trip
-  CK(cudaGetLastError());
   // tile-count upper bounds: every region adds at most one partial tile
   const uint32_t nts = (uint32_t)((ns + kTileS - 1) / kTileS) + W + 2;
   const uint32_t nte = (uint32_t)((ne + kTileE - 1) / kTileE) + W + 2;
@@ -432,6 +429,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   }
   if ((s = ensure(c, c->comps, (size_t)c->nc * sizeof(rtm_component_tasks)))) return s;
 
+  ClearList prep_cl;
   {
     const ResLayout L = res_layout(c, W);
     ClearList cl;
@@ -444,7 +442,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     // long H, call shorter than H: the hang kernel stops at the first window its prefix AND empties
     if (c->H > 64 && W < c->H) cl.add(c->hung.p, Wn * c->ncw * 4);
     cl.add(c->unit_ctr.p, 16);
-    launch_clear(cl, c->st);
+    prep_cl = cl;
   }
 
   p.tdesc = (TileDesc *)c->tdesc.p; p.tile_reg_s = (const uint32_t *)c->treg_s.p; p.tile_reg_e = (const uint32_t *)c->treg_e.p;
@@ -473,7 +471,10 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   cudaMemsetAsync(dbg, 0, 64, c->st);
   p.dbg = dbg;
 #endif
-  launch_fill_tile_regions(p, c->st);
+  // clear the call's accumulators, region boundaries, tile tables: one cooperative launch
+  LAUNCH(KT_SPLIT, 0,
+         launch_prep(p, prep_cl, (long long *)c->Bs.p, (long long *)c->Be.p, c->n_sms, c->st));
+  CK(cudaGetLastError());
   // Task events are independent of the sample path.  Lane-major partition path: the persistent
   // partition kernel runs the event tiles after its sample tiles (claimed dynamically), so no
   // concurrent kernel competes with the issue-bound fold.  Otherwise: a side stream, overlapped

@@ -1,8 +1,10 @@
 // rtm_internal.h — device data layout and kernel launchers of librtm (sm_100a).
 //
 // Data path of one rtm_window_reduce call (DESIGN.md §4 has the rationale and rooflines):
-//   K0 split      : per window boundary, warp 33-ary search for the first record position whose
-//                   field-valid successors all have ts >= boundary  -> region [B_r, B_r+1) per window
+//   K0 prep       : one cooperative launch: zero the call's accumulators; per window boundary,
+//                   warp 33-ary search for the first record position whose field-valid successors
+//                   all have ts >= boundary -> region [B_r, B_r+1) per window; grid sync; region ->
+//                   tile tables; grid sync; per-tile descriptors
 //   K1 partition  : one CTA per 4096-sample tile of one region; validate, order-check, stable
 //                   multisplit of kept samples by 256-buffer bin into 8-byte staging entries
 //   K3 events     : one CTA per 4096-event tile; progress deltas, component activity bitmaps
@@ -146,9 +148,9 @@ struct Params {
 };
 
 // launchers (rtm_kernels.cu); all asynchronous on `st`
-void launch_split(const Params &p, long long *outBs, long long *outBe, cudaStream_t st);
-void launch_regions(const Params &p, cudaStream_t st);
-void launch_fill_tile_regions(const Params &p, cudaStream_t st);
+struct ClearList;
+// clear + region boundaries + tile tables, one cooperative launch (p.Bs/Be/rts/rte/tdesc/tile_reg set)
+void launch_prep(const Params &p, const ClearList &cl, long long *Bs, long long *Be, int n_sms, cudaStream_t st);
 void launch_partition(const Params &p, int n_sms, cudaStream_t st);
 void launch_events(const Params &p, cudaStream_t st);
 bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s);  // lane-major partition path

@@ -1,6 +1,7 @@
 // rtm_kernels.cu — sm_100a kernels of the window-snapshot reduction (see rtm_internal.h and
 // DESIGN.md §4).  No tensor cores: nothing here is a dense contraction; the path is bound by
 // the one compulsory HBM read of 16 B per trace record.
+#include <cooperative_groups.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdlib.h>
@@ -183,12 +184,6 @@ __device__ __forceinline__ void split_one(const Params &p, unsigned q, long long
   if (lane == 0) outB[q] = (long long)ans;
 }
 
-// Both streams in one launch: warps 0..W split the samples, warps W+1..2W+1 the events.
-__global__ void k_split(Params p, long long *outBs, long long *outBe) {
-  const unsigned q = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;  // warp-uniform
-  if (q <= p.W) split_one<true>(p, q, outBs);
-  else if (q <= 2 * p.W + 1) split_one<false>(p, q - (p.W + 1), outBe);
-}
 
 // Region boundaries -> tile table on the device (no host round trip): B[0] = 0, B[W+2] = N, the
 // split positions made monotone (only an unsorted stream can break that; it is reported by the
@@ -241,44 +236,69 @@ __device__ __forceinline__ void regions_one(long long *B, unsigned long long N, 
   }
 }
 
-// CTA 0: sample regions, CTA 1: event regions.
-__global__ void __launch_bounds__(1024) k_regions(Params p, long long *Bs, long long *Be, uint32_t *rts, uint32_t *rte) {
-  if (blockIdx.x == 0) regions_one(Bs, p.ns, p.W, rts, kTileS);
-  else regions_one(Be, p.ne, p.W, rte, kTileE);
-}
-
-// first half of the grid: sample tiles (region id + descriptor: start, bounds, size, window);
-// second half: event tiles (region id)
-__global__ void k_fill_tiles(Params p) {
-  const uint32_t nr = p.W + 2, half = gridDim.x / 2;
-  if (blockIdx.x >= half) {
-    for (uint32_t r = blockIdx.x - half; r < nr; r += half)
-      for (uint32_t t = p.rte[r] + threadIdx.x; t < p.rte[r + 1]; t += blockDim.x)
-        const_cast<uint32_t *>(p.tile_reg_e)[t] = r;
-    return;
-  }
-  for (uint32_t r = blockIdx.x; r < nr; r += half) {
-    const Region g = region_of(p, r);
-    const long long lo = g.lo_ts;
-    const unsigned long long wlen =
-        g.hi_ts == kTsMax ? (unsigned long long)(kTsMax - lo) + 1ull : (unsigned long long)(g.hi_ts - lo);
-    for (uint32_t t = p.rts[r] + threadIdx.x; t < p.rts[r + 1]; t += blockDim.x) {
-      const_cast<uint32_t *>(p.tile_reg_s)[t] = r;
-      TileDesc d;
-      d.start = p.Bs[r] + (long long)(t - p.rts[r]) * kTileS;
-      long long endp = p.Bs[r + 1];
-      if (endp > d.start + kTileS) endp = d.start + kTileS;
-      d.n = (int)(endp - d.start);
-      d.lo = lo;
-      d.wlen = wlen;
-      d.window = g.window;
-      d.charge = g.charge;
-      d.pad[0] = d.pad[1] = d.pad[2] = 0;
-      p.tdesc[t] = d;
-    }
+// tile tables of region r: the sample tiles' region id + descriptor (start, bounds, size, window)
+// and the event tiles' region id
+__device__ __forceinline__ void fill_region(const Params &p, uint32_t r, bool samples, bool events) {
+  if (events)
+    for (uint32_t t = p.rte[r] + threadIdx.x; t < p.rte[r + 1]; t += blockDim.x)
+      const_cast<uint32_t *>(p.tile_reg_e)[t] = r;
+  if (!samples) return;
+  const Region g = region_of(p, r);
+  const long long lo = g.lo_ts;
+  const unsigned long long wlen =
+      g.hi_ts == kTsMax ? (unsigned long long)(kTsMax - lo) + 1ull : (unsigned long long)(g.hi_ts - lo);
+  for (uint32_t t = p.rts[r] + threadIdx.x; t < p.rts[r + 1]; t += blockDim.x) {
+    const_cast<uint32_t *>(p.tile_reg_s)[t] = r;
+    TileDesc d;
+    d.start = p.Bs[r] + (long long)(t - p.rts[r]) * kTileS;
+    long long endp = p.Bs[r + 1];
+    if (endp > d.start + kTileS) endp = d.start + kTileS;
+    d.n = (int)(endp - d.start);
+    d.lo = lo;
+    d.wlen = wlen;
+    d.window = g.window;
+    d.charge = g.charge;
+    d.pad[0] = d.pad[1] = d.pad[2] = 0;
+    p.tdesc[t] = d;
   }
 }
 
+// zero every range of the list: 16-byte stores over each range's 16-byte-aligned body, bytes
+// for the ends (ranges come from cudaMalloc'd buffers and may have any length)
+__device__ __forceinline__ void clear_ranges(const ClearList &cl) {
+  const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (size_t)gridDim.x * blockDim.x;
+  for (int r = 0; r < cl.n; ++r) {
+    unsigned char *b = static_cast<unsigned char *>(cl.ptr[r]);
+    const size_t n = cl.bytes[r];
+    const size_t head = (16 - ((uintptr_t)b & 15)) & 15;
+    const size_t h = head < n ? head : n;
+    const size_t body = (n - h) / 16;
+    if (tid < h) b[tid] = 0;
+    uint4 *b4 = reinterpret_cast<uint4 *>(b + h);
+    for (size_t i = tid; i < body; i += nth) b4[i] = make_uint4(0, 0, 0, 0);
+    for (size_t i = h + body * 16 + tid; i < n; i += nth) b[i] = 0;
+  }
+}
+
+// The prologue of a reduce call in ONE cooperative launch (it was four: clear, split, regions,
+// tile tables): (A) zero the call's accumulators and find the region boundaries (one warp per
+// window boundary and stream), grid barrier, (B) boundaries -> per-region tile counts (blocks 0 and
+// 1), grid barrier, (C) the tile tables.  Every phase is grid-strided, so any co-resident grid works.
+__global__ void __launch_bounds__(256, 4) k_prep(Params p, ClearList cl, long long *Bs, long long *Be) {
+  namespace cg = cooperative_groups;
+  cg::grid_group grid = cg::this_grid();
+  clear_ranges(cl);
+  const unsigned nwarps = gridDim.x * (blockDim.x >> 5);
+  for (unsigned q = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; q <= 2 * p.W + 1; q += nwarps) {
+    if (q <= p.W) split_one<true>(p, q, Bs + 1);
+    else split_one<false>(p, q - (p.W + 1), Be + 1);
+  }
+  grid.sync();
+  if (blockIdx.x == 0) regions_one(Bs, p.ns, p.W, const_cast<uint32_t *>(p.rts), kTileS);
+  if (blockIdx.x == (gridDim.x > 1 ? 1u : 0u)) regions_one(Be, p.ne, p.W, const_cast<uint32_t *>(p.rte), kTileE);
+  grid.sync();
+  for (uint32_t r = blockIdx.x; r < p.W + 2; r += gridDim.x) fill_region(p, r, true, true);
+}
 
 // ============================================================================================
 // K3: task events.  One CTA per tile of <= 4096 events of one region: validate, order-check,
@@ -2586,22 +2606,7 @@ __global__ void k_scatter_bstat(Params p) {
 // ============================================================================================
 // launchers
 // ============================================================================================
-// zero every range of the list: 16-byte stores over each range's 16-byte-aligned body, bytes
-// for the ends (ranges come from cudaMalloc'd buffers and may have any length)
-__global__ void k_clear(ClearList cl) {
-  const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (size_t)gridDim.x * blockDim.x;
-  for (int r = 0; r < cl.n; ++r) {
-    unsigned char *b = static_cast<unsigned char *>(cl.ptr[r]);
-    const size_t n = cl.bytes[r];
-    const size_t head = (16 - ((uintptr_t)b & 15)) & 15;
-    const size_t h = head < n ? head : n;
-    const size_t body = (n - h) / 16;
-    if (tid < h) b[tid] = 0;
-    uint4 *b4 = reinterpret_cast<uint4 *>(b + h);
-    for (size_t i = tid; i < body; i += nth) b4[i] = make_uint4(0, 0, 0, 0);
-    for (size_t i = h + body * 16 + tid; i < n; i += nth) b[i] = 0;
-  }
-}
+__global__ void k_clear(ClearList cl) { clear_ranges(cl); }
 
 std::atomic<unsigned long long> g_kernel_launches{0};
 inline void count_launch() { g_kernel_launches.fetch_add(1, std::memory_order_relaxed); }
@@ -2630,20 +2635,25 @@ size_t topk_smem_bytes(uint32_t nb) {
   return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8 + kTopkCand * 4;
 }
 
-void launch_split(const Params &p, long long *outBs, long long *outBe, cudaStream_t st) {
-  const unsigned warps = 2 * (p.W + 1);
-  const unsigned threads = 128;
-  const unsigned blocks = (warps * 32 + threads - 1) / threads;
-  { k_split<<<blocks, threads, 0, st>>>(p, outBs, outBe); count_launch(); }
-}
-void launch_regions(const Params &p, cudaStream_t st) {
-  { k_regions<<<2, 1024, 0, st>>>(p, const_cast<long long *>(p.Bs), const_cast<long long *>(p.Be),
-                                   const_cast<uint32_t *>(p.rts), const_cast<uint32_t *>(p.rte)); count_launch(); }
-}
-void launch_fill_tile_regions(const Params &p, cudaStream_t st) {
-  const unsigned nr = p.W + 2;
-  const unsigned blocks = nr < 2048 ? nr : 2048;
-  { k_fill_tiles<<<2 * blocks, 64, 0, st>>>(p); count_launch(); }
+void launch_prep(const Params &p, const ClearList &cl, long long *Bs, long long *Be, int n_sms, cudaStream_t st) {
+  static int per_sm[128] = {0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 0 && dev < 128 && !per_sm[dev]) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[dev], k_prep, 256, 0);
+    if (per_sm[dev] < 1) per_sm[dev] = 1;
+  }
+  const unsigned cap = (unsigned)(n_sms * per_sm[dev >= 0 && dev < 128 ? dev : 0]);
+  unsigned long long mx = 0;
+  for (int r = 0; r < cl.n; ++r) mx = cl.bytes[r] > mx ? cl.bytes[r] : mx;
+  unsigned grid = (unsigned)std::max<unsigned long long>({(2ull * (p.W + 1) + 7) / 8, (mx / 16 + 255) / 256 + 1,
+                                                          (unsigned long long)(p.W + 2), 2ull});
+  if (grid > cap) grid = cap;
+  Params pp = p;
+  ClearList cc = cl;
+  void *args[] = {&pp, &cc, &Bs, &Be};
+  cudaLaunchCooperativeKernel((const void *)k_prep, dim3(grid), dim3(256), args, 0, st);
+  count_launch();
 }
 
 bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s) { return n_tiles_s && nbins <= kLmMaxBins; }

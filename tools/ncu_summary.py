@@ -13,7 +13,7 @@ ki, vi = h.index("Kernel Name"), h.index("Metric Value")
 lst = [(r[ki], float(r[vi])) for r in rows[hdr + 1:] if len(r) > vi]
 # second reduce step only (the first launches are the generator + warm-up step)
 names = [n for n, _ in lst]
-start = max(i for i, n in enumerate(names) if "k_split" in n and i > 0 and "k_split" not in names[i - 1]) if names else 0
+start = max(i for i, n in enumerate(names) if "k_prep" in n and i > 0 and "k_prep" not in names[i - 1]) if names else 0
 step = lst[start:]
 tot = sum(v for _, v in step)
 lines = [f"# {tag}: ncu summaries (C2, 1 x B200)", "",

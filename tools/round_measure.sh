@@ -4,7 +4,7 @@ NCU=/usr/local/cuda/bin/ncu
 mkdir -p gpurun_out
 timeout 600 $NCU --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/r02_launches.csv \
   python tools/prof_step.py --warmup 1 --steps 1 > /dev/null 2>&1; echo "launches rc=$?"
-timeout 1200 $NCU --set full --clock-control none --import-source on -k regex:"k_partition|k_fold|k_topk|k_split|k_hang|k_progress|k_order" \
+timeout 1200 $NCU --set full --clock-control none --import-source on -k regex:"k_partition|k_fold|k_topk|k_prep|k_hang|k_progress|k_order" \
   -s 9 -c 7 -f -o gpurun_out/r02_full python tools/prof_step.py --warmup 1 --steps 1 > gpurun_out/r02_full.log 2>&1; echo "full rc=$?"
 timeout 900 python bench.py --steps 50 --warmup 5 > gpurun_out/r02_bench_final.log 2>&1; echo "bench rc=$?"; tail -1 gpurun_out/r02_bench_final.log
 for c in C3-4gpu C4-skewed; do timeout 600 python bench.py --config $c --steps 5 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/r02_bench_$c.log 2>&1; echo "$c rc=$?"; done
