@@ -31,9 +31,10 @@ struct Chunk {
   uint64_t n;
 };
 
-enum KernelId { KT_SPLIT, KT_PARTITION, KT_EVENTS, KT_FOLD, KT_ORDER, KT_TOPK, KT_HANG, KT_PROGRESS, KT_MERGE, KT_N };
+enum KernelId { KT_SPLIT, KT_PARTITION, KT_EVENTS, KT_FOLD, KT_ORDER, KT_TOPK, KT_HANG, KT_PROGRESS, KT_MERGE,
+                KT_SUBPART, KT_N };
 const char *kKernelNames[KT_N] = {"k_prep", "k_partition", "k_events", "k_fold", "k_order_check",
-                                  "k_topk", "k_hang", "k_progress", "k_merge"};
+                                  "k_topk", "k_hang", "k_progress", "k_merge", "k_subpart"};
 
 }  // namespace
 
@@ -86,7 +87,7 @@ struct rtm_ctx {
   DevBuf s_own, e_own;              // internal concatenation
   uint64_t s_own_n = 0, e_own_n = 0;
   // per-call workspaces
-  DevBuf T, Bs, Be, rts, rte, treg_s, treg_e, tdesc, soff, stage, smeta, emeta, lastlvl, res, kdelta, cdelta, active,
+  DevBuf T, Bs, Be, rts, rte, treg_s, treg_e, tdesc, soff, stage, stage2, woff, smeta, emeta, lastlvl, res, kdelta, cdelta, active,
       anyfull, hung, unit_ctr, bstat, comps, pack, gathered;
   Pinned h_small, h_res;
   // results of the last call
@@ -397,6 +398,12 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   if ((s = ensure(c, c->tdesc, (size_t)nts * sizeof(TileDesc)))) return s;
   if ((s = ensure(c, c->soff, (size_t)nts * (c->nbins + 1) * 2))) return s;
   if ((s = ensure(c, c->stage, (size_t)nts * kTileS * 8))) return s;
+  // more than 170 bins: two-pass partition (superbins, then bins per (window, superbin))
+  const bool two_pass = partition_two_pass(c->nbins, p.narrow != 0);
+  if (two_pass) {
+    if ((s = ensure(c, c->stage2, (size_t)nts * kTileS * 8))) return s;
+    if ((s = ensure(c, c->woff, (size_t)W * (c->nbins + 1) * 4))) return s;
+  }
   if ((s = ensure(c, c->smeta, (size_t)nts * sizeof(TileMeta)))) return s;
   if ((s = ensure(c, c->emeta, (size_t)nte * sizeof(TileMeta)))) return s;
   if ((s = ensure(c, c->lastlvl, Wn * c->nb * 2))) return s;
@@ -448,6 +455,11 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.tdesc = (TileDesc *)c->tdesc.p; p.tile_reg_s = (const uint32_t *)c->treg_s.p; p.tile_reg_e = (const uint32_t *)c->treg_e.p;
   p.n_tiles_s = nts; p.n_tiles_e = nte;
   p.soff = (uint16_t *)c->soff.p; p.stage = (unsigned long long *)c->stage.p;
+  if (two_pass) {
+    p.nsb = (c->nb + (1u << kSupLog) - 1) >> kSupLog;
+    p.stage2 = (unsigned long long *)c->stage2.p;
+    p.woff = (uint32_t *)c->woff.p;
+  }
   p.smeta = (TileMeta *)c->smeta.p; p.emeta = (TileMeta *)c->emeta.p;
   p.lastlvl = (uint16_t *)c->lastlvl.p; p.flags = (uint32_t *)c->flags.p;
   set_result_ptrs(c, W, p);
@@ -479,7 +491,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   // partition kernel runs the event tiles after its sample tiles (claimed dynamically), so no
   // concurrent kernel competes with the issue-bound fold.  Otherwise: a side stream, overlapped
   // with the partition and the fold, joined before the kernels that read the event outputs.
-  p.fuse_events = partition_fuses_events(p.nbins, nts) ? 1 : 0;
+  p.fuse_events = partition_fuses_events(p.nbins, nts, two_pass) ? 1 : 0;
   if (!p.fuse_events) {
     CK(cudaEventRecord(c->ev_fork, c->st));
     CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
@@ -508,6 +520,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     if (c->prof) prof_end_on(c, c->st2);
     CK(cudaEventRecord(c->ev_join, c->st2));
   }
+  if (p.nsb) LAUNCH(KT_SUBPART, 0, launch_subpart(p, c->n_sms, c->st));
   LAUNCH(KT_FOLD, 0, launch_fold(p, c->n_sms, c->st));
   if (side || !p.fuse_events) CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
   if (!side) LAUNCH(KT_ORDER, 0, launch_order_check(p, c->st));
@@ -535,6 +548,8 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     unsigned long long h[8];
     cudaMemcpyAsync(h, p.dbg, 64, cudaMemcpyDeviceToHost, c->st);
     cudaStreamSynchronize(c->st);
+    fprintf(stderr, "[lookback] units=%llu steps=%llu (%.2f / unit) spins=%llu\n", (unsigned long long)W * c->nbins,
+            h[0], (double)h[0] / ((double)W * c->nbins), h[6]);
     if (h[7])
       fprintf(stderr, "[phase] tiles=%llu  -=%.0f wait_raw=%.0f scan=%.0f rank=%.0f B1=%.0f bases+scatter=%.0f -=%.0f (cycles/tile, thread 0)\n",
               h[7], (double)h[0] / h[7], (double)h[1] / h[7], (double)h[2] / h[7], (double)h[3] / h[7],
@@ -774,7 +789,7 @@ void rtm_destroy(rtm_ctx *c) {
   DevBuf *bufs[] = {&c->cap, &c->owner, &c->elig, &c->ktotal, &c->carry[0], &c->carry[1], &c->run[0], &c->run[1],
                     &c->kstart, &c->rcp, &c->elig_ids, &c->gid, &c->bstat_g,
                     &c->kend, &c->cstart, &c->cend, &c->flags, &c->s_own, &c->e_own, &c->T, &c->Bs, &c->Be,
-                    &c->rts, &c->rte, &c->treg_s, &c->treg_e, &c->tdesc, &c->soff, &c->stage, &c->smeta, &c->emeta,
+                    &c->rts, &c->rte, &c->treg_s, &c->treg_e, &c->tdesc, &c->soff, &c->stage, &c->stage2, &c->woff, &c->smeta, &c->emeta,
                     &c->lastlvl, &c->res, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
                     &c->unit_ctr, &c->bstat, &c->comps, &c->pack,
                     &c->gathered, &c->tkscr, &c->mkey, &c->rcp64, &c->tkey, &c->persist, &c->klive,

@@ -7,6 +7,8 @@
 //                   tile tables; grid sync; per-tile descriptors
 //   K1 partition  : one CTA per 4096-sample tile of one region; validate, order-check, stable
 //                   multisplit of kept samples by 256-buffer bin into 8-byte staging entries
+//   K1b subpart   : (> 170 bins) K1 keys by superbin; per (window, superbin) a stable counting sort
+//                   by bin into (window, bin)-contiguous staging
 //   K3 events     : one CTA per 4096-event tile; progress deltas, component activity bitmaps
 //   K2 fold       : one warp per (window, bin) unit, dequeued in window order; in-order fold of
 //                   the bin's samples (delta form of the integral), carry-in resolved by
@@ -37,7 +39,8 @@ constexpr int kK3Threads = 256;
 constexpr int kFoldWarps = RTM_FOLD_WARPS;  // warps per fold CTA (compile-time A/B override)
 constexpr uint16_t kSent = 0xFFFFu;         // "no kept sample in this window" marker
 constexpr uint32_t kMaxBins = 4096;         // n_buffers <= 2^20 (fallback partition smem 160 KB)
-constexpr uint32_t kTopkSmemKeys = 40960;   // keys held in shared memory by the top-k kernel
+constexpr uint32_t kTopkSmemKeys = 40960;
+constexpr int kSupLog = 14;                 // two-pass partition: superbins of 2^14 buffers (<= 64 of them)   // keys held in shared memory by the top-k kernel
 // ts offset field of a staging entry: 48 - bin_log bits (entry = off << (16 + bin_log) | level << bin_log | lid)
 inline int64_t max_window_len(int bin_log) { return (int64_t)1 << (bin_log >= 8 ? 40 : 48 - bin_log > 40 ? 40 : 48 - bin_log); }
 
@@ -145,6 +148,12 @@ struct Params {
   uint32_t watch[RTM_WATCH_MAX];
   rtm_buffer_stat *wstat;    // [W * RTM_WATCH_MAX] per-window statistics of the watched buffers
   unsigned long long *dbg;   // phase-timing scratch (RTM_PHASE_TIMING builds only)
+  // two-pass path (> 170 bins, narrow windows): pass 1 partitions by superbin (buffer_id >> kSupLog)
+  // into stage / soff (rows of nsb + 1); k_subpart re-partitions every (window, superbin) by bin
+  // into stage2, (window, bin)-contiguous: bin b of window w is stage2[woff[w][b] .. woff[w][b+1])
+  uint32_t nsb;              // superbins (0: one-pass path)
+  unsigned long long *stage2;// [n_tiles_s * kTileS]
+  uint32_t *woff;            // [W * (nbins + 1)]
 };
 
 // launchers (rtm_kernels.cu); all asynchronous on `st`
@@ -153,7 +162,9 @@ struct ClearList;
 void launch_prep(const Params &p, const ClearList &cl, long long *Bs, long long *Be, int n_sms, cudaStream_t st);
 void launch_partition(const Params &p, int n_sms, cudaStream_t st);
 void launch_events(const Params &p, cudaStream_t st);
-bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s);  // lane-major partition path
+bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s, bool two_pass);  // lane-major partition path
+bool partition_two_pass(uint32_t nbins, bool narrow);  // > 170 bins: superbins + k_subpart
+void launch_subpart(const Params &p, int n_sms, cudaStream_t st);
 void launch_fold(const Params &p, int n_sms, cudaStream_t st);
 void launch_order_check(const Params &p, cudaStream_t st);
 void launch_topk(const Params &p, cudaStream_t st);

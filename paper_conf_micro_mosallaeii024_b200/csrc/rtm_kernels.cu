@@ -522,10 +522,11 @@ __device__ __forceinline__ void k1_tile_summary(const Params &p, const K1Tile &t
 
 // After B1 (window tiles): this warp's bin bases -> myb; warp 0 writes the soff row.  Returns the
 // tile's kept total.
+template <int KS>
 __device__ __forceinline__ unsigned k1_bin_bases(const Params &p, unsigned tile, const unsigned short *wt,
                                                  unsigned short *myb) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const unsigned nbins = p.nbins;
+  const unsigned nbins = KS == 8 ? p.nbins : p.nsb;
   uint16_t *offs = p.soff + (size_t)tile * (nbins + 1);
   unsigned carry = 0;
   for (unsigned b0 = 0; b0 < nbins; b0 += 32) {
@@ -577,7 +578,9 @@ __device__ __forceinline__ void k1_publish(K1WarpSum *wsum, unsigned long long f
 // One lane's 16 consecutive records: field check, running min / max of the field-valid offsets
 // (an inversion inside the lane shows up as an offset below the running max), entries, keys.
 // NAR: windows shorter than 2^32 ticks, so offsets are compared and packed in 32 bits.
-template <bool NAR, int BL, bool CAPS>
+// KS: key = buffer_id >> KS.  KS == 8: the bin (entries as above).  KS == kSupLog: the superbin
+// of the two-pass path (narrow windows only): entry = o << 32 | level << 16 | (buffer_id & 0x3FFF).
+template <bool NAR, int BL, bool CAPS, int KS>
 __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool is_win, const int4 *raw,
                                         const unsigned short *capS, int sub0, unsigned long long (&e)[kPerLane],
                                         unsigned (&kp)[kPerLane], unsigned long long &first,
@@ -601,9 +604,13 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
       mx = max(mx, valid ? o : 0u);
       mn = min(mn, valid ? o : ~0u);
       hiacc |= valid ? (unsigned)(off >> 32) : 0u;
-      // (o << 24) | (level << 8) | (buffer_id & 255), o < 2^32
-      const unsigned lo = __byte_perm(__byte_perm((unsigned)v.z, (unsigned)v.w, 0x0540), o, 0x4210);
-      e[k] = ((unsigned long long)(o >> 8) << 32) | lo;
+      if constexpr (KS == kSupLog) {
+        e[k] = ((unsigned long long)o << 32) | (lvl << 16) | (b & ((1u << kSupLog) - 1u));
+      } else {
+        // (o << 24) | (level << 8) | (buffer_id & 255), o < 2^32
+        const unsigned lo = __byte_perm(__byte_perm((unsigned)v.z, (unsigned)v.w, 0x0540), o, 0x4210);
+        e[k] = ((unsigned long long)(o >> 8) << 32) | lo;
+      }
     } else {
       bad |= valid & (off < mx64);
       mx64 = max(mx64, valid ? off : 0ull);
@@ -612,7 +619,7 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
     }
     const bool keep = valid & is_win;
     kept += keep;
-    kp[k] = (keep ? (b >> BL) : kNoKey) << 16;
+    kp[k] = (keep ? (b >> KS) : kNoKey) << 16;
   }
   if (NAR) {
     bad |= hv & ((hiacc != 0u) | ((unsigned long long)mx >= t.wlen));
@@ -648,14 +655,15 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
 // and only then prefetch their next raw records (named barrier among themselves); warps 4-7
 // prefetch before the first barrier (measured 813 -> 692 us on C2 against direct 8-byte scatter
 // stores from every lane, which touched 32 sectors per store instruction).
-template <int BL, bool CAPS>
+template <int BL, bool CAPS, int KS>
 __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   static_assert(BL == 8, "lane-major entries pack the buffer id in one byte");
+  static_assert(KS == 8 || KS == kSupLog, "bins or superbins");
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ K1WarpSum wsum[2][kK1Warps];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
-  const unsigned nbins = p.nbins;
+  const unsigned nbins = KS == 8 ? p.nbins : p.nsb;  // keys of this pass
   const size_t vb = k1_vec_bytes(nbins);
   unsigned char *tail = smem + (size_t)kTileS * 16;
   unsigned short *wt2 = reinterpret_cast<unsigned short *>(tail);            // [2][8][nbins]
@@ -726,8 +734,8 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     unsigned long long first, last;
     bool has, viol;
     unsigned kept = 0;
-    if (p.narrow && is_win) lm_scan<true, BL, CAPS>(p, t, is_win, raw, capS, sub0, e, kp, first, last, has, viol, kept);
-    else lm_scan<false, BL, CAPS>(p, t, is_win, raw, capS, sub0, e, kp, first, last, has, viol, kept);
+    if (p.narrow && is_win) lm_scan<true, BL, CAPS, KS>(p, t, is_win, raw, capS, sub0, e, kp, first, last, has, viol, kept);
+    else lm_scan<false, BL, CAPS, KS>(p, t, is_win, raw, capS, sub0, e, kp, first, last, has, viol, kept);
     {  // order across lanes: my first vs the last of the nearest earlier lane with a valid record
       const unsigned hm = __ballot_sync(kFull, has);
       const unsigned lower = hm & lt;
@@ -799,7 +807,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     {
       unsigned total = 0;
       if (is_win) {
-        total = k1_bin_bases(p, tile, wt, myb);
+        total = k1_bin_bases<KS>(p, tile, wt, myb);
         unsigned long long *sst = reinterpret_cast<unsigned long long *>(smem);
 #pragma unroll
         for (int k = 0; k < kPerLane; ++k) {
@@ -963,6 +971,243 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
   for (unsigned q = threadIdx.x; q < (total + 1) / 2; q += kK1Threads) d4[q] = s4[q];
 }
 
+
+// ============================================================================================
+// K1b (two-pass path: more than 170 bins, windows shorter than 2^32 ticks).  Pass 1 is the
+// lane-major partition keyed by superbin (buffer_id >> 14, <= 64 keys), entries
+// o << 32 | level << 16 | (buffer_id & 0x3FFF).  Here, one warp per (window, superbin) unit,
+// claimed in window order: the unit's entries (its (tile, superbin) segments in ingest order)
+// are re-partitioned by bin into (window, bin)-contiguous staging in the fold's entry format.
+// Sweep 1 counts the unit's entries per bin (shared atomics) and fixes every bin's output range
+// (woff); sweep 2 takes 512-entry chunks in ingest order, lane-major (lane l: chunk entries
+// 16l .. 16l+15) as in K1, so the stable rank is a u8 (bin, lane) counter plus earlier lanes'
+// counts (byte-SIMD prefix); the chunk is permuted by bin in shared memory and each bin's run is
+// appended at its cursor.  The fold then reads one contiguous range per (window, bin) unit
+// instead of one segment per tile of the window (C4: ~220 tiles per window, ~1 entry per
+// segment).
+// ============================================================================================
+constexpr int kSubWarps = 8;
+template <int BL>
+struct SubSmem {
+  static constexpr int kNB = 1 << (kSupLog - BL);  // bins per superbin: 64 (BL 8) or 128 (BL 7)
+  unsigned long long buf[kSub];  // the loaded chunk (swizzled), then its permutation by bin
+  unsigned char rows[kNB * 48];  // per bin: 32 u8 lane counters / in-word prefixes + 8 u16 word bases
+  unsigned cur[kNB];             // sweep 1: counts; sweep 2: output cursor of each bin
+  unsigned short cb[kNB];        // chunk base of each bin
+  unsigned short ct[kNB];        // chunk count of each bin
+  unsigned seg_base[32];
+};
+
+template <int BL>
+__global__ void __launch_bounds__(kSubWarps * 32, 2) k_subpart(Params p) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  using SS = SubSmem<BL>;
+  constexpr int kNB = SS::kNB, kPerB = kNB / 32;
+  SS &Q = reinterpret_cast<SS *>(smem)[threadIdx.x >> 5];
+  const int lane = threadIdx.x & 31;
+  const unsigned lt = lanemask_lt(), le = (2u << lane) - 1u;
+  const unsigned nsb = p.nsb, nbins = p.nbins, rs = nsb + 1;
+  const unsigned n_units = p.W * nsb;
+  // the unit's tile group [tg, tg + 32): flattened segment table -> Q.seg_base, returns the total
+  auto group = [&](unsigned tg, unsigned t_hi, unsigned S, unsigned &my_end) -> unsigned {
+    unsigned seg_lo = 0, seg_len = 0;
+    if (tg + lane < t_hi) {
+      const uint16_t *o = p.soff + (size_t)(tg + lane) * rs + S;
+      seg_lo = __ldg(o);
+      seg_len = (unsigned)__ldg(o + 1) - seg_lo;
+    }
+    unsigned pre = seg_len;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned y = __shfl_up_sync(kFull, pre, o);
+      if (lane >= o) pre += y;
+    }
+    const unsigned nonempty = __ballot_sync(kFull, seg_len != 0);
+    __syncwarp();  // the previous group's seg_base reads are done
+    if (seg_len) Q.seg_base[__popc(nonempty & lt)] = (tg + lane) * (unsigned)kTileS + seg_lo - (pre - seg_len);
+    my_end = seg_len ? pre : 0xFFFFFFFFu;
+    __syncwarp();
+    return __shfl_sync(kFull, pre, 31);
+  };
+  // staging index of flattened position c + lane of the group, ~0u past its end (c advances by
+  // 32 per call).  Addresses first, loads after: a unit's loads are issued in batches, so the
+  // warp waits for DRAM once per batch instead of once per 32 entries.
+  auto addr = [&](unsigned c, unsigned total, unsigned my_end, unsigned &seg_before) -> unsigned {
+    const unsigned x = my_end - c;
+    const unsigned ends = __reduce_or_sync(kFull, x < 32u ? 1u << x : 0u);
+    const unsigned sgi = seg_before + __popc(ends & le);
+    seg_before += __popc(ends);
+    const unsigned g = c + lane;
+    return g < total ? Q.seg_base[sgi] + g : ~0u;
+  };
+  auto ld = [&](unsigned i) -> unsigned long long { return i != ~0u ? __ldcs(p.stage + i) : 0ull; };
+  for (;;) {
+    unsigned u = 0;
+    if (lane == 0) u = atomicAdd(p.unit_ctr + 3, 1u);
+    u = __shfl_sync(kFull, u, 0);
+    if (u >= n_units) break;
+    const unsigned w = u / nsb, S = u % nsb;
+    const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
+    // the unit's output base: the window's staging region + its entries of lower superbins
+    unsigned before = 0;
+    for (unsigned t = t_lo + lane; t < t_hi; t += 32) before += __ldg(p.soff + (size_t)t * rs + S);
+    before = warp_sum(before);
+    const unsigned ubase = t_lo * (unsigned)kTileS + before;
+#pragma unroll
+    for (int j = 0; j < kPerB; ++j) Q.cur[lane + 32 * j] = 0;
+    __syncwarp();
+    // ---- sweep 1: entries per bin
+    for (unsigned tg = t_lo; tg < t_hi; tg += 32) {
+      unsigned my_end;
+      const unsigned total = group(tg, t_hi, S, my_end);
+      unsigned sb = 0;
+      for (unsigned c = 0; c < total; c += 256) {  // 8 steps per batch
+        unsigned ix[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) ix[j] = c + 32u * j < total ? addr(c + 32u * j, total, my_end, sb) : ~0u;
+        unsigned long long v[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[j] = ld(ix[j]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+          if (ix[j] != ~0u) atomicAdd(&Q.cur[((unsigned)v[j] & ((1u << kSupLog) - 1u)) >> BL], 1u);
+      }
+    }
+    __syncwarp();
+    {  // bin ranges: exclusive scan of the counts (lane: kPerB consecutive bins)
+      unsigned v[kPerB], tot = 0;
+#pragma unroll
+      for (int j = 0; j < kPerB; ++j) {
+        v[j] = Q.cur[kPerB * lane + j];
+        tot += v[j];
+      }
+      unsigned incl = tot;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+      }
+      unsigned run = ubase + incl - tot;
+      unsigned *wo = p.woff + (size_t)w * (nbins + 1);
+#pragma unroll
+      for (int j = 0; j < kPerB; ++j) {
+        const unsigned bin = S * kNB + kPerB * lane + j;
+        if (bin < nbins) wo[bin] = run;
+        Q.cur[kPerB * lane + j] = run;
+        run += v[j];
+      }
+      if (S == nsb - 1 && lane == 31) wo[nbins] = run;  // the window's end
+    }
+    __syncwarp();
+    // ---- sweep 2: stable scatter, 512-entry chunks
+    for (unsigned tg = t_lo; tg < t_hi; tg += 32) {
+      unsigned my_end;
+      const unsigned total = group(tg, t_hi, S, my_end);
+      unsigned sb = 0;
+      for (unsigned c0 = 0; c0 < total; c0 += kSub) {
+        const unsigned n = total - c0 < (unsigned)kSub ? total - c0 : (unsigned)kSub;
+        // load (coalesced, lane-strided) into the swizzled chunk: entry i at row i >> 4, column
+        // (i & 15) ^ (row & 15), so the lane-major read below is conflict-free per half-warp
+        {
+          unsigned ix[kPerLane];
+          // warp-uniform condition: addr is a warp collective, called once per 32-position step
+#pragma unroll
+          for (int j = 0; j < kPerLane; ++j) ix[j] = 32u * j < n ? addr(c0 + 32u * j, total, my_end, sb) : ~0u;
+          unsigned long long v[kPerLane];
+#pragma unroll
+          for (int j = 0; j < kPerLane; ++j) v[j] = ld(ix[j]);
+#pragma unroll
+          for (int j = 0; j < kPerLane; ++j) {
+            const unsigned i = 32u * j + lane;
+            Q.buf[(i & ~15u) | ((i & 15u) ^ ((i >> 4) & 15u))] = v[j];
+          }
+        }
+        __syncwarp();
+        uint4 *r4 = reinterpret_cast<uint4 *>(Q.rows);
+        for (unsigned q = lane; q < (unsigned)kNB * 3; q += 32) r4[q] = make_uint4(0, 0, 0, 0);
+        __syncwarp();
+        unsigned long long e[kPerLane];
+        unsigned kp[kPerLane];
+#pragma unroll
+        for (int k = 0; k < kPerLane; ++k) {
+          e[k] = Q.buf[16 * lane + (k ^ (lane & 15))];
+          const unsigned key = 16u * lane + k < n ? ((unsigned)e[k] & ((1u << kSupLog) - 1u)) >> BL : kNoKey;
+          kp[k] = key << 16;
+          if (key != kNoKey) {
+            unsigned char *ctr = Q.rows + key * 48 + lane;
+            const unsigned r = *ctr;
+            *ctr = (unsigned char)(r + 1);
+            kp[k] |= r;
+          }
+        }
+        __syncwarp();
+#pragma unroll
+        for (int j = 0; j < kPerB; ++j) {  // one bin row per lane and step: byte-SIMD prefix
+          const unsigned b = lane + 32 * j;
+          uint4 *row = reinterpret_cast<uint4 *>(Q.rows + b * 48);
+          const uint4 q0 = row[0], q1 = row[1];
+          unsigned wv[8] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w};
+          unsigned base[8];
+          unsigned run = 0;
+#pragma unroll
+          for (int x = 0; x < 8; ++x) {
+            const unsigned incl = wv[x] * 0x01010101u;
+            base[x] = run;
+            run += incl >> 24;
+            wv[x] = incl - wv[x];
+          }
+          row[0] = make_uint4(wv[0], wv[1], wv[2], wv[3]);
+          row[1] = make_uint4(wv[4], wv[5], wv[6], wv[7]);
+          row[2] = make_uint4(base[0] | (base[1] << 16), base[2] | (base[3] << 16), base[4] | (base[5] << 16),
+                              base[6] | (base[7] << 16));
+          Q.ct[b] = (unsigned short)run;
+        }
+        __syncwarp();
+        {  // chunk bases: exclusive scan of the chunk counts
+          unsigned v[kPerB], tot = 0;
+#pragma unroll
+          for (int j = 0; j < kPerB; ++j) {
+            v[j] = Q.ct[kPerB * lane + j];
+            tot += v[j];
+          }
+          unsigned incl = tot;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const unsigned y = __shfl_up_sync(kFull, incl, o);
+            if (lane >= o) incl += y;
+          }
+          unsigned run = incl - tot;
+#pragma unroll
+          for (int j = 0; j < kPerB; ++j) {
+            Q.cb[kPerB * lane + j] = (unsigned short)run;
+            run += v[j];
+          }
+        }
+        __syncwarp();
+        const unsigned short *rows16 = reinterpret_cast<const unsigned short *>(Q.rows);
+#pragma unroll
+        for (int k = 0; k < kPerLane; ++k) {
+          const unsigned key = kp[k] >> 16;
+          if (key != kNoKey)
+            Q.buf[Q.cb[key] + (kp[k] & 0xFFFFu) + Q.rows[key * 48 + lane] + rows16[key * 24 + 16 + (lane >> 2)]] = e[k];
+        }
+        __syncwarp();
+        // copy out: each bin's run of the chunk appended at its cursor, in the fold's format
+        for (unsigned q = lane; q < n; q += 32) {
+          const unsigned long long x = Q.buf[q];
+          const unsigned key = ((unsigned)x & ((1u << kSupLog) - 1u)) >> BL;
+          const unsigned dst = Q.cur[key] + (q - Q.cb[key]);
+          const unsigned long long lvl = (x >> 16) & 0xFFFFull;
+          __stcg(p.stage2 + dst, ((x >> 32) << (16 + BL)) | (lvl << BL) | (x & ((1u << BL) - 1u)));
+        }
+        __syncwarp();
+#pragma unroll
+        for (int j = 0; j < kPerB; ++j) Q.cur[lane + 32 * j] += Q.ct[lane + 32 * j];
+        __syncwarp();
+      }
+    }
+  }
+}
 
 // Persistence ranking key (rank mode MEAN): floor(I * 2^32 / c), exact.  Within a window the
 // mean occupancy I / (c * W) orders like I / c; distinct ratios I1/c1 != I2/c2 differ by at least
@@ -1171,7 +1416,13 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
           }
         }
         if (RTM_SPIN_RELAXED) (void)ld_acquire_u32(f);
+#ifdef RTM_PHASE_TIMING
+        if (p.dbg) atomicAdd(p.dbg + 6, (unsigned long long)spins);
+#endif
       }
+#ifdef RTM_PHASE_TIMING
+      if (lane == 0 && p.dbg) atomicAdd(p.dbg + 0, 1ull);
+#endif
       __syncwarp();
       const unsigned short *lj = p.lastlvl + (size_t)j * p.nb + b_base + lane;
       if constexpr (kStep > 1) {
@@ -1310,6 +1561,20 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
 template <bool NAR, int BL>
 __device__ __forceinline__ void fold_phase1(const Params &p, FoldSmem<BL> &S, unsigned w, unsigned bin,
                                             unsigned long long Wlen, int lane, unsigned lt) {
+  if (p.woff) {  // two-pass path: the unit's entries are one contiguous range
+    const unsigned *wo = p.woff + (size_t)w * (p.nbins + 1) + bin;
+    const unsigned lo = __ldg(wo), total = __ldg(wo + 1) - lo;
+    const unsigned long long *src = p.stage2 + lo;
+    auto fetch = [&](unsigned c) -> unsigned long long { return c + lane < total ? __ldcs(src + c + lane) : 0ull; };
+    unsigned long long e0 = fetch(0), e1 = fetch(32);
+    for (unsigned c = 0; c < total; c += 32) {
+      const unsigned long long en = fetch(c + 64);
+      fold_chunk<NAR, BL>(S, lane, lt, c + lane < total, e0, Wlen);
+      e0 = e1;
+      e1 = en;
+    }
+    return;
+  }
   const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
   {
     // ---- phase 1: the (tile, bin) segments of window w, flattened into one stream of chunks
@@ -1586,6 +1851,38 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
     // segment offsets are in flight, window w-1 is finalized (a window's chain of dependent
     // loads - tile range, segment offsets, entries - would otherwise stall the warp every window).
     // Fast path: a window's segments for this bin span <= 32 tiles; else fold_phase1.
+    if (p.woff) {  // two-pass path: one contiguous range per (window, bin)
+      const unsigned rs = p.nbins + 1;
+      unsigned n_lo = __ldg(p.woff + bin), n_hi = __ldg(p.woff + bin + 1);
+      bool pend = false;
+      unsigned pw = 0;
+      unsigned long long pWlen = 0;
+      for (unsigned w = 0; w < p.W; ++w) {
+        const long long tb = p.T[w], te = p.T[w + 1];
+        const unsigned long long Wlen = (unsigned long long)(te - tb);
+        const unsigned total = n_hi - n_lo;
+        const unsigned long long *src = p.stage2 + n_lo;
+        auto fetch = [&](unsigned c) -> unsigned long long { return c + lane < total ? __ldcs(src + c + lane) : 0ull; };
+        unsigned long long e0 = fetch(0), e1 = total > 32u ? fetch(32) : 0ull;
+        if (w + 1 < p.W) {  // the next window's range (in flight during the finalize)
+          n_lo = __ldg(p.woff + (size_t)(w + 1) * rs + bin);
+          n_hi = __ldg(p.woff + (size_t)(w + 1) * rs + bin + 1);
+        }
+        if (pend) finalize(pw, pWlen);
+        for (unsigned c = 0; c < total; c += 32) {
+          const unsigned long long en = c + 64 < total ? fetch(c + 64) : 0ull;
+          fold_chunk<NAR, BL>(S, lane, lt, c + lane < total, e0, Wlen);
+          e0 = e1;
+          e1 = en;
+        }
+        __syncwarp();
+        pend = true;
+        pw = w;
+        pWlen = Wlen;
+      }
+      if (pend) finalize(pw, pWlen);
+      continue;
+    }
     unsigned n_tlo = p.rts[1], n_thi = p.rts[2];
     unsigned n_lo = 0, n_len = 0;
     bool n_ok = n_thi - n_tlo <= 32u;
@@ -2656,26 +2953,59 @@ void launch_prep(const Params &p, const ClearList &cl, long long *Bs, long long 
   count_launch();
 }
 
-bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s) { return n_tiles_s && nbins <= kLmMaxBins; }
+// measured (1 x B200, full-size configs): 320 bins (C3) the match-based partition and the two-pass
+// path tie (28.5 vs 29.4 ms per step: k_subpart reads the entries twice at ~4 warp instructions
+// each); 2560 bins (C5) fold 22.4 -> 17.9 ms per 10k windows; 4096 bins (C4) 132.5 -> 77.5 ms
+constexpr uint32_t kTwoPassMinBins = 1024;
+bool partition_two_pass(uint32_t nbins, bool narrow) { return nbins >= kTwoPassMinBins && narrow; }
+bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s, bool two_pass) {
+  return n_tiles_s && (nbins <= kLmMaxBins || two_pass);
+}
 
-template <int BL, bool CAPS>
+template <int BL>
+void launch_subpart_bl(const Params &p, int n_sms, cudaStream_t st) {
+  const size_t sm = sizeof(SubSmem<BL>) * kSubWarps;
+  int per_sm = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_subpart<BL>, kSubWarps * 32, sm);
+  if (per_sm < 1) per_sm = 1;
+  unsigned grid = (unsigned)(n_sms * per_sm);
+  const unsigned need = (p.W * p.nsb + kSubWarps - 1) / kSubWarps;
+  if (grid > need) grid = need;
+  if (grid == 0) grid = 1;
+  { k_subpart<BL><<<grid, kSubWarps * 32, sm, st>>>(p); count_launch(); }
+}
+
+void launch_subpart(const Params &p, int n_sms, cudaStream_t st) {
+  if (!p.nsb || !p.n_tiles_s) return;
+  if (p.bin_log == 7) launch_subpart_bl<7>(p, n_sms, st);
+  else launch_subpart_bl<8>(p, n_sms, st);
+}
+
+template <int BL, bool CAPS, int KS>
 void launch_partition_lm(const Params &p, int n_sms, size_t sm, cudaStream_t st) {
   int per_sm = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm<BL, CAPS>, kK1Threads, sm);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm<BL, CAPS, KS>, kK1Threads, sm);
   if (per_sm < 1) per_sm = 1;
   unsigned grid = (unsigned)(n_sms * per_sm);
   const unsigned work = p.n_tiles_s + (p.fuse_events ? p.n_tiles_e : 0u);
   if (grid > work) grid = work;
-  { k_partition_lm<BL, CAPS><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
+  { k_partition_lm<BL, CAPS, KS><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
 }
 
 void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   if (!p.n_tiles_s) return;
+  if (p.nsb) {  // two-pass path, pass 1: superbin keys (capacities through L1: > 2^15 buffers)
+    const bool caps = partition_caps_smem(p.nsb, p.nb);
+    const size_t sm = k1_smem_lm(p.nsb, p.nb, caps);
+    if (caps) launch_partition_lm<8, true, kSupLog>(p, n_sms, sm, st);
+    else launch_partition_lm<8, false, kSupLog>(p, n_sms, sm, st);
+    return;
+  }
   const size_t sm = partition_smem_bytes(p.nbins, p.nb);
   if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM
     // bin_log 8 here: bin_log 7 is only chosen for > 131072 buffers (> 170 bins)
-    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true>(p, n_sms, sm, st);
-    else launch_partition_lm<8, false>(p, n_sms, sm, st);
+    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 8>(p, n_sms, sm, st);
+    else launch_partition_lm<8, false, 8>(p, n_sms, sm, st);
   } else {
     if (p.bin_log == 7) { k_partition_mx<7><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
     else { k_partition_mx<8><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
@@ -2807,8 +3137,12 @@ void configure_kernels_once() {
   done[dev] = true;
   const int lm_caps = (int)k1_smem_lm(kLmMaxBins, 113 * 512, true);  // <= 113 KB by partition_caps_smem
   const int lm_glob = (int)k1_smem_lm(kLmMaxBins, 0, false);
-  cudaFuncSetAttribute(k_partition_lm<8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
-  cudaFuncSetAttribute(k_partition_lm<8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  cudaFuncSetAttribute(k_partition_lm<8, true, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  cudaFuncSetAttribute(k_partition_lm<8, true, kSupLog>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false, kSupLog>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  cudaFuncSetAttribute(k_subpart<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(SubSmem<7>) * kSubWarps));
+  cudaFuncSetAttribute(k_subpart<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(SubSmem<8>) * kSubWarps));
   cudaFuncSetAttribute(k_partition_mx<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
   cudaFuncSetAttribute(k_partition_mx<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
   cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));

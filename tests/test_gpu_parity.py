@@ -521,6 +521,41 @@ def test_many_bins_partition_paths(n_buffers):
     assert_same(got, ref, mon)
 
 
+@pytest.mark.parametrize("case", ["ragged_invalid", "mean_1m", "very_sparse_bl7", "wide_windows"])
+def test_two_pass_partition_paths(case):
+    """Registries of >= 1024 bins take the two-pass partition (lane-major by 16384-buffer superbin,
+    then k_subpart sorts every (window, superbin) by bin into (window, bin)-contiguous staging)
+    when every window is shorter than 2^32 ticks; wider windows keep the match-based partition.
+    Cases: a ragged last superbin (262444 buffers) with 1 % invalid records and empty windows;
+    2^20 buffers in rank mode MEAN (windowed fold + 64-bit keys); 327680 buffers (bins of 128)
+    in a very sparse call (sequential fold); a window of 2^33 ticks (fallback partition)."""
+    n_buffers = {"ragged_invalid": 262444, "mean_1m": 1 << 20, "very_sparse_bl7": 327680,
+                 "wide_windows": 262144}[case]
+    n_samples = 60_000 if case == "very_sparse_bl7" else 500_000
+    wl = gen.C1.scaled("C1-2p", n_samples=n_samples, n_events=n_samples // 10, n_buffers=n_buffers, n_windows=6,
+                       invalid_ppm=10_000 if case == "ragged_invalid" else 0)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    if case == "mean_1m":
+        kw["rank_mode"] = 2  # RTM_RANK_MEAN
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    s, e = gen.samples(wl), gen.events(wl)
+    t_end = wl.t_end()
+    if case == "ragged_invalid":  # empty windows: repeated ends
+        t_end = np.array([t_end[0], t_end[0], t_end[1], t_end[2], t_end[2], t_end[3], t_end[4], t_end[5]], np.int64)
+    elif case == "very_sparse_bl7":  # 60k samples over 327680 buffers x 40 windows: sequential fold
+        t_end = np.linspace(wl.t0 + 1, int(t_end[-1]), 40).astype(np.int64)
+        assert len(s) * 8 < n_buffers * len(t_end)
+    elif case == "wide_windows":
+        t_end = np.array([int(t_end[2]), int(t_end[2]) + (1 << 33)], np.int64)
+    ref = orc.reduce(s, e, t_end, want_all_stats=True)
+    mon.ingest(_dev(s), _dev(e))
+    got = mon.window_reduce(t_end)
+    assert_same(got, ref, mon)
+    if case == "ragged_invalid":
+        assert int(np.sum(ref["summary"]["n_dropped"])) > 0
+
+
 @pytest.mark.parametrize("n_buffers,k,calls", [(20480, 64, (1, 1, 3, 37, 1)), (65536, 1024, (1, 2)),
                                                 (16384, 16, (5, 1)), (20482, 64, (1, 2))])
 def test_topk_slices_few_window_calls(n_buffers, k, calls):
