@@ -300,6 +300,23 @@ rtm_status rtm_watch(rtm_ctx *ctx, const uint32_t *buffer_ids, uint32_t n);
  * *n_out that count.  RTM_E_INVALID for slot >= the watched count. */
 rtm_status rtm_watch_series(rtm_ctx *ctx, uint32_t slot, rtm_watch_point *out, uint32_t *n_out);
 
+/* Launch mechanism of rtm_window_reduce / rtm_window_reduce_local (results are identical).
+ * The call's kernels and copies form a fixed sequence for a given launch shape (window count,
+ * tile counts of the pending records, partition / fold variant): it can be captured once into a
+ * CUDA graph and replayed with only the kernels' arguments replaced, which removes the per-kernel
+ * launch cost of small calls (the list is refreshed for every window).
+ *   RTM_GRAPHS_OFF     direct launches
+ *   RTM_GRAPHS_AUTO    graphs for calls of <= 64 windows (default)
+ *   RTM_GRAPHS_ALWAYS  graphs for every call
+ * Up to 8 shapes are cached per context (least recently used evicted); a workspace growth drops
+ * them.  Profiling (rtm_profile) uses direct launches.  If the driver cannot capture the sequence
+ * the context falls back to direct launches for good.  RTM_E_INVALID for another mode. */
+typedef enum { RTM_GRAPHS_OFF = 0, RTM_GRAPHS_AUTO = 1, RTM_GRAPHS_ALWAYS = 2 } rtm_graph_mode;
+rtm_status rtm_use_graphs(rtm_ctx *ctx, int32_t mode);
+/* Calls of this context launched from a newly captured graph / by replaying a cached one
+ * (host outputs; the rest were direct launches). */
+rtm_status rtm_graph_stats(rtm_ctx *ctx, uint64_t *captured, uint64_t *replayed);
+
 /* Per-kernel CUDA-event timing on the context stream (off by default). */
 rtm_status rtm_profile(rtm_ctx *ctx, int32_t enable);
 rtm_status rtm_profile_read(rtm_ctx *ctx, rtm_kernel_time *out, uint32_t cap, uint32_t *n);

@@ -282,6 +282,18 @@ class Monitor:
         N.check(N.lib().rtm_watch_series(self._h, slot, out.ctypes.data, ctypes.byref(n)), "rtm_watch_series")
         return out[: n.value]
 
+    def use_graphs(self, mode: int = N.RTM_GRAPHS_AUTO):
+        """Launch mechanism of window_reduce (include/rtm.h rtm_use_graphs): RTM_GRAPHS_OFF direct
+        launches, RTM_GRAPHS_AUTO CUDA-graph replay for calls of <= 64 windows (default),
+        RTM_GRAPHS_ALWAYS for every call.  Results are identical."""
+        N.check(N.lib().rtm_use_graphs(self._h, int(mode)), "rtm_use_graphs")
+
+    def graph_stats(self):
+        """(calls launched from a newly captured CUDA graph, calls that replayed a cached one)."""
+        a, b = ctypes.c_uint64(), ctypes.c_uint64()
+        N.check(N.lib().rtm_graph_stats(self._h, ctypes.byref(a), ctypes.byref(b)), "rtm_graph_stats")
+        return int(a.value), int(b.value)
+
     def profile(self, enable: bool = True):
         N.check(N.lib().rtm_profile(self._h, 1 if enable else 0), "rtm_profile")
 

@@ -17,6 +17,7 @@ RTM_OK, RTM_E_INVALID, RTM_E_CUDA, RTM_E_COMM, RTM_E_ORDER, RTM_E_TOO_SMALL, RTM
     0, -1, -2, -3, -4, -5, -6, -7)
 RTM_MEM_HOST, RTM_MEM_DEVICE = 0, 1
 RTM_RANK_PERCENT, RTM_RANK_SIZE, RTM_RANK_MEAN = 0, 1, 2
+RTM_GRAPHS_OFF, RTM_GRAPHS_AUTO, RTM_GRAPHS_ALWAYS = 0, 1, 2
 
 # record and result layouts (include/rtm.h)
 SAMPLE_DTYPE = np.dtype([("ts", "<i8"), ("buffer_id", "<u4"), ("level", "<u2"), ("capacity", "<u2")])
@@ -63,7 +64,8 @@ EXPORTS = ("rtm_create", "rtm_destroy", "rtm_reset", "rtm_ingest", "rtm_window_r
            "rtm_merge", "rtm_profile", "rtm_profile_read", "rtm_status_str", "rtm_version",
            "rtm_kernel_launches", "rtm_watch", "rtm_watch_series", "rtm_topk_persistence",
            "rtm_bar_create", "rtm_bar_update", "rtm_bar_destroy", "rtm_set_links", "rtm_hang_roots",
-           "rtm_exchange_bytes", "rtm_sync_tables", "rtm_tables_local", "rtm_tables_merge")
+           "rtm_exchange_bytes", "rtm_sync_tables", "rtm_tables_local", "rtm_tables_merge", "rtm_use_graphs",
+           "rtm_graph_stats")
 
 _lib = None
 
@@ -104,10 +106,13 @@ def lib():
     L.rtm_sync_tables.argtypes = [vp]
     L.rtm_tables_local.argtypes = [vp, P(vp), P(u64)]
     L.rtm_tables_merge.argtypes = [vp, vp, u32]
+    L.rtm_use_graphs.argtypes = [vp, i32]
+    L.rtm_graph_stats.argtypes = [vp, P(u64), P(u64)]
     for fn in ("rtm_watch", "rtm_watch_series", "rtm_topk_persistence", "rtm_bar_create", "rtm_bar_update",
                "rtm_bar_destroy", "rtm_set_links", "rtm_hang_roots", "rtm_create", "rtm_reset", "rtm_ingest", "rtm_window_reduce", "rtm_topk_buffers", "rtm_progress",
                "rtm_hang_check", "rtm_buffer_stats", "rtm_window_reduce_local", "rtm_merge", "rtm_profile",
-               "rtm_profile_read", "rtm_window_results", "rtm_sync_tables", "rtm_tables_local", "rtm_tables_merge"):
+               "rtm_profile_read", "rtm_window_results", "rtm_sync_tables", "rtm_tables_local", "rtm_tables_merge",
+               "rtm_use_graphs", "rtm_graph_stats"):
         getattr(L, fn).restype = ctypes.c_int
     L.rtm_status_str.argtypes = [ctypes.c_int]
     L.rtm_status_str.restype = ctypes.c_char_p

@@ -31,6 +31,9 @@ struct Chunk {
   uint64_t n;
 };
 
+constexpr uint32_t kGraphAutoMaxWindows = 64;  // RTM_GRAPHS_AUTO: calls of at most this many windows
+constexpr size_t kGraphCacheSize = 8;           // launch shapes cached per context
+
 enum KernelId { KT_SPLIT, KT_PARTITION, KT_EVENTS, KT_FOLD, KT_ORDER, KT_TOPK, KT_HANG, KT_PROGRESS, KT_MERGE,
                 KT_SUBPART, KT_N };
 const char *kKernelNames[KT_N] = {"k_prep", "k_partition", "k_events", "k_fold", "k_order_check",
@@ -50,6 +53,21 @@ struct rtm_ctx {
   cudaStream_t st2 = nullptr;            // side stream (task events), joined per call
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   int n_sms;
+  // CUDA graphs of the reduce launch sequence (rtm_use_graphs): one per launch shape, replayed with
+  // the call's Params; valid while no workspace was reallocated (gen)
+  struct GraphEntry {
+    uint64_t key[3], gen, used;
+    cudaGraph_t g;
+    cudaGraphExec_t x;
+    std::vector<cudaGraphNode_t> kn;      // kernel nodes
+    std::vector<cudaKernelNodeParams> kp;  // their launch configurations
+  };
+  int32_t graph_mode = RTM_GRAPHS_AUTO;
+  cudaStream_t cap_st = nullptr;  // capture stream (the context stream may be the legacy default stream)
+  bool graph_broken = false;  // capture / instantiation unsupported here: direct launches only
+  uint64_t gen = 0, graph_tick = 0;
+  uint64_t graph_captures = 0, graph_replays = 0;  // rtm_graph_stats
+  std::vector<GraphEntry> graphs;
   DevBuf cap, owner, elig, ktotal, rcp, elig_ids;
   DevBuf gid, bstat_g;      // rank-local numbering: global id per local buffer, table by global id
   DevBuf tkscr;             // per-slice top-k candidates (few-window calls)
@@ -131,6 +149,7 @@ rtm_status ensure(rtm_ctx *c, DevBuf &b, size_t bytes, bool zero_new = false) {
   b.p = nullptr;
   b.cap = 0;
   size_t want = bytes + bytes / 4;
+  ++c->gen;  // cached CUDA graphs hold the old pointers
   cudaError_t e = cudaMalloc(&b.p, want);
   if (e != cudaSuccess) {
     cudaGetLastError();
@@ -153,6 +172,7 @@ rtm_status grow_keep(rtm_ctx *c, DevBuf &b, size_t bytes, size_t keep) {
   if (b.cap >= bytes) return RTM_OK;
   size_t want = std::max(bytes + bytes / 2, (size_t)1 << 20);
   void *np = nullptr;
+  ++c->gen;
   if (cudaMalloc(&np, want) != cudaSuccess) {
     cudaGetLastError();
     c->sticky = RTM_E_NOMEM;
@@ -170,6 +190,7 @@ rtm_status ensure_pinned(rtm_ctx *c, Pinned &h, size_t bytes) {
   if (h.cap >= bytes) return RTM_OK;
   if (h.p) cudaFreeHost(h.p);
   h.p = nullptr;
+  ++c->gen;
   size_t want = std::max(bytes + bytes / 4, (size_t)1 << 16);
   if (cudaMallocHost(&h.p, want) != cudaSuccess) {
     cudaGetLastError();
@@ -333,6 +354,116 @@ void set_result_ptrs(rtm_ctx *c, uint32_t W, Params &p) {
   p.wstat = (rtm_buffer_stat *)(d + L.watch);
 }
 
+// ---- CUDA graphs of the launch sequence (rtm_use_graphs) ------------------------------------
+bool graph_use(const rtm_ctx *c, uint32_t W) {
+#ifdef RTM_PHASE_TIMING
+  (void)c; (void)W;
+  return false;
+#else
+  if (c->prof || c->graph_broken) return false;
+  return c->graph_mode == RTM_GRAPHS_ALWAYS || (c->graph_mode == RTM_GRAPHS_AUTO && W <= kGraphAutoMaxWindows);
+#endif
+}
+
+void graph_free(rtm_ctx::GraphEntry &e) {
+  if (e.x) cudaGraphExecDestroy(e.x);
+  if (e.g) cudaGraphDestroy(e.g);
+  e.x = nullptr;
+  e.g = nullptr;
+}
+
+void graphs_clear(rtm_ctx *c) {
+  for (auto &e : c->graphs) graph_free(e);
+  c->graphs.clear();
+}
+
+// Replays the graph captured for this call's launch shape (capturing it first if needed).  A
+// replay replaces every kernel node's arguments with this call's (Params; k_prep: Params, clear
+// list, split buffers): the shape key fixes everything else - kernel variants, grids, shared
+// memory, the memcpy of the window bounds from the pinned staging (its pointer is guarded by the
+// workspace generation).
+template <typename F>
+rtm_status graph_launch(rtm_ctx *c, Params &p, const ClearList &cl, F &&enqueue) {
+  uint64_t key[3];
+  launch_shape(p, key);
+  rtm_ctx::GraphEntry *hit = nullptr;
+  for (auto &e : c->graphs)
+    if (e.gen == c->gen && e.key[0] == key[0] && e.key[1] == key[1] && e.key[2] == key[2]) hit = &e;
+  if (!hit) {
+    if (!c->graphs.empty() && c->graphs.front().gen != c->gen) graphs_clear(c);  // stale pointers
+    // Captured on a private non-blocking stream (capture is not permitted on the legacy default
+    // stream, which the context stream may be); replayed on the context stream.
+    if (!c->cap_st) CK(cudaStreamCreateWithFlags(&c->cap_st, cudaStreamNonBlocking));
+    cudaGraph_t g = nullptr;
+    cudaStream_t user = c->st;
+    cudaError_t ce = cudaStreamBeginCapture(c->cap_st, cudaStreamCaptureModeThreadLocal);
+    rtm_status s = RTM_OK;
+    if (ce == cudaSuccess) {
+      c->st = c->cap_st;
+      s = enqueue();
+      c->st = user;
+      ce = cudaStreamEndCapture(c->cap_st, &g);
+    }
+    if (s) {
+      if (g) cudaGraphDestroy(g);
+      return s;
+    }
+    cudaGraphExec_t x = nullptr;
+    if (ce != cudaSuccess || !g || cudaGraphInstantiate(&x, g, 0) != cudaSuccess) {
+      cudaGetLastError();  // capture of this sequence unsupported here: launch directly from now on
+      if (g) cudaGraphDestroy(g);
+      c->graph_broken = true;
+      return enqueue();
+    }
+    rtm_ctx::GraphEntry e;
+    memcpy(e.key, key, sizeof(key));
+    e.gen = c->gen;
+    e.g = g;
+    e.x = x;
+    size_t n = 0;
+    CK(cudaGraphGetNodes(g, nullptr, &n));
+    std::vector<cudaGraphNode_t> nodes(n);
+    CK(cudaGraphGetNodes(g, nodes.data(), &n));
+    for (cudaGraphNode_t nd : nodes) {
+      cudaGraphNodeType t;
+      CK(cudaGraphNodeGetType(nd, &t));
+      if (t != cudaGraphNodeTypeKernel) continue;
+      cudaKernelNodeParams kp;
+      CK(cudaGraphKernelNodeGetParams(nd, &kp));
+      kp.kernelParams = nullptr;
+      kp.extra = nullptr;
+      e.kn.push_back(nd);
+      e.kp.push_back(kp);
+    }
+    if (c->graphs.size() >= kGraphCacheSize) {  // evict the least recently used shape
+      size_t lru = 0;
+      for (size_t i = 1; i < c->graphs.size(); ++i)
+        if (c->graphs[i].used < c->graphs[lru].used) lru = i;
+      graph_free(c->graphs[lru]);
+      c->graphs.erase(c->graphs.begin() + (long)lru);
+    }
+    c->graphs.push_back(std::move(e));
+    hit = &c->graphs.back();  // captured with this call's arguments: launch as is
+    ++c->graph_captures;
+  } else {
+    void *a1[] = {&p};
+    ClearList cc = cl;
+    long long *Bs = (long long *)c->Bs.p, *Be = (long long *)c->Be.p;
+    void *a4[] = {&p, &cc, &Bs, &Be};
+    const void *prep = prep_kernel_fn();
+    for (size_t i = 0; i < hit->kn.size(); ++i) {
+      cudaKernelNodeParams kp = hit->kp[i];
+      kp.kernelParams = kp.func == prep ? a4 : a1;
+      CK(cudaGraphExecKernelNodeSetParams(hit->x, hit->kn[i], &kp));
+    }
+    count_launches((unsigned)hit->kn.size());
+    ++c->graph_replays;
+  }
+  hit->used = ++c->graph_tick;
+  CK(cudaGraphLaunch(hit->x, c->st));
+  return RTM_OK;
+}
+
 rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p) {
   if (c->sticky) return (rtm_status)c->sticky;
   if (c->merge_pending) return RTM_E_STATE;  // the previous local reduce awaits rtm_merge
@@ -361,7 +492,6 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   long long *hT = (long long *)c->h_small.p;
   hT[0] = c->t_prev;
   for (uint32_t w = 0; w < W; ++w) hT[w + 1] = t_end[w];
-  CK(cudaMemcpyAsync(c->T.p, hT, (size_t)(W + 1) * 8, cudaMemcpyHostToDevice, c->st));
 
   memset(&p, 0, sizeof(p));
   p.nb = c->nb; p.nc = c->nc; p.nk = c->nk; p.nbins = c->nbins; p.ncw = c->ncw; p.k = c->k;
@@ -483,15 +613,21 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   cudaMemsetAsync(dbg, 0, 64, c->st);
   p.dbg = dbg;
 #endif
-  // clear the call's accumulators, region boundaries, tile tables: one cooperative launch
-  LAUNCH(KT_SPLIT, 0,
-         launch_prep(p, prep_cl, (long long *)c->Bs.p, (long long *)c->Be.p, c->n_sms, c->st));
-  CK(cudaGetLastError());
   // Task events are independent of the sample path.  Lane-major partition path: the persistent
   // partition kernel runs the event tiles after its sample tiles (claimed dynamically), so no
   // concurrent kernel competes with the issue-bound fold.  Otherwise: a side stream, overlapped
   // with the partition and the fold, joined before the kernels that read the event outputs.
   p.fuse_events = partition_fuses_events(p.nbins, nts, two_pass) ? 1 : 0;
+  p.persist_inline = c->world == 1 && p.persist;  // the top-k kernels count their winners (world 1)
+  // The launch sequence (every kernel takes this call's Params by value; k_prep also the clear
+  // list and the split buffers).  Direct launches, or captured once per launch shape into a CUDA
+  // graph and replayed (rtm_use_graphs).
+  auto enqueue = [&]() -> rtm_status {
+  CK(cudaMemcpyAsync(c->T.p, hT, (size_t)(W + 1) * 8, cudaMemcpyHostToDevice, c->st));
+  // clear the call's accumulators, region boundaries, tile tables: one cooperative launch
+  LAUNCH(KT_SPLIT, 0,
+         launch_prep(p, prep_cl, (long long *)c->Bs.p, (long long *)c->Be.p, c->n_sms, c->st));
+  CK(cudaGetLastError());
   if (!p.fuse_events) {
     CK(cudaEventRecord(c->ev_fork, c->st));
     CK(cudaStreamWaitEvent(c->st2, c->ev_fork, 0));
@@ -536,13 +672,17 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     if (c->prof) prof_end_on(c, c->st2);
     CK(cudaEventRecord(c->ev_join, c->st2));
   }
-  p.persist_inline = c->world == 1 && p.persist;  // world > 1: counted from the merged lists
-  LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));
-  p.persist_inline = 0;
+  LAUNCH(KT_TOPK, 0, launch_topk(p, c->st));  // world > 1: persistence counted from the merged lists
   if (side_hang) CK(cudaStreamWaitEvent(c->st, c->ev_join, 0));
   else LAUNCH(KT_HANG, 0, launch_hang(p, c->st));
   if (!side) LAUNCH(KT_PROGRESS, 0, launch_progress(p, c->st));
   CK(cudaGetLastError());
+  return RTM_OK;
+  };
+  if (graph_use(c, W)) s = graph_launch(c, p, prep_cl, enqueue);
+  else s = enqueue();
+  p.persist_inline = 0;
+  if (s) return s;
 #ifdef RTM_PHASE_TIMING
   {
     unsigned long long h[8];
@@ -794,6 +934,8 @@ void rtm_destroy(rtm_ctx *c) {
                     &c->unit_ctr, &c->bstat, &c->comps, &c->pack,
                     &c->gathered, &c->tkscr, &c->mkey, &c->rcp64, &c->tkey, &c->persist, &c->klive,
                     &c->gcum, &c->tpack, &c->tgathered};
+  graphs_clear(c);
+  if (c->cap_st) cudaStreamDestroy(c->cap_st);
   for (DevBuf *b : bufs) free_buf(*b);
   if (c->h_small.p) cudaFreeHost(c->h_small.p);
   if (c->h_res.p) cudaFreeHost(c->h_res.p);
@@ -1259,6 +1401,20 @@ rtm_status rtm_buffer_stats(rtm_ctx *c, uint32_t first, uint32_t count, rtm_buff
                      cudaMemcpyDeviceToHost, c->st));
   CK(cudaStreamSynchronize(c->st));
   for (uint32_t i = 0; i < count; ++i) out[i].reserved = 0;
+  return RTM_OK;
+}
+
+rtm_status rtm_use_graphs(rtm_ctx *c, int32_t mode) {
+  if (!c || mode < RTM_GRAPHS_OFF || mode > RTM_GRAPHS_ALWAYS) return RTM_E_INVALID;
+  c->graph_mode = mode;
+  if (mode == RTM_GRAPHS_OFF) graphs_clear(c);
+  return RTM_OK;
+}
+
+rtm_status rtm_graph_stats(rtm_ctx *c, uint64_t *captured, uint64_t *replayed) {
+  if (!c || !captured || !replayed) return RTM_E_INVALID;
+  *captured = c->graph_captures;
+  *replayed = c->graph_replays;
   return RTM_OK;
 }
 

@@ -184,6 +184,9 @@ void launch_merge_tables(const Params &p, const void *gathered, uint32_t world, 
 bool merge_fits(uint32_t world, uint32_t k);  // world * k candidates fit the merge's shared memory
 void launch_scatter_bstat(const Params &p, cudaStream_t st);  // gid set, world == 1
 unsigned long long kernel_launches();  // kernels launched by this library in this process
+void count_launches(unsigned n);       // kernels launched by a CUDA graph replay
+void launch_shape(const Params &p, uint64_t key[3]);  // launch-sequence shape (graph cache key)
+const void *prep_kernel_fn();          // k_prep (the one kernel with arguments besides Params)
 
 // Device ranges zeroed by ONE kernel launch (replaces per-buffer cudaMemsetAsync calls).
 struct ClearList {

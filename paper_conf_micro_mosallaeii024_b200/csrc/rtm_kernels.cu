@@ -3102,6 +3102,22 @@ void launch_topk(const Params &p, cudaStream_t st) {
   else { k_topk<false><<<p.W, kTopkThreads, topk_smem_bytes(p.n_elig), st>>>(p); count_launch(); }
 }
 
+// Every host-side decision of rtm_window_reduce's launch sequence that is not a kernel argument
+// (kernel variants, grid sizes, which kernels run): two calls with equal shapes on the same
+// workspaces launch the same kernels with the same configurations, so a CUDA graph captured for
+// one replays the other with only the Params argument replaced (rtm_api.cpp, rtm_use_graphs).
+void launch_shape(const Params &p, uint64_t key[3]) {
+  key[0] = (uint64_t)p.W | (uint64_t)p.n_tiles_s << 32;
+  key[1] = (uint64_t)p.n_tiles_e | (uint64_t)p.tk_slices << 32;
+  key[2] = (uint64_t)(p.narrow != 0) | (uint64_t)(p.fuse_events != 0) << 1 | (uint64_t)(p.nsb != 0) << 2 |
+           (uint64_t)fold_sequential(p) << 3 | (uint64_t)(p.ns < 2ull * p.nb * p.W) << 4 |
+           (uint64_t)(p.mkey != nullptr) << 5 | (uint64_t)(p.n_elig == p.nb) << 6 |
+           (uint64_t)hang_prefix_path(p.W, p.H) << 7 | (uint64_t)(p.n_tiles_s != 0) << 8 |
+           (uint64_t)(p.n_tiles_e != 0) << 9;
+}
+const void *prep_kernel_fn() { return (const void *)k_prep; }
+void count_launches(unsigned n) { g_kernel_launches.fetch_add(n, std::memory_order_relaxed); }
+
 void launch_persist(const Params &p, cudaStream_t st) {
   const size_t n = (size_t)p.W * p.k;
   if (!n || !p.persist) return;

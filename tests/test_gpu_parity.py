@@ -521,6 +521,51 @@ def test_many_bins_partition_paths(n_buffers):
     assert_same(got, ref, mon)
 
 
+@pytest.mark.parametrize("n_buffers", [1000, 327680])
+def test_graph_replay_equals_direct_launches(n_buffers):
+    """rtm_use_graphs: a context replaying captured CUDA graphs (RTM_GRAPHS_ALWAYS) and one
+    launching directly (RTM_GRAPHS_OFF) stream the same trace in calls of 1, 1, 3, 1, 2, 1, 1
+    windows (shapes repeat, so most calls are replays with new arguments) with watched buffers;
+    both equal the oracle call by call, including the value-monitor rings.  327680 buffers take the
+    two-pass partition; 1000 the lane-major one."""
+    wl = gen.C1.scaled("C1-graph", n_samples=300_000, n_events=30_000, n_buffers=n_buffers, n_windows=10)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
+    orc = oracle.Oracle(owner, cap, tot, n_components=wl.n_components, **kw)
+    mons = [Monitor(owner, cap, tot, n_components=wl.n_components, **kw) for _ in range(2)]
+    mons[0].use_graphs(N.RTM_GRAPHS_OFF)
+    mons[1].use_graphs(N.RTM_GRAPHS_ALWAYS)
+    watched = [0, 7, n_buffers - 1]
+    for m in mons:
+        m.watch(watched)
+    s, e = gen.samples(wl), gen.events(wl)
+    t_end = wl.t_end()
+    w0 = 0
+    launches = []
+    for m_w in (1, 1, 3, 1, 2, 1, 1):
+        w1 = w0 + m_w
+        sl = slice(wl.index_at("samples", wl.t_begin(w0)), wl.index_at("samples", wl.t_begin(w1)))
+        el = slice(wl.index_at("events", wl.t_begin(w0)), wl.index_at("events", wl.t_begin(w1)))
+        ref = orc.reduce(s[sl], e[el], t_end[w0:w1], want_all_stats=True)
+        for i, m in enumerate(mons):
+            k0 = N.lib().rtm_kernel_launches()
+            m.ingest(_dev(s[sl]), _dev(e[el]))
+            got = m.window_reduce(t_end[w0:w1])
+            launches.append((i, int(N.lib().rtm_kernel_launches() - k0)))
+            assert_same(got, ref, m)
+        w0 = w1
+    for q in range(len(watched)):
+        a, b = mons[0].watch_series(q), mons[1].watch_series(q)
+        assert np.array_equal(a.view(np.uint8), b.view(np.uint8))
+    captured, replayed = mons[1].graph_stats()
+    assert captured >= 1 and replayed >= 1 and captured + replayed == 7, (captured, replayed)
+    assert mons[0].graph_stats() == (0, 0)
+    # a replay launches (and counts) the same kernels as a direct call of the same shape
+    direct = [n for i, n in launches if i == 0]
+    graph = [n for i, n in launches if i == 1]
+    assert direct == graph
+
+
 @pytest.mark.parametrize("case", ["ragged_invalid", "mean_1m", "very_sparse_bl7", "wide_windows"])
 def test_two_pass_partition_paths(case):
     """Registries of >= 1024 bins take the two-pass partition (lane-major by 16384-buffer superbin,

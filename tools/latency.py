@@ -24,6 +24,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C5-long")
 ap.add_argument("--windows", type=int, default=2000)
 ap.add_argument("--warmup", type=int, default=50)
+ap.add_argument("--graphs", type=int, default=1, help="rtm_use_graphs mode: 0 off, 1 auto (default), 2 always")
 args = ap.parse_args()
 wl = gen.CONFIGS[args.config]
 W = args.windows + args.warmup
@@ -36,6 +37,7 @@ gen.fill_device("events", wl, de.data_ptr(), 0, ne)
 torch.cuda.synchronize()
 owner, cap, tot = gen.registry(wl)
 mon = Monitor(owner, cap, tot, n_components=wl.n_components, t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k)
+mon.use_graphs(args.graphs)
 t_end = wl.t_end(0, W)
 lat = []
 recs = 0
@@ -63,7 +65,7 @@ for w in range(n_prof):
 prof = {k: round(v["total_ms"] * 1e3 / n_prof, 2) for k, v in mon.profile_read().items() if v["launches"]}
 mon.profile(False)
 print(json.dumps({"what": "per-window snapshot latency, one window per call (streaming)", "config": wl.name,
-                  "n_buffers": wl.n_buffers, "windows": args.windows, "records_per_window": recs / args.windows,
+                  "n_buffers": wl.n_buffers, "windows": args.windows, "graphs": args.graphs, "records_per_window": recs / args.windows,
                   "p50_us": float(np.percentile(lat, 50)), "p99_us": float(np.percentile(lat, 99)),
                   "mean_us": float(lat.mean()), "records_per_s": recs / (lat.sum() / 1e6),
                   "kernel_us_per_call": prof}))
