@@ -655,9 +655,10 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
 // and only then prefetch their next raw records (named barrier among themselves); warps 4-7
 // prefetch before the first barrier (measured 813 -> 692 us on C2 against direct 8-byte scatter
 // stores from every lane, which touched 32 sectors per store instruction).
-template <int BL, bool CAPS, int KS>
+template <int BL, bool CAPS, int KS, bool MP>
 __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   static_assert(BL == 8, "lane-major entries pack the buffer id in one byte");
+  static_assert(!MP || KS == 8, "multi-pass ranking: bins");
   static_assert(KS == 8 || KS == kSupLog, "bins or superbins");
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ K1WarpSum wsum[2][kK1Warps];
@@ -750,47 +751,97 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
     PTM(2);
     __syncwarp();  // every lane has consumed its raw records
     if (is_win) {  // rank = (lane, bin) counter; position = rank + earlier lanes' counts of the bin
-      uint4 *r4 = reinterpret_cast<uint4 *>(rows);
-      for (unsigned q = lane; q < nbins * 3; q += 32) r4[q] = make_uint4(0, 0, 0, 0);
-      __syncwarp();
+      // bins [kb, kb + nk): their count rows (48 B per bin) overlay the consumed raw slot.  MP
+      // (171 .. 1023 bins): the slot holds the rows of at most kLmMaxBins bins, so the keys are
+      // ranked in passes over bin ranges (each record in the pass of its bin).
+      if constexpr (MP) {
+        auto rank_pass = [&](unsigned kb, unsigned nk) {
+          uint4 *r4 = reinterpret_cast<uint4 *>(rows);
+          for (unsigned q = lane; q < nk * 3; q += 32) r4[q] = make_uint4(0, 0, 0, 0);
+          __syncwarp();
+  #pragma unroll
+          for (int k = 0; k < kPerLane; ++k) {
+            const unsigned key = kp[k] >> 16, rk = key - kb;
+            if (key != kNoKey && (!MP || rk < nk)) {
+              unsigned char *ctr = rows + rk * 48 + lane;
+              const unsigned r = *ctr;
+              *ctr = (unsigned char)(r + 1);
+              kp[k] |= r;
+            }
+          }
+          __syncwarp();
+          for (unsigned b = lane; b < nk; b += 32) {  // one bin row per lane: byte-SIMD prefix
+            uint4 *row = reinterpret_cast<uint4 *>(rows + b * 48);
+            const uint4 q0 = row[0], q1 = row[1];
+            unsigned w[8] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w};
+            unsigned base[8];
+            unsigned run = 0;
+  #pragma unroll
+            for (int x = 0; x < 8; ++x) {
+              const unsigned incl = w[x] * 0x01010101u;  // byte j = counts of lanes 4x .. 4x+j (<= 64)
+              base[x] = run;
+              run += incl >> 24;
+              w[x] = incl - w[x];
+            }
+            row[0] = make_uint4(w[0], w[1], w[2], w[3]);
+            row[1] = make_uint4(w[4], w[5], w[6], w[7]);
+            row[2] = make_uint4(base[0] | (base[1] << 16), base[2] | (base[3] << 16), base[4] | (base[5] << 16),
+                                base[6] | (base[7] << 16));
+            myt[kb + b] = (unsigned short)run;
+          }
+          __syncwarp();
+          const unsigned short *rows16 = reinterpret_cast<const unsigned short *>(rows);
+  #pragma unroll
+          for (int k = 0; k < kPerLane; ++k) {
+            const unsigned key = kp[k] >> 16, rk = key - kb;
+            if (key != kNoKey && (!MP || rk < nk)) kp[k] += rows[rk * 48 + lane] + rows16[rk * 24 + 16 + (lane >> 2)];
+          }
+          __syncwarp();  // the slot is free again
+        };
+        for (unsigned kb = 0; kb < nbins; kb += kLmMaxBins) rank_pass(kb, min(nbins - kb, kLmMaxBins));
+      } else {  // one pass (the C2 path: kept as its own code, the lambda form spills 8 B here)
+        uint4 *r4 = reinterpret_cast<uint4 *>(rows);
+        for (unsigned q = lane; q < nbins * 3; q += 32) r4[q] = make_uint4(0, 0, 0, 0);
+        __syncwarp();
 #pragma unroll
-      for (int k = 0; k < kPerLane; ++k) {
-        const unsigned key = kp[k] >> 16;
-        if (key != kNoKey) {
-          unsigned char *ctr = rows + key * 48 + lane;
-          const unsigned r = *ctr;
-          *ctr = (unsigned char)(r + 1);
-          kp[k] |= r;
+        for (int k = 0; k < kPerLane; ++k) {
+          const unsigned key = kp[k] >> 16;
+          if (key != kNoKey) {
+            unsigned char *ctr = rows + key * 48 + lane;
+            const unsigned r = *ctr;
+            *ctr = (unsigned char)(r + 1);
+            kp[k] |= r;
+          }
         }
-      }
-      __syncwarp();
-      for (unsigned b = lane; b < nbins; b += 32) {  // one bin row per lane: byte-SIMD prefix
-        uint4 *row = reinterpret_cast<uint4 *>(rows + b * 48);
-        const uint4 q0 = row[0], q1 = row[1];
-        unsigned w[8] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w};
-        unsigned base[8];
-        unsigned run = 0;
+        __syncwarp();
+        for (unsigned b = lane; b < nbins; b += 32) {  // one bin row per lane: byte-SIMD prefix
+          uint4 *row = reinterpret_cast<uint4 *>(rows + b * 48);
+          const uint4 q0 = row[0], q1 = row[1];
+          unsigned w[8] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w};
+          unsigned base[8];
+          unsigned run = 0;
 #pragma unroll
-        for (int x = 0; x < 8; ++x) {
-          const unsigned incl = w[x] * 0x01010101u;  // byte j = counts of lanes 4x .. 4x+j (<= 64)
-          base[x] = run;
-          run += incl >> 24;
-          w[x] = incl - w[x];
+          for (int x = 0; x < 8; ++x) {
+            const unsigned incl = w[x] * 0x01010101u;  // byte j = counts of lanes 4x .. 4x+j (<= 64)
+            base[x] = run;
+            run += incl >> 24;
+            w[x] = incl - w[x];
+          }
+          row[0] = make_uint4(w[0], w[1], w[2], w[3]);
+          row[1] = make_uint4(w[4], w[5], w[6], w[7]);
+          row[2] = make_uint4(base[0] | (base[1] << 16), base[2] | (base[3] << 16), base[4] | (base[5] << 16),
+                              base[6] | (base[7] << 16));
+          myt[b] = (unsigned short)run;
         }
-        row[0] = make_uint4(w[0], w[1], w[2], w[3]);
-        row[1] = make_uint4(w[4], w[5], w[6], w[7]);
-        row[2] = make_uint4(base[0] | (base[1] << 16), base[2] | (base[3] << 16), base[4] | (base[5] << 16),
-                            base[6] | (base[7] << 16));
-        myt[b] = (unsigned short)run;
-      }
-      __syncwarp();
-      const unsigned short *rows16 = reinterpret_cast<const unsigned short *>(rows);
+        __syncwarp();
+        const unsigned short *rows16 = reinterpret_cast<const unsigned short *>(rows);
 #pragma unroll
-      for (int k = 0; k < kPerLane; ++k) {
-        const unsigned key = kp[k] >> 16;
-        if (key != kNoKey) kp[k] += rows[key * 48 + lane] + rows16[key * 24 + 16 + (lane >> 2)];
+        for (int k = 0; k < kPerLane; ++k) {
+          const unsigned key = kp[k] >> 16;
+          if (key != kNoKey) kp[k] += rows[key * 48 + lane] + rows16[key * 24 + 16 + (lane >> 2)];
+        }
+        __syncwarp();  // the slot is free again
       }
-      __syncwarp();  // the slot is free again
     }
     PTM(3);
     // the next tile's records stream into the slot while this tile is published and written out
@@ -2920,13 +2971,19 @@ void launch_clear(const ClearList &cl, cudaStream_t st) {
 size_t fold_smem_bytes(int bin_log) {
   return (bin_log == 7 ? sizeof(FoldSmem<7>) : sizeof(FoldSmem<8>)) * kFoldWarps;
 }
+// measured (1 x B200, full-size configs): 320 bins (C3) the match-based partition and the two-pass
+// path tie (28.5 vs 29.4 ms per step: k_subpart reads the entries twice at ~4 warp instructions
+// each); 2560 bins (C5) fold 22.4 -> 17.9 ms per 10k windows; 4096 bins (C4) 132.5 -> 77.5 ms.
+// Below it, 171 .. 1023 bins take the lane-major partition with multi-pass ranking (MP).
+constexpr uint32_t kTwoPassMinBins = 1024;
 // lane-major partition: the capacity table in shared memory when two CTAs still fit per SM
 bool partition_caps_smem(uint32_t nbins, uint32_t nb) { return k1_smem_lm(nbins, nb, true) + 1024 <= 113 * 1024; }
 size_t partition_smem_bytes(uint32_t nbins, uint32_t nb) {
-  return nbins <= kLmMaxBins ? k1_smem_lm(nbins, nb, partition_caps_smem(nbins, nb)) : k1_smem_mx(nbins);
+  return nbins < kTwoPassMinBins ? k1_smem_lm(nbins, nb, partition_caps_smem(nbins, nb)) : k1_smem_mx(nbins);
 }
 static_assert(2 * (k1_smem_lm(80, 20480) + 1024 + 512) <= 228 * 1024, "C2-sized partition CTAs must fit 2 per SM");
-static_assert(k1_smem_lm(kLmMaxBins, 0, false) <= 113 * 1024 && k1_smem_mx(kMaxBins) <= 227 * 1024,
+static_assert(k1_smem_lm(kLmMaxBins, 0, false) <= 113 * 1024 && k1_smem_lm(kTwoPassMinBins - 1, 0, false) <= 227 * 1024 &&
+                  k1_smem_mx(kMaxBins) <= 227 * 1024,
               "partition shared memory exceeds the opt-in limit");
 size_t topk_smem_bytes(uint32_t nb) {
   return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8 + kTopkCand * 4;
@@ -2953,13 +3010,9 @@ void launch_prep(const Params &p, const ClearList &cl, long long *Bs, long long 
   count_launch();
 }
 
-// measured (1 x B200, full-size configs): 320 bins (C3) the match-based partition and the two-pass
-// path tie (28.5 vs 29.4 ms per step: k_subpart reads the entries twice at ~4 warp instructions
-// each); 2560 bins (C5) fold 22.4 -> 17.9 ms per 10k windows; 4096 bins (C4) 132.5 -> 77.5 ms
-constexpr uint32_t kTwoPassMinBins = 1024;
 bool partition_two_pass(uint32_t nbins, bool narrow) { return nbins >= kTwoPassMinBins && narrow; }
 bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s, bool two_pass) {
-  return n_tiles_s && (nbins <= kLmMaxBins || two_pass);
+  return n_tiles_s && (nbins < kTwoPassMinBins || two_pass);
 }
 
 template <int BL>
@@ -2981,15 +3034,15 @@ void launch_subpart(const Params &p, int n_sms, cudaStream_t st) {
   else launch_subpart_bl<8>(p, n_sms, st);
 }
 
-template <int BL, bool CAPS, int KS>
+template <int BL, bool CAPS, int KS, bool MP = false>
 void launch_partition_lm(const Params &p, int n_sms, size_t sm, cudaStream_t st) {
   int per_sm = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm<BL, CAPS, KS>, kK1Threads, sm);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm<BL, CAPS, KS, MP>, kK1Threads, sm);
   if (per_sm < 1) per_sm = 1;
   unsigned grid = (unsigned)(n_sms * per_sm);
   const unsigned work = p.n_tiles_s + (p.fuse_events ? p.n_tiles_e : 0u);
   if (grid > work) grid = work;
-  { k_partition_lm<BL, CAPS, KS><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
+  { k_partition_lm<BL, CAPS, KS, MP><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
 }
 
 void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
@@ -3003,9 +3056,12 @@ void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
   }
   const size_t sm = partition_smem_bytes(p.nbins, p.nb);
   if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM
-    // bin_log 8 here: bin_log 7 is only chosen for > 131072 buffers (> 170 bins)
+    // bin_log 8 here: bin_log 7 is only chosen for > 131072 buffers (> 1024 bins)
     if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 8>(p, n_sms, sm, st);
     else launch_partition_lm<8, false, 8>(p, n_sms, sm, st);
+  } else if (p.nbins < kTwoPassMinBins) {  // 171 .. 1023 bins: ranks in passes of <= 170 bins
+    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 8, true>(p, n_sms, sm, st);
+    else launch_partition_lm<8, false, 8, true>(p, n_sms, sm, st);
   } else {
     if (p.bin_log == 7) { k_partition_mx<7><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
     else { k_partition_mx<8><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
@@ -3153,10 +3209,13 @@ void configure_kernels_once() {
   done[dev] = true;
   const int lm_caps = (int)k1_smem_lm(kLmMaxBins, 113 * 512, true);  // <= 113 KB by partition_caps_smem
   const int lm_glob = (int)k1_smem_lm(kLmMaxBins, 0, false);
-  cudaFuncSetAttribute(k_partition_lm<8, true, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
-  cudaFuncSetAttribute(k_partition_lm<8, false, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
-  cudaFuncSetAttribute(k_partition_lm<8, true, kSupLog>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
-  cudaFuncSetAttribute(k_partition_lm<8, false, kSupLog>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  const int lm_mp = (int)k1_smem_lm(kTwoPassMinBins - 1, 0, false);
+  cudaFuncSetAttribute(k_partition_lm<8, true, 8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false, 8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  cudaFuncSetAttribute(k_partition_lm<8, true, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_mp);
+  cudaFuncSetAttribute(k_partition_lm<8, true, kSupLog, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false, kSupLog, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
   cudaFuncSetAttribute(k_subpart<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(SubSmem<7>) * kSubWarps));
   cudaFuncSetAttribute(k_subpart<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(SubSmem<8>) * kSubWarps));
   cudaFuncSetAttribute(k_partition_mx<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));

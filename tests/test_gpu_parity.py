@@ -506,10 +506,11 @@ def test_rank_local_numbering_rejects_unsorted_ids():
                 n_global_buffers=10)
 
 
-@pytest.mark.parametrize("n_buffers", [32768, 33000, 81920, 262144])
+@pytest.mark.parametrize("n_buffers", [32768, 33000, 43521, 81920, 261888, 262144])
 def test_many_bins_partition_paths(n_buffers):
-    """n_bins <= 128 takes the lane-major partition, more bins the match-based fallback
-    (k_partition_mx): both must agree with the oracle (C3-like buffer counts, short trace)."""
+    """Every partition path against the oracle (short trace): <= 170 bins the lane-major partition
+    in one ranking pass (128, 129 bins), 171 .. 1023 bins in passes of <= 170 bins (171: a
+    one-bin second pass; 320 as C3; 1023: one CTA per SM), 1024 bins the two-pass path."""
     wl = gen.C1.scaled("C1-bins", n_samples=400_000, n_events=40_000, n_buffers=n_buffers, n_windows=5)
     owner, cap, tot = gen.registry(wl)
     kw = dict(t0=wl.t0, hang_windows=2, k=wl.k)
