@@ -496,6 +496,13 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   memset(&p, 0, sizeof(p));
   p.nb = c->nb; p.nc = c->nc; p.nk = c->nk; p.nbins = c->nbins; p.ncw = c->ncw; p.k = c->k;
   p.bin_log = c->bin_log;
+  // Few-unit calls (fewer (window, bin) units than SMs: one-window streaming calls on a C2-sized
+  // registry) fold 128-buffer bins: twice the units, half the chain per unit.
+  if (p.bin_log == 8 && (uint64_t)W * p.nbins < (uint64_t)c->n_sms && ((c->nb + 127) >> 7) <= kLmMaxBins) {
+    p.bin_log = 7;
+    p.nbins = (c->nb + 127) >> 7;
+  }
+  const uint32_t nbins = p.nbins;
   p.rank_mode = c->rank_mode; p.H = c->H; p.hang_mode = c->hang_mode;
   p.cap = (const uint16_t *)c->cap.p; p.owner = (const uint32_t *)c->owner.p;
   p.elig = (const uint8_t *)c->elig.p; p.ktotal = (const int64_t *)c->ktotal.p;
@@ -526,19 +533,19 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   if ((s = ensure(c, c->treg_s, (size_t)nts * 4))) return s;
   if ((s = ensure(c, c->treg_e, (size_t)nte * 4))) return s;
   if ((s = ensure(c, c->tdesc, (size_t)nts * sizeof(TileDesc)))) return s;
-  if ((s = ensure(c, c->soff, (size_t)nts * (c->nbins + 1) * 2))) return s;
+  if ((s = ensure(c, c->soff, (size_t)nts * (nbins + 1) * 2))) return s;
   if ((s = ensure(c, c->stage, (size_t)nts * kTileS * 8))) return s;
   // more than 170 bins: two-pass partition (superbins, then bins per (window, superbin))
-  const bool two_pass = partition_two_pass(c->nbins, p.narrow != 0);
+  const bool two_pass = partition_two_pass(nbins, p.narrow != 0);
   if (two_pass) {
     if ((s = ensure(c, c->stage2, (size_t)nts * kTileS * 8))) return s;
-    if ((s = ensure(c, c->woff, (size_t)W * (c->nbins + 1) * 4))) return s;
+    if ((s = ensure(c, c->woff, (size_t)W * (nbins + 1) * 4))) return s;
   }
   if ((s = ensure(c, c->smeta, (size_t)nts * sizeof(TileMeta)))) return s;
   if ((s = ensure(c, c->emeta, (size_t)nte * sizeof(TileMeta)))) return s;
   if ((s = ensure(c, c->lastlvl, Wn * c->nb * 2))) return s;
-  if (c->flags.cap < Wn * c->nbins * 4) {
-    if ((s = ensure(c, c->flags, Wn * c->nbins * 4, true))) return s;
+  if (c->flags.cap < Wn * nbins * 4) {
+    if ((s = ensure(c, c->flags, Wn * nbins * 4, true))) return s;
   }
   if ((s = ensure(c, c->res, res_layout(c, W).bytes))) return s;
   if ((s = ensure(c, c->kdelta, Wn * c->nk * 2 * 4))) return s;
@@ -688,8 +695,8 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     unsigned long long h[8];
     cudaMemcpyAsync(h, p.dbg, 64, cudaMemcpyDeviceToHost, c->st);
     cudaStreamSynchronize(c->st);
-    fprintf(stderr, "[lookback] units=%llu steps=%llu (%.2f / unit) spins=%llu\n", (unsigned long long)W * c->nbins,
-            h[0], (double)h[0] / ((double)W * c->nbins), h[6]);
+    fprintf(stderr, "[lookback] units=%llu steps=%llu (%.2f / unit) spins=%llu\n", (unsigned long long)W * p.nbins,
+            h[0], (double)h[0] / ((double)W * p.nbins), h[6]);
     if (h[7])
       fprintf(stderr, "[phase] tiles=%llu  -=%.0f wait_raw=%.0f scan=%.0f rank=%.0f B1=%.0f bases+scatter=%.0f -=%.0f (cycles/tile, thread 0)\n",
               h[7], (double)h[0] / h[7], (double)h[1] / h[7], (double)h[2] / h[7], (double)h[3] / h[7],

@@ -40,6 +40,7 @@ constexpr int kFoldWarps = RTM_FOLD_WARPS;  // warps per fold CTA (compile-time 
 constexpr uint16_t kSent = 0xFFFFu;         // "no kept sample in this window" marker
 constexpr uint32_t kMaxBins = 4096;         // n_buffers <= 2^20 (fallback partition smem 160 KB)
 constexpr uint32_t kTopkSmemKeys = 40960;
+constexpr uint32_t kLmMaxBins = 170;        // lane-major partition: count rows (bins x 48 B) fit a warp's 8 KB slot
 constexpr int kSupLog = 14;                 // two-pass partition: superbins of 2^14 buffers (<= 64 of them)   // keys held in shared memory by the top-k kernel
 // ts offset field of a staging entry: 48 - bin_log bits (entry = off << (16 + bin_log) | level << bin_log | lid)
 inline int64_t max_window_len(int bin_log) { return (int64_t)1 << (bin_log >= 8 ? 40 : 48 - bin_log > 40 ? 40 : 48 - bin_log); }

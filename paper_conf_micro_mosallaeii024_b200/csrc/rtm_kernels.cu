@@ -442,7 +442,6 @@ constexpr int kSub = kTileS / (kK1Threads / 32);  // 512 samples per warp
 constexpr int kPerLane = kSub / 32;               // 16
 constexpr int kK1Warps = kK1Threads / 32;         // 8
 constexpr unsigned kNoKey = 0xFFFFu;
-constexpr uint32_t kLmMaxBins = 170;              // count rows (nbins x 48 B) fit the 8 KB raw slot
 static_assert(kPerLane == 16, "lane-major swizzle assumes 16 records per lane");
 static_assert((size_t)kLmMaxBins * 48 <= (size_t)kSub * 16, "count rows must fit the raw slot");
 
@@ -526,7 +525,7 @@ template <int KS>
 __device__ __forceinline__ unsigned k1_bin_bases(const Params &p, unsigned tile, const unsigned short *wt,
                                                  unsigned short *myb) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const unsigned nbins = KS == 8 ? p.nbins : p.nsb;
+  const unsigned nbins = KS == kSupLog ? p.nsb : p.nbins;
   uint16_t *offs = p.soff + (size_t)tile * (nbins + 1);
   unsigned carry = 0;
   for (unsigned b0 = 0; b0 < nbins; b0 += 32) {
@@ -578,8 +577,10 @@ __device__ __forceinline__ void k1_publish(K1WarpSum *wsum, unsigned long long f
 // One lane's 16 consecutive records: field check, running min / max of the field-valid offsets
 // (an inversion inside the lane shows up as an offset below the running max), entries, keys.
 // NAR: windows shorter than 2^32 ticks, so offsets are compared and packed in 32 bits.
-// KS: key = buffer_id >> KS.  KS == 8: the bin (entries as above).  KS == kSupLog: the superbin
-// of the two-pass path (narrow windows only): entry = o << 32 | level << 16 | (buffer_id & 0x3FFF).
+// KS: key = buffer_id >> KS.  KS == 8: the 256-buffer bin (entries as above); KS == 7: the
+// 128-buffer bin (entries off << 23 | level << 7 | buffer_id & 127: few-unit calls, see rtm_api.cpp);
+// KS == kSupLog: the superbin of the two-pass path (narrow windows only): entry =
+// o << 32 | level << 16 | (buffer_id & 0x3FFF).
 template <bool NAR, int BL, bool CAPS, int KS>
 __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool is_win, const int4 *raw,
                                         const unsigned short *capS, int sub0, unsigned long long (&e)[kPerLane],
@@ -606,6 +607,8 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
       hiacc |= valid ? (unsigned)(off >> 32) : 0u;
       if constexpr (KS == kSupLog) {
         e[k] = ((unsigned long long)o << 32) | (lvl << 16) | (b & ((1u << kSupLog) - 1u));
+      } else if constexpr (KS != 8) {
+        e[k] = ((unsigned long long)o << (16 + KS)) | (lvl << KS) | (b & ((1u << KS) - 1u));
       } else {
         // (o << 24) | (level << 8) | (buffer_id & 255), o < 2^32
         const unsigned lo = __byte_perm(__byte_perm((unsigned)v.z, (unsigned)v.w, 0x0540), o, 0x4210);
@@ -615,7 +618,8 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
       bad |= valid & (off < mx64);
       mx64 = max(mx64, valid ? off : 0ull);
       mn64 = min(mn64, valid ? off : ~0ull);
-      e[k] = (off << (16 + BL)) | ((unsigned long long)lvl << BL) | (b & ((1u << BL) - 1u));
+      constexpr int EB = KS == kSupLog ? BL : KS;  // bin bits of a fold entry
+      e[k] = (off << (16 + EB)) | ((unsigned long long)lvl << EB) | (b & ((1u << EB) - 1u));
     }
     const bool keep = valid & is_win;
     kept += keep;
@@ -658,13 +662,13 @@ __device__ __forceinline__ void lm_scan(const Params &p, const K1Tile &t, bool i
 template <int BL, bool CAPS, int KS, bool MP>
 __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   static_assert(BL == 8, "lane-major entries pack the buffer id in one byte");
-  static_assert(!MP || KS == 8, "multi-pass ranking: bins");
-  static_assert(KS == 8 || KS == kSupLog, "bins or superbins");
+  static_assert(!MP || KS != kSupLog, "multi-pass ranking: bins");
+  static_assert(KS == 8 || KS == 7 || KS == kSupLog, "bins or superbins");
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ K1WarpSum wsum[2][kK1Warps];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
-  const unsigned nbins = KS == 8 ? p.nbins : p.nsb;  // keys of this pass
+  const unsigned nbins = KS == kSupLog ? p.nsb : p.nbins;
   const size_t vb = k1_vec_bytes(nbins);
   unsigned char *tail = smem + (size_t)kTileS * 16;
   unsigned short *wt2 = reinterpret_cast<unsigned short *>(tail);            // [2][8][nbins]
@@ -3055,8 +3059,10 @@ void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
     return;
   }
   const size_t sm = partition_smem_bytes(p.nbins, p.nb);
-  if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM
-    // bin_log 8 here: bin_log 7 is only chosen for > 131072 buffers (> 1024 bins)
+  if (p.nbins <= kLmMaxBins && p.bin_log == 7) {  // few-unit calls on a small registry
+    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 7>(p, n_sms, sm, st);
+    else launch_partition_lm<8, false, 7>(p, n_sms, sm, st);
+  } else if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM
     if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 8>(p, n_sms, sm, st);
     else launch_partition_lm<8, false, 8>(p, n_sms, sm, st);
   } else if (p.nbins < kTwoPassMinBins) {  // 171 .. 1023 bins: ranks in passes of <= 170 bins
@@ -3169,7 +3175,7 @@ void launch_shape(const Params &p, uint64_t key[3]) {
            (uint64_t)fold_sequential(p) << 3 | (uint64_t)(p.ns < 2ull * p.nb * p.W) << 4 |
            (uint64_t)(p.mkey != nullptr) << 5 | (uint64_t)(p.n_elig == p.nb) << 6 |
            (uint64_t)hang_prefix_path(p.W, p.H) << 7 | (uint64_t)(p.n_tiles_s != 0) << 8 |
-           (uint64_t)(p.n_tiles_e != 0) << 9;
+           (uint64_t)(p.n_tiles_e != 0) << 9 | (uint64_t)p.bin_log << 16;
 }
 const void *prep_kernel_fn() { return (const void *)k_prep; }
 void count_launches(unsigned n) { g_kernel_launches.fetch_add(n, std::memory_order_relaxed); }
@@ -3212,6 +3218,8 @@ void configure_kernels_once() {
   const int lm_mp = (int)k1_smem_lm(kTwoPassMinBins - 1, 0, false);
   cudaFuncSetAttribute(k_partition_lm<8, true, 8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
   cudaFuncSetAttribute(k_partition_lm<8, false, 8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  cudaFuncSetAttribute(k_partition_lm<8, true, 7, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false, 7, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
   cudaFuncSetAttribute(k_partition_lm<8, true, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
   cudaFuncSetAttribute(k_partition_lm<8, false, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_mp);
   cudaFuncSetAttribute(k_partition_lm<8, true, kSupLog, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
