@@ -1339,9 +1339,10 @@ __device__ __forceinline__ void fold_chunk(FoldSmem<BL> &S, int lane, unsigned l
 #define RTM_FOLD_NODUP_FAST 1
 #endif
   // the buffer state update of a chain tail (sum / mm / count over the chain, head's offset)
+  // mm = max << 16 | (0xFFFF - min): one __vmaxu2 combines both halves
   auto update = [&](const uint4 &sv, bool c0, unsigned long long d, unsigned mm, unsigned n16,
                     unsigned long long off0) {
-    unsigned hi = mm >> 16, lo = mm & 0xFFFFu;
+    unsigned hi = mm >> 16, lo = (mm & 0xFFFFu) ^ 0xFFFFu;
     if (c0) {
       hi = max(hi, sv.z >> 16);
       lo = min(lo, sv.w & 0xFFFFu);
@@ -1365,7 +1366,7 @@ __device__ __forceinline__ void fold_chunk(FoldSmem<BL> &S, int lane, unsigned l
       const unsigned long long contrib =
           NAR ? (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(unsigned)(Wlen - off))
               : (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off));
-      update(sv, c0, contrib, (lvl << 16) | lvl, 1u, off);
+      update(sv, c0, contrib, (lvl << 16) | (lvl ^ 0xFFFFu), 1u, off);
     }
     __syncwarp();
     return;
@@ -1388,16 +1389,22 @@ __device__ __forceinline__ void fold_chunk(FoldSmem<BL> &S, int lane, unsigned l
       : NAR ? (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(unsigned)(Wlen - off))
             : (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off));
   unsigned long long sum = contrib;
-  unsigned mm = (lvl << 16) | lvl;  // max << 16 | min over the chain so far
+  unsigned mm = (lvl << 16) | (lvl ^ 0xFFFFu);  // max << 16 | (0xFFFF - min) over the chain so far
   const unsigned maxrank = __reduce_max_sync(kFull, rank);
-#pragma unroll 1  // chains are short (maxrank is 1 in most chunks): a tight loop beats the 4x unroll (-1 %)
-  for (unsigned k = 0; k < maxrank; ++k) {
-    const unsigned long long su = __shfl_sync(kFull, sum, pred);
-    const unsigned mu = __shfl_sync(kFull, mm, pred);
-    if (lower) {
-      sum = contrib + su;
-      const unsigned hi = max(lvl, mu >> 16), lo = min(lvl, mu & 0xFFFFu);
-      mm = (hi << 16) | lo;
+  // Pointer jumping along the chain: after s steps a lane holds the combination of its chain
+  // elements at distance < 2^s, so ceil(log2(maxrank + 1)) steps (a hot buffer filling the chunk
+  // - Zipf skew, C4 - takes 5 steps, not 31).  pj = predecessor lane | 0x100 while it has one.
+  unsigned pj = (unsigned)pred | (lower ? 0x100u : 0u);
+#pragma unroll 1
+  for (unsigned d = 1; d <= maxrank; d <<= 1) {
+    const int src = (int)(pj & 31u);
+    const unsigned long long su = __shfl_sync(kFull, sum, src);
+    const unsigned mu = __shfl_sync(kFull, mm, src);
+    const unsigned pp = __shfl_sync(kFull, pj, src);
+    if (pj & 0x100u) {
+      sum += su;
+      mm = __vmaxu2(mm, mu);
+      pj = pp;
     }
   }
   const unsigned long long off0 = __shfl_sync(kFull, off, __ffs(peers) - 1);  // chain head's offset
