@@ -163,7 +163,8 @@ rtm_status ensure(rtm_ctx *c, DevBuf &b, size_t bytes, bool zero_new = false) {
     return RTM_E_NOMEM;
   }
   b.cap = want;
-  if (zero_new && cudaMemset(b.p, 0, want) != cudaSuccess) return cuda_fail(c, cudaGetLastError(), "memset", __LINE__);
+  // stream-ordered: the kernels that first use the buffer run on the context stream
+  if (zero_new && cudaMemsetAsync(b.p, 0, want, c->st) != cudaSuccess) return cuda_fail(c, cudaGetLastError(), "memset", __LINE__);
   return RTM_OK;
 }
 
@@ -271,6 +272,7 @@ rtm_status zero_state(rtm_ctx *c) {
   cl.add(c->cend.p, (size_t)c->nc * 8);
   cl.add(c->persist.p, (size_t)(c->n_global ? c->n_global : c->nb) * 4);
   cl.add(c->gcum.p, (size_t)c->nk * 16);
+  cl.add(c->cdelta.p, (size_t)c->nc * 16);
   launch_clear(cl, c->st);
   CK(cudaGetLastError());
   if (c->bars_dirty) {  // every registered bar live with its registered total (only after changes:
@@ -519,6 +521,10 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     if (t_end[w] - (w ? t_end[w - 1] : c->t_prev) >= ((int64_t)1 << 32)) p.narrow = 0;
   if (c->rank_mode == RTM_RANK_MEAN && !p.narrow) return RTM_E_INVALID;  // before any launch
   p.T = (const long long *)c->T.p;
+  if (W + 1 <= kTInline) {
+    p.t_inline = 1;
+    for (uint32_t w = 0; w <= W; ++w) p.Tin[w] = hT[w];
+  }
   p.s = (const rtm_level_sample *)sp; p.ns = ns;
   p.e = (const rtm_task_event *)ep; p.ne = ne;
 
@@ -549,7 +555,9 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   }
   if ((s = ensure(c, c->res, res_layout(c, W).bytes))) return s;
   if ((s = ensure(c, c->kdelta, Wn * c->nk * 2 * 4))) return s;
-  if ((s = ensure(c, c->cdelta, (size_t)c->nc * 2 * 8))) return s;
+  // per-component event deltas: zeroed at allocation and by rtm_reset, re-zeroed by k_progress
+  // after it folds them into the cumulative counts (no per-call clear: C5 1.3 MB)
+  if ((s = ensure(c, c->cdelta, (size_t)c->nc * 2 * 8, true))) return s;
   if ((s = ensure(c, c->active, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->anyfull, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->hung, Wn * c->ncw * 4))) return s;
@@ -580,7 +588,6 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     cl.add(c->res.p, (size_t)kWinFields * Wn * 8);
     cl.add((char *)c->res.p + L.status, 16);
     cl.add(c->kdelta.p, Wn * c->nk * 2 * 4);
-    cl.add(c->cdelta.p, (size_t)c->nc * 2 * 8);
     cl.add(c->active.p, Wn * c->ncw * 4);
     cl.add(c->anyfull.p, Wn * c->ncw * 4);
     // long H, call shorter than H: the hang kernel stops at the first window its prefix AND empties
@@ -630,7 +637,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   // list and the split buffers).  Direct launches, or captured once per launch shape into a CUDA
   // graph and replayed (rtm_use_graphs).
   auto enqueue = [&]() -> rtm_status {
-  CK(cudaMemcpyAsync(c->T.p, hT, (size_t)(W + 1) * 8, cudaMemcpyHostToDevice, c->st));
+  if (!p.t_inline) CK(cudaMemcpyAsync(c->T.p, hT, (size_t)(W + 1) * 8, cudaMemcpyHostToDevice, c->st));
   // clear the call's accumulators, region boundaries, tile tables: one cooperative launch
   LAUNCH(KT_SPLIT, 0,
          launch_prep(p, prep_cl, (long long *)c->Bs.p, (long long *)c->Be.p, c->n_sms, c->st));

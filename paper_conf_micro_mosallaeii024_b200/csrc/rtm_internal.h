@@ -40,6 +40,7 @@ constexpr int kFoldWarps = RTM_FOLD_WARPS;  // warps per fold CTA (compile-time 
 constexpr uint16_t kSent = 0xFFFFu;         // "no kept sample in this window" marker
 constexpr uint32_t kMaxBins = 4096;         // n_buffers <= 2^20 (fallback partition smem 160 KB)
 constexpr uint32_t kTopkSmemKeys = 40960;
+constexpr uint32_t kTInline = 16;           // window bounds passed inline for W + 1 <= 16
 constexpr uint32_t kLmMaxBins = 170;        // lane-major partition: count rows (bins x 48 B) fit a warp's 8 KB slot
 constexpr int kSupLog = 14;                 // two-pass partition: superbins of 2^14 buffers (<= 64 of them)   // keys held in shared memory by the top-k kernel
 // ts offset field of a staging entry: 48 - bin_log bits (entry = off << (16 + bin_log) | level << bin_log | lid)
@@ -98,6 +99,10 @@ struct Params {
   int32_t narrow;            // every window shorter than 2^32 ticks (32-bit order check)
   uint32_t epoch;
   const long long *T;        // [W+1]: T[0] = t_begin, T[w+1] = t_end[w]
+  // few-window calls (W + 1 <= kTInline): the window bounds travel in the kernel arguments and
+  // k_prep writes T (no host-to-device copy in the call's launch sequence)
+  int32_t t_inline;
+  long long Tin[16];
   const rtm_level_sample *s;
   uint64_t ns;
   const rtm_task_event *e;

@@ -139,10 +139,35 @@ __device__ unsigned block_excl_scan(unsigned v, unsigned *scratch /*[32]*/, unsi
 template <bool SAMPLES>
 __device__ __forceinline__ void split_one(const Params &p, unsigned q, long long *outB) {
   const int lane = threadIdx.x & 31;
-  const long long T = p.T[q];
+  const long long T = p.t_inline ? p.Tin[q] : p.T[q];
   const unsigned long long N = SAMPLES ? p.ns : p.ne;
   const int4 *recs = SAMPLES ? reinterpret_cast<const int4 *>(p.s) : reinterpret_cast<const int4 *>(p.e);
   unsigned long long lo = 0, hi = N;
+  // Fast exits for the call's outer boundaries (one probe round instead of the search; the
+  // common streaming call ingests exactly its windows' records): the first boundary is 0 when the
+  // stream's first field-valid record is at or after it, the last is 1 + the index of the last
+  // field-valid record when that one is before it (sorted stream; an unsorted one is reported by
+  // the order check).
+  if ((q == 0 || q == p.W) && N > 0) {
+    const bool first = q == 0;
+    const unsigned long long i = first ? (unsigned long long)lane : N - 1 - (unsigned long long)lane;
+    bool ok = false;
+    long long ts = 0;
+    if (i < N) {
+      const int4 v = __ldcg(recs + i);
+      ok = SAMPLES ? sample_valid(p, v) : event_valid(p, v);
+      ts = rec_ts(v);
+    }
+    const unsigned m = __ballot_sync(kFull, ok);
+    if (m) {
+      const int src = __ffs(m) - 1;  // first: lowest index; last: lane 0 probes N - 1
+      const long long t = __shfl_sync(kFull, ts, src);
+      if (first ? t >= T : t < T) {
+        if (lane == 0) outB[q] = first ? 0 : (long long)(N - (unsigned long long)src);
+        return;
+      }
+    }
+  }
   while (hi - lo > 64) {  // then <= 2 dependent rounds of the final scan
     unsigned long long span = hi - lo;
     unsigned long long qq = lo + span * (unsigned long long)(lane + 1) / 33ull;
@@ -287,6 +312,7 @@ __device__ __forceinline__ void clear_ranges(const ClearList &cl) {
 __global__ void __launch_bounds__(256, 4) k_prep(Params p, ClearList cl, long long *Bs, long long *Be) {
   namespace cg = cooperative_groups;
   cg::grid_group grid = cg::this_grid();
+  if (p.t_inline && blockIdx.x == 0 && threadIdx.x <= p.W) const_cast<long long *>(p.T)[threadIdx.x] = p.Tin[threadIdx.x];
   clear_ranges(cl);
   const unsigned nwarps = gridDim.x * (blockDim.x >> 5);
   for (unsigned q = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; q <= 2 * p.W + 1; q += nwarps) {
@@ -1418,9 +1444,26 @@ __device__ __forceinline__ void fold_chunk(FoldSmem<BL> &S, int lane, unsigned l
 // carry-in, full bits, digest, mean-occupancy keys, watched buffers, the last window's table).
 // S holds the unit's per-buffer phase-1 state: st (D, last | max << 16, min | n16 << 16), hi
 // (n_hi | ts0_hi << 16) and ts0 (offset of the buffer's first kept sample in the window).
-template <bool NAR, bool SPARSE, typename FS>
+// digest term of one touched (window, buffer) (reading R17): odd-constant products
+// of (I, n | id, levels | capacity), XOR, one fmix64 (splitmix64 finalizer)
+__device__ __forceinline__ unsigned long long digest_term(unsigned long long I, unsigned cnt, unsigned bid, unsigned last,
+                                                          unsigned mx, unsigned mn, unsigned capb) {
+  unsigned long long h = (I * 0x9E3779B97F4A7C15ULL) ^ ((((unsigned long long)cnt << 32) | bid) * 0xC2B2AE3D27D4EB4FULL) ^
+                         (((unsigned long long)last | ((unsigned long long)mx << 16) | ((unsigned long long)mn << 32) |
+                           ((unsigned long long)capb << 48)) *
+                          0x165667B19E3779F9ULL);
+  h ^= h >> 30;
+  h *= 0xbf58476d1ce4e5b9ULL;
+  h ^= h >> 27;
+  h *= 0x94d049bb133111ebULL;
+  h ^= h >> 31;
+  return h;
+}
+
+template <bool NAR, bool SPARSE, typename FS, bool CF = false>
 __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, unsigned bin,
                                             unsigned long long Wlen, int lane) {
+  static_assert(!CF || (NAR && SPARSE), "compacted finalize: narrow windows, sparse units");
   {
     // ---- publish this window's last levels (kSent: untouched) and the phase-1 flag
     const unsigned b_base = bin * FS::kB;
@@ -1533,7 +1576,9 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
       const unsigned hw = S.hi[l];
       if (st_touched(sv)) {
         const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
-        I = (unsigned long long)L * (((unsigned long long)(hw >> 16) << 32) | S.ts0[l]) + st_D(sv);
+        // NAR: the first sample's offset fits 32 bits (hw's upper half is reused below)
+        I = (unsigned long long)L * (NAR ? (unsigned long long)S.ts0[l]
+                                         : (((unsigned long long)(hw >> 16) << 32) | S.ts0[l])) + st_D(sv);
         mx = hi > L ? hi : L;
         mn = lo < L ? lo : L;
         last = sv.z & 0xFFFFu;
@@ -1545,6 +1590,62 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
     };
     const unsigned nb = p.nb;
     const unsigned short *capp = p.cap;
+    const bool nonempty_mode = p.hang_mode == RTM_HANG_NONEMPTY;
+    if constexpr (CF) {  // compacted finalize (NAR, sparse units; launch_fold_bl decides)
+      // Sparse units (C3, C4): many of the bin's buffers are untouched in the window.  Pass A
+      // resolves every untouched cell (row, held-full bit from the carry-in, MEAN key) and
+      // compacts the touched buffers into a list (the phase-1 owner slots are free now; each
+      // touched buffer's carry-in goes to the upper half of its hi word, unused for narrow
+      // windows); pass B finalizes the touched ones 32 at a time, so the digest runs on full
+      // warps instead of once per slot for the few touched lanes.
+      unsigned nt = 0;
+#pragma unroll
+      for (int i = 0; i < FS::kB / 32; ++i) {
+        const unsigned l = lane + 32 * i, b = b_base + l;
+        const bool t = b < nb && st_touched(S.st[l]);
+        if (b < nb && !t) {
+          const unsigned L = lin[i];
+          lw[b] = (uint16_t)L;
+          const unsigned capb = __ldg(capp + b);
+          if (p.mkey) p.mkey[(size_t)w * nb + b] = mean_key((unsigned long long)L * Wlen, capb, p.rcp64);
+          if (nonempty_mode ? L >= 1u : L == capb) {
+            const unsigned c = __ldg(p.owner + b);
+            atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
+          }
+        }
+        const unsigned m = __ballot_sync(kFull, t);
+        if (t) {
+          S.hi[l] |= (unsigned)lin[i] << 16;
+          S.owner[nt + __popc(m & lanemask_lt())] = (unsigned char)l;
+        }
+        nt += __popc(m);
+      }
+      __syncwarp();
+      for (unsigned q0 = 0; q0 < nt; q0 += 32) {
+        const unsigned q = q0 + lane;
+        if (q < nt) {
+          const unsigned l = S.owner[q], b = b_base + l;
+          const uint4 sv = S.st[l];
+          const unsigned hw = S.hi[l], L = hw >> 16;
+          const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
+          const unsigned long long I = (unsigned long long)L * S.ts0[l] + st_D(sv);
+          const unsigned mx = hi > L ? hi : L, mn = lo < L ? lo : L, last = sv.z & 0xFFFFu;
+          const unsigned cnt = ((hw & 0xFFFFu) << 16) + (sv.w >> 16);
+          const unsigned capb = __ldg(capp + b);
+          if (p.mkey) p.mkey[(size_t)w * nb + b] = mean_key(I, capb, p.rcp64);
+          if (nonempty_mode ? mn >= 1u : mn == capb) {
+            const unsigned c = __ldg(p.owner + b);
+            atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
+          }
+          const unsigned bid = p.gid ? __ldg(p.gid + b) : b;
+          dig += digest_term(I, cnt, bid, last, mx, mn, capb);
+        }
+      }
+      touched = lane == 0 ? nt : 0u;  // summed over the warp below
+      __syncwarp();
+      // the last-window / value-monitor pass below reads the carry-in from lin[] and the
+      // first-sample offset from ts0 only (NAR), so the reused hi bits do not matter
+    } else {
 #pragma unroll
     for (int i = 0; i < FS::kB / 32; ++i) {
       const unsigned b = b_base + lane + 32 * i;
@@ -1575,6 +1676,7 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
         dig += h;
         ++touched;
       }
+    }
     }
     // rare, uniform: the call's last window (per-buffer table, next call's carry) and the value
     // monitor's watched buffers - a second pass, so the loop above stays small
@@ -1690,7 +1792,7 @@ __device__ __forceinline__ void fold_phase1(const Params &p, FoldSmem<BL> &S, un
 // several consecutive windows, so the look-back walks several windows; it takes RTM_LB_STEP of
 // them per step (their flags waited for by as many lanes, all rows loaded before any is used),
 // dividing the dependent round trips.  A separate instantiation: the dense (C2) code is unchanged.
-template <bool NAR, bool SPARSE, int BL>
+template <bool NAR, bool SPARSE, int BL, bool CF = false>
 __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   using FS = FoldSmem<BL>;
@@ -1713,7 +1815,7 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
     }
     __syncwarp();
     fold_phase1<NAR, BL>(p, S, w, bin, Wlen, lane, lt);
-    fold_finish<NAR, SPARSE>(p, S, w, bin, Wlen, lane);
+    fold_finish<NAR, SPARSE, FoldSmem<BL>, CF>(p, S, w, bin, Wlen, lane);
   }
 }
 
@@ -2722,6 +2824,7 @@ __global__ void __launch_bounds__(1024) k_progress(Params p) {
   } else {
     for (unsigned c = (k - p.nk) * blockDim.x + threadIdx.x; c < p.nc; c += (gridDim.x - p.nk) * blockDim.x) {
       long long s = p.cstart[c] + (long long)p.cdelta[2 * c], e = p.cend[c] + (long long)p.cdelta[2 * c + 1];
+      p.cdelta[2 * c] = p.cdelta[2 * c + 1] = 0;  // consumed: zero for the next call
       p.cstart[c] = s;
       p.cend[c] = e;
       rtm_component_tasks t;
@@ -3101,7 +3204,11 @@ void launch_fold_bl(const Params &p, int n_sms, cudaStream_t st) {
   // sparse: fewer than 2 samples per buffer and window on average (C3-C5 shapes), so many of a
   // unit's buffers are untouched and the look-back walks several windows
   const bool sparse = p.ns < 2ull * p.nb * p.W;
-  if (p.narrow && sparse) { k_fold<true, true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  // compacted finalize when fewer samples than buffer-windows (C4: 0.86, Zipf, ~40 % of a unit's
+  // buffers touched: fold 31.8 -> 28.3 ms; C3 at 1.1 (2/3 touched) is faster without: 13.1 vs 15.9)
+  const bool very_sparse = p.ns < 1ull * p.nb * p.W;
+  if (p.narrow && very_sparse) { k_fold<true, true, BL, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else if (p.narrow && sparse) { k_fold<true, true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else if (p.narrow) { k_fold<true, false, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else if (sparse) { k_fold<false, true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else { k_fold<false, false, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
@@ -3180,9 +3287,10 @@ void launch_shape(const Params &p, uint64_t key[3]) {
   key[1] = (uint64_t)p.n_tiles_e | (uint64_t)p.tk_slices << 32;
   key[2] = (uint64_t)(p.narrow != 0) | (uint64_t)(p.fuse_events != 0) << 1 | (uint64_t)(p.nsb != 0) << 2 |
            (uint64_t)fold_sequential(p) << 3 | (uint64_t)(p.ns < 2ull * p.nb * p.W) << 4 |
+           (uint64_t)(p.ns < 1ull * p.nb * p.W) << 11 |
            (uint64_t)(p.mkey != nullptr) << 5 | (uint64_t)(p.n_elig == p.nb) << 6 |
            (uint64_t)hang_prefix_path(p.W, p.H) << 7 | (uint64_t)(p.n_tiles_s != 0) << 8 |
-           (uint64_t)(p.n_tiles_e != 0) << 9 | (uint64_t)p.bin_log << 16;
+           (uint64_t)(p.n_tiles_e != 0) << 9 | (uint64_t)(p.t_inline != 0) << 10 | (uint64_t)p.bin_log << 16;
 }
 const void *prep_kernel_fn() { return (const void *)k_prep; }
 void count_launches(unsigned n) { g_kernel_launches.fetch_add(n, std::memory_order_relaxed); }
@@ -3243,6 +3351,8 @@ void configure_kernels_once() {
   RTM_FOLD_ATTR(true, false, 8); RTM_FOLD_ATTR(false, false, 8); RTM_FOLD_ATTR(true, true, 8); RTM_FOLD_ATTR(false, true, 8);
   RTM_FOLD_ATTR(true, false, 7); RTM_FOLD_ATTR(false, false, 7); RTM_FOLD_ATTR(true, true, 7); RTM_FOLD_ATTR(false, true, 7);
 #undef RTM_FOLD_ATTR
+  cudaFuncSetAttribute(k_fold<true, true, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes(8));
+  cudaFuncSetAttribute(k_fold<true, true, 7, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes(7));
   cudaFuncSetAttribute(k_fold_seq<true, 7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<7>) * kFoldWarps));
   cudaFuncSetAttribute(k_fold_seq<false, 7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<7>) * kFoldWarps));
   cudaFuncSetAttribute(k_fold_seq<true, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<8>) * kFoldWarps));

@@ -961,6 +961,41 @@ def test_very_sparse_calls_sequential_fold(hang_mode):
             assert np.array_equal(ser[f], A[-300:, b][f]), (b, f)
 
 
+@pytest.mark.parametrize("hang_mode,rank_mode", [(0, 0), (1, 0), (0, 2)])
+def test_windowed_fold_compacted_finalize(hang_mode, rank_mode):
+    """Calls with 1/8 .. 1 kept samples per buffer-window (C4's density) take the windowed fold with
+    the compacted finalize (untouched cells resolved in one pass, touched buffers finalized 32 at a
+    time): 20 000 buffers, 0.5 samples per buffer-window, calls of 40 and 23 windows, watched
+    buffers, both hang criteria and the MEAN ranking - summaries, top-k, progress, hang lists, the
+    last window's table and the value-monitor rings equal the oracle's."""
+    wl = gen.C1.scaled("C1-cf", n_samples=630_000, n_events=63_000, n_buffers=20_000, n_windows=63, k=32,
+                       hang_windows=3)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=3, k=wl.k, hang_mode=hang_mode, rank_mode=rank_mode)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    watched = [0, 777, 19999]
+    mon.watch(watched)
+    s, e = gen.samples(wl), gen.events(wl)
+    t_end = wl.t_end()
+    rows, w0 = [], 0
+    for m in (40, 23):
+        w1 = w0 + m
+        sl = slice(wl.index_at("samples", wl.t_begin(w0)), wl.index_at("samples", wl.t_begin(w1)))
+        el = slice(wl.index_at("events", wl.t_begin(w0)), wl.index_at("events", wl.t_begin(w1)))
+        n = sl.stop - sl.start
+        assert wl.n_buffers * m / 8 < n < wl.n_buffers * m  # windowed fold, compacted finalize
+        ref = orc.reduce(s[sl], e[el], t_end[w0:w1], want_all_stats=True)
+        rows.append(ref["all_stats"])
+        mon.ingest(_dev(s[sl]), _dev(e[el]))
+        assert_same(mon.window_reduce(t_end[w0:w1]), ref, mon)
+        w0 = w1
+    A = np.concatenate(rows)
+    for q, b in enumerate(watched):
+        ser = mon.watch_series(q)
+        for f in ("integral", "last", "max", "min", "capacity", "n_samples", "mean_occ"):
+            assert np.array_equal(ser[f], A[-len(ser):, b][f]), (b, f)
+
+
 def test_large_registry_bins_of_128_dense_and_sparse_calls():
     """Registries of 131073 .. 524288 buffers use bins of 128 buffers (C5's 327680): the fallback
     partition with 128-buffer bins and every fold path on them - a dense call (>= 2 samples per

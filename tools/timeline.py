@@ -23,6 +23,7 @@ ap.add_argument("--windows", type=int, default=1000, help="windows per call")
 ap.add_argument("--calls", type=int, default=2)
 ap.add_argument("--warmup", type=int, default=2)
 ap.add_argument("--trace", default="")
+ap.add_argument("--graphs", type=int, default=1, help="rtm_use_graphs mode: 0 off, 1 auto, 2 always")
 args = ap.parse_args()
 wl = gen.CONFIGS[args.config]
 W = args.windows
@@ -36,6 +37,7 @@ gen.fill_device("events", wl, de.data_ptr(), 0, ne)
 torch.cuda.synchronize()
 owner, cap, tot = gen.registry(wl)
 mon = Monitor(owner, cap, tot, n_components=wl.n_components, t0=wl.t0, hang_windows=wl.hang_windows, k=wl.k)
+mon.use_graphs(args.graphs)
 
 
 def call(i):
