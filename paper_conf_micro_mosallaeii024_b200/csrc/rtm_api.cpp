@@ -77,6 +77,7 @@ struct rtm_ctx {
   DevBuf klive;             // progress bar ids in use
   std::vector<uint8_t> klive_h;
   std::vector<int64_t> ktotal0;  // bar totals registered at create (restored by reset)
+  uint32_t cap_max = 0;          // largest registered capacity (the fold's 32-bit D condition)
   bool bars_dirty = true;        // registry changed since create / the last reset
   std::vector<uint32_t> link_off, link_dst;  // component connection graph (CSR by source)
   // value monitor: watched ids (as given), their local ids (~0: not on this rank), rings
@@ -517,8 +518,14 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   c->epoch = c->epoch == 0xFFFFFFFFu ? 1u : c->epoch + 1u;
   p.W = W; p.epoch = c->epoch;
   p.narrow = 1;
-  for (uint32_t w = 0; w < W; ++w)
-    if (t_end[w] - (w ? t_end[w - 1] : c->t_prev) >= ((int64_t)1 << 32)) p.narrow = 0;
+  int64_t wlen_max = 0;
+  for (uint32_t w = 0; w < W; ++w) {
+    const int64_t len = t_end[w] - (w ? t_end[w - 1] : c->t_prev);
+    wlen_max = std::max(wlen_max, len);
+    if (len >= ((int64_t)1 << 32)) p.narrow = 0;
+  }
+  // the fold's integral term D lies in [0, cap * Wlen]: 32 bits when that is < 2^32
+  p.narrow_d = p.narrow && (uint64_t)c->cap_max * (uint64_t)wlen_max < ((uint64_t)1 << 32);
   if (c->rank_mode == RTM_RANK_MEAN && !p.narrow) return RTM_E_INVALID;  // before any launch
   p.T = (const long long *)c->T.p;
   if (W + 1 <= kTInline) {
@@ -889,6 +896,7 @@ rtm_status rtm_create(const rtm_config *cfg, rtm_ctx **out) {
       (s = ensure(c, c->klive, (size_t)c->nk)) || (s = ensure(c, c->gcum, (size_t)c->nk * 16)))
     return fail(s);
   c->ktotal0.assign(cfg->kernel_total, cfg->kernel_total + c->nk);
+  for (uint32_t b = 0; b < c->nb; ++b) c->cap_max = std::max<uint32_t>(c->cap_max, cfg->buffer_capacity[b]);
   if (c->rank_mode == RTM_RANK_MEAN) {
     if ((s = ensure(c, c->rcp64, (size_t)65536 * 8))) return fail(s);
     std::vector<unsigned long long> r64(65536, 0);

@@ -97,6 +97,7 @@ struct Params {
   // call
   uint32_t W;                // windows in the call
   int32_t narrow;            // every window shorter than 2^32 ticks (32-bit order check)
+  int32_t narrow_d;          // max capacity * every window length < 2^32: the fold's D in 32 bits
   uint32_t epoch;
   const long long *T;        // [W+1]: T[0] = t_begin, T[w+1] = t_end[w]
   // few-window calls (W + 1 <= kTInline): the window bounds travel in the kernel arguments and
@@ -210,6 +211,9 @@ struct ClearList {
 };
 void launch_clear(const ClearList &cl, cudaStream_t st);
 void configure_kernels_once();  // opt-in shared-memory limits, once per device
+void configure_partition_once();  // (rtm_partition.cu) the partition kernels' shared-memory limits
+int occupancy(const void *fn, int threads, size_t smem);  // resident blocks per SM (cached)
+bool partition_caps_smem(uint32_t nbins, uint32_t nb);  // the lane-major partition keeps cap[] in shared memory
 size_t fold_smem_bytes(int bin_log);
 size_t partition_smem_bytes(uint32_t nbins, uint32_t nb);
 size_t topk_smem_bytes(uint32_t nb);

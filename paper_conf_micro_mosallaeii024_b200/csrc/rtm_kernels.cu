@@ -10,6 +10,9 @@
 
 #include <algorithm>
 #include <atomic>
+#include <map>
+#include <mutex>
+#include <tuple>
 
 #include "rtm_internal.h"
 
@@ -309,6 +312,7 @@ __device__ __forceinline__ void clear_ranges(const ClearList &cl) {
 // tile tables): (A) zero the call's accumulators and find the region boundaries (one warp per
 // window boundary and stream), grid barrier, (B) boundaries -> per-region tile counts (blocks 0 and
 // 1), grid barrier, (C) the tile tables.  Every phase is grid-strided, so any co-resident grid works.
+#ifndef RTM_TU_PARTITION
 __global__ void __launch_bounds__(256, 4) k_prep(Params p, ClearList cl, long long *Bs, long long *Be) {
   namespace cg = cooperative_groups;
   cg::grid_group grid = cg::this_grid();
@@ -325,6 +329,7 @@ __global__ void __launch_bounds__(256, 4) k_prep(Params p, ClearList cl, long lo
   grid.sync();
   for (uint32_t r = blockIdx.x; r < p.W + 2; r += gridDim.x) fill_region(p, r, true, true);
 }
+#endif
 
 // ============================================================================================
 // K3: task events.  One CTA per tile of <= 4096 events of one region: validate, order-check,
@@ -438,11 +443,13 @@ __device__ __forceinline__ void events_tile(const Params &p, unsigned tile, unsi
   __syncthreads();  // shared memory free for the next tile
 }
 
+#ifndef RTM_TU_PARTITION
 __global__ void __launch_bounds__(kK3Threads) k_events(Params p) {
   if (blockIdx.x >= p.rte[p.W + 2]) return;  // grid sized by an upper bound
   extern __shared__ __align__(16) unsigned char smem[];
   events_tile(p, blockIdx.x, smem);
 }
+#endif
 
 // ============================================================================================
 // K1: sample partition.  A tile is <= 4096 samples of ONE region, handled by one CTA of 8 warps;
@@ -487,6 +494,7 @@ __host__ __device__ constexpr size_t k1_smem_lm(uint32_t nbins, uint32_t nb, boo
 }
 __host__ __device__ constexpr size_t k1_smem_mx(uint32_t nbins) { return (size_t)kTileS * 8 + 2 * k1_vec_bytes(nbins); }
 
+#ifdef RTM_TU_PARTITION  // the partition kernels: compiled in their own module (rtm_partition.cu)
 struct K1Tile {
   unsigned tile;
   int n;
@@ -1052,6 +1060,7 @@ __global__ void __launch_bounds__(kK1Threads) k_partition_mx(Params p) {
   for (unsigned q = threadIdx.x; q < (total + 1) / 2; q += kK1Threads) d4[q] = s4[q];
 }
 
+#endif  // RTM_TU_PARTITION
 
 // ============================================================================================
 // K1b (two-pass path: more than 170 bins, windows shorter than 2^32 ticks).  Pass 1 is the
@@ -1338,6 +1347,11 @@ __device__ __forceinline__ bool st_touched(const uint4 &v) { return (v.z & 0xFFF
 __device__ __forceinline__ unsigned long long st_D(const uint4 &v) {
   return ((unsigned long long)v.y << 32) | v.x;
 }
+// D and the first sample's offset (low 32 bits) of a touched state, either layout (ND: fold_chunk)
+template <bool ND>
+__device__ __forceinline__ unsigned long long st_Dn(const uint4 &v) { return ND ? (unsigned long long)v.x : st_D(v); }
+template <bool ND, typename FS>
+__device__ __forceinline__ unsigned st_ts0(const FS &S, const uint4 &v, unsigned l) { return ND ? v.y : S.ts0[l]; }
 
 // One chunk of <= 32 consecutive records (ingest order) of one (window, bin) unit.  Records of
 // the same buffer (peers, found with __match_any_sync) form a chain in lane order: each record's
@@ -1345,12 +1359,20 @@ __device__ __forceinline__ unsigned long long st_D(const uint4 &v) {
 // Contributions are computed in parallel; the group's sum / max / min travel down the chain in
 // `maxrank` shuffle steps and only the chain's last lane updates the shared state, so every
 // state update in a chunk touches a distinct buffer.
-template <bool NAR, int BL>
+// ND ("narrow D"): every registered capacity times every window length of the call
+// is below 2^32.  D's partial sums then stay in [0, cap * Wlen] (Abel summation: D_j = l_j u_j +
+// sum_{i<j} l_i (u_i - u_{i+1}) with u_i = t_end - ts_i non-increasing), so D is exact in unsigned
+// 32-bit wrapping arithmetic, and st.y holds the first sample's offset instead of D's high word
+// (one 16-byte state access per update, 32-bit products and chain shuffles).
+template <bool NAR, int BL, bool ND = false>
 __device__ __forceinline__ void fold_chunk(FoldSmem<BL> &S, int lane, unsigned lt, bool act, unsigned long long e,
                                            unsigned long long Wlen) {
+  static_assert(!ND || NAR, "narrow D implies narrow windows");
+  using DT = typename std::conditional<ND, unsigned, unsigned long long>::type;
+  using OT = typename std::conditional<NAR, unsigned, unsigned long long>::type;
   const unsigned lid = (unsigned)(e & ((1u << BL) - 1u));
   const unsigned lvl = (unsigned)(e >> BL) & 0xFFFFu;
-  const unsigned long long off = e >> (16 + BL);
+  const OT off = (OT)(e >> (16 + BL));
   // Peers = lanes holding the same buffer.  Most lanes hold a buffer no other lane of the chunk
   // holds, and __match_any_sync costs ~2 cycles of SM throughput per DISTINCT key in the warp
   // (tools/microbench.cu), so duplicates are found first through a shared-memory slot per
@@ -1364,35 +1386,49 @@ __device__ __forceinline__ void fold_chunk(FoldSmem<BL> &S, int lane, unsigned l
 #ifndef RTM_FOLD_NODUP_FAST
 #define RTM_FOLD_NODUP_FAST 1
 #endif
+  // (l - prev) * (t_end - ts): NAR one wide multiply; ND one 32-bit multiply (mod 2^32, exact at the end)
+  auto contrib_of = [&](unsigned prev) -> DT {
+    if constexpr (ND) return (unsigned)(lvl - prev) * (unsigned)((unsigned)Wlen - off);
+    else if constexpr (NAR)
+      return (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(unsigned)((unsigned)Wlen - off));
+    else return (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off));
+  };
   // the buffer state update of a chain tail (sum / mm / count over the chain, head's offset)
   // mm = max << 16 | (0xFFFF - min): one __vmaxu2 combines both halves
-  auto update = [&](const uint4 &sv, bool c0, unsigned long long d, unsigned mm, unsigned n16,
-                    unsigned long long off0) {
+  auto update = [&](const uint4 &sv, bool c0, DT d, unsigned mm, unsigned n16, OT off0) {
     unsigned hi = mm >> 16, lo = (mm & 0xFFFFu) ^ 0xFFFFu;
+    unsigned y;  // ND: first sample's offset; else D's high word
     if (c0) {
       hi = max(hi, sv.z >> 16);
       lo = min(lo, sv.w & 0xFFFFu);
-      d += st_D(sv);
+      if constexpr (ND) {
+        d += sv.x;
+        y = sv.y;
+      } else {
+        d += st_D(sv);
+      }
       n16 += sv.w >> 16;
       if (n16 > 0xFFFFu) {  // rare: more than 65535 samples of one buffer in one window
         S.hi[lid] += 1;
         n16 -= 0x10000u;
       }
     } else {
-      S.ts0[lid] = (unsigned)off0;
-      if (!NAR && (off0 >> 32)) S.hi[lid] += (unsigned)(off0 >> 32) << 16;  // windows >= 2^32 ticks
+      if constexpr (ND) {
+        y = (unsigned)off0;
+      } else {
+        S.ts0[lid] = (unsigned)off0;
+        if constexpr (!NAR)
+          if (off0 >> 32) S.hi[lid] += (unsigned)((unsigned long long)off0 >> 32) << 16;  // windows >= 2^32 ticks
+      }
     }
-    S.st[lid] = make_uint4((unsigned)d, (unsigned)(d >> 32), lvl | (hi << 16), lo | (n16 << 16));
+    if constexpr (!ND) y = (unsigned)((unsigned long long)d >> 32);
+    S.st[lid] = make_uint4((unsigned)d, y, lvl | (hi << 16), lo | (n16 << 16));
   };
   if (RTM_FOLD_NODUP_FAST && told == 0) {  // warp-uniform: every buffer of the chunk is distinct
     if (act) {  // each lane is its buffer's whole chain: no match, no chain propagation
       const uint4 sv = S.st[lid];
       const bool c0 = st_touched(sv);
-      const unsigned prev = c0 ? (sv.z & 0xFFFFu) : 0u;
-      const unsigned long long contrib =
-          NAR ? (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(unsigned)(Wlen - off))
-              : (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off));
-      update(sv, c0, contrib, (lvl << 16) | (lvl ^ 0xFFFFu), 1u, off);
+      update(sv, c0, contrib_of(c0 ? (sv.z & 0xFFFFu) : 0u), (lvl << 16) | (lvl ^ 0xFFFFu), 1u, off);
     }
     __syncwarp();
     return;
@@ -1409,12 +1445,8 @@ __device__ __forceinline__ void fold_chunk(FoldSmem<BL> &S, int lane, unsigned l
   if (act && (!lower || tail)) sv = S.st[lid];  // chain heads need the level, tails the state
   const bool c0 = st_touched(sv);
   const unsigned prev = lower ? plv : (c0 ? (sv.z & 0xFFFFu) : 0u);
-  // NAR: windows shorter than 2^32 ticks, (t_end - ts) fits 32 bits: one wide multiply
-  const unsigned long long contrib =
-      !act ? 0ull
-      : NAR ? (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(unsigned)(Wlen - off))
-            : (unsigned long long)((long long)((int)lvl - (int)prev) * (long long)(Wlen - off));
-  unsigned long long sum = contrib;
+  const DT contrib = act ? contrib_of(prev) : (DT)0;
+  DT sum = contrib;
   unsigned mm = (lvl << 16) | (lvl ^ 0xFFFFu);  // max << 16 | (0xFFFF - min) over the chain so far
   const unsigned maxrank = __reduce_max_sync(kFull, rank);
   // Pointer jumping along the chain: after s steps a lane holds the combination of its chain
@@ -1424,7 +1456,7 @@ __device__ __forceinline__ void fold_chunk(FoldSmem<BL> &S, int lane, unsigned l
 #pragma unroll 1
   for (unsigned d = 1; d <= maxrank; d <<= 1) {
     const int src = (int)(pj & 31u);
-    const unsigned long long su = __shfl_sync(kFull, sum, src);
+    const DT su = __shfl_sync(kFull, sum, src);
     const unsigned mu = __shfl_sync(kFull, mm, src);
     const unsigned pp = __shfl_sync(kFull, pj, src);
     if (pj & 0x100u) {
@@ -1433,7 +1465,7 @@ __device__ __forceinline__ void fold_chunk(FoldSmem<BL> &S, int lane, unsigned l
       pj = pp;
     }
   }
-  const unsigned long long off0 = __shfl_sync(kFull, off, __ffs(peers) - 1);  // chain head's offset
+  const OT off0 = __shfl_sync(kFull, off, __ffs(peers) - 1);  // chain head's offset
   if (act && tail) update(sv, c0, sum, mm, rank + 1, off0);
   __syncwarp();
 }
@@ -1460,7 +1492,7 @@ __device__ __forceinline__ unsigned long long digest_term(unsigned long long I, 
   return h;
 }
 
-template <bool NAR, bool SPARSE, typename FS, bool CF = false>
+template <bool NAR, bool SPARSE, typename FS, bool CF = false, bool ND = false>
 __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, unsigned bin,
                                             unsigned long long Wlen, int lane) {
   static_assert(!CF || (NAR && SPARSE), "compacted finalize: narrow windows, sparse units");
@@ -1577,8 +1609,8 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
       if (st_touched(sv)) {
         const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
         // NAR: the first sample's offset fits 32 bits (hw's upper half is reused below)
-        I = (unsigned long long)L * (NAR ? (unsigned long long)S.ts0[l]
-                                         : (((unsigned long long)(hw >> 16) << 32) | S.ts0[l])) + st_D(sv);
+        I = (unsigned long long)L * (NAR ? (unsigned long long)st_ts0<ND>(S, sv, l)
+                                         : (((unsigned long long)(hw >> 16) << 32) | S.ts0[l])) + st_Dn<ND>(sv);
         mx = hi > L ? hi : L;
         mn = lo < L ? lo : L;
         last = sv.z & 0xFFFFu;
@@ -1628,7 +1660,7 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
           const uint4 sv = S.st[l];
           const unsigned hw = S.hi[l], L = hw >> 16;
           const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
-          const unsigned long long I = (unsigned long long)L * S.ts0[l] + st_D(sv);
+          const unsigned long long I = (unsigned long long)L * st_ts0<ND>(S, sv, l) + st_Dn<ND>(sv);
           const unsigned mx = hi > L ? hi : L, mn = lo < L ? lo : L, last = sv.z & 0xFFFFu;
           const unsigned cnt = ((hw & 0xFFFFu) << 16) + (sv.w >> 16);
           const unsigned capb = __ldg(capp + b);
@@ -1722,7 +1754,7 @@ __device__ __forceinline__ void fold_finish(const Params &p, FS &S, unsigned w, 
 
 // Phase 1 of a fold unit (window w, bin): the (tile, bin) segments of window w flattened into one
 // stream of 32-sample chunks, each folded by fold_chunk into S (carry-in left symbolic).
-template <bool NAR, int BL>
+template <bool NAR, int BL, bool ND = false>
 __device__ __forceinline__ void fold_phase1(const Params &p, FoldSmem<BL> &S, unsigned w, unsigned bin,
                                             unsigned long long Wlen, int lane, unsigned lt) {
   if (p.woff) {  // two-pass path: the unit's entries are one contiguous range
@@ -1733,7 +1765,7 @@ __device__ __forceinline__ void fold_phase1(const Params &p, FoldSmem<BL> &S, un
     unsigned long long e0 = fetch(0), e1 = fetch(32);
     for (unsigned c = 0; c < total; c += 32) {
       const unsigned long long en = fetch(c + 64);
-      fold_chunk<NAR, BL>(S, lane, lt, c + lane < total, e0, Wlen);
+      fold_chunk<NAR, BL, ND>(S, lane, lt, c + lane < total, e0, Wlen);
       e0 = e1;
       e1 = en;
     }
@@ -1780,7 +1812,7 @@ __device__ __forceinline__ void fold_phase1(const Params &p, FoldSmem<BL> &S, un
       unsigned long long e0 = fetch(0), e1 = fetch(32);
       for (unsigned c = 0; c < total; c += 32) {
         const unsigned long long en = fetch(c + 64);
-        fold_chunk<NAR, BL>(S, lane, lt, c + lane < total, e0, Wlen);
+        fold_chunk<NAR, BL, ND>(S, lane, lt, c + lane < total, e0, Wlen);
         e0 = e1;
         e1 = en;
       }
@@ -1792,7 +1824,7 @@ __device__ __forceinline__ void fold_phase1(const Params &p, FoldSmem<BL> &S, un
 // several consecutive windows, so the look-back walks several windows; it takes RTM_LB_STEP of
 // them per step (their flags waited for by as many lanes, all rows loaded before any is used),
 // dividing the dependent round trips.  A separate instantiation: the dense (C2) code is unchanged.
-template <bool NAR, bool SPARSE, int BL, bool CF = false>
+template <bool NAR, bool SPARSE, int BL, bool CF = false, bool ND = false>
 __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   using FS = FoldSmem<BL>;
@@ -1814,8 +1846,8 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
       S.hi[lane + 32 * i] = 0;
     }
     __syncwarp();
-    fold_phase1<NAR, BL>(p, S, w, bin, Wlen, lane, lt);
-    fold_finish<NAR, SPARSE, FoldSmem<BL>, CF>(p, S, w, bin, Wlen, lane);
+    fold_phase1<NAR, BL, ND>(p, S, w, bin, Wlen, lane, lt);
+    fold_finish<NAR, SPARSE, FoldSmem<BL>, CF, ND>(p, S, w, bin, Wlen, lane);
   }
 }
 
@@ -1835,8 +1867,12 @@ __global__ void __launch_bounds__(kFoldWarps * 32, 32 / kFoldWarps) k_fold(Param
 // ============================================================================================
 template <int BL>
 struct FoldSeqSmem {
-  static constexpr int kB = 1 << BL, kPer = kB / 32;
+  static constexpr int kB = 1 << BL, kPer = kB / 32, kQ = 64;
   FoldSmem<BL> f;
+  // touched (window, buffer) results awaiting their finalize, 32 at a time: state; hi word, window,
+  // lid | carried level << 16, first sample's offset (wide layout)
+  uint4 qst[kQ];
+  uint4 qmeta[kQ];
   unsigned short lvl[kB];   // carried level of every buffer of the bin
   unsigned short list[kB];  // the window's touched buffers (compacted)
   unsigned short capS[kB];  // capacities and owners of the bin (the touched finalize reads them)
@@ -1844,7 +1880,7 @@ struct FoldSeqSmem {
   unsigned tmask[kPer];     // the window's touched buffers (bit lid)
 };
 
-template <bool NAR, int BL>
+template <bool NAR, int BL, bool ND = false>
 __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   using QS = FoldSeqSmem<BL>;
@@ -1880,8 +1916,54 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
       Q.ownS[l] = b < p.nb ? __ldg(p.owner + b) : 0;
     }
     __syncwarp();
-    // finalize of window w (its samples are folded into S): touched buffers, the last-level row,
-    // held-full bits, the window's digest and touched count
+    // finalize queue entries [base, base + m), one per lane: integral, max / min with the carried
+    // level, digest (added to its window's sum), held-full bit, the call's table / value monitor
+    unsigned qn = 0;
+    auto flush = [&](unsigned base, unsigned m) {
+      if ((unsigned)lane < m) {
+        const uint4 sv = Q.qst[base + lane], mt = Q.qmeta[base + lane];
+        const unsigned hw = mt.x, w = mt.y, l = mt.z & 0xFFFFu, L = mt.z >> 16, b = b_base + l;
+        const unsigned cnt = ((hw & 0xFFFFu) << 16) + (sv.w >> 16);
+        const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
+        const unsigned long long I =
+            (unsigned long long)L * (ND ? (unsigned long long)sv.y : (((unsigned long long)(hw >> 16) << 32) | mt.w)) +
+            st_Dn<ND>(sv);
+        const unsigned mx = hi > L ? hi : L, mn = lo < L ? lo : L, last = sv.z & 0xFFFFu;
+        const unsigned capb = Q.capS[l];
+        const unsigned bid = p.gid ? __ldg(p.gid + b) : b;
+        atomicAdd(p.win + WF_DIGEST * p.W + w, digest_term(I, cnt, bid, last, mx, mn, capb));
+        if (nonempty_mode ? mn >= 1u : mn == capb) {  // held the whole window
+          const unsigned c = Q.ownS[l];
+          atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
+        }
+        const bool last_window = (w == p.W - 1);
+        if (last_window || p.n_watch) {  // rare: the call's table, the value monitor
+          int wq = -1;
+          for (unsigned k2 = 0; k2 < p.n_watch; ++k2)
+            if (p.watch[k2] == b) wq = (int)k2;
+          if (last_window || wq >= 0) {
+            const unsigned long long Wlen = (unsigned long long)(p.T[w + 1] - p.T[w]);
+            rtm_buffer_stat st;
+            st.integral = (int64_t)I;
+            st.last = (uint16_t)last;
+            st.max = (uint16_t)mx;
+            st.min = (uint16_t)mn;
+            st.capacity = (uint16_t)capb;
+            st.n_samples = cnt;
+            st.reserved = __ldg(p.elig + b);
+            st.mean_occ = Wlen ? __ddiv_rn((double)(long long)I, (double)((long long)capb * (long long)Wlen)) : 0.0;
+            if (wq >= 0) p.wstat[(size_t)w * RTM_WATCH_MAX + wq] = st;
+            if (last_window) {
+              p.bstat[b] = st;
+              p.carry_out[b] = (uint16_t)last;
+            }
+          }
+        }
+      }
+      __syncwarp();
+    };
+    // finalize of window w (its samples are folded into S): touched buffers queued, the
+    // last-level row, held-full bits of the untouched ones, the window's touched count
     auto finalize = [&](unsigned w, unsigned long long Wlen) {
       const bool last_window = (w == p.W - 1);
         // ---- compact the touched buffers (owner-strided scan of the state)
@@ -1895,61 +1977,29 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
           nt += __popc(m);
         }
         __syncwarp();
-        // ---- finalize the touched buffers, 32 at a time
-        unsigned long long dig = 0;
+        // ---- queue the touched buffers (state, carried level, window), advance their carried
+        // level and reset their state; the queue is finalized 32 entries at a time (flush), so
+        // the digest runs on full warps across windows instead of a few lanes per window
         for (unsigned q0 = 0; q0 < nt; q0 += 32) {
-          const unsigned q = q0 + lane;
-          if (q < nt) {
-            const unsigned l = Q.list[q], b = b_base + l;
-            const unsigned L = Q.lvl[l];
+          const unsigned n = nt - q0 < 32u ? nt - q0 : 32u;
+          if (qn + n > (unsigned)QS::kQ) {  // warp-uniform: make room
+            flush(0, qn);
+            qn = 0;
+          }
+          if ((unsigned)lane < n) {
+            const unsigned l = Q.list[q0 + lane];
             const uint4 sv = S.st[l];
-            const unsigned hw = S.hi[l];
-            const unsigned cnt = ((hw & 0xFFFFu) << 16) + (sv.w >> 16);
-            const unsigned hi = sv.z >> 16, lo = sv.w & 0xFFFFu;
-            const unsigned long long I =
-                (unsigned long long)L * (((unsigned long long)(hw >> 16) << 32) | S.ts0[l]) + st_D(sv);
-            const unsigned mx = hi > L ? hi : L, mn = lo < L ? lo : L, last = sv.z & 0xFFFFu;
-            const unsigned capb = Q.capS[l];
-            const unsigned bid = p.gid ? __ldg(p.gid + b) : b;
-            unsigned long long h = (I * 0x9E3779B97F4A7C15ULL) ^
-                                   ((((unsigned long long)cnt << 32) | bid) * 0xC2B2AE3D27D4EB4FULL) ^
-                                   (((unsigned long long)last | ((unsigned long long)mx << 16) |
-                                     ((unsigned long long)mn << 32) | ((unsigned long long)capb << 48)) *
-                                    0x165667B19E3779F9ULL);
-            h ^= h >> 30;
-            h *= 0xbf58476d1ce4e5b9ULL;
-            h ^= h >> 27;
-            h *= 0x94d049bb133111ebULL;
-            h ^= h >> 31;
-            dig += h;
-            if (nonempty_mode ? mn >= 1u : mn == capb) {  // held the whole window
-              const unsigned c = Q.ownS[l];
-              atomicOr(p.anyfull + (size_t)w * p.ncw + (c >> 5), 1u << (c & 31));
-            }
-            if (last_window || p.n_watch) {  // rare: the call's table, the value monitor
-              int wq = -1;
-              for (unsigned k2 = 0; k2 < p.n_watch; ++k2)
-                if (p.watch[k2] == b) wq = (int)k2;
-              if (last_window || wq >= 0) {
-                rtm_buffer_stat st;
-                st.integral = (int64_t)I;
-                st.last = (uint16_t)last;
-                st.max = (uint16_t)mx;
-                st.min = (uint16_t)mn;
-                st.capacity = (uint16_t)capb;
-                st.n_samples = cnt;
-                st.reserved = __ldg(p.elig + b);
-                st.mean_occ = Wlen ? __ddiv_rn((double)(long long)I, (double)((long long)capb * (long long)Wlen)) : 0.0;
-                if (wq >= 0) p.wstat[(size_t)w * RTM_WATCH_MAX + wq] = st;
-                if (last_window) {
-                  p.bstat[b] = st;
-                  p.carry_out[b] = (uint16_t)last;
-                }
-              }
-            }
-            Q.lvl[l] = (unsigned short)last;
+            Q.qst[qn + lane] = sv;
+            Q.qmeta[qn + lane] = make_uint4(S.hi[l], w, l | ((unsigned)Q.lvl[l] << 16), ND ? 0u : S.ts0[l]);
+            Q.lvl[l] = (unsigned short)(sv.z & 0xFFFFu);
             S.st[l] = make_uint4(0, 0, kUntouchedZ, 0);
             S.hi[l] = 0;
+          }
+          qn += n;
+          __syncwarp();
+          if (qn >= 32u) {
+            flush(qn - 32u, 32u);
+            qn -= 32u;
           }
         }
         __syncwarp();
@@ -2004,11 +2054,7 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
             }
           }
         }
-        dig = warp_sum(dig);
-        if (lane == 0) {
-          if (dig) atomicAdd(p.win + WF_DIGEST * p.W + w, dig);
-          if (nt) atomicAdd(p.win + WF_TOUCHED * p.W + w, (unsigned long long)nt);
-        }
+        if (lane == 0 && nt) atomicAdd(p.win + WF_TOUCHED * p.W + w, (unsigned long long)nt);
         __syncwarp();
     };
     // Software pipeline over the windows: while window w's staging entries and window w+1's
@@ -2035,7 +2081,7 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
         if (pend) finalize(pw, pWlen);
         for (unsigned c = 0; c < total; c += 32) {
           const unsigned long long en = c + 64 < total ? fetch(c + 64) : 0ull;
-          fold_chunk<NAR, BL>(S, lane, lt, c + lane < total, e0, Wlen);
+          fold_chunk<NAR, BL, ND>(S, lane, lt, c + lane < total, e0, Wlen);
           e0 = e1;
           e1 = en;
         }
@@ -2045,6 +2091,7 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
         pWlen = Wlen;
       }
       if (pend) finalize(pw, pWlen);
+      flush(0, qn);
       continue;
     }
     unsigned n_tlo = p.rts[1], n_thi = p.rts[2];
@@ -2102,14 +2149,14 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
         if (pend) finalize(pw, pWlen);
         for (unsigned c = 0; c < total; c += 32) {
           const unsigned long long en = c + 64 < total ? fetch(c + 64) : 0ull;
-          fold_chunk<NAR, BL>(S, lane, lt, c + lane < total, e0, Wlen);
+          fold_chunk<NAR, BL, ND>(S, lane, lt, c + lane < total, e0, Wlen);
           e0 = e1;
           e1 = en;
         }
         __syncwarp();
       } else {  // many tiles in one window: the general phase 1, no overlap
         if (pend) finalize(pw, pWlen);
-        fold_phase1<NAR, BL>(p, S, w, bin, Wlen, lane, lt);
+        fold_phase1<NAR, BL, ND>(p, S, w, bin, Wlen, lane, lt);
         __syncwarp();
         if (w + 1 < p.W) {
           n_tlo = p.rts[w + 2];
@@ -2128,9 +2175,11 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
       pWlen = Wlen;
     }
     if (pend) finalize(pw, pWlen);
+    flush(0, qn);
   }
 }
 
+#ifndef RTM_TU_PARTITION  // (to the end of the file but the partition launchers)
 // ============================================================================================
 // K4: cross-tile order check.  Every tile has its in-tile verdict (flag bit 1: range / order
 // inside the tile) and the offsets of its first / last field-valid record.  The field-valid
@@ -3063,11 +3112,17 @@ __global__ void k_scatter_bstat(Params p) {
     p.bstat_g[__ldg(p.gid + b)] = p.bstat[b];
 }
 
+#endif  // RTM_TU_PARTITION
 }  // namespace
 
 // ============================================================================================
 // launchers
 // ============================================================================================
+constexpr uint32_t kTwoPassMinBins = 1024;
+#ifdef RTM_TU_PARTITION
+extern std::atomic<unsigned long long> g_kernel_launches;
+inline void count_launch() { g_kernel_launches.fetch_add(1, std::memory_order_relaxed); }
+#else
 __global__ void k_clear(ClearList cl) { clear_ranges(cl); }
 
 std::atomic<unsigned long long> g_kernel_launches{0};
@@ -3089,7 +3144,6 @@ size_t fold_smem_bytes(int bin_log) {
 // path tie (28.5 vs 29.4 ms per step: k_subpart reads the entries twice at ~4 warp instructions
 // each); 2560 bins (C5) fold 22.4 -> 17.9 ms per 10k windows; 4096 bins (C4) 132.5 -> 77.5 ms.
 // Below it, 171 .. 1023 bins take the lane-major partition with multi-pass ranking (MP).
-constexpr uint32_t kTwoPassMinBins = 1024;
 // lane-major partition: the capacity table in shared memory when two CTAs still fit per SM
 bool partition_caps_smem(uint32_t nbins, uint32_t nb) { return k1_smem_lm(nbins, nb, true) + 1024 <= 113 * 1024; }
 size_t partition_smem_bytes(uint32_t nbins, uint32_t nb) {
@@ -3101,6 +3155,39 @@ static_assert(k1_smem_lm(kLmMaxBins, 0, false) <= 113 * 1024 && k1_smem_lm(kTwoP
               "partition shared memory exceeds the opt-in limit");
 size_t topk_smem_bytes(uint32_t nb) {
   return (size_t)(nb <= kTopkSmemKeys ? ((nb + 1) & ~1u) : 0) * 4 + 8 * 256 * 4 + 1024 * 8 + kTopkCand * 4;
+}
+
+// Resident blocks per SM of a kernel at a block size / dynamic shared memory, cached per device:
+// the occupancy query is a driver call of tens of microseconds, made on the launch path of every
+// call otherwise (the GPU idled behind it between k_prep and the partition).
+int occupancy(const void *fn, int threads, size_t smem) {
+  struct Key {
+    const void *fn;
+    int threads, dev;
+    size_t smem;
+    bool operator<(const Key &o) const {
+      return std::tie(fn, threads, dev, smem) < std::tie(o.fn, o.threads, o.dev, o.smem);
+    }
+  };
+  static std::mutex mu;
+  static std::map<Key, int> cache;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const Key k{fn, threads, dev, smem};
+  {
+    std::lock_guard<std::mutex> g(mu);
+    auto it = cache.find(k);
+    if (it != cache.end()) return it->second;
+  }
+  int n = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, threads, smem) != cudaSuccess) {
+    cudaGetLastError();
+    n = 0;
+  }
+  if (n < 1) n = 1;
+  std::lock_guard<std::mutex> g(mu);
+  cache[k] = n;
+  return n;
 }
 
 void launch_prep(const Params &p, const ClearList &cl, long long *Bs, long long *Be, int n_sms, cudaStream_t st) {
@@ -3132,9 +3219,7 @@ bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s, bool two_pass) {
 template <int BL>
 void launch_subpart_bl(const Params &p, int n_sms, cudaStream_t st) {
   const size_t sm = sizeof(SubSmem<BL>) * kSubWarps;
-  int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_subpart<BL>, kSubWarps * 32, sm);
-  if (per_sm < 1) per_sm = 1;
+  const int per_sm = occupancy((const void *)k_subpart<BL>, kSubWarps * 32, sm);
   unsigned grid = (unsigned)(n_sms * per_sm);
   const unsigned need = (p.W * p.nsb + kSubWarps - 1) / kSubWarps;
   if (grid > need) grid = need;
@@ -3148,42 +3233,6 @@ void launch_subpart(const Params &p, int n_sms, cudaStream_t st) {
   else launch_subpart_bl<8>(p, n_sms, st);
 }
 
-template <int BL, bool CAPS, int KS, bool MP = false>
-void launch_partition_lm(const Params &p, int n_sms, size_t sm, cudaStream_t st) {
-  int per_sm = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition_lm<BL, CAPS, KS, MP>, kK1Threads, sm);
-  if (per_sm < 1) per_sm = 1;
-  unsigned grid = (unsigned)(n_sms * per_sm);
-  const unsigned work = p.n_tiles_s + (p.fuse_events ? p.n_tiles_e : 0u);
-  if (grid > work) grid = work;
-  { k_partition_lm<BL, CAPS, KS, MP><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
-}
-
-void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
-  if (!p.n_tiles_s) return;
-  if (p.nsb) {  // two-pass path, pass 1: superbin keys (capacities through L1: > 2^15 buffers)
-    const bool caps = partition_caps_smem(p.nsb, p.nb);
-    const size_t sm = k1_smem_lm(p.nsb, p.nb, caps);
-    if (caps) launch_partition_lm<8, true, kSupLog>(p, n_sms, sm, st);
-    else launch_partition_lm<8, false, kSupLog>(p, n_sms, sm, st);
-    return;
-  }
-  const size_t sm = partition_smem_bytes(p.nbins, p.nb);
-  if (p.nbins <= kLmMaxBins && p.bin_log == 7) {  // few-unit calls on a small registry
-    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 7>(p, n_sms, sm, st);
-    else launch_partition_lm<8, false, 7>(p, n_sms, sm, st);
-  } else if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM
-    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 8>(p, n_sms, sm, st);
-    else launch_partition_lm<8, false, 8>(p, n_sms, sm, st);
-  } else if (p.nbins < kTwoPassMinBins) {  // 171 .. 1023 bins: ranks in passes of <= 170 bins
-    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 8, true>(p, n_sms, sm, st);
-    else launch_partition_lm<8, false, 8, true>(p, n_sms, sm, st);
-  } else {
-    if (p.bin_log == 7) { k_partition_mx<7><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
-    else { k_partition_mx<8><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
-  }
-}
-
 void launch_events(const Params &p, cudaStream_t st) {
   if (!p.n_tiles_e) return;
   const size_t sm = (size_t)2 * p.nk * 4 + (p.ncw <= 2048 ? (size_t)p.ncw * 4 : 0);
@@ -3193,9 +3242,7 @@ void launch_events(const Params &p, cudaStream_t st) {
 template <int BL>
 void launch_fold_bl(const Params &p, int n_sms, cudaStream_t st) {
   const size_t sm = fold_smem_bytes(BL);
-  int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fold<true, false, BL>, kFoldWarps * 32, sm);
-  if (per_sm < 1) per_sm = 1;
+  const int per_sm = occupancy((const void *)k_fold<true, false, BL>, kFoldWarps * 32, sm);
   unsigned grid = (unsigned)(n_sms * per_sm);
   const unsigned units = p.W * p.nbins;
   const unsigned need = (units + kFoldWarps - 1) / kFoldWarps;
@@ -3207,7 +3254,10 @@ void launch_fold_bl(const Params &p, int n_sms, cudaStream_t st) {
   // compacted finalize when fewer samples than buffer-windows (C4: 0.86, Zipf, ~40 % of a unit's
   // buffers touched: fold 31.8 -> 28.3 ms; C3 at 1.1 (2/3 touched) is faster without: 13.1 vs 15.9)
   const bool very_sparse = p.ns < 1ull * p.nb * p.W;
-  if (p.narrow && very_sparse) { k_fold<true, true, BL, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  if (p.narrow_d && very_sparse) { k_fold<true, true, BL, true, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else if (p.narrow_d && sparse) { k_fold<true, true, BL, false, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else if (p.narrow_d) { k_fold<true, false, BL, false, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else if (p.narrow && very_sparse) { k_fold<true, true, BL, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else if (p.narrow && sparse) { k_fold<true, true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else if (p.narrow) { k_fold<true, false, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else if (sparse) { k_fold<false, true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
@@ -3222,13 +3272,12 @@ bool fold_sequential(const Params &p) {
 template <int BL>
 void launch_fold_seq(const Params &p, int n_sms, cudaStream_t st) {
   const size_t sm = sizeof(FoldSeqSmem<BL>) * kFoldWarps;
-  int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fold_seq<true, BL>, kFoldWarps * 32, sm);
-  if (per_sm < 1) per_sm = 1;
+  const int per_sm = occupancy((const void *)k_fold_seq<true, BL>, kFoldWarps * 32, sm);
   unsigned grid = (unsigned)(n_sms * per_sm);
   const unsigned need = (p.nbins + kFoldWarps - 1) / kFoldWarps;
   if (grid > need) grid = need;
-  if (p.narrow) { k_fold_seq<true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  if (p.narrow_d) { k_fold_seq<true, BL, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
+  else if (p.narrow) { k_fold_seq<true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else { k_fold_seq<false, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
 }
 
@@ -3287,7 +3336,7 @@ void launch_shape(const Params &p, uint64_t key[3]) {
   key[1] = (uint64_t)p.n_tiles_e | (uint64_t)p.tk_slices << 32;
   key[2] = (uint64_t)(p.narrow != 0) | (uint64_t)(p.fuse_events != 0) << 1 | (uint64_t)(p.nsb != 0) << 2 |
            (uint64_t)fold_sequential(p) << 3 | (uint64_t)(p.ns < 2ull * p.nb * p.W) << 4 |
-           (uint64_t)(p.ns < 1ull * p.nb * p.W) << 11 |
+           (uint64_t)(p.ns < 1ull * p.nb * p.W) << 11 | (uint64_t)(p.narrow_d != 0) << 12 |
            (uint64_t)(p.mkey != nullptr) << 5 | (uint64_t)(p.n_elig == p.nb) << 6 |
            (uint64_t)hang_prefix_path(p.W, p.H) << 7 | (uint64_t)(p.n_tiles_s != 0) << 8 |
            (uint64_t)(p.n_tiles_e != 0) << 9 | (uint64_t)(p.t_inline != 0) << 10 | (uint64_t)p.bin_log << 16;
@@ -3328,21 +3377,9 @@ void configure_kernels_once() {
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 128 || done[dev]) return;
   done[dev] = true;
-  const int lm_caps = (int)k1_smem_lm(kLmMaxBins, 113 * 512, true);  // <= 113 KB by partition_caps_smem
-  const int lm_glob = (int)k1_smem_lm(kLmMaxBins, 0, false);
-  const int lm_mp = (int)k1_smem_lm(kTwoPassMinBins - 1, 0, false);
-  cudaFuncSetAttribute(k_partition_lm<8, true, 8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
-  cudaFuncSetAttribute(k_partition_lm<8, false, 8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
-  cudaFuncSetAttribute(k_partition_lm<8, true, 7, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
-  cudaFuncSetAttribute(k_partition_lm<8, false, 7, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
-  cudaFuncSetAttribute(k_partition_lm<8, true, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
-  cudaFuncSetAttribute(k_partition_lm<8, false, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_mp);
-  cudaFuncSetAttribute(k_partition_lm<8, true, kSupLog, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
-  cudaFuncSetAttribute(k_partition_lm<8, false, kSupLog, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  configure_partition_once();
   cudaFuncSetAttribute(k_subpart<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(SubSmem<7>) * kSubWarps));
   cudaFuncSetAttribute(k_subpart<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(SubSmem<8>) * kSubWarps));
-  cudaFuncSetAttribute(k_partition_mx<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
-  cudaFuncSetAttribute(k_partition_mx<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
   cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
   cudaFuncSetAttribute(k_topk<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)topk_smem_bytes(kTopkSmemKeys));
@@ -3353,6 +3390,13 @@ void configure_kernels_once() {
 #undef RTM_FOLD_ATTR
   cudaFuncSetAttribute(k_fold<true, true, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes(8));
   cudaFuncSetAttribute(k_fold<true, true, 7, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes(7));
+#define RTM_FOLD_ATTR_ND(SP_, BL_, CF_) \
+  cudaFuncSetAttribute(k_fold<true, SP_, BL_, CF_, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fold_smem_bytes(BL_))
+  RTM_FOLD_ATTR_ND(true, 8, true); RTM_FOLD_ATTR_ND(true, 8, false); RTM_FOLD_ATTR_ND(false, 8, false);
+  RTM_FOLD_ATTR_ND(true, 7, true); RTM_FOLD_ATTR_ND(true, 7, false); RTM_FOLD_ATTR_ND(false, 7, false);
+#undef RTM_FOLD_ATTR_ND
+  cudaFuncSetAttribute(k_fold_seq<true, 7, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<7>) * kFoldWarps));
+  cudaFuncSetAttribute(k_fold_seq<true, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<8>) * kFoldWarps));
   cudaFuncSetAttribute(k_fold_seq<true, 7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<7>) * kFoldWarps));
   cudaFuncSetAttribute(k_fold_seq<false, 7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<7>) * kFoldWarps));
   cudaFuncSetAttribute(k_fold_seq<true, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(FoldSeqSmem<8>) * kFoldWarps));
@@ -3417,4 +3461,57 @@ void launch_merge(const Params &p, const void *gathered, uint32_t world, long lo
   { k_merge_progress<<<p.nk, 1024, 0, st>>>(p, static_cast<const unsigned char *>(gathered), world, stride, gcum); count_launch(); }
 }
 
+#endif  // !RTM_TU_PARTITION
+#ifdef RTM_TU_PARTITION  // the sample partition kernels' launchers: a module of their own
+// (rtm_partition.cu); the partition kernels and their device helpers are compiled only there
+template <int BL, bool CAPS, int KS, bool MP = false>
+void launch_partition_lm(const Params &p, int n_sms, size_t sm, cudaStream_t st) {
+  const int per_sm = occupancy((const void *)k_partition_lm<BL, CAPS, KS, MP>, kK1Threads, sm);
+  unsigned grid = (unsigned)(n_sms * per_sm);
+  const unsigned work = p.n_tiles_s + (p.fuse_events ? p.n_tiles_e : 0u);
+  if (grid > work) grid = work;
+  { k_partition_lm<BL, CAPS, KS, MP><<<grid, kK1Threads, sm, st>>>(p); count_launch(); }
+}
+
+void launch_partition(const Params &p, int n_sms, cudaStream_t st) {
+  if (!p.n_tiles_s) return;
+  if (p.nsb) {  // two-pass path, pass 1: superbin keys (capacities through L1: > 2^15 buffers)
+    const bool caps = partition_caps_smem(p.nsb, p.nb);
+    const size_t sm = k1_smem_lm(p.nsb, p.nb, caps);
+    if (caps) launch_partition_lm<8, true, kSupLog>(p, n_sms, sm, st);
+    else launch_partition_lm<8, false, kSupLog>(p, n_sms, sm, st);
+    return;
+  }
+  const size_t sm = partition_smem_bytes(p.nbins, p.nb);
+  if (p.nbins <= kLmMaxBins && p.bin_log == 7) {  // few-unit calls on a small registry
+    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 7>(p, n_sms, sm, st);
+    else launch_partition_lm<8, false, 7>(p, n_sms, sm, st);
+  } else if (p.nbins <= kLmMaxBins) {  // persistent: one or two CTAs per SM
+    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 8>(p, n_sms, sm, st);
+    else launch_partition_lm<8, false, 8>(p, n_sms, sm, st);
+  } else if (p.nbins < kTwoPassMinBins) {  // 171 .. 1023 bins: ranks in passes of <= 170 bins
+    if (partition_caps_smem(p.nbins, p.nb)) launch_partition_lm<8, true, 8, true>(p, n_sms, sm, st);
+    else launch_partition_lm<8, false, 8, true>(p, n_sms, sm, st);
+  } else {
+    if (p.bin_log == 7) { k_partition_mx<7><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
+    else { k_partition_mx<8><<<p.n_tiles_s, kK1Threads, sm, st>>>(p); count_launch(); }
+  }
+}
+
+void configure_partition_once() {
+  const int lm_caps = (int)k1_smem_lm(kLmMaxBins, 113 * 512, true);  // <= 113 KB by partition_caps_smem
+  const int lm_glob = (int)k1_smem_lm(kLmMaxBins, 0, false);
+  const int lm_mp = (int)k1_smem_lm(kTwoPassMinBins - 1, 0, false);
+  cudaFuncSetAttribute(k_partition_lm<8, true, 8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false, 8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  cudaFuncSetAttribute(k_partition_lm<8, true, 7, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false, 7, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  cudaFuncSetAttribute(k_partition_lm<8, true, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_mp);
+  cudaFuncSetAttribute(k_partition_lm<8, true, kSupLog, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_caps);
+  cudaFuncSetAttribute(k_partition_lm<8, false, kSupLog, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, lm_glob);
+  cudaFuncSetAttribute(k_partition_mx<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
+  cudaFuncSetAttribute(k_partition_mx<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem_mx(kMaxBins));
+}
+#endif  // RTM_TU_PARTITION
 }  // namespace rtm

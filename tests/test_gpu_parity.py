@@ -854,6 +854,42 @@ def test_limits_max_sizes_wide_windows_and_hot_buffer():
         assert_same(got, ref, mon)  # window 3's digest covers the hot buffer's > 65535-sample count
 
 
+@pytest.mark.parametrize("dense", [True, False])
+def test_narrow_integral_boundary(dense):
+    """The fold keeps its integral term D in 32 bits when every capacity times every window length
+    of the call is below 2^32 (D lies in [0, cap * Wlen]).  Capacities up to 65534 at levels near
+    capacity, a call whose windows are 65538 ticks (65534 * 65538 = 2^32 - 4: the 32-bit path at
+    its edge, one buffer with more than 65535 samples in a window) and a call with 65539-tick
+    windows (just past it: the 64-bit path), dense and sparse, then very sparse calls of 40 such
+    windows (the sequential fold, both layouts), against the oracle."""
+    rng = np.random.default_rng(4242 + dense)
+    nb, nc, nk = 2000 if dense else 60_000, 500, 4
+    owner = (np.arange(nb) % nc).astype(np.uint32)
+    cap = rng.choice([1, 1024, 65534], size=nb).astype(np.uint16)
+    tot = np.full(nk, 10, np.int64)
+    orc, mon = _pair(owner, cap, tot, nc, t0=0, hang_windows=2, k=16)
+    t = 0
+    # windowed fold (32-bit D at its edge, then 64-bit), then very sparse calls (sequential fold)
+    for lens, n in (([65538, 1000, 0, 65538], 400_000), ([65539, 70000, 3], 400_000), ([65539] * 40, 500),
+                    ([65538] * 40, 500)):
+        ends = np.cumsum([t] + lens)[1:].astype(np.int64)
+        ts = np.sort(rng.integers(t, ends[-1], n))
+        b = rng.integers(0, nb, n).astype(np.uint32)
+        if n > 1000 and lens[0] == 65538:  # > 65535 samples of buffer 5 in the first window
+            hot = (ts < ends[0]) & (rng.random(n) < 0.5)
+            b[hot] = 5
+            assert int(hot.sum()) > 65535
+        hi = rng.random(n) < 0.8
+        lvl = np.where(hi, cap[b], (rng.random(n) * cap[b]).astype(np.int64)).astype(np.uint16)
+        s_ = np.zeros(n, gen.SAMPLE_DTYPE)
+        s_["ts"], s_["buffer_id"], s_["level"], s_["capacity"] = ts, b, lvl, cap[b]
+        ref = orc.reduce(s_, event_array([]), ends)
+        assert ref["rc"] == 0
+        mon.ingest(_dev(s_), None)
+        assert_same(mon.window_reduce(ends), ref, mon)
+        t = int(ends[-1])
+
+
 def test_order_error_then_reset_then_multiwindow_lookback():
     """A multi-window call that fails with RTM_E_ORDER has already run its fold (which publishes
     look-back flags); after rtm_reset the next multi-window call must not read those flags as

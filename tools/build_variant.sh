@@ -8,5 +8,5 @@ else git show $REV:paper_conf_micro_mosallaeii024_b200/csrc/rtm_kernels.cu > $TM
      git show $REV:paper_conf_micro_mosallaeii024_b200/csrc/rtm_internal.h > $TMP/rtm_internal.h
      git show $REV:include/rtm.h > $TMP/rtm.h; fi
 /usr/local/cuda/bin/nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -shared \
-  --expt-relaxed-constexpr -I $TMP "$@" -o $OUT $TMP/rtm_api.cpp $TMP/rtm_kernels.cu && echo built $OUT
+  --expt-relaxed-constexpr -I $TMP "$@" -o $OUT $TMP/rtm_api.cpp $TMP/rtm_kernels.cu $( [ -f $TMP/rtm_partition.cu ] && echo $TMP/rtm_partition.cu ) && echo built $OUT
 rm -rf $TMP
