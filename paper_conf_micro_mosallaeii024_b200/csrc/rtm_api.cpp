@@ -107,7 +107,7 @@ struct rtm_ctx {
   uint64_t s_own_n = 0, e_own_n = 0;
   // per-call workspaces
   DevBuf T, Bs, Be, rts, rte, treg_s, treg_e, tdesc, soff, stage, stage2, woff, smeta, emeta, lastlvl, res, kdelta, cdelta, active,
-      anyfull, hung, unit_ctr, bstat, comps, pack, gathered;
+      anyfull, hung, unit_ctr, bstat, comps, pack, gathered, endkey;
   Pinned h_small, h_res;
   // results of the last call
   bool have = false;
@@ -587,6 +587,27 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     p.tk_scratch = (unsigned long long *)c->tkscr.p;
   }
   if ((s = ensure(c, c->comps, (size_t)c->nc * sizeof(rtm_component_tasks)))) return s;
+  // Very sparse calls on the two-pass path (C5): the sequential fold walks the windows of a bin in
+  // seq_ranges ranges at once, so ~2 warps per SM slot instead of one per bin (C5: 2560 bins).
+  size_t endkey_bytes = 0;
+  {
+    Params q = p;
+    q.ns = ns;
+    if (two_pass && fold_sequential(q) && W >= 128) {
+      const uint32_t want = (uint32_t)((2u * (uint32_t)c->n_sms * 24u + nbins - 1) / nbins);
+      uint32_t R = std::min<uint32_t>({want, 8u, W / 64u});
+      if (R > 1) {
+        p.seq_range_len = (W + R - 1) / R;
+        R = (W + p.seq_range_len - 1) / p.seq_range_len;
+      }
+      if (R > 1) {
+        p.seq_ranges = R;
+        endkey_bytes = (size_t)(R - 1) * c->nb * 8;
+        if ((s = ensure(c, c->endkey, endkey_bytes))) return s;
+        p.endkey = (unsigned long long *)c->endkey.p;
+      }
+    }
+  }
 
   ClearList prep_cl;
   {
@@ -600,6 +621,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
     // long H, call shorter than H: the hang kernel stops at the first window its prefix AND empties
     if (c->H > 64 && W < c->H) cl.add(c->hung.p, Wn * c->ncw * 4);
     cl.add(c->unit_ctr.p, 16);
+    if (endkey_bytes) cl.add(c->endkey.p, endkey_bytes);
     prep_cl = cl;
   }
 
@@ -955,7 +977,7 @@ void rtm_destroy(rtm_ctx *c) {
                     &c->lastlvl, &c->res, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
                     &c->unit_ctr, &c->bstat, &c->comps, &c->pack,
                     &c->gathered, &c->tkscr, &c->mkey, &c->rcp64, &c->tkey, &c->persist, &c->klive,
-                    &c->gcum, &c->tpack, &c->tgathered};
+                    &c->gcum, &c->tpack, &c->tgathered, &c->endkey};
   graphs_clear(c);
   if (c->cap_st) cudaStreamDestroy(c->cap_st);
   for (DevBuf *b : bufs) free_buf(*b);

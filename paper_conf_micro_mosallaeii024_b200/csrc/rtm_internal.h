@@ -161,6 +161,11 @@ struct Params {
   uint32_t nsb;              // superbins (0: one-pass path)
   unsigned long long *stage2;// [n_tiles_s * kTileS]
   uint32_t *woff;            // [W * (nbins + 1)]
+  // range-parallel sequential fold (two-pass path, very sparse calls): the call's windows in
+  // seq_ranges ranges of seq_range_len, one unit per (bin, range); endkey[r][b] = max over buffer
+  // b's kept samples in range r of (staging index + 1) << 16 | level (k_subpart), 0 if none
+  uint32_t seq_ranges, seq_range_len;
+  unsigned long long *endkey;  // [(seq_ranges - 1) * nb]
 };
 
 // launchers (rtm_kernels.cu); all asynchronous on `st`
@@ -171,6 +176,7 @@ void launch_partition(const Params &p, int n_sms, cudaStream_t st);
 void launch_events(const Params &p, cudaStream_t st);
 bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s, bool two_pass);  // lane-major partition path
 bool partition_two_pass(uint32_t nbins, bool narrow);  // > 170 bins: superbins + k_subpart
+bool fold_sequential(const Params &p);  // very sparse call: the sequential fold (one warp per bin)
 void launch_subpart(const Params &p, int n_sms, cudaStream_t st);
 void launch_fold(const Params &p, int n_sms, cudaStream_t st);
 void launch_order_check(const Params &p, cudaStream_t st);

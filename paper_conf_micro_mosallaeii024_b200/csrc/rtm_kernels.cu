@@ -1137,6 +1137,8 @@ __global__ void __launch_bounds__(kSubWarps * 32, 2) k_subpart(Params p) {
     u = __shfl_sync(kFull, u, 0);
     if (u >= n_units) break;
     const unsigned w = u / nsb, S = u % nsb;
+    // window range of the range-parallel sequential fold (seq_ranges == 1: none)
+    const unsigned rng = p.seq_ranges > 1u ? w / p.seq_range_len : ~0u;
     const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
     // the unit's output base: the window's staging region + its entries of lower superbins
     unsigned before = 0;
@@ -1289,6 +1291,9 @@ __global__ void __launch_bounds__(kSubWarps * 32, 2) k_subpart(Params p) {
           const unsigned dst = Q.cur[key] + (q - Q.cb[key]);
           const unsigned long long lvl = (x >> 16) & 0xFFFFull;
           __stcg(p.stage2 + dst, ((x >> 32) << (16 + BL)) | (lvl << BL) | (x & ((1u << BL) - 1u)));
+          if (rng < p.seq_ranges - 1u)  // range-parallel sequential fold: latest level per buffer and range
+            atomicMax(p.endkey + (size_t)rng * p.nb + (S << kSupLog) + ((unsigned)x & ((1u << kSupLog) - 1u)),
+                      ((unsigned long long)(dst + 1u) << 16) | lvl);
         }
         __syncwarp();
 #pragma unroll
@@ -1890,11 +1895,18 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
   const int lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
   const bool nonempty_mode = p.hang_mode == RTM_HANG_NONEMPTY;
+  const unsigned n_ranges = p.seq_ranges > 1u ? p.seq_ranges : 1u;
   for (;;) {
-    unsigned bin = 0;
-    if (lane == 0) bin = atomicAdd(p.unit_ctr, 1u);
-    bin = __shfl_sync(kFull, bin, 0);
-    if (bin >= p.nbins) break;
+    unsigned u = 0;
+    if (lane == 0) u = atomicAdd(p.unit_ctr, 1u);
+    u = __shfl_sync(kFull, u, 0);
+    if (u >= p.nbins * n_ranges) break;
+    // unit = (bin, range of windows): range r starts from the carried levels at the end of range
+    // r - 1, i.e. each buffer's latest kept sample in the ranges before it (k_subpart's end keys),
+    // else the call's carry-in
+    const unsigned bin = u % p.nbins, rg = u / p.nbins;
+    const unsigned w_lo = n_ranges > 1u ? rg * p.seq_range_len : 0u;
+    const unsigned w_hi = n_ranges > 1u ? min(p.W, w_lo + p.seq_range_len) : p.W;
     const unsigned b_base = bin * (unsigned)kB;
     // this lane's contiguous buffers kPer lane .. kPer lane + kPer - 1 (row stores, held-full bits)
     const unsigned c0 = b_base + kPer * lane;
@@ -1911,7 +1923,15 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
       const unsigned l = lane + 32 * i, b = b_base + l;
       S.st[l] = make_uint4(0, 0, kUntouchedZ, 0);
       S.hi[l] = 0;
-      Q.lvl[l] = b < p.nb ? __ldg(p.carry_in + b) : 0;
+      unsigned short L = b < p.nb ? __ldg(p.carry_in + b) : 0;
+      for (int r2 = (int)rg - 1; r2 >= 0 && b < p.nb; --r2) {
+        const unsigned long long k = __ldcg(p.endkey + (size_t)r2 * p.nb + b);
+        if (k) {
+          L = (unsigned short)(k & 0xFFFFu);
+          break;
+        }
+      }
+      Q.lvl[l] = L;
       Q.capS[l] = b < p.nb ? __ldg(p.cap + b) : 0xFFFFu;
       Q.ownS[l] = b < p.nb ? __ldg(p.owner + b) : 0;
     }
@@ -2063,18 +2083,18 @@ __global__ void __launch_bounds__(kFoldWarps * 32) k_fold_seq(Params p) {
     // Fast path: a window's segments for this bin span <= 32 tiles; else fold_phase1.
     if (p.woff) {  // two-pass path: one contiguous range per (window, bin)
       const unsigned rs = p.nbins + 1;
-      unsigned n_lo = __ldg(p.woff + bin), n_hi = __ldg(p.woff + bin + 1);
+      unsigned n_lo = __ldg(p.woff + (size_t)w_lo * rs + bin), n_hi = __ldg(p.woff + (size_t)w_lo * rs + bin + 1);
       bool pend = false;
       unsigned pw = 0;
       unsigned long long pWlen = 0;
-      for (unsigned w = 0; w < p.W; ++w) {
+      for (unsigned w = w_lo; w < w_hi; ++w) {
         const long long tb = p.T[w], te = p.T[w + 1];
         const unsigned long long Wlen = (unsigned long long)(te - tb);
         const unsigned total = n_hi - n_lo;
         const unsigned long long *src = p.stage2 + n_lo;
         auto fetch = [&](unsigned c) -> unsigned long long { return c + lane < total ? __ldcs(src + c + lane) : 0ull; };
         unsigned long long e0 = fetch(0), e1 = total > 32u ? fetch(32) : 0ull;
-        if (w + 1 < p.W) {  // the next window's range (in flight during the finalize)
+        if (w + 1 < w_hi) {  // the next window's range (in flight during the finalize)
           n_lo = __ldg(p.woff + (size_t)(w + 1) * rs + bin);
           n_hi = __ldg(p.woff + (size_t)(w + 1) * rs + bin + 1);
         }
@@ -3274,7 +3294,7 @@ void launch_fold_seq(const Params &p, int n_sms, cudaStream_t st) {
   const size_t sm = sizeof(FoldSeqSmem<BL>) * kFoldWarps;
   const int per_sm = occupancy((const void *)k_fold_seq<true, BL>, kFoldWarps * 32, sm);
   unsigned grid = (unsigned)(n_sms * per_sm);
-  const unsigned need = (p.nbins + kFoldWarps - 1) / kFoldWarps;
+  const unsigned need = (p.nbins * (p.seq_ranges > 1u ? p.seq_ranges : 1u) + kFoldWarps - 1) / kFoldWarps;
   if (grid > need) grid = need;
   if (p.narrow_d) { k_fold_seq<true, BL, true><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
   else if (p.narrow) { k_fold_seq<true, BL><<<grid, kFoldWarps * 32, sm, st>>>(p); count_launch(); }
@@ -3337,6 +3357,7 @@ void launch_shape(const Params &p, uint64_t key[3]) {
   key[2] = (uint64_t)(p.narrow != 0) | (uint64_t)(p.fuse_events != 0) << 1 | (uint64_t)(p.nsb != 0) << 2 |
            (uint64_t)fold_sequential(p) << 3 | (uint64_t)(p.ns < 2ull * p.nb * p.W) << 4 |
            (uint64_t)(p.ns < 1ull * p.nb * p.W) << 11 | (uint64_t)(p.narrow_d != 0) << 12 |
+           (uint64_t)(p.seq_ranges & 0xFu) << 20 |
            (uint64_t)(p.mkey != nullptr) << 5 | (uint64_t)(p.n_elig == p.nb) << 6 |
            (uint64_t)hang_prefix_path(p.W, p.H) << 7 | (uint64_t)(p.n_tiles_s != 0) << 8 |
            (uint64_t)(p.n_tiles_e != 0) << 9 | (uint64_t)(p.t_inline != 0) << 10 | (uint64_t)p.bin_log << 16;

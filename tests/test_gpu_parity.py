@@ -1032,6 +1032,41 @@ def test_windowed_fold_compacted_finalize(hang_mode, rank_mode):
             assert np.array_equal(ser[f], A[-len(ser):, b][f]), (b, f)
 
 
+@pytest.mark.parametrize("hang_mode", [0, 1])
+def test_range_parallel_sequential_fold(hang_mode):
+    """Very sparse calls of >= 128 windows on the two-pass path (C5's shape: 327 680 buffers, ~0.02
+    samples per buffer-window) fold each bin's windows in several ranges at once: a range starts
+    from every buffer's latest kept sample in the earlier ranges (k_subpart's end keys), else the
+    call's carry-in.  Two calls of 260 windows, H small enough to flag components, watched buffers:
+    every window's summary, top-k, progress, hang list, the last window's table and the rings."""
+    wl = gen.C5.scaled("C5-ranges", n_samples=1_800_000, n_events=180_000, n_windows=520, hang_windows=6)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=6, k=wl.k, hang_mode=hang_mode)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    watched = [3, 100_000, wl.n_buffers - 1]
+    mon.watch(watched)
+    s, e = gen.samples(wl), gen.events(wl)
+    t_end = wl.t_end()
+    rows, w0, flagged = [], 0, 0
+    for m in (260, 260):
+        w1 = w0 + m
+        sl = slice(wl.index_at("samples", wl.t_begin(w0)), wl.index_at("samples", wl.t_begin(w1)))
+        el = slice(wl.index_at("events", wl.t_begin(w0)), wl.index_at("events", wl.t_begin(w1)))
+        assert (sl.stop - sl.start) * 8 < wl.n_buffers * m  # sequential fold, ranges (W >= 128)
+        ref = orc.reduce(s[sl], e[el], t_end[w0:w1], want_all_stats=True)
+        rows.append(ref["all_stats"])
+        mon.ingest(_dev(s[sl]), _dev(e[el]))
+        assert_same(mon.window_reduce(t_end[w0:w1]), ref, mon)
+        flagged += int(ref["summary"]["n_hung"].sum())
+        w0 = w1
+    assert flagged > 0
+    A = np.concatenate(rows)
+    for q, b in enumerate(watched):
+        ser = mon.watch_series(q)
+        for f in ("integral", "last", "max", "min", "capacity", "n_samples", "mean_occ"):
+            assert np.array_equal(ser[f], A[-300:, b][f]), (b, f)
+
+
 def test_large_registry_bins_of_128_dense_and_sparse_calls():
     """Registries of 131073 .. 524288 buffers use bins of 128 buffers (C5's 327680): the fallback
     partition with 128-buffer bins and every fold path on them - a dense call (>= 2 samples per
