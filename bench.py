@@ -59,6 +59,11 @@ class ClockSampler:
             pynvml.nvmlInit()
             self._nvml = pynvml
             self._h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            # the max clock is constant and its query slow (~3 ms): once, before the timed region;
+            # one warm-up sample too (the first NVML queries of a process take several ms, which
+            # left a 30 ms region with a single sample)
+            self._max = float(pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM))
+            self._sample()
         except Exception:
             self._nvml = None
 
@@ -66,9 +71,8 @@ class ClockSampler:
         if self._nvml is not None:
             n = self._nvml
             sm = n.nvmlDeviceGetClockInfo(self._h, n.NVML_CLOCK_SM)
-            mx = n.nvmlDeviceGetMaxClockInfo(self._h, n.NVML_CLOCK_SM)
             rs = n.nvmlDeviceGetCurrentClocksEventReasons(self._h)
-            return float(sm), float(mx), int(rs)
+            return float(sm), self._max, int(rs)
         q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.sw_power_cap,"
              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.hw_thermal_slowdown")
         out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}", "--format=csv,noheader,nounits"],
@@ -87,6 +91,10 @@ class ClockSampler:
             self._stop.wait(self.period)
 
     def __enter__(self):
+        # the timed loop holds the GIL between its (GIL-releasing) library calls: a short switch
+        # interval lets the sampler thread run every period instead of every 5 ms or less often
+        self._switch = sys.getswitchinterval()
+        sys.setswitchinterval(2e-4)
         self._t = threading.Thread(target=self._run, daemon=True)
         self._t.start()
         return self
@@ -94,6 +102,7 @@ class ClockSampler:
     def __exit__(self, *a):
         self._stop.set()
         self._t.join(timeout=10)
+        sys.setswitchinterval(self._switch)
 
     def summary(self):
         if not self.rows:

@@ -1088,7 +1088,7 @@ struct SubSmem {
   unsigned seg_base[32];
 };
 
-template <int BL>
+template <int BL, bool ENDK = false>  // ENDK: record the end keys of the range-parallel sequential fold
 __global__ void __launch_bounds__(kSubWarps * 32, 2) k_subpart(Params p) {
   extern __shared__ __align__(16) unsigned char smem[];
   using SS = SubSmem<BL>;
@@ -1138,7 +1138,7 @@ __global__ void __launch_bounds__(kSubWarps * 32, 2) k_subpart(Params p) {
     if (u >= n_units) break;
     const unsigned w = u / nsb, S = u % nsb;
     // window range of the range-parallel sequential fold (seq_ranges == 1: none)
-    const unsigned rng = p.seq_ranges > 1u ? w / p.seq_range_len : ~0u;
+    const unsigned rng = ENDK && p.seq_ranges > 1u ? w / p.seq_range_len : ~0u;
     const unsigned t_lo = p.rts[w + 1], t_hi = p.rts[w + 2];
     // the unit's output base: the window's staging region + its entries of lower superbins
     unsigned before = 0;
@@ -1291,7 +1291,7 @@ __global__ void __launch_bounds__(kSubWarps * 32, 2) k_subpart(Params p) {
           const unsigned dst = Q.cur[key] + (q - Q.cb[key]);
           const unsigned long long lvl = (x >> 16) & 0xFFFFull;
           __stcg(p.stage2 + dst, ((x >> 32) << (16 + BL)) | (lvl << BL) | (x & ((1u << BL) - 1u)));
-          if (rng < p.seq_ranges - 1u)  // range-parallel sequential fold: latest level per buffer and range
+          if (ENDK && rng < p.seq_ranges - 1u)  // range-parallel sequential fold: latest level per buffer and range
             atomicMax(p.endkey + (size_t)rng * p.nb + (S << kSupLog) + ((unsigned)x & ((1u << kSupLog) - 1u)),
                       ((unsigned long long)(dst + 1u) << 16) | lvl);
         }
@@ -3244,7 +3244,8 @@ void launch_subpart_bl(const Params &p, int n_sms, cudaStream_t st) {
   const unsigned need = (p.W * p.nsb + kSubWarps - 1) / kSubWarps;
   if (grid > need) grid = need;
   if (grid == 0) grid = 1;
-  { k_subpart<BL><<<grid, kSubWarps * 32, sm, st>>>(p); count_launch(); }
+  if (p.seq_ranges > 1u) { k_subpart<BL, true><<<grid, kSubWarps * 32, sm, st>>>(p); count_launch(); }
+  else { k_subpart<BL><<<grid, kSubWarps * 32, sm, st>>>(p); count_launch(); }
 }
 
 void launch_subpart(const Params &p, int n_sms, cudaStream_t st) {
@@ -3401,6 +3402,8 @@ void configure_kernels_once() {
   configure_partition_once();
   cudaFuncSetAttribute(k_subpart<7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(SubSmem<7>) * kSubWarps));
   cudaFuncSetAttribute(k_subpart<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(SubSmem<8>) * kSubWarps));
+  cudaFuncSetAttribute(k_subpart<7, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(SubSmem<7>) * kSubWarps));
+  cudaFuncSetAttribute(k_subpart<8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(SubSmem<8>) * kSubWarps));
   cudaFuncSetAttribute(k_topk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)topk_smem_bytes(kTopkSmemKeys));
   cudaFuncSetAttribute(k_topk<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)topk_smem_bytes(kTopkSmemKeys));

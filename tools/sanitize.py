@@ -1,7 +1,9 @@
 """Workload for compute-sanitizer (SURVEY.md §4 "Sanitizers", §5): a C1-shaped trace through the
 C-ABI in the launch configurations the tests use — one multi-window call (partition, fold with
 look-back, top-k, hang, progress), single-window calls (top-k slices + merge), rank modes SIZE and
-MEAN, invalid records — every result compared with the oracle so a silent corruption also fails.
+MEAN, invalid records, a very sparse call (sequential fold, prefix hang), a windowed call with the
+compacted finalize, a two-pass call over window ranges — every result compared with the oracle so
+a silent corruption also fails.
 
     compute-sanitizer --tool memcheck python tools/sanitize.py [--small]
 """
@@ -78,6 +80,33 @@ def main():
     ref = orc.reduce(sp, np.zeros(0, gen.EVENT_DTYPE), ends)
     mon.ingest(_dev(sp), None)
     check(mon.window_reduce(ends), ref, len(ends))
+    # a windowed call with fewer samples than buffer-windows (compacted finalize, 32-bit D)
+    cf = gen.C1.scaled("C1-cf-sanitize", n_samples=40_000 if small else 120_000, n_events=4_000, n_buffers=20_000,
+                       n_windows=8)
+    owner3, cap3, tot3 = gen.registry(cf)
+    kw = dict(t0=cf.t0, hang_windows=2, k=cf.k)
+    orc = oracle.Oracle(owner3, cap3, tot3, n_components=cf.n_components, **kw)
+    mon = Monitor(owner3, cap3, tot3, n_components=cf.n_components, **kw)
+    ref = orc.reduce(gen.samples(cf), gen.events(cf), cf.t_end())
+    mon.ingest(_dev(gen.samples(cf)), _dev(gen.events(cf)))
+    check(mon.window_reduce(cf.t_end()), ref, 8)
+    # a very sparse two-pass call of >= 128 windows: the sequential fold over window ranges
+    # (k_subpart's end keys) with its batched finalize queue
+    nb4 = 262_144
+    owner4 = (np.arange(nb4) // 4).astype(np.uint32)
+    cap4 = np.full(nb4, 16, np.uint16)
+    m4 = 6000 if small else 20_000
+    ts4 = np.sort(rng.integers(0, 130_000, m4))
+    s4 = np.zeros(m4, gen.SAMPLE_DTYPE)
+    s4["ts"], s4["buffer_id"] = ts4, rng.integers(0, nb4, m4)
+    s4["level"], s4["capacity"] = rng.integers(0, 17, m4), 16
+    ends4 = np.arange(1, 131, dtype=np.int64) * 1000
+    kw = dict(t0=0, hang_windows=4, k=16)
+    orc = oracle.Oracle(owner4, cap4, tot2, n_components=nb4 // 4, **kw)
+    mon = Monitor(owner4, cap4, tot2, n_components=nb4 // 4, **kw)
+    ref = orc.reduce(s4, np.zeros(0, gen.EVENT_DTYPE), ends4)
+    mon.ingest(_dev(s4), None)
+    check(mon.window_reduce(ends4), ref, len(ends4))
     mon.close()
     print("sanitize workload OK")
 
