@@ -51,6 +51,13 @@ for row in r[2:]:
 lines.append("")
 lines.append("Units row: " + ", ".join(f"{w}={r[1][H.index(w)]}" for w in want if w in H))
 open(out_md, "w").write("\n".join(lines) + "\n")
-json.dump({"what": "dram__bytes_read.sum + dram__bytes_write.sum per launch (ncu --set full, C2)", "all": traffic,
-           "source": rep, "tag": tag}, open(os.path.join(os.path.dirname(out_md), "traffic.json"), "w"), indent=1)
+# merge into the existing table: a capture that skipped a kernel keeps that kernel's earlier entry
+tpath = os.path.join(os.path.dirname(out_md), "traffic.json")
+old = json.load(open(tpath)) if os.path.exists(tpath) else {}
+merged = dict(old.get("all", {}))
+merged.update(traffic)
+srcs = dict(old.get("sources", {}))
+srcs.update({k: rep for k in traffic})
+json.dump({"what": "dram__bytes_read.sum + dram__bytes_write.sum per launch (ncu --set full, C2)", "all": merged,
+           "sources": srcs, "tag": tag}, open(tpath, "w"), indent=1)
 print("\n".join(lines))

@@ -11,5 +11,5 @@ for c in C2-1gpu C5-long; do timeout 400 python tools/latency.py --config $c --w
 timeout 600 $NCU --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/r02g_launches.csv \
   python tools/prof_step.py --warmup 1 --steps 1 > /dev/null 2>&1; echo "launches rc=$?"
 timeout 1200 $NCU --set full --clock-control none --import-source on -k regex:"k_partition|k_fold|k_topk|k_prep|k_hang|k_progress|k_order" \
-  -s 9 -c 7 -f -o gpurun_out/r02g_full python tools/prof_step.py --warmup 1 --steps 1 > gpurun_out/r02g_full.log 2>&1; echo "full rc=$?"
+  -s 7 -c 7 -f -o gpurun_out/r02g_full python tools/prof_step.py --warmup 1 --steps 1 > gpurun_out/r02g_full.log 2>&1; echo "full rc=$?"
 timeout 2400 python tools/c5_full.py --windows 1000000 --batch 1000 --oracle --out gpurun_out/r02g_c5_full.json > gpurun_out/r02g_c5_full.log 2>&1; echo "c5 rc=$?"; tail -3 gpurun_out/r02g_c5_full.log
