@@ -376,9 +376,10 @@ def run_streaming(mon, ds, de, wl, t_end, n_windows: int = 300, warmup: int = 20
     for w in range(warmup + n_windows):
         s0, s1 = wl.index_at("samples", wl.t_begin(w)), wl.index_at("samples", wl.t_begin(w + 1))
         e0, e1 = wl.index_at("events", wl.t_begin(w)), wl.index_at("events", wl.t_begin(w + 1))
+        sv, ev, te = ds[s0 * 16:s1 * 16], de[e0 * 16:e1 * 16], t_end[w:w + 1]  # views made before the clock
         t = time.perf_counter()
-        mon.ingest(ds[s0 * 16:s1 * 16], de[e0 * 16:e1 * 16])
-        mon.window_reduce(t_end[w:w + 1])
+        mon.ingest(sv, ev)
+        mon.window_reduce(te)
         dt = time.perf_counter() - t
         if w >= warmup:
             lat.append(dt * 1e6)

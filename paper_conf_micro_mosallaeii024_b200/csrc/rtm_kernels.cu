@@ -323,10 +323,15 @@ __global__ void __launch_bounds__(256, 4) k_prep(Params p, ClearList cl, long lo
     if (q <= p.W) split_one<true>(p, q, Bs + 1);
     else split_one<false>(p, q - (p.W + 1), Be + 1);
   }
-  grid.sync();
+  // a one-block grid (few-window calls) synchronises with a block barrier
+  auto gsync = [&]() {
+    if (gridDim.x == 1) __syncthreads();
+    else grid.sync();
+  };
+  gsync();
   if (blockIdx.x == 0) regions_one(Bs, p.ns, p.W, const_cast<uint32_t *>(p.rts), kTileS);
   if (blockIdx.x == (gridDim.x > 1 ? 1u : 0u)) regions_one(Be, p.ne, p.W, const_cast<uint32_t *>(p.rte), kTileE);
-  grid.sync();
+  gsync();
   for (uint32_t r = blockIdx.x; r < p.W + 2; r += gridDim.x) fill_region(p, r, true, true);
 }
 #endif
@@ -714,7 +719,13 @@ __global__ void __launch_bounds__(kK1Threads, 2) k_partition_lm(Params p) {
   // exclusive in-word prefixes) + 8 u16 word bases
   unsigned char *rows = reinterpret_cast<unsigned char *>(raw);
   if (CAPS)  // the capacity table in shared memory (the field check gathers it per sample)
-    for (unsigned i = threadIdx.x; i < p.nb; i += kK1Threads) capS[i] = __ldg(p.cap + i);
+  {  // 16-byte loads (8 capacities each): this fill is on the critical path of one-window calls
+    const unsigned n8 = p.nb >> 3;
+    const uint4 *src = reinterpret_cast<const uint4 *>(p.cap);
+    uint4 *dst = reinterpret_cast<uint4 *>(capS);
+    for (unsigned i = threadIdx.x; i < n8; i += kK1Threads) dst[i] = __ldg(src + i);
+    for (unsigned i = (n8 << 3) + threadIdx.x; i < p.nb; i += kK1Threads) capS[i] = __ldg(p.cap + i);
+  }
   // Tiles are claimed dynamically (p.unit_ctr[1]) so a CTA that starts late - the side-stream
   // event kernel holds SMs at first - simply takes fewer tiles.  Claims run two ahead:
   // ring[i & 3] is iteration i's tile, written by thread 0 in iteration i - 2 and read after
@@ -3224,6 +3235,8 @@ void launch_prep(const Params &p, const ClearList &cl, long long *Bs, long long 
   unsigned grid = (unsigned)std::max<unsigned long long>({(2ull * (p.W + 1) + 7) / 8, (mx / 16 + 255) / 256 + 1,
                                                           (unsigned long long)(p.W + 2), 2ull});
   if (grid > cap) grid = cap;
+  // few-window calls (streaming): one block, block barriers instead of grid barriers
+  if (p.W <= 4 && mx <= 64 * 1024) grid = 1;
   Params pp = p;
   ClearList cc = cl;
   void *args[] = {&pp, &cc, &Bs, &Be};
