@@ -107,7 +107,7 @@ struct rtm_ctx {
   uint64_t s_own_n = 0, e_own_n = 0;
   // per-call workspaces
   DevBuf T, Bs, Be, rts, rte, treg_s, treg_e, tdesc, soff, stage, stage2, woff, smeta, emeta, lastlvl, res, kdelta, cdelta, active,
-      anyfull, hung, unit_ctr, bstat, comps, pack, gathered, endkey;
+      anyfull, hung, unit_ctr, bstat, comps, pack, gathered, endkey, hsfx;
   Pinned h_small, h_res;
   // results of the last call
   bool have = false;
@@ -568,6 +568,9 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   if ((s = ensure(c, c->active, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->anyfull, Wn * c->ncw * 4))) return s;
   if ((s = ensure(c, c->hung, Wn * c->ncw * 4))) return s;
+  if (hang_block_path(W, c->H)) {
+    if ((s = ensure(c, c->hsfx, Wn * c->ncw * 4))) return s;
+  }
   if ((s = ensure(c, c->unit_ctr, 16))) return s;
   if ((s = ensure(c, c->bstat, (size_t)c->nb * sizeof(rtm_buffer_stat)))) return s;
   if (c->rank_mode == RTM_RANK_MEAN) {  // order keys (windows shorter than 2^32 ticks, checked above)
@@ -639,6 +642,7 @@ rtm_status reduce_local(rtm_ctx *c, const int64_t *t_end, uint32_t W, Params &p)
   p.kdelta = (uint32_t *)c->kdelta.p;
   p.cdelta = (unsigned long long *)c->cdelta.p; p.active = (uint32_t *)c->active.p;
   p.anyfull = (uint32_t *)c->anyfull.p; p.hung = (uint32_t *)c->hung.p;
+  p.hsfx = hang_block_path(W, c->H) ? (uint32_t *)c->hsfx.p : nullptr;
   p.unit_ctr = (uint32_t *)c->unit_ctr.p;
   p.carry_in = (const uint16_t *)c->carry[c->cur].p; p.carry_out = (uint16_t *)c->carry[c->cur ^ 1].p;
   p.run = (const uint32_t *)c->run[c->cur].p;
@@ -977,7 +981,7 @@ void rtm_destroy(rtm_ctx *c) {
                     &c->lastlvl, &c->res, &c->kdelta, &c->cdelta, &c->active, &c->anyfull, &c->hung,
                     &c->unit_ctr, &c->bstat, &c->comps, &c->pack,
                     &c->gathered, &c->tkscr, &c->mkey, &c->rcp64, &c->tkey, &c->persist, &c->klive,
-                    &c->gcum, &c->tpack, &c->tgathered, &c->endkey};
+                    &c->gcum, &c->tpack, &c->tgathered, &c->endkey, &c->hsfx};
   graphs_clear(c);
   if (c->cap_st) cudaStreamDestroy(c->cap_st);
   for (DevBuf *b : bufs) free_buf(*b);

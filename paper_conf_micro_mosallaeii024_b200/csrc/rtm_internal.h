@@ -128,6 +128,7 @@ struct Params {
   uint32_t *active;          // [W * ncw]
   uint32_t *anyfull;         // [W * ncw]
   uint32_t *hung;            // [W * ncw]
+  uint32_t *hsfx;            // [W * ncw] suffix ANDs of the block-parallel long-H hang path, or nullptr
   uint32_t *unit_ctr;        // [0] fold units dequeued, [1] partition tiles, [2] fused event tiles claimed
   int32_t fuse_events;       // the persistent partition also runs the event tiles (K3 in K1)
   uint32_t *status;          // bit0 sample order, bit1 event order
@@ -177,6 +178,7 @@ void launch_events(const Params &p, cudaStream_t st);
 bool partition_fuses_events(uint32_t nbins, uint32_t n_tiles_s, bool two_pass);  // lane-major partition path
 bool partition_two_pass(uint32_t nbins, bool narrow);  // > 170 bins: superbins + k_subpart
 bool fold_sequential(const Params &p);  // very sparse call: the sequential fold (one warp per bin)
+bool hang_block_path(uint32_t W, uint32_t H);  // long H and W >= H: block-parallel van Herk hang passes
 void launch_subpart(const Params &p, int n_sms, cudaStream_t st);
 void launch_fold(const Params &p, int n_sms, cudaStream_t st);
 void launch_order_check(const Params &p, cudaStream_t st);
