@@ -416,6 +416,30 @@ def test_long_hang_window_across_calls(H):
     assert w0 == wl.n_windows and total_hung > 0  # the long-run path was exercised
 
 
+def test_long_hang_block_edges():
+    """Long H with calls of H - 1, H, H + 1 and 2H windows: the prefix path (W < H) and the
+    block-parallel van Herk path at its edges (one full block, a one-window second block, two full
+    blocks), runs carried across all of them."""
+    H = 100
+    wl = gen.C1.scaled("C1-longH-edges", n_samples=400_000, n_events=2_000, n_windows=500, hang_windows=H)
+    owner, cap, tot = gen.registry(wl)
+    kw = dict(t0=wl.t0, hang_windows=H, k=wl.k)
+    orc, mon = _pair(owner, cap, tot, wl.n_components, **kw)
+    s, e = gen.samples(wl), gen.events(wl)
+    t_end = wl.t_end()
+    w0, total_hung = 0, 0
+    for m in (H - 1, H, H + 1, 2 * H):
+        w1 = w0 + m
+        sl = slice(wl.index_at("samples", wl.t_begin(w0)), wl.index_at("samples", wl.t_begin(w1)))
+        el = slice(wl.index_at("events", wl.t_begin(w0)), wl.index_at("events", wl.t_begin(w1)))
+        ref = orc.reduce(s[sl], e[el], t_end[w0:w1])
+        mon.ingest(_dev(s[sl]), _dev(e[el]))
+        assert_same(mon.window_reduce(t_end[w0:w1]), ref, mon, stats=False, comps=False)
+        total_hung += int(ref["summary"]["n_hung"].sum())
+        w0 = w1
+    assert total_hung > 0
+
+
 @pytest.mark.parametrize("disorder", [False, True])
 @pytest.mark.parametrize("stream", ["samples", "events"])
 def test_order_check_across_tiles_with_invalid_gap(disorder, stream):
